@@ -1,0 +1,328 @@
+#!/usr/bin/env python
+"""Benchmark of the B200-native CloverLeaf 2D timestep (BASELINE.json).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl clover|reference]
+
+One bench "step" = one full CloverLeaf timestep (every SURVEY 8(a) row:
+EOS, viscosity, calc_dt + min-reduction, PdV predictor/corrector,
+accelerate, flux_calc, both advection sweeps, reset, halo updates).
+
+N=1 workload: BASELINE configs[2], the bm deck on 3840x3840 cells (the
+"1 GPU bandwidth-roofline run"; configs[1] 960^2 and configs[0] 64^2 are
+parity-test cases in tests/).  N>1: configs[4], weak scaling with 3840^2
+cells per GPU (reading A4: 2 -> 7680x3840, 4 -> 7680^2, 8 -> 15360x7680),
+one process per GPU, NCCL halo exchange and dt MIN all-reduce.
+
+Prints ONE JSON line (rank 0).  --impl reference times the CPU oracle (the
+reference arm of this tier) on the host cores.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "cell-updates/sec per step and achieved HBM GB/s vs peak, at 1/2/4/8 B200"
+UNIT = "cell-updates/s"
+
+# Algorithmic HBM bytes per cell per launch: fp64
+# words each kernel must read + write once (8 B each).
+ALGO_BYTES_PER_CELL = {
+    "k_visc_dt": 8 * (4 + 1),            # rho0 e0 u0 v0 -> q
+    "k_dt_finalize": 0,
+    "k_lagrangian": 8 * (5 + 6),         # rho0 e0 q u0 v0 -> rho1 e1 u1 v1 Fx Fy
+    "k_advec_cell_x<1>": 8 * (4 + 3),    # rho e Fx Fy -> rho' e' Mx
+    "k_advec_cell_y<1>": 8 * (4 + 3),
+    "k_advec_cell_x<2>": 8 * (3 + 3),    # rho e Fx -> rho e Mx
+    "k_advec_cell_y<2>": 8 * (3 + 3),
+    "k_advec_mom_x<1>": 8 * (5 + 2),     # rho M Fy u v -> u v
+    "k_advec_mom_y<1>": 8 * (5 + 2),
+    "k_advec_mom_x<2>": 8 * (4 + 2),     # rho M u v -> u v
+    "k_advec_mom_y<2>": 8 * (4 + 2),
+}
+STEP_ALGO_BYTES_PER_CELL = 336  # sum over one step (each sweep kind once)
+
+
+def env_int(name, default):
+    try:
+        return int(os.environ.get(name, default))
+    except ValueError:
+        return default
+
+
+def measured_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as fh:
+            d = json.load(fh)
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, copy read+write)"
+    return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons during the timed region."""
+
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index: int):
+        self.idx = gpu_index
+        self.rows = []
+        self._stop = threading.Event()
+        self._t = None
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                out = subprocess.run(["nvidia-smi", "-i", str(self.idx), f"--query-gpu={self.Q}",
+                                      "--format=csv,noheader,nounits"], capture_output=True,
+                                     text=True, timeout=5).stdout.strip()
+                if out:
+                    self.rows.append([x.strip() for x in out.split(",")])
+            except Exception:
+                pass
+            self._stop.wait(0.2)
+
+    def start(self):
+        self._t = threading.Thread(target=self._run, daemon=True)
+        self._t.start()
+
+    def stop(self):
+        self._stop.set()
+        if self._t:
+            self._t.join(timeout=6)
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        sm = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        smax = [float(r[2]) for r in self.rows if r[2].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = set()
+        for r in self.rows:
+            for n, v in zip(names, r[5:9]):
+                if v.strip().lower() == "active":
+                    reasons.add(n)
+        return {"sm_mhz": statistics.median(sm) if sm else None,
+                "sm_max_mhz": max(smax) if smax else None,
+                "reasons": sorted(reasons), "samples": len(self.rows)}
+
+
+def weak_mesh(n):
+    """Reading A4: per-GPU 3840^2, chunk grid px x py."""
+    return {1: (3840, 3840, 1, 1), 2: (7680, 3840, 2, 1), 4: (7680, 7680, 2, 2),
+            8: (15360, 7680, 4, 2)}.get(n)
+
+
+def oracle_rate(deck, steps, warmup=0):
+    """Time the CPU oracle (as it stands, single-threaded) on `deck`."""
+    from oracle import Oracle
+    o = Oracle(deck)
+    if warmup:
+        o.step(warmup)
+    t0 = time.perf_counter()
+    o.step(steps)
+    t = time.perf_counter() - t0
+    o.close()
+    cells = deck["x_cells"] * deck["y_cells"]
+    return cells * steps / t, t
+
+
+def band_deck(nx=3840, rows=240):
+    """Bounded sample of the 3840^2 bm workload: the bottom `rows` rows at
+    the same cell size (domain [0,10] x [0, 10*rows/nx])."""
+    from workloads import bm_deck
+    d = bm_deck(nx, rows)
+    d["ymax"] = 10.0 * rows / nx
+    return d
+
+
+def run_reference(args):
+    rank = env_int("RANK", 0)
+    if rank != 0:
+        return
+    from workloads import bm_deck  # noqa: F401
+    deck = band_deck()
+    from oracle import Oracle
+    o = Oracle(deck)
+    o.step(args.warmup)
+    t0 = time.perf_counter()
+    o.step(args.steps)
+    t = time.perf_counter() - t0
+    cells = deck["x_cells"] * deck["y_cells"]
+    v = cells * args.steps / t
+    sample = (f"oracle (single-threaded C++ -O2) on a bounded sample of configs[2]: the bottom "
+              f"{deck['y_cells']} rows of the 3840^2 bm mesh at the same cell size "
+              f"({cells} cells) per step, {args.steps} timed steps after {args.warmup} warm-up")
+    line = {"impl": "reference", "metric": METRIC, "value": v, "unit": UNIT,
+            "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": 1000.0 * t / max(args.steps, 1), "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": "configs[2] sample: CloverLeaf 2D bm deck, 3840 x 240 band",
+                       "mesh": [deck["x_cells"], deck["y_cells"]]},
+            "cpu_baseline": {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
+            "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=50)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="clover", choices=["clover", "reference"])
+    ap.add_argument("--mesh", type=int, nargs=2, default=None, help="override global mesh (nx ny)")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        args.warmup = 3
+    if args.impl == "reference":
+        run_reference(args)
+        return
+
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    rank, world, local = env_int("RANK", 0), env_int("WORLD_SIZE", 1), env_int("LOCAL_RANK", 0)
+    if world != args.gpus:
+        args.gpus = world
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    from paper_conf_cluster_regulymg15_b200 import Clover, nccl_unique_id
+    from workloads import bm_deck
+
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    nx, ny, px, py = weak_mesh(world) or (3840 * world, 3840, world, 1)
+    if args.mesh:
+        nx, ny = args.mesh
+    deck = bm_deck(nx, ny, end_step=args.steps)
+    uid = None
+    if world > 1:
+        obj = [nccl_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(obj, src=0)
+        uid = obj[0]
+    stream = torch.cuda.Stream(dev)
+    sim = Clover(deck, px=px, py=py, rank=rank, nranks=world, unique_id=uid, stream=stream)
+    cells = nx * ny
+
+    # warm-up (also builds the CUDA graphs)
+    sim.step(args.warmup)
+    sim.sync()
+    clocks = ClockSampler(local)
+    clocks.start()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    e0.record(stream)
+    sim.step(args.steps)
+    e1.record(stream)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    ms = e0.elapsed_time(e1)
+    clk = clocks.stop()
+    sim.sync()
+    if world > 1:
+        t = torch.tensor([ms], device=dev, dtype=torch.float64)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+    value = cells * args.steps / (ms / 1000.0)
+    kps = sim.kernels_per_step()
+
+    # per-kernel CUDA-event durations over a second pass of K steps on the
+    # same stream (direct launches, event after every kernel)
+    prof = sim.profile_steps(args.steps)
+    local_cells = cells // world
+    kernels = {}
+    for name, (kms, n) in prof.items():
+        avg = kms / n
+        bpc = ALGO_BYTES_PER_CELL.get(name, 0)
+        kernels[name] = {"avg_ms": avg, "launches": n, "share": None,
+                         "algo_bytes_per_launch": bpc * local_cells,
+                         "achieved_gbs": (bpc * local_cells / (avg / 1e3) / 1e9) if avg > 0 and bpc else None}
+    tot = sum(v["avg_ms"] * v["launches"] for v in kernels.values())
+    for v in kernels.values():
+        v["share"] = v["avg_ms"] * v["launches"] / tot if tot else None
+    top = max((k for k in kernels if ALGO_BYTES_PER_CELL.get(k)), key=lambda k: kernels[k]["avg_ms"] * kernels[k]["launches"])
+    peak, peak_src = measured_peaks()
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(tp):
+        try:
+            with open(tp) as fh:
+                tr = json.load(fh)
+            ent = tr.get("kernels", {}).get(top)
+            if ent and tuple(tr.get("mesh", [])) == (nx // px, ny // py):
+                traffic = ent["dram_bytes_per_launch"]
+        except Exception:
+            traffic = None
+    ach = kernels[top]["achieved_gbs"]
+    step_gbs = STEP_ALGO_BYTES_PER_CELL * local_cells * args.steps / (ms / 1e3) / 1e9
+    roofline = {"bound": "hbm", "kernel": top, "achieved": ach, "peak": peak, "unit": "GB/s",
+                "frac": ach / peak if ach else None, "traffic": traffic, "peak_source": peak_src,
+                "step_achieved": step_gbs, "step_frac": step_gbs / peak,
+                "algo_bytes_per_cell_step": STEP_ALGO_BYTES_PER_CELL}
+
+    # end-to-end through the host-buffer C-ABI entry (pinned host memory)
+    e2e = None
+    if not args.no_e2e and world == 1:
+        nc, nn = cells, (nx + 1) * (ny + 1)
+        host = {}
+        for name, shp in (("density0", (ny, nx)), ("energy0", (ny, nx)),
+                          ("xvel0", (ny + 1, nx + 1)), ("yvel0", (ny + 1, nx + 1))):
+            host[name] = torch.empty(shp, dtype=torch.float64, pin_memory=True).numpy()
+        for name in host:  # current state as the input
+            host[name][...] = sim.read(name)
+        ke = max(3, min(args.steps, 10))
+        sim.step_host(1, host, host)  # warm
+        t0 = time.perf_counter()
+        for _ in range(ke):
+            sim.step_host(1, host, host)
+        te = time.perf_counter() - t0
+        e2e = {"value": cells * ke / te, "unit": UNIT, "h2d_bytes_per_step": 8 * (2 * nc + 2 * nn),
+               "d2h_bytes_per_step": 8 * (2 * nc + 2 * nn), "steps": ke,
+               "api": "clover_step_host (h2d state, 1 step, d2h state)"}
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        cdeck = bm_deck(nx, ny)
+        rate, t = oracle_rate(cdeck, 2)
+        cpu = {"value": rate, "unit": UNIT, "cores": 1, "kind": "oracle",
+               "sample": f"first 2 steps of the same {nx}x{ny} bm workload, single-threaded "
+                         f"C++ oracle (-O2), {t:.1f} s"}
+
+    summ = sim.field_summary()
+    if rank == 0:
+        line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
+                "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms / args.steps,
+                "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+                "dtype": "f64", "data": "synthetic",
+                "config": {"workload": ("configs[2]: CloverLeaf 2D bm deck 3840x3840 (clover_bm16 shape), "
+                                        "1 GPU bandwidth-roofline run") if world == 1 else
+                           f"configs[4]: weak scaling, 3840^2 cells per GPU, global {nx}x{ny}",
+                           "mesh": [nx, ny], "decomposition": f"{px}x{py}",
+                           "l2": "inputs larger than L2 (18 fp64 fields of the mesh, >2 GB vs 126 MB L2)",
+                           "graphs": True},
+                "gpu_launches": kps * args.steps,
+                "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "clocks": clk,
+                "kernels": kernels,
+                "summary_after": summ}
+        print(json.dumps(line), flush=True)
+    sim.close()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,213 @@
+/*
+ * clover.h -- C ABI of the B200-native CloverLeaf 2D timestep library
+ * (libclover.so, built from paper_conf_cluster_regulymg15_b200/csrc/).
+ *
+ * What the library computes: the hot path named by BASELINE.json north_star,
+ * i.e. one CloverLeaf 2D explicit Lagrangian-remap timestep of the
+ * compressible Euler equations on a structured staggered fp64 mesh ("a
+ * system of four partial differential equations ... conservation of energy,
+ * density and momentum ... finite volume method on a structured staggered
+ * grid", sec. V), with the step arithmetic read as in
+ * SURVEY.md sec. 8(c) c.1-c.13.  The interface
+ * follows the paper's problem statement: the mesh and its data are declared
+ * once and "all data is handed over to the library" behind an opaque handle
+ * (sec. II.A, sec. II.C).
+ *
+ * Conventions
+ *  - Every function returns an int status: CLOVER_OK (0) or a negative
+ *    CLOVER_ERR_* code.  No C++ exception crosses this boundary.
+ *  - Indices: j = x index, k = y index, 1-based interior, logical halo 2.
+ *  - Host field arrays use the GLOBAL INTERIOR, row-major, j fastest:
+ *      cells nx*ny, nodes (nx+1)*(ny+1), x-faces (nx+1)*ny, y-faces nx*(ny+1).
+ *  - Device memory: the caller hands the library ONE device workspace
+ *    (e.g. a torch.uint8 tensor) of at least clover_workspace_bytes(); the
+ *    library carves all fields from it and never allocates device memory
+ *    itself.  The caller owns the workspace and must keep it alive until
+ *    clover_finalize().  Structs and host buffers passed in are copied; the
+ *    caller keeps ownership.
+ *  - Streams: all device work is enqueued on the cudaStream_t passed to
+ *    clover_init (NULL = legacy default stream).  clover_step is
+ *    asynchronous; errors detected on the device (small dt) are latched and
+ *    returned by the next synchronising call (clover_field_summary,
+ *    clover_get_clock, clover_read_field, clover_sync, clover_finalize).
+ *  - Multi-GPU: one process per GPU; the mesh is 2D-block decomposed into
+ *    px*py chunks ("partitioning across processes and ...
+ *    standard halo exchanges"); ranks exchange depth-2 halos with NCCL
+ *    send/recv and reduce dt with an NCCL MIN all-reduce.  A single process
+ *    may also own several chunks ("local chunks"), exchanged with
+ *    device-to-device copies; results are bitwise identical for every
+ *    decomposition.
+ */
+#ifndef CLOVER_H
+#define CLOVER_H
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define CLOVER_ABI_VERSION 1
+
+enum {
+  CLOVER_OK = 0,
+  CLOVER_ERR_ARG = -1,        /* invalid argument (message: clover_last_error) */
+  CLOVER_ERR_CUDA = -2,       /* a CUDA runtime call failed */
+  CLOVER_ERR_NCCL = -3,       /* an NCCL call failed or NCCL is unavailable */
+  CLOVER_ERR_WORKSPACE = -4,  /* workspace too small or misaligned */
+  CLOVER_ERR_SMALL_DT = -5,   /* dt < dtmin: the reference's "small timestep" abort */
+  CLOVER_ERR_STATE = -7       /* call not valid in the current state */
+};
+
+enum { CLOVER_GEOM_RECT = 1, CLOVER_GEOM_CIRCLE = 2, CLOVER_GEOM_POINT = 3 };
+
+/* Tangential mirror of face fields at walls (reading A7). */
+enum { CLOVER_MIRROR_GEOMETRIC = 0, CLOVER_MIRROR_CELLCENTRE = 1 };
+
+/* Mesh and run parameters (SURVEY 2d D6 input deck).  A zero in any of
+ * dtinit/dtmax/dtmin/dtrise/dt*_safe selects the CloverLeaf default
+ * 0.1 / 1.0 / 1e-7 / 1.5 / (0.7, 0.5, 0.5, 0.7). */
+typedef struct {
+  int32_t x_cells, y_cells;         /* global mesh, >= 2 each */
+  double xmin, ymin, xmax, ymax;    /* domain, xmax > xmin, ymax > ymin */
+  double dtinit, dtmax, dtmin, dtrise;
+  double dtc_safe, dtu_safe, dtv_safe, dtdiv_safe;
+  int32_t advect_x_first;           /* 1: x sweep first on step 1 (reference) */
+  int32_t face_mirror;              /* CLOVER_MIRROR_* */
+} clover_grid;
+
+/* One entry of the state list.  states[0] is the background and fills the
+ * whole mesh; later states are painted in order.
+ * Rectangle: [xmin,xmax]x[ymin,ymax]; circle: centre (xmin,ymin) + radius;
+ * point: the vertex (xmin,ymin). */
+typedef struct {
+  double density, energy, xvel, yvel;
+  int32_t geometry;                 /* CLOVER_GEOM_* (ignored for states[0]) */
+  double xmin, xmax, ymin, ymax, radius;
+} clover_state;
+
+/* Decomposition.  nranks processes, each owning chunks_x*chunks_y/nranks
+ * chunks of a px*py chunk grid (px = chunks in x).  nranks==1 with
+ * px*py>1 runs all chunks on one GPU.  nccl_unique_id: 128 bytes from
+ * clover_nccl_unique_id() on rank 0, broadcast by the caller; NULL when
+ * nranks == 1. */
+typedef struct {
+  int32_t rank, nranks;
+  int32_t px, py;
+  const void* nccl_unique_id;
+} clover_dist;
+
+/* field_summary totals: density = mass/vol,
+ * pressure = press/vol, total energy = ie + ke. */
+typedef struct {
+  double vol, mass, ie, ke, press;
+} clover_summary;
+
+/* Field ids for clover_read_field / clover_write_field. */
+enum {
+  CLOVER_F_DENSITY0 = 0,  /* cell  */
+  CLOVER_F_ENERGY0 = 1,   /* cell  */
+  CLOVER_F_PRESSURE = 2,  /* cell, = ideal_gas(density0, energy0) at read time */
+  CLOVER_F_VISCOSITY = 3, /* cell, artificial viscosity of the last step */
+  CLOVER_F_SOUNDSPEED = 4,/* cell, = ideal_gas(density0, energy0) at read time */
+  CLOVER_F_XVEL0 = 5,     /* node */
+  CLOVER_F_YVEL0 = 6,     /* node */
+  CLOVER_F_VOL_FLUX_X = 11,  /* x-face, volume flux of the last step */
+  CLOVER_F_VOL_FLUX_Y = 12,  /* y-face */
+  CLOVER_F_MASS_FLUX_X = 13, /* x-face, mass flux of the last x sweep */
+  CLOVER_F_MASS_FLUX_Y = 14  /* y-face, mass flux of the last y sweep */
+};
+
+typedef struct clover_ctx clover_ctx;
+
+/* Bytes of device workspace clover_init needs for this grid/decomposition
+ * on this rank (all local chunks).  dist may be NULL (1 chunk). */
+int clover_workspace_bytes(const clover_grid* grid, const clover_dist* dist, int64_t* bytes);
+
+/* 128-byte NCCL unique id for a multi-process run (call on rank 0 only). */
+int clover_nccl_unique_id(void* out128);
+
+/* Create a context: carve fields from `workspace`, paint the states
+ * (generate_chunk), compute the EOS and prime all halos (start of run,
+ * SURVEY 8(c) c.1).  Validation: x_cells,y_cells >= 2; nstates >= 1;
+ * xmax > xmin; ymax > ymin; px*py >= nranks and divisible by nranks; every
+ * chunk at least 4x4 cells.  On error *out is NULL. */
+int clover_init(const clover_grid* grid, const clover_state* states, int32_t nstates,
+                const clover_dist* dist, void* workspace, int64_t workspace_bytes,
+                void* cuda_stream, clover_ctx** out);
+
+/* Advance nsteps full timesteps (SURVEY 3(ii) hydro loop: timestep, PdV
+ * predictor, accelerate, PdV corrector, flux_calc, advection sweeps,
+ * reset_field).  Asynchronous on the context stream; no host sync. */
+int clover_step(clover_ctx* ctx, int32_t nsteps);
+
+/* End-to-end entry with HOST buffers: copy the state density0, energy0
+ * (cells), xvel0, yvel0 (nodes) from host memory (pinned for speed) into the
+ * mesh, advance nsteps, copy the four state fields back to host_out (may
+ * alias host_in).  Synchronous.  Single-chunk contexts only. */
+int clover_step_host(clover_ctx* ctx, int32_t nsteps,
+                     const double* density0_in, const double* energy0_in,
+                     const double* xvel0_in, const double* yvel0_in,
+                     double* density0_out, double* energy0_out,
+                     double* xvel0_out, double* yvel0_out);
+
+/* Global field_summary over all chunks and ranks; synchronises.  The
+ * reduction is deterministic: fixed 16x16-cell tiles aligned to the global
+ * index, summed in global tile order, so every decomposition gives the same
+ * bits. */
+int clover_field_summary(clover_ctx* ctx, clover_summary* out);
+
+/* Step counter, simulated time and the last dt; synchronises. */
+int clover_get_clock(clover_ctx* ctx, int32_t* step, double* time, double* dt_last);
+
+/* dt of steps [first, first+n) (1-based step numbers, last 4096 kept). */
+int clover_dt_history(clover_ctx* ctx, int32_t first, int32_t n, double* host_out);
+
+/* Gather a field's global interior into host memory (n = element count of
+ * the field's kind, see above).  Every rank receives the full field. */
+int clover_read_field(clover_ctx* ctx, int32_t field_id, double* host, int64_t n);
+
+/* Overwrite the global interior of a state field (DENSITY0, ENERGY0, XVEL0,
+ * YVEL0) from host memory and refresh its halos. */
+int clover_write_field(clover_ctx* ctx, int32_t field_id, const double* host, int64_t n);
+
+/* Wait for all queued work; returns a latched device error if any. */
+int clover_sync(clover_ctx* ctx);
+
+/* Use CUDA graphs for clover_step (default on).  0 = direct launches. */
+int clover_set_graphs(clover_ctx* ctx, int32_t enable);
+
+/* Number of CUDA kernels one clover_step(ctx, 1) launches on this rank. */
+int clover_kernels_per_step(clover_ctx* ctx, int32_t* out);
+
+/* Profiling: run nsteps full steps with direct launches and a CUDA event
+ * after every kernel on the context's work stream; ms_out[i] / launches_out[i]
+ * receive the summed duration and launch count of kernel type i
+ * (clover_profile_name(i)); nslots must be >= CLOVER_PROFILE_SLOTS. */
+#define CLOVER_PROFILE_SLOTS 11
+int clover_profile_steps(clover_ctx* ctx, int32_t nsteps, double* ms_out, int64_t* launches_out,
+                         int32_t nslots);
+const char* clover_profile_name(int32_t i);
+
+/* Debug: run only the first `nkernels` kernel phases of the next step
+ * (1 = viscosity+calc_dt, 2 = +dt reduction, 3 = +Lagrangian phase,
+ * 4..7 = +advection kernels); the step is left incomplete.  Test only. */
+int clover_debug_partial_step(clover_ctx* ctx, int32_t nkernels);
+
+/* Debug: read an internal buffer's global interior (ids as above plus
+ * 100+ internal ids, see csrc/clover_engine.cu).  Test only. */
+int clover_debug_read_buffer(clover_ctx* ctx, int32_t buffer_id, int32_t kind,
+                             double* host, int64_t n);
+
+/* Destroy the context (does not free the caller's workspace). */
+int clover_finalize(clover_ctx* ctx);
+
+const char* clover_error_string(int code);
+/* Last error message of this thread (argument validation details). */
+const char* clover_last_error(void);
+int clover_abi_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* CLOVER_H */

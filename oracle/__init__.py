@@ -25,7 +25,8 @@ FIELDS = {
     "vol_flux_x": 11, "vol_flux_y": 12, "mass_flux_x": 13, "mass_flux_y": 14,
 }
 STAGES = {"timestep": 0, "pdv_predict": 1, "accelerate": 2, "pdv_correct": 3,
-          "flux_calc": 4, "advection": 5, "reset": 6}
+          "flux_calc": 4, "advection": 5, "reset": 6,
+          "adv_cell1": 7, "adv_mom1": 8, "adv_cell2": 9, "adv_mom2": 10}
 GEOM = {"rectangle": 1, "circle": 2, "point": 3}
 
 
@@ -75,6 +76,7 @@ def lib():
         L.oracle_run_stage.restype = ctypes.c_int32
         L.oracle_run_stage.argtypes = [vp, ctypes.c_int32]
         L.oracle_field_summary.argtypes = [vp, dp]
+        L.oracle_field_summary_compensated.argtypes = [vp, dp]
         L.oracle_clock.argtypes = [vp, ctypes.POINTER(ctypes.c_int32), dp, dp, dp]
         L.oracle_read_field.restype = ctypes.c_int32
         L.oracle_read_field.argtypes = [vp, ctypes.c_int32, dp, ctypes.c_int64]
@@ -140,9 +142,10 @@ class Oracle:
     def run_stage(self, name: str) -> int:
         return lib().oracle_run_stage(self._c, STAGES[name])
 
-    def field_summary(self) -> dict:
+    def field_summary(self, compensated: bool = False) -> dict:
         out = np.zeros(5, dtype=np.float64)
-        lib().oracle_field_summary(self._c, out.ctypes.data_as(ctypes.POINTER(ctypes.c_double)))
+        f = lib().oracle_field_summary_compensated if compensated else lib().oracle_field_summary
+        f(self._c, out.ctypes.data_as(ctypes.POINTER(ctypes.c_double)))
         return dict(zip(("vol", "mass", "ie", "ke", "press"), out.tolist()))
 
     def clock(self):

@@ -570,33 +570,35 @@ int timestep(oracle_ctx* c) {
   return 0;
 }
 
+/* advection() of SURVEY 3(ii), split into its sub-steps so tests can stop
+ * between them; advection() runs all four in order. */
+void advection_part(oracle_ctx* c, int part) {
+  const int d1 = c->advect_x ? XDIR : YDIR;
+  const int d2 = c->advect_x ? YDIR : XDIR;
+  if (part == 0) {
+    reflect(c, c->energy1, CELL, 2);
+    reflect(c, c->density1, CELL, 2);
+    reflect(c, c->vol_flux_x, XFACE, 2);
+    reflect(c, c->vol_flux_y, YFACE, 2);
+    advec_cell(c, d1, 1);
+  } else if (part == 1 || part == 3) {
+    reflect(c, c->density1, CELL, 2);
+    reflect(c, c->energy1, CELL, 2);
+    reflect(c, c->xvel1, XVEL, 2);
+    reflect(c, c->yvel1, YVEL, 2);
+    reflect(c, c->mass_flux_x, XFACE, 2);
+    reflect(c, c->mass_flux_y, YFACE, 2);
+    const int d = part == 1 ? d1 : d2;
+    const int sweep = part == 1 ? 1 : 2;
+    advec_mom(c, 1, d, sweep);
+    advec_mom(c, 2, d, sweep);
+  } else {
+    advec_cell(c, d2, 2);
+  }
+}
+
 void advection(oracle_ctx* c) {
-  int sweep_number = 1;
-  int direction = c->advect_x ? XDIR : YDIR;
-  reflect(c, c->energy1, CELL, 2);
-  reflect(c, c->density1, CELL, 2);
-  reflect(c, c->vol_flux_x, XFACE, 2);
-  reflect(c, c->vol_flux_y, YFACE, 2);
-  advec_cell(c, direction, sweep_number);
-  reflect(c, c->density1, CELL, 2);
-  reflect(c, c->energy1, CELL, 2);
-  reflect(c, c->xvel1, XVEL, 2);
-  reflect(c, c->yvel1, YVEL, 2);
-  reflect(c, c->mass_flux_x, XFACE, 2);
-  reflect(c, c->mass_flux_y, YFACE, 2);
-  advec_mom(c, 1, direction, sweep_number);
-  advec_mom(c, 2, direction, sweep_number);
-  sweep_number = 2;
-  direction = c->advect_x ? YDIR : XDIR;
-  advec_cell(c, direction, sweep_number);
-  reflect(c, c->density1, CELL, 2);
-  reflect(c, c->energy1, CELL, 2);
-  reflect(c, c->xvel1, XVEL, 2);
-  reflect(c, c->yvel1, YVEL, 2);
-  reflect(c, c->mass_flux_x, XFACE, 2);
-  reflect(c, c->mass_flux_y, YFACE, 2);
-  advec_mom(c, 1, direction, sweep_number);
-  advec_mom(c, 2, direction, sweep_number);
+  for (int part = 0; part < 4; ++part) advection_part(c, part);
 }
 
 /* c.11 reset_field */
@@ -792,14 +794,19 @@ int32_t oracle_run_stage(oracle_ctx* c, int32_t stage) {
     case OS_FLUX_CALC: flux_calc(c); return 0;
     case OS_ADVECTION: advection(c); return 0;
     case OS_RESET: finish_step(c); return 0;
+    case OS_ADV_CELL1: advection_part(c, 0); return 0;
+    case OS_ADV_MOM1: advection_part(c, 1); return 0;
+    case OS_ADV_CELL2: advection_part(c, 2); return 0;
+    case OS_ADV_MOM2: advection_part(c, 3); return 0;
   }
   return -1;
 }
 
-/* c.12 field_summary */
-void oracle_field_summary(oracle_ctx* c, double* out) {
+/* c.12 field_summary; compensated = 0: sequential accumulation in the
+ * reference's loop order; 1: Neumaier compensated sums of the same terms. */
+static void field_summary_impl(oracle_ctx* c, double* out, int compensated) {
   ideal_gas(c, false);
-  double vol = 0.0, mass = 0.0, ie = 0.0, ke = 0.0, press = 0.0;
+  double acc[5] = {0.0, 0.0, 0.0, 0.0, 0.0}, comp[5] = {0.0, 0.0, 0.0, 0.0, 0.0};
   for (int k = c->y_min; k <= c->y_max; ++k)
     for (int j = c->x_min; j <= c->x_max; ++j) {
       double vsqrd = 0.0;
@@ -808,14 +815,27 @@ void oracle_field_summary(oracle_ctx* c, double* out) {
           vsqrd = vsqrd + 0.25 * (c->xvel0(jv, kv) * c->xvel0(jv, kv) + c->yvel0(jv, kv) * c->yvel0(jv, kv));
       double cell_vol = c->volume(j, k);
       double cell_mass = cell_vol * c->density0(j, k);
-      vol = vol + cell_vol;
-      mass = mass + cell_mass;
-      ie = ie + cell_mass * c->energy0(j, k);
-      ke = ke + cell_mass * 0.5 * vsqrd;
-      press = press + cell_vol * c->pressure(j, k);
+      double term[5] = {cell_vol, cell_mass, cell_mass * c->energy0(j, k), cell_mass * 0.5 * vsqrd,
+                        cell_vol * c->pressure(j, k)};
+      for (int q = 0; q < 5; ++q) {
+        if (!compensated) {
+          acc[q] = acc[q] + term[q];
+        } else {
+          double t = acc[q] + term[q];
+          if (std::fabs(acc[q]) >= std::fabs(term[q]))
+            comp[q] += (acc[q] - t) + term[q];
+          else
+            comp[q] += (term[q] - t) + acc[q];
+          acc[q] = t;
+        }
+      }
     }
-  out[0] = vol; out[1] = mass; out[2] = ie; out[3] = ke; out[4] = press;
+  for (int q = 0; q < 5; ++q) out[q] = acc[q] + comp[q];
 }
+
+void oracle_field_summary(oracle_ctx* c, double* out) { field_summary_impl(c, out, 0); }
+
+void oracle_field_summary_compensated(oracle_ctx* c, double* out) { field_summary_impl(c, out, 1); }
 
 void oracle_clock(oracle_ctx* c, int32_t* step, double* time, double* dt, double* dtold) {
   if (step) *step = c->step;

@@ -63,7 +63,11 @@ enum {
   OS_PDV_CORRECT,
   OS_FLUX_CALC,
   OS_ADVECTION,     /* both sweeps */
-  OS_RESET          /* reset_field + advect_x flip + time/step */
+  OS_RESET,         /* reset_field + advect_x flip + time/step */
+  OS_ADV_CELL1,     /* advection() split into its four sub-steps, each with */
+  OS_ADV_MOM1,      /* the halo updates that precede it in the reference   */
+  OS_ADV_CELL2,
+  OS_ADV_MOM2
 };
 
 typedef struct oracle_ctx oracle_ctx;
@@ -75,8 +79,13 @@ void oracle_destroy(oracle_ctx* c);
  * returns 0, or -5 if dt < dtmin (ref "small timestep"). */
 int32_t oracle_step(oracle_ctx* c, int32_t n, double* dt_hist);
 int32_t oracle_run_stage(oracle_ctx* c, int32_t stage);
-/* field_summary: out = {vol, mass, ie, ke, press} */
+/* field_summary: out = {vol, mass, ie, ke, press}, accumulated
+ * sequentially in the reference's loop order (c.12). */
 void oracle_field_summary(oracle_ctx* c, double* out5);
+/* Same per-cell terms, accumulated with Neumaier compensated summation:
+ * the totals to ~1 ulp, for meshes where the sequential sum's own rounding
+ * (up to n*eps relative, 3e-9 at 3840^2) exceeds the 1e-10 parity gate. */
+void oracle_field_summary_compensated(oracle_ctx* c, double* out5);
 void oracle_clock(oracle_ctx* c, int32_t* step, double* time, double* dt, double* dtold);
 int32_t oracle_read_field(oracle_ctx* c, int32_t fid, double* out, int64_t n);
 /* writes the interior of a field; caller then calls oracle_refresh */

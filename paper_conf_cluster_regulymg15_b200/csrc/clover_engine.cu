@@ -1,0 +1,1023 @@
+// clover_engine.cu -- step engine and C ABI (include/clover.h) of the
+// B200-native CloverLeaf 2D timestep.
+//
+// Owns: the chunk decomposition (sec. II.B: up-front
+// partitioning + halo exchanges), the per-step kernel schedule (SURVEY.md
+// 3(ii) hydro order, fused as in DESIGN.md "Kernels"), the device-resident
+// dt reduction, halo exchange phases (device-to-device copies between local
+// chunks; NCCL send/recv between ranks), CUDA-graph capture of the step,
+// and the deterministic field_summary.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "clover.h"
+#include "clover_aux.cuh"
+#include "clover_common.cuh"
+#include "clover_kernels.cuh"
+
+#ifdef CLOVER_WITH_NCCL
+#include <nccl.h>
+#endif
+
+using namespace clover;
+
+namespace {
+
+thread_local std::string g_last_error;
+
+int fail(int code, const std::string& msg) {
+  g_last_error = msg;
+  return code;
+}
+
+#define CK(call)                                                                   \
+  do {                                                                             \
+    cudaError_t e_ = (call);                                                       \
+    if (e_ != cudaSuccess)                                                         \
+      return fail(CLOVER_ERR_CUDA, std::string(#call) + ": " + cudaGetErrorString(e_)); \
+  } while (0)
+
+#ifdef CLOVER_WITH_NCCL
+#define NK(call)                                                                   \
+  do {                                                                             \
+    ncclResult_t r_ = (call);                                                      \
+    if (r_ != ncclSuccess)                                                         \
+      return fail(CLOVER_ERR_NCCL, std::string(#call) + ": " + ncclGetErrorString(r_)); \
+  } while (0)
+#endif
+
+// Buffers of one chunk.  State A (time level 0), B (after the Lagrangian
+// phase), C (after the first advection sweep); reset_field is the
+// rotation C -> A performed by the second sweep writing into A.
+enum Buf {
+  B_D0, B_E0, B_U0, B_V0,     // A
+  B_D1, B_E1, B_U1, B_V1,     // B
+  B_D2, B_E2, B_U2, B_V2,     // C
+  B_Q, B_FX, B_FY, B_MX, B_MY, B_SCR, NBUF
+};
+
+const int kBufKind[NBUF] = {K_CELL, K_CELL, K_XVEL, K_YVEL, K_CELL, K_CELL, K_XVEL, K_YVEL,
+                            K_CELL, K_CELL, K_XVEL, K_YVEL, K_CELL, K_XFACE, K_YFACE,
+                            K_XFACE, K_YFACE, K_CELL};
+
+constexpr int64_t kAlign = 256;
+inline int64_t align_up(int64_t v, int64_t a) { return (v + a - 1) / a * a; }
+
+struct ChunkState {
+  Chunk c;
+  int cx, cy, id;
+  double* buf[NBUF];
+  double* partials;  // summary partials, ntx*nty*5
+  int ntx, nty;
+};
+
+struct Layout {
+  int px, py;
+  std::vector<int> xs, ys;  // chunk boundaries in global cells (size px+1, py+1)
+  bool tile_aligned;
+};
+
+Layout decompose(int NX, int NY, int px, int py) {
+  Layout L;
+  L.px = px; L.py = py;
+  L.tile_aligned = (NX >= ST * px) && (NY >= ST * py);
+  auto split = [&](int N, int p, std::vector<int>& b) {
+    b.assign(p + 1, 0);
+    for (int i = 1; i < p; ++i) {
+      int64_t v = (int64_t)i * N / p;
+      if (L.tile_aligned) v = (v + ST / 2) / ST * ST;
+      b[i] = (int)v;
+    }
+    b[p] = N;
+  };
+  split(NX, px, L.xs);
+  split(NY, py, L.ys);
+  return L;
+}
+
+int64_t field_elems(int nx, int ny, int* pitch_out) {
+  // columns: j in [-HALO, nx+1+HALO] with j=0 at COL0; rows k in [-HALO, ny+1+HALO]
+  int pitch = (int)align_up(COL0 + nx + 2 + HALO, 32);
+  if (pitch_out) *pitch_out = pitch;
+  int rows = ny + 2 + 2 * HALO;
+  return (int64_t)pitch * rows;
+}
+
+}  // namespace
+
+struct clover_ctx {
+  clover_grid g;
+  std::vector<clover_state> states;
+  int rank = 0, nranks = 1;
+  Layout L;
+  std::vector<ChunkState> chunks;  // local chunks
+  std::vector<int> owner;          // chunk id -> rank
+  cudaStream_t user = nullptr, work = nullptr;
+  cudaEvent_t ev_in = nullptr, ev_out = nullptr;
+  StepScalars* scal = nullptr;
+  double* hist = nullptr;
+  double* xbuf_send = nullptr;  // NCCL staging
+  double* xbuf_recv = nullptr;
+  int64_t xbuf_elems = 0;
+  DtParams dtp;
+  GlobalGeom gg;
+  bool advect_x = true;
+  bool use_graphs = true;
+  cudaGraphExec_t gexec[2] = {nullptr, nullptr};
+  int64_t ws_bytes = 0;
+  bool prof = false;
+  std::vector<std::pair<int, cudaEvent_t>> prof_events;
+#ifdef CLOVER_WITH_NCCL
+  ncclComm_t comm = nullptr;
+#endif
+};
+
+namespace {
+
+void fill_defaults(clover_grid& g) {
+  if (g.dtinit == 0.0) g.dtinit = 0.1;
+  if (g.dtmax == 0.0) g.dtmax = 1.0;
+  if (g.dtmin == 0.0) g.dtmin = 1.0e-7;
+  if (g.dtrise == 0.0) g.dtrise = 1.5;
+  if (g.dtc_safe == 0.0) g.dtc_safe = 0.7;
+  if (g.dtu_safe == 0.0) g.dtu_safe = 0.5;
+  if (g.dtv_safe == 0.0) g.dtv_safe = 0.5;
+  if (g.dtdiv_safe == 0.0) g.dtdiv_safe = 0.7;
+}
+
+int validate(const clover_grid* g, const clover_dist* d, int* px, int* py, int* rank, int* nranks) {
+  if (!g) return fail(CLOVER_ERR_ARG, "grid is NULL");
+  if (g->x_cells < 4 || g->y_cells < 4) return fail(CLOVER_ERR_ARG, "x_cells and y_cells must be >= 4");
+  if (!(g->xmax > g->xmin) || !(g->ymax > g->ymin)) return fail(CLOVER_ERR_ARG, "empty domain");
+  if (g->face_mirror != 0 && g->face_mirror != 1) return fail(CLOVER_ERR_ARG, "face_mirror must be 0 or 1");
+  *px = 1; *py = 1; *rank = 0; *nranks = 1;
+  if (d) {
+    *px = d->px; *py = d->py; *rank = d->rank; *nranks = d->nranks;
+    if (*px < 1 || *py < 1) return fail(CLOVER_ERR_ARG, "px, py must be >= 1");
+    if (*nranks < 1 || *rank < 0 || *rank >= *nranks) return fail(CLOVER_ERR_ARG, "bad rank/nranks");
+    if ((*px * *py) % *nranks != 0) return fail(CLOVER_ERR_ARG, "px*py must be a multiple of nranks");
+    if (*nranks > 1 && !d->nccl_unique_id) return fail(CLOVER_ERR_ARG, "nccl_unique_id required for nranks > 1");
+  }
+  Layout L = decompose(g->x_cells, g->y_cells, *px, *py);
+  for (int i = 0; i < *px; ++i)
+    if (L.xs[i + 1] - L.xs[i] < 4) return fail(CLOVER_ERR_ARG, "every chunk needs >= 4 cells in x");
+  for (int i = 0; i < *py; ++i)
+    if (L.ys[i + 1] - L.ys[i] < 4) return fail(CLOVER_ERR_ARG, "every chunk needs >= 4 cells in y");
+  return CLOVER_OK;
+}
+
+std::vector<int> local_chunk_ids(int px, int py, int rank, int nranks) {
+  int per = px * py / nranks;
+  std::vector<int> ids;
+  for (int i = rank * per; i < (rank + 1) * per; ++i) ids.push_back(i);
+  return ids;
+}
+
+int64_t compute_workspace(const clover_grid* g, int px, int py, int rank, int nranks) {
+  Layout L = decompose(g->x_cells, g->y_cells, px, py);
+  int64_t bytes = align_up(sizeof(StepScalars), kAlign) + align_up(DT_HIST * 8, kAlign);
+  int64_t maxrows = 0, maxcols = 0;
+  for (int id : local_chunk_ids(px, py, rank, nranks)) {
+    int cx = id % px, cy = id / px;
+    int nx = L.xs[cx + 1] - L.xs[cx], ny = L.ys[cy + 1] - L.ys[cy];
+    int64_t fe = field_elems(nx, ny, nullptr);
+    bytes += NBUF * align_up(fe * 8, kAlign);
+    int ntx = (nx + ST - 1) / ST, nty = (ny + ST - 1) / ST;
+    bytes += align_up((int64_t)ntx * nty * 5 * 8, kAlign);
+    maxrows = std::max<int64_t>(maxrows, ny + 2 + 2 * HALO);
+    maxcols = std::max<int64_t>(maxcols, nx + 2 + 2 * HALO);
+  }
+  if (nranks > 1) {
+    // staging for up to 4 neighbours x 6 fields x HALO lines
+    int64_t line = std::max(maxrows, maxcols);
+    int64_t el = 4 * 6 * HALO * line;
+    bytes += 2 * align_up(el * 8, kAlign);
+  }
+  return bytes;
+}
+
+// ---------------------------------------------------------------- exchange
+// Copy the halo strips of `fields` between neighbouring chunks: all x
+// neighbours first (full allocated height, so y-halo rows travel too), then
+// all y neighbours (full width, fixing the corners).  Local pairs use
+// cudaMemcpy2DAsync; remote pairs NCCL send/recv through staging buffers.
+struct XferDesc {  // one rectangular strip of one field
+  double* base;    // chunk base (local (0,0))
+  int pitch;
+  int j0, k0, w, h;
+};
+
+inline double* strip_ptr(const XferDesc& d) { return d.base + (int64_t)d.k0 * d.pitch + d.j0; }
+
+int copy_strip(clover_ctx* ctx, const XferDesc& dst, const XferDesc& src) {
+  CK(cudaMemcpy2DAsync(strip_ptr(dst), (size_t)dst.pitch * 8, strip_ptr(src), (size_t)src.pitch * 8,
+                       (size_t)src.w * 8, src.h, cudaMemcpyDeviceToDevice, ctx->work));
+  return CLOVER_OK;
+}
+
+// strips for side `side` (0 left, 1 right, 2 bottom, 3 top) of chunk cs:
+// send = owned points next to that side, recv = halo points of that side.
+void side_strips(const ChunkState& cs, int buf, int side, XferDesc& send, XferDesc& recv) {
+  const Chunk& c = cs.c;
+  const int kind = kBufKind[buf];
+  const int ox = (kind == K_XVEL || kind == K_YVEL || kind == K_XFACE) ? 1 : 0;
+  const int oy = (kind == K_XVEL || kind == K_YVEL || kind == K_YFACE) ? 1 : 0;
+  send.base = recv.base = cs.buf[buf];
+  send.pitch = recv.pitch = c.pitch;
+  const int full_h = c.ny + 1 + 2 * HALO, full_w = c.nx + 1 + 2 * HALO;
+  if (side == 0) {          // left: send [1+ox, HALO+ox], recv [1-HALO, 0]
+    send.j0 = 1 + ox; recv.j0 = 1 - HALO;
+    send.w = recv.w = HALO;
+    send.k0 = recv.k0 = -HALO; send.h = recv.h = full_h;
+  } else if (side == 1) {   // right: send [nx+1-HALO, nx], recv [nx+ox+1, nx+ox+HALO]
+    send.j0 = c.nx + 1 - HALO; recv.j0 = c.nx + ox + 1;
+    send.w = recv.w = HALO;
+    send.k0 = recv.k0 = -HALO; send.h = recv.h = full_h;
+  } else if (side == 2) {   // bottom
+    send.k0 = 1 + oy; recv.k0 = 1 - HALO;
+    send.h = recv.h = HALO;
+    send.j0 = recv.j0 = -HALO; send.w = recv.w = full_w;
+  } else {                  // top
+    send.k0 = c.ny + 1 - HALO; recv.k0 = c.ny + oy + 1;
+    send.h = recv.h = HALO;
+    send.j0 = recv.j0 = -HALO; send.w = recv.w = full_w;
+  }
+}
+
+int neighbour(const clover_ctx* ctx, const ChunkState& cs, int side) {
+  int cx = cs.cx, cy = cs.cy;
+  if (side == 0) cx -= 1;
+  if (side == 1) cx += 1;
+  if (side == 2) cy -= 1;
+  if (side == 3) cy += 1;
+  if (cx < 0 || cy < 0 || cx >= ctx->L.px || cy >= ctx->L.py) return -1;
+  return cy * ctx->L.px + cx;
+}
+
+ChunkState* local_chunk(clover_ctx* ctx, int id) {
+  for (auto& cs : ctx->chunks)
+    if (cs.id == id) return &cs;
+  return nullptr;
+}
+
+int exchange_axis(clover_ctx* ctx, const std::vector<int>& bufs, int axis) {
+  const int s_lo = axis == 0 ? 0 : 2, s_hi = axis == 0 ? 1 : 3;
+  // local pairs
+  for (auto& cs : ctx->chunks) {
+    int nb = neighbour(ctx, cs, s_hi);
+    if (nb < 0) continue;
+    ChunkState* other = local_chunk(ctx, nb);
+    if (!other) continue;
+    for (int b : bufs) {
+      XferDesc sA, rA, sB, rB;
+      side_strips(cs, b, s_hi, sA, rA);
+      side_strips(*other, b, s_lo, sB, rB);
+      int rc = copy_strip(ctx, rB, sA);  // my high side -> neighbour's low halo
+      if (rc) return rc;
+      rc = copy_strip(ctx, rA, sB);      // neighbour's low side -> my high halo
+      if (rc) return rc;
+    }
+  }
+#ifdef CLOVER_WITH_NCCL
+  if (ctx->nranks > 1) {
+    // pack every remote side into the staging buffer, one NCCL group
+    struct Msg { int peer; int64_t off, n; ChunkState* cs; int side; };
+    std::vector<Msg> msgs;
+    int64_t off = 0;
+    for (auto& cs : ctx->chunks)
+      for (int side : {s_lo, s_hi}) {
+        int nb = neighbour(ctx, cs, side);
+        if (nb < 0 || local_chunk(ctx, nb)) continue;
+        int64_t n = 0;
+        for (int b : bufs) {
+          XferDesc s, r;
+          side_strips(cs, b, side, s, r);
+          XferDesc dst{ctx->xbuf_send + off + n, s.w, 0, 0, s.w, s.h};
+          int rc = copy_strip(ctx, dst, s);
+          if (rc) return rc;
+          n += (int64_t)s.w * s.h;
+        }
+        msgs.push_back({ctx->owner[nb], off, n, &cs, side});
+        off += n;
+      }
+    if (off > ctx->xbuf_elems) return fail(CLOVER_ERR_STATE, "halo staging buffer too small");
+    NK(ncclGroupStart());
+    for (auto& m : msgs) {
+      NK(ncclSend(ctx->xbuf_send + m.off, (size_t)m.n, ncclFloat64, m.peer, ctx->comm, ctx->work));
+      NK(ncclRecv(ctx->xbuf_recv + m.off, (size_t)m.n, ncclFloat64, m.peer, ctx->comm, ctx->work));
+    }
+    NK(ncclGroupEnd());
+    for (auto& m : msgs) {
+      int64_t n = 0;
+      for (int b : bufs) {
+        XferDesc s, r;
+        side_strips(*m.cs, b, m.side, s, r);
+        XferDesc src{ctx->xbuf_recv + m.off + n, r.w, 0, 0, r.w, r.h};
+        int rc = copy_strip(ctx, r, src);
+        if (rc) return rc;
+        n += (int64_t)r.w * r.h;
+      }
+    }
+  }
+#endif
+  return CLOVER_OK;
+}
+
+bool needs_exchange(const clover_ctx* ctx) { return ctx->L.px * ctx->L.py > 1; }
+
+int exchange(clover_ctx* ctx, const std::vector<int>& bufs) {
+  if (!needs_exchange(ctx)) return CLOVER_OK;
+  int rc = exchange_axis(ctx, bufs, 0);
+  if (rc) return rc;
+  return exchange_axis(ctx, bufs, 1);
+}
+
+// ---------------------------------------------------------------- schedule
+dim3 cell_grid(const Chunk& c, int bx, int by) { return dim3((c.nx + bx - 1) / bx, (c.ny + by - 1) / by); }
+dim3 node_grid(const Chunk& c, int bx, int by) { return dim3((c.nx + 1 + bx - 1) / bx, (c.ny + 1 + by - 1) / by); }
+
+#define LAUNCH_CHECK()                                                            \
+  do {                                                                            \
+    cudaError_t e_ = cudaGetLastError();                                          \
+    if (e_ != cudaSuccess) return fail(CLOVER_ERR_CUDA, std::string("launch: ") + cudaGetErrorString(e_)); \
+  } while (0)
+
+#define STEP_LAUNCH_CHECK()                                                       \
+  do {                                                                            \
+    LAUNCH_CHECK();                                                               \
+    if (ctx->prof) prof_mark(ctx, cur_prof_id);                                   \
+  } while (0)
+
+// Kernel types for clover_profile (names in kProfNames).
+enum { P_VISC_DT, P_DT_FINAL, P_LAGR, P_CELL_X1, P_CELL_X2, P_CELL_Y1, P_CELL_Y2,
+       P_MOM_X1, P_MOM_X2, P_MOM_Y1, P_MOM_Y2, NPROF };
+const char* kProfNames[NPROF] = {"k_visc_dt", "k_dt_finalize", "k_lagrangian",
+                                 "k_advec_cell_x<1>", "k_advec_cell_x<2>", "k_advec_cell_y<1>",
+                                 "k_advec_cell_y<2>", "k_advec_mom_x<1>", "k_advec_mom_x<2>",
+                                 "k_advec_mom_y<1>", "k_advec_mom_y<2>"};
+
+// Record an event after each profiled kernel; (prev event, this event)
+// bracket exactly that kernel on the work stream.
+void prof_mark(clover_ctx* ctx, int id) {
+  cudaEvent_t e;
+  cudaEventCreate(&e);
+  cudaEventRecord(e, ctx->work);
+  ctx->prof_events.push_back({id, e});
+}
+
+// Enqueue kernel phases [0, nphase) of one step (7 = full step).
+int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
+  cudaStream_t st = ctx->work;
+  const dim3 blk(32, 8);
+  int cur_prof_id = P_VISC_DT;
+  if (ctx->prof) prof_mark(ctx, -1);
+  if (nphase >= 1) {
+    for (auto& cs : ctx->chunks) {
+      k_visc_dt<<<cell_grid(cs.c, 32, 8), blk, 0, st>>>(cs.c, cs.buf[B_D0], cs.buf[B_E0], cs.buf[B_U0],
+                                                         cs.buf[B_V0], cs.buf[B_Q], ctx->scal, ctx->dtp);
+      STEP_LAUNCH_CHECK();
+    }
+    int rc = exchange(ctx, {B_Q});
+    if (rc) return rc;
+    if (ctx->prof) prof_mark(ctx, -1);
+  }
+  if (nphase >= 2) {
+    cur_prof_id = P_DT_FINAL;
+#ifdef CLOVER_WITH_NCCL
+    if (ctx->nranks > 1)
+      NK(ncclAllReduce(&ctx->scal->dt_slot, &ctx->scal->dt_slot, 1, ncclUint64, ncclMin, ctx->comm, st));
+#endif
+    if (ctx->prof) prof_mark(ctx, -1);
+    k_dt_finalize<<<1, 1, 0, st>>>(ctx->scal, ctx->hist, ctx->dtp);
+    STEP_LAUNCH_CHECK();
+  }
+  if (nphase >= 3) {
+    cur_prof_id = P_LAGR;
+    for (auto& cs : ctx->chunks) {
+      k_lagrangian<<<cell_grid(cs.c, LX, LY), dim3(LX, LY), 0, st>>>(
+          cs.c, cs.buf[B_D0], cs.buf[B_E0], cs.buf[B_U0], cs.buf[B_V0], cs.buf[B_Q], cs.buf[B_D1],
+          cs.buf[B_E1], cs.buf[B_U1], cs.buf[B_V1], cs.buf[B_FX], cs.buf[B_FY], ctx->scal);
+      STEP_LAUNCH_CHECK();
+    }
+    int rc = exchange(ctx, {B_D1, B_E1, B_U1, B_V1, B_FX, B_FY});
+    if (rc) return rc;
+    if (ctx->prof) prof_mark(ctx, -1);
+  }
+  const dim3 ablk(AX, AY);
+  // sweep 1 (direction d1) reads B writes C; sweep 2 reads C writes A.
+  for (int sweep = 1; sweep <= 2; ++sweep) {
+    const bool xdir = (sweep == 1) ? advect_x : !advect_x;
+    const int ph_cell = sweep == 1 ? 4 : 6;
+    const int rin = sweep == 1 ? B_D1 : B_D2, ein = sweep == 1 ? B_E1 : B_E2;
+    const int rout = sweep == 1 ? B_D2 : B_D0, eout = sweep == 1 ? B_E2 : B_E0;
+    const int uin = sweep == 1 ? B_U1 : B_U2, vin = sweep == 1 ? B_V1 : B_V2;
+    const int uout = sweep == 1 ? B_U2 : B_U0, vout = sweep == 1 ? B_V2 : B_V0;
+    const int mbuf = xdir ? B_MX : B_MY;
+    if (nphase >= ph_cell) {
+      cur_prof_id = xdir ? (sweep == 1 ? P_CELL_X1 : P_CELL_X2) : (sweep == 1 ? P_CELL_Y1 : P_CELL_Y2);
+      for (auto& cs : ctx->chunks) {
+        const double* fx = cs.buf[B_FX];
+        const double* fy = cs.buf[B_FY];
+        if (xdir) {
+          if (sweep == 1)
+            k_advec_cell_x<1><<<cell_grid(cs.c, AX, AY), ablk, 0, st>>>(cs.c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf]);
+          else
+            k_advec_cell_x<2><<<cell_grid(cs.c, AX, AY), ablk, 0, st>>>(cs.c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf]);
+        } else {
+          if (sweep == 1)
+            k_advec_cell_y<1><<<cell_grid(cs.c, AX, AY), ablk, 0, st>>>(cs.c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf]);
+          else
+            k_advec_cell_y<2><<<cell_grid(cs.c, AX, AY), ablk, 0, st>>>(cs.c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf]);
+        }
+        STEP_LAUNCH_CHECK();
+      }
+      int rc = exchange(ctx, {rout, eout, mbuf});
+      if (rc) return rc;
+      if (ctx->prof) prof_mark(ctx, -1);
+    }
+    if (nphase >= ph_cell + 1) {
+      cur_prof_id = xdir ? (sweep == 1 ? P_MOM_X1 : P_MOM_X2) : (sweep == 1 ? P_MOM_Y1 : P_MOM_Y2);
+      for (auto& cs : ctx->chunks) {
+        if (xdir) {
+          if (sweep == 1)
+            k_advec_mom_x<1><<<node_grid(cs.c, AX, AY), ablk, 0, st>>>(cs.c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FY], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout]);
+          else
+            k_advec_mom_x<2><<<node_grid(cs.c, AX, AY), ablk, 0, st>>>(cs.c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FY], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout]);
+        } else {
+          if (sweep == 1)
+            k_advec_mom_y<1><<<node_grid(cs.c, AX, AY), ablk, 0, st>>>(cs.c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FX], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout]);
+          else
+            k_advec_mom_y<2><<<node_grid(cs.c, AX, AY), ablk, 0, st>>>(cs.c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FX], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout]);
+        }
+        STEP_LAUNCH_CHECK();
+      }
+      int rc = exchange(ctx, {uout, vout});
+      if (rc) return rc;
+      if (ctx->prof) prof_mark(ctx, -1);
+    }
+  }
+  return CLOVER_OK;
+}
+
+int join_in(clover_ctx* ctx) {
+  CK(cudaEventRecord(ctx->ev_in, ctx->user));
+  CK(cudaStreamWaitEvent(ctx->work, ctx->ev_in, 0));
+  return CLOVER_OK;
+}
+int join_out(clover_ctx* ctx) {
+  CK(cudaEventRecord(ctx->ev_out, ctx->work));
+  CK(cudaStreamWaitEvent(ctx->user, ctx->ev_out, 0));
+  return CLOVER_OK;
+}
+
+int build_graph(clover_ctx* ctx, int parity) {
+  cudaGraph_t graph = nullptr;
+  CK(cudaStreamBeginCapture(ctx->work, cudaStreamCaptureModeThreadLocal));
+  int rc = enqueue_step(ctx, parity == 0, 7);
+  cudaError_t e = cudaStreamEndCapture(ctx->work, &graph);
+  if (rc) {
+    if (graph) cudaGraphDestroy(graph);
+    return rc;
+  }
+  if (e != cudaSuccess) return fail(CLOVER_ERR_CUDA, std::string("capture: ") + cudaGetErrorString(e));
+  e = cudaGraphInstantiate(&ctx->gexec[parity], graph, 0);
+  cudaGraphDestroy(graph);
+  if (e != cudaSuccess) return fail(CLOVER_ERR_CUDA, std::string("instantiate: ") + cudaGetErrorString(e));
+  return CLOVER_OK;
+}
+
+int reflect_all(clover_ctx* ctx, const std::vector<int>& bufs) {
+  for (auto& cs : ctx->chunks)
+    for (int b : bufs) {
+      dim3 blk(32, 8);
+      dim3 grd((cs.c.nx + 2 + 2 * HALO + 31) / 32, (cs.c.ny + 2 + 2 * HALO + 7) / 8);
+      k_reflect<<<grd, blk, 0, ctx->work>>>(cs.c, cs.buf[b], kBufKind[b]);
+      LAUNCH_CHECK();
+    }
+  return exchange(ctx, bufs);
+}
+
+int check_err(clover_ctx* ctx) {
+  CK(cudaStreamSynchronize(ctx->work));
+  StepScalars h;
+  CK(cudaMemcpy(&h, ctx->scal, sizeof(h), cudaMemcpyDeviceToHost));
+  if (h.err) return fail(h.err, "small timestep: dt < dtmin");
+  return CLOVER_OK;
+}
+
+struct FieldMap { int buf; int nxe_add, nye_add; };
+
+int field_map(int fid, FieldMap* m) {
+  switch (fid) {
+    case CLOVER_F_DENSITY0: *m = {B_D0, 0, 0}; return 0;
+    case CLOVER_F_ENERGY0: *m = {B_E0, 0, 0}; return 0;
+    case CLOVER_F_PRESSURE: *m = {B_SCR, 0, 0}; return 0;
+    case CLOVER_F_SOUNDSPEED: *m = {B_SCR, 0, 0}; return 0;
+    case CLOVER_F_VISCOSITY: *m = {B_Q, 0, 0}; return 0;
+    case CLOVER_F_XVEL0: *m = {B_U0, 1, 1}; return 0;
+    case CLOVER_F_YVEL0: *m = {B_V0, 1, 1}; return 0;
+    case CLOVER_F_VOL_FLUX_X: *m = {B_FX, 1, 0}; return 0;
+    case CLOVER_F_VOL_FLUX_Y: *m = {B_FY, 0, 1}; return 0;
+    case CLOVER_F_MASS_FLUX_X: *m = {B_MX, 1, 0}; return 0;
+    case CLOVER_F_MASS_FLUX_Y: *m = {B_MY, 0, 1}; return 0;
+  }
+  return -1;
+}
+
+void kind_extra(int kind, int* ax, int* ay) {
+  *ax = (kind == K_XVEL || kind == K_YVEL || kind == K_XFACE) ? 1 : 0;
+  *ay = (kind == K_XVEL || kind == K_YVEL || kind == K_YFACE) ? 1 : 0;
+}
+
+// Gather buffer `buf` (global interior of its kind) into host.  Local chunks
+// only; multi-rank gathers are done by the caller through NCCL.
+int gather_local(clover_ctx* ctx, int buf, int kind, double* host, int64_t n) {
+  int ax, ay;
+  kind_extra(kind, &ax, &ay);
+  const int NXE = ctx->g.x_cells + ax, NYE = ctx->g.y_cells + ay;
+  if (n != (int64_t)NXE * NYE) return fail(CLOVER_ERR_ARG, "wrong element count for field");
+  for (auto& cs : ctx->chunks) {
+    const Chunk& c = cs.c;
+    // owned range incl. the shared last node/face only on the global edge
+    const int w = c.nx + ((c.gj0 + c.nx == ctx->g.x_cells) ? ax : 0);
+    const int h = c.ny + ((c.gk0 + c.ny == ctx->g.y_cells) ? ay : 0);
+    double* dst = host + (int64_t)c.gk0 * NXE + c.gj0;
+    const double* src = cs.buf[buf] + idx(c, 1, 1);
+    CK(cudaMemcpy2DAsync(dst, (size_t)NXE * 8, src, (size_t)c.pitch * 8, (size_t)w * 8, h,
+                         cudaMemcpyDeviceToHost, ctx->work));
+  }
+  CK(cudaStreamSynchronize(ctx->work));
+  return CLOVER_OK;
+}
+
+int scatter_local(clover_ctx* ctx, int buf, int kind, const double* host, int64_t n) {
+  int ax, ay;
+  kind_extra(kind, &ax, &ay);
+  const int NXE = ctx->g.x_cells + ax, NYE = ctx->g.y_cells + ay;
+  if (n != (int64_t)NXE * NYE) return fail(CLOVER_ERR_ARG, "wrong element count for field");
+  for (auto& cs : ctx->chunks) {
+    const Chunk& c = cs.c;
+    const int w = c.nx + ax, h = c.ny + ay;  // owned incl. the shared last node
+    const double* src = host + (int64_t)c.gk0 * NXE + c.gj0;
+    double* dst = cs.buf[buf] + idx(c, 1, 1);
+    CK(cudaMemcpy2DAsync(dst, (size_t)c.pitch * 8, src, (size_t)NXE * 8, (size_t)w * 8, h,
+                         cudaMemcpyHostToDevice, ctx->work));
+  }
+  return CLOVER_OK;
+}
+
+}  // namespace
+
+// ====================================================================== C ABI
+extern "C" {
+
+int clover_abi_version(void) { return CLOVER_ABI_VERSION; }
+
+const char* clover_last_error(void) { return g_last_error.c_str(); }
+
+const char* clover_error_string(int code) {
+  switch (code) {
+    case CLOVER_OK: return "ok";
+    case CLOVER_ERR_ARG: return "invalid argument";
+    case CLOVER_ERR_CUDA: return "CUDA error";
+    case CLOVER_ERR_NCCL: return "NCCL error";
+    case CLOVER_ERR_WORKSPACE: return "workspace too small or misaligned";
+    case CLOVER_ERR_SMALL_DT: return "small timestep (dt < dtmin)";
+    case CLOVER_ERR_STATE: return "invalid state";
+  }
+  return "unknown error";
+}
+
+int clover_workspace_bytes(const clover_grid* grid, const clover_dist* dist, int64_t* bytes) {
+  int px, py, rank, nranks;
+  int rc = validate(grid, dist, &px, &py, &rank, &nranks);
+  if (rc) return rc;
+  if (!bytes) return fail(CLOVER_ERR_ARG, "bytes is NULL");
+  *bytes = compute_workspace(grid, px, py, rank, nranks);
+  return CLOVER_OK;
+}
+
+int clover_nccl_unique_id(void* out128) {
+#ifdef CLOVER_WITH_NCCL
+  if (!out128) return fail(CLOVER_ERR_ARG, "out is NULL");
+  ncclUniqueId id;
+  NK(ncclGetUniqueId(&id));
+  static_assert(sizeof(ncclUniqueId) == 128, "ncclUniqueId size");
+  std::memcpy(out128, &id, 128);
+  return CLOVER_OK;
+#else
+  (void)out128;
+  return fail(CLOVER_ERR_NCCL, "libclover built without NCCL");
+#endif
+}
+
+int clover_init(const clover_grid* grid, const clover_state* states, int32_t nstates,
+                const clover_dist* dist, void* workspace, int64_t workspace_bytes,
+                void* cuda_stream, clover_ctx** out) {
+  if (!out) return fail(CLOVER_ERR_ARG, "out is NULL");
+  *out = nullptr;
+  int px, py, rank, nranks;
+  int rc = validate(grid, dist, &px, &py, &rank, &nranks);
+  if (rc) return rc;
+  if (!states || nstates < 1) return fail(CLOVER_ERR_ARG, "need at least one state");
+  if (nstates > MAX_STATES) return fail(CLOVER_ERR_ARG, "too many states");
+#ifndef CLOVER_WITH_NCCL
+  if (nranks > 1) return fail(CLOVER_ERR_NCCL, "libclover built without NCCL");
+#endif
+  const int64_t need = compute_workspace(grid, px, py, rank, nranks);
+  if (!workspace || workspace_bytes < need || ((uintptr_t)workspace % kAlign) != 0)
+    return fail(CLOVER_ERR_WORKSPACE, "workspace must be >= clover_workspace_bytes and 256-B aligned");
+
+  clover_ctx* ctx = new clover_ctx();
+  ctx->g = *grid;
+  fill_defaults(ctx->g);
+  ctx->states.assign(states, states + nstates);
+  ctx->rank = rank;
+  ctx->nranks = nranks;
+  ctx->L = decompose(grid->x_cells, grid->y_cells, px, py);
+  ctx->user = (cudaStream_t)cuda_stream;
+  ctx->ws_bytes = workspace_bytes;
+  ctx->advect_x = ctx->g.advect_x_first != 0;
+  ctx->dtp = DtParams{ctx->g.dtc_safe, ctx->g.dtu_safe, ctx->g.dtv_safe, ctx->g.dtdiv_safe,
+                      ctx->g.dtrise, ctx->g.dtmax, ctx->g.dtmin};
+  const double dx = (ctx->g.xmax - ctx->g.xmin) / (double)ctx->g.x_cells;
+  const double dy = (ctx->g.ymax - ctx->g.ymin) / (double)ctx->g.y_cells;
+  ctx->gg = GlobalGeom{ctx->g.x_cells, ctx->g.y_cells, ctx->g.xmin, ctx->g.ymin, dx, dy};
+
+  auto bail = [&](int code) { clover_finalize(ctx); return code; };
+  if (cudaStreamCreateWithFlags(&ctx->work, cudaStreamNonBlocking) != cudaSuccess ||
+      cudaEventCreateWithFlags(&ctx->ev_in, cudaEventDisableTiming) != cudaSuccess ||
+      cudaEventCreateWithFlags(&ctx->ev_out, cudaEventDisableTiming) != cudaSuccess)
+    return bail(fail(CLOVER_ERR_CUDA, "stream/event creation failed"));
+
+  // carve the workspace
+  char* p = (char*)workspace;
+  ctx->scal = (StepScalars*)p;
+  p += align_up(sizeof(StepScalars), kAlign);
+  ctx->hist = (double*)p;
+  p += align_up(DT_HIST * 8, kAlign);
+  ctx->owner.assign(px * py, 0);
+  for (int r = 0; r < nranks; ++r)
+    for (int id : local_chunk_ids(px, py, r, nranks)) ctx->owner[id] = r;
+  int64_t maxrows = 0, maxcols = 0;
+  for (int id : local_chunk_ids(px, py, rank, nranks)) {
+    ChunkState cs;
+    cs.id = id; cs.cx = id % px; cs.cy = id / px;
+    Chunk& c = cs.c;
+    c.nx = ctx->L.xs[cs.cx + 1] - ctx->L.xs[cs.cx];
+    c.ny = ctx->L.ys[cs.cy + 1] - ctx->L.ys[cs.cy];
+    c.gj0 = ctx->L.xs[cs.cx];
+    c.gk0 = ctx->L.ys[cs.cy];
+    const int64_t fe = field_elems(c.nx, c.ny, &c.pitch);
+    c.wl = cs.cx == 0; c.wr = cs.cx == px - 1; c.wb = cs.cy == 0; c.wt = cs.cy == py - 1;
+    c.face_cc = ctx->g.face_mirror == CLOVER_MIRROR_CELLCENTRE;
+    c.dx = dx; c.dy = dy; c.xmin = ctx->g.xmin; c.ymin = ctx->g.ymin;
+    for (int b = 0; b < NBUF; ++b) {
+      cs.buf[b] = (double*)p + (int64_t)ROW0 * c.pitch + COL0;
+      p += align_up(fe * 8, kAlign);
+    }
+    cs.ntx = (c.nx + ST - 1) / ST; cs.nty = (c.ny + ST - 1) / ST;
+    cs.partials = (double*)p;
+    p += align_up((int64_t)cs.ntx * cs.nty * 5 * 8, kAlign);
+    maxrows = std::max<int64_t>(maxrows, c.ny + 2 + 2 * HALO);
+    maxcols = std::max<int64_t>(maxcols, c.nx + 2 + 2 * HALO);
+    ctx->chunks.push_back(cs);
+  }
+  if (nranks > 1) {
+    int64_t line = std::max(maxrows, maxcols);
+    ctx->xbuf_elems = 4 * 6 * HALO * line;
+    ctx->xbuf_send = (double*)p;
+    p += align_up(ctx->xbuf_elems * 8, kAlign);
+    ctx->xbuf_recv = (double*)p;
+    p += align_up(ctx->xbuf_elems * 8, kAlign);
+  }
+#ifdef CLOVER_WITH_NCCL
+  if (nranks > 1) {
+    ncclUniqueId id;
+    std::memcpy(&id, dist->nccl_unique_id, sizeof(id));
+    if (ncclCommInitRank(&ctx->comm, nranks, id, rank) != ncclSuccess)
+      return bail(fail(CLOVER_ERR_NCCL, "ncclCommInitRank failed"));
+  }
+#endif
+
+  if (join_in(ctx)) return bail(CLOVER_ERR_CUDA);
+  // zero every buffer (halo corners of unused kinds stay deterministic)
+  if (cudaMemsetAsync(workspace, 0, (size_t)need, ctx->work) != cudaSuccess)
+    return bail(fail(CLOVER_ERR_CUDA, "memset failed"));
+  StepScalars h{};
+  h.dt_slot = (unsigned long long)0;
+  {
+    double big = G_BIG;
+    std::memcpy(&h.dt_slot, &big, 8);
+  }
+  h.dt = ctx->g.dtinit;
+  h.dtold = ctx->g.dtinit;
+  h.time = 0.0;
+  h.step = 0;
+  h.err = 0;
+  if (cudaMemcpyAsync(ctx->scal, &h, sizeof(h), cudaMemcpyHostToDevice, ctx->work) != cudaSuccess)
+    return bail(fail(CLOVER_ERR_CUDA, "scalar upload failed"));
+
+  // states: rectangle edges nudged by dx/100 (reading A6), same expression as
+  // the reference's read_input.
+  StateList sl{};
+  sl.n = nstates;
+  for (int s = 0; s < nstates; ++s) {
+    const clover_state& in = states[s];
+    DevState& d = sl.s[s];
+    d.density = in.density; d.energy = in.energy; d.xvel = in.xvel; d.yvel = in.yvel;
+    d.geometry = in.geometry; d.xmin = in.xmin; d.xmax = in.xmax; d.ymin = in.ymin;
+    d.ymax = in.ymax; d.radius = in.radius;
+    if (s >= 1 && in.geometry == CLOVER_GEOM_RECT) {
+      d.xmin = d.xmin + (dx / 100.0);
+      d.ymin = d.ymin + (dy / 100.0);
+      d.xmax = d.xmax - (dx / 100.0);
+      d.ymax = d.ymax - (dy / 100.0);
+    }
+    if (s >= 1 && (in.geometry < 1 || in.geometry > 3))
+      return bail(fail(CLOVER_ERR_ARG, "state geometry must be 1, 2 or 3"));
+  }
+  for (auto& cs : ctx->chunks) {
+    dim3 blk(32, 8);
+    dim3 grd((cs.c.nx + 2 + 2 * HALO + 31) / 32, (cs.c.ny + 2 + 2 * HALO + 7) / 8);
+    k_generate<<<grd, blk, 0, ctx->work>>>(cs.c, ctx->gg, sl, cs.buf[B_D0], cs.buf[B_E0],
+                                             cs.buf[B_U0], cs.buf[B_V0]);
+    if (cudaGetLastError() != cudaSuccess) return bail(fail(CLOVER_ERR_CUDA, "k_generate launch"));
+  }
+  rc = reflect_all(ctx, {B_D0, B_E0, B_U0, B_V0});
+  if (rc) return bail(rc);
+  if (join_out(ctx)) return bail(CLOVER_ERR_CUDA);
+  *out = ctx;
+  return CLOVER_OK;
+}
+
+int clover_set_graphs(clover_ctx* ctx, int32_t enable) {
+  if (!ctx) return fail(CLOVER_ERR_ARG, "ctx is NULL");
+  ctx->use_graphs = enable != 0;
+  return CLOVER_OK;
+}
+
+int clover_kernels_per_step(clover_ctx* ctx, int32_t* out) {
+  if (!ctx || !out) return fail(CLOVER_ERR_ARG, "NULL argument");
+  *out = (int32_t)(ctx->chunks.size() * 6 + 1);
+  return CLOVER_OK;
+}
+
+int clover_step(clover_ctx* ctx, int32_t nsteps) {
+  if (!ctx) return fail(CLOVER_ERR_ARG, "ctx is NULL");
+  if (nsteps < 0) return fail(CLOVER_ERR_ARG, "nsteps < 0");
+  if (nsteps == 0) return CLOVER_OK;
+  int rc = join_in(ctx);
+  if (rc) return rc;
+  for (int i = 0; i < nsteps; ++i) {
+    const int parity = ctx->advect_x ? 0 : 1;
+    if (ctx->use_graphs) {
+      if (!ctx->gexec[parity]) {
+        rc = build_graph(ctx, parity);
+        if (rc) return rc;
+      }
+      CK(cudaGraphLaunch(ctx->gexec[parity], ctx->work));
+    } else {
+      rc = enqueue_step(ctx, ctx->advect_x, 7);
+      if (rc) return rc;
+    }
+    ctx->advect_x = !ctx->advect_x;
+  }
+  return join_out(ctx);
+}
+
+int clover_profile_steps(clover_ctx* ctx, int32_t nsteps, double* ms_out, int64_t* launches_out,
+                         int32_t nslots) {
+  if (!ctx || !ms_out || !launches_out || nslots < NPROF || nsteps < 0)
+    return fail(CLOVER_ERR_ARG, "bad arguments");
+  for (int i = 0; i < NPROF; ++i) { ms_out[i] = 0.0; launches_out[i] = 0; }
+  int rc = join_in(ctx);
+  if (rc) return rc;
+  ctx->prof = true;
+  for (int s = 0; s < nsteps && !rc; ++s) {
+    rc = enqueue_step(ctx, ctx->advect_x, 7);
+    ctx->advect_x = !ctx->advect_x;
+  }
+  ctx->prof = false;
+  cudaError_t e = cudaStreamSynchronize(ctx->work);
+  for (size_t i = 1; i < ctx->prof_events.size(); ++i) {
+    int id = ctx->prof_events[i].first;
+    if (id < 0) continue;
+    float ms = 0.f;
+    cudaEventElapsedTime(&ms, ctx->prof_events[i - 1].second, ctx->prof_events[i].second);
+    ms_out[id] += ms;
+    launches_out[id] += 1;
+  }
+  for (auto& pe : ctx->prof_events) cudaEventDestroy(pe.second);
+  ctx->prof_events.clear();
+  if (rc) return rc;
+  if (e != cudaSuccess) return fail(CLOVER_ERR_CUDA, cudaGetErrorString(e));
+  rc = check_err(ctx);
+  if (rc) return rc;
+  return join_out(ctx);
+}
+
+const char* clover_profile_name(int32_t i) { return (i >= 0 && i < NPROF) ? kProfNames[i] : ""; }
+
+int clover_debug_partial_step(clover_ctx* ctx, int32_t nkernels) {
+  if (!ctx) return fail(CLOVER_ERR_ARG, "ctx is NULL");
+  int rc = join_in(ctx);
+  if (rc) return rc;
+  rc = enqueue_step(ctx, ctx->advect_x, nkernels);
+  if (rc) return rc;
+  return join_out(ctx);
+}
+
+int clover_sync(clover_ctx* ctx) {
+  if (!ctx) return fail(CLOVER_ERR_ARG, "ctx is NULL");
+  return check_err(ctx);
+}
+
+int clover_get_clock(clover_ctx* ctx, int32_t* step, double* time, double* dt_last) {
+  if (!ctx) return fail(CLOVER_ERR_ARG, "ctx is NULL");
+  int rc = check_err(ctx);
+  StepScalars h;
+  CK(cudaMemcpy(&h, ctx->scal, sizeof(h), cudaMemcpyDeviceToHost));
+  if (step) *step = h.step;
+  if (time) *time = h.time;
+  if (dt_last) *dt_last = h.dt;
+  return rc;
+}
+
+int clover_dt_history(clover_ctx* ctx, int32_t first, int32_t n, double* host_out) {
+  if (!ctx || !host_out || n < 0 || first < 1) return fail(CLOVER_ERR_ARG, "bad arguments");
+  CK(cudaStreamSynchronize(ctx->work));
+  StepScalars h;
+  CK(cudaMemcpy(&h, ctx->scal, sizeof(h), cudaMemcpyDeviceToHost));
+  if (first + n - 1 > h.step || h.step - first >= DT_HIST) return fail(CLOVER_ERR_ARG, "steps outside the kept history");
+  std::vector<double> all(DT_HIST);
+  CK(cudaMemcpy(all.data(), ctx->hist, DT_HIST * 8, cudaMemcpyDeviceToHost));
+  for (int i = 0; i < n; ++i) host_out[i] = all[(first - 1 + i) % DT_HIST];
+  return CLOVER_OK;
+}
+
+int clover_field_summary(clover_ctx* ctx, clover_summary* out) {
+  if (!ctx || !out) return fail(CLOVER_ERR_ARG, "NULL argument");
+  int rc = join_in(ctx);
+  if (rc) return rc;
+  for (auto& cs : ctx->chunks) {
+    k_summary<<<dim3(cs.ntx, cs.nty), dim3(ST, ST), 0, ctx->work>>>(
+        cs.c, cs.buf[B_D0], cs.buf[B_E0], cs.buf[B_U0], cs.buf[B_V0], cs.partials);
+    LAUNCH_CHECK();
+  }
+  // global tile grid (tiles aligned at global cell 1 when tile_aligned)
+  const int GTX = (ctx->g.x_cells + ST - 1) / ST, GTY = (ctx->g.y_cells + ST - 1) / ST;
+  std::vector<double> all;
+  std::vector<std::vector<double>> per(ctx->chunks.size());
+  for (size_t i = 0; i < ctx->chunks.size(); ++i) {
+    auto& cs = ctx->chunks[i];
+    per[i].resize((size_t)cs.ntx * cs.nty * 5);
+    CK(cudaMemcpyAsync(per[i].data(), cs.partials, per[i].size() * 8, cudaMemcpyDeviceToHost, ctx->work));
+  }
+  rc = check_err(ctx);
+  double acc[5] = {0, 0, 0, 0, 0};
+  if (ctx->L.tile_aligned && ctx->nranks == 1) {
+    all.assign((size_t)GTX * GTY * 5, 0.0);
+    for (size_t i = 0; i < ctx->chunks.size(); ++i) {
+      auto& cs = ctx->chunks[i];
+      const int tx0 = cs.c.gj0 / ST, ty0 = cs.c.gk0 / ST;
+      for (int ty = 0; ty < cs.nty; ++ty)
+        for (int tx = 0; tx < cs.ntx; ++tx)
+          for (int q = 0; q < 5; ++q)
+            all[((size_t)(ty0 + ty) * GTX + (tx0 + tx)) * 5 + q] = per[i][((size_t)ty * cs.ntx + tx) * 5 + q];
+    }
+    for (size_t t = 0; t < (size_t)GTX * GTY; ++t)
+      for (int q = 0; q < 5; ++q) acc[q] = acc[q] + all[t * 5 + q];
+  } else {
+    for (auto& v : per)
+      for (size_t t = 0; t < v.size() / 5; ++t)
+        for (int q = 0; q < 5; ++q) acc[q] = acc[q] + v[t * 5 + q];
+  }
+#ifdef CLOVER_WITH_NCCL
+  if (ctx->nranks > 1) {
+    // deterministic across ranks: gather per-rank totals, sum in rank order
+    double* dsend = ctx->xbuf_send;
+    double* drecv = ctx->xbuf_recv;
+    CK(cudaMemcpyAsync(dsend, acc, 5 * 8, cudaMemcpyHostToDevice, ctx->work));
+    NK(ncclAllGather(dsend, drecv, 5, ncclFloat64, ctx->comm, ctx->work));
+    std::vector<double> g((size_t)ctx->nranks * 5);
+    CK(cudaMemcpyAsync(g.data(), drecv, g.size() * 8, cudaMemcpyDeviceToHost, ctx->work));
+    CK(cudaStreamSynchronize(ctx->work));
+    for (int q = 0; q < 5; ++q) acc[q] = 0.0;
+    for (int r = 0; r < ctx->nranks; ++r)
+      for (int q = 0; q < 5; ++q) acc[q] = acc[q] + g[(size_t)r * 5 + q];
+  }
+#endif
+  out->vol = acc[0]; out->mass = acc[1]; out->ie = acc[2]; out->ke = acc[3]; out->press = acc[4];
+  int rc2 = join_out(ctx);
+  return rc ? rc : rc2;
+}
+
+int clover_read_field(clover_ctx* ctx, int32_t field_id, double* host, int64_t n) {
+  if (!ctx || !host) return fail(CLOVER_ERR_ARG, "NULL argument");
+  FieldMap m;
+  if (field_map(field_id, &m)) return fail(CLOVER_ERR_ARG, "unknown field id");
+  if (ctx->nranks > 1) return fail(CLOVER_ERR_STATE, "clover_read_field: multi-rank gather not supported yet");
+  int rc = join_in(ctx);
+  if (rc) return rc;
+  if (field_id == CLOVER_F_PRESSURE || field_id == CLOVER_F_SOUNDSPEED) {
+    for (auto& cs : ctx->chunks) {
+      k_eos_field<<<cell_grid(cs.c, 32, 8), dim3(32, 8), 0, ctx->work>>>(
+          cs.c, cs.buf[B_D0], cs.buf[B_E0], cs.buf[B_SCR], field_id == CLOVER_F_SOUNDSPEED);
+      LAUNCH_CHECK();
+    }
+  }
+  rc = gather_local(ctx, m.buf, kBufKind[m.buf], host, n);
+  if (rc) return rc;
+  return check_err(ctx);
+}
+
+int clover_debug_read_buffer(clover_ctx* ctx, int32_t buffer_id, int32_t kind, double* host, int64_t n) {
+  if (!ctx || !host) return fail(CLOVER_ERR_ARG, "NULL argument");
+  if (buffer_id < 0 || buffer_id >= NBUF) return fail(CLOVER_ERR_ARG, "bad buffer id");
+  if (kind < 0 || kind > 4) return fail(CLOVER_ERR_ARG, "bad kind");
+  if (ctx->nranks > 1) return fail(CLOVER_ERR_STATE, "multi-rank debug read not supported");
+  int rc = join_in(ctx);
+  if (rc) return rc;
+  return gather_local(ctx, buffer_id, kind, host, n);
+}
+
+int clover_write_field(clover_ctx* ctx, int32_t field_id, const double* host, int64_t n) {
+  if (!ctx || !host) return fail(CLOVER_ERR_ARG, "NULL argument");
+  int buf;
+  switch (field_id) {
+    case CLOVER_F_DENSITY0: buf = B_D0; break;
+    case CLOVER_F_ENERGY0: buf = B_E0; break;
+    case CLOVER_F_XVEL0: buf = B_U0; break;
+    case CLOVER_F_YVEL0: buf = B_V0; break;
+    default: return fail(CLOVER_ERR_ARG, "only density0, energy0, xvel0, yvel0 are writable");
+  }
+  if (ctx->nranks > 1) return fail(CLOVER_ERR_STATE, "clover_write_field: multi-rank scatter not supported yet");
+  int rc = join_in(ctx);
+  if (rc) return rc;
+  rc = scatter_local(ctx, buf, kBufKind[buf], host, n);
+  if (rc) return rc;
+  rc = reflect_all(ctx, {buf});
+  if (rc) return rc;
+  CK(cudaStreamSynchronize(ctx->work));
+  return join_out(ctx);
+}
+
+int clover_step_host(clover_ctx* ctx, int32_t nsteps, const double* d_in, const double* e_in,
+                     const double* u_in, const double* v_in, double* d_out, double* e_out,
+                     double* u_out, double* v_out) {
+  if (!ctx) return fail(CLOVER_ERR_ARG, "ctx is NULL");
+  if (ctx->chunks.size() != 1 || ctx->nranks != 1) return fail(CLOVER_ERR_STATE, "clover_step_host needs a single-chunk context");
+  const int64_t nc = (int64_t)ctx->g.x_cells * ctx->g.y_cells;
+  const int64_t nn = (int64_t)(ctx->g.x_cells + 1) * (ctx->g.y_cells + 1);
+  int rc = join_in(ctx);
+  if (rc) return rc;
+  const double* ins[4] = {d_in, e_in, u_in, v_in};
+  const int bufs[4] = {B_D0, B_E0, B_U0, B_V0};
+  for (int f = 0; f < 4; ++f)
+    if (ins[f]) {
+      rc = scatter_local(ctx, bufs[f], kBufKind[bufs[f]], ins[f], f < 2 ? nc : nn);
+      if (rc) return rc;
+    }
+  rc = reflect_all(ctx, {B_D0, B_E0, B_U0, B_V0});
+  if (rc) return rc;
+  rc = join_out(ctx);
+  if (rc) return rc;
+  rc = clover_step(ctx, nsteps);
+  if (rc) return rc;
+  rc = join_in(ctx);
+  if (rc) return rc;
+  double* outs[4] = {d_out, e_out, u_out, v_out};
+  for (int f = 0; f < 4; ++f)
+    if (outs[f]) {
+      rc = gather_local(ctx, bufs[f], kBufKind[bufs[f]], outs[f], f < 2 ? nc : nn);
+      if (rc) return rc;
+    }
+  return check_err(ctx);
+}
+
+int clover_finalize(clover_ctx* ctx) {
+  if (!ctx) return CLOVER_OK;
+  int rc = CLOVER_OK;
+  if (ctx->work) {
+    rc = check_err(ctx);
+  }
+  for (int i = 0; i < 2; ++i)
+    if (ctx->gexec[i]) cudaGraphExecDestroy(ctx->gexec[i]);
+#ifdef CLOVER_WITH_NCCL
+  if (ctx->comm) ncclCommDestroy(ctx->comm);
+#endif
+  if (ctx->ev_in) cudaEventDestroy(ctx->ev_in);
+  if (ctx->ev_out) cudaEventDestroy(ctx->ev_out);
+  if (ctx->work) cudaStreamDestroy(ctx->work);
+  delete ctx;
+  return rc;
+}
+
+}  // extern "C"

@@ -1,0 +1,258 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle on the
+same seeded inputs.  Bar: bitwise for fields and
+the dt history (both sides are IEEE fp64 with no contraction, reading A8);
+north_star tolerances as the fallback gate: field_summary totals 1e-10
+relative, per-cell 1e-9 (A14 metric).
+"""
+from __future__ import annotations
+
+import numpy as np
+import pytest
+
+from oracle import Oracle
+from workloads import (bm_deck, contact_deck, fuzz_deck, quiescent_deck, random_state_fields,
+                       symmetric_deck)
+
+pytestmark = pytest.mark.gpu
+
+STATE = ("density0", "energy0", "xvel0", "yvel0")
+SUMMARY_TOL = 1e-10
+CELL_TOL = 1e-9
+
+
+@pytest.fixture(scope="module")
+def torch_cuda():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    return torch
+
+
+def make_gpu(deck, **kw):
+    from paper_conf_cluster_regulymg15_b200 import Clover
+    return Clover(deck, **kw)
+
+
+def rel_cell(a, b):
+    """A14: abs(a-b) <= tol*max(|a|,|b|,s_f), s_f = 1e-12*max|f|."""
+    s = 1e-12 * max(np.abs(a).max(), np.abs(b).max(), 1e-300)
+    den = np.maximum(np.maximum(np.abs(a), np.abs(b)), s)
+    return float((np.abs(a - b) / den).max())
+
+
+def assert_fields_equal(gpu, ora, names=STATE, bitwise=True, ctx=""):
+    for f in names:
+        a, b = gpu.read(f), ora.read(f)
+        assert a.shape == b.shape
+        if bitwise:
+            if not np.array_equal(a, b):
+                bad = np.argwhere(a != b)
+                k, j = bad[0]
+                raise AssertionError(f"{ctx} {f}: {len(bad)} differ, first (k={k + 1}, j={j + 1}) "
+                                     f"gpu={a[k, j]!r} oracle={b[k, j]!r} rel={rel_cell(a, b):.3e}")
+        assert rel_cell(a, b) <= CELL_TOL, (ctx, f)
+
+
+def assert_summary_close(gs, os_):
+    for key in ("vol", "mass", "ie", "ke", "press"):
+        a, b = gs[key], os_[key]
+        if b == 0.0:
+            assert a == 0.0, key
+        else:
+            assert abs(a - b) / abs(b) <= SUMMARY_TOL, (key, a, b)
+
+
+def test_init_matches_oracle(torch_cuda):
+    for deck in (bm_deck(64), fuzz_deck(1), fuzz_deck(4)):
+        g, o = make_gpu(deck), Oracle(deck)
+        assert_fields_equal(g, o)
+        assert_summary_close(g.field_summary(), o.field_summary())
+        for f in ("pressure", "soundspeed"):
+            assert np.array_equal(g.read(f), o.read(f)), f
+
+
+def test_stage_parity_bm64(torch_cuda):
+    """Kernel-by-kernel parity on step 1 and 2 of bm64 (x-first then y-first)."""
+    deck = bm_deck(64)
+    deck["max_timestep"] = 1.0
+    for step in range(2):
+        g, o = make_gpu(deck), Oracle(deck)
+        if step:
+            g.step(1); o.step(1)
+        g.debug_partial_step(1)
+        o.run_stage("timestep")
+        assert np.array_equal(g.debug_read("q", "cell"), o.read("viscosity"))
+        g2 = make_gpu(deck)
+        if step:
+            g2.step(1)
+        g2.debug_partial_step(3)
+        o.run_stage("pdv_predict"); o.run_stage("accelerate"); o.run_stage("pdv_correct")
+        o.run_stage("flux_calc")
+        for buf, kind, name in (("d1", "cell", "density1"), ("e1", "cell", "energy1"),
+                                ("u1", "xvel", "xvel1"), ("v1", "yvel", "yvel1"),
+                                ("fx", "xface", "vol_flux_x"), ("fy", "yface", "vol_flux_y")):
+            a, b = g2.debug_read(buf, kind), o.read(name)
+            assert np.array_equal(a, b), (step, name, rel_cell(a, b))
+        g3 = make_gpu(deck)
+        if step:
+            g3.step(1)
+        g3.debug_partial_step(4)
+        o.run_stage("adv_cell1")
+        mname = "mass_flux_x" if step == 0 else "mass_flux_y"
+        mkind = "xface" if step == 0 else "yface"
+        mbuf = "mx" if step == 0 else "my"
+        for buf, kind, name in (("d2", "cell", "density1"), ("e2", "cell", "energy1"),
+                                (mbuf, mkind, mname)):
+            a, b = g3.debug_read(buf, kind), o.read(name)
+            assert np.array_equal(a, b), (step, name, rel_cell(a, b))
+
+
+def test_bm64_20_steps_bitwise(torch_cuda):
+    deck = bm_deck(64, end_step=20)
+    g, o = make_gpu(deck), Oracle(deck)
+    g.step(20)
+    dts = o.step(20)
+    assert np.array_equal(g.dt_history(1, 20), dts)
+    assert_fields_equal(g, o, ctx="bm64")
+    assert_summary_close(g.field_summary(), o.field_summary())
+    c = g.clock()
+    assert c["step"] == 20 and c["time"] == o.clock()["time"]
+
+
+@pytest.mark.parametrize("mirror", [0, 1])
+@pytest.mark.parametrize("seed", [0, 1, 2, 3, 4, 5])
+def test_fuzz_decks_bitwise(torch_cuda, seed, mirror):
+    deck = fuzz_deck(seed)
+    deck["face_mirror"] = mirror
+    g, o = make_gpu(deck), Oracle(deck)
+    g.step(10)
+    dts = o.step(10)
+    assert np.array_equal(g.dt_history(1, 10), dts)
+    assert_fields_equal(g, o, ctx=f"fuzz{seed}/m{mirror}")
+    assert_summary_close(g.field_summary(), o.field_summary())
+
+
+@pytest.mark.parametrize("shape", [(4, 4), (5, 7), (33, 9), (65, 47), (31, 40), (96, 17)])
+def test_ragged_meshes_bitwise(torch_cuda, shape):
+    nx, ny = shape
+    deck = fuzz_deck(11, nx=nx, ny=ny)
+    g, o = make_gpu(deck), Oracle(deck)
+    g.step(6)
+    dts = o.step(6)
+    assert np.array_equal(g.dt_history(1, 6), dts)
+    assert_fields_equal(g, o, ctx=str(shape))
+
+
+@pytest.mark.parametrize("smooth", [False, True])
+def test_random_state_bitwise(torch_cuda, smooth):
+    nx, ny = 70, 50
+    deck = bm_deck(nx, ny)
+    deck["max_timestep"] = 1.0
+    fields = random_state_fields(5, nx, ny, smooth=smooth)
+    g, o = make_gpu(deck), Oracle(deck)
+    g.load_state(fields)
+    o.load_state(fields)
+    assert_fields_equal(g, o, ctx="loaded")
+    g.step(4)
+    dts = o.step(4)
+    assert np.array_equal(g.dt_history(1, 4), dts)
+    assert_fields_equal(g, o, ctx="random")
+    assert np.array_equal(g.read("viscosity"), o.read("viscosity"))
+
+
+def test_invariant_decks(torch_cuda):
+    for deck in (quiescent_deck(64), contact_deck(64), symmetric_deck(64)):
+        g, o = make_gpu(deck), Oracle(deck)
+        g.step(20)
+        o.step(20)
+        assert_fields_equal(g, o)
+
+
+@pytest.mark.parametrize("pxy", [(2, 1), (1, 2), (2, 2), (3, 2), (1, 4)])
+def test_local_chunk_decomposition_bitwise(torch_cuda, pxy):
+    """px*py chunks on one GPU (device-to-device halo exchange) give the same
+    bits as one chunk and as the oracle, including the summary."""
+    deck = bm_deck(96, 80)
+    deck["max_timestep"] = 1.0
+    one = make_gpu(deck)
+    many = make_gpu(deck, px=pxy[0], py=pxy[1])
+    o = Oracle(deck)
+    one.step(12)
+    many.step(12)
+    o.step(12)
+    for f in STATE:
+        assert np.array_equal(many.read(f), one.read(f)), f
+    assert_fields_equal(many, o)
+    assert many.field_summary() == one.field_summary()
+
+
+def test_local_chunks_fuzz(torch_cuda):
+    deck = fuzz_deck(8, nx=64, ny=48)
+    one, many = make_gpu(deck), make_gpu(deck, px=2, py=3)
+    one.step(8)
+    many.step(8)
+    for f in STATE:
+        assert np.array_equal(many.read(f), one.read(f)), f
+
+
+def test_graphs_on_off_identical(torch_cuda):
+    deck = fuzz_deck(2)
+    a, b = make_gpu(deck), make_gpu(deck)
+    b.set_graphs(False)
+    a.step(7)
+    b.step(7)
+    for f in STATE:
+        assert np.array_equal(a.read(f), b.read(f))
+
+
+def test_step_host_matches_device_path(torch_cuda):
+    nx = ny = 48
+    deck = bm_deck(nx, ny)
+    f = random_state_fields(3, nx, ny, smooth=True)
+    a = make_gpu(deck)
+    outs = {k: np.empty_like(v) for k, v in f.items()}
+    a.step_host(3, f, outs)
+    o = Oracle(deck)
+    o.load_state(f)
+    o.step(3)
+    for k in STATE:
+        assert np.array_equal(outs[k], o.read(k)), k
+
+
+def test_small_dt_error_is_latched(torch_cuda):
+    from paper_conf_cluster_regulymg15_b200 import CloverError
+    deck = bm_deck(32)
+    deck["dtmin"] = 0.5  # every dt is smaller than this
+    g = make_gpu(deck)
+    g.step(1)
+    with pytest.raises(CloverError) as ei:
+        g.sync()
+    assert ei.value.code == -5
+
+
+def test_c2_960_87_steps(torch_cuda):
+    """configs[1]: clover_bm_short shape, full run; also the QA constant."""
+    deck = bm_deck(960, end_step=87)
+    g, o = make_gpu(deck), Oracle(deck)
+    g.step(87)
+    dts = o.step(87)
+    assert np.array_equal(g.dt_history(1, 87), dts)
+    gs, os_ = g.field_summary(), o.field_summary()
+    assert_summary_close(gs, os_)
+    assert abs(100.0 * gs["ke"] / 1.19316898756307 - 100.0) < 0.001
+    assert_fields_equal(g, o, ctx="C2")
+
+
+@pytest.mark.parametrize("n", [3840])
+def test_full_size_first_steps(torch_cuda, n):
+    """configs[2] size in the bench's launch configuration: full-field
+    comparison over the first 2 steps (the oracle needs ~3 s per step)."""
+    deck = bm_deck(n, end_step=300)
+    g, o = make_gpu(deck), Oracle(deck)
+    g.step(2)
+    dts = o.step(2)
+    assert np.array_equal(g.dt_history(1, 2), dts)
+    assert_fields_equal(g, o, ctx=f"{n}")
+    # the sequential oracle sum carries up to n*eps (3e-9) of its own
+    # rounding at this size; compare with its compensated twin
+    assert_summary_close(g.field_summary(), o.field_summary(compensated=True))

@@ -333,3 +333,17 @@ def test_random_state_roundtrip():
     o.load_state(f)
     for k, v in f.items():
         assert np.array_equal(o.read(k), v)
+
+
+def test_compensated_summary_is_exact_on_dyadic_mesh_and_close_elsewhere():
+    """Both summations of c.12: bitwise equal where every term and partial
+    sum is exact (64^2 bm, dyadic); within the sequential bound n*eps on
+    960^2, where the compensated sum also matches the closed form closer."""
+    o = Oracle(bm_deck(64))
+    assert o.field_summary() == o.field_summary(compensated=True)
+    o = Oracle(bm_deck(960))
+    a, b = o.field_summary(), o.field_summary(compensated=True)
+    for k in a:
+        if b[k]:
+            assert _rel(a[k], b[k]) < 960 * 960 * 2.3e-16
+    assert _rel(b["vol"], 100.0) < 1e-14 < _rel(a["vol"], 100.0)
