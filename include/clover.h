@@ -199,6 +199,13 @@ int clover_debug_partial_step(clover_ctx* ctx, int32_t nkernels);
 int clover_debug_read_buffer(clover_ctx* ctx, int32_t buffer_id, int32_t kind,
                              double* host, int64_t n);
 
+/* Test: compare the library's internal fp64 division (div_rn) with IEEE
+ * a/b bit for bit on n random operand pairs (exponents in [-emax, emax],
+ * 1/16 zero numerators); *mismatches receives the count, example_ab (may be
+ * NULL) the first mismatching pair.  Uses the current CUDA device. */
+int clover_debug_div_check(int64_t n, uint64_t seed, int32_t emax, int64_t* mismatches,
+                           double* example_ab);
+
 /* Destroy the context (does not free the caller's workspace). */
 int clover_finalize(clover_ctx* ctx);
 

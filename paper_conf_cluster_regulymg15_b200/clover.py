@@ -38,7 +38,7 @@ EXPORTS = ["clover_workspace_bytes", "clover_nccl_unique_id", "clover_init", "cl
            "clover_step_host", "clover_field_summary", "clover_get_clock", "clover_dt_history",
            "clover_read_field", "clover_write_field", "clover_sync", "clover_set_graphs",
            "clover_kernels_per_step", "clover_debug_partial_step", "clover_debug_read_buffer",
-           "clover_profile_steps", "clover_profile_name", "clover_finalize", "clover_error_string", "clover_last_error", "clover_abi_version"]
+           "clover_profile_steps", "clover_profile_name", "clover_debug_div_check", "clover_finalize", "clover_error_string", "clover_last_error", "clover_abi_version"]
 
 
 class CloverGrid(ctypes.Structure):
@@ -102,6 +102,7 @@ def load(build_if_missing: bool = True):
     L.clover_profile_steps.argtypes = [c_void_p, c_int32, dptr, ctypes.POINTER(c_int64), c_int32]
     L.clover_profile_name.argtypes = [c_int32]
     L.clover_profile_name.restype = ctypes.c_char_p
+    L.clover_debug_div_check.argtypes = [c_int64, ctypes.c_uint64, c_int32, ctypes.POINTER(c_int64), dptr]
     L.clover_finalize.argtypes = [c_void_p]
     L.clover_error_string.argtypes = [c_int32]
     L.clover_error_string.restype = ctypes.c_char_p
@@ -163,6 +164,15 @@ def field_shape(name_or_kind: str, nx: int, ny: int):
     if k in ("vol_flux_y", "mass_flux_y", "yface"):
         return (ny + 1, nx)
     return (ny, nx)
+
+
+def debug_div_check(n: int, seed: int = 1, emax: int = 60):
+    """Bitwise check of the library's fp64 division against IEEE a/b."""
+    bad = c_int64()
+    ex = np.zeros(2, dtype=np.float64)
+    _check(load().clover_debug_div_check(n, seed, emax, ctypes.byref(bad), ex.ctypes.data_as(dptr)),
+           "clover_debug_div_check")
+    return bad.value, (float(ex[0]), float(ex[1]))
 
 
 class Clover:

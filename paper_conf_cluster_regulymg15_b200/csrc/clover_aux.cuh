@@ -69,7 +69,7 @@ __global__ void k_generate(Chunk c, GlobalGeom g, StateList sl, double* __restri
   const int k = blockIdx.y * blockDim.y + threadIdx.y - HALO;
   if (j > c.nx + 1 + HALO || k > c.ny + 1 + HALO) return;
   const int gj = c.gj0 + j, gk = c.gk0 + k;
-  const int64_t i = idx(c, j, k);
+  const int i = idx(c, j, k);
   if (gj >= 1 && gj <= g.NX && gk >= 1 && gk <= g.NY && j <= c.nx + HALO && k <= c.ny + HALO) {
     const int s = cell_state(g, sl, gj, gk);
     d0[i] = sl.s[s].density;
@@ -121,8 +121,8 @@ __global__ void k_eos_field(Chunk c, const double* __restrict__ d0, const double
   const int j = blockIdx.x * blockDim.x + threadIdx.x + 1;
   const int k = blockIdx.y * blockDim.y + threadIdx.y + 1;
   if (j > c.nx || k > c.ny) return;
-  const int64_t i = idx(c, j, k);
-  out[i] = soundspeed ? eos_soundspeed(d0[i], e0[i]) : eos_pressure(d0[i], e0[i]);
+  const int i = idx(c, j, k);
+  out[i] = soundspeed ? eos_soundspeed_ieee(d0[i], e0[i]) : eos_pressure(d0[i], e0[i]);
 }
 
 // field_summary (c.12): one 16x16 tile of cells per CTA; per-cell terms
@@ -138,8 +138,8 @@ k_summary(Chunk c, const double* __restrict__ d0, const double* __restrict__ e0,
   const int t = threadIdx.y * ST + threadIdx.x;
   double a0 = 0.0, a1 = 0.0, a2 = 0.0, a3 = 0.0, a4 = 0.0;
   if (j <= c.nx && k <= c.ny) {
-    const int64_t i = idx(c, j, k);
-    const int64_t P = c.pitch;
+    const int i = idx(c, j, k);
+    const int P = c.pitch;
     double vsqrd = 0.0;
     vsqrd = vsqrd + 0.25 * (u0[i] * u0[i] + v0[i] * v0[i]);
     vsqrd = vsqrd + 0.25 * (u0[i + 1] * u0[i + 1] + v0[i + 1] * v0[i + 1]);

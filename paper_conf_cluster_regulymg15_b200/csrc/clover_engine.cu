@@ -166,6 +166,10 @@ int validate(const clover_grid* g, const clover_dist* d, int* px, int* py, int* 
   }
   Layout L = decompose(g->x_cells, g->y_cells, *px, *py);
   for (int i = 0; i < *px; ++i)
+    for (int jj = 0; jj < *py; ++jj)
+      if (field_elems(L.xs[i + 1] - L.xs[i], L.ys[jj + 1] - L.ys[jj], nullptr) >= (int64_t)1 << 31)
+        return fail(CLOVER_ERR_ARG, "a chunk field exceeds 2^31 elements: use more chunks");
+  for (int i = 0; i < *px; ++i)
     if (L.xs[i + 1] - L.xs[i] < 4) return fail(CLOVER_ERR_ARG, "every chunk needs >= 4 cells in x");
   for (int i = 0; i < *py; ++i)
     if (L.ys[i + 1] - L.ys[i] < 4) return fail(CLOVER_ERR_ARG, "every chunk needs >= 4 cells in y");
@@ -821,6 +825,65 @@ int clover_profile_steps(clover_ctx* ctx, int32_t nsteps, double* ms_out, int64_
   rc = check_err(ctx);
   if (rc) return rc;
   return join_out(ctx);
+}
+
+// Self-check of div_rn (clover_common.cuh) against IEEE a/b on random
+// operands: exponents in [-emax, emax], random signs and mantissas, one
+// numerator in 16 is +-0.  Counts bitwise mismatches.
+__device__ __forceinline__ unsigned long long splitmix(unsigned long long x) {
+  x += 0x9E3779B97F4A7C15ull;
+  x = (x ^ (x >> 30)) * 0xBF58476D1CE4E5B9ull;
+  x = (x ^ (x >> 27)) * 0x94D049BB133111EBull;
+  return x ^ (x >> 31);
+}
+__device__ __forceinline__ double rand_double(unsigned long long r, int emin, int emax) {
+  const unsigned long long mant = r & 0xFFFFFFFFFFFFFull;
+  const int e = (int)((r >> 52) % (unsigned long long)(emax - emin + 1)) + emin;
+  const unsigned long long sign = (r >> 63) << 63;
+  const unsigned long long bits = sign | ((unsigned long long)(1023 + e) << 52) | mant;
+  return __longlong_as_double((long long)bits);
+}
+__global__ void k_div_check(long long n, unsigned long long seed, int emax,
+                            unsigned long long* bad, double* example) {
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n;
+       i += (long long)gridDim.x * blockDim.x) {
+    const unsigned long long r1 = splitmix(seed ^ (2 * i)), r2 = splitmix(seed ^ (2 * i + 1));
+    // contract of DivFast (clover_common.cuh): divisor in [2^-900, 2^900]
+    // (here [2^-300, 2^300]), quotient below 2^900; numerators anywhere
+    // down to denormals and zero.
+    double a = rand_double(r1, -emax, emax < 600 ? emax : 600);
+    double b = rand_double(r2 >> 1, -(emax < 300 ? emax : 300), emax < 300 ? emax : 300);
+    if ((r2 & 15) == 0) a = (r1 & 1) ? -0.0 : 0.0;
+    clover::DivFast f;
+    double q1 = f(a, b);
+    if (f.bad) q1 = a / b;
+    const double q2 = a / b;
+    if (__double_as_longlong(q1) != __double_as_longlong(q2)) {
+      if (atomicAdd(bad, 1ull) == 0) { example[0] = a; example[1] = b; }
+    }
+  }
+}
+
+int clover_debug_div_check(int64_t n, uint64_t seed, int32_t emax, int64_t* mismatches,
+                           double* example_ab) {
+  if (!mismatches || n < 0 || emax < 1 || emax > 1023) return fail(CLOVER_ERR_ARG, "bad arguments");
+  unsigned long long* d_bad = nullptr;
+  double* d_ex = nullptr;
+  CK(cudaMalloc(&d_bad, sizeof(unsigned long long)));
+  CK(cudaMalloc(&d_ex, 2 * sizeof(double)));
+  CK(cudaMemset(d_bad, 0, sizeof(unsigned long long)));
+  CK(cudaMemset(d_ex, 0, 2 * sizeof(double)));
+  k_div_check<<<148 * 16, 256>>>(n, seed, emax, d_bad, d_ex);
+  CK(cudaGetLastError());
+  unsigned long long h = 0;
+  double ex[2] = {0, 0};
+  CK(cudaMemcpy(&h, d_bad, sizeof(h), cudaMemcpyDeviceToHost));
+  CK(cudaMemcpy(ex, d_ex, sizeof(ex), cudaMemcpyDeviceToHost));
+  cudaFree(d_bad);
+  cudaFree(d_ex);
+  *mismatches = (int64_t)h;
+  if (example_ab) { example_ab[0] = ex[0]; example_ab[1] = ex[1]; }
+  return CLOVER_OK;
 }
 
 const char* clover_profile_name(int32_t i) { return (i >= 0 && i < NPROF) ? kProfNames[i] : ""; }
