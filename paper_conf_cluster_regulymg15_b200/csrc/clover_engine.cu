@@ -20,6 +20,7 @@
 #include "clover_aux.cuh"
 #include "clover_common.cuh"
 #include "clover_kernels.cuh"
+#include "clover_stream.cuh"
 
 #ifdef CLOVER_WITH_NCCL
 #include <nccl.h>
@@ -375,16 +376,23 @@ void prof_mark(clover_ctx* ctx, int id) {
   ctx->prof_events.push_back({id, e});
 }
 
+// Launch geometry of the streaming kernels (clover_stream.cuh).
+inline int cdiv(int a, int b) { return (a + b - 1) / b; }
+dim3 grid_cols(int ncols, int nrows, int ks) { return dim3(cdiv(ncols, SB), cdiv(nrows, ks)); }
+dim3 grid_strip(int ncols, int width, int nrows, int ks) {
+  return dim3(cdiv(cdiv(ncols, width), SB / 32), cdiv(nrows, ks));
+}
+
 // Enqueue kernel phases [0, nphase) of one step (7 = full step).
 int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
   cudaStream_t st = ctx->work;
-  const dim3 blk(32, 8);
   int cur_prof_id = P_VISC_DT;
   if (ctx->prof) prof_mark(ctx, -1);
   if (nphase >= 1) {
     for (auto& cs : ctx->chunks) {
-      k_visc_dt<<<cell_grid(cs.c, 32, 8), blk, 0, st>>>(cs.c, cs.buf[B_D0], cs.buf[B_E0], cs.buf[B_U0],
-                                                         cs.buf[B_V0], cs.buf[B_Q], ctx->scal, ctx->dtp);
+      const Chunk& c = cs.c;
+      ks_visc_dt<<<grid_cols(c.nx, c.ny, VKS), SB, 0, st>>>(c, cs.buf[B_D0], cs.buf[B_E0], cs.buf[B_U0],
+                                                             cs.buf[B_V0], cs.buf[B_Q], ctx->scal, ctx->dtp);
       STEP_LAUNCH_CHECK();
     }
     int rc = exchange(ctx, {B_Q});
@@ -404,8 +412,9 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
   if (nphase >= 3) {
     cur_prof_id = P_LAGR;
     for (auto& cs : ctx->chunks) {
-      k_lagrangian<<<cell_grid(cs.c, LX, LY), dim3(LX, LY), 0, st>>>(
-          cs.c, cs.buf[B_D0], cs.buf[B_E0], cs.buf[B_U0], cs.buf[B_V0], cs.buf[B_Q], cs.buf[B_D1],
+      const Chunk& c = cs.c;
+      ks_lagrangian<<<grid_strip(c.nx, LW, c.ny, LKS), SB, 0, st>>>(
+          c, cs.buf[B_D0], cs.buf[B_E0], cs.buf[B_U0], cs.buf[B_V0], cs.buf[B_Q], cs.buf[B_D1],
           cs.buf[B_E1], cs.buf[B_U1], cs.buf[B_V1], cs.buf[B_FX], cs.buf[B_FY], ctx->scal);
       STEP_LAUNCH_CHECK();
     }
@@ -413,7 +422,6 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
     if (rc) return rc;
     if (ctx->prof) prof_mark(ctx, -1);
   }
-  const dim3 ablk(AX, AY);
   // sweep 1 (direction d1) reads B writes C; sweep 2 reads C writes A.
   for (int sweep = 1; sweep <= 2; ++sweep) {
     const bool xdir = (sweep == 1) ? advect_x : !advect_x;
@@ -426,18 +434,21 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
     if (nphase >= ph_cell) {
       cur_prof_id = xdir ? (sweep == 1 ? P_CELL_X1 : P_CELL_X2) : (sweep == 1 ? P_CELL_Y1 : P_CELL_Y2);
       for (auto& cs : ctx->chunks) {
+        const Chunk& c = cs.c;
         const double* fx = cs.buf[B_FX];
         const double* fy = cs.buf[B_FY];
         if (xdir) {
+          const dim3 g = grid_strip(c.nx, CW_X, c.ny, CKS);
           if (sweep == 1)
-            k_advec_cell_x<1><<<cell_grid(cs.c, AX, AY), ablk, 0, st>>>(cs.c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf]);
+            ks_advec_cell_x<1><<<g, SB, 0, st>>>(c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf]);
           else
-            k_advec_cell_x<2><<<cell_grid(cs.c, AX, AY), ablk, 0, st>>>(cs.c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf]);
+            ks_advec_cell_x<2><<<g, SB, 0, st>>>(c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf]);
         } else {
+          const dim3 g = grid_cols(c.nx, c.ny, CKS_Y);
           if (sweep == 1)
-            k_advec_cell_y<1><<<cell_grid(cs.c, AX, AY), ablk, 0, st>>>(cs.c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf]);
+            ks_advec_cell_y<1><<<g, SB, 0, st>>>(c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf]);
           else
-            k_advec_cell_y<2><<<cell_grid(cs.c, AX, AY), ablk, 0, st>>>(cs.c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf]);
+            ks_advec_cell_y<2><<<g, SB, 0, st>>>(c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf]);
         }
         STEP_LAUNCH_CHECK();
       }
@@ -448,16 +459,19 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
     if (nphase >= ph_cell + 1) {
       cur_prof_id = xdir ? (sweep == 1 ? P_MOM_X1 : P_MOM_X2) : (sweep == 1 ? P_MOM_Y1 : P_MOM_Y2);
       for (auto& cs : ctx->chunks) {
+        const Chunk& c = cs.c;
         if (xdir) {
+          const dim3 g = grid_strip(c.nx + 1, MW_X, c.ny + 1, MKS);
           if (sweep == 1)
-            k_advec_mom_x<1><<<node_grid(cs.c, AX, AY), ablk, 0, st>>>(cs.c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FY], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout]);
+            ks_advec_mom_x<1><<<g, SB, 0, st>>>(c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FY], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout]);
           else
-            k_advec_mom_x<2><<<node_grid(cs.c, AX, AY), ablk, 0, st>>>(cs.c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FY], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout]);
+            ks_advec_mom_x<2><<<g, SB, 0, st>>>(c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FY], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout]);
         } else {
+          const dim3 g = grid_cols(c.nx + 1, c.ny + 1, MKS_Y);
           if (sweep == 1)
-            k_advec_mom_y<1><<<node_grid(cs.c, AX, AY), ablk, 0, st>>>(cs.c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FX], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout]);
+            ks_advec_mom_y<1><<<g, SB, 0, st>>>(c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FX], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout]);
           else
-            k_advec_mom_y<2><<<node_grid(cs.c, AX, AY), ablk, 0, st>>>(cs.c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FX], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout]);
+            ks_advec_mom_y<2><<<g, SB, 0, st>>>(c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FX], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout]);
         }
         STEP_LAUNCH_CHECK();
       }

@@ -1,0 +1,567 @@
+// clover_stream.cuh -- row-streaming sm_100a kernels of the CloverLeaf 2D
+// step (the production path; clover_kernels.cuh holds the per-point math).
+//
+// Thread mapping: one thread per mesh column j, each
+// thread walks a segment of rows k keeping the rows it still needs in
+// registers, so every field element is loaded once per kernel and index
+// arithmetic is one add per row.  Warps are 32 consecutive columns
+// (coalesced 256-B row segments).  Neighbour values along x that are
+// COMPUTED in the same kernel (half-step pressure, face fluxes, node masses,
+// momentum fluxes) come from the adjacent lane via warp shuffles; the
+// kernels whose x stencil reaches computed values overlap their warps by
+// 1-3 "halo lanes".  Raw inputs at x-neighbours are plain L1-cached loads.
+//
+// All arithmetic is in the per-point functions of clover_kernels.cuh
+// (evaluation order of SURVEY 8(c)); division policy DivFast with a
+// per-point IEEE recompute when flagged.
+#pragma once
+#include "clover_common.cuh"
+#include "clover_kernels.cuh"
+
+namespace clover {
+
+constexpr unsigned FULL = 0xffffffffu;
+constexpr int SB = 128;  // threads per block (4 warps)
+
+// ================================================================ visc_dt
+// Column j = block*128 + tid + 1, rows [k0, k0+VKS).  Rolling: pressure of
+// the row below, density/energy of the row above, the 4 node velocities.
+constexpr int VKS = 16;
+
+__global__ void __launch_bounds__(SB)
+ks_visc_dt(Chunk c, const double* __restrict__ d0, const double* __restrict__ e0,
+           const double* __restrict__ u0, const double* __restrict__ v0, double* __restrict__ q,
+           StepScalars* __restrict__ s, DtParams prm) {
+  const int j = blockIdx.x * SB + threadIdx.x + 1;
+  const int k0 = blockIdx.y * VKS + 1;
+  const int k1 = min(k0 + VKS, c.ny + 1);
+  double dtl = G_BIG;
+  if (j <= c.nx) {
+    const int P = c.pitch;
+    int i = idx(c, j, k0);
+    double pcm = eos_pressure(d0[i - P], e0[i - P]);
+    double rho = d0[i], ein = e0[i];
+    double pc = eos_pressure(rho, ein);
+    double ua = u0[i], ub = u0[i + 1], va = v0[i], vb = v0[i + 1];
+    for (int k = k0; k < k1; ++k, i += P) {
+      const double rhon = d0[i + P], en = e0[i + P];
+      ViscIn I;
+      I.rho = rho; I.e = ein;
+      I.pb = pcm;
+      I.pt = eos_pressure(rhon, en);
+      I.pl = eos_pressure(d0[i - 1], e0[i - 1]);
+      I.pr = eos_pressure(d0[i + 1], e0[i + 1]);
+      const double uc = u0[i + P], ud = u0[i + P + 1], vc = v0[i + P], vd = v0[i + P + 1];
+      I.u00 = ua; I.u10 = ub; I.u01 = uc; I.u11 = ud;
+      I.v00 = va; I.v10 = vb; I.v01 = vc; I.v11 = vd;
+      double qv;
+      DivFast f;
+      double dtc = visc_dt_cell(f, I, c.dx, c.dy, prm, qv);
+      if (f.bad) {
+        DivIEEE x;
+        dtc = visc_dt_cell(x, I, c.dx, c.dy, prm, qv);
+      }
+      dtl = fmin(dtl, dtc);
+      store_field(c, q, K_CELL, j, k, qv);
+      pcm = pc; pc = I.pt; rho = rhon; ein = en;
+      ua = uc; ub = ud; va = vc; vb = vd;
+    }
+  }
+  for (int o = 16; o > 0; o >>= 1) dtl = fmin(dtl, __shfl_xor_sync(FULL, dtl, o));
+  __shared__ double wmin[SB / 32];
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  if (lane == 0) wmin[warp] = dtl;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    double m = wmin[0];
+    for (int w = 1; w < SB / 32; ++w) m = fmin(m, wmin[w]);
+    atomicMin(&s->dt_slot, (unsigned long long)__double_as_longlong(m));
+  }
+}
+
+// ================================================================ Lagrangian
+// Warp strip: lane l <-> column j = J0 - 1 + l, J0 = 1 + 30 * (global warp);
+// lanes 1..30 own cells/nodes j (lane 0 and 31 are halo lanes).  Rows are
+// streamed k = k0-1 .. k1: at row k the thread computes the PdV predictor +
+// EOS of cell (j,k), accelerate at node (j,k) and the PdV corrector +
+// flux_calc of cell (j,k-1).  Reflective walls: the half-step pressure of a
+// ring cell outside the mesh is the mirror of the computed interior value
+// (rows: recomputed from the mirrored row; columns: taken from the mirrored
+// lane), exactly the reference's update_halo{pressure} after the predictor.
+constexpr int LW = 30;   // owned columns per warp
+constexpr int LKS = 32;  // rows per segment
+
+__global__ void __launch_bounds__(SB)
+ks_lagrangian(Chunk c, const double* __restrict__ d0, const double* __restrict__ e0,
+              const double* __restrict__ u0, const double* __restrict__ v0,
+              const double* __restrict__ q, double* __restrict__ d1, double* __restrict__ e1,
+              double* __restrict__ u1, double* __restrict__ v1, double* __restrict__ fx,
+              double* __restrict__ fy, const StepScalars* __restrict__ s) {
+  const int lane = threadIdx.x & 31;
+  const int gw = blockIdx.x * (SB / 32) + (threadIdx.x >> 5);
+  const int J0 = 1 + LW * gw;
+  const int j = J0 - 1 + lane;
+  if (J0 > c.nx) return;  // whole warp beyond the chunk
+  const int k0 = blockIdx.y * LKS + 1;
+  const int k1 = min(k0 + LKS, c.ny + 1);  // cell rows [k0, k1)
+  const double dt = s->dt, dx = c.dx, dy = c.dy;
+  const int P = c.pitch;
+  // column validity: cells exist for j in [0, nx+1] (ring incl.)
+  const bool colok = j <= c.nx + 1;
+  // mirrored-lane sources for the x walls
+  int src = lane;
+  if (c.wl && j == 0) src = lane + 1;
+  if (c.wr && j == c.nx + 1) src = lane - 1;
+  const bool xwall_warp = __any_sync(FULL, src != lane);
+
+  // rolling state (row k-1)
+  double r_m = 1.0, e_m = 0.0, q_m = 0.0, ph_m = 0.0;     // cell (j, k-1)
+  double rl_m = 1.0, phl_m = 0.0, ql_m = 0.0;             // cell (j-1, k-1)
+  double u0_m = 0.0, v0_m = 0.0, u0r_m = 0.0, v0r_m = 0.0; // nodes (j,k-1), (j+1,k-1)
+  double u1_m = 0.0, v1_m = 0.0;                          // node (j, k-1) after accelerate
+  double u0_c = 0.0, v0_c = 0.0, u0r_c = 0.0, v0r_c = 0.0; // nodes (j,k), (j+1,k)
+
+  // node row k0-1 (bottom of the first ring cell row)
+  if (colok) {
+    const int in = idx(c, j, k0 - 1);
+    u0_c = u0[in]; v0_c = v0[in]; u0r_c = u0[in + 1]; v0r_c = v0[in + 1];
+  }
+  for (int k = k0 - 1; k <= k1; ++k) {
+    // ---- A: cell row k (ring rows k0-1 and k1 included)
+    double r = 1.0, e = 0.0, qq = 0.0, ph = 0.0;
+    double u0_n = 0.0, v0_n = 0.0, u0r_n = 0.0, v0r_n = 0.0;  // nodes (j,k+1), (j+1,k+1)
+    if (colok) {
+      const int i = idx(c, j, k);
+      r = d0[i]; e = e0[i]; qq = q[i];
+      u0_n = u0[i + P]; v0_n = v0[i + P]; u0r_n = u0[i + P + 1]; v0r_n = v0[i + P + 1];
+      // rows outside a reflective wall take the mirrored row's predictor
+      int kp = k;
+      if (c.wb && k == 0) kp = 1;
+      if (c.wt && k == c.ny + 1) kp = c.ny;
+      double pr_, pe_, pq_, ua, ub, uc, ud, va, vb, vc, vd;
+      if (kp == k) {
+        pr_ = r; pe_ = e; pq_ = qq;
+        ua = u0_c; ub = u0_n; uc = u0r_c; ud = u0r_n;
+        va = v0_c; vb = v0r_c; vc = v0_n; vd = v0r_n;
+      } else {
+        const int ip = idx(c, j, kp);
+        pr_ = d0[ip]; pe_ = e0[ip]; pq_ = q[ip];
+        ua = u0[ip]; ub = u0[ip + P]; uc = u0[ip + 1]; ud = u0[ip + P + 1];
+        va = v0[ip]; vb = v0[ip + 1]; vc = v0[ip + P]; vd = v0[ip + P + 1];
+      }
+      DivFast f;
+      ph = pdv_predict_pressure(f, pr_, pe_, pq_, ua, ub, uc, ud, va, vb, vc, vd, dx, dy, dt);
+      if (f.bad) {
+        DivIEEE x;
+        ph = pdv_predict_pressure(x, pr_, pe_, pq_, ua, ub, uc, ud, va, vb, vc, vd, dx, dy, dt);
+      }
+    }
+    if (xwall_warp) ph = __shfl_sync(FULL, ph, src);
+    const double rl = __shfl_up_sync(FULL, r, 1);
+    const double phl = __shfl_up_sync(FULL, ph, 1);
+    const double ql = __shfl_up_sync(FULL, qq, 1);
+
+    // ---- B: accelerate at node (j,k), node rows [k0, k1]
+    double u1_c = 0.0, v1_c = 0.0;
+    if (k >= k0 && colok) {
+      const double rr[4] = {rl_m, r_m, r, rl};
+      const double pp[4] = {phl_m, ph_m, ph, phl};
+      const double qv[4] = {ql_m, q_m, qq, ql};
+      DivFast f;
+      accelerate_node(f, rr, pp, qv, u0_c, v0_c, dx, dy, dt, u1_c, v1_c);
+      if (f.bad) {
+        DivIEEE x;
+        accelerate_node(x, rr, pp, qv, u0_c, v0_c, dx, dy, dt, u1_c, v1_c);
+      }
+    }
+    const double u1r_c = __shfl_down_sync(FULL, u1_c, 1);
+    const double v1r_c = __shfl_down_sync(FULL, v1_c, 1);
+    const double u1r_m = __shfl_down_sync(FULL, u1_m, 1);
+    const double v1r_m = __shfl_down_sync(FULL, v1_m, 1);
+
+    // ---- C: PdV corrector + flux_calc of cell (j, k-1), rows [k0, k1)
+    const int kc = k - 1;
+    if (kc >= k0 && lane >= 1 && lane <= LW && j <= c.nx) {
+      // nodes: a=(j,kc) b=(j,kc+1) c=(j+1,kc) d=(j+1,kc+1)
+      const double lsum = u0_m + u0_c + u1_m + u1_c;
+      const double rsum = u0r_m + u0r_c + u1r_m + u1r_c;
+      const double bsum = v0_m + v0r_m + v1_m + v1r_m;
+      const double tsum = v0_c + v0r_c + v1_c + v1r_c;
+      double ev, dvv;
+      DivFast f;
+      pdv_correct(f, r_m, e_m, ph_m, q_m, lsum, rsum, bsum, tsum, dx, dy, dt, ev, dvv);
+      if (f.bad) {
+        DivIEEE x;
+        pdv_correct(x, r_m, e_m, ph_m, q_m, lsum, rsum, bsum, tsum, dx, dy, dt, ev, dvv);
+      }
+      store_field(c, e1, K_CELL, j, kc, ev);
+      store_field(c, d1, K_CELL, j, kc, dvv);
+      const double cx = 0.25 * dt * dy, cy = 0.25 * dt * dx;
+      store_field(c, fx, K_XFACE, j, kc, cx * lsum);
+      store_field(c, fy, K_YFACE, j, kc, cy * bsum);
+      if (j == c.nx) store_field(c, fx, K_XFACE, j + 1, kc, cx * rsum);
+      if (kc == c.ny) store_field(c, fy, K_YFACE, j, kc + 1, cy * tsum);
+      store_field(c, u1, K_XVEL, j, kc, u1_m);
+      store_field(c, v1, K_YVEL, j, kc, v1_m);
+      if (j == c.nx) {
+        store_field(c, u1, K_XVEL, j + 1, kc, u1r_m);
+        store_field(c, v1, K_YVEL, j + 1, kc, v1r_m);
+      }
+      if (kc == c.ny) {
+        store_field(c, u1, K_XVEL, j, kc + 1, u1_c);
+        store_field(c, v1, K_YVEL, j, kc + 1, v1_c);
+      }
+      if (j == c.nx && kc == c.ny) {
+        store_field(c, u1, K_XVEL, j + 1, kc + 1, u1r_c);
+        store_field(c, v1, K_YVEL, j + 1, kc + 1, v1r_c);
+      }
+    }
+    // ---- roll
+    r_m = r; e_m = e; q_m = qq; ph_m = ph;
+    rl_m = rl; phl_m = phl; ql_m = ql;
+    u0_m = u0_c; v0_m = v0_c; u0r_m = u0r_c; v0r_m = v0r_c;
+    u0_c = u0_n; v0_c = v0_n; u0r_c = u0r_n; v0r_c = v0r_n;
+    u1_m = u1_c; v1_m = v1_c;
+  }
+}
+
+// ================================================================ advec_cell x
+// Warp strip: lane l <-> face/cell column j = J0 + l, J0 = 1 + 31*(warp);
+// every lane computes the flux of face j, lanes 0..30 update cell j using
+// face j+1 from the next lane.  Rows [k0, k0+CKS).
+constexpr int CW_X = 31;
+constexpr int CKS = 16;
+
+template <int SWEEP>
+__global__ void __launch_bounds__(SB)
+ks_advec_cell_x(Chunk c, const double* __restrict__ rho, const double* __restrict__ en,
+                const double* __restrict__ fx, const double* __restrict__ fy,
+                double* __restrict__ rho_out, double* __restrict__ en_out,
+                double* __restrict__ mfx) {
+  const int lane = threadIdx.x & 31;
+  const int gw = blockIdx.x * (SB / 32) + (threadIdx.x >> 5);
+  const int J0 = 1 + CW_X * gw;
+  if (J0 > c.nx) return;
+  const int j = J0 + lane;
+  const int k0 = blockIdx.y * CKS + 1;
+  const int k1 = min(k0 + CKS, c.ny + 1);
+  const double vol = c.dx * c.dy;
+  const int P = c.pitch;
+  const bool faceok = j <= c.nx + 1;
+  for (int k = k0; k < k1; ++k) {
+    const int i = idx(c, j, k);
+    double pv = 0.0, pvl = 0.0, F = 0.0, m = 0.0, ef = 0.0, rr = 0.0, ee = 0.0, flo = 0.0, fhi = 0.0;
+    if (faceok) {
+      flo = fx[i]; fhi = fx[i + 1];
+      F = flo;
+      pv = (SWEEP == 1) ? vol + (fhi - flo + fy[i + P] - fy[i]) : vol + fhi - flo;
+      rr = rho[i]; ee = en[i];
+    }
+    pvl = __shfl_up_sync(FULL, pv, 1);
+    if (faceok) {
+      if (lane == 0) {
+        const double fl = fx[i - 1];
+        pvl = (SWEEP == 1) ? vol + (flo - fl + fy[i - 1 + P] - fy[i - 1]) : vol + flo - fl;
+      }
+      double ru, rd, rw, eu, ed, ew, pvd;
+      if (F > 0.0) {
+        ru = rho[i - 2]; rd = rho[i - 1]; rw = rr;
+        eu = en[i - 2]; ed = en[i - 1]; ew = ee;
+        pvd = pvl;
+      } else {
+        const int up = min(j + 1, c.nx + 2) - j;
+        ru = rho[i + up]; rd = rr; rw = rho[i - 1];
+        eu = en[i + up]; ed = ee; ew = en[i - 1];
+        pvd = pv;
+      }
+      DivFast f;
+      cell_face_flux(f, F, pvd, ru, rd, rw, eu, ed, ew, m, ef);
+      if (f.bad) {
+        DivIEEE x;
+        cell_face_flux(x, F, pvd, ru, rd, rw, eu, ed, ew, m, ef);
+      }
+    }
+    const double mh = __shfl_down_sync(FULL, m, 1);
+    const double efh = __shfl_down_sync(FULL, ef, 1);
+    if (lane < CW_X && j <= c.nx) {
+      double ro, eo;
+      DivFast f;
+      cell_update(f, rr, ee, pv, m, mh, ef, efh, flo, fhi, ro, eo);
+      if (f.bad) {
+        DivIEEE x;
+        cell_update(x, rr, ee, pv, m, mh, ef, efh, flo, fhi, ro, eo);
+      }
+      store_field(c, rho_out, K_CELL, j, k, ro);
+      store_field(c, en_out, K_CELL, j, k, eo);
+      store_field(c, mfx, K_XFACE, j, k, m);
+      if (j == c.nx) store_field(c, mfx, K_XFACE, j + 1, k, mh);
+    }
+  }
+}
+
+// ================================================================ advec_cell y
+// Column j = block*128 + tid + 1; streams cell rows [k0, k1).  Iteration k
+// computes the flux of face k+1 and updates cell k (face k from the previous
+// iteration).  Registers hold density/energy of rows k-1..k+2 and the
+// pre-sweep volume of rows k, k+1.
+constexpr int CKS_Y = 32;
+
+template <int SWEEP>
+__global__ void __launch_bounds__(SB)
+ks_advec_cell_y(Chunk c, const double* __restrict__ rho, const double* __restrict__ en,
+                const double* __restrict__ fx, const double* __restrict__ fy,
+                double* __restrict__ rho_out, double* __restrict__ en_out,
+                double* __restrict__ mfy) {
+  const int j = blockIdx.x * SB + threadIdx.x + 1;
+  if (j > c.nx) return;
+  const int k0 = blockIdx.y * CKS_Y + 1;
+  const int k1 = min(k0 + CKS_Y, c.ny + 1);
+  const double vol = c.dx * c.dy;
+  const int P = c.pitch;
+  auto pre_vol = [&](int i) -> double {
+    if (SWEEP == 1) return vol + (fy[i + P] - fy[i] + fx[i + 1] - fx[i]);
+    return vol + fy[i + P] - fy[i];
+  };
+  int i = idx(c, j, k0);
+  // rows k0-2 .. k0+1
+  double R0 = rho[i - 2 * P], R1 = rho[i - P], R2 = rho[i], R3 = rho[i + P];
+  double E0 = en[i - 2 * P], E1 = en[i - P], E2 = en[i], E3 = en[i + P];
+  double pvm = pre_vol(i - P), pv0 = pre_vol(i);
+  // face k0
+  double m0, ef0;
+  {
+    const double F = fy[i];
+    double ru, rd, rw, eu, ed, ew, pvd;
+    if (F > 0.0) {
+      ru = R0; rd = R1; rw = R2; eu = E0; ed = E1; ew = E2; pvd = pvm;
+    } else {
+      ru = R3; rd = R2; rw = R1; eu = E3; ed = E2; ew = E1; pvd = pv0;
+    }
+    DivFast f;
+    cell_face_flux(f, F, pvd, ru, rd, rw, eu, ed, ew, m0, ef0);
+    if (f.bad) {
+      DivIEEE x;
+      cell_face_flux(x, F, pvd, ru, rd, rw, eu, ed, ew, m0, ef0);
+    }
+  }
+  for (int k = k0; k < k1; ++k, i += P) {
+    // registers: R1..R3 = rows k-1..k+1; load row k+2
+    const double R4 = rho[i + 2 * P], E4 = en[i + 2 * P];
+    const double pv1 = pre_vol(i + P);
+    // face k+1: up = k (F>0: k-1+1), don = k, dw = k+1 ; else up = k+2, don = k+1, dw = k
+    double m1, ef1;
+    {
+      const double F = fy[i + P];
+      double ru, rd, rw, eu, ed, ew, pvd;
+      if (F > 0.0) {
+        ru = R1; rd = R2; rw = R3; eu = E1; ed = E2; ew = E3; pvd = pv0;
+      } else {
+        ru = R4; rd = R3; rw = R2; eu = E4; ed = E3; ew = E2; pvd = pv1;
+      }
+      DivFast f;
+      cell_face_flux(f, F, pvd, ru, rd, rw, eu, ed, ew, m1, ef1);
+      if (f.bad) {
+        DivIEEE x;
+        cell_face_flux(x, F, pvd, ru, rd, rw, eu, ed, ew, m1, ef1);
+      }
+    }
+    double ro, eo;
+    {
+      const double flo = fy[i], fhi = fy[i + P];
+      DivFast f;
+      cell_update(f, R2, E2, pv0, m0, m1, ef0, ef1, flo, fhi, ro, eo);
+      if (f.bad) {
+        DivIEEE x;
+        cell_update(x, R2, E2, pv0, m0, m1, ef0, ef1, flo, fhi, ro, eo);
+      }
+    }
+    store_field(c, rho_out, K_CELL, j, k, ro);
+    store_field(c, en_out, K_CELL, j, k, eo);
+    store_field(c, mfy, K_YFACE, j, k, m0);
+    if (k == c.ny) store_field(c, mfy, K_YFACE, j, k + 1, m1);
+    R0 = R1; R1 = R2; R2 = R3; R3 = R4;
+    E0 = E1; E1 = E2; E2 = E3; E3 = E4;
+    pvm = pv0; pv0 = pv1;
+    m0 = m1; ef0 = ef1;
+  }
+}
+
+// ================================================================ advec_mom x
+// Warp strip: lane l <-> node column j = J0 - 2 + l, J0 = 1 + 29*(warp);
+// lanes 2..30 update nodes j.  Per node row k: node flux from the mass
+// fluxes of faces j, j+1 (rows k-1, k), node masses from cells j-1, j
+// (rows k-1, k; column j-1 via shuffle), momentum fluxes for u and v.
+constexpr int MW_X = 29;
+constexpr int MKS = 16;
+
+template <int SWEEP>
+__global__ void __launch_bounds__(SB)
+ks_advec_mom_x(Chunk c, const double* __restrict__ rho, const double* __restrict__ mfx,
+               const double* __restrict__ fy, const double* __restrict__ uin,
+               const double* __restrict__ vin, double* __restrict__ uout,
+               double* __restrict__ vout) {
+  const int lane = threadIdx.x & 31;
+  const int gw = blockIdx.x * (SB / 32) + (threadIdx.x >> 5);
+  const int J0 = 1 + MW_X * gw;
+  if (J0 > c.nx + 1) return;
+  const int j = J0 - 2 + lane;
+  const int k0 = blockIdx.y * MKS + 1;
+  const int k1 = min(k0 + MKS, c.ny + 2);  // node rows [k0, k1)
+  const double vol = c.dx * c.dy;
+  const int P = c.pitch;
+  const bool nfok = j <= c.nx + 2;   // node flux / node mass columns
+  auto mass_post = [&](int i) -> double {
+    const double pv = (SWEEP == 1) ? vol + fy[i + P] - fy[i] : vol;
+    return rho[i] * pv;
+  };
+  double mA_m = 0.0, mB_m = 0.0, mp_m = 0.0;  // row k-1: Mx(j), Mx(j+1), mass of cell (j,k-1)
+  if (nfok) {
+    const int i = idx(c, j, k0 - 1);
+    mA_m = mfx[i]; mB_m = mfx[i + 1]; mp_m = mass_post(i);
+  }
+  double mpl_m = __shfl_up_sync(FULL, mp_m, 1);
+  for (int k = k0; k < k1; ++k) {
+    const int i = idx(c, j, k);
+    double mA = 0.0, mB = 0.0, mp = 0.0;
+    if (nfok) {
+      mA = mfx[i]; mB = mfx[i + 1]; mp = mass_post(i);
+    }
+    const double mpl = __shfl_up_sync(FULL, mp, 1);
+    const double nf = 0.25 * (mA_m + mA + mB_m + mB);
+    const double post = 0.25 * (mp_m + mp + mpl_m + mpl);
+    const double nfl = __shfl_up_sync(FULL, nf, 1);
+    const double pre = post - nfl + nf;
+    const double prer = __shfl_down_sync(FULL, pre, 1);
+    double mu = 0.0, mv = 0.0;
+    if (lane >= 1 && lane <= 30 && j <= c.nx + 1) {
+      int up, don, dw;
+      double nmp;
+      if (nf < 0.0) {
+        up = 2; don = 1; dw = 0; nmp = prer;
+      } else {
+        up = -1; don = 0; dw = 1; nmp = pre;
+      }
+      const double uu[3] = {uin[i + up], uin[i + don], uin[i + dw]};
+      const double vv[3] = {vin[i + up], vin[i + don], vin[i + dw]};
+      DivFast f;
+      mom_flux2(f, nf, nmp, uu, vv, c.dx, mu, mv);
+      if (f.bad) {
+        DivIEEE x;
+        mom_flux2(x, nf, nmp, uu, vv, c.dx, mu, mv);
+      }
+    }
+    const double mul = __shfl_up_sync(FULL, mu, 1);
+    const double mvl = __shfl_up_sync(FULL, mv, 1);
+    if (lane >= 2 && lane <= MW_X + 1 && j <= c.nx + 1) {
+      const double u = uin[i], v = vin[i];
+      double un, vn;
+      DivFast f;
+      mom_update(f, u, v, pre, post, mul, mu, mvl, mv, un, vn);
+      if (f.bad) {
+        DivIEEE x;
+        mom_update(x, u, v, pre, post, mul, mu, mvl, mv, un, vn);
+      }
+      store_field(c, uout, K_XVEL, j, k, un);
+      store_field(c, vout, K_YVEL, j, k, vn);
+    }
+    mA_m = mA; mB_m = mB; mp_m = mp; mpl_m = mpl;
+  }
+}
+
+// ================================================================ advec_mom y
+// Column j = block*128 + tid + 1 (node column), streams node rows [k0, k1).
+// Iteration k computes node flux / node masses of row k+1, the momentum
+// flux of row k and updates node k.
+constexpr int MKS_Y = 32;
+
+template <int SWEEP>
+__global__ void __launch_bounds__(SB)
+ks_advec_mom_y(Chunk c, const double* __restrict__ rho, const double* __restrict__ mfy,
+               const double* __restrict__ fx, const double* __restrict__ uin,
+               const double* __restrict__ vin, double* __restrict__ uout,
+               double* __restrict__ vout) {
+  const int j = blockIdx.x * SB + threadIdx.x + 1;
+  if (j > c.nx + 1) return;
+  const int k0 = blockIdx.y * MKS_Y + 1;
+  const int k1 = min(k0 + MKS_Y, c.ny + 2);
+  const double vol = c.dx * c.dy;
+  const int P = c.pitch;
+  auto mass_post = [&](int i) -> double {  // rho * post_vol of the cell at offset i
+    const double pv = (SWEEP == 1) ? vol + fx[i + 1] - fx[i] : vol;
+    return rho[i] * pv;
+  };
+  // node flux of row r uses My(j-1,r), My(j,r), My(j-1,r+1), My(j,r+1)
+  auto node_flux = [&](int i) -> double {
+    return 0.25 * (mfy[i - 1] + mfy[i] + mfy[i - 1 + P] + mfy[i + P]);
+  };
+  // node mass post of row r uses cells (j,r-1), (j,r), (j-1,r-1), (j-1,r)
+  auto node_post = [&](double mj_m, double mj, double ml_m, double ml) -> double {
+    return 0.25 * (mj_m + mj + ml_m + ml);
+  };
+  int i = idx(c, j, k0);
+  // prologue: rows k0-2 .. k0
+  double mpj_a = mass_post(i - 2 * P), mpl_a = mass_post(i - 2 * P - 1);  // row k0-2
+  double mpj_b = mass_post(i - P), mpl_b = mass_post(i - P - 1);          // row k0-1
+  double mpj_c = mass_post(i), mpl_c = mass_post(i - 1);                  // row k0
+  const double nf_m2 = node_flux(i - 2 * P);
+  double nf_m = node_flux(i - P);                  // nf(k0-1)
+  double nf_0 = node_flux(i);                      // nf(k0)
+  const double post_m = node_post(mpj_a, mpj_b, mpl_a, mpl_b);   // nmpost(k0-1)
+  double post_0 = node_post(mpj_b, mpj_c, mpl_b, mpl_c);         // nmpost(k0)
+  const double pre_m = post_m - nf_m2 + nf_m;                    // nmp(k0-1)
+  double pre_0 = post_0 - nf_m + nf_0;                           // nmp(k0)
+  double U0 = uin[i - 2 * P], U1 = uin[i - P], U2 = uin[i], U3 = uin[i + P];  // rows k0-2..k0+1
+  double V0 = vin[i - 2 * P], V1 = vin[i - P], V2 = vin[i], V3 = vin[i + P];
+  double mu_m, mv_m;  // mom flux of row k0-1
+  {
+    const double nf = nf_m;
+    const double nmp = (nf < 0.0) ? pre_0 : pre_m;
+    const double uu[3] = {nf < 0.0 ? U3 : U0, nf < 0.0 ? U2 : U1, nf < 0.0 ? U1 : U2};
+    const double vv[3] = {nf < 0.0 ? V3 : V0, nf < 0.0 ? V2 : V1, nf < 0.0 ? V1 : V2};
+    DivFast f;
+    mom_flux2(f, nf, nmp, uu, vv, c.dy, mu_m, mv_m);
+    if (f.bad) {
+      DivIEEE x;
+      mom_flux2(x, nf, nmp, uu, vv, c.dy, mu_m, mv_m);
+    }
+  }
+  for (int k = k0; k < k1; ++k, i += P) {
+    // registers: U1..U3 = rows k-1..k+1 ; load row k+2
+    const double U4 = uin[i + 2 * P], V4 = vin[i + 2 * P];
+    const double mpj_d = mass_post(i + P), mpl_d = mass_post(i + P - 1);  // row k+1
+    const double nf_1 = node_flux(i + P);                                 // nf(k+1)
+    const double post_1 = node_post(mpj_c, mpj_d, mpl_c, mpl_d);          // nmpost(k+1)
+    const double pre_1 = post_1 - nf_0 + nf_1;                            // nmp(k+1)
+    double mu, mv;
+    {
+      const double nf = nf_0;
+      const double nmp = (nf < 0.0) ? pre_1 : pre_0;
+      const double uu[3] = {nf < 0.0 ? U4 : U1, nf < 0.0 ? U3 : U2, nf < 0.0 ? U2 : U3};
+      const double vv[3] = {nf < 0.0 ? V4 : V1, nf < 0.0 ? V3 : V2, nf < 0.0 ? V2 : V3};
+      DivFast f;
+      mom_flux2(f, nf, nmp, uu, vv, c.dy, mu, mv);
+      if (f.bad) {
+        DivIEEE x;
+        mom_flux2(x, nf, nmp, uu, vv, c.dy, mu, mv);
+      }
+    }
+    double un, vn;
+    {
+      DivFast f;
+      mom_update(f, U2, V2, pre_0, post_0, mu_m, mu, mv_m, mv, un, vn);
+      if (f.bad) {
+        DivIEEE x;
+        mom_update(x, U2, V2, pre_0, post_0, mu_m, mu, mv_m, mv, un, vn);
+      }
+    }
+    store_field(c, uout, K_XVEL, j, k, un);
+    store_field(c, vout, K_YVEL, j, k, vn);
+    U1 = U2; U2 = U3; U3 = U4;
+    V1 = V2; V2 = V3; V3 = V4;
+    mpj_c = mpj_d; mpl_c = mpl_d;
+    nf_0 = nf_1; post_0 = post_1; pre_0 = pre_1;
+    mu_m = mu; mv_m = mv;
+  }
+}
+
+}  // namespace clover
