@@ -48,12 +48,17 @@ def stale() -> bool:
     return any(os.path.getmtime(s) > t for s in sources())
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    if not force and not stale():
+def build(force: bool = False, verbose: bool = False, out: str | None = None,
+          defines: tuple = ()) -> str:
+    """Build libclover.so (or a variant at `out` with extra -D defines, for
+    A/B experiments: scripts/ab_variants.py)."""
+    target = out or LIB
+    if out is None and not force and not stale():
         return LIB
     cmd = [nvcc(), "-O3", "-std=c++17", ARCH, "-lineinfo", "-fmad=false",
            "-Xcompiler", "-fPIC", "-shared", "-I", os.path.join(ROOT, "include"),
-           "-o", LIB + ".tmp", os.path.join(CSRC, "clover_engine.cu")]
+           "-o", target + ".tmp", os.path.join(CSRC, "clover_engine.cu")]
+    cmd += ["-D" + d for d in defines]
     nd = nccl_dir()
     if nd:
         cmd += ["-DCLOVER_WITH_NCCL", "-I", os.path.join(nd, "include"),
@@ -63,8 +68,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
         cmd += ["-Xptxas", "-v"]
         print(" ".join(cmd))
     subprocess.check_call(cmd)
-    os.replace(LIB + ".tmp", LIB)
-    return LIB
+    os.replace(target + ".tmp", target)
+    return target
 
 
 if __name__ == "__main__":

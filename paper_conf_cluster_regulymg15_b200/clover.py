@@ -69,7 +69,8 @@ _lib = None
 
 
 def lib_path() -> str:
-    return _build.LIB
+    # CLOVER_LIB: path of an A/B variant of the same library (scripts/ab_variants.py)
+    return os.environ.get("CLOVER_LIB", _build.LIB)
 
 
 def load(build_if_missing: bool = True):
@@ -77,11 +78,12 @@ def load(build_if_missing: bool = True):
     global _lib
     if _lib is not None:
         return _lib
-    if build_if_missing:
+    path = lib_path()
+    if build_if_missing and path == _build.LIB:
         _build.build()
-    if not os.path.exists(_build.LIB):
-        raise RuntimeError(f"libclover.so not found at {_build.LIB}; run __graft_entry__.build()")
-    L = ctypes.CDLL(_build.LIB)
+    if not os.path.exists(path):
+        raise RuntimeError(f"libclover.so not found at {path}; run __graft_entry__.build()")
+    L = ctypes.CDLL(path)
     P = ctypes.POINTER
     L.clover_workspace_bytes.argtypes = [P(CloverGrid), P(CloverDist), P(c_int64)]
     L.clover_nccl_unique_id.argtypes = [c_void_p]

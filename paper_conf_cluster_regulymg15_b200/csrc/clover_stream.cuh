@@ -23,12 +23,58 @@ namespace clover {
 constexpr unsigned FULL = 0xffffffffu;
 constexpr int SB = 128;  // threads per block (4 warps)
 
+// Tunables (defaults = measured best; scripts/ab_variants.py builds others).
+#define CLOVER_STR2(x) #x
+#define CLOVER_STR(x) CLOVER_STR2(x)
+#ifdef CLOVER_UNROLL  // default: the compiler's own unrolling (measured best)
+#define STREAM_LOOP _Pragma(CLOVER_STR(unroll CLOVER_UNROLL))
+#else
+#define STREAM_LOOP
+#endif
+// min resident blocks/SM (register cap) for visc_dt+lagrangian / advection;
+// 0 = plain __launch_bounds__(SB) (ptxas heuristic).  Measured on B200 at
+// 3840^2 (scripts/ab_variants.py): 5 / 8 best (1.79 -> 1.68 ms/step).
+#ifndef CLOVER_MINB_HEAVY
+#define CLOVER_MINB_HEAVY 5
+#endif
+#ifndef CLOVER_MINB_ADV
+#define CLOVER_MINB_ADV 8
+#endif
+#if CLOVER_MINB_HEAVY > 0
+#define LB_HEAVY __launch_bounds__(SB, CLOVER_MINB_HEAVY)
+#else
+#define LB_HEAVY __launch_bounds__(SB)
+#endif
+#if CLOVER_MINB_ADV > 0
+#define LB_ADV __launch_bounds__(SB, CLOVER_MINB_ADV)
+#else
+#define LB_ADV __launch_bounds__(SB)
+#endif
+#ifndef CLOVER_VKS
+#define CLOVER_VKS 16
+#endif
+#ifndef CLOVER_LKS
+#define CLOVER_LKS 32
+#endif
+#ifndef CLOVER_CKS
+#define CLOVER_CKS 16
+#endif
+#ifndef CLOVER_CKS_Y
+#define CLOVER_CKS_Y 32
+#endif
+#ifndef CLOVER_MKS
+#define CLOVER_MKS 16
+#endif
+#ifndef CLOVER_MKS_Y
+#define CLOVER_MKS_Y 32
+#endif
+
 // ================================================================ visc_dt
 // Column j = block*128 + tid + 1, rows [k0, k0+VKS).  Rolling: pressure of
 // the row below, density/energy of the row above, the 4 node velocities.
-constexpr int VKS = 16;
+constexpr int VKS = CLOVER_VKS;
 
-__global__ void __launch_bounds__(SB)
+__global__ void LB_HEAVY
 ks_visc_dt(Chunk c, const double* __restrict__ d0, const double* __restrict__ e0,
            const double* __restrict__ u0, const double* __restrict__ v0, double* __restrict__ q,
            StepScalars* __restrict__ s, DtParams prm) {
@@ -43,6 +89,7 @@ ks_visc_dt(Chunk c, const double* __restrict__ d0, const double* __restrict__ e0
     double rho = d0[i], ein = e0[i];
     double pc = eos_pressure(rho, ein);
     double ua = u0[i], ub = u0[i + 1], va = v0[i], vb = v0[i + 1];
+    STREAM_LOOP
     for (int k = k0; k < k1; ++k, i += P) {
       const double rhon = d0[i + P], en = e0[i + P];
       ViscIn I;
@@ -89,9 +136,9 @@ ks_visc_dt(Chunk c, const double* __restrict__ d0, const double* __restrict__ e0
 // (rows: recomputed from the mirrored row; columns: taken from the mirrored
 // lane), exactly the reference's update_halo{pressure} after the predictor.
 constexpr int LW = 30;   // owned columns per warp
-constexpr int LKS = 32;  // rows per segment
+constexpr int LKS = CLOVER_LKS;  // rows per segment
 
-__global__ void __launch_bounds__(SB)
+__global__ void LB_HEAVY
 ks_lagrangian(Chunk c, const double* __restrict__ d0, const double* __restrict__ e0,
               const double* __restrict__ u0, const double* __restrict__ v0,
               const double* __restrict__ q, double* __restrict__ d1, double* __restrict__ e1,
@@ -126,6 +173,7 @@ ks_lagrangian(Chunk c, const double* __restrict__ d0, const double* __restrict__
     const int in = idx(c, j, k0 - 1);
     u0_c = u0[in]; v0_c = v0[in]; u0r_c = u0[in + 1]; v0r_c = v0[in + 1];
   }
+  STREAM_LOOP
   for (int k = k0 - 1; k <= k1; ++k) {
     // ---- A: cell row k (ring rows k0-1 and k1 included)
     double r = 1.0, e = 0.0, qq = 0.0, ph = 0.0;
@@ -230,10 +278,10 @@ ks_lagrangian(Chunk c, const double* __restrict__ d0, const double* __restrict__
 // every lane computes the flux of face j, lanes 0..30 update cell j using
 // face j+1 from the next lane.  Rows [k0, k0+CKS).
 constexpr int CW_X = 31;
-constexpr int CKS = 16;
+constexpr int CKS = CLOVER_CKS;
 
 template <int SWEEP>
-__global__ void __launch_bounds__(SB)
+__global__ void LB_ADV
 ks_advec_cell_x(Chunk c, const double* __restrict__ rho, const double* __restrict__ en,
                 const double* __restrict__ fx, const double* __restrict__ fy,
                 double* __restrict__ rho_out, double* __restrict__ en_out,
@@ -248,6 +296,7 @@ ks_advec_cell_x(Chunk c, const double* __restrict__ rho, const double* __restric
   const double vol = c.dx * c.dy;
   const int P = c.pitch;
   const bool faceok = j <= c.nx + 1;
+  STREAM_LOOP
   for (int k = k0; k < k1; ++k) {
     const int i = idx(c, j, k);
     double pv = 0.0, pvl = 0.0, F = 0.0, m = 0.0, ef = 0.0, rr = 0.0, ee = 0.0, flo = 0.0, fhi = 0.0;
@@ -304,10 +353,10 @@ ks_advec_cell_x(Chunk c, const double* __restrict__ rho, const double* __restric
 // computes the flux of face k+1 and updates cell k (face k from the previous
 // iteration).  Registers hold density/energy of rows k-1..k+2 and the
 // pre-sweep volume of rows k, k+1.
-constexpr int CKS_Y = 32;
+constexpr int CKS_Y = CLOVER_CKS_Y;
 
 template <int SWEEP>
-__global__ void __launch_bounds__(SB)
+__global__ void LB_ADV
 ks_advec_cell_y(Chunk c, const double* __restrict__ rho, const double* __restrict__ en,
                 const double* __restrict__ fx, const double* __restrict__ fy,
                 double* __restrict__ rho_out, double* __restrict__ en_out,
@@ -344,6 +393,7 @@ ks_advec_cell_y(Chunk c, const double* __restrict__ rho, const double* __restric
       cell_face_flux(x, F, pvd, ru, rd, rw, eu, ed, ew, m0, ef0);
     }
   }
+  STREAM_LOOP
   for (int k = k0; k < k1; ++k, i += P) {
     // registers: R1..R3 = rows k-1..k+1; load row k+2
     const double R4 = rho[i + 2 * P], E4 = en[i + 2 * P];
@@ -392,10 +442,10 @@ ks_advec_cell_y(Chunk c, const double* __restrict__ rho, const double* __restric
 // fluxes of faces j, j+1 (rows k-1, k), node masses from cells j-1, j
 // (rows k-1, k; column j-1 via shuffle), momentum fluxes for u and v.
 constexpr int MW_X = 29;
-constexpr int MKS = 16;
+constexpr int MKS = CLOVER_MKS;
 
 template <int SWEEP>
-__global__ void __launch_bounds__(SB)
+__global__ void LB_ADV
 ks_advec_mom_x(Chunk c, const double* __restrict__ rho, const double* __restrict__ mfx,
                const double* __restrict__ fy, const double* __restrict__ uin,
                const double* __restrict__ vin, double* __restrict__ uout,
@@ -420,6 +470,7 @@ ks_advec_mom_x(Chunk c, const double* __restrict__ rho, const double* __restrict
     mA_m = mfx[i]; mB_m = mfx[i + 1]; mp_m = mass_post(i);
   }
   double mpl_m = __shfl_up_sync(FULL, mp_m, 1);
+  STREAM_LOOP
   for (int k = k0; k < k1; ++k) {
     const int i = idx(c, j, k);
     double mA = 0.0, mB = 0.0, mp = 0.0;
@@ -472,10 +523,10 @@ ks_advec_mom_x(Chunk c, const double* __restrict__ rho, const double* __restrict
 // Column j = block*128 + tid + 1 (node column), streams node rows [k0, k1).
 // Iteration k computes node flux / node masses of row k+1, the momentum
 // flux of row k and updates node k.
-constexpr int MKS_Y = 32;
+constexpr int MKS_Y = CLOVER_MKS_Y;
 
 template <int SWEEP>
-__global__ void __launch_bounds__(SB)
+__global__ void LB_ADV
 ks_advec_mom_y(Chunk c, const double* __restrict__ rho, const double* __restrict__ mfy,
                const double* __restrict__ fx, const double* __restrict__ uin,
                const double* __restrict__ vin, double* __restrict__ uout,
@@ -525,6 +576,7 @@ ks_advec_mom_y(Chunk c, const double* __restrict__ rho, const double* __restrict
       mom_flux2(x, nf, nmp, uu, vv, c.dy, mu_m, mv_m);
     }
   }
+  STREAM_LOOP
   for (int k = k0; k < k1; ++k, i += P) {
     // registers: U1..U3 = rows k-1..k+1 ; load row k+2
     const double U4 = uin[i + 2 * P], V4 = vin[i + 2 * P];
