@@ -138,6 +138,172 @@ ks_visc_dt(Chunk c, const double* __restrict__ d0, const double* __restrict__ e0
 constexpr int LW = 30;   // owned columns per warp
 constexpr int LKS = CLOVER_LKS;  // rows per segment
 
+#ifndef CLOVER_TMA_LAGR
+#define CLOVER_TMA_LAGR 1
+#endif
+#if CLOVER_TMA_LAGR
+// TMA-staged variant: rows of d0, e0, q (cells) and u0, v0 (nodes) stream
+// through a per-warp LSTG-stage shared-memory ring filled by cp.async.bulk,
+// so the DRAM latency of row k+LSTG-1 overlaps the compute of row k.
+constexpr int LRW = 36;   // doubles per staged row segment (>= 34, 16-B multiple)
+constexpr int LSTG = 4;   // ring stages
+enum { LF_R, LF_E, LF_Q, LF_U, LF_V, LNF };
+
+__global__ void LB_HEAVY
+ks_lagrangian(Chunk c, const double* __restrict__ d0, const double* __restrict__ e0,
+              const double* __restrict__ u0, const double* __restrict__ v0,
+              const double* __restrict__ q, double* __restrict__ d1, double* __restrict__ e1,
+              double* __restrict__ u1, double* __restrict__ v1, double* __restrict__ fx,
+              double* __restrict__ fy, const StepScalars* __restrict__ s) {
+  __shared__ __align__(128) double ring[SB / 32][LSTG][LNF][LRW];
+  __shared__ __align__(8) unsigned long long bars[SB / 32][LSTG];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const int gw = blockIdx.x * (SB / 32) + w;
+  const int J0 = 1 + LW * gw;
+  const int j = J0 - 1 + lane;
+  if (J0 > c.nx) return;  // whole warp beyond the chunk (rings are per warp)
+  const int k0 = blockIdx.y * LKS + 1;
+  const int k1 = min(k0 + LKS, c.ny + 1);  // cell rows [k0, k1)
+  const double dt = s->dt, dx = c.dx, dy = c.dy;
+  const int P = c.pitch;
+  const bool colok = j <= c.nx + 1;
+  int src = lane;
+  if (c.wl && j == 0) src = lane + 1;
+  if (c.wr && j == c.nx + 1) src = lane - 1;
+  const bool xwall_warp = __any_sync(FULL, src != lane);
+
+  // staged window: memory columns [mstart, mstart+ncopy), covering j-1..j+1
+  const int mstart = (COL0 + J0 - 1) & ~1;
+  int ncopy = ((COL0 + J0 + 31 - mstart + 1) + 1) & ~1;
+  if (mstart + ncopy > P) ncopy = P - mstart;
+  const int off = COL0 + j - mstart;  // smem index of column j
+  const unsigned bytes = (unsigned)ncopy * 8u;
+  const double* fields[LNF] = {d0, e0, q, u0, v0};
+  const int r_first = k0 - 1, r_last = k1 + 1;  // staged rows
+  auto issue = [&](int r) {
+    const int rel = r - r_first, slot = rel % LSTG;
+    mbar_arrive_expect_tx(&bars[w][slot], bytes * LNF);
+#pragma unroll
+    for (int f = 0; f < LNF; ++f)
+      tma_load_1d(&ring[w][slot][f][0], fields[f] + (size_t)r * P + (mstart - COL0), bytes, &bars[w][slot]);
+  };
+  auto wait_row = [&](int r) {
+    const int rel = r - r_first;
+    mbar_wait(&bars[w][rel % LSTG], (unsigned)((rel / LSTG) & 1));
+  };
+  if (lane == 0) {
+    for (int t = 0; t < LSTG; ++t) mbar_init(&bars[w][t], 1);
+    fence_mbar_init();
+    fence_proxy_async();
+    for (int r = r_first; r < r_first + LSTG && r <= r_last; ++r) issue(r);
+  }
+  __syncwarp();
+
+  double r_m = 1.0, e_m = 0.0, q_m = 0.0, ph_m = 0.0;
+  double rl_m = 1.0, phl_m = 0.0, ql_m = 0.0;
+  double u0_m = 0.0, v0_m = 0.0, u0r_m = 0.0, v0r_m = 0.0;
+  double u1_m = 0.0, v1_m = 0.0;
+  wait_row(r_first);
+  for (int k = k0 - 1; k <= k1; ++k) {
+    wait_row(k + 1);
+    const double* rowc = &ring[w][(k - r_first) % LSTG][0][0];
+    const double* rown = &ring[w][(k + 1 - r_first) % LSTG][0][0];
+    const double u0_c = rowc[LF_U * LRW + off], v0_c = rowc[LF_V * LRW + off];
+    const double u0r_c = rowc[LF_U * LRW + off + 1], v0r_c = rowc[LF_V * LRW + off + 1];
+    double r = 1.0, e = 0.0, qq = 0.0, ph = 0.0;
+    if (colok) {
+      r = rowc[LF_R * LRW + off]; e = rowc[LF_E * LRW + off]; qq = rowc[LF_Q * LRW + off];
+      const double u0_n = rown[LF_U * LRW + off], v0_n = rown[LF_V * LRW + off];
+      const double u0r_n = rown[LF_U * LRW + off + 1], v0r_n = rown[LF_V * LRW + off + 1];
+      int kp = k;
+      if (c.wb && k == 0) kp = 1;
+      if (c.wt && k == c.ny + 1) kp = c.ny;
+      double pr_, pe_, pq_, ua, ub, uc, ud, va, vb, vc, vd;
+      if (kp == k) {
+        pr_ = r; pe_ = e; pq_ = qq;
+        ua = u0_c; ub = u0_n; uc = u0r_c; ud = u0r_n;
+        va = v0_c; vb = v0r_c; vc = v0_n; vd = v0r_n;
+      } else {
+        const int ip = idx(c, j, kp);
+        pr_ = d0[ip]; pe_ = e0[ip]; pq_ = q[ip];
+        ua = u0[ip]; ub = u0[ip + P]; uc = u0[ip + 1]; ud = u0[ip + P + 1];
+        va = v0[ip]; vb = v0[ip + 1]; vc = v0[ip + P]; vd = v0[ip + P + 1];
+      }
+      DivFast f;
+      ph = pdv_predict_pressure(f, pr_, pe_, pq_, ua, ub, uc, ud, va, vb, vc, vd, dx, dy, dt);
+      if (f.bad) {
+        DivIEEE x;
+        ph = pdv_predict_pressure(x, pr_, pe_, pq_, ua, ub, uc, ud, va, vb, vc, vd, dx, dy, dt);
+      }
+    }
+    if (xwall_warp) ph = __shfl_sync(FULL, ph, src);
+    const double rl = __shfl_up_sync(FULL, r, 1);
+    const double phl = __shfl_up_sync(FULL, ph, 1);
+    const double ql = __shfl_up_sync(FULL, qq, 1);
+
+    double u1_c = 0.0, v1_c = 0.0;
+    if (k >= k0 && colok) {
+      const double rr[4] = {rl_m, r_m, r, rl};
+      const double pp[4] = {phl_m, ph_m, ph, phl};
+      const double qv[4] = {ql_m, q_m, qq, ql};
+      DivFast f;
+      accelerate_node(f, rr, pp, qv, u0_c, v0_c, dx, dy, dt, u1_c, v1_c);
+      if (f.bad) {
+        DivIEEE x;
+        accelerate_node(x, rr, pp, qv, u0_c, v0_c, dx, dy, dt, u1_c, v1_c);
+      }
+    }
+    const double u1r_c = __shfl_down_sync(FULL, u1_c, 1);
+    const double v1r_c = __shfl_down_sync(FULL, v1_c, 1);
+    const double u1r_m = __shfl_down_sync(FULL, u1_m, 1);
+    const double v1r_m = __shfl_down_sync(FULL, v1_m, 1);
+
+    const int kc = k - 1;
+    if (kc >= k0 && lane >= 1 && lane <= LW && j <= c.nx) {
+      const double lsum = u0_m + u0_c + u1_m + u1_c;
+      const double rsum = u0r_m + u0r_c + u1r_m + u1r_c;
+      const double bsum = v0_m + v0r_m + v1_m + v1r_m;
+      const double tsum = v0_c + v0r_c + v1_c + v1r_c;
+      double ev, dvv;
+      DivFast f;
+      pdv_correct(f, r_m, e_m, ph_m, q_m, lsum, rsum, bsum, tsum, dx, dy, dt, ev, dvv);
+      if (f.bad) {
+        DivIEEE x;
+        pdv_correct(x, r_m, e_m, ph_m, q_m, lsum, rsum, bsum, tsum, dx, dy, dt, ev, dvv);
+      }
+      store_field(c, e1, K_CELL, j, kc, ev);
+      store_field(c, d1, K_CELL, j, kc, dvv);
+      const double cx = 0.25 * dt * dy, cy = 0.25 * dt * dx;
+      store_field(c, fx, K_XFACE, j, kc, cx * lsum);
+      store_field(c, fy, K_YFACE, j, kc, cy * bsum);
+      if (j == c.nx) store_field(c, fx, K_XFACE, j + 1, kc, cx * rsum);
+      if (kc == c.ny) store_field(c, fy, K_YFACE, j, kc + 1, cy * tsum);
+      store_field(c, u1, K_XVEL, j, kc, u1_m);
+      store_field(c, v1, K_YVEL, j, kc, v1_m);
+      if (j == c.nx) {
+        store_field(c, u1, K_XVEL, j + 1, kc, u1r_m);
+        store_field(c, v1, K_YVEL, j + 1, kc, v1r_m);
+      }
+      if (kc == c.ny) {
+        store_field(c, u1, K_XVEL, j, kc + 1, u1_c);
+        store_field(c, v1, K_YVEL, j, kc + 1, v1_c);
+      }
+      if (j == c.nx && kc == c.ny) {
+        store_field(c, u1, K_XVEL, j + 1, kc + 1, u1r_c);
+        store_field(c, v1, K_YVEL, j + 1, kc + 1, v1r_c);
+      }
+    }
+    r_m = r; e_m = e; q_m = qq; ph_m = ph;
+    rl_m = rl; phl_m = phl; ql_m = ql;
+    u0_m = u0_c; v0_m = v0_c; u0r_m = u0r_c; v0r_m = v0r_c;
+    u1_m = u1_c; v1_m = v1_c;
+    // row k is consumed: refill its slot with row k+LSTG
+    fence_proxy_async();
+    __syncwarp();
+    if (lane == 0 && k + LSTG <= r_last) issue(k + LSTG);
+  }
+}
+#else
 __global__ void LB_HEAVY
 ks_lagrangian(Chunk c, const double* __restrict__ d0, const double* __restrict__ e0,
               const double* __restrict__ u0, const double* __restrict__ v0,
@@ -272,6 +438,8 @@ ks_lagrangian(Chunk c, const double* __restrict__ d0, const double* __restrict__
     u1_m = u1_c; v1_m = v1_c;
   }
 }
+
+#endif  // CLOVER_TMA_LAGR
 
 // ================================================================ advec_cell x
 // Warp strip: lane l <-> face/cell column j = J0 + l, J0 = 1 + 31*(warp);
