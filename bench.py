@@ -115,12 +115,6 @@ class ClockSampler:
                 "reasons": sorted(reasons), "samples": len(self.rows)}
 
 
-def weak_mesh(n):
-    """Reading A4: per-GPU 3840^2, chunk grid px x py."""
-    return {1: (3840, 3840, 1, 1), 2: (7680, 3840, 2, 1), 4: (7680, 7680, 2, 2),
-            8: (15360, 7680, 4, 2)}.get(n)
-
-
 def oracle_rate(deck, steps, warmup=0):
     """Time the CPU oracle (as it stands, single-threaded) on `deck`."""
     from oracle import Oracle
@@ -181,6 +175,8 @@ def main():
     ap.add_argument("--mesh", type=int, nargs=2, default=None, help="override global mesh (nx ny)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--strong", action="store_true",
+                    help="configs[3]: 7680^2 strong-scaled over the ranks (default: configs[4] weak)")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
@@ -198,19 +194,21 @@ def main():
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     from paper_conf_cluster_regulymg15_b200 import Clover, nccl_unique_id
+    from paper_conf_cluster_regulymg15_b200 import dist as cdist
     from workloads import bm_deck
 
     if world > 1:
         dist.init_process_group("nccl", device_id=dev)
-    nx, ny, px, py = weak_mesh(world) or (3840 * world, 3840, world, 1)
+    if args.strong:
+        nx, ny = 7680, 7680
+        px, py = cdist.chunk_grid(world, nx, ny)
+    else:
+        nx, ny, px, py = cdist.weak_mesh(world)
     if args.mesh:
         nx, ny = args.mesh
+        px, py = cdist.chunk_grid(world, nx, ny)
     deck = bm_deck(nx, ny, end_step=args.steps)
-    uid = None
-    if world > 1:
-        obj = [nccl_unique_id() if rank == 0 else None]
-        dist.broadcast_object_list(obj, src=0)
-        uid = obj[0]
+    uid = cdist.share_unique_id(nccl_unique_id) if world > 1 else None
     stream = torch.cuda.Stream(dev)
     sim = Clover(deck, px=px, py=py, rank=rank, nranks=world, unique_id=uid, stream=stream)
     cells = nx * ny
@@ -233,10 +231,7 @@ def main():
     ms = e0.elapsed_time(e1)
     clk = clocks.stop()
     sim.sync()
-    if world > 1:
-        t = torch.tensor([ms], device=dev, dtype=torch.float64)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        ms = float(t.item())
+    ms = cdist.max_over_ranks(ms, dev)
     value = cells * args.steps / (ms / 1000.0)
     kps = sim.kernels_per_step()
 
@@ -306,11 +301,14 @@ def main():
     if rank == 0:
         line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
                 "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms / args.steps,
-                "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+                "higher_is_better": True, "scaling": "strong" if args.strong else "weak",
+                "vs_baseline": None,
                 "dtype": "f64", "data": "synthetic",
-                "config": {"workload": ("configs[2]: CloverLeaf 2D bm deck 3840x3840 (clover_bm16 shape), "
-                                        "1 GPU bandwidth-roofline run") if world == 1 else
-                           f"configs[4]: weak scaling, 3840^2 cells per GPU, global {nx}x{ny}",
+                "config": {"workload": ("configs[3]: CloverLeaf 2D bm deck 7680x7680 strong-scaled"
+                                        if args.strong else
+                                        "configs[2]: CloverLeaf 2D bm deck 3840x3840 (clover_bm16 shape), "
+                                        "1 GPU bandwidth-roofline run" if world == 1 else
+                                        f"configs[4]: weak scaling, 3840^2 cells per GPU, global {nx}x{ny}"),
                            "mesh": [nx, ny], "decomposition": f"{px}x{py}",
                            "l2": "inputs larger than L2 (18 fp64 fields of the mesh, >2 GB vs 126 MB L2)",
                            "graphs": True},

@@ -1,0 +1,53 @@
+"""Multi-process plumbing for one-process-per-GPU runs (torch.distributed):
+chunk-grid choice, NCCL unique-id broadcast and max-over-ranks timing.
+The halo exchange and the dt MIN all-reduce themselves run inside
+libclover.so over NCCL; this module only sets them up.
+"""
+from __future__ import annotations
+
+import torch
+import torch.distributed as dist
+
+
+def chunk_grid(nranks: int, nx: int, ny: int) -> tuple[int, int]:
+    """px x py chunks for nranks ranks, one chunk per rank: the most square
+    chunks, splitting the longer axis first (the reference's
+    clover_decompose idea; 2 -> 1x2 on a square mesh)."""
+    best = None
+    for px in range(1, nranks + 1):
+        if nranks % px:
+            continue
+        py = nranks // px
+        lx, ly = nx / px, ny / py
+        score = (max(lx, ly) / min(lx, ly), -py)  # squarest, then prefer y splits
+        if best is None or score < best[0]:
+            best = (score, px, py)
+    return best[1], best[2]
+
+
+def weak_mesh(nranks: int, per: int = 3840) -> tuple[int, int, int, int]:
+    """Reading A4: per-rank per^2 cells; global mesh and chunk grid."""
+    table = {1: (1, 1), 2: (2, 1), 4: (2, 2), 8: (4, 2)}
+    px, py = table.get(nranks, (nranks, 1))
+    return per * px, per * py, px, py
+
+
+def share_unique_id(make_id) -> bytes:
+    """Rank 0 creates the 128-byte NCCL unique id (make_id()), every rank
+    returns the same bytes."""
+    obj = [make_id() if dist.get_rank() == 0 else None]
+    dist.broadcast_object_list(obj, src=0)
+    uid = obj[0]
+    if not isinstance(uid, (bytes, bytearray)) or len(uid) != 128:
+        raise ValueError("bad NCCL unique id")
+    return bytes(uid)
+
+
+def max_over_ranks(value: float, device=None) -> float:
+    """Max of a per-rank timing over all ranks (the bench reports the
+    slowest rank)."""
+    if not dist.is_initialized() or dist.get_world_size() == 1:
+        return float(value)
+    t = torch.tensor([float(value)], dtype=torch.float64, device=device)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())

@@ -72,9 +72,11 @@ if os.path.exists(rep):
           "(units as reported: " + units[hdr.index('dram__bytes_read.sum')] + ").\n",
           "| kernel | time us | DRAM read | DRAM write | DRAM GB/s | issue % | fp64 pipe % | warps active % | regs | thread inst/cell |",
           "|---|---|---|---|---|---|---|---|---|---|"]
+    tunit = units[hdr.index("gpu__time_duration.sum")]
+    tscale = {"ns": 1.0, "nsecond": 1.0, "us": 1e3, "usecond": 1e3, "ms": 1e6, "msecond": 1e6}.get(tunit, 1.0)
     for r in data:
         n = short(r[hdr.index("Kernel Name")])
-        t = g(r, "gpu__time_duration.sum")
+        t = g(r, "gpu__time_duration.sum") * tscale  # ns
         rd, wr = g(r, "dram__bytes_read.sum"), g(r, "dram__bytes_write.sum")
         unit = units[hdr.index("dram__bytes_read.sum")]
         scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}.get(unit, 1)
