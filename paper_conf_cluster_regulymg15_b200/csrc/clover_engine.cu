@@ -345,7 +345,6 @@ int exchange(clover_ctx* ctx, const std::vector<int>& bufs) {
 
 // ---------------------------------------------------------------- schedule
 dim3 cell_grid(const Chunk& c, int bx, int by) { return dim3((c.nx + bx - 1) / bx, (c.ny + by - 1) / by); }
-dim3 node_grid(const Chunk& c, int bx, int by) { return dim3((c.nx + 1 + bx - 1) / bx, (c.ny + 1 + by - 1) / by); }
 
 #define LAUNCH_CHECK()                                                            \
   do {                                                                            \
@@ -696,6 +695,10 @@ int clover_init(const clover_grid* grid, const clover_state* states, int32_t nst
     c.wl = cs.cx == 0; c.wr = cs.cx == px - 1; c.wb = cs.cy == 0; c.wt = cs.cy == py - 1;
     c.face_cc = ctx->g.face_mirror == CLOVER_MIRROR_CELLCENTRE;
     c.dx = dx; c.dy = dy; c.xmin = ctx->g.xmin; c.ymin = ctx->g.ymin;
+    // correctly rounded reciprocals of the constant divisors (IEEE host division)
+    c.rdx = 1.0 / dx; c.rdy = 1.0 / dy;
+    c.r2dx = 1.0 / (dx + dx); c.r2dy = 1.0 / (dy + dy);
+    c.rvol = 1.0 / (dx * dy); c.r2vol = 1.0 / (2.0 * (dx * dy));
     for (int b = 0; b < NBUF; ++b) {
       cs.buf[b] = (double*)p + (int64_t)ROW0 * c.pitch + COL0;
       p += align_up(fe * 8, kAlign);
@@ -872,7 +875,13 @@ __global__ void k_div_check(long long n, unsigned long long seed, int emax,
     double q1 = f(a, b);
     if (f.bad) q1 = a / b;
     const double q2 = a / b;
-    if (__double_as_longlong(q1) != __double_as_longlong(q2)) {
+    // constant-divisor form with the correctly rounded reciprocal
+    clover::DivFast fc;
+    const double rb = 1.0 / b;
+    double q3 = fc.c(a, b, rb);
+    if (fc.bad) q3 = a / b;
+    if (__double_as_longlong(q1) != __double_as_longlong(q2) ||
+        __double_as_longlong(q3) != __double_as_longlong(q2)) {
       if (atomicAdd(bad, 1ull) == 0) { example[0] = a; example[1] = b; }
     }
   }

@@ -103,10 +103,10 @@ ks_visc_dt(Chunk c, const double* __restrict__ d0, const double* __restrict__ e0
       I.v00 = va; I.v10 = vb; I.v01 = vc; I.v11 = vd;
       double qv;
       DivFast f;
-      double dtc = visc_dt_cell(f, I, c.dx, c.dy, prm, qv);
+      double dtc = visc_dt_cell(f, I, c, prm, qv);
       if (f.bad) {
         DivIEEE x;
-        dtc = visc_dt_cell(x, I, c.dx, c.dy, prm, qv);
+        dtc = visc_dt_cell(x, I, c, prm, qv);
       }
       dtl = fmin(dtl, dtc);
       store_field(c, q, K_CELL, j, k, qv);
@@ -230,10 +230,10 @@ ks_lagrangian(Chunk c, const double* __restrict__ d0, const double* __restrict__
         va = v0[ip]; vb = v0[ip + 1]; vc = v0[ip + P]; vd = v0[ip + P + 1];
       }
       DivFast f;
-      ph = pdv_predict_pressure(f, pr_, pe_, pq_, ua, ub, uc, ud, va, vb, vc, vd, dx, dy, dt);
+      ph = pdv_predict_pressure(f, pr_, pe_, pq_, ua, ub, uc, ud, va, vb, vc, vd, dx, dy, c.rvol, dt);
       if (f.bad) {
         DivIEEE x;
-        ph = pdv_predict_pressure(x, pr_, pe_, pq_, ua, ub, uc, ud, va, vb, vc, vd, dx, dy, dt);
+        ph = pdv_predict_pressure(x, pr_, pe_, pq_, ua, ub, uc, ud, va, vb, vc, vd, dx, dy, c.rvol, dt);
       }
     }
     if (xwall_warp) ph = __shfl_sync(FULL, ph, src);
@@ -266,10 +266,10 @@ ks_lagrangian(Chunk c, const double* __restrict__ d0, const double* __restrict__
       const double tsum = v0_c + v0r_c + v1_c + v1r_c;
       double ev, dvv;
       DivFast f;
-      pdv_correct(f, r_m, e_m, ph_m, q_m, lsum, rsum, bsum, tsum, dx, dy, dt, ev, dvv);
+      pdv_correct(f, r_m, e_m, ph_m, q_m, lsum, rsum, bsum, tsum, dx, dy, c.rvol, dt, ev, dvv);
       if (f.bad) {
         DivIEEE x;
-        pdv_correct(x, r_m, e_m, ph_m, q_m, lsum, rsum, bsum, tsum, dx, dy, dt, ev, dvv);
+        pdv_correct(x, r_m, e_m, ph_m, q_m, lsum, rsum, bsum, tsum, dx, dy, c.rvol, dt, ev, dvv);
       }
       store_field(c, e1, K_CELL, j, kc, ev);
       store_field(c, d1, K_CELL, j, kc, dvv);
@@ -364,10 +364,10 @@ ks_lagrangian(Chunk c, const double* __restrict__ d0, const double* __restrict__
         va = v0[ip]; vb = v0[ip + 1]; vc = v0[ip + P]; vd = v0[ip + P + 1];
       }
       DivFast f;
-      ph = pdv_predict_pressure(f, pr_, pe_, pq_, ua, ub, uc, ud, va, vb, vc, vd, dx, dy, dt);
+      ph = pdv_predict_pressure(f, pr_, pe_, pq_, ua, ub, uc, ud, va, vb, vc, vd, dx, dy, c.rvol, dt);
       if (f.bad) {
         DivIEEE x;
-        ph = pdv_predict_pressure(x, pr_, pe_, pq_, ua, ub, uc, ud, va, vb, vc, vd, dx, dy, dt);
+        ph = pdv_predict_pressure(x, pr_, pe_, pq_, ua, ub, uc, ud, va, vb, vc, vd, dx, dy, c.rvol, dt);
       }
     }
     if (xwall_warp) ph = __shfl_sync(FULL, ph, src);
@@ -403,10 +403,10 @@ ks_lagrangian(Chunk c, const double* __restrict__ d0, const double* __restrict__
       const double tsum = v0_c + v0r_c + v1_c + v1r_c;
       double ev, dvv;
       DivFast f;
-      pdv_correct(f, r_m, e_m, ph_m, q_m, lsum, rsum, bsum, tsum, dx, dy, dt, ev, dvv);
+      pdv_correct(f, r_m, e_m, ph_m, q_m, lsum, rsum, bsum, tsum, dx, dy, c.rvol, dt, ev, dvv);
       if (f.bad) {
         DivIEEE x;
-        pdv_correct(x, r_m, e_m, ph_m, q_m, lsum, rsum, bsum, tsum, dx, dy, dt, ev, dvv);
+        pdv_correct(x, r_m, e_m, ph_m, q_m, lsum, rsum, bsum, tsum, dx, dy, c.rvol, dt, ev, dvv);
       }
       store_field(c, e1, K_CELL, j, kc, ev);
       store_field(c, d1, K_CELL, j, kc, dvv);
@@ -663,10 +663,10 @@ ks_advec_mom_x(Chunk c, const double* __restrict__ rho, const double* __restrict
       const double uu[3] = {uin[i + up], uin[i + don], uin[i + dw]};
       const double vv[3] = {vin[i + up], vin[i + don], vin[i + dw]};
       DivFast f;
-      mom_flux2(f, nf, nmp, uu, vv, c.dx, mu, mv);
+      mom_flux2(f, nf, nmp, uu, vv, c.dx, c.rdx, mu, mv);
       if (f.bad) {
         DivIEEE x;
-        mom_flux2(x, nf, nmp, uu, vv, c.dx, mu, mv);
+        mom_flux2(x, nf, nmp, uu, vv, c.dx, c.rdx, mu, mv);
       }
     }
     const double mul = __shfl_up_sync(FULL, mu, 1);
@@ -738,10 +738,10 @@ ks_advec_mom_y(Chunk c, const double* __restrict__ rho, const double* __restrict
     const double uu[3] = {nf < 0.0 ? U3 : U0, nf < 0.0 ? U2 : U1, nf < 0.0 ? U1 : U2};
     const double vv[3] = {nf < 0.0 ? V3 : V0, nf < 0.0 ? V2 : V1, nf < 0.0 ? V1 : V2};
     DivFast f;
-    mom_flux2(f, nf, nmp, uu, vv, c.dy, mu_m, mv_m);
+    mom_flux2(f, nf, nmp, uu, vv, c.dy, c.rdy, mu_m, mv_m);
     if (f.bad) {
       DivIEEE x;
-      mom_flux2(x, nf, nmp, uu, vv, c.dy, mu_m, mv_m);
+      mom_flux2(x, nf, nmp, uu, vv, c.dy, c.rdy, mu_m, mv_m);
     }
   }
   STREAM_LOOP
@@ -759,10 +759,10 @@ ks_advec_mom_y(Chunk c, const double* __restrict__ rho, const double* __restrict
       const double uu[3] = {nf < 0.0 ? U4 : U1, nf < 0.0 ? U3 : U2, nf < 0.0 ? U2 : U3};
       const double vv[3] = {nf < 0.0 ? V4 : V1, nf < 0.0 ? V3 : V2, nf < 0.0 ? V2 : V3};
       DivFast f;
-      mom_flux2(f, nf, nmp, uu, vv, c.dy, mu, mv);
+      mom_flux2(f, nf, nmp, uu, vv, c.dy, c.rdy, mu, mv);
       if (f.bad) {
         DivIEEE x;
-        mom_flux2(x, nf, nmp, uu, vv, c.dy, mu, mv);
+        mom_flux2(x, nf, nmp, uu, vv, c.dy, c.rdy, mu, mv);
       }
     }
     double un, vn;
