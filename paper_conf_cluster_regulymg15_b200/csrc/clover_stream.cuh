@@ -33,17 +33,34 @@ constexpr int SB = 128;  // threads per block (4 warps)
 #endif
 // min resident blocks/SM (register cap) for visc_dt+lagrangian / advection;
 // 0 = plain __launch_bounds__(SB) (ptxas heuristic).  Measured on B200 at
-// 3840^2 (scripts/ab_variants.py): 5 / 8 best (1.79 -> 1.68 ms/step).
+// 3840^2 (scripts/ab_variants.py): lagrangian 5, visc_dt uncapped,
+// advection 8 (mom_y 7).
 #ifndef CLOVER_MINB_HEAVY
 #define CLOVER_MINB_HEAVY 5
 #endif
 #ifndef CLOVER_MINB_ADV
 #define CLOVER_MINB_ADV 8
 #endif
+#ifndef CLOVER_MINB_VISC
+#define CLOVER_MINB_VISC 0
+#endif
+#ifndef CLOVER_MINB_MOMY
+#define CLOVER_MINB_MOMY 7
+#endif
+#if CLOVER_MINB_MOMY > 0
+#define LB_MOMY __launch_bounds__(SB, CLOVER_MINB_MOMY)
+#else
+#define LB_MOMY __launch_bounds__(SB)
+#endif
 #if CLOVER_MINB_HEAVY > 0
 #define LB_HEAVY __launch_bounds__(SB, CLOVER_MINB_HEAVY)
 #else
 #define LB_HEAVY __launch_bounds__(SB)
+#endif
+#if CLOVER_MINB_VISC > 0
+#define LB_VISC __launch_bounds__(SB, CLOVER_MINB_VISC)
+#else
+#define LB_VISC __launch_bounds__(SB)
 #endif
 #if CLOVER_MINB_ADV > 0
 #define LB_ADV __launch_bounds__(SB, CLOVER_MINB_ADV)
@@ -74,7 +91,7 @@ constexpr int SB = 128;  // threads per block (4 warps)
 // the row below, density/energy of the row above, the 4 node velocities.
 constexpr int VKS = CLOVER_VKS;
 
-__global__ void LB_HEAVY
+__global__ void LB_VISC
 ks_visc_dt(Chunk c, const double* __restrict__ d0, const double* __restrict__ e0,
            const double* __restrict__ u0, const double* __restrict__ v0, double* __restrict__ q,
            StepScalars* __restrict__ s, DtParams prm) {
@@ -84,6 +101,7 @@ ks_visc_dt(Chunk c, const double* __restrict__ d0, const double* __restrict__ e0
   double dtl = G_BIG;
   if (j <= c.nx) {
     const int P = c.pitch;
+    const bool ncol = near_wall_col(c, j);
     int i = idx(c, j, k0);
     double pcm = eos_pressure(d0[i - P], e0[i - P]);
     double rho = d0[i], ein = e0[i];
@@ -109,7 +127,7 @@ ks_visc_dt(Chunk c, const double* __restrict__ d0, const double* __restrict__ e0
         dtc = visc_dt_cell(x, I, c, prm, qv);
       }
       dtl = fmin(dtl, dtc);
-      store_field(c, q, K_CELL, j, k, qv);
+      store_at(c, q, K_CELL, j, k, i, ncol || near_wall_row(c, k), qv);
       pcm = pc; pc = I.pt; rho = rhon; ein = en;
       ua = uc; ub = ud; va = vc; vb = vd;
     }
@@ -167,6 +185,7 @@ ks_lagrangian(Chunk c, const double* __restrict__ d0, const double* __restrict__
   const double dt = s->dt, dx = c.dx, dy = c.dy;
   const int P = c.pitch;
   const bool colok = j <= c.nx + 1;
+  const bool ncol = near_wall_col(c, j);
   int src = lane;
   if (c.wl && j == 0) src = lane + 1;
   if (c.wr && j == c.nx + 1) src = lane - 1;
@@ -271,15 +290,17 @@ ks_lagrangian(Chunk c, const double* __restrict__ d0, const double* __restrict__
         DivIEEE x;
         pdv_correct(x, r_m, e_m, ph_m, q_m, lsum, rsum, bsum, tsum, dx, dy, c.rvol, dt, ev, dvv);
       }
-      store_field(c, e1, K_CELL, j, kc, ev);
-      store_field(c, d1, K_CELL, j, kc, dvv);
+      const int ic = idx(c, j, kc);
+      const bool near = ncol || near_wall_row(c, kc);
+      store_at(c, e1, K_CELL, j, kc, ic, near, ev);
+      store_at(c, d1, K_CELL, j, kc, ic, near, dvv);
       const double cx = 0.25 * dt * dy, cy = 0.25 * dt * dx;
-      store_field(c, fx, K_XFACE, j, kc, cx * lsum);
-      store_field(c, fy, K_YFACE, j, kc, cy * bsum);
+      store_at(c, fx, K_XFACE, j, kc, ic, near, cx * lsum);
+      store_at(c, fy, K_YFACE, j, kc, ic, near, cy * bsum);
       if (j == c.nx) store_field(c, fx, K_XFACE, j + 1, kc, cx * rsum);
       if (kc == c.ny) store_field(c, fy, K_YFACE, j, kc + 1, cy * tsum);
-      store_field(c, u1, K_XVEL, j, kc, u1_m);
-      store_field(c, v1, K_YVEL, j, kc, v1_m);
+      store_at(c, u1, K_XVEL, j, kc, ic, near, u1_m);
+      store_at(c, v1, K_YVEL, j, kc, ic, near, v1_m);
       if (j == c.nx) {
         store_field(c, u1, K_XVEL, j + 1, kc, u1r_m);
         store_field(c, v1, K_YVEL, j + 1, kc, v1r_m);
@@ -408,15 +429,17 @@ ks_lagrangian(Chunk c, const double* __restrict__ d0, const double* __restrict__
         DivIEEE x;
         pdv_correct(x, r_m, e_m, ph_m, q_m, lsum, rsum, bsum, tsum, dx, dy, c.rvol, dt, ev, dvv);
       }
-      store_field(c, e1, K_CELL, j, kc, ev);
-      store_field(c, d1, K_CELL, j, kc, dvv);
+      const int ic = idx(c, j, kc);
+      const bool near = ncol || near_wall_row(c, kc);
+      store_at(c, e1, K_CELL, j, kc, ic, near, ev);
+      store_at(c, d1, K_CELL, j, kc, ic, near, dvv);
       const double cx = 0.25 * dt * dy, cy = 0.25 * dt * dx;
-      store_field(c, fx, K_XFACE, j, kc, cx * lsum);
-      store_field(c, fy, K_YFACE, j, kc, cy * bsum);
+      store_at(c, fx, K_XFACE, j, kc, ic, near, cx * lsum);
+      store_at(c, fy, K_YFACE, j, kc, ic, near, cy * bsum);
       if (j == c.nx) store_field(c, fx, K_XFACE, j + 1, kc, cx * rsum);
       if (kc == c.ny) store_field(c, fy, K_YFACE, j, kc + 1, cy * tsum);
-      store_field(c, u1, K_XVEL, j, kc, u1_m);
-      store_field(c, v1, K_YVEL, j, kc, v1_m);
+      store_at(c, u1, K_XVEL, j, kc, ic, near, u1_m);
+      store_at(c, v1, K_YVEL, j, kc, ic, near, v1_m);
       if (j == c.nx) {
         store_field(c, u1, K_XVEL, j + 1, kc, u1r_m);
         store_field(c, v1, K_YVEL, j + 1, kc, v1r_m);
@@ -464,6 +487,7 @@ ks_advec_cell_x(Chunk c, const double* __restrict__ rho, const double* __restric
   const double vol = c.dx * c.dy;
   const int P = c.pitch;
   const bool faceok = j <= c.nx + 1;
+  const bool ncol = near_wall_col(c, j);
   STREAM_LOOP
   for (int k = k0; k < k1; ++k) {
     const int i = idx(c, j, k);
@@ -508,9 +532,10 @@ ks_advec_cell_x(Chunk c, const double* __restrict__ rho, const double* __restric
         DivIEEE x;
         cell_update(x, rr, ee, pv, m, mh, ef, efh, flo, fhi, ro, eo);
       }
-      store_field(c, rho_out, K_CELL, j, k, ro);
-      store_field(c, en_out, K_CELL, j, k, eo);
-      store_field(c, mfx, K_XFACE, j, k, m);
+      const bool near = ncol || near_wall_row(c, k);
+      store_at(c, rho_out, K_CELL, j, k, i, near, ro);
+      store_at(c, en_out, K_CELL, j, k, i, near, eo);
+      store_at(c, mfx, K_XFACE, j, k, i, near, m);
       if (j == c.nx) store_field(c, mfx, K_XFACE, j + 1, k, mh);
     }
   }
@@ -539,6 +564,7 @@ ks_advec_cell_y(Chunk c, const double* __restrict__ rho, const double* __restric
     if (SWEEP == 1) return vol + (fy[i + P] - fy[i] + fx[i + 1] - fx[i]);
     return vol + fy[i + P] - fy[i];
   };
+  const bool ncol = near_wall_col(c, j);
   int i = idx(c, j, k0);
   // rows k0-2 .. k0+1
   double R0 = rho[i - 2 * P], R1 = rho[i - P], R2 = rho[i], R3 = rho[i + P];
@@ -593,9 +619,10 @@ ks_advec_cell_y(Chunk c, const double* __restrict__ rho, const double* __restric
         cell_update(x, R2, E2, pv0, m0, m1, ef0, ef1, flo, fhi, ro, eo);
       }
     }
-    store_field(c, rho_out, K_CELL, j, k, ro);
-    store_field(c, en_out, K_CELL, j, k, eo);
-    store_field(c, mfy, K_YFACE, j, k, m0);
+    const bool near = ncol || near_wall_row(c, k);
+    store_at(c, rho_out, K_CELL, j, k, i, near, ro);
+    store_at(c, en_out, K_CELL, j, k, i, near, eo);
+    store_at(c, mfy, K_YFACE, j, k, i, near, m0);
     if (k == c.ny) store_field(c, mfy, K_YFACE, j, k + 1, m1);
     R0 = R1; R1 = R2; R2 = R3; R3 = R4;
     E0 = E1; E1 = E2; E2 = E3; E3 = E4;
@@ -628,6 +655,7 @@ ks_advec_mom_x(Chunk c, const double* __restrict__ rho, const double* __restrict
   const double vol = c.dx * c.dy;
   const int P = c.pitch;
   const bool nfok = j <= c.nx + 2;   // node flux / node mass columns
+  const bool ncol = near_wall_col(c, j);
   auto mass_post = [&](int i) -> double {
     const double pv = (SWEEP == 1) ? vol + fy[i + P] - fy[i] : vol;
     return rho[i] * pv;
@@ -680,8 +708,9 @@ ks_advec_mom_x(Chunk c, const double* __restrict__ rho, const double* __restrict
         DivIEEE x;
         mom_update(x, u, v, pre, post, mul, mu, mvl, mv, un, vn);
       }
-      store_field(c, uout, K_XVEL, j, k, un);
-      store_field(c, vout, K_YVEL, j, k, vn);
+      const bool near = ncol || near_wall_row(c, k);
+      store_at(c, uout, K_XVEL, j, k, i, near, un);
+      store_at(c, vout, K_YVEL, j, k, i, near, vn);
     }
     mA_m = mA; mB_m = mB; mp_m = mp; mpl_m = mpl;
   }
@@ -694,7 +723,7 @@ ks_advec_mom_x(Chunk c, const double* __restrict__ rho, const double* __restrict
 constexpr int MKS_Y = CLOVER_MKS_Y;
 
 template <int SWEEP>
-__global__ void LB_ADV
+__global__ void LB_MOMY
 ks_advec_mom_y(Chunk c, const double* __restrict__ rho, const double* __restrict__ mfy,
                const double* __restrict__ fx, const double* __restrict__ uin,
                const double* __restrict__ vin, double* __restrict__ uout,
@@ -709,6 +738,7 @@ ks_advec_mom_y(Chunk c, const double* __restrict__ rho, const double* __restrict
     const double pv = (SWEEP == 1) ? vol + fx[i + 1] - fx[i] : vol;
     return rho[i] * pv;
   };
+  const bool ncol = near_wall_col(c, j);
   // node flux of row r uses My(j-1,r), My(j,r), My(j-1,r+1), My(j,r+1)
   auto node_flux = [&](int i) -> double {
     return 0.25 * (mfy[i - 1] + mfy[i] + mfy[i - 1 + P] + mfy[i + P]);
@@ -774,8 +804,9 @@ ks_advec_mom_y(Chunk c, const double* __restrict__ rho, const double* __restrict
         mom_update(x, U2, V2, pre_0, post_0, mu_m, mu, mv_m, mv, un, vn);
       }
     }
-    store_field(c, uout, K_XVEL, j, k, un);
-    store_field(c, vout, K_YVEL, j, k, vn);
+    const bool near = ncol || near_wall_row(c, k);
+    store_at(c, uout, K_XVEL, j, k, i, near, un);
+    store_at(c, vout, K_YVEL, j, k, i, near, vn);
     U1 = U2; U2 = U3; U3 = U4;
     V1 = V2; V2 = V3; V3 = V4;
     mpj_c = mpj_d; mpl_c = mpl_d;
