@@ -206,6 +206,25 @@ int clover_debug_read_buffer(clover_ctx* ctx, int32_t buffer_id, int32_t kind,
 int clover_debug_div_check(int64_t n, uint64_t seed, int32_t emax, int64_t* mismatches,
                            double* example_ab);
 
+/* ---- checkpoint / restart (sec. VI)
+ * The library's access-execute description of one step (the reference's
+ * loops with their read/write datasets) decides what a checkpoint must hold:
+ * entering checkpoint mode before loop `loop` (0 = ideal_gas, i.e. the step
+ * boundary ... 12 = reset_field), a dataset is saved iff its first access in
+ * the periodic loop sequence is a read.  clover_checkpoint_plan returns that
+ * set as a bit mask (bit order: density0, energy0, xvel0, yvel0, pressure,
+ * soundspeed, viscosity, density1, energy1, xvel1, yvel1, vol_flux_x,
+ * vol_flux_y, mass_flux_x, mass_flux_y), its size and the loop's name.
+ * At the step boundary -- the optimum, where clover_checkpoint operates --
+ * it is {density0, energy0, xvel0, yvel0}; plus the clock (step, time, dt,
+ * dtold, sweep order).  Restarting from a checkpoint continues bit for bit.
+ * Single-process contexts; the buffer is host memory owned by the caller. */
+int clover_checkpoint_plan(int32_t loop, uint32_t* save_mask, int32_t* nsaved, const char** name);
+int clover_checkpoint_bytes(clover_ctx* ctx, int64_t* bytes);
+int clover_checkpoint(clover_ctx* ctx, void* host, int64_t bytes);
+/* Restore a checkpoint taken on the same mesh (CLOVER_ERR_ARG otherwise). */
+int clover_restart(clover_ctx* ctx, const void* host, int64_t bytes);
+
 /* Destroy the context (does not free the caller's workspace). */
 int clover_finalize(clover_ctx* ctx);
 

@@ -38,7 +38,8 @@ EXPORTS = ["clover_workspace_bytes", "clover_nccl_unique_id", "clover_init", "cl
            "clover_step_host", "clover_field_summary", "clover_get_clock", "clover_dt_history",
            "clover_read_field", "clover_write_field", "clover_sync", "clover_set_graphs",
            "clover_kernels_per_step", "clover_debug_partial_step", "clover_debug_read_buffer",
-           "clover_profile_steps", "clover_profile_name", "clover_debug_div_check", "clover_finalize", "clover_error_string", "clover_last_error", "clover_abi_version"]
+           "clover_profile_steps", "clover_profile_name", "clover_debug_div_check",
+           "clover_checkpoint_plan", "clover_checkpoint_bytes", "clover_checkpoint", "clover_restart", "clover_finalize", "clover_error_string", "clover_last_error", "clover_abi_version"]
 
 
 class CloverGrid(ctypes.Structure):
@@ -105,6 +106,11 @@ def load(build_if_missing: bool = True):
     L.clover_profile_name.argtypes = [c_int32]
     L.clover_profile_name.restype = ctypes.c_char_p
     L.clover_debug_div_check.argtypes = [c_int64, ctypes.c_uint64, c_int32, ctypes.POINTER(c_int64), dptr]
+    L.clover_checkpoint_plan.argtypes = [c_int32, ctypes.POINTER(ctypes.c_uint32), ctypes.POINTER(c_int32),
+                                         ctypes.POINTER(ctypes.c_char_p)]
+    L.clover_checkpoint_bytes.argtypes = [c_void_p, ctypes.POINTER(c_int64)]
+    L.clover_checkpoint.argtypes = [c_void_p, c_void_p, c_int64]
+    L.clover_restart.argtypes = [c_void_p, c_void_p, c_int64]
     L.clover_finalize.argtypes = [c_void_p]
     L.clover_error_string.argtypes = [c_int32]
     L.clover_error_string.restype = ctypes.c_char_p
@@ -166,6 +172,19 @@ def field_shape(name_or_kind: str, nx: int, ny: int):
     if k in ("vol_flux_y", "mass_flux_y", "yface"):
         return (ny + 1, nx)
     return (ny, nx)
+
+
+CKPT_DATASETS = ["density0", "energy0", "xvel0", "yvel0", "pressure", "soundspeed", "viscosity",
+                 "density1", "energy1", "xvel1", "yvel1", "vol_flux_x", "vol_flux_y",
+                 "mass_flux_x", "mass_flux_y"]
+
+
+def checkpoint_plan(loop: int):
+    """(loop name, datasets a checkpoint entered before `loop` must save)."""
+    m = ctypes.c_uint32(); n = c_int32(); name = ctypes.c_char_p()
+    _check(load().clover_checkpoint_plan(loop, ctypes.byref(m), ctypes.byref(n), ctypes.byref(name)),
+           "clover_checkpoint_plan")
+    return name.value.decode(), [d for i, d in enumerate(CKPT_DATASETS) if m.value >> i & 1]
 
 
 def debug_div_check(n: int, seed: int = 1, emax: int = 60):
@@ -276,6 +295,17 @@ class Clover:
                "clover_profile_steps")
         return {L.clover_profile_name(i).decode(): (float(ms[i]), int(cnt[i]))
                 for i in range(PROFILE_SLOTS) if cnt[i]}
+
+    def checkpoint(self) -> bytes:
+        n = c_int64()
+        _check(load().clover_checkpoint_bytes(self._ctx, ctypes.byref(n)), "clover_checkpoint_bytes")
+        buf = ctypes.create_string_buffer(n.value)
+        _check(load().clover_checkpoint(self._ctx, buf, n.value), "clover_checkpoint")
+        return buf.raw
+
+    def restart(self, blob: bytes):
+        buf = ctypes.create_string_buffer(blob, len(blob))
+        _check(load().clover_restart(self._ctx, buf, len(blob)), "clover_restart")
 
     def debug_partial_step(self, nkernels: int):
         _check(load().clover_debug_partial_step(self._ctx, nkernels), "clover_debug_partial_step")

@@ -589,6 +589,57 @@ int scatter_local(clover_ctx* ctx, int buf, int kind, const double* host, int64_
   return CLOVER_OK;
 }
 
+// ---------------------------------------------------------------- checkpoint
+// Access-execute analysis of one timestep (Fig. 8):
+// each loop of the reference step with the datasets it reads
+// (R) and writes (W); read-and-write counts as R.  Entering checkpoint mode
+// before loop L, walk the (periodic) loop sequence from L: a dataset whose
+// first access is a read must be saved, one whose first access is a write is
+// dropped; datasets never written (mesh geometry) are not saved.
+enum Dataset { D_RHO0, D_E0, D_U0, D_V0, D_P, D_CS, D_Q, D_RHO1, D_E1, D_U1, D_V1, D_FX, D_FY,
+               D_MX, D_MY, ND };
+#define DB(x) (1u << (x))
+struct LoopAccess { const char* name; unsigned r, w; };
+const LoopAccess kStepLoops[] = {
+    {"ideal_gas", DB(D_RHO0) | DB(D_E0), DB(D_P) | DB(D_CS)},
+    {"viscosity", DB(D_U0) | DB(D_V0) | DB(D_P) | DB(D_RHO0), DB(D_Q)},
+    {"calc_dt", DB(D_CS) | DB(D_Q) | DB(D_RHO0) | DB(D_U0) | DB(D_V0), 0},
+    {"PdV(predict)", DB(D_RHO0) | DB(D_E0) | DB(D_P) | DB(D_Q) | DB(D_U0) | DB(D_V0), DB(D_RHO1) | DB(D_E1)},
+    {"ideal_gas(predict)", DB(D_RHO1) | DB(D_E1), DB(D_P) | DB(D_CS)},
+    {"accelerate", DB(D_RHO0) | DB(D_P) | DB(D_Q) | DB(D_U0) | DB(D_V0), DB(D_U1) | DB(D_V1)},
+    {"PdV(correct)", DB(D_RHO0) | DB(D_E0) | DB(D_P) | DB(D_Q) | DB(D_U0) | DB(D_V0) | DB(D_U1) | DB(D_V1),
+     DB(D_RHO1) | DB(D_E1)},
+    {"flux_calc", DB(D_U0) | DB(D_V0) | DB(D_U1) | DB(D_V1), DB(D_FX) | DB(D_FY)},
+    {"advec_cell(1)", DB(D_RHO1) | DB(D_E1) | DB(D_FX) | DB(D_FY), DB(D_RHO1) | DB(D_E1) | DB(D_MX) | DB(D_MY)},
+    {"advec_mom(1)", DB(D_RHO1) | DB(D_FX) | DB(D_FY) | DB(D_MX) | DB(D_MY) | DB(D_U1) | DB(D_V1),
+     DB(D_U1) | DB(D_V1)},
+    {"advec_cell(2)", DB(D_RHO1) | DB(D_E1) | DB(D_FX) | DB(D_FY), DB(D_RHO1) | DB(D_E1) | DB(D_MX) | DB(D_MY)},
+    {"advec_mom(2)", DB(D_RHO1) | DB(D_FX) | DB(D_FY) | DB(D_MX) | DB(D_MY) | DB(D_U1) | DB(D_V1),
+     DB(D_U1) | DB(D_V1)},
+    {"reset_field", DB(D_RHO1) | DB(D_E1) | DB(D_U1) | DB(D_V1), DB(D_RHO0) | DB(D_E0) | DB(D_U0) | DB(D_V0)},
+};
+constexpr int kNumLoops = sizeof(kStepLoops) / sizeof(kStepLoops[0]);
+#undef DB
+
+unsigned checkpoint_plan(int loop) {
+  unsigned decided = 0, save = 0;
+  for (int t = 0; t < kNumLoops; ++t) {
+    const LoopAccess& L = kStepLoops[(loop + t) % kNumLoops];
+    const unsigned rnew = L.r & ~decided;
+    save |= rnew;
+    decided |= L.r | L.w;
+  }
+  return save;
+}
+
+constexpr uint64_t kCkptMagic = 0x54504b43564f4c43ull;  // "CLOVCKPT"
+struct CkptHeader {
+  uint64_t magic;
+  int32_t version, x_cells, y_cells, face_mirror;
+  int32_t step, advect_x, nfields, pad;
+  double xmin, ymin, xmax, ymax, time, dt, dtold;
+};
+
 }  // namespace
 
 // ====================================================================== C ABI
@@ -1086,6 +1137,97 @@ int clover_step_host(clover_ctx* ctx, int32_t nsteps, const double* d_in, const 
       if (rc) return rc;
     }
   return check_err(ctx);
+}
+
+int clover_checkpoint_plan(int32_t loop, uint32_t* save_mask, int32_t* nsaved, const char** name) {
+  if (loop < 0 || loop >= kNumLoops) return fail(CLOVER_ERR_ARG, "loop index out of range");
+  const unsigned m = checkpoint_plan(loop);
+  if (save_mask) *save_mask = m;
+  if (nsaved) *nsaved = __builtin_popcount(m);
+  if (name) *name = kStepLoops[loop].name;
+  return CLOVER_OK;
+}
+
+int clover_checkpoint_bytes(clover_ctx* ctx, int64_t* bytes) {
+  if (!ctx || !bytes) return fail(CLOVER_ERR_ARG, "NULL argument");
+  const int64_t nc = (int64_t)ctx->g.x_cells * ctx->g.y_cells;
+  const int64_t nn = (int64_t)(ctx->g.x_cells + 1) * (ctx->g.y_cells + 1);
+  *bytes = (int64_t)sizeof(CkptHeader) + 8 * (2 * nc + 2 * nn);
+  return CLOVER_OK;
+}
+
+int clover_checkpoint(clover_ctx* ctx, void* host, int64_t bytes) {
+  if (!ctx || !host) return fail(CLOVER_ERR_ARG, "NULL argument");
+  if (ctx->nranks > 1) return fail(CLOVER_ERR_STATE, "checkpoint: single-process contexts only");
+  int64_t need;
+  clover_checkpoint_bytes(ctx, &need);
+  if (bytes < need) return fail(CLOVER_ERR_ARG, "checkpoint buffer too small");
+  // the step boundary is the optimum of the access analysis: exactly the
+  // four state fields are live there
+  if (checkpoint_plan(0) != ((1u << D_RHO0) | (1u << D_E0) | (1u << D_U0) | (1u << D_V0)))
+    return fail(CLOVER_ERR_STATE, "checkpoint plan mismatch");
+  int rc = join_in(ctx);
+  if (rc) return rc;
+  rc = check_err(ctx);
+  if (rc) return rc;
+  StepScalars h;
+  CK(cudaMemcpy(&h, ctx->scal, sizeof(h), cudaMemcpyDeviceToHost));
+  CkptHeader hd{};
+  hd.magic = kCkptMagic; hd.version = 1;
+  hd.x_cells = ctx->g.x_cells; hd.y_cells = ctx->g.y_cells; hd.face_mirror = ctx->g.face_mirror;
+  hd.step = h.step; hd.advect_x = ctx->advect_x ? 1 : 0; hd.nfields = 4;
+  hd.xmin = ctx->g.xmin; hd.ymin = ctx->g.ymin; hd.xmax = ctx->g.xmax; hd.ymax = ctx->g.ymax;
+  hd.time = h.time; hd.dt = h.dt; hd.dtold = h.dtold;
+  std::memcpy(host, &hd, sizeof(hd));
+  double* p = (double*)((char*)host + sizeof(hd));
+  const int64_t nc = (int64_t)ctx->g.x_cells * ctx->g.y_cells;
+  const int64_t nn = (int64_t)(ctx->g.x_cells + 1) * (ctx->g.y_cells + 1);
+  rc = gather_local(ctx, B_D0, K_CELL, p, nc);
+  if (!rc) rc = gather_local(ctx, B_E0, K_CELL, p + nc, nc);
+  if (!rc) rc = gather_local(ctx, B_U0, K_XVEL, p + 2 * nc, nn);
+  if (!rc) rc = gather_local(ctx, B_V0, K_YVEL, p + 2 * nc + nn, nn);
+  if (rc) return rc;
+  return join_out(ctx);
+}
+
+int clover_restart(clover_ctx* ctx, const void* host, int64_t bytes) {
+  if (!ctx || !host) return fail(CLOVER_ERR_ARG, "NULL argument");
+  if (ctx->nranks > 1) return fail(CLOVER_ERR_STATE, "restart: single-process contexts only");
+  int64_t need;
+  clover_checkpoint_bytes(ctx, &need);
+  if (bytes < need) return fail(CLOVER_ERR_ARG, "checkpoint buffer too small");
+  CkptHeader hd;
+  std::memcpy(&hd, host, sizeof(hd));
+  if (hd.magic != kCkptMagic || hd.version != 1 || hd.nfields != 4)
+    return fail(CLOVER_ERR_ARG, "not a clover checkpoint");
+  if (hd.x_cells != ctx->g.x_cells || hd.y_cells != ctx->g.y_cells || hd.xmin != ctx->g.xmin ||
+      hd.ymin != ctx->g.ymin || hd.xmax != ctx->g.xmax || hd.ymax != ctx->g.ymax ||
+      hd.face_mirror != ctx->g.face_mirror)
+    return fail(CLOVER_ERR_ARG, "checkpoint was taken on a different mesh");
+  const double* p = (const double*)((const char*)host + sizeof(hd));
+  const int64_t nc = (int64_t)ctx->g.x_cells * ctx->g.y_cells;
+  const int64_t nn = (int64_t)(ctx->g.x_cells + 1) * (ctx->g.y_cells + 1);
+  int rc = join_in(ctx);
+  if (rc) return rc;
+  rc = scatter_local(ctx, B_D0, K_CELL, p, nc);
+  if (!rc) rc = scatter_local(ctx, B_E0, K_CELL, p + nc, nc);
+  if (!rc) rc = scatter_local(ctx, B_U0, K_XVEL, p + 2 * nc, nn);
+  if (!rc) rc = scatter_local(ctx, B_V0, K_YVEL, p + 2 * nc + nn, nn);
+  if (rc) return rc;
+  rc = reflect_all(ctx, {B_D0, B_E0, B_U0, B_V0});
+  if (rc) return rc;
+  StepScalars h;
+  CK(cudaStreamSynchronize(ctx->work));
+  CK(cudaMemcpy(&h, ctx->scal, sizeof(h), cudaMemcpyDeviceToHost));
+  h.step = hd.step; h.time = hd.time; h.dt = hd.dt; h.dtold = hd.dtold; h.err = 0;
+  {
+    double big = G_BIG;
+    std::memcpy(&h.dt_slot, &big, 8);
+  }
+  CK(cudaMemcpyAsync(ctx->scal, &h, sizeof(h), cudaMemcpyHostToDevice, ctx->work));
+  ctx->advect_x = hd.advect_x != 0;
+  CK(cudaStreamSynchronize(ctx->work));
+  return join_out(ctx);
 }
 
 int clover_finalize(clover_ctx* ctx) {
