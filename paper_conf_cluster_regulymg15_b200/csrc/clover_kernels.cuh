@@ -32,7 +32,7 @@ __device__ __forceinline__ double eos_pressure(double rho, double e) {
 template <class D>
 __device__ __forceinline__ double eos_soundspeed(D& dv, double rho, double e) {
   const double gm1 = 1.4 - 1.0;
-  double v = dv(1.0, rho);
+  double v = dv.nz(1.0, rho);
   double p = gm1 * rho * e;
   double pbe = gm1 * rho;
   double pbv = -rho * p;
@@ -91,18 +91,18 @@ __device__ __forceinline__ double visc_dt_cell(D& dv, const ViscIn& I, const Chu
   double cc = cs * cs;
   cc = cc + dv(2.0 * qv, I.rho);
   cc = fmax(sqrt(cc), G_SMALL);
-  double dtct = dv(prm.dtc_safe * fmin(dx, dy), cc);
+  double dtct = dv.nz(prm.dtc_safe * fmin(dx, dy), cc);
   double dvv = 0.0;
   double dv1 = (u00 + u01) * dy;
   double dv2 = (u10 + u11) * dy;
   dvv = dvv + dv2 - dv1;
-  double dtut = dv(prm.dtu_safe * 2.0 * vol, fmax(fmax(fabs(dv1), fabs(dv2)), G_SMALL * vol));
+  double dtut = dv.nz(prm.dtu_safe * 2.0 * vol, fmax(fmax(fabs(dv1), fabs(dv2)), G_SMALL * vol));
   dv1 = (v00 + v10) * dx;
   dv2 = (v01 + v11) * dx;
   dvv = dvv + dv2 - dv1;
-  double dtvt = dv(prm.dtv_safe * 2.0 * vol, fmax(fmax(fabs(dv1), fabs(dv2)), G_SMALL * vol));
+  double dtvt = dv.nz(prm.dtv_safe * 2.0 * vol, fmax(fmax(fabs(dv1), fabs(dv2)), G_SMALL * vol));
   dvv = dv.c(dvv, 2.0 * vol, C.r2vol);
-  double dtdivt = (dvv < -G_SMALL) ? prm.dtdiv_safe * dv(-1.0, dvv) : G_BIG;
+  double dtdivt = (dvv < -G_SMALL) ? prm.dtdiv_safe * dv.nz(-1.0, dvv) : G_BIG;
   return fmin(fmin(dtct, dtut), fmin(dtvt, dtdivt));
 }
 
@@ -138,7 +138,7 @@ __device__ __forceinline__ double pdv_predict_pressure(D& dv, double r, double e
   double bottom_flux = (dx * (va + vb + va + vb)) * 0.25 * dt * 0.5;
   double top_flux = (dx * (vc + vd + vc + vd)) * 0.25 * dt * 0.5;
   double total_flux = right_flux - left_flux + top_flux - bottom_flux;
-  double volume_change = dv(vol, vol + total_flux);
+  double volume_change = dv.nz(vol, vol + total_flux);
   double recip_volume = rvol;  // = RN(1.0/vol), precomputed
   double p0 = eos_pressure(r, e);
   double energy_change = (dv(p0, r) + dv(q, r)) * total_flux * recip_volume;
@@ -156,7 +156,7 @@ __device__ __forceinline__ void accelerate_node(D& dv, const double* rr, const d
   const double vol = dx * dy;
   const double halfdt = 0.5 * dt;
   double nodal_mass = (rr[0] * vol + rr[1] * vol + rr[2] * vol + rr[3] * vol) * 0.25;
-  double stepbymass = dv(halfdt, nodal_mass);
+  double stepbymass = dv.nz(halfdt, nodal_mass);
   // p(j,k)=pp[2], p(j-1,k)=pp[3], p(j,k-1)=pp[1], p(j-1,k-1)=pp[0]
   uu = u0v - stepbymass * (dy * (pp[2] - pp[3]) + dy * (pp[1] - pp[0]));
   vv = v0v - stepbymass * (dx * (pp[2] - pp[1]) + dx * (pp[3] - pp[0]));
@@ -176,7 +176,7 @@ __device__ __forceinline__ void pdv_correct(D& dv, double r, double e, double ph
   double bottom_flux = (dx * bsum) * 0.25 * dt;
   double top_flux = (dx * tsum) * 0.25 * dt;
   double total_flux = right_flux - left_flux + top_flux - bottom_flux;
-  double volume_change = dv(vol, vol + total_flux);
+  double volume_change = dv.nz(vol, vol + total_flux);
   double recip_volume = rvol;  // = RN(1.0/vol), precomputed
   double energy_change = (dv(ph, r) + dv(q, r)) * total_flux * recip_volume;
   e1v = e - energy_change;
