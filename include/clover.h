@@ -189,6 +189,12 @@ int clover_profile_steps(clover_ctx* ctx, int32_t nsteps, double* ms_out, int64_
                          int32_t nslots);
 const char* clover_profile_name(int32_t i);
 
+/* Test: route every chunk boundary of a single-process multi-chunk context
+ * through the remote-neighbour path (pack -> staging -> unpack, exactly the
+ * code around the NCCL send/recv pair, which a device copy replaces), so the
+ * multi-GPU message layout is exercised on one GPU. */
+int clover_debug_set_virtual_remote(clover_ctx* ctx, int32_t enable);
+
 /* Debug: run only the first `nkernels` kernel phases of the next step
  * (1 = viscosity+calc_dt, 2 = +dt reduction, 3 = +Lagrangian phase,
  * 4..7 = +advection kernels); the step is left incomplete.  Test only. */

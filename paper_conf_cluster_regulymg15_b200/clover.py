@@ -39,7 +39,7 @@ EXPORTS = ["clover_workspace_bytes", "clover_nccl_unique_id", "clover_init", "cl
            "clover_read_field", "clover_write_field", "clover_sync", "clover_set_graphs",
            "clover_kernels_per_step", "clover_debug_partial_step", "clover_debug_read_buffer",
            "clover_profile_steps", "clover_profile_name", "clover_debug_div_check",
-           "clover_checkpoint_plan", "clover_checkpoint_bytes", "clover_checkpoint", "clover_restart", "clover_finalize", "clover_error_string", "clover_last_error", "clover_abi_version"]
+           "clover_checkpoint_plan", "clover_debug_set_virtual_remote", "clover_checkpoint_bytes", "clover_checkpoint", "clover_restart", "clover_finalize", "clover_error_string", "clover_last_error", "clover_abi_version"]
 
 
 class CloverGrid(ctypes.Structure):
@@ -111,6 +111,7 @@ def load(build_if_missing: bool = True):
     L.clover_checkpoint_bytes.argtypes = [c_void_p, ctypes.POINTER(c_int64)]
     L.clover_checkpoint.argtypes = [c_void_p, c_void_p, c_int64]
     L.clover_restart.argtypes = [c_void_p, c_void_p, c_int64]
+    L.clover_debug_set_virtual_remote.argtypes = [c_void_p, c_int32]
     L.clover_finalize.argtypes = [c_void_p]
     L.clover_error_string.argtypes = [c_int32]
     L.clover_error_string.restype = ctypes.c_char_p
@@ -306,6 +307,10 @@ class Clover:
     def restart(self, blob: bytes):
         buf = ctypes.create_string_buffer(blob, len(blob))
         _check(load().clover_restart(self._ctx, buf, len(blob)), "clover_restart")
+
+    def debug_set_virtual_remote(self, on: bool):
+        _check(load().clover_debug_set_virtual_remote(self._ctx, 1 if on else 0),
+               "clover_debug_set_virtual_remote")
 
     def debug_partial_step(self, nkernels: int):
         _check(load().clover_debug_partial_step(self._ctx, nkernels), "clover_debug_partial_step")

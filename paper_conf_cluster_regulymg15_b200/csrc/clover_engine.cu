@@ -133,6 +133,7 @@ struct clover_ctx {
   cudaGraphExec_t gexec[2] = {nullptr, nullptr};
   int64_t ws_bytes = 0;
   bool prof = false;
+  bool virtual_remote = false;  // test mode: every chunk boundary takes the NCCL packing path
   std::vector<std::pair<int, cudaEvent_t>> prof_events;
 #ifdef CLOVER_WITH_NCCL
   ncclComm_t comm = nullptr;
@@ -198,10 +199,11 @@ int64_t compute_workspace(const clover_grid* g, int px, int py, int rank, int nr
     maxrows = std::max<int64_t>(maxrows, ny + 2 + 2 * HALO);
     maxcols = std::max<int64_t>(maxcols, nx + 2 + 2 * HALO);
   }
-  if (nranks > 1) {
-    // staging for up to 4 neighbours x 6 fields x HALO lines
+  if (px * py > 1) {
+    // staging for the remote-neighbour path: every local chunk x 4 sides x
+    // 6 fields x HALO lines (also used by the virtual-remote test mode)
     int64_t line = std::max(maxrows, maxcols);
-    int64_t el = 4 * 6 * HALO * line;
+    int64_t el = (int64_t)local_chunk_ids(px, py, rank, nranks).size() * 4 * 6 * HALO * line;
     bytes += 2 * align_up(el * 8, kAlign);
   }
   return bytes;
@@ -235,7 +237,10 @@ void side_strips(const ChunkState& cs, int buf, int side, XferDesc& send, XferDe
   const int oy = (kind == K_XVEL || kind == K_YVEL || kind == K_YFACE) ? 1 : 0;
   send.base = recv.base = cs.buf[buf];
   send.pitch = recv.pitch = c.pitch;
-  const int full_h = c.ny + 1 + 2 * HALO, full_w = c.nx + 1 + 2 * HALO;
+  // full extent of this kind including both halos: rows [-HALO, ny+oy+HALO],
+  // columns [-HALO, nx+ox+HALO] (x strips carry every row, y strips every
+  // column, so 4-chunk corners are refreshed by the second axis)
+  const int full_h = c.ny + oy + 1 + 2 * HALO, full_w = c.nx + ox + 1 + 2 * HALO;
   if (side == 0) {          // left: send [1+ox, HALO+ox], recv [1-HALO, 0]
     send.j0 = 1 + ox; recv.j0 = 1 - HALO;
     send.w = recv.w = HALO;
@@ -275,6 +280,7 @@ int exchange_axis(clover_ctx* ctx, const std::vector<int>& bufs, int axis) {
   const int s_lo = axis == 0 ? 0 : 2, s_hi = axis == 0 ? 1 : 3;
   // local pairs
   for (auto& cs : ctx->chunks) {
+    if (ctx->virtual_remote) break;
     int nb = neighbour(ctx, cs, s_hi);
     if (nb < 0) continue;
     ChunkState* other = local_chunk(ctx, nb);
@@ -289,17 +295,27 @@ int exchange_axis(clover_ctx* ctx, const std::vector<int>& bufs, int axis) {
       if (rc) return rc;
     }
   }
-#ifdef CLOVER_WITH_NCCL
-  if (ctx->nranks > 1) {
-    // pack every remote side into the staging buffer, one NCCL group
-    struct Msg { int peer; int64_t off, n; ChunkState* cs; int side; };
+  if (ctx->nranks > 1 || ctx->virtual_remote) {
+    // remote neighbours: pack every remote side into the staging buffer,
+    // exchange all messages in one NCCL group, unpack.  In virtual-remote
+    // mode (one process, test only) the NCCL pair is replaced by a device
+    // copy from the partner message's send slot into this message's receive
+    // slot; packing, offsets and unpacking are the NCCL path's own.
+    struct Msg { int peer, nb; int64_t off, n; ChunkState* cs; int side; };
     std::vector<Msg> msgs;
     int64_t off = 0;
     for (auto& cs : ctx->chunks)
       for (int side : {s_lo, s_hi}) {
         int nb = neighbour(ctx, cs, side);
-        if (nb < 0 || local_chunk(ctx, nb)) continue;
+        if (nb < 0 || (!ctx->virtual_remote && local_chunk(ctx, nb))) continue;
         int64_t n = 0;
+        for (int b : bufs) {
+          XferDesc s, r;
+          side_strips(cs, b, side, s, r);
+          n += (int64_t)s.w * s.h;
+        }
+        if (off + n > ctx->xbuf_elems) return fail(CLOVER_ERR_STATE, "halo staging buffer too small");
+        n = 0;
         for (int b : bufs) {
           XferDesc s, r;
           side_strips(cs, b, side, s, r);
@@ -308,16 +324,30 @@ int exchange_axis(clover_ctx* ctx, const std::vector<int>& bufs, int axis) {
           if (rc) return rc;
           n += (int64_t)s.w * s.h;
         }
-        msgs.push_back({ctx->owner[nb], off, n, &cs, side});
+        msgs.push_back({ctx->owner[nb], nb, off, n, &cs, side});
         off += n;
       }
-    if (off > ctx->xbuf_elems) return fail(CLOVER_ERR_STATE, "halo staging buffer too small");
-    NK(ncclGroupStart());
-    for (auto& m : msgs) {
-      NK(ncclSend(ctx->xbuf_send + m.off, (size_t)m.n, ncclFloat64, m.peer, ctx->comm, ctx->work));
-      NK(ncclRecv(ctx->xbuf_recv + m.off, (size_t)m.n, ncclFloat64, m.peer, ctx->comm, ctx->work));
+    if (ctx->virtual_remote) {
+      for (auto& m : msgs) {
+        const Msg* partner = nullptr;
+        for (auto& q : msgs)
+          if (q.cs->id == m.nb && q.side == (m.side ^ 1)) partner = &q;
+        if (!partner || partner->n != m.n) return fail(CLOVER_ERR_STATE, "virtual remote: unmatched message");
+        CK(cudaMemcpyAsync(ctx->xbuf_recv + m.off, ctx->xbuf_send + partner->off, (size_t)m.n * 8,
+                           cudaMemcpyDeviceToDevice, ctx->work));
+      }
+    } else {
+#ifdef CLOVER_WITH_NCCL
+      NK(ncclGroupStart());
+      for (auto& m : msgs) {
+        NK(ncclSend(ctx->xbuf_send + m.off, (size_t)m.n, ncclFloat64, m.peer, ctx->comm, ctx->work));
+        NK(ncclRecv(ctx->xbuf_recv + m.off, (size_t)m.n, ncclFloat64, m.peer, ctx->comm, ctx->work));
+      }
+      NK(ncclGroupEnd());
+#else
+      return fail(CLOVER_ERR_NCCL, "libclover built without NCCL");
+#endif
     }
-    NK(ncclGroupEnd());
     for (auto& m : msgs) {
       int64_t n = 0;
       for (int b : bufs) {
@@ -330,7 +360,6 @@ int exchange_axis(clover_ctx* ctx, const std::vector<int>& bufs, int axis) {
       }
     }
   }
-#endif
   return CLOVER_OK;
 }
 
@@ -761,9 +790,9 @@ int clover_init(const clover_grid* grid, const clover_state* states, int32_t nst
     maxcols = std::max<int64_t>(maxcols, c.nx + 2 + 2 * HALO);
     ctx->chunks.push_back(cs);
   }
-  if (nranks > 1) {
+  if (px * py > 1) {
     int64_t line = std::max(maxrows, maxcols);
-    ctx->xbuf_elems = 4 * 6 * HALO * line;
+    ctx->xbuf_elems = (int64_t)ctx->chunks.size() * 4 * 6 * HALO * line;
     ctx->xbuf_send = (double*)p;
     p += align_up(ctx->xbuf_elems * 8, kAlign);
     ctx->xbuf_recv = (double*)p;
@@ -832,6 +861,19 @@ int clover_init(const clover_grid* grid, const clover_state* states, int32_t nst
 int clover_set_graphs(clover_ctx* ctx, int32_t enable) {
   if (!ctx) return fail(CLOVER_ERR_ARG, "ctx is NULL");
   ctx->use_graphs = enable != 0;
+  return CLOVER_OK;
+}
+
+int clover_debug_set_virtual_remote(clover_ctx* ctx, int32_t enable) {
+  if (!ctx) return fail(CLOVER_ERR_ARG, "ctx is NULL");
+  if (ctx->nranks > 1) return fail(CLOVER_ERR_STATE, "virtual remote is a single-process test mode");
+  if (enable && ctx->L.px * ctx->L.py < 2) return fail(CLOVER_ERR_STATE, "virtual remote needs px*py > 1");
+  ctx->virtual_remote = enable != 0;
+  for (int i = 0; i < 2; ++i)
+    if (ctx->gexec[i]) {
+      cudaGraphExecDestroy(ctx->gexec[i]);
+      ctx->gexec[i] = nullptr;
+    }
   return CLOVER_OK;
 }
 

@@ -186,13 +186,36 @@ def test_local_chunk_decomposition_bitwise(torch_cuda, pxy):
     assert many.field_summary() == one.field_summary()
 
 
-def test_local_chunks_fuzz(torch_cuda):
-    deck = fuzz_deck(8, nx=64, ny=48)
-    one, many = make_gpu(deck), make_gpu(deck, px=2, py=3)
-    one.step(8)
-    many.step(8)
+@pytest.mark.parametrize("pxy", [(2, 1), (1, 2), (2, 2), (3, 2), (2, 4)])
+def test_virtual_remote_exchange_bitwise(torch_cuda, pxy):
+    """Every chunk boundary through the multi-GPU packing path (pack ->
+    staging -> unpack, the NCCL pair replaced by a device copy): same bits
+    as one chunk, including the dt history."""
+    deck = fuzz_deck(9, nx=96, ny=80)
+    one = make_gpu(deck)
+    many = make_gpu(deck, px=pxy[0], py=pxy[1])
+    many.debug_set_virtual_remote(True)
+    one.step(10)
+    many.step(10)
     for f in STATE:
         assert np.array_equal(many.read(f), one.read(f)), f
+    assert np.array_equal(many.dt_history(1, 10), one.dt_history(1, 10))
+
+
+@pytest.mark.parametrize("seed,pxy", [(8, (2, 3)), (9, (3, 2)), (9, (2, 4)), (12, (4, 4)),
+                                      (13, (3, 3))])
+def test_local_chunks_fuzz(torch_cuda, seed, pxy):
+    """Fuzz decks put flow on the 4-chunk corners (the bm deck never does):
+    the corner halos of node/face fields must be refreshed by the second
+    exchange axis (regression: x-face Mx(nx+3, ny+1) was once missed)."""
+    deck = fuzz_deck(seed, nx=96, ny=80)
+    deck["max_timestep"] = 1.0
+    one, many = make_gpu(deck), make_gpu(deck, px=pxy[0], py=pxy[1])
+    one.step(12)
+    many.step(12)
+    for f in STATE:
+        assert np.array_equal(many.read(f), one.read(f)), f
+    assert np.array_equal(many.dt_history(1, 12), one.dt_history(1, 12))
 
 
 def test_graphs_on_off_identical(torch_cuda):
