@@ -164,7 +164,9 @@ int clover_get_clock(clover_ctx* ctx, int32_t* step, double* time, double* dt_la
 int clover_dt_history(clover_ctx* ctx, int32_t first, int32_t n, double* host_out);
 
 /* Gather a field's global interior into host memory (n = element count of
- * the field's kind, see above).  Every rank receives the full field. */
+ * the field's kind, see above).  Every rank receives the full field
+ * (multi-rank: NCCL all-gather through a temporary device buffer -- the one
+ * place the library allocates device memory, a debug/I-O path). */
 int clover_read_field(clover_ctx* ctx, int32_t field_id, double* host, int64_t n);
 
 /* Overwrite the global interior of a state field (DENSITY0, ENERGY0, XVEL0,
@@ -224,7 +226,9 @@ int clover_debug_div_check(int64_t n, uint64_t seed, int32_t emax, int64_t* mism
  * At the step boundary -- the optimum, where clover_checkpoint operates --
  * it is {density0, energy0, xvel0, yvel0}; plus the clock (step, time, dt,
  * dtold, sweep order).  Restarting from a checkpoint continues bit for bit.
- * Single-process contexts; the buffer is host memory owned by the caller. */
+ * Multi-rank: every rank gathers (and may write) the full checkpoint;
+ * restart scatters each rank's part.  The buffer is host memory owned by the
+ * caller. */
 int clover_checkpoint_plan(int32_t loop, uint32_t* save_mask, int32_t* nsaved, const char** name);
 int clover_checkpoint_bytes(clover_ctx* ctx, int64_t* bytes);
 int clover_checkpoint(clover_ctx* ctx, void* host, int64_t bytes);

@@ -618,6 +618,80 @@ int scatter_local(clover_ctx* ctx, int buf, int kind, const double* host, int64_
   return CLOVER_OK;
 }
 
+// All-gather `count` doubles per rank (device `send`) into host `out`
+// (nranks*count, rank-major).  Uses a temporary device buffer: this is the
+// debug / I/O path (field readback, summaries, checkpoints), not the step.
+int allgather_to_host(clover_ctx* ctx, const double* send, int64_t count, double* out) {
+#ifdef CLOVER_WITH_NCCL
+  double* recv = nullptr;
+  CK(cudaMallocAsync((void**)&recv, (size_t)count * ctx->nranks * 8, ctx->work));
+  ncclResult_t r = ncclAllGather(send, recv, (size_t)count, ncclFloat64, ctx->comm, ctx->work);
+  cudaError_t e = cudaMemcpyAsync(out, recv, (size_t)count * ctx->nranks * 8, cudaMemcpyDeviceToHost, ctx->work);
+  cudaFreeAsync(recv, ctx->work);
+  if (r != ncclSuccess) return fail(CLOVER_ERR_NCCL, std::string("ncclAllGather: ") + ncclGetErrorString(r));
+  if (e != cudaSuccess) return fail(CLOVER_ERR_CUDA, cudaGetErrorString(e));
+  CK(cudaStreamSynchronize(ctx->work));
+  return CLOVER_OK;
+#else
+  (void)ctx; (void)send; (void)count; (void)out;
+  return fail(CLOVER_ERR_NCCL, "libclover built without NCCL");
+#endif
+}
+
+// Owned block of chunk `id` for a field kind: global origin and extent (the
+// shared last node/face column/row belongs to the chunk on the global edge).
+void owned_block(const clover_ctx* ctx, int id, int ax, int ay, int* gj0, int* gk0, int* w, int* h) {
+  const int cx = id % ctx->L.px, cy = id / ctx->L.px;
+  *gj0 = ctx->L.xs[cx];
+  *gk0 = ctx->L.ys[cy];
+  const int nx = ctx->L.xs[cx + 1] - ctx->L.xs[cx], ny = ctx->L.ys[cy + 1] - ctx->L.ys[cy];
+  *w = nx + ((ctx->L.xs[cx + 1] == ctx->g.x_cells) ? ax : 0);
+  *h = ny + ((ctx->L.ys[cy + 1] == ctx->g.y_cells) ? ay : 0);
+}
+
+// Gather a field's global interior on every rank.  Single process: device to
+// host copies.  Multi-rank: each rank packs its owned blocks (padded to the
+// largest block) into one device buffer, NCCL all-gather, every rank unpacks
+// all blocks into the host array.
+int gather_all(clover_ctx* ctx, int buf, int kind, double* host, int64_t n) {
+  if (ctx->nranks == 1) return gather_local(ctx, buf, kind, host, n);
+  int ax, ay;
+  kind_extra(kind, &ax, &ay);
+  const int NXE = ctx->g.x_cells + ax, NYE = ctx->g.y_cells + ay;
+  if (n != (int64_t)NXE * NYE) return fail(CLOVER_ERR_ARG, "wrong element count for field");
+  int64_t maxblk = 0;
+  for (int id = 0; id < ctx->L.px * ctx->L.py; ++id) {
+    int gj, gk, w, h;
+    owned_block(ctx, id, ax, ay, &gj, &gk, &w, &h);
+    maxblk = std::max<int64_t>(maxblk, (int64_t)w * h);
+  }
+  const int64_t per = (int64_t)ctx->chunks.size() * maxblk;
+  double* pack = nullptr;
+  CK(cudaMallocAsync((void**)&pack, (size_t)per * 8, ctx->work));
+  for (size_t t = 0; t < ctx->chunks.size(); ++t) {
+    const ChunkState& cs = ctx->chunks[t];
+    int gj, gk, w, h;
+    owned_block(ctx, cs.id, ax, ay, &gj, &gk, &w, &h);
+    CK(cudaMemcpy2DAsync(pack + t * maxblk, (size_t)w * 8, cs.buf[buf] + idx(cs.c, 1, 1),
+                         (size_t)cs.c.pitch * 8, (size_t)w * 8, h, cudaMemcpyDeviceToDevice, ctx->work));
+  }
+  std::vector<double> all((size_t)per * ctx->nranks);
+  int rc = allgather_to_host(ctx, pack, per, all.data());
+  cudaFreeAsync(pack, ctx->work);
+  if (rc) return rc;
+  for (int r = 0; r < ctx->nranks; ++r) {
+    const std::vector<int> ids = local_chunk_ids(ctx->L.px, ctx->L.py, r, ctx->nranks);
+    for (size_t t = 0; t < ids.size(); ++t) {
+      int gj, gk, w, h;
+      owned_block(ctx, ids[t], ax, ay, &gj, &gk, &w, &h);
+      const double* blk = all.data() + (size_t)r * per + t * maxblk;
+      for (int k = 0; k < h; ++k)
+        std::memcpy(host + (int64_t)(gk + k) * NXE + gj, blk + (int64_t)k * w, (size_t)w * 8);
+    }
+  }
+  return CLOVER_OK;
+}
+
 // ---------------------------------------------------------------- checkpoint
 // Access-execute analysis of one timestep (Fig. 8):
 // each loop of the reference step with the datasets it reads
@@ -1050,49 +1124,71 @@ int clover_field_summary(clover_ctx* ctx, clover_summary* out) {
         cs.c, cs.buf[B_D0], cs.buf[B_E0], cs.buf[B_U0], cs.buf[B_V0], cs.partials);
     LAUNCH_CHECK();
   }
-  // global tile grid (tiles aligned at global cell 1 when tile_aligned)
-  const int GTX = (ctx->g.x_cells + ST - 1) / ST, GTY = (ctx->g.y_cells + ST - 1) / ST;
-  std::vector<double> all;
-  std::vector<std::vector<double>> per(ctx->chunks.size());
-  for (size_t i = 0; i < ctx->chunks.size(); ++i) {
-    auto& cs = ctx->chunks[i];
-    per[i].resize((size_t)cs.ntx * cs.nty * 5);
-    CK(cudaMemcpyAsync(per[i].data(), cs.partials, per[i].size() * 8, cudaMemcpyDeviceToHost, ctx->work));
+  // tile partials of every chunk of the mesh, in chunk-id order (all ranks'
+  // chunks after an all-gather of the padded per-rank blocks)
+  const int nch = ctx->L.px * ctx->L.py;
+  auto ntiles = [&](int id) {
+    const int cx = id % ctx->L.px, cy = id / ctx->L.px;
+    const int nx = ctx->L.xs[cx + 1] - ctx->L.xs[cx], ny = ctx->L.ys[cy + 1] - ctx->L.ys[cy];
+    return std::make_pair((nx + ST - 1) / ST, (ny + ST - 1) / ST);
+  };
+  std::vector<std::vector<double>> per(nch);
+  if (ctx->nranks == 1) {
+    for (auto& cs : ctx->chunks) {
+      per[cs.id].resize((size_t)cs.ntx * cs.nty * 5);
+      CK(cudaMemcpyAsync(per[cs.id].data(), cs.partials, per[cs.id].size() * 8, cudaMemcpyDeviceToHost,
+                         ctx->work));
+    }
+    rc = check_err(ctx);
+  } else {
+    int64_t maxt = 0;
+    for (int id = 0; id < nch; ++id) {
+      auto t = ntiles(id);
+      maxt = std::max<int64_t>(maxt, (int64_t)t.first * t.second * 5);
+    }
+    const int64_t cnt = (int64_t)ctx->chunks.size() * maxt;
+    double* pack = nullptr;
+    CK(cudaMallocAsync((void**)&pack, (size_t)cnt * 8, ctx->work));
+    for (size_t t = 0; t < ctx->chunks.size(); ++t) {
+      auto& cs = ctx->chunks[t];
+      CK(cudaMemcpyAsync(pack + t * maxt, cs.partials, (size_t)cs.ntx * cs.nty * 5 * 8,
+                         cudaMemcpyDeviceToDevice, ctx->work));
+    }
+    std::vector<double> all((size_t)cnt * ctx->nranks);
+    rc = allgather_to_host(ctx, pack, cnt, all.data());
+    cudaFreeAsync(pack, ctx->work);
+    if (rc) return rc;
+    for (int r = 0; r < ctx->nranks; ++r) {
+      const std::vector<int> ids = local_chunk_ids(ctx->L.px, ctx->L.py, r, ctx->nranks);
+      for (size_t t = 0; t < ids.size(); ++t) {
+        auto nt = ntiles(ids[t]);
+        const double* blk = all.data() + (size_t)r * cnt + t * maxt;
+        per[ids[t]].assign(blk, blk + (size_t)nt.first * nt.second * 5);
+      }
+    }
+    rc = check_err(ctx);
   }
-  rc = check_err(ctx);
   double acc[5] = {0, 0, 0, 0, 0};
-  if (ctx->L.tile_aligned && ctx->nranks == 1) {
-    all.assign((size_t)GTX * GTY * 5, 0.0);
-    for (size_t i = 0; i < ctx->chunks.size(); ++i) {
-      auto& cs = ctx->chunks[i];
-      const int tx0 = cs.c.gj0 / ST, ty0 = cs.c.gk0 / ST;
-      for (int ty = 0; ty < cs.nty; ++ty)
-        for (int tx = 0; tx < cs.ntx; ++tx)
+  if (ctx->L.tile_aligned) {
+    // 16x16 tiles aligned at global cell 1: sum in global tile order, so
+    // every decomposition (chunks, ranks) gives the same bits
+    const int GTX = (ctx->g.x_cells + ST - 1) / ST, GTY = (ctx->g.y_cells + ST - 1) / ST;
+    std::vector<double> glob((size_t)GTX * GTY * 5, 0.0);
+    for (int id = 0; id < nch; ++id) {
+      auto nt = ntiles(id);
+      const int tx0 = ctx->L.xs[id % ctx->L.px] / ST, ty0 = ctx->L.ys[id / ctx->L.px] / ST;
+      for (int ty = 0; ty < nt.second; ++ty)
+        for (int tx = 0; tx < nt.first; ++tx)
           for (int q = 0; q < 5; ++q)
-            all[((size_t)(ty0 + ty) * GTX + (tx0 + tx)) * 5 + q] = per[i][((size_t)ty * cs.ntx + tx) * 5 + q];
+            glob[((size_t)(ty0 + ty) * GTX + (tx0 + tx)) * 5 + q] = per[id][((size_t)ty * nt.first + tx) * 5 + q];
     }
     for (size_t t = 0; t < (size_t)GTX * GTY; ++t)
-      for (int q = 0; q < 5; ++q) acc[q] = acc[q] + all[t * 5 + q];
+      for (int q = 0; q < 5; ++q) acc[q] = acc[q] + glob[t * 5 + q];
   } else {
     for (auto& v : per)
       for (size_t t = 0; t < v.size() / 5; ++t)
         for (int q = 0; q < 5; ++q) acc[q] = acc[q] + v[t * 5 + q];
   }
-#ifdef CLOVER_WITH_NCCL
-  if (ctx->nranks > 1) {
-    // deterministic across ranks: gather per-rank totals, sum in rank order
-    double* dsend = ctx->xbuf_send;
-    double* drecv = ctx->xbuf_recv;
-    CK(cudaMemcpyAsync(dsend, acc, 5 * 8, cudaMemcpyHostToDevice, ctx->work));
-    NK(ncclAllGather(dsend, drecv, 5, ncclFloat64, ctx->comm, ctx->work));
-    std::vector<double> g((size_t)ctx->nranks * 5);
-    CK(cudaMemcpyAsync(g.data(), drecv, g.size() * 8, cudaMemcpyDeviceToHost, ctx->work));
-    CK(cudaStreamSynchronize(ctx->work));
-    for (int q = 0; q < 5; ++q) acc[q] = 0.0;
-    for (int r = 0; r < ctx->nranks; ++r)
-      for (int q = 0; q < 5; ++q) acc[q] = acc[q] + g[(size_t)r * 5 + q];
-  }
-#endif
   out->vol = acc[0]; out->mass = acc[1]; out->ie = acc[2]; out->ke = acc[3]; out->press = acc[4];
   int rc2 = join_out(ctx);
   return rc ? rc : rc2;
@@ -1102,7 +1198,6 @@ int clover_read_field(clover_ctx* ctx, int32_t field_id, double* host, int64_t n
   if (!ctx || !host) return fail(CLOVER_ERR_ARG, "NULL argument");
   FieldMap m;
   if (field_map(field_id, &m)) return fail(CLOVER_ERR_ARG, "unknown field id");
-  if (ctx->nranks > 1) return fail(CLOVER_ERR_STATE, "clover_read_field: multi-rank gather not supported yet");
   int rc = join_in(ctx);
   if (rc) return rc;
   if (field_id == CLOVER_F_PRESSURE || field_id == CLOVER_F_SOUNDSPEED) {
@@ -1112,7 +1207,7 @@ int clover_read_field(clover_ctx* ctx, int32_t field_id, double* host, int64_t n
       LAUNCH_CHECK();
     }
   }
-  rc = gather_local(ctx, m.buf, kBufKind[m.buf], host, n);
+  rc = gather_all(ctx, m.buf, kBufKind[m.buf], host, n);
   if (rc) return rc;
   return check_err(ctx);
 }
@@ -1137,7 +1232,6 @@ int clover_write_field(clover_ctx* ctx, int32_t field_id, const double* host, in
     case CLOVER_F_YVEL0: buf = B_V0; break;
     default: return fail(CLOVER_ERR_ARG, "only density0, energy0, xvel0, yvel0 are writable");
   }
-  if (ctx->nranks > 1) return fail(CLOVER_ERR_STATE, "clover_write_field: multi-rank scatter not supported yet");
   int rc = join_in(ctx);
   if (rc) return rc;
   rc = scatter_local(ctx, buf, kBufKind[buf], host, n);
@@ -1200,7 +1294,6 @@ int clover_checkpoint_bytes(clover_ctx* ctx, int64_t* bytes) {
 
 int clover_checkpoint(clover_ctx* ctx, void* host, int64_t bytes) {
   if (!ctx || !host) return fail(CLOVER_ERR_ARG, "NULL argument");
-  if (ctx->nranks > 1) return fail(CLOVER_ERR_STATE, "checkpoint: single-process contexts only");
   int64_t need;
   clover_checkpoint_bytes(ctx, &need);
   if (bytes < need) return fail(CLOVER_ERR_ARG, "checkpoint buffer too small");
@@ -1224,17 +1317,16 @@ int clover_checkpoint(clover_ctx* ctx, void* host, int64_t bytes) {
   double* p = (double*)((char*)host + sizeof(hd));
   const int64_t nc = (int64_t)ctx->g.x_cells * ctx->g.y_cells;
   const int64_t nn = (int64_t)(ctx->g.x_cells + 1) * (ctx->g.y_cells + 1);
-  rc = gather_local(ctx, B_D0, K_CELL, p, nc);
-  if (!rc) rc = gather_local(ctx, B_E0, K_CELL, p + nc, nc);
-  if (!rc) rc = gather_local(ctx, B_U0, K_XVEL, p + 2 * nc, nn);
-  if (!rc) rc = gather_local(ctx, B_V0, K_YVEL, p + 2 * nc + nn, nn);
+  rc = gather_all(ctx, B_D0, K_CELL, p, nc);
+  if (!rc) rc = gather_all(ctx, B_E0, K_CELL, p + nc, nc);
+  if (!rc) rc = gather_all(ctx, B_U0, K_XVEL, p + 2 * nc, nn);
+  if (!rc) rc = gather_all(ctx, B_V0, K_YVEL, p + 2 * nc + nn, nn);
   if (rc) return rc;
   return join_out(ctx);
 }
 
 int clover_restart(clover_ctx* ctx, const void* host, int64_t bytes) {
   if (!ctx || !host) return fail(CLOVER_ERR_ARG, "NULL argument");
-  if (ctx->nranks > 1) return fail(CLOVER_ERR_STATE, "restart: single-process contexts only");
   int64_t need;
   clover_checkpoint_bytes(ctx, &need);
   if (bytes < need) return fail(CLOVER_ERR_ARG, "checkpoint buffer too small");
