@@ -175,6 +175,8 @@ def main():
     ap.add_argument("--mesh", type=int, nargs=2, default=None, help="override global mesh (nx ny)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-active", action="store_true",
+                    help="skip the fully-active-flow side measurement")
     ap.add_argument("--strong", action="store_true",
                     help="configs[3]: 7680^2 strong-scaled over the ranks (default: configs[4] weak)")
     args = ap.parse_args()
@@ -289,6 +291,33 @@ def main():
                "d2h_bytes_per_step": 8 * (2 * nc + 2 * nn), "steps": ke,
                "api": "clover_step_host (h2d state, 1 step, d2h state)"}
 
+    # side measurement: the same mesh with every cell moving (seeded smooth
+    # random state + noise, workloads.random_state_fields), so the headline
+    # is not an artifact of the bm deck's quiescent regions
+    active = None
+    if world == 1 and not args.no_active:
+        from workloads import random_state_fields
+        adeck = bm_deck(nx, ny)
+        adeck["max_timestep"] = 1.0
+        sim.close()
+        act = Clover(adeck, stream=stream)
+        act.load_state(random_state_fields(7, nx, ny, smooth=True))
+        act.step(args.warmup)
+        act.sync()
+        a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        torch.cuda.synchronize()
+        a0.record(stream)
+        act.step(args.steps)
+        a1.record(stream)
+        torch.cuda.synchronize()
+        act.sync()
+        ams = a0.elapsed_time(a1) / args.steps
+        active = {"ms_per_step": ams, "value": cells / (ams / 1e3), "unit": UNIT,
+                  "state": "workloads.random_state_fields(7, smooth=True): every cell moving, limiters active"}
+        act.close()
+        sim = Clover(deck, px=px, py=py, rank=rank, nranks=world, unique_id=uid, stream=stream)
+        sim.step(args.steps + args.warmup)
+
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         cdeck = bm_deck(nx, ny)
@@ -315,6 +344,7 @@ def main():
                 "gpu_launches": kps * args.steps,
                 "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "clocks": clk,
                 "kernels": kernels,
+                "active_flow": active,
                 "summary_after": summ}
         print(json.dumps(line), flush=True)
     sim.close()
