@@ -156,8 +156,9 @@ ks_visc_dt(Chunk c, const double* __restrict__ d0, const double* __restrict__ e0
 constexpr int LW = 30;   // owned columns per warp
 constexpr int LKS = CLOVER_LKS;  // rows per segment
 
-#ifndef CLOVER_TMA_LAGR
 #define CLOVER_TMA_LAGR 1
+#ifndef CLOVER_TMA_RELEASE_FENCE  // proxy fence before refilling a slot (A/B: no measurable cost)
+#define CLOVER_TMA_RELEASE_FENCE 1
 #endif
 #if CLOVER_TMA_LAGR
 // TMA-staged variant: rows of d0, e0, q (cells) and u0, v0 (nodes) stream
@@ -318,151 +319,16 @@ ks_lagrangian(Chunk c, const double* __restrict__ d0, const double* __restrict__
     rl_m = rl; phl_m = phl; ql_m = ql;
     u0_m = u0_c; v0_m = v0_c; u0r_m = u0r_c; v0r_m = v0r_c;
     u1_m = u1_c; v1_m = v1_c;
-    // row k is consumed: refill its slot with row k+LSTG
+    // row k is consumed (every value read from its slot is already in
+    // registers and used): refill its slot with row k+LSTG
+#if CLOVER_TMA_RELEASE_FENCE
     fence_proxy_async();
+#endif
     __syncwarp();
     if (lane == 0 && k + LSTG <= r_last) issue(k + LSTG);
   }
 }
-#else
-__global__ void LB_HEAVY
-ks_lagrangian(Chunk c, const double* __restrict__ d0, const double* __restrict__ e0,
-              const double* __restrict__ u0, const double* __restrict__ v0,
-              const double* __restrict__ q, double* __restrict__ d1, double* __restrict__ e1,
-              double* __restrict__ u1, double* __restrict__ v1, double* __restrict__ fx,
-              double* __restrict__ fy, const StepScalars* __restrict__ s) {
-  const int lane = threadIdx.x & 31;
-  const int gw = blockIdx.x * (SB / 32) + (threadIdx.x >> 5);
-  const int J0 = 1 + LW * gw;
-  const int j = J0 - 1 + lane;
-  if (J0 > c.nx) return;  // whole warp beyond the chunk
-  const int k0 = blockIdx.y * LKS + 1;
-  const int k1 = min(k0 + LKS, c.ny + 1);  // cell rows [k0, k1)
-  const double dt = s->dt, dx = c.dx, dy = c.dy;
-  const int P = c.pitch;
-  // column validity: cells exist for j in [0, nx+1] (ring incl.)
-  const bool colok = j <= c.nx + 1;
-  // mirrored-lane sources for the x walls
-  int src = lane;
-  if (c.wl && j == 0) src = lane + 1;
-  if (c.wr && j == c.nx + 1) src = lane - 1;
-  const bool xwall_warp = __any_sync(FULL, src != lane);
-
-  // rolling state (row k-1)
-  double r_m = 1.0, e_m = 0.0, q_m = 0.0, ph_m = 0.0;     // cell (j, k-1)
-  double rl_m = 1.0, phl_m = 0.0, ql_m = 0.0;             // cell (j-1, k-1)
-  double u0_m = 0.0, v0_m = 0.0, u0r_m = 0.0, v0r_m = 0.0; // nodes (j,k-1), (j+1,k-1)
-  double u1_m = 0.0, v1_m = 0.0;                          // node (j, k-1) after accelerate
-  double u0_c = 0.0, v0_c = 0.0, u0r_c = 0.0, v0r_c = 0.0; // nodes (j,k), (j+1,k)
-
-  // node row k0-1 (bottom of the first ring cell row)
-  if (colok) {
-    const int in = idx(c, j, k0 - 1);
-    u0_c = u0[in]; v0_c = v0[in]; u0r_c = u0[in + 1]; v0r_c = v0[in + 1];
-  }
-  STREAM_LOOP
-  for (int k = k0 - 1; k <= k1; ++k) {
-    // ---- A: cell row k (ring rows k0-1 and k1 included)
-    double r = 1.0, e = 0.0, qq = 0.0, ph = 0.0;
-    double u0_n = 0.0, v0_n = 0.0, u0r_n = 0.0, v0r_n = 0.0;  // nodes (j,k+1), (j+1,k+1)
-    if (colok) {
-      const int i = idx(c, j, k);
-      r = d0[i]; e = e0[i]; qq = q[i];
-      u0_n = u0[i + P]; v0_n = v0[i + P]; u0r_n = u0[i + P + 1]; v0r_n = v0[i + P + 1];
-      // rows outside a reflective wall take the mirrored row's predictor
-      int kp = k;
-      if (c.wb && k == 0) kp = 1;
-      if (c.wt && k == c.ny + 1) kp = c.ny;
-      double pr_, pe_, pq_, ua, ub, uc, ud, va, vb, vc, vd;
-      if (kp == k) {
-        pr_ = r; pe_ = e; pq_ = qq;
-        ua = u0_c; ub = u0_n; uc = u0r_c; ud = u0r_n;
-        va = v0_c; vb = v0r_c; vc = v0_n; vd = v0r_n;
-      } else {
-        const int ip = idx(c, j, kp);
-        pr_ = d0[ip]; pe_ = e0[ip]; pq_ = q[ip];
-        ua = u0[ip]; ub = u0[ip + P]; uc = u0[ip + 1]; ud = u0[ip + P + 1];
-        va = v0[ip]; vb = v0[ip + 1]; vc = v0[ip + P]; vd = v0[ip + P + 1];
-      }
-      DivFast f;
-      ph = pdv_predict_pressure(f, pr_, pe_, pq_, ua, ub, uc, ud, va, vb, vc, vd, dx, dy, c.rvol, dt);
-      if (f.bad) {
-        DivIEEE x;
-        ph = pdv_predict_pressure(x, pr_, pe_, pq_, ua, ub, uc, ud, va, vb, vc, vd, dx, dy, c.rvol, dt);
-      }
-    }
-    if (xwall_warp) ph = __shfl_sync(FULL, ph, src);
-    const double rl = __shfl_up_sync(FULL, r, 1);
-    const double phl = __shfl_up_sync(FULL, ph, 1);
-    const double ql = __shfl_up_sync(FULL, qq, 1);
-
-    // ---- B: accelerate at node (j,k), node rows [k0, k1]
-    double u1_c = 0.0, v1_c = 0.0;
-    if (k >= k0 && colok) {
-      const double rr[4] = {rl_m, r_m, r, rl};
-      const double pp[4] = {phl_m, ph_m, ph, phl};
-      const double qv[4] = {ql_m, q_m, qq, ql};
-      DivFast f;
-      accelerate_node(f, rr, pp, qv, u0_c, v0_c, dx, dy, dt, u1_c, v1_c);
-      if (f.bad) {
-        DivIEEE x;
-        accelerate_node(x, rr, pp, qv, u0_c, v0_c, dx, dy, dt, u1_c, v1_c);
-      }
-    }
-    const double u1r_c = __shfl_down_sync(FULL, u1_c, 1);
-    const double v1r_c = __shfl_down_sync(FULL, v1_c, 1);
-    const double u1r_m = __shfl_down_sync(FULL, u1_m, 1);
-    const double v1r_m = __shfl_down_sync(FULL, v1_m, 1);
-
-    // ---- C: PdV corrector + flux_calc of cell (j, k-1), rows [k0, k1)
-    const int kc = k - 1;
-    if (kc >= k0 && lane >= 1 && lane <= LW && j <= c.nx) {
-      // nodes: a=(j,kc) b=(j,kc+1) c=(j+1,kc) d=(j+1,kc+1)
-      const double lsum = u0_m + u0_c + u1_m + u1_c;
-      const double rsum = u0r_m + u0r_c + u1r_m + u1r_c;
-      const double bsum = v0_m + v0r_m + v1_m + v1r_m;
-      const double tsum = v0_c + v0r_c + v1_c + v1r_c;
-      double ev, dvv;
-      DivFast f;
-      pdv_correct(f, r_m, e_m, ph_m, q_m, lsum, rsum, bsum, tsum, dx, dy, c.rvol, dt, ev, dvv);
-      if (f.bad) {
-        DivIEEE x;
-        pdv_correct(x, r_m, e_m, ph_m, q_m, lsum, rsum, bsum, tsum, dx, dy, c.rvol, dt, ev, dvv);
-      }
-      const int ic = idx(c, j, kc);
-      const bool near = ncol || near_wall_row(c, kc);
-      store_at(c, e1, K_CELL, j, kc, ic, near, ev);
-      store_at(c, d1, K_CELL, j, kc, ic, near, dvv);
-      const double cx = 0.25 * dt * dy, cy = 0.25 * dt * dx;
-      store_at(c, fx, K_XFACE, j, kc, ic, near, cx * lsum);
-      store_at(c, fy, K_YFACE, j, kc, ic, near, cy * bsum);
-      if (j == c.nx) store_field(c, fx, K_XFACE, j + 1, kc, cx * rsum);
-      if (kc == c.ny) store_field(c, fy, K_YFACE, j, kc + 1, cy * tsum);
-      store_at(c, u1, K_XVEL, j, kc, ic, near, u1_m);
-      store_at(c, v1, K_YVEL, j, kc, ic, near, v1_m);
-      if (j == c.nx) {
-        store_field(c, u1, K_XVEL, j + 1, kc, u1r_m);
-        store_field(c, v1, K_YVEL, j + 1, kc, v1r_m);
-      }
-      if (kc == c.ny) {
-        store_field(c, u1, K_XVEL, j, kc + 1, u1_c);
-        store_field(c, v1, K_YVEL, j, kc + 1, v1_c);
-      }
-      if (j == c.nx && kc == c.ny) {
-        store_field(c, u1, K_XVEL, j + 1, kc + 1, u1r_c);
-        store_field(c, v1, K_YVEL, j + 1, kc + 1, v1r_c);
-      }
-    }
-    // ---- roll
-    r_m = r; e_m = e; q_m = qq; ph_m = ph;
-    rl_m = rl; phl_m = phl; ql_m = ql;
-    u0_m = u0_c; v0_m = v0_c; u0r_m = u0r_c; v0r_m = v0r_c;
-    u0_c = u0_n; v0_c = v0_n; u0r_c = u0r_n; v0r_c = v0r_n;
-    u1_m = u1_c; v1_m = v1_c;
-  }
-}
-
-#endif  // CLOVER_TMA_LAGR
+#endif  // CLOVER_TMA_LAGR (the register-only variant was measured 3% slower; see git history)
 
 // ================================================================ advec_cell x
 // Warp strip: lane l <-> face/cell column j = J0 + l, J0 = 1 + 31*(warp);
@@ -602,6 +468,16 @@ ks_advec_cell_y(Chunk c, const double* __restrict__ rho, const double* __restric
       } else {
         ru = R4; rd = R3; rw = R2; eu = E4; ed = E3; ew = E2; pvd = pv1;
       }
+#ifdef CLOVER_DIAG_TRIVIAL
+      m1 = F * rd + pvd * (ru + rw); ef1 = m1 * (ed + eu + ew);
+    }
+    double ro, eo;
+    {
+      const double flo = fy[i], fhi = fy[i + P];
+      // keep every load live, keep the state physical
+      ro = R2 + 0.0 * (pv0 + m0 - m1 + flo - fhi); eo = E2 + 0.0 * (ef0 - ef1);
+    }
+#else
       DivFast f;
       cell_face_flux(f, F, pvd, ru, rd, rw, eu, ed, ew, m1, ef1);
       if (f.bad) {
@@ -619,6 +495,7 @@ ks_advec_cell_y(Chunk c, const double* __restrict__ rho, const double* __restric
         cell_update(x, R2, E2, pv0, m0, m1, ef0, ef1, flo, fhi, ro, eo);
       }
     }
+#endif
     const bool near = ncol || near_wall_row(c, k);
     store_at(c, rho_out, K_CELL, j, k, i, near, ro);
     store_at(c, en_out, K_CELL, j, k, i, near, eo);
