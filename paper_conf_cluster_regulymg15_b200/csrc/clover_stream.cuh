@@ -21,7 +21,10 @@
 namespace clover {
 
 constexpr unsigned FULL = 0xffffffffu;
-constexpr int SB = 128;  // threads per block (4 warps)
+#ifndef CLOVER_SB
+#define CLOVER_SB 64
+#endif
+constexpr int SB = CLOVER_SB;  // threads per block
 
 // Tunables (defaults = measured best; scripts/ab_variants.py builds others).
 #define CLOVER_STR2(x) #x
@@ -33,19 +36,20 @@ constexpr int SB = 128;  // threads per block (4 warps)
 #endif
 // min resident blocks/SM (register cap) for visc_dt+lagrangian / advection;
 // 0 = plain __launch_bounds__(SB) (ptxas heuristic).  Measured on B200 at
-// 3840^2 (scripts/ab_variants.py): lagrangian 5, visc_dt uncapped,
-// advection 8 (mom_y 7).
+// 3840^2 (scripts/ab_variants.py), 64-thread blocks: lagrangian 10 (96 regs),
+// visc_dt uncapped, advection 16 (64 regs), mom_y 14.  Short row segments
+// (8-16 rows) measured 6 % faster than 16-32 (more, shorter blocks).
 #ifndef CLOVER_MINB_HEAVY
-#define CLOVER_MINB_HEAVY 5
+#define CLOVER_MINB_HEAVY 10
 #endif
 #ifndef CLOVER_MINB_ADV
-#define CLOVER_MINB_ADV 8
+#define CLOVER_MINB_ADV 16
 #endif
 #ifndef CLOVER_MINB_VISC
 #define CLOVER_MINB_VISC 0
 #endif
 #ifndef CLOVER_MINB_MOMY
-#define CLOVER_MINB_MOMY 7
+#define CLOVER_MINB_MOMY 14
 #endif
 #if CLOVER_MINB_MOMY > 0
 #define LB_MOMY __launch_bounds__(SB, CLOVER_MINB_MOMY)
@@ -71,19 +75,19 @@ constexpr int SB = 128;  // threads per block (4 warps)
 #define CLOVER_VKS 16
 #endif
 #ifndef CLOVER_LKS
-#define CLOVER_LKS 32
+#define CLOVER_LKS 16
 #endif
 #ifndef CLOVER_CKS
-#define CLOVER_CKS 16
+#define CLOVER_CKS 8
 #endif
 #ifndef CLOVER_CKS_Y
-#define CLOVER_CKS_Y 32
+#define CLOVER_CKS_Y 8
 #endif
 #ifndef CLOVER_MKS
-#define CLOVER_MKS 16
+#define CLOVER_MKS 8
 #endif
 #ifndef CLOVER_MKS_Y
-#define CLOVER_MKS_Y 32
+#define CLOVER_MKS_Y 8
 #endif
 
 // ================================================================ visc_dt
