@@ -56,10 +56,10 @@ struct ViscIn {
   double u00, u10, u01, u11, v00, v10, v01, v11;
 };
 
-// c.3 viscosity then c.4 calc_dt for one cell; returns dt_cell, writes q.
+// c.3 viscosity of one cell (writes q) and the c.4 sound-speed term cc.
 template <class D>
-__device__ __forceinline__ double visc_dt_cell(D& dv, const ViscIn& I, const Chunk& C,
-                                               const DtParams& prm, double& qv) {
+__device__ __forceinline__ void visc_cell(D& dv, const ViscIn& I, const Chunk& C, double& qv,
+                                          double& cc) {
   const double dx = C.dx, dy = C.dy;
   const double u00 = I.u00, u10 = I.u10, u01 = I.u01, u11 = I.u11;
   const double v00 = I.v00, v10 = I.v10, v01 = I.v01, v11 = I.v11;
@@ -86,25 +86,49 @@ __device__ __forceinline__ double visc_dt_cell(D& dv, const ViscIn& I, const Chu
     double grad2 = grad * grad;
     qv = 2.0 * I.rho * grad2 * limiter * limiter;
   }
-  const double vol = dx * dy;
   double cs = eos_soundspeed(dv, I.rho, I.e);
-  double cc = cs * cs;
+  cc = cs * cs;
   cc = cc + dv(2.0 * qv, I.rho);
   cc = fmax(sqrt(cc), G_SMALL);
-  double dtct = dv.nz(prm.dtc_safe * fmin(dx, dy), cc);
-  double dvv = 0.0;
-  double dv1 = (u00 + u01) * dy;
-  double dv2 = (u10 + u11) * dy;
-  dvv = dvv + dv2 - dv1;
-  double dtut = dv.nz(prm.dtu_safe * 2.0 * vol, fmax(fmax(fabs(dv1), fabs(dv2)), G_SMALL * vol));
-  dv1 = (v00 + v10) * dx;
-  dv2 = (v01 + v11) * dx;
-  dvv = dvv + dv2 - dv1;
-  double dtvt = dv.nz(prm.dtv_safe * 2.0 * vol, fmax(fmax(fabs(dv1), fabs(dv2)), G_SMALL * vol));
-  dvv = dv.c(dvv, 2.0 * vol, C.r2vol);
-  double dtdivt = (dvv < -G_SMALL) ? prm.dtdiv_safe * dv.nz(-1.0, dvv) : G_BIG;
-  return fmin(fmin(dtct, dtut), fmin(dtvt, dtdivt));
 }
+
+// c.4 calc_dt, reduced over a set of cells without per-cell divisions.
+// Per cell the reading takes
+//   dt_cell = min( A_c / cc, A_u / du, A_v / dv', dtdiv_safe * (-1 / (w / 2vol)) )
+// (the last term only when w / 2vol < -g_small, else g_big), with A_c, A_u,
+// A_v and 2vol launch constants and every quotient correctly rounded.
+// Correct rounding is monotone (x <= y => RN(x) <= RN(y)), so the minimum
+// over cells of RN(A / d) is RN(A / max d), that of RN(w / 2vol) is
+// RN(min w / 2vol), and -1/x grows with x < 0: the minimum of the per-cell
+// dt over the set equals the dt computed once from the four extremes below,
+// bit for bit.  The kernel keeps the extremes per thread and divides once.
+struct DtAcc {
+  double ccmax = 0.0, dumax = 0.0, dvmax = 0.0, wmin = G_BIG;
+  __device__ __forceinline__ void add(const ViscIn& I, const Chunk& C, double cc) {
+    const double dx = C.dx, dy = C.dy, vol = dx * dy;
+    double dvv = 0.0;
+    double dv1 = (I.u00 + I.u01) * dy;
+    double dv2 = (I.u10 + I.u11) * dy;
+    dvv = dvv + dv2 - dv1;
+    dumax = fmax(dumax, fmax(fmax(fabs(dv1), fabs(dv2)), G_SMALL * vol));
+    dv1 = (I.v00 + I.v10) * dx;
+    dv2 = (I.v01 + I.v11) * dx;
+    dvv = dvv + dv2 - dv1;
+    dvmax = fmax(dvmax, fmax(fmax(fabs(dv1), fabs(dv2)), G_SMALL * vol));
+    wmin = fmin(wmin, dvv);
+    ccmax = fmax(ccmax, cc);
+  }
+  // dt of the set (call only if at least one cell was added)
+  __device__ __forceinline__ double dt(const Chunk& C, const DtParams& prm) const {
+    const double dx = C.dx, dy = C.dy, vol = dx * dy;
+    double dtct = div_fast_nz(prm.dtc_safe * fmin(dx, dy), ccmax);
+    double dtut = div_fast_nz(prm.dtu_safe * 2.0 * vol, dumax);
+    double dtvt = div_fast_nz(prm.dtv_safe * 2.0 * vol, dvmax);
+    double dvv = wmin / (2.0 * vol);
+    double dtdivt = (dvv < -G_SMALL) ? prm.dtdiv_safe * div_fast_nz(-1.0, dvv) : G_BIG;
+    return fmin(fmin(dtct, dtut), fmin(dtvt, dtdivt));
+  }
+};
 
 // ------------------------------------------------ k_dt_finalize (c.4 tail)
 __global__ void k_dt_finalize(StepScalars* __restrict__ s, double* __restrict__ hist,

@@ -111,6 +111,7 @@ ks_visc_dt(Chunk c, const double* __restrict__ d0, const double* __restrict__ e0
     double rho = d0[i], ein = e0[i];
     double pc = eos_pressure(rho, ein);
     double ua = u0[i], ub = u0[i + 1], va = v0[i], vb = v0[i + 1];
+    DtAcc acc;
     STREAM_LOOP
     for (int k = k0; k < k1; ++k, i += P) {
       const double rhon = d0[i + P], en = e0[i + P];
@@ -123,18 +124,19 @@ ks_visc_dt(Chunk c, const double* __restrict__ d0, const double* __restrict__ e0
       const double uc = u0[i + P], ud = u0[i + P + 1], vc = v0[i + P], vd = v0[i + P + 1];
       I.u00 = ua; I.u10 = ub; I.u01 = uc; I.u11 = ud;
       I.v00 = va; I.v10 = vb; I.v01 = vc; I.v11 = vd;
-      double qv;
+      double qv, cc;
       DivFast f;
-      double dtc = visc_dt_cell(f, I, c, prm, qv);
+      visc_cell(f, I, c, qv, cc);
       if (f.bad) {
         DivIEEE x;
-        dtc = visc_dt_cell(x, I, c, prm, qv);
+        visc_cell(x, I, c, qv, cc);
       }
-      dtl = fmin(dtl, dtc);
+      acc.add(I, c, cc);
       store_at(c, q, K_CELL, j, k, i, ncol || near_wall_row(c, k), qv);
       pcm = pc; pc = I.pt; rho = rhon; ein = en;
       ua = uc; ub = ud; va = vc; vb = vd;
     }
+    dtl = acc.dt(c, prm);
   }
   for (int o = 16; o > 0; o >>= 1) dtl = fmin(dtl, __shfl_xor_sync(FULL, dtl, o));
   __shared__ double wmin[SB / 32];
