@@ -1,0 +1,42 @@
+"""Host checks of the arithmetic identities the CUDA path relies on to
+restructure work without changing a single bit.
+
+These run numpy fp64 (IEEE, round-to-nearest-even) on CPU; the GPU parity
+tests then confirm the kernels end to end (dt history bitwise).
+"""
+import numpy as np
+
+
+def _logu(rng, lo, hi, n):
+    return np.exp(rng.uniform(np.log(lo), np.log(hi), n))
+
+
+def test_min_of_rounded_quotients_is_quotient_of_extreme():
+    # DtAcc (clover_kernels.cuh): min_i RN(A / d_i) == RN(A / max_i d_i)
+    rng = np.random.default_rng(11)
+    for trial in range(200):
+        A = float(_logu(rng, 1e-6, 1e3, 1)[0])
+        n = int(rng.integers(1, 64))
+        if trial % 3 == 0:  # near-ties: d differing in the last few ulps
+            d = np.nextafter(np.full(n, _logu(rng, 1e-3, 1e3, 1)[0]), np.inf)
+            d = d * (1 + rng.integers(0, 8, n) * 2.0**-52)
+        else:
+            d = _logu(rng, 1e-16, 1e6, n)
+        per_cell = np.min(A / d)
+        once = A / np.max(d)
+        assert per_cell.tobytes() == np.float64(once).tobytes()
+
+
+def test_min_of_divergence_term_is_term_of_min():
+    # dtdivt: per cell (w/2vol < -g_small) ? s * RN(-1 / RN(w/2vol)) : g_big
+    rng = np.random.default_rng(12)
+    g_small, g_big, s = 1.0e-16, 1.0e21, 0.7
+    for _ in range(200):
+        vol2 = 2.0 * float(_logu(rng, 1e-8, 1.0, 1)[0])
+        n = int(rng.integers(1, 64))
+        w = rng.normal(0.0, 1.0, n) * float(_logu(rng, 1e-20, 1.0, 1)[0])
+        dvv = w / vol2
+        cell = np.where(dvv < -g_small, s * (-1.0 / np.where(dvv < -g_small, dvv, -1.0)), g_big)
+        m = np.min(w) / vol2
+        once = s * (-1.0 / m) if m < -g_small else g_big
+        assert np.float64(np.min(cell)).tobytes() == np.float64(once).tobytes()
