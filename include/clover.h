@@ -207,6 +207,12 @@ int clover_debug_partial_step(clover_ctx* ctx, int32_t nkernels);
 int clover_debug_read_buffer(clover_ctx* ctx, int32_t buffer_id, int32_t kind,
                              double* host, int64_t n);
 
+/* Debug: total number of warp segments the IEEE-division fixup launches
+ * have recomputed since clover_init (DivFast flagged a numerator below
+ * 2^-900 there), summed over local chunks.  Synchronises
+ * the context's stream.  Test only. */
+int clover_debug_fix_count(clover_ctx* ctx, int64_t* out);
+
 /* Test: compare the library's internal fp64 division (div_rn) with IEEE
  * a/b bit for bit on n random operand pairs (exponents in [-emax, emax],
  * 1/16 zero numerators); *mismatches receives the count, example_ab (may be

@@ -39,6 +39,7 @@ EXPORTS = ["clover_workspace_bytes", "clover_nccl_unique_id", "clover_init", "cl
            "clover_read_field", "clover_write_field", "clover_sync", "clover_set_graphs",
            "clover_kernels_per_step", "clover_debug_partial_step", "clover_debug_read_buffer",
            "clover_profile_steps", "clover_profile_name", "clover_debug_div_check",
+           "clover_debug_fix_count",
            "clover_checkpoint_plan", "clover_debug_set_virtual_remote", "clover_checkpoint_bytes", "clover_checkpoint", "clover_restart", "clover_finalize", "clover_error_string", "clover_last_error", "clover_abi_version"]
 
 
@@ -105,6 +106,8 @@ def load(build_if_missing: bool = True):
     L.clover_profile_steps.argtypes = [c_void_p, c_int32, dptr, ctypes.POINTER(c_int64), c_int32]
     L.clover_profile_name.argtypes = [c_int32]
     L.clover_profile_name.restype = ctypes.c_char_p
+    if hasattr(L, "clover_debug_fix_count"):  # absent from older builds (A/B harness)
+        L.clover_debug_fix_count.argtypes = [c_void_p, ctypes.POINTER(c_int64)]
     L.clover_debug_div_check.argtypes = [c_int64, ctypes.c_uint64, c_int32, ctypes.POINTER(c_int64), dptr]
     L.clover_checkpoint_plan.argtypes = [c_int32, ctypes.POINTER(ctypes.c_uint32), ctypes.POINTER(c_int32),
                                          ctypes.POINTER(ctypes.c_char_p)]
@@ -117,6 +120,8 @@ def load(build_if_missing: bool = True):
     L.clover_error_string.restype = ctypes.c_char_p
     L.clover_last_error.restype = ctypes.c_char_p
     for name in EXPORTS:
+        if os.environ.get("CLOVER_LIB") and not hasattr(L, name):
+            continue  # an older build under the A/B harness
         if name not in ("clover_error_string", "clover_last_error", "clover_profile_name"):
             getattr(L, name).restype = c_int32
     _lib = L
@@ -314,6 +319,12 @@ class Clover:
 
     def debug_partial_step(self, nkernels: int):
         _check(load().clover_debug_partial_step(self._ctx, nkernels), "clover_debug_partial_step")
+
+    def debug_fix_count(self) -> int:
+        """Warp segments recomputed so far by the IEEE-division fixup launches."""
+        n = c_int64()
+        _check(load().clover_debug_fix_count(self._ctx, ctypes.byref(n)), "clover_debug_fix_count")
+        return n.value
 
     def debug_read(self, buf: str, kind: str) -> np.ndarray:
         a = np.zeros(field_shape(kind, self.nx, self.ny), dtype=np.float64)

@@ -76,6 +76,7 @@ struct ChunkState {
   double* buf[NBUF];
   double* partials;  // summary partials, ntx*nty*5
   int ntx, nty;
+  FixSlot fix;       // warps to redo with IEEE division (clover_stream.cuh)
 };
 
 struct Layout {
@@ -109,6 +110,23 @@ int64_t field_elems(int nx, int ny, int* pitch_out) {
   int rows = ny + 2 + 2 * HALO;
   return (int64_t)pitch * rows;
 }
+
+// Fix-list capacity of a chunk: the most warps any step kernel's grid has
+// (grid shapes as in enqueue_step).
+inline int cdiv(int a, int b) { return (a + b - 1) / b; }
+dim3 grid_cols(int ncols, int nrows, int ks) { return dim3(cdiv(ncols, SB), cdiv(nrows, ks)); }
+dim3 grid_strip(int ncols, int width, int nrows, int ks) {
+  return dim3(cdiv(cdiv(ncols, width), SB / 32), cdiv(nrows, ks));
+}
+int64_t fix_capacity(int nx, int ny) {
+  const dim3 g[6] = {grid_cols(nx, ny, VKS),          grid_strip(nx, LW, ny, LKS),
+                     grid_strip(nx, CW_X, ny, CKS),    grid_cols(nx, ny, CKS_Y),
+                     grid_strip(nx + 1, MW_X, ny + 1, MKS), grid_cols(nx + 1, ny + 1, MKS_Y)};
+  int64_t m = 0;
+  for (const dim3& d : g) m = std::max<int64_t>(m, (int64_t)d.x * d.y * (SB / 32));
+  return m;
+}
+int64_t fix_bytes(int nx, int ny) { return kAlign + align_up(fix_capacity(nx, ny) * 8, kAlign); }
 
 }  // namespace
 
@@ -196,6 +214,7 @@ int64_t compute_workspace(const clover_grid* g, int px, int py, int rank, int nr
     bytes += NBUF * align_up(fe * 8, kAlign);
     int ntx = (nx + ST - 1) / ST, nty = (ny + ST - 1) / ST;
     bytes += align_up((int64_t)ntx * nty * 5 * 8, kAlign);
+    bytes += fix_bytes(nx, ny);
     maxrows = std::max<int64_t>(maxrows, ny + 2 + 2 * HALO);
     maxcols = std::max<int64_t>(maxcols, nx + 2 + 2 * HALO);
   }
@@ -404,12 +423,6 @@ void prof_mark(clover_ctx* ctx, int id) {
   ctx->prof_events.push_back({id, e});
 }
 
-// Launch geometry of the streaming kernels (clover_stream.cuh).
-inline int cdiv(int a, int b) { return (a + b - 1) / b; }
-dim3 grid_cols(int ncols, int nrows, int ks) { return dim3(cdiv(ncols, SB), cdiv(nrows, ks)); }
-dim3 grid_strip(int ncols, int width, int nrows, int ks) {
-  return dim3(cdiv(cdiv(ncols, width), SB / 32), cdiv(nrows, ks));
-}
 
 // Enqueue kernel phases [0, nphase) of one step (7 = full step).
 int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
@@ -420,7 +433,10 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
     for (auto& cs : ctx->chunks) {
       const Chunk& c = cs.c;
       ks_visc_dt<<<grid_cols(c.nx, c.ny, VKS), SB, 0, st>>>(c, cs.buf[B_D0], cs.buf[B_E0], cs.buf[B_U0],
-                                                             cs.buf[B_V0], cs.buf[B_Q], ctx->scal, ctx->dtp);
+                                                             cs.buf[B_V0], cs.buf[B_Q], ctx->scal, ctx->dtp, cs.fix);
+      STEP_LAUNCH_CHECK();
+      kf_visc_dt<<<FIX_BLOCKS, SB, 0, st>>>(c, cs.buf[B_D0], cs.buf[B_E0], cs.buf[B_U0], cs.buf[B_V0],
+                                            cs.buf[B_Q], ctx->scal, ctx->dtp, cs.fix);
       STEP_LAUNCH_CHECK();
     }
     int rc = exchange(ctx, {B_Q});
@@ -443,7 +459,11 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
       const Chunk& c = cs.c;
       ks_lagrangian<<<grid_strip(c.nx, LW, c.ny, LKS), SB, 0, st>>>(
           c, cs.buf[B_D0], cs.buf[B_E0], cs.buf[B_U0], cs.buf[B_V0], cs.buf[B_Q], cs.buf[B_D1],
-          cs.buf[B_E1], cs.buf[B_U1], cs.buf[B_V1], cs.buf[B_FX], cs.buf[B_FY], ctx->scal);
+          cs.buf[B_E1], cs.buf[B_U1], cs.buf[B_V1], cs.buf[B_FX], cs.buf[B_FY], ctx->scal, cs.fix);
+      STEP_LAUNCH_CHECK();
+      kf_lagrangian<<<FIX_BLOCKS, SB, 0, st>>>(
+          c, cs.buf[B_D0], cs.buf[B_E0], cs.buf[B_U0], cs.buf[B_V0], cs.buf[B_Q], cs.buf[B_D1],
+          cs.buf[B_E1], cs.buf[B_U1], cs.buf[B_V1], cs.buf[B_FX], cs.buf[B_FY], ctx->scal, cs.fix);
       STEP_LAUNCH_CHECK();
     }
     int rc = exchange(ctx, {B_D1, B_E1, B_U1, B_V1, B_FX, B_FY});
@@ -467,16 +487,26 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
         const double* fy = cs.buf[B_FY];
         if (xdir) {
           const dim3 g = grid_strip(c.nx, CW_X, c.ny, CKS);
-          if (sweep == 1)
-            ks_advec_cell_x<1><<<g, SB, 0, st>>>(c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf]);
-          else
-            ks_advec_cell_x<2><<<g, SB, 0, st>>>(c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf]);
+          if (sweep == 1) {
+            ks_advec_cell_x<1><<<g, SB, 0, st>>>(c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf], cs.fix);
+            STEP_LAUNCH_CHECK();
+            kf_advec_cell_x<1><<<FIX_BLOCKS, SB, 0, st>>>(c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf], cs.fix);
+          } else {
+            ks_advec_cell_x<2><<<g, SB, 0, st>>>(c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf], cs.fix);
+            STEP_LAUNCH_CHECK();
+            kf_advec_cell_x<2><<<FIX_BLOCKS, SB, 0, st>>>(c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf], cs.fix);
+          }
         } else {
           const dim3 g = grid_cols(c.nx, c.ny, CKS_Y);
-          if (sweep == 1)
-            ks_advec_cell_y<1><<<g, SB, 0, st>>>(c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf]);
-          else
-            ks_advec_cell_y<2><<<g, SB, 0, st>>>(c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf]);
+          if (sweep == 1) {
+            ks_advec_cell_y<1><<<g, SB, 0, st>>>(c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf], cs.fix);
+            STEP_LAUNCH_CHECK();
+            kf_advec_cell_y<1><<<FIX_BLOCKS, SB, 0, st>>>(c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf], cs.fix);
+          } else {
+            ks_advec_cell_y<2><<<g, SB, 0, st>>>(c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf], cs.fix);
+            STEP_LAUNCH_CHECK();
+            kf_advec_cell_y<2><<<FIX_BLOCKS, SB, 0, st>>>(c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf], cs.fix);
+          }
         }
         STEP_LAUNCH_CHECK();
       }
@@ -490,16 +520,26 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
         const Chunk& c = cs.c;
         if (xdir) {
           const dim3 g = grid_strip(c.nx + 1, MW_X, c.ny + 1, MKS);
-          if (sweep == 1)
-            ks_advec_mom_x<1><<<g, SB, 0, st>>>(c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FY], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout]);
-          else
-            ks_advec_mom_x<2><<<g, SB, 0, st>>>(c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FY], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout]);
+          if (sweep == 1) {
+            ks_advec_mom_x<1><<<g, SB, 0, st>>>(c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FY], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout], cs.fix);
+            STEP_LAUNCH_CHECK();
+            kf_advec_mom_x<1><<<FIX_BLOCKS, SB, 0, st>>>(c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FY], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout], cs.fix);
+          } else {
+            ks_advec_mom_x<2><<<g, SB, 0, st>>>(c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FY], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout], cs.fix);
+            STEP_LAUNCH_CHECK();
+            kf_advec_mom_x<2><<<FIX_BLOCKS, SB, 0, st>>>(c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FY], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout], cs.fix);
+          }
         } else {
           const dim3 g = grid_cols(c.nx + 1, c.ny + 1, MKS_Y);
-          if (sweep == 1)
-            ks_advec_mom_y<1><<<g, SB, 0, st>>>(c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FX], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout]);
-          else
-            ks_advec_mom_y<2><<<g, SB, 0, st>>>(c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FX], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout]);
+          if (sweep == 1) {
+            ks_advec_mom_y<1><<<g, SB, 0, st>>>(c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FX], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout], cs.fix);
+            STEP_LAUNCH_CHECK();
+            kf_advec_mom_y<1><<<FIX_BLOCKS, SB, 0, st>>>(c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FX], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout], cs.fix);
+          } else {
+            ks_advec_mom_y<2><<<g, SB, 0, st>>>(c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FX], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout], cs.fix);
+            STEP_LAUNCH_CHECK();
+            kf_advec_mom_y<2><<<FIX_BLOCKS, SB, 0, st>>>(c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FX], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout], cs.fix);
+          }
         }
         STEP_LAUNCH_CHECK();
       }
@@ -860,6 +900,9 @@ int clover_init(const clover_grid* grid, const clover_state* states, int32_t nst
     cs.ntx = (c.nx + ST - 1) / ST; cs.nty = (c.ny + ST - 1) / ST;
     cs.partials = (double*)p;
     p += align_up((int64_t)cs.ntx * cs.nty * 5 * 8, kAlign);
+    cs.fix.hdr = (unsigned*)p;
+    cs.fix.e = (uint2*)(p + kAlign);
+    p += fix_bytes(c.nx, c.ny);
     maxrows = std::max<int64_t>(maxrows, c.ny + 2 + 2 * HALO);
     maxcols = std::max<int64_t>(maxcols, c.nx + 2 + 2 * HALO);
     ctx->chunks.push_back(cs);
@@ -951,9 +994,22 @@ int clover_debug_set_virtual_remote(clover_ctx* ctx, int32_t enable) {
   return CLOVER_OK;
 }
 
+int clover_debug_fix_count(clover_ctx* ctx, int64_t* out) {
+  if (!ctx || !out) return fail(CLOVER_ERR_ARG, "NULL argument");
+  CK(cudaStreamSynchronize(ctx->work));
+  int64_t t = 0;
+  for (auto& cs : ctx->chunks) {
+    unsigned h[3];
+    CK(cudaMemcpy(h, cs.fix.hdr, sizeof(h), cudaMemcpyDeviceToHost));
+    t += h[2];
+  }
+  *out = t;
+  return CLOVER_OK;
+}
+
 int clover_kernels_per_step(clover_ctx* ctx, int32_t* out) {
   if (!ctx || !out) return fail(CLOVER_ERR_ARG, "NULL argument");
-  *out = (int32_t)(ctx->chunks.size() * 6 + 1);
+  *out = (int32_t)(ctx->chunks.size() * 12 + 1);  // 6 step kernels + 6 fixups per chunk
   return CLOVER_OK;
 }
 

@@ -12,8 +12,13 @@
 // 1-3 "halo lanes".  Raw inputs at x-neighbours are plain L1-cached loads.
 //
 // All arithmetic is in the per-point functions of clover_kernels.cuh
-// (evaluation order of SURVEY 8(c)); division policy DivFast with a
-// per-point IEEE recompute when flagged.
+// (evaluation order of SURVEY 8(c)).  Each kernel is a warp-segment body
+// templated on the division policy.  The production launch runs it with
+// DivFast (no IEEE code in the kernel at all); a warp whose sticky
+// tiny-numerator flag is set pushes (warp, segment) onto a fix list, and a
+// small fixup launch right after (kf_*) recomputes exactly those warp
+// segments with IEEE division, overwriting the same outputs.  Every kernel
+// is out-of-place, so the inputs are still intact for the redo.
 #pragma once
 #include "clover_common.cuh"
 #include "clover_kernels.cuh"
@@ -90,19 +95,64 @@ constexpr int SB = CLOVER_SB;  // threads per block
 #define CLOVER_MKS_Y 8
 #endif
 
+// ---------------------------------------------------------------- fix lists
+// hdr[0] = number of entries, hdr[1] = finished fixup blocks, hdr[2] =
+// entries fixed so far (debug counter); e[] = (global
+// warp, segment) of every warp whose fast pass flagged.  Capacity = warps
+// of the fast grid (each warp pushes at most once), sized by the engine.
+struct FixSlot {
+  unsigned* hdr;
+  uint2* e;
+};
+__device__ __forceinline__ void fix_push(FixSlot f, int lane, unsigned gw, unsigned seg) {
+  if (lane == 0) {
+    const unsigned n = atomicAdd(f.hdr, 1u);
+    f.e[n] = make_uint2(gw, seg);
+  }
+}
+// Fixup driver: every flagged segment of ks rows is redone one row per warp
+// (row-parallel, so the fixup's latency is one row, not one segment); the
+// last block to finish resets the list.  run(gw, k0, k1, lane, w) with
+// k1 = k0 + 1; rows at or beyond `lim` are skipped.
+template <class Run>
+__device__ __forceinline__ void fix_loop(FixSlot f, int ks, int lim, Run&& run) {
+  const unsigned n = *(volatile unsigned*)f.hdr;
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const unsigned items = n * (unsigned)ks;
+  for (unsigned it = blockIdx.x * (SB / 32) + w; it < items; it += gridDim.x * (SB / 32)) {
+    const uint2 t = f.e[it / ks];
+    const int k0 = (int)t.y * ks + 1 + (int)(it % ks);
+    if (k0 < lim) run((int)t.x, k0, k0 + 1, lane, w);
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    if (atomicAdd(f.hdr + 1, 1u) == gridDim.x - 1) {
+      f.hdr[2] += n;  // cumulative (clover_debug_fix_count)
+      f.hdr[0] = 0u;
+      f.hdr[1] = 0u;
+    }
+  }
+}
+constexpr int FIX_BLOCKS = 148;  // fixup grid (one block per SM)
+
 // ================================================================ visc_dt
 // Column j = block*128 + tid + 1, rows [k0, k0+VKS).  Rolling: pressure of
 // the row below, density/energy of the row above, the 4 node velocities.
 constexpr int VKS = CLOVER_VKS;
 
-__global__ void LB_VISC
-ks_visc_dt(Chunk c, const double* __restrict__ d0, const double* __restrict__ e0,
-           const double* __restrict__ u0, const double* __restrict__ v0, double* __restrict__ q,
-           StepScalars* __restrict__ s, DtParams prm) {
-  const int j = blockIdx.x * SB + threadIdx.x + 1;
-  const int k0 = blockIdx.y * VKS + 1;
-  const int k1 = min(k0 + VKS, c.ny + 1);
+// Warp segment: columns j = 32*gw + lane + 1, rows [k0, k1).
+// Returns whether any lane flagged; dtw = the warp's dt minimum (lane 0).
+template <class D>
+__device__ __forceinline__ bool visc_body(const Chunk& c, const double* __restrict__ d0,
+                                          const double* __restrict__ e0,
+                                          const double* __restrict__ u0,
+                                          const double* __restrict__ v0, double* __restrict__ q,
+                                          const DtParams& prm, int gw, int k0, int k1, int lane,
+                                          double& dtw) {
+  const int j = gw * 32 + lane + 1;
   double dtl = G_BIG;
+  D dv;
   if (j <= c.nx) {
     const int P = c.pitch;
     const bool ncol = near_wall_col(c, j);
@@ -125,12 +175,7 @@ ks_visc_dt(Chunk c, const double* __restrict__ d0, const double* __restrict__ e0
       I.u00 = ua; I.u10 = ub; I.u01 = uc; I.u11 = ud;
       I.v00 = va; I.v10 = vb; I.v01 = vc; I.v11 = vd;
       double qv, cc;
-      DivFast f;
-      visc_cell(f, I, c, qv, cc);
-      if (f.bad) {
-        DivIEEE x;
-        visc_cell(x, I, c, qv, cc);
-      }
+      visc_cell(dv, I, c, qv, cc);
       acc.add(I, c, cc);
       store_at(c, q, K_CELL, j, k, i, ncol || near_wall_row(c, k), qv);
       pcm = pc; pc = I.pt; rho = rhon; ein = en;
@@ -139,15 +184,41 @@ ks_visc_dt(Chunk c, const double* __restrict__ d0, const double* __restrict__ e0
     dtl = acc.dt(c, prm);
   }
   for (int o = 16; o > 0; o >>= 1) dtl = fmin(dtl, __shfl_xor_sync(FULL, dtl, o));
-  __shared__ double wmin[SB / 32];
+  dtw = dtl;
+  return __any_sync(FULL, dv.bad);
+}
+
+__global__ void LB_VISC
+ks_visc_dt(Chunk c, const double* __restrict__ d0, const double* __restrict__ e0,
+           const double* __restrict__ u0, const double* __restrict__ v0, double* __restrict__ q,
+           StepScalars* __restrict__ s, DtParams prm, FixSlot fix) {
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  if (lane == 0) wmin[warp] = dtl;
+  const int gw = blockIdx.x * (SB / 32) + warp;
+  double dtw;
+  const int k0 = blockIdx.y * VKS + 1, k1 = min(k0 + VKS, c.ny + 1);
+  if (visc_body<DivFast>(c, d0, e0, u0, v0, q, prm, gw, k0, k1, lane, dtw)) {
+    fix_push(fix, lane, gw, blockIdx.y);
+    dtw = G_BIG;  // this warp's dt comes from the fixup
+  }
+  __shared__ double wmin[SB / 32];
+  if (lane == 0) wmin[warp] = dtw;
   __syncthreads();
   if (threadIdx.x == 0) {
     double m = wmin[0];
     for (int w = 1; w < SB / 32; ++w) m = fmin(m, wmin[w]);
     atomicMin(&s->dt_slot, (unsigned long long)__double_as_longlong(m));
   }
+}
+
+__global__ void __launch_bounds__(SB)
+kf_visc_dt(Chunk c, const double* __restrict__ d0, const double* __restrict__ e0,
+           const double* __restrict__ u0, const double* __restrict__ v0, double* __restrict__ q,
+           StepScalars* __restrict__ s, DtParams prm, FixSlot fix) {
+  fix_loop(fix, VKS, c.ny + 1, [&](int gw, int k0, int k1, int lane, int) {
+    double dtw;
+    visc_body<DivIEEE>(c, d0, e0, u0, v0, q, prm, gw, k0, k1, lane, dtw);
+    if (lane == 0) atomicMin(&s->dt_slot, (unsigned long long)__double_as_longlong(dtw));
+  });
 }
 
 // ================================================================ Lagrangian
@@ -162,11 +233,9 @@ ks_visc_dt(Chunk c, const double* __restrict__ d0, const double* __restrict__ e0
 constexpr int LW = 30;   // owned columns per warp
 constexpr int LKS = CLOVER_LKS;  // rows per segment
 
-#define CLOVER_TMA_LAGR 1
 #ifndef CLOVER_TMA_RELEASE_FENCE  // proxy fence before refilling a slot (A/B: no measurable cost)
 #define CLOVER_TMA_RELEASE_FENCE 1
 #endif
-#if CLOVER_TMA_LAGR
 // TMA-staged variant: rows of d0, e0, q (cells) and u0, v0 (nodes) stream
 // through a per-warp LSTG-stage shared-memory ring filled by cp.async.bulk,
 // so the DRAM latency of row k+LSTG-1 overlaps the compute of row k.
@@ -174,21 +243,22 @@ constexpr int LRW = 36;   // doubles per staged row segment (>= 34, 16-B multipl
 constexpr int LSTG = 4;   // ring stages
 enum { LF_R, LF_E, LF_Q, LF_U, LF_V, LNF };
 
-__global__ void LB_HEAVY
-ks_lagrangian(Chunk c, const double* __restrict__ d0, const double* __restrict__ e0,
-              const double* __restrict__ u0, const double* __restrict__ v0,
-              const double* __restrict__ q, double* __restrict__ d1, double* __restrict__ e1,
-              double* __restrict__ u1, double* __restrict__ v1, double* __restrict__ fx,
-              double* __restrict__ fy, const StepScalars* __restrict__ s) {
-  __shared__ __align__(128) double ring[SB / 32][LSTG][LNF][LRW];
-  __shared__ __align__(8) unsigned long long bars[SB / 32][LSTG];
-  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-  const int gw = blockIdx.x * (SB / 32) + w;
+template <class D>
+__device__ __forceinline__ bool lagr_body(const Chunk& c, const double* __restrict__ d0,
+                                          const double* __restrict__ e0,
+                                          const double* __restrict__ u0,
+                                          const double* __restrict__ v0,
+                                          const double* __restrict__ q, double* __restrict__ d1,
+                                          double* __restrict__ e1, double* __restrict__ u1,
+                                          double* __restrict__ v1, double* __restrict__ fx,
+                                          double* __restrict__ fy,
+                                          const StepScalars* __restrict__ s, int gw, int k0,
+                                          int k1, int lane, double (*ring)[LNF][LRW],
+                                          unsigned long long* bars) {
   const int J0 = 1 + LW * gw;
   const int j = J0 - 1 + lane;
-  if (J0 > c.nx) return;  // whole warp beyond the chunk (rings are per warp)
-  const int k0 = blockIdx.y * LKS + 1;
-  const int k1 = min(k0 + LKS, c.ny + 1);  // cell rows [k0, k1)
+  if (J0 > c.nx) return false;  // whole warp beyond the chunk (rings are per warp)
+  D dv;
   const double dt = s->dt, dx = c.dx, dy = c.dy;
   const int P = c.pitch;
   const bool colok = j <= c.nx + 1;
@@ -208,17 +278,17 @@ ks_lagrangian(Chunk c, const double* __restrict__ d0, const double* __restrict__
   const int r_first = k0 - 1, r_last = k1 + 1;  // staged rows
   auto issue = [&](int r) {
     const int rel = r - r_first, slot = rel % LSTG;
-    mbar_arrive_expect_tx(&bars[w][slot], bytes * LNF);
+    mbar_arrive_expect_tx(&bars[slot], bytes * LNF);
 #pragma unroll
     for (int f = 0; f < LNF; ++f)
-      tma_load_1d(&ring[w][slot][f][0], fields[f] + (size_t)r * P + (mstart - COL0), bytes, &bars[w][slot]);
+      tma_load_1d(&ring[slot][f][0], fields[f] + (size_t)r * P + (mstart - COL0), bytes, &bars[slot]);
   };
   auto wait_row = [&](int r) {
     const int rel = r - r_first;
-    mbar_wait(&bars[w][rel % LSTG], (unsigned)((rel / LSTG) & 1));
+    mbar_wait(&bars[rel % LSTG], (unsigned)((rel / LSTG) & 1));
   };
   if (lane == 0) {
-    for (int t = 0; t < LSTG; ++t) mbar_init(&bars[w][t], 1);
+    for (int t = 0; t < LSTG; ++t) mbar_init(&bars[t], 1);
     fence_mbar_init();
     fence_proxy_async();
     for (int r = r_first; r < r_first + LSTG && r <= r_last; ++r) issue(r);
@@ -232,8 +302,8 @@ ks_lagrangian(Chunk c, const double* __restrict__ d0, const double* __restrict__
   wait_row(r_first);
   for (int k = k0 - 1; k <= k1; ++k) {
     wait_row(k + 1);
-    const double* rowc = &ring[w][(k - r_first) % LSTG][0][0];
-    const double* rown = &ring[w][(k + 1 - r_first) % LSTG][0][0];
+    const double* rowc = &ring[(k - r_first) % LSTG][0][0];
+    const double* rown = &ring[(k + 1 - r_first) % LSTG][0][0];
     const double u0_c = rowc[LF_U * LRW + off], v0_c = rowc[LF_V * LRW + off];
     const double u0r_c = rowc[LF_U * LRW + off + 1], v0r_c = rowc[LF_V * LRW + off + 1];
     double r = 1.0, e = 0.0, qq = 0.0, ph = 0.0;
@@ -255,12 +325,7 @@ ks_lagrangian(Chunk c, const double* __restrict__ d0, const double* __restrict__
         ua = u0[ip]; ub = u0[ip + P]; uc = u0[ip + 1]; ud = u0[ip + P + 1];
         va = v0[ip]; vb = v0[ip + 1]; vc = v0[ip + P]; vd = v0[ip + P + 1];
       }
-      DivFast f;
-      ph = pdv_predict_pressure(f, pr_, pe_, pq_, ua, ub, uc, ud, va, vb, vc, vd, dx, dy, c.rvol, dt);
-      if (f.bad) {
-        DivIEEE x;
-        ph = pdv_predict_pressure(x, pr_, pe_, pq_, ua, ub, uc, ud, va, vb, vc, vd, dx, dy, c.rvol, dt);
-      }
+      ph = pdv_predict_pressure(dv, pr_, pe_, pq_, ua, ub, uc, ud, va, vb, vc, vd, dx, dy, c.rvol, dt);
     }
     if (xwall_warp) ph = __shfl_sync(FULL, ph, src);
     const double rl = __shfl_up_sync(FULL, r, 1);
@@ -272,12 +337,7 @@ ks_lagrangian(Chunk c, const double* __restrict__ d0, const double* __restrict__
       const double rr[4] = {rl_m, r_m, r, rl};
       const double pp[4] = {phl_m, ph_m, ph, phl};
       const double qv[4] = {ql_m, q_m, qq, ql};
-      DivFast f;
-      accelerate_node(f, rr, pp, qv, u0_c, v0_c, dx, dy, dt, u1_c, v1_c);
-      if (f.bad) {
-        DivIEEE x;
-        accelerate_node(x, rr, pp, qv, u0_c, v0_c, dx, dy, dt, u1_c, v1_c);
-      }
+      accelerate_node(dv, rr, pp, qv, u0_c, v0_c, dx, dy, dt, u1_c, v1_c);
     }
     const double u1r_c = __shfl_down_sync(FULL, u1_c, 1);
     const double v1r_c = __shfl_down_sync(FULL, v1_c, 1);
@@ -291,12 +351,7 @@ ks_lagrangian(Chunk c, const double* __restrict__ d0, const double* __restrict__
       const double bsum = v0_m + v0r_m + v1_m + v1r_m;
       const double tsum = v0_c + v0r_c + v1_c + v1r_c;
       double ev, dvv;
-      DivFast f;
-      pdv_correct(f, r_m, e_m, ph_m, q_m, lsum, rsum, bsum, tsum, dx, dy, c.rvol, dt, ev, dvv);
-      if (f.bad) {
-        DivIEEE x;
-        pdv_correct(x, r_m, e_m, ph_m, q_m, lsum, rsum, bsum, tsum, dx, dy, c.rvol, dt, ev, dvv);
-      }
+      pdv_correct(dv, r_m, e_m, ph_m, q_m, lsum, rsum, bsum, tsum, dx, dy, c.rvol, dt, ev, dvv);
       const int ic = idx(c, j, kc);
       const bool near = ncol || near_wall_row(c, kc);
       store_at(c, e1, K_CELL, j, kc, ic, near, ev);
@@ -333,8 +388,44 @@ ks_lagrangian(Chunk c, const double* __restrict__ d0, const double* __restrict__
     __syncwarp();
     if (lane == 0 && k + LSTG <= r_last) issue(k + LSTG);
   }
+  __syncwarp();
+  if (lane == 0)
+    for (int t = 0; t < LSTG; ++t) mbar_inval(&bars[t]);  // the ring may be reused (fixup)
+  __syncwarp();
+  return __any_sync(FULL, dv.bad);
 }
-#endif  // CLOVER_TMA_LAGR (the register-only variant was measured 3% slower; see git history)
+
+__global__ void LB_HEAVY
+ks_lagrangian(Chunk c, const double* __restrict__ d0, const double* __restrict__ e0,
+              const double* __restrict__ u0, const double* __restrict__ v0,
+              const double* __restrict__ q, double* __restrict__ d1, double* __restrict__ e1,
+              double* __restrict__ u1, double* __restrict__ v1, double* __restrict__ fx,
+              double* __restrict__ fy, const StepScalars* __restrict__ s, FixSlot fix) {
+  __shared__ __align__(128) double ring[SB / 32][LSTG][LNF][LRW];
+  __shared__ __align__(8) unsigned long long bars[SB / 32][LSTG];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const int gw = blockIdx.x * (SB / 32) + w;
+  const int k0 = blockIdx.y * LKS + 1, k1 = min(k0 + LKS, c.ny + 1);
+  if (lagr_body<DivFast>(c, d0, e0, u0, v0, q, d1, e1, u1, v1, fx, fy, s, gw, k0, k1, lane,
+                         ring[w], bars[w])) {
+    fix_push(fix, lane, gw, blockIdx.y);
+  }
+}
+
+__global__ void __launch_bounds__(SB)
+kf_lagrangian(Chunk c, const double* __restrict__ d0, const double* __restrict__ e0,
+              const double* __restrict__ u0, const double* __restrict__ v0,
+              const double* __restrict__ q, double* __restrict__ d1, double* __restrict__ e1,
+              double* __restrict__ u1, double* __restrict__ v1, double* __restrict__ fx,
+              double* __restrict__ fy, const StepScalars* __restrict__ s, FixSlot fix) {
+  __shared__ __align__(128) double ring[SB / 32][LSTG][LNF][LRW];
+  __shared__ __align__(8) unsigned long long bars[SB / 32][LSTG];
+  fix_loop(fix, LKS, c.ny + 1, [&](int gw, int k0, int k1, int lane, int w) {
+    lagr_body<DivIEEE>(c, d0, e0, u0, v0, q, d1, e1, u1, v1, fx, fy, s, gw, k0, k1, lane, ring[w],
+                       bars[w]);
+  });
+}
+// (a register-only Lagrangian variant was measured 3% slower; see git history)
 
 // ================================================================ advec_cell x
 // Warp strip: lane l <-> face/cell column j = J0 + l, J0 = 1 + 31*(warp);
@@ -343,19 +434,16 @@ ks_lagrangian(Chunk c, const double* __restrict__ d0, const double* __restrict__
 constexpr int CW_X = 31;
 constexpr int CKS = CLOVER_CKS;
 
-template <int SWEEP>
-__global__ void LB_ADV
-ks_advec_cell_x(Chunk c, const double* __restrict__ rho, const double* __restrict__ en,
+template <int SWEEP, class D>
+__device__ __forceinline__ bool advec_cell_x_body(const Chunk& c, const double* __restrict__ rho, const double* __restrict__ en,
                 const double* __restrict__ fx, const double* __restrict__ fy,
                 double* __restrict__ rho_out, double* __restrict__ en_out,
-                double* __restrict__ mfx) {
-  const int lane = threadIdx.x & 31;
-  const int gw = blockIdx.x * (SB / 32) + (threadIdx.x >> 5);
+                double* __restrict__ mfx,
+    int gw, int k0, int k1, int lane) {
+  D dv;
   const int J0 = 1 + CW_X * gw;
-  if (J0 > c.nx) return;
+  if (J0 > c.nx) return false;
   const int j = J0 + lane;
-  const int k0 = blockIdx.y * CKS + 1;
-  const int k1 = min(k0 + CKS, c.ny + 1);
   const double vol = c.dx * c.dy;
   const int P = c.pitch;
   const bool faceok = j <= c.nx + 1;
@@ -387,23 +475,13 @@ ks_advec_cell_x(Chunk c, const double* __restrict__ rho, const double* __restric
         eu = en[i + up]; ed = ee; ew = en[i - 1];
         pvd = pv;
       }
-      DivFast f;
-      cell_face_flux(f, F, pvd, ru, rd, rw, eu, ed, ew, m, ef);
-      if (f.bad) {
-        DivIEEE x;
-        cell_face_flux(x, F, pvd, ru, rd, rw, eu, ed, ew, m, ef);
-      }
+      cell_face_flux(dv, F, pvd, ru, rd, rw, eu, ed, ew, m, ef);
     }
     const double mh = __shfl_down_sync(FULL, m, 1);
     const double efh = __shfl_down_sync(FULL, ef, 1);
     if (lane < CW_X && j <= c.nx) {
       double ro, eo;
-      DivFast f;
-      cell_update(f, rr, ee, pv, m, mh, ef, efh, flo, fhi, ro, eo);
-      if (f.bad) {
-        DivIEEE x;
-        cell_update(x, rr, ee, pv, m, mh, ef, efh, flo, fhi, ro, eo);
-      }
+      cell_update(dv, rr, ee, pv, m, mh, ef, efh, flo, fhi, ro, eo);
       const bool near = ncol || near_wall_row(c, k);
       store_at(c, rho_out, K_CELL, j, k, i, near, ro);
       store_at(c, en_out, K_CELL, j, k, i, near, eo);
@@ -411,6 +489,32 @@ ks_advec_cell_x(Chunk c, const double* __restrict__ rho, const double* __restric
       if (j == c.nx) store_field(c, mfx, K_XFACE, j + 1, k, mh);
     }
   }
+  return __any_sync(FULL, dv.bad);
+}
+
+template <int SWEEP>
+__global__ void LB_ADV
+ks_advec_cell_x(Chunk c, const double* __restrict__ rho, const double* __restrict__ en,
+                const double* __restrict__ fx, const double* __restrict__ fy,
+                double* __restrict__ rho_out, double* __restrict__ en_out,
+                double* __restrict__ mfx, FixSlot fix) {
+  const int lane = threadIdx.x & 31;
+  const int gw = blockIdx.x * (SB / 32) + (threadIdx.x >> 5);
+  const int k0 = blockIdx.y * CKS + 1, k1 = min(k0 + CKS, c.ny + 1);
+  if (advec_cell_x_body<SWEEP, DivFast>(c, rho, en, fx, fy, rho_out, en_out, mfx, gw, k0, k1, lane)) {
+    fix_push(fix, lane, gw, blockIdx.y);
+  }
+}
+
+template <int SWEEP>
+__global__ void __launch_bounds__(SB)
+kf_advec_cell_x(Chunk c, const double* __restrict__ rho, const double* __restrict__ en,
+                const double* __restrict__ fx, const double* __restrict__ fy,
+                double* __restrict__ rho_out, double* __restrict__ en_out,
+                double* __restrict__ mfx, FixSlot fix) {
+  fix_loop(fix, CKS, c.ny + 1, [&](int gw, int k0, int k1, int lane, int) {
+    advec_cell_x_body<SWEEP, DivIEEE>(c, rho, en, fx, fy, rho_out, en_out, mfx, gw, k0, k1, lane);
+  });
 }
 
 // ================================================================ advec_cell y
@@ -420,98 +524,98 @@ ks_advec_cell_x(Chunk c, const double* __restrict__ rho, const double* __restric
 // pre-sweep volume of rows k, k+1.
 constexpr int CKS_Y = CLOVER_CKS_Y;
 
+template <int SWEEP, class D>
+__device__ __forceinline__ bool advec_cell_y_body(const Chunk& c, const double* __restrict__ rho, const double* __restrict__ en,
+                const double* __restrict__ fx, const double* __restrict__ fy,
+                double* __restrict__ rho_out, double* __restrict__ en_out,
+                double* __restrict__ mfy,
+    int gw, int k0, int k1, int lane) {
+  D dv;
+  const int j = gw * 32 + lane + 1;
+  if (j <= c.nx) {
+    const double vol = c.dx * c.dy;
+    const int P = c.pitch;
+    auto pre_vol = [&](int i) -> double {
+      if (SWEEP == 1) return vol + (fy[i + P] - fy[i] + fx[i + 1] - fx[i]);
+      return vol + fy[i + P] - fy[i];
+    };
+    const bool ncol = near_wall_col(c, j);
+    int i = idx(c, j, k0);
+    // rows k0-2 .. k0+1
+    double R0 = rho[i - 2 * P], R1 = rho[i - P], R2 = rho[i], R3 = rho[i + P];
+    double E0 = en[i - 2 * P], E1 = en[i - P], E2 = en[i], E3 = en[i + P];
+    double pvm = pre_vol(i - P), pv0 = pre_vol(i);
+    // face k0
+    double m0, ef0;
+    {
+      const double F = fy[i];
+      double ru, rd, rw, eu, ed, ew, pvd;
+      if (F > 0.0) {
+        ru = R0; rd = R1; rw = R2; eu = E0; ed = E1; ew = E2; pvd = pvm;
+      } else {
+        ru = R3; rd = R2; rw = R1; eu = E3; ed = E2; ew = E1; pvd = pv0;
+      }
+      cell_face_flux(dv, F, pvd, ru, rd, rw, eu, ed, ew, m0, ef0);
+    }
+    STREAM_LOOP
+    for (int k = k0; k < k1; ++k, i += P) {
+      // registers: R1..R3 = rows k-1..k+1; load row k+2
+      const double R4 = rho[i + 2 * P], E4 = en[i + 2 * P];
+      const double pv1 = pre_vol(i + P);
+      // face k+1: up = k (F>0: k-1+1), don = k, dw = k+1 ; else up = k+2, don = k+1, dw = k
+      double m1, ef1;
+      {
+        const double F = fy[i + P];
+        double ru, rd, rw, eu, ed, ew, pvd;
+        if (F > 0.0) {
+          ru = R1; rd = R2; rw = R3; eu = E1; ed = E2; ew = E3; pvd = pv0;
+        } else {
+          ru = R4; rd = R3; rw = R2; eu = E4; ed = E3; ew = E2; pvd = pv1;
+        }
+        cell_face_flux(dv, F, pvd, ru, rd, rw, eu, ed, ew, m1, ef1);
+      }
+      double ro, eo;
+      {
+        const double flo = fy[i], fhi = fy[i + P];
+        cell_update(dv, R2, E2, pv0, m0, m1, ef0, ef1, flo, fhi, ro, eo);
+      }
+      const bool near = ncol || near_wall_row(c, k);
+      store_at(c, rho_out, K_CELL, j, k, i, near, ro);
+      store_at(c, en_out, K_CELL, j, k, i, near, eo);
+      store_at(c, mfy, K_YFACE, j, k, i, near, m0);
+      if (k == c.ny) store_field(c, mfy, K_YFACE, j, k + 1, m1);
+      R0 = R1; R1 = R2; R2 = R3; R3 = R4;
+      E0 = E1; E1 = E2; E2 = E3; E3 = E4;
+      pvm = pv0; pv0 = pv1;
+      m0 = m1; ef0 = ef1;
+    }
+  }
+  return __any_sync(FULL, dv.bad);
+}
+
 template <int SWEEP>
 __global__ void LB_ADV
 ks_advec_cell_y(Chunk c, const double* __restrict__ rho, const double* __restrict__ en,
                 const double* __restrict__ fx, const double* __restrict__ fy,
                 double* __restrict__ rho_out, double* __restrict__ en_out,
-                double* __restrict__ mfy) {
-  const int j = blockIdx.x * SB + threadIdx.x + 1;
-  if (j > c.nx) return;
-  const int k0 = blockIdx.y * CKS_Y + 1;
-  const int k1 = min(k0 + CKS_Y, c.ny + 1);
-  const double vol = c.dx * c.dy;
-  const int P = c.pitch;
-  auto pre_vol = [&](int i) -> double {
-    if (SWEEP == 1) return vol + (fy[i + P] - fy[i] + fx[i + 1] - fx[i]);
-    return vol + fy[i + P] - fy[i];
-  };
-  const bool ncol = near_wall_col(c, j);
-  int i = idx(c, j, k0);
-  // rows k0-2 .. k0+1
-  double R0 = rho[i - 2 * P], R1 = rho[i - P], R2 = rho[i], R3 = rho[i + P];
-  double E0 = en[i - 2 * P], E1 = en[i - P], E2 = en[i], E3 = en[i + P];
-  double pvm = pre_vol(i - P), pv0 = pre_vol(i);
-  // face k0
-  double m0, ef0;
-  {
-    const double F = fy[i];
-    double ru, rd, rw, eu, ed, ew, pvd;
-    if (F > 0.0) {
-      ru = R0; rd = R1; rw = R2; eu = E0; ed = E1; ew = E2; pvd = pvm;
-    } else {
-      ru = R3; rd = R2; rw = R1; eu = E3; ed = E2; ew = E1; pvd = pv0;
-    }
-    DivFast f;
-    cell_face_flux(f, F, pvd, ru, rd, rw, eu, ed, ew, m0, ef0);
-    if (f.bad) {
-      DivIEEE x;
-      cell_face_flux(x, F, pvd, ru, rd, rw, eu, ed, ew, m0, ef0);
-    }
+                double* __restrict__ mfy, FixSlot fix) {
+  const int lane = threadIdx.x & 31;
+  const int gw = blockIdx.x * (SB / 32) + (threadIdx.x >> 5);
+  const int k0 = blockIdx.y * CKS_Y + 1, k1 = min(k0 + CKS_Y, c.ny + 1);
+  if (advec_cell_y_body<SWEEP, DivFast>(c, rho, en, fx, fy, rho_out, en_out, mfy, gw, k0, k1, lane)) {
+    fix_push(fix, lane, gw, blockIdx.y);
   }
-  STREAM_LOOP
-  for (int k = k0; k < k1; ++k, i += P) {
-    // registers: R1..R3 = rows k-1..k+1; load row k+2
-    const double R4 = rho[i + 2 * P], E4 = en[i + 2 * P];
-    const double pv1 = pre_vol(i + P);
-    // face k+1: up = k (F>0: k-1+1), don = k, dw = k+1 ; else up = k+2, don = k+1, dw = k
-    double m1, ef1;
-    {
-      const double F = fy[i + P];
-      double ru, rd, rw, eu, ed, ew, pvd;
-      if (F > 0.0) {
-        ru = R1; rd = R2; rw = R3; eu = E1; ed = E2; ew = E3; pvd = pv0;
-      } else {
-        ru = R4; rd = R3; rw = R2; eu = E4; ed = E3; ew = E2; pvd = pv1;
-      }
-#ifdef CLOVER_DIAG_TRIVIAL
-      m1 = F * rd + pvd * (ru + rw); ef1 = m1 * (ed + eu + ew);
-    }
-    double ro, eo;
-    {
-      const double flo = fy[i], fhi = fy[i + P];
-      // keep every load live, keep the state physical
-      ro = R2 + 0.0 * (pv0 + m0 - m1 + flo - fhi); eo = E2 + 0.0 * (ef0 - ef1);
-    }
-#else
-      DivFast f;
-      cell_face_flux(f, F, pvd, ru, rd, rw, eu, ed, ew, m1, ef1);
-      if (f.bad) {
-        DivIEEE x;
-        cell_face_flux(x, F, pvd, ru, rd, rw, eu, ed, ew, m1, ef1);
-      }
-    }
-    double ro, eo;
-    {
-      const double flo = fy[i], fhi = fy[i + P];
-      DivFast f;
-      cell_update(f, R2, E2, pv0, m0, m1, ef0, ef1, flo, fhi, ro, eo);
-      if (f.bad) {
-        DivIEEE x;
-        cell_update(x, R2, E2, pv0, m0, m1, ef0, ef1, flo, fhi, ro, eo);
-      }
-    }
-#endif
-    const bool near = ncol || near_wall_row(c, k);
-    store_at(c, rho_out, K_CELL, j, k, i, near, ro);
-    store_at(c, en_out, K_CELL, j, k, i, near, eo);
-    store_at(c, mfy, K_YFACE, j, k, i, near, m0);
-    if (k == c.ny) store_field(c, mfy, K_YFACE, j, k + 1, m1);
-    R0 = R1; R1 = R2; R2 = R3; R3 = R4;
-    E0 = E1; E1 = E2; E2 = E3; E3 = E4;
-    pvm = pv0; pv0 = pv1;
-    m0 = m1; ef0 = ef1;
-  }
+}
+
+template <int SWEEP>
+__global__ void __launch_bounds__(SB)
+kf_advec_cell_y(Chunk c, const double* __restrict__ rho, const double* __restrict__ en,
+                const double* __restrict__ fx, const double* __restrict__ fy,
+                double* __restrict__ rho_out, double* __restrict__ en_out,
+                double* __restrict__ mfy, FixSlot fix) {
+  fix_loop(fix, CKS_Y, c.ny + 1, [&](int gw, int k0, int k1, int lane, int) {
+    advec_cell_y_body<SWEEP, DivIEEE>(c, rho, en, fx, fy, rho_out, en_out, mfy, gw, k0, k1, lane);
+  });
 }
 
 // ================================================================ advec_mom x
@@ -522,19 +626,16 @@ ks_advec_cell_y(Chunk c, const double* __restrict__ rho, const double* __restric
 constexpr int MW_X = 29;
 constexpr int MKS = CLOVER_MKS;
 
-template <int SWEEP>
-__global__ void LB_ADV
-ks_advec_mom_x(Chunk c, const double* __restrict__ rho, const double* __restrict__ mfx,
+template <int SWEEP, class D>
+__device__ __forceinline__ bool advec_mom_x_body(const Chunk& c, const double* __restrict__ rho, const double* __restrict__ mfx,
                const double* __restrict__ fy, const double* __restrict__ uin,
                const double* __restrict__ vin, double* __restrict__ uout,
-               double* __restrict__ vout) {
-  const int lane = threadIdx.x & 31;
-  const int gw = blockIdx.x * (SB / 32) + (threadIdx.x >> 5);
+               double* __restrict__ vout,
+    int gw, int k0, int k1, int lane) {
+  D dv;
   const int J0 = 1 + MW_X * gw;
-  if (J0 > c.nx + 1) return;
+  if (J0 > c.nx + 1) return false;
   const int j = J0 - 2 + lane;
-  const int k0 = blockIdx.y * MKS + 1;
-  const int k1 = min(k0 + MKS, c.ny + 2);  // node rows [k0, k1)
   const double vol = c.dx * c.dy;
   const int P = c.pitch;
   const bool nfok = j <= c.nx + 2;   // node flux / node mass columns
@@ -573,30 +674,46 @@ ks_advec_mom_x(Chunk c, const double* __restrict__ rho, const double* __restrict
       }
       const double uu[3] = {uin[i + up], uin[i + don], uin[i + dw]};
       const double vv[3] = {vin[i + up], vin[i + don], vin[i + dw]};
-      DivFast f;
-      mom_flux2(f, nf, nmp, uu, vv, c.dx, c.rdx, mu, mv);
-      if (f.bad) {
-        DivIEEE x;
-        mom_flux2(x, nf, nmp, uu, vv, c.dx, c.rdx, mu, mv);
-      }
+      mom_flux2(dv, nf, nmp, uu, vv, c.dx, c.rdx, mu, mv);
     }
     const double mul = __shfl_up_sync(FULL, mu, 1);
     const double mvl = __shfl_up_sync(FULL, mv, 1);
     if (lane >= 2 && lane <= MW_X + 1 && j <= c.nx + 1) {
       const double u = uin[i], v = vin[i];
       double un, vn;
-      DivFast f;
-      mom_update(f, u, v, pre, post, mul, mu, mvl, mv, un, vn);
-      if (f.bad) {
-        DivIEEE x;
-        mom_update(x, u, v, pre, post, mul, mu, mvl, mv, un, vn);
-      }
+      mom_update(dv, u, v, pre, post, mul, mu, mvl, mv, un, vn);
       const bool near = ncol || near_wall_row(c, k);
       store_at(c, uout, K_XVEL, j, k, i, near, un);
       store_at(c, vout, K_YVEL, j, k, i, near, vn);
     }
     mA_m = mA; mB_m = mB; mp_m = mp; mpl_m = mpl;
   }
+  return __any_sync(FULL, dv.bad);
+}
+
+template <int SWEEP>
+__global__ void LB_ADV
+ks_advec_mom_x(Chunk c, const double* __restrict__ rho, const double* __restrict__ mfx,
+               const double* __restrict__ fy, const double* __restrict__ uin,
+               const double* __restrict__ vin, double* __restrict__ uout,
+               double* __restrict__ vout, FixSlot fix) {
+  const int lane = threadIdx.x & 31;
+  const int gw = blockIdx.x * (SB / 32) + (threadIdx.x >> 5);
+  const int k0 = blockIdx.y * MKS + 1, k1 = min(k0 + MKS, c.ny + 2);
+  if (advec_mom_x_body<SWEEP, DivFast>(c, rho, mfx, fy, uin, vin, uout, vout, gw, k0, k1, lane)) {
+    fix_push(fix, lane, gw, blockIdx.y);
+  }
+}
+
+template <int SWEEP>
+__global__ void __launch_bounds__(SB)
+kf_advec_mom_x(Chunk c, const double* __restrict__ rho, const double* __restrict__ mfx,
+               const double* __restrict__ fy, const double* __restrict__ uin,
+               const double* __restrict__ vin, double* __restrict__ uout,
+               double* __restrict__ vout, FixSlot fix) {
+  fix_loop(fix, MKS, c.ny + 2, [&](int gw, int k0, int k1, int lane, int) {
+    advec_mom_x_body<SWEEP, DivIEEE>(c, rho, mfx, fy, uin, vin, uout, vout, gw, k0, k1, lane);
+  });
 }
 
 // ================================================================ advec_mom y
@@ -605,97 +722,108 @@ ks_advec_mom_x(Chunk c, const double* __restrict__ rho, const double* __restrict
 // flux of row k and updates node k.
 constexpr int MKS_Y = CLOVER_MKS_Y;
 
+template <int SWEEP, class D>
+__device__ __forceinline__ bool advec_mom_y_body(const Chunk& c, const double* __restrict__ rho, const double* __restrict__ mfy,
+               const double* __restrict__ fx, const double* __restrict__ uin,
+               const double* __restrict__ vin, double* __restrict__ uout,
+               double* __restrict__ vout,
+    int gw, int k0, int k1, int lane) {
+  D dv;
+  const int j = gw * 32 + lane + 1;
+  if (j <= c.nx + 1) {
+    const double vol = c.dx * c.dy;
+    const int P = c.pitch;
+    auto mass_post = [&](int i) -> double {  // rho * post_vol of the cell at offset i
+      const double pv = (SWEEP == 1) ? vol + fx[i + 1] - fx[i] : vol;
+      return rho[i] * pv;
+    };
+    const bool ncol = near_wall_col(c, j);
+    // node flux of row r uses My(j-1,r), My(j,r), My(j-1,r+1), My(j,r+1)
+    auto node_flux = [&](int i) -> double {
+      return 0.25 * (mfy[i - 1] + mfy[i] + mfy[i - 1 + P] + mfy[i + P]);
+    };
+    // node mass post of row r uses cells (j,r-1), (j,r), (j-1,r-1), (j-1,r)
+    auto node_post = [&](double mj_m, double mj, double ml_m, double ml) -> double {
+      return 0.25 * (mj_m + mj + ml_m + ml);
+    };
+    int i = idx(c, j, k0);
+    // prologue: rows k0-2 .. k0
+    double mpj_a = mass_post(i - 2 * P), mpl_a = mass_post(i - 2 * P - 1);  // row k0-2
+    double mpj_b = mass_post(i - P), mpl_b = mass_post(i - P - 1);          // row k0-1
+    double mpj_c = mass_post(i), mpl_c = mass_post(i - 1);                  // row k0
+    const double nf_m2 = node_flux(i - 2 * P);
+    double nf_m = node_flux(i - P);                  // nf(k0-1)
+    double nf_0 = node_flux(i);                      // nf(k0)
+    const double post_m = node_post(mpj_a, mpj_b, mpl_a, mpl_b);   // nmpost(k0-1)
+    double post_0 = node_post(mpj_b, mpj_c, mpl_b, mpl_c);         // nmpost(k0)
+    const double pre_m = post_m - nf_m2 + nf_m;                    // nmp(k0-1)
+    double pre_0 = post_0 - nf_m + nf_0;                           // nmp(k0)
+    double U0 = uin[i - 2 * P], U1 = uin[i - P], U2 = uin[i], U3 = uin[i + P];  // rows k0-2..k0+1
+    double V0 = vin[i - 2 * P], V1 = vin[i - P], V2 = vin[i], V3 = vin[i + P];
+    double mu_m, mv_m;  // mom flux of row k0-1
+    {
+      const double nf = nf_m;
+      const double nmp = (nf < 0.0) ? pre_0 : pre_m;
+      const double uu[3] = {nf < 0.0 ? U3 : U0, nf < 0.0 ? U2 : U1, nf < 0.0 ? U1 : U2};
+      const double vv[3] = {nf < 0.0 ? V3 : V0, nf < 0.0 ? V2 : V1, nf < 0.0 ? V1 : V2};
+      mom_flux2(dv, nf, nmp, uu, vv, c.dy, c.rdy, mu_m, mv_m);
+    }
+    STREAM_LOOP
+    for (int k = k0; k < k1; ++k, i += P) {
+      // registers: U1..U3 = rows k-1..k+1 ; load row k+2
+      const double U4 = uin[i + 2 * P], V4 = vin[i + 2 * P];
+      const double mpj_d = mass_post(i + P), mpl_d = mass_post(i + P - 1);  // row k+1
+      const double nf_1 = node_flux(i + P);                                 // nf(k+1)
+      const double post_1 = node_post(mpj_c, mpj_d, mpl_c, mpl_d);          // nmpost(k+1)
+      const double pre_1 = post_1 - nf_0 + nf_1;                            // nmp(k+1)
+      double mu, mv;
+      {
+        const double nf = nf_0;
+        const double nmp = (nf < 0.0) ? pre_1 : pre_0;
+        const double uu[3] = {nf < 0.0 ? U4 : U1, nf < 0.0 ? U3 : U2, nf < 0.0 ? U2 : U3};
+        const double vv[3] = {nf < 0.0 ? V4 : V1, nf < 0.0 ? V3 : V2, nf < 0.0 ? V2 : V3};
+        mom_flux2(dv, nf, nmp, uu, vv, c.dy, c.rdy, mu, mv);
+      }
+      double un, vn;
+      {
+        mom_update(dv, U2, V2, pre_0, post_0, mu_m, mu, mv_m, mv, un, vn);
+      }
+      const bool near = ncol || near_wall_row(c, k);
+      store_at(c, uout, K_XVEL, j, k, i, near, un);
+      store_at(c, vout, K_YVEL, j, k, i, near, vn);
+      U1 = U2; U2 = U3; U3 = U4;
+      V1 = V2; V2 = V3; V3 = V4;
+      mpj_c = mpj_d; mpl_c = mpl_d;
+      nf_0 = nf_1; post_0 = post_1; pre_0 = pre_1;
+      mu_m = mu; mv_m = mv;
+    }
+  }
+  return __any_sync(FULL, dv.bad);
+}
+
 template <int SWEEP>
 __global__ void LB_MOMY
 ks_advec_mom_y(Chunk c, const double* __restrict__ rho, const double* __restrict__ mfy,
                const double* __restrict__ fx, const double* __restrict__ uin,
                const double* __restrict__ vin, double* __restrict__ uout,
-               double* __restrict__ vout) {
-  const int j = blockIdx.x * SB + threadIdx.x + 1;
-  if (j > c.nx + 1) return;
-  const int k0 = blockIdx.y * MKS_Y + 1;
-  const int k1 = min(k0 + MKS_Y, c.ny + 2);
-  const double vol = c.dx * c.dy;
-  const int P = c.pitch;
-  auto mass_post = [&](int i) -> double {  // rho * post_vol of the cell at offset i
-    const double pv = (SWEEP == 1) ? vol + fx[i + 1] - fx[i] : vol;
-    return rho[i] * pv;
-  };
-  const bool ncol = near_wall_col(c, j);
-  // node flux of row r uses My(j-1,r), My(j,r), My(j-1,r+1), My(j,r+1)
-  auto node_flux = [&](int i) -> double {
-    return 0.25 * (mfy[i - 1] + mfy[i] + mfy[i - 1 + P] + mfy[i + P]);
-  };
-  // node mass post of row r uses cells (j,r-1), (j,r), (j-1,r-1), (j-1,r)
-  auto node_post = [&](double mj_m, double mj, double ml_m, double ml) -> double {
-    return 0.25 * (mj_m + mj + ml_m + ml);
-  };
-  int i = idx(c, j, k0);
-  // prologue: rows k0-2 .. k0
-  double mpj_a = mass_post(i - 2 * P), mpl_a = mass_post(i - 2 * P - 1);  // row k0-2
-  double mpj_b = mass_post(i - P), mpl_b = mass_post(i - P - 1);          // row k0-1
-  double mpj_c = mass_post(i), mpl_c = mass_post(i - 1);                  // row k0
-  const double nf_m2 = node_flux(i - 2 * P);
-  double nf_m = node_flux(i - P);                  // nf(k0-1)
-  double nf_0 = node_flux(i);                      // nf(k0)
-  const double post_m = node_post(mpj_a, mpj_b, mpl_a, mpl_b);   // nmpost(k0-1)
-  double post_0 = node_post(mpj_b, mpj_c, mpl_b, mpl_c);         // nmpost(k0)
-  const double pre_m = post_m - nf_m2 + nf_m;                    // nmp(k0-1)
-  double pre_0 = post_0 - nf_m + nf_0;                           // nmp(k0)
-  double U0 = uin[i - 2 * P], U1 = uin[i - P], U2 = uin[i], U3 = uin[i + P];  // rows k0-2..k0+1
-  double V0 = vin[i - 2 * P], V1 = vin[i - P], V2 = vin[i], V3 = vin[i + P];
-  double mu_m, mv_m;  // mom flux of row k0-1
-  {
-    const double nf = nf_m;
-    const double nmp = (nf < 0.0) ? pre_0 : pre_m;
-    const double uu[3] = {nf < 0.0 ? U3 : U0, nf < 0.0 ? U2 : U1, nf < 0.0 ? U1 : U2};
-    const double vv[3] = {nf < 0.0 ? V3 : V0, nf < 0.0 ? V2 : V1, nf < 0.0 ? V1 : V2};
-    DivFast f;
-    mom_flux2(f, nf, nmp, uu, vv, c.dy, c.rdy, mu_m, mv_m);
-    if (f.bad) {
-      DivIEEE x;
-      mom_flux2(x, nf, nmp, uu, vv, c.dy, c.rdy, mu_m, mv_m);
-    }
+               double* __restrict__ vout, FixSlot fix) {
+  const int lane = threadIdx.x & 31;
+  const int gw = blockIdx.x * (SB / 32) + (threadIdx.x >> 5);
+  const int k0 = blockIdx.y * MKS_Y + 1, k1 = min(k0 + MKS_Y, c.ny + 2);
+  if (advec_mom_y_body<SWEEP, DivFast>(c, rho, mfy, fx, uin, vin, uout, vout, gw, k0, k1, lane)) {
+    fix_push(fix, lane, gw, blockIdx.y);
   }
-  STREAM_LOOP
-  for (int k = k0; k < k1; ++k, i += P) {
-    // registers: U1..U3 = rows k-1..k+1 ; load row k+2
-    const double U4 = uin[i + 2 * P], V4 = vin[i + 2 * P];
-    const double mpj_d = mass_post(i + P), mpl_d = mass_post(i + P - 1);  // row k+1
-    const double nf_1 = node_flux(i + P);                                 // nf(k+1)
-    const double post_1 = node_post(mpj_c, mpj_d, mpl_c, mpl_d);          // nmpost(k+1)
-    const double pre_1 = post_1 - nf_0 + nf_1;                            // nmp(k+1)
-    double mu, mv;
-    {
-      const double nf = nf_0;
-      const double nmp = (nf < 0.0) ? pre_1 : pre_0;
-      const double uu[3] = {nf < 0.0 ? U4 : U1, nf < 0.0 ? U3 : U2, nf < 0.0 ? U2 : U3};
-      const double vv[3] = {nf < 0.0 ? V4 : V1, nf < 0.0 ? V3 : V2, nf < 0.0 ? V2 : V3};
-      DivFast f;
-      mom_flux2(f, nf, nmp, uu, vv, c.dy, c.rdy, mu, mv);
-      if (f.bad) {
-        DivIEEE x;
-        mom_flux2(x, nf, nmp, uu, vv, c.dy, c.rdy, mu, mv);
-      }
-    }
-    double un, vn;
-    {
-      DivFast f;
-      mom_update(f, U2, V2, pre_0, post_0, mu_m, mu, mv_m, mv, un, vn);
-      if (f.bad) {
-        DivIEEE x;
-        mom_update(x, U2, V2, pre_0, post_0, mu_m, mu, mv_m, mv, un, vn);
-      }
-    }
-    const bool near = ncol || near_wall_row(c, k);
-    store_at(c, uout, K_XVEL, j, k, i, near, un);
-    store_at(c, vout, K_YVEL, j, k, i, near, vn);
-    U1 = U2; U2 = U3; U3 = U4;
-    V1 = V2; V2 = V3; V3 = V4;
-    mpj_c = mpj_d; mpl_c = mpl_d;
-    nf_0 = nf_1; post_0 = post_1; pre_0 = pre_1;
-    mu_m = mu; mv_m = mv;
-  }
+}
+
+template <int SWEEP>
+__global__ void __launch_bounds__(SB)
+kf_advec_mom_y(Chunk c, const double* __restrict__ rho, const double* __restrict__ mfy,
+               const double* __restrict__ fx, const double* __restrict__ uin,
+               const double* __restrict__ vin, double* __restrict__ uout,
+               double* __restrict__ vout, FixSlot fix) {
+  fix_loop(fix, MKS_Y, c.ny + 2, [&](int gw, int k0, int k1, int lane, int) {
+    advec_mom_y_body<SWEEP, DivIEEE>(c, rho, mfy, fx, uin, vin, uout, vout, gw, k0, k1, lane);
+  });
 }
 
 }  // namespace clover

@@ -160,6 +160,29 @@ def test_random_state_bitwise(torch_cuda, smooth):
     assert np.array_equal(g.read("viscosity"), o.read("viscosity"))
 
 
+@pytest.mark.parametrize("scale", [1e-300, 1e-306])
+def test_tiny_numerators_take_the_ieee_fixup_bitwise(torch_cuda, scale):
+    """Velocities of 1e-300 (and subnormal-adjacent 1e-306) in the left half:
+    numerators below 2^-900 make DivFast flag, so those warp segments are
+    recomputed by the IEEE fixup launches.  Bitwise vs the
+    oracle, and the fixup path must actually have run."""
+    nx, ny = 96, 64
+    deck = bm_deck(nx, ny)
+    deck["max_timestep"] = 1.0
+    fields = random_state_fields(9, nx, ny)
+    for f in ("xvel0", "yvel0"):
+        fields[f][:, : (nx + 1) // 2] *= scale
+    g, o = make_gpu(deck), Oracle(deck)
+    g.load_state(fields)
+    o.load_state(fields)
+    g.step(3)
+    dts = o.step(3)
+    assert np.array_equal(g.dt_history(1, 3), dts)
+    assert_fields_equal(g, o, ctx=f"tiny {scale}")
+    assert np.array_equal(g.read("viscosity"), o.read("viscosity"))
+    assert g.debug_fix_count() > 0
+
+
 def test_invariant_decks(torch_cuda):
     for deck in (quiescent_deck(64), contact_deck(64), symmetric_deck(64)):
         g, o = make_gpu(deck), Oracle(deck)
@@ -264,6 +287,7 @@ def test_c2_960_87_steps(torch_cuda):
     assert_summary_close(gs, os_)
     assert abs(100.0 * gs["ke"] / 1.19316898756307 - 100.0) < 0.001
     assert_fields_equal(g, o, ctx="C2")
+    print("C2 IEEE fixup warp segments:", g.debug_fix_count())
 
 
 @pytest.mark.parametrize("n", [3840])
