@@ -14,6 +14,7 @@
 #include <cstdio>
 #include <cstring>
 #include <string>
+#include <utility>
 #include <vector>
 
 #include "clover.h"
@@ -424,6 +425,29 @@ void prof_mark(clover_ctx* ctx, int id) {
 }
 
 
+#ifndef CLOVER_PDL
+#define CLOVER_PDL 1
+#endif
+// Launch a step kernel with programmatic dependent launch (the kernels call
+// pdl_trigger/pdl_wait, clover_common.cuh), so launch latency and the next
+// grid's block scheduling overlap the previous grid's tail.  Graph capture
+// keeps the programmatic edges.
+template <typename... KArgs, typename... Args>
+cudaError_t launch_step(void (*kernel)(KArgs...), dim3 grid, dim3 block, cudaStream_t st,
+                        Args&&... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = 0;
+  cfg.stream = st;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = CLOVER_PDL;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, kernel, std::forward<Args>(args)...);
+}
+
 // Enqueue kernel phases [0, nphase) of one step (7 = full step).
 int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
   cudaStream_t st = ctx->work;
@@ -432,11 +456,11 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
   if (nphase >= 1) {
     for (auto& cs : ctx->chunks) {
       const Chunk& c = cs.c;
-      ks_visc_dt<<<grid_cols(c.nx, c.ny, VKS), SB, 0, st>>>(c, cs.buf[B_D0], cs.buf[B_E0], cs.buf[B_U0],
-                                                             cs.buf[B_V0], cs.buf[B_Q], ctx->scal, ctx->dtp, cs.fix);
+      launch_step(ks_visc_dt, grid_cols(c.nx, c.ny, VKS), SB, st, c, cs.buf[B_D0], cs.buf[B_E0],
+                  cs.buf[B_U0], cs.buf[B_V0], cs.buf[B_Q], ctx->scal, ctx->dtp, cs.fix);
       STEP_LAUNCH_CHECK();
-      kf_visc_dt<<<FIX_BLOCKS, SB, 0, st>>>(c, cs.buf[B_D0], cs.buf[B_E0], cs.buf[B_U0], cs.buf[B_V0],
-                                            cs.buf[B_Q], ctx->scal, ctx->dtp, cs.fix);
+      launch_step(kf_visc_dt, FIX_BLOCKS, SB, st, c, cs.buf[B_D0], cs.buf[B_E0], cs.buf[B_U0],
+                  cs.buf[B_V0], cs.buf[B_Q], ctx->scal, ctx->dtp, cs.fix);
       STEP_LAUNCH_CHECK();
     }
     int rc = exchange(ctx, {B_Q});
@@ -450,18 +474,18 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
       NK(ncclAllReduce(&ctx->scal->dt_slot, &ctx->scal->dt_slot, 1, ncclUint64, ncclMin, ctx->comm, st));
 #endif
     if (ctx->prof) prof_mark(ctx, -1);
-    k_dt_finalize<<<1, 1, 0, st>>>(ctx->scal, ctx->hist, ctx->dtp);
+    launch_step(k_dt_finalize, 1, 1, st, ctx->scal, ctx->hist, ctx->dtp);
     STEP_LAUNCH_CHECK();
   }
   if (nphase >= 3) {
     cur_prof_id = P_LAGR;
     for (auto& cs : ctx->chunks) {
       const Chunk& c = cs.c;
-      ks_lagrangian<<<grid_strip(c.nx, LW, c.ny, LKS), SB, 0, st>>>(
+      launch_step(ks_lagrangian, grid_strip(c.nx, LW, c.ny, LKS), SB, st,
           c, cs.buf[B_D0], cs.buf[B_E0], cs.buf[B_U0], cs.buf[B_V0], cs.buf[B_Q], cs.buf[B_D1],
           cs.buf[B_E1], cs.buf[B_U1], cs.buf[B_V1], cs.buf[B_FX], cs.buf[B_FY], ctx->scal, cs.fix);
       STEP_LAUNCH_CHECK();
-      kf_lagrangian<<<FIX_BLOCKS, SB, 0, st>>>(
+      launch_step(kf_lagrangian, FIX_BLOCKS, SB, st,
           c, cs.buf[B_D0], cs.buf[B_E0], cs.buf[B_U0], cs.buf[B_V0], cs.buf[B_Q], cs.buf[B_D1],
           cs.buf[B_E1], cs.buf[B_U1], cs.buf[B_V1], cs.buf[B_FX], cs.buf[B_FY], ctx->scal, cs.fix);
       STEP_LAUNCH_CHECK();
@@ -488,24 +512,24 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
         if (xdir) {
           const dim3 g = grid_strip(c.nx, CW_X, c.ny, CKS);
           if (sweep == 1) {
-            ks_advec_cell_x<1><<<g, SB, 0, st>>>(c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf], cs.fix);
+            launch_step(ks_advec_cell_x<1>, g, SB, st, c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf], cs.fix);
             STEP_LAUNCH_CHECK();
-            kf_advec_cell_x<1><<<FIX_BLOCKS, SB, 0, st>>>(c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf], cs.fix);
+            launch_step(kf_advec_cell_x<1>, FIX_BLOCKS, SB, st, c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf], cs.fix);
           } else {
-            ks_advec_cell_x<2><<<g, SB, 0, st>>>(c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf], cs.fix);
+            launch_step(ks_advec_cell_x<2>, g, SB, st, c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf], cs.fix);
             STEP_LAUNCH_CHECK();
-            kf_advec_cell_x<2><<<FIX_BLOCKS, SB, 0, st>>>(c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf], cs.fix);
+            launch_step(kf_advec_cell_x<2>, FIX_BLOCKS, SB, st, c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf], cs.fix);
           }
         } else {
           const dim3 g = grid_cols(c.nx, c.ny, CKS_Y);
           if (sweep == 1) {
-            ks_advec_cell_y<1><<<g, SB, 0, st>>>(c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf], cs.fix);
+            launch_step(ks_advec_cell_y<1>, g, SB, st, c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf], cs.fix);
             STEP_LAUNCH_CHECK();
-            kf_advec_cell_y<1><<<FIX_BLOCKS, SB, 0, st>>>(c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf], cs.fix);
+            launch_step(kf_advec_cell_y<1>, FIX_BLOCKS, SB, st, c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf], cs.fix);
           } else {
-            ks_advec_cell_y<2><<<g, SB, 0, st>>>(c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf], cs.fix);
+            launch_step(ks_advec_cell_y<2>, g, SB, st, c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf], cs.fix);
             STEP_LAUNCH_CHECK();
-            kf_advec_cell_y<2><<<FIX_BLOCKS, SB, 0, st>>>(c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf], cs.fix);
+            launch_step(kf_advec_cell_y<2>, FIX_BLOCKS, SB, st, c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf], cs.fix);
           }
         }
         STEP_LAUNCH_CHECK();
@@ -521,24 +545,24 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
         if (xdir) {
           const dim3 g = grid_strip(c.nx + 1, MW_X, c.ny + 1, MKS);
           if (sweep == 1) {
-            ks_advec_mom_x<1><<<g, SB, 0, st>>>(c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FY], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout], cs.fix);
+            launch_step(ks_advec_mom_x<1>, g, SB, st, c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FY], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout], cs.fix);
             STEP_LAUNCH_CHECK();
-            kf_advec_mom_x<1><<<FIX_BLOCKS, SB, 0, st>>>(c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FY], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout], cs.fix);
+            launch_step(kf_advec_mom_x<1>, FIX_BLOCKS, SB, st, c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FY], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout], cs.fix);
           } else {
-            ks_advec_mom_x<2><<<g, SB, 0, st>>>(c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FY], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout], cs.fix);
+            launch_step(ks_advec_mom_x<2>, g, SB, st, c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FY], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout], cs.fix);
             STEP_LAUNCH_CHECK();
-            kf_advec_mom_x<2><<<FIX_BLOCKS, SB, 0, st>>>(c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FY], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout], cs.fix);
+            launch_step(kf_advec_mom_x<2>, FIX_BLOCKS, SB, st, c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FY], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout], cs.fix);
           }
         } else {
           const dim3 g = grid_cols(c.nx + 1, c.ny + 1, MKS_Y);
           if (sweep == 1) {
-            ks_advec_mom_y<1><<<g, SB, 0, st>>>(c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FX], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout], cs.fix);
+            launch_step(ks_advec_mom_y<1>, g, SB, st, c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FX], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout], cs.fix);
             STEP_LAUNCH_CHECK();
-            kf_advec_mom_y<1><<<FIX_BLOCKS, SB, 0, st>>>(c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FX], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout], cs.fix);
+            launch_step(kf_advec_mom_y<1>, FIX_BLOCKS, SB, st, c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FX], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout], cs.fix);
           } else {
-            ks_advec_mom_y<2><<<g, SB, 0, st>>>(c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FX], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout], cs.fix);
+            launch_step(ks_advec_mom_y<2>, g, SB, st, c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FX], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout], cs.fix);
             STEP_LAUNCH_CHECK();
-            kf_advec_mom_y<2><<<FIX_BLOCKS, SB, 0, st>>>(c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FX], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout], cs.fix);
+            launch_step(kf_advec_mom_y<2>, FIX_BLOCKS, SB, st, c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FX], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout], cs.fix);
           }
         }
         STEP_LAUNCH_CHECK();

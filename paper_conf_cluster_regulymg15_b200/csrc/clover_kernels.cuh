@@ -133,6 +133,8 @@ struct DtAcc {
 // ------------------------------------------------ k_dt_finalize (c.4 tail)
 __global__ void k_dt_finalize(StepScalars* __restrict__ s, double* __restrict__ hist,
                               DtParams prm) {
+  pdl_trigger();
+  pdl_wait();
   double dtc = __longlong_as_double((long long)s->dt_slot);
   double dt = fmin(fmin(dtc, (s->dtold * prm.dtrise)), prm.dtmax);
   s->dt = dt;

@@ -192,6 +192,8 @@ __global__ void LB_VISC
 ks_visc_dt(Chunk c, const double* __restrict__ d0, const double* __restrict__ e0,
            const double* __restrict__ u0, const double* __restrict__ v0, double* __restrict__ q,
            StepScalars* __restrict__ s, DtParams prm, FixSlot fix) {
+  pdl_trigger();
+  pdl_wait();
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const int gw = blockIdx.x * (SB / 32) + warp;
   double dtw;
@@ -214,6 +216,8 @@ __global__ void __launch_bounds__(SB)
 kf_visc_dt(Chunk c, const double* __restrict__ d0, const double* __restrict__ e0,
            const double* __restrict__ u0, const double* __restrict__ v0, double* __restrict__ q,
            StepScalars* __restrict__ s, DtParams prm, FixSlot fix) {
+  pdl_trigger();
+  pdl_wait();
   fix_loop(fix, VKS, c.ny + 1, [&](int gw, int k0, int k1, int lane, int) {
     double dtw;
     visc_body<DivIEEE>(c, d0, e0, u0, v0, q, prm, gw, k0, k1, lane, dtw);
@@ -401,6 +405,8 @@ ks_lagrangian(Chunk c, const double* __restrict__ d0, const double* __restrict__
               const double* __restrict__ q, double* __restrict__ d1, double* __restrict__ e1,
               double* __restrict__ u1, double* __restrict__ v1, double* __restrict__ fx,
               double* __restrict__ fy, const StepScalars* __restrict__ s, FixSlot fix) {
+  pdl_trigger();
+  pdl_wait();
   __shared__ __align__(128) double ring[SB / 32][LSTG][LNF][LRW];
   __shared__ __align__(8) unsigned long long bars[SB / 32][LSTG];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
@@ -418,6 +424,8 @@ kf_lagrangian(Chunk c, const double* __restrict__ d0, const double* __restrict__
               const double* __restrict__ q, double* __restrict__ d1, double* __restrict__ e1,
               double* __restrict__ u1, double* __restrict__ v1, double* __restrict__ fx,
               double* __restrict__ fy, const StepScalars* __restrict__ s, FixSlot fix) {
+  pdl_trigger();
+  pdl_wait();
   __shared__ __align__(128) double ring[SB / 32][LSTG][LNF][LRW];
   __shared__ __align__(8) unsigned long long bars[SB / 32][LSTG];
   fix_loop(fix, LKS, c.ny + 1, [&](int gw, int k0, int k1, int lane, int w) {
@@ -498,6 +506,8 @@ ks_advec_cell_x(Chunk c, const double* __restrict__ rho, const double* __restric
                 const double* __restrict__ fx, const double* __restrict__ fy,
                 double* __restrict__ rho_out, double* __restrict__ en_out,
                 double* __restrict__ mfx, FixSlot fix) {
+  pdl_trigger();
+  pdl_wait();
   const int lane = threadIdx.x & 31;
   const int gw = blockIdx.x * (SB / 32) + (threadIdx.x >> 5);
   const int k0 = blockIdx.y * CKS + 1, k1 = min(k0 + CKS, c.ny + 1);
@@ -512,6 +522,8 @@ kf_advec_cell_x(Chunk c, const double* __restrict__ rho, const double* __restric
                 const double* __restrict__ fx, const double* __restrict__ fy,
                 double* __restrict__ rho_out, double* __restrict__ en_out,
                 double* __restrict__ mfx, FixSlot fix) {
+  pdl_trigger();
+  pdl_wait();
   fix_loop(fix, CKS, c.ny + 1, [&](int gw, int k0, int k1, int lane, int) {
     advec_cell_x_body<SWEEP, DivIEEE>(c, rho, en, fx, fy, rho_out, en_out, mfx, gw, k0, k1, lane);
   });
@@ -599,6 +611,8 @@ ks_advec_cell_y(Chunk c, const double* __restrict__ rho, const double* __restric
                 const double* __restrict__ fx, const double* __restrict__ fy,
                 double* __restrict__ rho_out, double* __restrict__ en_out,
                 double* __restrict__ mfy, FixSlot fix) {
+  pdl_trigger();
+  pdl_wait();
   const int lane = threadIdx.x & 31;
   const int gw = blockIdx.x * (SB / 32) + (threadIdx.x >> 5);
   const int k0 = blockIdx.y * CKS_Y + 1, k1 = min(k0 + CKS_Y, c.ny + 1);
@@ -613,6 +627,8 @@ kf_advec_cell_y(Chunk c, const double* __restrict__ rho, const double* __restric
                 const double* __restrict__ fx, const double* __restrict__ fy,
                 double* __restrict__ rho_out, double* __restrict__ en_out,
                 double* __restrict__ mfy, FixSlot fix) {
+  pdl_trigger();
+  pdl_wait();
   fix_loop(fix, CKS_Y, c.ny + 1, [&](int gw, int k0, int k1, int lane, int) {
     advec_cell_y_body<SWEEP, DivIEEE>(c, rho, en, fx, fy, rho_out, en_out, mfy, gw, k0, k1, lane);
   });
@@ -697,6 +713,8 @@ ks_advec_mom_x(Chunk c, const double* __restrict__ rho, const double* __restrict
                const double* __restrict__ fy, const double* __restrict__ uin,
                const double* __restrict__ vin, double* __restrict__ uout,
                double* __restrict__ vout, FixSlot fix) {
+  pdl_trigger();
+  pdl_wait();
   const int lane = threadIdx.x & 31;
   const int gw = blockIdx.x * (SB / 32) + (threadIdx.x >> 5);
   const int k0 = blockIdx.y * MKS + 1, k1 = min(k0 + MKS, c.ny + 2);
@@ -711,6 +729,8 @@ kf_advec_mom_x(Chunk c, const double* __restrict__ rho, const double* __restrict
                const double* __restrict__ fy, const double* __restrict__ uin,
                const double* __restrict__ vin, double* __restrict__ uout,
                double* __restrict__ vout, FixSlot fix) {
+  pdl_trigger();
+  pdl_wait();
   fix_loop(fix, MKS, c.ny + 2, [&](int gw, int k0, int k1, int lane, int) {
     advec_mom_x_body<SWEEP, DivIEEE>(c, rho, mfx, fy, uin, vin, uout, vout, gw, k0, k1, lane);
   });
@@ -807,6 +827,8 @@ ks_advec_mom_y(Chunk c, const double* __restrict__ rho, const double* __restrict
                const double* __restrict__ fx, const double* __restrict__ uin,
                const double* __restrict__ vin, double* __restrict__ uout,
                double* __restrict__ vout, FixSlot fix) {
+  pdl_trigger();
+  pdl_wait();
   const int lane = threadIdx.x & 31;
   const int gw = blockIdx.x * (SB / 32) + (threadIdx.x >> 5);
   const int k0 = blockIdx.y * MKS_Y + 1, k1 = min(k0 + MKS_Y, c.ny + 2);
@@ -821,6 +843,8 @@ kf_advec_mom_y(Chunk c, const double* __restrict__ rho, const double* __restrict
                const double* __restrict__ fx, const double* __restrict__ uin,
                const double* __restrict__ vin, double* __restrict__ uout,
                double* __restrict__ vout, FixSlot fix) {
+  pdl_trigger();
+  pdl_wait();
   fix_loop(fix, MKS_Y, c.ny + 2, [&](int gw, int k0, int k1, int lane, int) {
     advec_mom_y_body<SWEEP, DivIEEE>(c, rho, mfy, fx, uin, vin, uout, vout, gw, k0, k1, lane);
   });
