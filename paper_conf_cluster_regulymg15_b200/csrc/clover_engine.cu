@@ -406,6 +406,13 @@ dim3 cell_grid(const Chunk& c, int bx, int by) { return dim3((c.nx + bx - 1) / b
     LAUNCH_CHECK();                                                               \
     if (ctx->prof) prof_mark(ctx, cur_prof_id);                                   \
   } while (0)
+// after a fixup launch: its time joins the phase, it is not counted as a launch
+constexpr int PROF_FIXUP = 0x100;
+#define FIX_LAUNCH_CHECK()                                                        \
+  do {                                                                            \
+    LAUNCH_CHECK();                                                               \
+    if (ctx->prof) prof_mark(ctx, cur_prof_id | PROF_FIXUP);                      \
+  } while (0)
 
 // Kernel types for clover_profile (names in kProfNames).
 enum { P_VISC_DT, P_DT_FINAL, P_LAGR, P_CELL_X1, P_CELL_X2, P_CELL_Y1, P_CELL_Y2,
@@ -461,7 +468,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
       STEP_LAUNCH_CHECK();
       launch_step(kf_visc_dt, FIX_BLOCKS, SB, st, c, cs.buf[B_D0], cs.buf[B_E0], cs.buf[B_U0],
                   cs.buf[B_V0], cs.buf[B_Q], ctx->scal, ctx->dtp, cs.fix);
-      STEP_LAUNCH_CHECK();
+      FIX_LAUNCH_CHECK();
     }
     int rc = exchange(ctx, {B_Q});
     if (rc) return rc;
@@ -488,7 +495,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
       launch_step(kf_lagrangian, FIX_BLOCKS, SB, st,
           c, cs.buf[B_D0], cs.buf[B_E0], cs.buf[B_U0], cs.buf[B_V0], cs.buf[B_Q], cs.buf[B_D1],
           cs.buf[B_E1], cs.buf[B_U1], cs.buf[B_V1], cs.buf[B_FX], cs.buf[B_FY], ctx->scal, cs.fix);
-      STEP_LAUNCH_CHECK();
+      FIX_LAUNCH_CHECK();
     }
     int rc = exchange(ctx, {B_D1, B_E1, B_U1, B_V1, B_FX, B_FY});
     if (rc) return rc;
@@ -515,10 +522,12 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
             launch_step(ks_advec_cell_x<1>, g, SB, st, c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf], cs.fix);
             STEP_LAUNCH_CHECK();
             launch_step(kf_advec_cell_x<1>, FIX_BLOCKS, SB, st, c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf], cs.fix);
+            FIX_LAUNCH_CHECK();
           } else {
             launch_step(ks_advec_cell_x<2>, g, SB, st, c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf], cs.fix);
             STEP_LAUNCH_CHECK();
             launch_step(kf_advec_cell_x<2>, FIX_BLOCKS, SB, st, c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf], cs.fix);
+            FIX_LAUNCH_CHECK();
           }
         } else {
           const dim3 g = grid_cols(c.nx, c.ny, CKS_Y);
@@ -526,13 +535,14 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
             launch_step(ks_advec_cell_y<1>, g, SB, st, c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf], cs.fix);
             STEP_LAUNCH_CHECK();
             launch_step(kf_advec_cell_y<1>, FIX_BLOCKS, SB, st, c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf], cs.fix);
+            FIX_LAUNCH_CHECK();
           } else {
             launch_step(ks_advec_cell_y<2>, g, SB, st, c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf], cs.fix);
             STEP_LAUNCH_CHECK();
             launch_step(kf_advec_cell_y<2>, FIX_BLOCKS, SB, st, c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf], cs.fix);
+            FIX_LAUNCH_CHECK();
           }
         }
-        STEP_LAUNCH_CHECK();
       }
       int rc = exchange(ctx, {rout, eout, mbuf});
       if (rc) return rc;
@@ -548,10 +558,12 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
             launch_step(ks_advec_mom_x<1>, g, SB, st, c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FY], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout], cs.fix);
             STEP_LAUNCH_CHECK();
             launch_step(kf_advec_mom_x<1>, FIX_BLOCKS, SB, st, c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FY], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout], cs.fix);
+            FIX_LAUNCH_CHECK();
           } else {
             launch_step(ks_advec_mom_x<2>, g, SB, st, c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FY], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout], cs.fix);
             STEP_LAUNCH_CHECK();
             launch_step(kf_advec_mom_x<2>, FIX_BLOCKS, SB, st, c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FY], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout], cs.fix);
+            FIX_LAUNCH_CHECK();
           }
         } else {
           const dim3 g = grid_cols(c.nx + 1, c.ny + 1, MKS_Y);
@@ -559,13 +571,14 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
             launch_step(ks_advec_mom_y<1>, g, SB, st, c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FX], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout], cs.fix);
             STEP_LAUNCH_CHECK();
             launch_step(kf_advec_mom_y<1>, FIX_BLOCKS, SB, st, c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FX], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout], cs.fix);
+            FIX_LAUNCH_CHECK();
           } else {
             launch_step(ks_advec_mom_y<2>, g, SB, st, c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FX], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout], cs.fix);
             STEP_LAUNCH_CHECK();
             launch_step(kf_advec_mom_y<2>, FIX_BLOCKS, SB, st, c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FX], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout], cs.fix);
+            FIX_LAUNCH_CHECK();
           }
         }
-        STEP_LAUNCH_CHECK();
       }
       int rc = exchange(ctx, {uout, vout});
       if (rc) return rc;
@@ -1079,8 +1092,8 @@ int clover_profile_steps(clover_ctx* ctx, int32_t nsteps, double* ms_out, int64_
     if (id < 0) continue;
     float ms = 0.f;
     cudaEventElapsedTime(&ms, ctx->prof_events[i - 1].second, ctx->prof_events[i].second);
-    ms_out[id] += ms;
-    launches_out[id] += 1;
+    ms_out[id & (PROF_FIXUP - 1)] += ms;
+    if (!(id & PROF_FIXUP)) launches_out[id] += 1;
   }
   for (auto& pe : ctx->prof_events) cudaEventDestroy(pe.second);
   ctx->prof_events.clear();
