@@ -47,8 +47,13 @@ ALGO_BYTES_PER_CELL = {
     "k_advec_mom_y<1>": 8 * (5 + 2),
     "k_advec_mom_x<2>": 8 * (4 + 2),     # rho M u v -> u v
     "k_advec_mom_y<2>": 8 * (4 + 2),
+    "k_advec_x<1>": 8 * (6 + 4),         # fused x sweep: rho e Fx Fy u v -> rho' e' u v
+    "k_advec_x<2>": 8 * (5 + 4),         # rho e Fx u v -> rho' e' u v
 }
-STEP_ALGO_BYTES_PER_CELL = 336  # sum over one step (each sweep kind once)
+# sum over one step of the kernels actually launched (the profile pass
+# below); with the fused x sweep 304/312 B for the x-first/y-first step,
+# 336 with separate kernels
+STEP_ALGO_BYTES_PER_CELL = 336
 
 
 def env_int(name, default):
@@ -265,11 +270,12 @@ def main():
         except Exception:
             traffic = None
     ach = kernels[top]["achieved_gbs"]
-    step_gbs = STEP_ALGO_BYTES_PER_CELL * local_cells * args.steps / (ms / 1e3) / 1e9
+    step_bpc = sum(ALGO_BYTES_PER_CELL.get(k, 0) * v["launches"] for k, v in kernels.items()) / args.steps
+    step_gbs = step_bpc * local_cells * args.steps / (ms / 1e3) / 1e9
     roofline = {"bound": "hbm", "kernel": top, "achieved": ach, "peak": peak, "unit": "GB/s",
                 "frac": ach / peak if ach else None, "traffic": traffic, "peak_source": peak_src,
                 "step_achieved": step_gbs, "step_frac": step_gbs / peak,
-                "algo_bytes_per_cell_step": STEP_ALGO_BYTES_PER_CELL}
+                "algo_bytes_per_cell_step": step_bpc}
 
     # end-to-end through the host-buffer C-ABI entry (pinned host memory)
     e2e = None

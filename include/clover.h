@@ -186,7 +186,7 @@ int clover_kernels_per_step(clover_ctx* ctx, int32_t* out);
  * after every kernel on the context's work stream; ms_out[i] / launches_out[i]
  * receive the summed duration and launch count of kernel type i
  * (clover_profile_name(i)); nslots must be >= CLOVER_PROFILE_SLOTS. */
-#define CLOVER_PROFILE_SLOTS 11
+#define CLOVER_PROFILE_SLOTS 13
 int clover_profile_steps(clover_ctx* ctx, int32_t nsteps, double* ms_out, int64_t* launches_out,
                          int32_t nslots);
 const char* clover_profile_name(int32_t i);
@@ -206,6 +206,13 @@ int clover_debug_partial_step(clover_ctx* ctx, int32_t nkernels);
  * 100+ internal ids, see csrc/clover_engine.cu).  Test only. */
 int clover_debug_read_buffer(clover_ctx* ctx, int32_t buffer_id, int32_t kind,
                              double* host, int64_t n);
+
+/* Debug: enable (default) or disable the fused x-sweep kernel (advec_cell x
+ * + advec_mom x in one pass, used when every local chunk has reflective
+ * walls on both x sides and the geometric face mirror).  Disabled, the
+ * x sweep runs the separate cell and momentum kernels.  Both paths are
+ * bitwise identical; tests compare them.  Test only. */
+int clover_debug_set_fusion(clover_ctx* ctx, int32_t enable);
 
 /* Debug: total number of warp segments the IEEE-division fixup launches
  * have recomputed since clover_init (DivFast flagged a numerator below

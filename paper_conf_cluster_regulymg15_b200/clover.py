@@ -22,7 +22,7 @@ c_void_p = ctypes.c_void_p
 dptr = ctypes.POINTER(c_double)
 
 CLOVER_OK = 0
-PROFILE_SLOTS = 11
+PROFILE_SLOTS = 13
 ERRORS = {-1: "ARG", -2: "CUDA", -3: "NCCL", -4: "WORKSPACE", -5: "SMALL_DT", -7: "STATE"}
 
 FIELDS = {"density0": 0, "energy0": 1, "pressure": 2, "viscosity": 3, "soundspeed": 4,
@@ -39,7 +39,7 @@ EXPORTS = ["clover_workspace_bytes", "clover_nccl_unique_id", "clover_init", "cl
            "clover_read_field", "clover_write_field", "clover_sync", "clover_set_graphs",
            "clover_kernels_per_step", "clover_debug_partial_step", "clover_debug_read_buffer",
            "clover_profile_steps", "clover_profile_name", "clover_debug_div_check",
-           "clover_debug_fix_count",
+           "clover_debug_fix_count", "clover_debug_set_fusion",
            "clover_checkpoint_plan", "clover_debug_set_virtual_remote", "clover_checkpoint_bytes", "clover_checkpoint", "clover_restart", "clover_finalize", "clover_error_string", "clover_last_error", "clover_abi_version"]
 
 
@@ -108,6 +108,8 @@ def load(build_if_missing: bool = True):
     L.clover_profile_name.restype = ctypes.c_char_p
     if hasattr(L, "clover_debug_fix_count"):  # absent from older builds (A/B harness)
         L.clover_debug_fix_count.argtypes = [c_void_p, ctypes.POINTER(c_int64)]
+    if hasattr(L, "clover_debug_set_fusion"):
+        L.clover_debug_set_fusion.argtypes = [c_void_p, c_int32]
     L.clover_debug_div_check.argtypes = [c_int64, ctypes.c_uint64, c_int32, ctypes.POINTER(c_int64), dptr]
     L.clover_checkpoint_plan.argtypes = [c_int32, ctypes.POINTER(ctypes.c_uint32), ctypes.POINTER(c_int32),
                                          ctypes.POINTER(ctypes.c_char_p)]
@@ -319,6 +321,10 @@ class Clover:
 
     def debug_partial_step(self, nkernels: int):
         _check(load().clover_debug_partial_step(self._ctx, nkernels), "clover_debug_partial_step")
+
+    def debug_set_fusion(self, enable: bool):
+        """Fused x sweep on (default) or off (separate cell / momentum kernels)."""
+        _check(load().clover_debug_set_fusion(self._ctx, 1 if enable else 0), "clover_debug_set_fusion")
 
     def debug_fix_count(self) -> int:
         """Warp segments recomputed so far by the IEEE-division fixup launches."""

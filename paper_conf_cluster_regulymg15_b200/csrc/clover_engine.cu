@@ -120,9 +120,10 @@ dim3 grid_strip(int ncols, int width, int nrows, int ks) {
   return dim3(cdiv(cdiv(ncols, width), SB / 32), cdiv(nrows, ks));
 }
 int64_t fix_capacity(int nx, int ny) {
-  const dim3 g[6] = {grid_cols(nx, ny, VKS),          grid_strip(nx, LW, ny, LKS),
+  const dim3 g[7] = {grid_cols(nx, ny, VKS),          grid_strip(nx, LW, ny, LKS),
                      grid_strip(nx, CW_X, ny, CKS),    grid_cols(nx, ny, CKS_Y),
-                     grid_strip(nx + 1, MW_X, ny + 1, MKS), grid_cols(nx + 1, ny + 1, MKS_Y)};
+                     grid_strip(nx + 1, MW_X, ny + 1, MKS), grid_cols(nx + 1, ny + 1, MKS_Y),
+                     grid_strip(nx + 1, XW, ny + 1, XKS)};
   int64_t m = 0;
   for (const dim3& d : g) m = std::max<int64_t>(m, (int64_t)d.x * d.y * (SB / 32));
   return m;
@@ -149,6 +150,7 @@ struct clover_ctx {
   GlobalGeom gg;
   bool advect_x = true;
   bool use_graphs = true;
+  bool fuse_x = true;  // fused x sweep where every chunk has both x walls (see fuse_x_ok)
   cudaGraphExec_t gexec[2] = {nullptr, nullptr};
   int64_t ws_bytes = 0;
   bool prof = false;
@@ -416,11 +418,13 @@ constexpr int PROF_FIXUP = 0x100;
 
 // Kernel types for clover_profile (names in kProfNames).
 enum { P_VISC_DT, P_DT_FINAL, P_LAGR, P_CELL_X1, P_CELL_X2, P_CELL_Y1, P_CELL_Y2,
-       P_MOM_X1, P_MOM_X2, P_MOM_Y1, P_MOM_Y2, NPROF };
+       P_MOM_X1, P_MOM_X2, P_MOM_Y1, P_MOM_Y2, P_ADV_X1, P_ADV_X2, NPROF };
 const char* kProfNames[NPROF] = {"k_visc_dt", "k_dt_finalize", "k_lagrangian",
                                  "k_advec_cell_x<1>", "k_advec_cell_x<2>", "k_advec_cell_y<1>",
                                  "k_advec_cell_y<2>", "k_advec_mom_x<1>", "k_advec_mom_x<2>",
-                                 "k_advec_mom_y<1>", "k_advec_mom_y<2>"};
+                                 "k_advec_mom_y<1>", "k_advec_mom_y<2>", "k_advec_x<1>",
+                                 "k_advec_x<2>"};
+static_assert(NPROF == CLOVER_PROFILE_SLOTS, "profile slots");
 
 // Record an event after each profiled kernel; (prev event, this event)
 // bracket exactly that kernel on the work stream.
@@ -453,6 +457,17 @@ cudaError_t launch_step(void (*kernel)(KArgs...), dim3 grid, dim3 block, cudaStr
   cfg.attrs = at;
   cfg.numAttrs = 1;
   return cudaLaunchKernelEx(&cfg, kernel, std::forward<Args>(args)...);
+}
+
+// The fused x sweep needs every chunk to have reflective walls on both x
+// sides (its wall halo columns are mirrors of lanes in the same warp; at a
+// chunk boundary the x stencil would need depth-3 halos) and the geometric
+// face mirror.
+bool fuse_x_ok(const clover_ctx* ctx) {
+  if (!ctx->fuse_x || ctx->g.face_mirror == CLOVER_MIRROR_CELLCENTRE) return false;
+  for (const auto& cs : ctx->chunks)
+    if (!cs.c.wl || !cs.c.wr) return false;
+  return true;
 }
 
 // Enqueue kernel phases [0, nphase) of one step (7 = full step).
@@ -510,6 +525,40 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
     const int uin = sweep == 1 ? B_U1 : B_U2, vin = sweep == 1 ? B_V1 : B_V2;
     const int uout = sweep == 1 ? B_U2 : B_U0, vout = sweep == 1 ? B_V2 : B_V0;
     const int mbuf = xdir ? B_MX : B_MY;
+    if (xdir && fuse_x_ok(ctx)) {
+      // advec_cell x + advec_mom x in one kernel (ks_advec_x): phase ph_cell
+      // runs both, phase ph_cell + 1 is empty
+      if (nphase >= ph_cell) {
+        cur_prof_id = sweep == 1 ? P_ADV_X1 : P_ADV_X2;
+        for (auto& cs : ctx->chunks) {
+          const Chunk& c = cs.c;
+          const dim3 g = grid_strip(c.nx + 1, XW, c.ny + 1, XKS);
+          const double* fx = cs.buf[B_FX];
+          const double* fy = cs.buf[B_FY];
+          if (sweep == 1) {
+            launch_step(ks_advec_x<1>, g, SB, st, c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[uin],
+                        cs.buf[vin], cs.buf[rout], cs.buf[eout], cs.buf[uout], cs.buf[vout], cs.fix);
+            STEP_LAUNCH_CHECK();
+            launch_step(kf_advec_x<1>, FIX_BLOCKS, SB, st, c, cs.buf[rin], cs.buf[ein], fx, fy,
+                        cs.buf[uin], cs.buf[vin], cs.buf[rout], cs.buf[eout], cs.buf[uout],
+                        cs.buf[vout], cs.fix);
+            FIX_LAUNCH_CHECK();
+          } else {
+            launch_step(ks_advec_x<2>, g, SB, st, c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[uin],
+                        cs.buf[vin], cs.buf[rout], cs.buf[eout], cs.buf[uout], cs.buf[vout], cs.fix);
+            STEP_LAUNCH_CHECK();
+            launch_step(kf_advec_x<2>, FIX_BLOCKS, SB, st, c, cs.buf[rin], cs.buf[ein], fx, fy,
+                        cs.buf[uin], cs.buf[vin], cs.buf[rout], cs.buf[eout], cs.buf[uout],
+                        cs.buf[vout], cs.fix);
+            FIX_LAUNCH_CHECK();
+          }
+        }
+        int rc = exchange(ctx, {rout, eout, uout, vout});
+        if (rc) return rc;
+        if (ctx->prof) prof_mark(ctx, -1);
+      }
+      continue;
+    }
     if (nphase >= ph_cell) {
       cur_prof_id = xdir ? (sweep == 1 ? P_CELL_X1 : P_CELL_X2) : (sweep == 1 ? P_CELL_Y1 : P_CELL_Y2);
       for (auto& cs : ctx->chunks) {
@@ -1023,6 +1072,17 @@ int clover_debug_set_virtual_remote(clover_ctx* ctx, int32_t enable) {
   if (ctx->nranks > 1) return fail(CLOVER_ERR_STATE, "virtual remote is a single-process test mode");
   if (enable && ctx->L.px * ctx->L.py < 2) return fail(CLOVER_ERR_STATE, "virtual remote needs px*py > 1");
   ctx->virtual_remote = enable != 0;
+  for (int i = 0; i < 2; ++i)
+    if (ctx->gexec[i]) {
+      cudaGraphExecDestroy(ctx->gexec[i]);
+      ctx->gexec[i] = nullptr;
+    }
+  return CLOVER_OK;
+}
+
+int clover_debug_set_fusion(clover_ctx* ctx, int32_t enable) {
+  if (!ctx) return fail(CLOVER_ERR_ARG, "ctx is NULL");
+  ctx->fuse_x = enable != 0;
   for (int i = 0; i < 2; ++i)
     if (ctx->gexec[i]) {
       cudaGraphExecDestroy(ctx->gexec[i]);

@@ -53,6 +53,14 @@ constexpr int SB = CLOVER_SB;  // threads per block
 #ifndef CLOVER_MINB_VISC
 #define CLOVER_MINB_VISC 0
 #endif
+#ifndef CLOVER_MINB_ADVX
+#define CLOVER_MINB_ADVX 0
+#endif
+#if CLOVER_MINB_ADVX > 0
+#define LB_ADVX __launch_bounds__(SB, CLOVER_MINB_ADVX)
+#else
+#define LB_ADVX __launch_bounds__(SB)
+#endif
 #ifndef CLOVER_MINB_MOMY
 #define CLOVER_MINB_MOMY 14
 #endif
@@ -733,6 +741,197 @@ kf_advec_mom_x(Chunk c, const double* __restrict__ rho, const double* __restrict
   pdl_wait();
   fix_loop(fix, MKS, c.ny + 2, [&](int gw, int k0, int k1, int lane, int) {
     advec_mom_x_body<SWEEP, DivIEEE>(c, rho, mfx, fy, uin, vin, uout, vout, gw, k0, k1, lane);
+  });
+}
+
+// ================================================================ fused x sweep
+// advec_cell (x) and advec_mom (x) of one sweep in one pass, for chunks with
+// reflective walls on both x sides (px == 1) and the geometric face mirror.
+// Warp strip: lane l <-> column j = J0 - 2 + l, J0 = 1 + 28*(warp).  At cell
+// row r every lane computes the x-face flux of face j and (lanes 0..30) the
+// cell update of cell j; lanes on wall halo columns take the mirror image of
+// the computed interior value instead (the reference's update_halo after
+// advec_cell: density/energy mirror with +, x-face mass flux with -), so
+// the mass flux and post-advection density the momentum update reads never
+// travel through memory.  Node row r then follows as in ks_advec_mom_x
+// (node flux from rows r-1, r; masses of cells j-1, j).  Lanes 2..29 own
+// cells and nodes.  Cell rows k0-1 .. k1-1 are computed (the first one
+// repeats the previous segment's last row).  Halo rows: at a y wall the
+// mirror of the adjacent interior row, at a chunk boundary computed from the
+// depth-2 input halos (bitwise what the neighbour computes).
+constexpr int XW = 28;
+#ifndef CLOVER_XKS
+#define CLOVER_XKS 8
+#endif
+constexpr int XKS = CLOVER_XKS;
+
+template <int SWEEP, class D>
+__device__ __forceinline__ bool advec_x_body(const Chunk& c, const double* __restrict__ rho,
+                                             const double* __restrict__ en,
+                                             const double* __restrict__ fx,
+                                             const double* __restrict__ fy,
+                                             const double* __restrict__ uin,
+                                             const double* __restrict__ vin,
+                                             double* __restrict__ rho_out,
+                                             double* __restrict__ en_out,
+                                             double* __restrict__ uout,
+                                             double* __restrict__ vout, int gw, int k0, int k1,
+                                             int lane) {
+  D dv;
+  const int J0 = 1 + XW * gw;
+  if (J0 > c.nx + 1) return false;
+  const int j = J0 - 2 + lane;
+  const double vol = c.dx * c.dy;
+  const int P = c.pitch;
+  const int nx = c.nx;
+  const bool faceok = j >= 1 && j <= nx + 1;  // faces computed here (others mirrored)
+  const bool cellok = j >= 0 && j <= nx + 2;  // pre_vol inputs exist
+  const bool mpok = j >= -1 && j <= nx + 2;   // node-mass columns
+  const bool ncol = near_wall_col(c, j);
+  const bool own = lane >= 2 && lane < 2 + XW;
+  // mirror sources at the x walls (lanes of this warp, see header)
+  int src_m = lane, src_r = lane;
+  double sgn_m = 1.0;
+  if (j <= 0) { src_m = lane + 2 - 2 * j; src_r = lane + 1 - 2 * j; sgn_m = -1.0; }
+  if (j >= nx + 2) { src_m = lane + 2 * nx + 2 - 2 * j; sgn_m = -1.0; }
+  if (j >= nx + 1) src_r = lane + 2 * nx + 1 - 2 * j;
+  if (src_m < 0 || src_m > 31) src_m = lane;
+  if (src_r < 0 || src_r > 31) src_r = lane;
+  const bool xwall_warp = __any_sync(FULL, src_m != lane || src_r != lane);
+  auto pv_mom = [&](int i) -> double { return (SWEEP == 1) ? vol + fy[i + P] - fy[i] : vol; };
+
+  double mA_m = 0.0, mp_m = 0.0, mB_m = 0.0, mpl_m = 0.0, ro_m = 0.0;
+  for (int r = k0 - 1; r < k1; ++r) {
+    const int i = idx(c, j, r);
+    const bool mir_bot = c.wb && r == 0;
+    const bool mir_top = c.wt && r == c.ny + 1;
+    if (mir_bot) continue;  // synthesised from row 1 below
+    double mA = 0.0, ro = 0.0;
+    if (mir_top) {
+      // row ny+1 = mirror of row ny (already mirrored along x)
+      mA = mA_m; ro = ro_m;
+    } else {
+      // ---- advec_cell x, row r
+      double pv = 0.0, F = 0.0, m = 0.0, ef = 0.0, rr = 0.0, ee = 0.0, flo = 0.0, fhi = 0.0;
+      if (cellok) {
+        flo = fx[i]; fhi = fx[i + 1];
+        F = flo;
+        pv = (SWEEP == 1) ? vol + (fhi - flo + fy[i + P] - fy[i]) : vol + fhi - flo;
+        rr = rho[i]; ee = en[i];
+      }
+      double pvl = __shfl_up_sync(FULL, pv, 1);
+      if (faceok) {
+        if (lane == 0) {
+          const double fl = fx[i - 1];
+          pvl = (SWEEP == 1) ? vol + (flo - fl + fy[i - 1 + P] - fy[i - 1]) : vol + flo - fl;
+        }
+        double ru, rd, rw, eu, ed, ew, pvd;
+        if (F > 0.0) {
+          ru = rho[i - 2]; rd = rho[i - 1]; rw = rr;
+          eu = en[i - 2]; ed = en[i - 1]; ew = ee;
+          pvd = pvl;
+        } else {
+          const int up = min(j + 1, nx + 2) - j;
+          ru = rho[i + up]; rd = rr; rw = rho[i - 1];
+          eu = en[i + up]; ed = ee; ew = en[i - 1];
+          pvd = pv;
+        }
+        cell_face_flux(dv, F, pvd, ru, rd, rw, eu, ed, ew, m, ef);
+      }
+      const double mh = __shfl_down_sync(FULL, m, 1);
+      const double efh = __shfl_down_sync(FULL, ef, 1);
+      double eo = 0.0;
+      if (j >= 1 && j <= nx && lane < 31) {
+        cell_update(dv, rr, ee, pv, m, mh, ef, efh, flo, fhi, ro, eo);
+        if (own && r >= k0 && r <= c.ny) {
+          const bool near = ncol || near_wall_row(c, r);
+          store_at(c, rho_out, K_CELL, j, r, i, near, ro);
+          store_at(c, en_out, K_CELL, j, r, i, near, eo);
+        }
+      }
+      mA = m;
+      if (xwall_warp) {
+        const double ms = __shfl_sync(FULL, m, src_m);
+        const double rs = __shfl_sync(FULL, ro, src_r);
+        if (src_m != lane) mA = sgn_m * ms;
+        if (src_r != lane) ro = rs;
+      }
+    }
+    const double mB = __shfl_down_sync(FULL, mA, 1);
+    double mp = 0.0;
+    if (mpok) mp = ro * pv_mom(i);
+    const double mpl = __shfl_up_sync(FULL, mp, 1);
+    if (c.wb && r == 1) {
+      // row 0 = mirror of row 1: same mass fluxes and density, row-0 volumes
+      mA_m = mA; mB_m = mB;
+      mp_m = mpok ? ro * pv_mom(i - P) : 0.0;
+      mpl_m = __shfl_up_sync(FULL, mp_m, 1);
+    }
+    if (r >= k0) {
+      // ---- advec_mom x, node row r
+      const double nf = 0.25 * (mA_m + mA + mB_m + mB);
+      const double post = 0.25 * (mp_m + mp + mpl_m + mpl);
+      const double nfl = __shfl_up_sync(FULL, nf, 1);
+      const double pre = post - nfl + nf;
+      const double prer = __shfl_down_sync(FULL, pre, 1);
+      double mu = 0.0, mv = 0.0;
+      if (lane >= 1 && lane <= 29 && j <= nx + 1) {
+        int up, don, dw;
+        double nmp;
+        if (nf < 0.0) {
+          up = 2; don = 1; dw = 0; nmp = prer;
+        } else {
+          up = -1; don = 0; dw = 1; nmp = pre;
+        }
+        const double uu[3] = {uin[i + up], uin[i + don], uin[i + dw]};
+        const double vv[3] = {vin[i + up], vin[i + don], vin[i + dw]};
+        mom_flux2(dv, nf, nmp, uu, vv, c.dx, c.rdx, mu, mv);
+      }
+      const double mul = __shfl_up_sync(FULL, mu, 1);
+      const double mvl = __shfl_up_sync(FULL, mv, 1);
+      if (own && j >= 1 && j <= nx + 1) {
+        const double u = uin[i], v = vin[i];
+        double un, vn;
+        mom_update(dv, u, v, pre, post, mul, mu, mvl, mv, un, vn);
+        const bool near = ncol || near_wall_row(c, r);
+        store_at(c, uout, K_XVEL, j, r, i, near, un);
+        store_at(c, vout, K_YVEL, j, r, i, near, vn);
+      }
+    }
+    mA_m = mA; mB_m = mB; mp_m = mp; mpl_m = mpl; ro_m = ro;
+  }
+  return __any_sync(FULL, dv.bad);
+}
+
+template <int SWEEP>
+__global__ void LB_ADVX
+ks_advec_x(Chunk c, const double* __restrict__ rho, const double* __restrict__ en,
+           const double* __restrict__ fx, const double* __restrict__ fy,
+           const double* __restrict__ uin, const double* __restrict__ vin,
+           double* __restrict__ rho_out, double* __restrict__ en_out, double* __restrict__ uout,
+           double* __restrict__ vout, FixSlot fix) {
+  pdl_trigger();
+  pdl_wait();
+  const int lane = threadIdx.x & 31;
+  const int gw = blockIdx.x * (SB / 32) + (threadIdx.x >> 5);
+  const int k0 = blockIdx.y * XKS + 1, k1 = min(k0 + XKS, c.ny + 2);
+  if (advec_x_body<SWEEP, DivFast>(c, rho, en, fx, fy, uin, vin, rho_out, en_out, uout, vout, gw,
+                                   k0, k1, lane))
+    fix_push(fix, lane, gw, blockIdx.y);
+}
+
+template <int SWEEP>
+__global__ void __launch_bounds__(SB)
+kf_advec_x(Chunk c, const double* __restrict__ rho, const double* __restrict__ en,
+           const double* __restrict__ fx, const double* __restrict__ fy,
+           const double* __restrict__ uin, const double* __restrict__ vin,
+           double* __restrict__ rho_out, double* __restrict__ en_out, double* __restrict__ uout,
+           double* __restrict__ vout, FixSlot fix) {
+  pdl_trigger();
+  pdl_wait();
+  fix_loop(fix, XKS, c.ny + 2, [&](int gw, int k0, int k1, int lane, int) {
+    advec_x_body<SWEEP, DivIEEE>(c, rho, en, fx, fy, uin, vin, rho_out, en_out, uout, vout, gw,
+                                 k0, k1, lane);
   });
 }
 
