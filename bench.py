@@ -214,7 +214,9 @@ def main():
     if args.mesh:
         nx, ny = args.mesh
         px, py = cdist.chunk_grid(world, nx, ny)
-    deck = bm_deck(nx, ny, end_step=args.steps)
+    # square cells: the domain grows with the mesh (weak scaling stacks
+    # per-rank 3840^2 blocks along y)
+    deck = bm_deck(nx, ny, end_step=args.steps, ymax=10.0 * ny / nx)
     uid = cdist.share_unique_id(nccl_unique_id) if world > 1 else None
     stream = torch.cuda.Stream(dev)
     sim = Clover(deck, px=px, py=py, rank=rank, nranks=world, unique_id=uid, stream=stream)

@@ -9,10 +9,15 @@ import torch
 import torch.distributed as dist
 
 
-def chunk_grid(nranks: int, nx: int, ny: int) -> tuple[int, int]:
-    """px x py chunks for nranks ranks, one chunk per rank: the most square
-    chunks, splitting the longer axis first (the reference's
-    clover_decompose idea; 2 -> 1x2 on a square mesh)."""
+def chunk_grid(nranks: int, nx: int, ny: int, strips: bool = True) -> tuple[int, int]:
+    """px x py chunks for nranks ranks, one chunk per rank.  Default: y
+    strips (px = 1) while each strip keeps >= 16 rows, so every chunk has
+    both x walls and the fused x-sweep kernel applies (DESIGN.md 5);
+    otherwise, or with strips=False, the most square chunks, splitting the
+    longer axis first (the reference's clover_decompose idea; SURVEY 8(e):
+    2 -> 1x2 on a square mesh)."""
+    if strips and ny // nranks >= 16:
+        return 1, nranks
     best = None
     for px in range(1, nranks + 1):
         if nranks % px:
@@ -26,10 +31,9 @@ def chunk_grid(nranks: int, nx: int, ny: int) -> tuple[int, int]:
 
 
 def weak_mesh(nranks: int, per: int = 3840) -> tuple[int, int, int, int]:
-    """Reading A4: per-rank per^2 cells; global mesh and chunk grid."""
-    table = {1: (1, 1), 2: (2, 1), 4: (2, 2), 8: (4, 2)}
-    px, py = table.get(nranks, (nranks, 1))
-    return per * px, per * py, px, py
+    """Reading A4: per-rank per^2 cells, stacked along y (1 x nranks chunk
+    grid): global mesh per x (per * nranks) and the chunk grid."""
+    return per, per * nranks, 1, nranks
 
 
 def share_unique_id(make_id) -> bytes:
