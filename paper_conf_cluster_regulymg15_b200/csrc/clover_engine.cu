@@ -57,15 +57,22 @@ int fail(int code, const std::string& msg) {
 // Buffers of one chunk.  State A (time level 0), B (after the Lagrangian
 // phase), C (after the first advection sweep); reset_field is the
 // rotation C -> A performed by the second sweep writing into A.
+// Buffers are carved in enum order at one common stride, so A + q (the five
+// inputs of the Lagrangian phase, in the order of its staged rows LF_*) are
+// one 3D tensor {pitch, rows, 5} for the TMA.
 enum Buf {
   B_D0, B_E0, B_U0, B_V0,     // A
+  B_Q,
   B_D1, B_E1, B_U1, B_V1,     // B
   B_D2, B_E2, B_U2, B_V2,     // C
-  B_Q, B_FX, B_FY, B_MX, B_MY, B_SCR, NBUF
+  B_FX, B_FY, B_MX, B_MY, B_SCR, NBUF
 };
+static_assert(B_E0 == B_D0 + LF_E && B_U0 == B_D0 + LF_U && B_V0 == B_D0 + LF_V &&
+                  B_Q == B_D0 + LF_Q, "Lagrangian tensor order");
 
-const int kBufKind[NBUF] = {K_CELL, K_CELL, K_XVEL, K_YVEL, K_CELL, K_CELL, K_XVEL, K_YVEL,
-                            K_CELL, K_CELL, K_XVEL, K_YVEL, K_CELL, K_XFACE, K_YFACE,
+const int kBufKind[NBUF] = {K_CELL, K_CELL, K_XVEL, K_YVEL, K_CELL,
+                            K_CELL, K_CELL, K_XVEL, K_YVEL,
+                            K_CELL, K_CELL, K_XVEL, K_YVEL, K_XFACE, K_YFACE,
                             K_XFACE, K_YFACE, K_CELL};
 
 constexpr int64_t kAlign = 256;
@@ -78,6 +85,7 @@ struct ChunkState {
   double* partials;  // summary partials, ntx*nty*5
   int ntx, nty;
   FixSlot fix;       // warps to redo with IEEE division (clover_stream.cuh)
+  CUtensorMap tm_lag;  // d0 e0 u0 v0 q as one {pitch, rows, 5} fp64 tensor, box {LRW, 1, 5}
 };
 
 struct Layout {
@@ -129,6 +137,40 @@ int64_t fix_capacity(int nx, int ny) {
   return m;
 }
 int64_t fix_bytes(int nx, int ny) { return kAlign + align_up(fix_capacity(nx, ny) * 8, kAlign); }
+
+// cuTensorMapEncodeTiled through the runtime's driver entry point (no -lcuda).
+typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*,
+                                  const cuuint64_t*, const cuuint64_t*, const cuuint32_t*,
+                                  const cuuint32_t*, CUtensorMapInterleave, CUtensorMapSwizzle,
+                                  CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+EncodeTiledFn encode_tiled() {
+  static EncodeTiledFn fn = nullptr;
+  if (!fn) {
+    void* p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = (EncodeTiledFn)p;
+  }
+  return fn;
+}
+
+// d0 e0 u0 v0 q of one chunk as a 3D fp64 tensor {pitch, rows, 5} (buffer
+// stride fstride bytes); box {LRW, 1, 5} = one staged row of the Lagrangian
+// ring.  Out-of-range columns (the last warp strip) read as zeros.
+int encode_lagr_map(CUtensorMap* m, const double* base, int pitch, int rows, int64_t fstride) {
+  EncodeTiledFn fn = encode_tiled();
+  if (!fn) return fail(CLOVER_ERR_CUDA, "cuTensorMapEncodeTiled unavailable");
+  const cuuint64_t dims[3] = {(cuuint64_t)pitch, (cuuint64_t)rows, (cuuint64_t)LNF};
+  const cuuint64_t strides[2] = {(cuuint64_t)pitch * 8, (cuuint64_t)fstride};
+  const cuuint32_t box[3] = {(cuuint32_t)LRW, 1, (cuuint32_t)LNF};
+  const cuuint32_t es[3] = {1, 1, 1};
+  CUresult r = fn(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 3, (void*)base, dims, strides, box, es,
+                  CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                  CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return fail(CLOVER_ERR_CUDA, "cuTensorMapEncodeTiled failed: " + std::to_string((int)r));
+  return CLOVER_OK;
+}
 
 }  // namespace
 
@@ -503,13 +545,13 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
     cur_prof_id = P_LAGR;
     for (auto& cs : ctx->chunks) {
       const Chunk& c = cs.c;
-      launch_step(ks_lagrangian, grid_strip(c.nx, LW, c.ny, LKS), SB, st,
-          c, cs.buf[B_D0], cs.buf[B_E0], cs.buf[B_U0], cs.buf[B_V0], cs.buf[B_Q], cs.buf[B_D1],
-          cs.buf[B_E1], cs.buf[B_U1], cs.buf[B_V1], cs.buf[B_FX], cs.buf[B_FY], ctx->scal, cs.fix);
+      launch_step(ks_lagrangian, grid_strip(c.nx, LW, c.ny, LKS), SB, st, c, cs.tm_lag,
+          cs.buf[B_D1], cs.buf[B_E1], cs.buf[B_U1], cs.buf[B_V1], cs.buf[B_FX], cs.buf[B_FY],
+          ctx->scal, cs.fix);
       STEP_LAUNCH_CHECK();
-      launch_step(kf_lagrangian, FIX_BLOCKS, SB, st,
-          c, cs.buf[B_D0], cs.buf[B_E0], cs.buf[B_U0], cs.buf[B_V0], cs.buf[B_Q], cs.buf[B_D1],
-          cs.buf[B_E1], cs.buf[B_U1], cs.buf[B_V1], cs.buf[B_FX], cs.buf[B_FY], ctx->scal, cs.fix);
+      launch_step(kf_lagrangian, FIX_BLOCKS, SB, st, c, cs.tm_lag,
+          cs.buf[B_D1], cs.buf[B_E1], cs.buf[B_U1], cs.buf[B_V1], cs.buf[B_FX], cs.buf[B_FY],
+          ctx->scal, cs.fix);
       FIX_LAUNCH_CHECK();
     }
     int rc = exchange(ctx, {B_D1, B_E1, B_U1, B_V1, B_FX, B_FY});
@@ -982,6 +1024,11 @@ int clover_init(const clover_grid* grid, const clover_state* states, int32_t nst
     for (int b = 0; b < NBUF; ++b) {
       cs.buf[b] = (double*)p + (int64_t)ROW0 * c.pitch + COL0;
       p += align_up(fe * 8, kAlign);
+    }
+    {
+      int rc = encode_lagr_map(&cs.tm_lag, cs.buf[B_D0] - (int64_t)ROW0 * c.pitch - COL0, c.pitch,
+                               c.ny + 2 + 2 * HALO, align_up(fe * 8, kAlign));
+      if (rc) return bail(rc);
     }
     cs.ntx = (c.nx + ST - 1) / ST; cs.nty = (c.ny + ST - 1) / ST;
     cs.partials = (double*)p;

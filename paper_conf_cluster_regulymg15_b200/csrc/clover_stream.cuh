@@ -248,31 +248,39 @@ constexpr int LKS = CLOVER_LKS;  // rows per segment
 #ifndef CLOVER_TMA_RELEASE_FENCE  // proxy fence before refilling a slot (A/B: no measurable cost)
 #define CLOVER_TMA_RELEASE_FENCE 1
 #endif
-// TMA-staged variant: rows of d0, e0, q (cells) and u0, v0 (nodes) stream
-// through a per-warp LSTG-stage shared-memory ring filled by cp.async.bulk,
-// so the DRAM latency of row k+LSTG-1 overlaps the compute of row k.
-constexpr int LRW = 36;   // doubles per staged row segment (>= 34, 16-B multiple)
-constexpr int LSTG = 4;   // ring stages
-enum { LF_R, LF_E, LF_Q, LF_U, LF_V, LNF };
+#ifndef CLOVER_LSTG
+#define CLOVER_LSTG 6
+#endif
+// TMA-staged rows: one 3D tensor copy per mesh row brings the row segment of
+// all five inputs (the engine keeps d0, e0, u0, v0, q as consecutive,
+// equally spaced buffers: tensor dims {pitch, rows, field}) into a per-warp
+// LSTG-row shared-memory ring, so the DRAM latency of row k+LSTG-2 overlaps
+// the compute of row k.  Smem column t of a slot holds memory column
+// COL0 + J0 - 2 + t: lane l reads its own column at t = l+1 and both x
+// neighbours without shuffles.  Iteration k reads rows k-1, k and k+1 from
+// the ring (raw inputs are never carried in registers), then releases row
+// k-1's slot.
+constexpr int LSTG = CLOVER_LSTG;  // ring rows
+constexpr int LRW = 36;            // staged columns (>= 34, 16-B multiple)
+enum { LF_R, LF_E, LF_U, LF_V, LF_Q, LNF };  // = buffer order B_D0 B_E0 B_U0 B_V0 B_Q
+constexpr int LSLOT = 192;         // doubles per slot: LNF*LRW = 180 padded to 128 B
+constexpr unsigned LBYTES = LNF * LRW * 8;
+static_assert(LSLOT >= LNF * LRW && (LSLOT * 8) % 128 == 0, "slot");
+static_assert(LSTG >= 3, "ring");
 
 template <class D>
-__device__ __forceinline__ bool lagr_body(const Chunk& c, const double* __restrict__ d0,
-                                          const double* __restrict__ e0,
-                                          const double* __restrict__ u0,
-                                          const double* __restrict__ v0,
-                                          const double* __restrict__ q, double* __restrict__ d1,
-                                          double* __restrict__ e1, double* __restrict__ u1,
-                                          double* __restrict__ v1, double* __restrict__ fx,
-                                          double* __restrict__ fy,
+__device__ __forceinline__ bool lagr_body(const Chunk& c, const CUtensorMap* __restrict__ tm,
+                                          double* __restrict__ d1, double* __restrict__ e1,
+                                          double* __restrict__ u1, double* __restrict__ v1,
+                                          double* __restrict__ fx, double* __restrict__ fy,
                                           const StepScalars* __restrict__ s, int gw, int k0,
-                                          int k1, int lane, double (*ring)[LNF][LRW],
+                                          int k1, int lane, double* ring,
                                           unsigned long long* bars) {
   const int J0 = 1 + LW * gw;
   const int j = J0 - 1 + lane;
   if (J0 > c.nx) return false;  // whole warp beyond the chunk (rings are per warp)
   D dv;
   const double dt = s->dt, dx = c.dx, dy = c.dy;
-  const int P = c.pitch;
   const bool colok = j <= c.nx + 1;
   const bool ncol = near_wall_col(c, j);
   int src = lane;
@@ -280,24 +288,25 @@ __device__ __forceinline__ bool lagr_body(const Chunk& c, const double* __restri
   if (c.wr && j == c.nx + 1) src = lane - 1;
   const bool xwall_warp = __any_sync(FULL, src != lane);
 
-  // staged window: memory columns [mstart, mstart+ncopy), covering j-1..j+1
-  const int mstart = (COL0 + J0 - 1) & ~1;
-  int ncopy = ((COL0 + J0 + 31 - mstart + 1) + 1) & ~1;
-  if (mstart + ncopy > P) ncopy = P - mstart;
-  const int off = COL0 + j - mstart;  // smem index of column j
-  const unsigned bytes = (unsigned)ncopy * 8u;
-  const double* fields[LNF] = {d0, e0, q, u0, v0};
   const int r_first = k0 - 1, r_last = k1 + 1;  // staged rows
+  const int xcol = COL0 + J0 - 2;
+  auto slot_of = [&](int r) { return (unsigned)(r - r_first) % (unsigned)LSTG; };
   auto issue = [&](int r) {
-    const int rel = r - r_first, slot = rel % LSTG;
-    mbar_arrive_expect_tx(&bars[slot], bytes * LNF);
-#pragma unroll
-    for (int f = 0; f < LNF; ++f)
-      tma_load_1d(&ring[slot][f][0], fields[f] + (size_t)r * P + (mstart - COL0), bytes, &bars[slot]);
+    const unsigned sl = slot_of(r);
+    mbar_arrive_expect_tx(&bars[sl], LBYTES);
+    tma_load_3d(ring + sl * LSLOT, tm, xcol, ROW0 + r, 0, &bars[sl]);
   };
   auto wait_row = [&](int r) {
-    const int rel = r - r_first;
-    mbar_wait(&bars[rel % LSTG], (unsigned)((rel / LSTG) & 1));
+    const unsigned rel = (unsigned)(r - r_first);
+    mbar_wait(&bars[rel % LSTG], (rel / LSTG) & 1u);
+  };
+  auto row = [&](int r) -> const double* { return ring + slot_of(r) * LSLOT + lane + 1; };
+  // PdV predictor + EOS of the cell in row rc, node rows rc and rn (c.5)
+  auto predict = [&](const double* rc, const double* rn) -> double {
+    return pdv_predict_pressure(dv, rc[LF_R * LRW], rc[LF_E * LRW], rc[LF_Q * LRW],
+                                rc[LF_U * LRW], rn[LF_U * LRW], rc[LF_U * LRW + 1],
+                                rn[LF_U * LRW + 1], rc[LF_V * LRW], rc[LF_V * LRW + 1],
+                                rn[LF_V * LRW], rn[LF_V * LRW + 1], dx, dy, c.rvol, dt);
   };
   if (lane == 0) {
     for (int t = 0; t < LSTG; ++t) mbar_init(&bars[t], 1);
@@ -307,98 +316,100 @@ __device__ __forceinline__ bool lagr_body(const Chunk& c, const double* __restri
   }
   __syncwarp();
 
-  double r_m = 1.0, e_m = 0.0, q_m = 0.0, ph_m = 0.0;
-  double rl_m = 1.0, phl_m = 0.0, ql_m = 0.0;
-  double u0_m = 0.0, v0_m = 0.0, u0r_m = 0.0, v0r_m = 0.0;
-  double u1_m = 0.0, v1_m = 0.0;
-  wait_row(r_first);
-  for (int k = k0 - 1; k <= k1; ++k) {
-    wait_row(k + 1);
-    const double* rowc = &ring[(k - r_first) % LSTG][0][0];
-    const double* rown = &ring[(k + 1 - r_first) % LSTG][0][0];
-    const double u0_c = rowc[LF_U * LRW + off], v0_c = rowc[LF_V * LRW + off];
-    const double u0r_c = rowc[LF_U * LRW + off + 1], v0r_c = rowc[LF_V * LRW + off + 1];
-    double r = 1.0, e = 0.0, qq = 0.0, ph = 0.0;
-    if (colok) {
-      r = rowc[LF_R * LRW + off]; e = rowc[LF_E * LRW + off]; qq = rowc[LF_Q * LRW + off];
-      const double u0_n = rown[LF_U * LRW + off], v0_n = rown[LF_V * LRW + off];
-      const double u0r_n = rown[LF_U * LRW + off + 1], v0r_n = rown[LF_V * LRW + off + 1];
-      int kp = k;
-      if (c.wb && k == 0) kp = 1;
-      if (c.wt && k == c.ny + 1) kp = c.ny;
-      double pr_, pe_, pq_, ua, ub, uc, ud, va, vb, vc, vd;
-      if (kp == k) {
-        pr_ = r; pe_ = e; pq_ = qq;
-        ua = u0_c; ub = u0_n; uc = u0r_c; ud = u0r_n;
-        va = v0_c; vb = v0r_c; vc = v0_n; vd = v0r_n;
-      } else {
-        const int ip = idx(c, j, kp);
-        pr_ = d0[ip]; pe_ = e0[ip]; pq_ = q[ip];
-        ua = u0[ip]; ub = u0[ip + P]; uc = u0[ip + 1]; ud = u0[ip + P + 1];
-        va = v0[ip]; vb = v0[ip + 1]; vc = v0[ip + P]; vd = v0[ip + P + 1];
-      }
-      ph = pdv_predict_pressure(dv, pr_, pe_, pq_, ua, ub, uc, ud, va, vb, vc, vd, dx, dy, c.rvol, dt);
-    }
+  // row k0-1: half-step pressure only.  At a reflective bottom wall the
+  // ring row 0 takes the mirror of row 1 (update_halo{pressure}), which is
+  // the predictor evaluated on row 1's inputs.
+  double ph_m, phl_m;
+  {
+    const int kp = (c.wb && k0 == 1) ? 1 : k0 - 1;
+    for (int r = r_first; r <= kp + 1; ++r) wait_row(r);
+    double ph = 0.0;
+    if (colok) ph = predict(row(kp), row(kp + 1));
     if (xwall_warp) ph = __shfl_sync(FULL, ph, src);
-    const double rl = __shfl_up_sync(FULL, r, 1);
+    ph_m = ph;
+    phl_m = __shfl_up_sync(FULL, ph, 1);
+  }
+  double u1_m = 0.0, v1_m = 0.0, u1r_m = 0.0, v1r_m = 0.0;
+  for (int k = k0; k <= k1; ++k) {
+    wait_row(k + 1);
+    const double* rm = row(k - 1);
+    const double* rc = row(k);
+    double ph = 0.0;
+    if (c.wt && k == c.ny + 1)
+      ph = ph_m;  // reflective top: mirror of row ny
+    else if (colok)
+      ph = predict(rc, row(k + 1));
+    if (xwall_warp) ph = __shfl_sync(FULL, ph, src);
     const double phl = __shfl_up_sync(FULL, ph, 1);
-    const double ql = __shfl_up_sync(FULL, qq, 1);
 
+    // accelerate at node (j,k): cells (j-1,k-1), (j,k-1), (j,k), (j-1,k)
     double u1_c = 0.0, v1_c = 0.0;
-    if (k >= k0 && colok) {
-      const double rr[4] = {rl_m, r_m, r, rl};
+    if (colok) {
+      const double rr[4] = {rm[LF_R * LRW - 1], rm[LF_R * LRW], rc[LF_R * LRW], rc[LF_R * LRW - 1]};
       const double pp[4] = {phl_m, ph_m, ph, phl};
-      const double qv[4] = {ql_m, q_m, qq, ql};
-      accelerate_node(dv, rr, pp, qv, u0_c, v0_c, dx, dy, dt, u1_c, v1_c);
+      const double qv[4] = {rm[LF_Q * LRW - 1], rm[LF_Q * LRW], rc[LF_Q * LRW], rc[LF_Q * LRW - 1]};
+      accelerate_node(dv, rr, pp, qv, rc[LF_U * LRW], rc[LF_V * LRW], dx, dy, dt, u1_c, v1_c);
     }
     const double u1r_c = __shfl_down_sync(FULL, u1_c, 1);
     const double v1r_c = __shfl_down_sync(FULL, v1_c, 1);
-    const double u1r_m = __shfl_down_sync(FULL, u1_m, 1);
-    const double v1r_m = __shfl_down_sync(FULL, v1_m, 1);
 
+    // PdV corrector + flux_calc of cell (j,k-1)
     const int kc = k - 1;
     if (kc >= k0 && lane >= 1 && lane <= LW && j <= c.nx) {
+      const double u0_m = rm[LF_U * LRW], u0r_m = rm[LF_U * LRW + 1];
+      const double v0_m = rm[LF_V * LRW], v0r_m = rm[LF_V * LRW + 1];
+      const double u0_c = rc[LF_U * LRW], u0r_c = rc[LF_U * LRW + 1];
+      const double v0_c = rc[LF_V * LRW], v0r_c = rc[LF_V * LRW + 1];
       const double lsum = u0_m + u0_c + u1_m + u1_c;
       const double rsum = u0r_m + u0r_c + u1r_m + u1r_c;
       const double bsum = v0_m + v0r_m + v1_m + v1r_m;
       const double tsum = v0_c + v0r_c + v1_c + v1r_c;
       double ev, dvv;
-      pdv_correct(dv, r_m, e_m, ph_m, q_m, lsum, rsum, bsum, tsum, dx, dy, c.rvol, dt, ev, dvv);
+      pdv_correct(dv, rm[LF_R * LRW], rm[LF_E * LRW], ph_m, rm[LF_Q * LRW], lsum, rsum, bsum, tsum,
+                  dx, dy, c.rvol, dt, ev, dvv);
       const int ic = idx(c, j, kc);
-      const bool near = ncol || near_wall_row(c, kc);
-      store_at(c, e1, K_CELL, j, kc, ic, near, ev);
-      store_at(c, d1, K_CELL, j, kc, ic, near, dvv);
       const double cx = 0.25 * dt * dy, cy = 0.25 * dt * dx;
-      store_at(c, fx, K_XFACE, j, kc, ic, near, cx * lsum);
-      store_at(c, fy, K_YFACE, j, kc, ic, near, cy * bsum);
-      if (j == c.nx) store_field(c, fx, K_XFACE, j + 1, kc, cx * rsum);
-      if (kc == c.ny) store_field(c, fy, K_YFACE, j, kc + 1, cy * tsum);
-      store_at(c, u1, K_XVEL, j, kc, ic, near, u1_m);
-      store_at(c, v1, K_YVEL, j, kc, ic, near, v1_m);
-      if (j == c.nx) {
-        store_field(c, u1, K_XVEL, j + 1, kc, u1r_m);
-        store_field(c, v1, K_YVEL, j + 1, kc, v1r_m);
+      if (!(ncol || near_wall_row(c, kc))) {
+        e1[ic] = ev;
+        d1[ic] = dvv;
+        fx[ic] = cx * lsum;
+        fy[ic] = cy * bsum;
+        u1[ic] = u1_m;
+        v1[ic] = v1_m;
+      } else {
+        store_mirrored(c, e1, K_CELL, j, kc, ev);
+        store_mirrored(c, d1, K_CELL, j, kc, dvv);
+        store_mirrored(c, fx, K_XFACE, j, kc, cx * lsum);
+        store_mirrored(c, fy, K_YFACE, j, kc, cy * bsum);
+        store_mirrored(c, u1, K_XVEL, j, kc, u1_m);
+        store_mirrored(c, v1, K_YVEL, j, kc, v1_m);
       }
-      if (kc == c.ny) {
-        store_field(c, u1, K_XVEL, j, kc + 1, u1_c);
-        store_field(c, v1, K_YVEL, j, kc + 1, v1_c);
-      }
-      if (j == c.nx && kc == c.ny) {
-        store_field(c, u1, K_XVEL, j + 1, kc + 1, u1r_c);
-        store_field(c, v1, K_YVEL, j + 1, kc + 1, v1r_c);
+      if (j == c.nx || kc == c.ny) {
+        if (j == c.nx) {
+          store_field(c, fx, K_XFACE, j + 1, kc, cx * rsum);
+          store_field(c, u1, K_XVEL, j + 1, kc, u1r_m);
+          store_field(c, v1, K_YVEL, j + 1, kc, v1r_m);
+        }
+        if (kc == c.ny) {
+          store_field(c, fy, K_YFACE, j, kc + 1, cy * tsum);
+          store_field(c, u1, K_XVEL, j, kc + 1, u1_c);
+          store_field(c, v1, K_YVEL, j, kc + 1, v1_c);
+        }
+        if (j == c.nx && kc == c.ny) {
+          store_field(c, u1, K_XVEL, j + 1, kc + 1, u1r_c);
+          store_field(c, v1, K_YVEL, j + 1, kc + 1, v1r_c);
+        }
       }
     }
-    r_m = r; e_m = e; q_m = qq; ph_m = ph;
-    rl_m = rl; phl_m = phl; ql_m = ql;
-    u0_m = u0_c; v0_m = v0_c; u0r_m = u0r_c; v0r_m = v0r_c;
-    u1_m = u1_c; v1_m = v1_c;
-    // row k is consumed (every value read from its slot is already in
-    // registers and used): refill its slot with row k+LSTG
+    ph_m = ph; phl_m = phl;
+    u1_m = u1_c; v1_m = v1_c; u1r_m = u1r_c; v1r_m = v1r_c;
+    // row k-1 is consumed (rows k, k+1 are still read next iteration):
+    // refill its slot with row k-1+LSTG
 #if CLOVER_TMA_RELEASE_FENCE
     fence_proxy_async();
 #endif
     __syncwarp();
-    if (lane == 0 && k + LSTG <= r_last) issue(k + LSTG);
+    if (lane == 0 && k - 1 + LSTG <= r_last) issue(k - 1 + LSTG);
   }
   __syncwarp();
   if (lane == 0)
@@ -408,37 +419,32 @@ __device__ __forceinline__ bool lagr_body(const Chunk& c, const double* __restri
 }
 
 __global__ void LB_HEAVY
-ks_lagrangian(Chunk c, const double* __restrict__ d0, const double* __restrict__ e0,
-              const double* __restrict__ u0, const double* __restrict__ v0,
-              const double* __restrict__ q, double* __restrict__ d1, double* __restrict__ e1,
-              double* __restrict__ u1, double* __restrict__ v1, double* __restrict__ fx,
-              double* __restrict__ fy, const StepScalars* __restrict__ s, FixSlot fix) {
+ks_lagrangian(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__ d1,
+              double* __restrict__ e1, double* __restrict__ u1, double* __restrict__ v1,
+              double* __restrict__ fx, double* __restrict__ fy, const StepScalars* __restrict__ s,
+              FixSlot fix) {
   pdl_trigger();
   pdl_wait();
-  __shared__ __align__(128) double ring[SB / 32][LSTG][LNF][LRW];
+  __shared__ __align__(128) double ring[SB / 32][LSTG * LSLOT];
   __shared__ __align__(8) unsigned long long bars[SB / 32][LSTG];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const int gw = blockIdx.x * (SB / 32) + w;
   const int k0 = blockIdx.y * LKS + 1, k1 = min(k0 + LKS, c.ny + 1);
-  if (lagr_body<DivFast>(c, d0, e0, u0, v0, q, d1, e1, u1, v1, fx, fy, s, gw, k0, k1, lane,
-                         ring[w], bars[w])) {
+  if (lagr_body<DivFast>(c, &tm, d1, e1, u1, v1, fx, fy, s, gw, k0, k1, lane, ring[w], bars[w]))
     fix_push(fix, lane, gw, blockIdx.y);
-  }
 }
 
 __global__ void __launch_bounds__(SB)
-kf_lagrangian(Chunk c, const double* __restrict__ d0, const double* __restrict__ e0,
-              const double* __restrict__ u0, const double* __restrict__ v0,
-              const double* __restrict__ q, double* __restrict__ d1, double* __restrict__ e1,
-              double* __restrict__ u1, double* __restrict__ v1, double* __restrict__ fx,
-              double* __restrict__ fy, const StepScalars* __restrict__ s, FixSlot fix) {
+kf_lagrangian(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__ d1,
+              double* __restrict__ e1, double* __restrict__ u1, double* __restrict__ v1,
+              double* __restrict__ fx, double* __restrict__ fy, const StepScalars* __restrict__ s,
+              FixSlot fix) {
   pdl_trigger();
   pdl_wait();
-  __shared__ __align__(128) double ring[SB / 32][LSTG][LNF][LRW];
+  __shared__ __align__(128) double ring[SB / 32][LSTG * LSLOT];
   __shared__ __align__(8) unsigned long long bars[SB / 32][LSTG];
   fix_loop(fix, LKS, c.ny + 1, [&](int gw, int k0, int k1, int lane, int w) {
-    lagr_body<DivIEEE>(c, d0, e0, u0, v0, q, d1, e1, u1, v1, fx, fy, s, gw, k0, k1, lane, ring[w],
-                       bars[w]);
+    lagr_body<DivIEEE>(c, &tm, d1, e1, u1, v1, fx, fy, s, gw, k0, k1, lane, ring[w], bars[w]);
   });
 }
 // (a register-only Lagrangian variant was measured 3% slower; see git history)

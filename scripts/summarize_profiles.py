@@ -22,7 +22,8 @@ def short(name):
     for a, b in (("ks_advec_cell_x<1>", "k_advec_cell_x<1>"), ("ks_advec_cell_x<2>", "k_advec_cell_x<2>"),
                  ("ks_advec_cell_y<1>", "k_advec_cell_y<1>"), ("ks_advec_cell_y<2>", "k_advec_cell_y<2>"),
                  ("ks_advec_mom_x<1>", "k_advec_mom_x<1>"), ("ks_advec_mom_x<2>", "k_advec_mom_x<2>"),
-                 ("ks_advec_mom_y<1>", "k_advec_mom_y<1>"), ("ks_advec_mom_y<2>", "k_advec_mom_y<2>")):
+                 ("ks_advec_mom_y<1>", "k_advec_mom_y<1>"), ("ks_advec_mom_y<2>", "k_advec_mom_y<2>"),
+                 ("ks_advec_x<1>", "k_advec_x<1>"), ("ks_advec_x<2>", "k_advec_x<2>")):
         if n.startswith(a):
             return b
     return NAMES.get(n, n)

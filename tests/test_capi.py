@@ -75,10 +75,10 @@ def test_sass_is_sm100a_and_has_no_cpu_fallback():
     sass = subprocess.run(["cuobjdump", "-sass", lib], capture_output=True, text=True).stdout
     for k in ("ks_visc_dt", "ks_lagrangian", "ks_advec_cell_x", "ks_advec_mom_y", "k_dt_finalize"):
         assert k in sass
-    # the Lagrangian kernel stages rows with the TMA bulk-copy engine
+    # the Lagrangian kernel stages rows with TMA tensor copies (3D: row x field)
     lag = sass[sass.index("Function : _ZN6clover13ks_lagrangian"):]
     lag = lag[:lag.index("Function :", 10)] if "Function :" in lag[10:] else lag
-    assert "UBLKCP" in lag and "SYNCS" in lag
+    assert "UTMALDG.3D" in lag and "SYNCS" in lag
 
 
 def test_product_package_does_not_touch_the_oracle():
