@@ -67,6 +67,8 @@ enum Buf {
   B_D2, B_E2, B_U2, B_V2,     // C
   B_FX, B_FY, B_MX, B_MY, B_SCR, NBUF
 };
+static_assert(B_E0 == B_D0 + VF_E && B_U0 == B_D0 + VF_U && B_V0 == B_D0 + VF_V,
+              "visc tensor order");
 static_assert(B_E0 == B_D0 + LF_E && B_U0 == B_D0 + LF_U && B_V0 == B_D0 + LF_V &&
                   B_Q == B_D0 + LF_Q, "Lagrangian tensor order");
 
@@ -85,7 +87,8 @@ struct ChunkState {
   double* partials;  // summary partials, ntx*nty*5
   int ntx, nty;
   FixSlot fix;       // warps to redo with IEEE division (clover_stream.cuh)
-  CUtensorMap tm_lag;  // d0 e0 u0 v0 q as one {pitch, rows, 5} fp64 tensor, box {LRW, 1, 5}
+  CUtensorMap tm_lag;   // d0 e0 u0 v0 q as one {pitch, rows, 5} fp64 tensor, box {LRW, 1, 5}
+  CUtensorMap tm_visc;  // d0 e0 u0 v0 as {pitch, rows, 4}, box {VRW, 1, 4}
 };
 
 struct Layout {
@@ -155,15 +158,17 @@ EncodeTiledFn encode_tiled() {
   return fn;
 }
 
-// d0 e0 u0 v0 q of one chunk as a 3D fp64 tensor {pitch, rows, 5} (buffer
-// stride fstride bytes); box {LRW, 1, 5} = one staged row of the Lagrangian
-// ring.  Out-of-range columns (the last warp strip) read as zeros.
-int encode_lagr_map(CUtensorMap* m, const double* base, int pitch, int rows, int64_t fstride) {
+// nf consecutive buffers of one chunk from `base` as a 3D fp64 tensor
+// {pitch, rows, nf} (buffer stride fstride bytes); box {boxw, 1, nf} = one
+// staged row of a kernel's ring.  Out-of-range columns (the last warp strip)
+// read as zeros.
+int encode_rows_map(CUtensorMap* m, const double* base, int pitch, int rows, int64_t fstride,
+                    int nf, int boxw) {
   EncodeTiledFn fn = encode_tiled();
   if (!fn) return fail(CLOVER_ERR_CUDA, "cuTensorMapEncodeTiled unavailable");
-  const cuuint64_t dims[3] = {(cuuint64_t)pitch, (cuuint64_t)rows, (cuuint64_t)LNF};
+  const cuuint64_t dims[3] = {(cuuint64_t)pitch, (cuuint64_t)rows, (cuuint64_t)nf};
   const cuuint64_t strides[2] = {(cuuint64_t)pitch * 8, (cuuint64_t)fstride};
-  const cuuint32_t box[3] = {(cuuint32_t)LRW, 1, (cuuint32_t)LNF};
+  const cuuint32_t box[3] = {(cuuint32_t)boxw, 1, (cuuint32_t)nf};
   const cuuint32_t es[3] = {1, 1, 1};
   CUresult r = fn(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 3, (void*)base, dims, strides, box, es,
                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
@@ -520,11 +525,11 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
   if (nphase >= 1) {
     for (auto& cs : ctx->chunks) {
       const Chunk& c = cs.c;
-      launch_step(ks_visc_dt, grid_cols(c.nx, c.ny, VKS), SB, st, c, cs.buf[B_D0], cs.buf[B_E0],
-                  cs.buf[B_U0], cs.buf[B_V0], cs.buf[B_Q], ctx->scal, ctx->dtp, cs.fix);
+      launch_step(ks_visc_dt, grid_cols(c.nx, c.ny, VKS), SB, st, c, cs.tm_visc, cs.buf[B_Q],
+                  ctx->scal, ctx->dtp, cs.fix);
       STEP_LAUNCH_CHECK();
-      launch_step(kf_visc_dt, FIX_BLOCKS, SB, st, c, cs.buf[B_D0], cs.buf[B_E0], cs.buf[B_U0],
-                  cs.buf[B_V0], cs.buf[B_Q], ctx->scal, ctx->dtp, cs.fix);
+      launch_step(kf_visc_dt, FIX_BLOCKS, SB, st, c, cs.tm_visc, cs.buf[B_Q], ctx->scal, ctx->dtp,
+                  cs.fix);
       FIX_LAUNCH_CHECK();
     }
     int rc = exchange(ctx, {B_Q});
@@ -1026,8 +1031,10 @@ int clover_init(const clover_grid* grid, const clover_state* states, int32_t nst
       p += align_up(fe * 8, kAlign);
     }
     {
-      int rc = encode_lagr_map(&cs.tm_lag, cs.buf[B_D0] - (int64_t)ROW0 * c.pitch - COL0, c.pitch,
-                               c.ny + 2 + 2 * HALO, align_up(fe * 8, kAlign));
+      const double* base = cs.buf[B_D0] - (int64_t)ROW0 * c.pitch - COL0;
+      const int rows = c.ny + 2 + 2 * HALO;
+      int rc = encode_rows_map(&cs.tm_lag, base, c.pitch, rows, align_up(fe * 8, kAlign), LNF, LRW);
+      if (!rc) rc = encode_rows_map(&cs.tm_visc, base, c.pitch, rows, align_up(fe * 8, kAlign), VNF, VRW);
       if (rc) return bail(rc);
     }
     cs.ntx = (c.nx + ST - 1) / ST; cs.nty = (c.ny + ST - 1) / ST;

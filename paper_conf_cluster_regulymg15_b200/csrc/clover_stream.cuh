@@ -103,6 +103,10 @@ constexpr int SB = CLOVER_SB;  // threads per block
 #define CLOVER_MKS_Y 8
 #endif
 
+#ifndef CLOVER_TMA_RELEASE_FENCE  // proxy fence before refilling a slot (A/B: no measurable cost)
+#define CLOVER_TMA_RELEASE_FENCE 1
+#endif
+
 // ---------------------------------------------------------------- fix lists
 // hdr[0] = number of entries, hdr[1] = finished fixup blocks, hdr[2] =
 // entries fixed so far (debug counter); e[] = (global
@@ -145,70 +149,125 @@ __device__ __forceinline__ void fix_loop(FixSlot f, int ks, int lim, Run&& run) 
 constexpr int FIX_BLOCKS = 148;  // fixup grid (one block per SM)
 
 // ================================================================ visc_dt
-// Column j = block*128 + tid + 1, rows [k0, k0+VKS).  Rolling: pressure of
-// the row below, density/energy of the row above, the 4 node velocities.
+// Warp w of the grid owns columns j = 32*w + lane + 1 over rows [k0, k0+VKS).
+// Rows of d0, e0, u0, v0 stream through a per-warp VSTG-row shared-memory
+// ring, one 3D TMA tensor copy per row (the four fields are consecutive
+// equally spaced buffers); smem column t of a slot holds memory column
+// COL0 - 1 + 32*w + t, so lane l reads its column at t = l+2 and both x
+// neighbours.  Iteration k reads rows k and k+1 (the pressures of rows k-1
+// and k are carried), then releases row k.  The box starts on an even
+// column: a tensor copy of fp64 rows must start 16-B aligned in global
+// memory (an odd start column faults with an illegal instruction on B200;
+// scripts/tma_probe.cu).
 constexpr int VKS = CLOVER_VKS;
+#ifndef CLOVER_VSTG
+#define CLOVER_VSTG 4
+#endif
+constexpr int VSTG = CLOVER_VSTG;
+constexpr int VRW = 36;
+enum { VF_R, VF_E, VF_U, VF_V, VNF };  // = buffer order B_D0 B_E0 B_U0 B_V0
+constexpr int VSLOT = VNF * VRW;       // 1152 B: a multiple of 128 B
+constexpr unsigned VBYTES = VNF * VRW * 8;
+static_assert((VSLOT * 8) % 128 == 0 && VSTG >= 2, "visc ring");
+static_assert(COL0 % 2 == 1, "visc ring box starts on an even (16-B aligned) column");
 
 // Warp segment: columns j = 32*gw + lane + 1, rows [k0, k1).
-// Returns whether any lane flagged; dtw = the warp's dt minimum (lane 0).
+// Returns whether any lane flagged; dtw = the warp's dt minimum (all lanes).
 template <class D>
-__device__ __forceinline__ bool visc_body(const Chunk& c, const double* __restrict__ d0,
-                                          const double* __restrict__ e0,
-                                          const double* __restrict__ u0,
-                                          const double* __restrict__ v0, double* __restrict__ q,
-                                          const DtParams& prm, int gw, int k0, int k1, int lane,
-                                          double& dtw) {
+__device__ __forceinline__ bool visc_body(const Chunk& c, const CUtensorMap* __restrict__ tm,
+                                          double* __restrict__ q, const DtParams& prm, int gw,
+                                          int k0, int k1, int lane, double* ring,
+                                          unsigned long long* bars, double& dtw) {
   const int j = gw * 32 + lane + 1;
   double dtl = G_BIG;
   D dv;
-  if (j <= c.nx) {
-    const int P = c.pitch;
-    const bool ncol = near_wall_col(c, j);
-    int i = idx(c, j, k0);
-    double pcm = eos_pressure(d0[i - P], e0[i - P]);
-    double rho = d0[i], ein = e0[i];
-    double pc = eos_pressure(rho, ein);
-    double ua = u0[i], ub = u0[i + 1], va = v0[i], vb = v0[i + 1];
-    DtAcc acc;
-    STREAM_LOOP
-    for (int k = k0; k < k1; ++k, i += P) {
-      const double rhon = d0[i + P], en = e0[i + P];
+  const int r_first = k0 - 1, r_last = k1;
+  const int xcol = COL0 - 1 + gw * 32;  // even (COL0 = 15)
+  auto slot_of = [&](int r) { return (unsigned)(r - r_first) % (unsigned)VSTG; };
+  auto issue = [&](int r) {
+    const unsigned sl = slot_of(r);
+    mbar_arrive_expect_tx(&bars[sl], VBYTES);
+    tma_load_3d(ring + sl * VSLOT, tm, xcol, ROW0 + r, 0, &bars[sl]);
+  };
+  auto wait_row = [&](int r) {
+    const unsigned rel = (unsigned)(r - r_first);
+    mbar_wait(&bars[rel % VSTG], (rel / VSTG) & 1u);
+  };
+  auto row = [&](int r) -> const double* { return ring + slot_of(r) * VSLOT + lane + 2; };
+  if (lane == 0) {
+    for (int t = 0; t < VSTG; ++t) mbar_init(&bars[t], 1);
+    fence_mbar_init();
+    fence_proxy_async();
+    for (int r = r_first; r < r_first + VSTG && r <= r_last; ++r) issue(r);
+  }
+  __syncwarp();
+  const bool ncol = near_wall_col(c, j);
+  wait_row(r_first);
+  wait_row(k0);
+  double pcm = eos_pressure(row(r_first)[VF_R * VRW], row(r_first)[VF_E * VRW]);  // p(k-1)
+  double pc = eos_pressure(row(k0)[VF_R * VRW], row(k0)[VF_E * VRW]);            // p(k)
+#if CLOVER_TMA_RELEASE_FENCE
+  fence_proxy_async();
+#endif
+  __syncwarp();
+  if (lane == 0 && r_first + VSTG <= r_last) issue(r_first + VSTG);  // row k0-1 is consumed
+  DtAcc acc;
+  int i = idx(c, j, k0);
+  for (int k = k0; k < k1; ++k, i += c.pitch) {
+    wait_row(k + 1);
+    const double* rc = row(k);
+    const double* rn = row(k + 1);
+    if (j <= c.nx) {
       ViscIn I;
-      I.rho = rho; I.e = ein;
+      I.rho = rc[VF_R * VRW]; I.e = rc[VF_E * VRW];
       I.pb = pcm;
-      I.pt = eos_pressure(rhon, en);
-      I.pl = eos_pressure(d0[i - 1], e0[i - 1]);
-      I.pr = eos_pressure(d0[i + 1], e0[i + 1]);
-      const double uc = u0[i + P], ud = u0[i + P + 1], vc = v0[i + P], vd = v0[i + P + 1];
-      I.u00 = ua; I.u10 = ub; I.u01 = uc; I.u11 = ud;
-      I.v00 = va; I.v10 = vb; I.v01 = vc; I.v11 = vd;
+      I.pt = eos_pressure(rn[VF_R * VRW], rn[VF_E * VRW]);
+      I.pl = eos_pressure(rc[VF_R * VRW - 1], rc[VF_E * VRW - 1]);
+      I.pr = eos_pressure(rc[VF_R * VRW + 1], rc[VF_E * VRW + 1]);
+      I.u00 = rc[VF_U * VRW]; I.u10 = rc[VF_U * VRW + 1];
+      I.u01 = rn[VF_U * VRW]; I.u11 = rn[VF_U * VRW + 1];
+      I.v00 = rc[VF_V * VRW]; I.v10 = rc[VF_V * VRW + 1];
+      I.v01 = rn[VF_V * VRW]; I.v11 = rn[VF_V * VRW + 1];
       double qv, cc;
       visc_cell(dv, I, c, qv, cc);
       acc.add(I, c, cc);
       store_at(c, q, K_CELL, j, k, i, ncol || near_wall_row(c, k), qv);
-      pcm = pc; pc = I.pt; rho = rhon; ein = en;
-      ua = uc; ub = ud; va = vc; vb = vd;
+      pcm = pc;
+      pc = I.pt;
     }
-    dtl = acc.dt(c, prm);
+    // row k is consumed (row k+1 is read again next iteration): refill
+#if CLOVER_TMA_RELEASE_FENCE
+    fence_proxy_async();
+#endif
+    __syncwarp();
+    if (lane == 0 && k + VSTG <= r_last) issue(k + VSTG);
   }
+  __syncwarp();
+  if (lane == 0)
+    for (int t = 0; t < VSTG; ++t) mbar_inval(&bars[t]);  // the ring may be reused (fixup)
+  __syncwarp();
+  if (j <= c.nx && k1 > k0) dtl = acc.dt(c, prm);
   for (int o = 16; o > 0; o >>= 1) dtl = fmin(dtl, __shfl_xor_sync(FULL, dtl, o));
   dtw = dtl;
   return __any_sync(FULL, dv.bad);
 }
 
 __global__ void LB_VISC
-ks_visc_dt(Chunk c, const double* __restrict__ d0, const double* __restrict__ e0,
-           const double* __restrict__ u0, const double* __restrict__ v0, double* __restrict__ q,
+ks_visc_dt(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__ q,
            StepScalars* __restrict__ s, DtParams prm, FixSlot fix) {
   pdl_trigger();
   pdl_wait();
+  __shared__ __align__(128) double ring[SB / 32][VSTG * VSLOT];
+  __shared__ __align__(8) unsigned long long bars[SB / 32][VSTG];
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const int gw = blockIdx.x * (SB / 32) + warp;
-  double dtw;
+  double dtw = G_BIG;
   const int k0 = blockIdx.y * VKS + 1, k1 = min(k0 + VKS, c.ny + 1);
-  if (visc_body<DivFast>(c, d0, e0, u0, v0, q, prm, gw, k0, k1, lane, dtw)) {
-    fix_push(fix, lane, gw, blockIdx.y);
-    dtw = G_BIG;  // this warp's dt comes from the fixup
+  if (gw * 32 < c.nx) {
+    if (visc_body<DivFast>(c, &tm, q, prm, gw, k0, k1, lane, ring[warp], bars[warp], dtw)) {
+      fix_push(fix, lane, gw, blockIdx.y);
+      dtw = G_BIG;  // this warp's dt comes from the fixup
+    }
   }
   __shared__ double wmin[SB / 32];
   if (lane == 0) wmin[warp] = dtw;
@@ -221,14 +280,15 @@ ks_visc_dt(Chunk c, const double* __restrict__ d0, const double* __restrict__ e0
 }
 
 __global__ void __launch_bounds__(SB)
-kf_visc_dt(Chunk c, const double* __restrict__ d0, const double* __restrict__ e0,
-           const double* __restrict__ u0, const double* __restrict__ v0, double* __restrict__ q,
+kf_visc_dt(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__ q,
            StepScalars* __restrict__ s, DtParams prm, FixSlot fix) {
   pdl_trigger();
   pdl_wait();
-  fix_loop(fix, VKS, c.ny + 1, [&](int gw, int k0, int k1, int lane, int) {
+  __shared__ __align__(128) double ring[SB / 32][VSTG * VSLOT];
+  __shared__ __align__(8) unsigned long long bars[SB / 32][VSTG];
+  fix_loop(fix, VKS, c.ny + 1, [&](int gw, int k0, int k1, int lane, int w) {
     double dtw;
-    visc_body<DivIEEE>(c, d0, e0, u0, v0, q, prm, gw, k0, k1, lane, dtw);
+    visc_body<DivIEEE>(c, &tm, q, prm, gw, k0, k1, lane, ring[w], bars[w], dtw);
     if (lane == 0) atomicMin(&s->dt_slot, (unsigned long long)__double_as_longlong(dtw));
   });
 }
@@ -243,11 +303,9 @@ kf_visc_dt(Chunk c, const double* __restrict__ d0, const double* __restrict__ e0
 // (rows: recomputed from the mirrored row; columns: taken from the mirrored
 // lane), exactly the reference's update_halo{pressure} after the predictor.
 constexpr int LW = 30;   // owned columns per warp
+static_assert((COL0 - 1 + LW) % 2 == 0 && LW % 2 == 0, "Lagrangian ring box starts on an even column");
 constexpr int LKS = CLOVER_LKS;  // rows per segment
 
-#ifndef CLOVER_TMA_RELEASE_FENCE  // proxy fence before refilling a slot (A/B: no measurable cost)
-#define CLOVER_TMA_RELEASE_FENCE 1
-#endif
 #ifndef CLOVER_LSTG
 #define CLOVER_LSTG 6
 #endif
@@ -289,7 +347,7 @@ __device__ __forceinline__ bool lagr_body(const Chunk& c, const CUtensorMap* __r
   const bool xwall_warp = __any_sync(FULL, src != lane);
 
   const int r_first = k0 - 1, r_last = k1 + 1;  // staged rows
-  const int xcol = COL0 + J0 - 2;
+  const int xcol = COL0 + J0 - 2;  // = 14 + 30*gw: even, 16-B aligned (see visc_body)
   auto slot_of = [&](int r) { return (unsigned)(r - r_first) % (unsigned)LSTG; };
   auto issue = [&](int r) {
     const unsigned sl = slot_of(r);
