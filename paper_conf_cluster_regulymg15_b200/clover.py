@@ -32,7 +32,7 @@ GEOM = {"rectangle": 1, "circle": 2, "point": 3}
 KIND = {"cell": 0, "xvel": 1, "yvel": 2, "xface": 3, "yface": 4}
 # internal buffer ids (csrc/clover_engine.cu enum Buf) for debug reads
 BUF = {"d0": 0, "e0": 1, "u0": 2, "v0": 3, "q": 4, "d1": 5, "e1": 6, "u1": 7, "v1": 8,
-       "d2": 9, "e2": 10, "u2": 11, "v2": 12, "fx": 13, "fy": 14, "mx": 15,
+       "fy": 9, "fx": 10, "d2": 11, "e2": 12, "u2": 13, "v2": 14, "mx": 15,
        "my": 16, "scr": 17}
 EXPORTS = ["clover_workspace_bytes", "clover_nccl_unique_id", "clover_init", "clover_step",
            "clover_step_host", "clover_field_summary", "clover_get_clock", "clover_dt_history",

@@ -60,21 +60,30 @@ int fail(int code, const std::string& msg) {
 // Buffers are carved in enum order at one common stride, so A + q (the five
 // inputs of the Lagrangian phase, in the order of its staged rows LF_*) are
 // one 3D tensor {pitch, rows, 5} for the TMA.
+// The fused x sweeps read d1 e1 u1 v1 fy fx (sweep 1) and fx d2 e2 u2 v2
+// (sweep 2) as one tensor each, so B is followed by fy, fx, then C.
 enum Buf {
   B_D0, B_E0, B_U0, B_V0,     // A
   B_Q,
   B_D1, B_E1, B_U1, B_V1,     // B
+  B_FY, B_FX,
   B_D2, B_E2, B_U2, B_V2,     // C
-  B_FX, B_FY, B_MX, B_MY, B_SCR, NBUF
+  B_MX, B_MY, B_SCR, NBUF
 };
+static_assert(B_E1 == B_D1 + XF<1>::E && B_U1 == B_D1 + XF<1>::U && B_V1 == B_D1 + XF<1>::V &&
+                  B_FY == B_D1 + XF<1>::FY && B_FX == B_D1 + XF<1>::FX,
+              "fused x sweep 1 tensor order");
+static_assert(B_D2 == B_FX + XF<2>::R && B_E2 == B_FX + XF<2>::E && B_U2 == B_FX + XF<2>::U &&
+                  B_V2 == B_FX + XF<2>::V,
+              "fused x sweep 2 tensor order");
 static_assert(B_E0 == B_D0 + VF_E && B_U0 == B_D0 + VF_U && B_V0 == B_D0 + VF_V,
               "visc tensor order");
 static_assert(B_E0 == B_D0 + LF_E && B_U0 == B_D0 + LF_U && B_V0 == B_D0 + LF_V &&
                   B_Q == B_D0 + LF_Q, "Lagrangian tensor order");
 
 const int kBufKind[NBUF] = {K_CELL, K_CELL, K_XVEL, K_YVEL, K_CELL,
+                            K_CELL, K_CELL, K_XVEL, K_YVEL, K_YFACE, K_XFACE,
                             K_CELL, K_CELL, K_XVEL, K_YVEL,
-                            K_CELL, K_CELL, K_XVEL, K_YVEL, K_XFACE, K_YFACE,
                             K_XFACE, K_YFACE, K_CELL};
 
 constexpr int64_t kAlign = 256;
@@ -89,6 +98,8 @@ struct ChunkState {
   FixSlot fix;       // warps to redo with IEEE division (clover_stream.cuh)
   CUtensorMap tm_lag;   // d0 e0 u0 v0 q as one {pitch, rows, 5} fp64 tensor, box {LRW, 1, 5}
   CUtensorMap tm_visc;  // d0 e0 u0 v0 as {pitch, rows, 4}, box {VRW, 1, 4}
+  CUtensorMap tm_x1;    // d1 e1 u1 v1 fy fx, box {XRW, 1, 6} (fused x sweep 1)
+  CUtensorMap tm_x2;    // fx d2 e2 u2 v2, box {XRW, 1, 5} (fused x sweep 2)
 };
 
 struct Layout {
@@ -583,20 +594,18 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
           const double* fx = cs.buf[B_FX];
           const double* fy = cs.buf[B_FY];
           if (sweep == 1) {
-            launch_step(ks_advec_x<1>, g, SB, st, c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[uin],
-                        cs.buf[vin], cs.buf[rout], cs.buf[eout], cs.buf[uout], cs.buf[vout], cs.fix);
+            launch_step(ks_advec_x<1>, g, SB, st, c, cs.tm_x1, cs.buf[rout], cs.buf[eout],
+                        cs.buf[uout], cs.buf[vout], cs.fix);
             STEP_LAUNCH_CHECK();
-            launch_step(kf_advec_x<1>, FIX_BLOCKS, SB, st, c, cs.buf[rin], cs.buf[ein], fx, fy,
-                        cs.buf[uin], cs.buf[vin], cs.buf[rout], cs.buf[eout], cs.buf[uout],
-                        cs.buf[vout], cs.fix);
+            launch_step(kf_advec_x<1>, FIX_BLOCKS, SB, st, c, cs.tm_x1, cs.buf[rout], cs.buf[eout],
+                        cs.buf[uout], cs.buf[vout], cs.fix);
             FIX_LAUNCH_CHECK();
           } else {
-            launch_step(ks_advec_x<2>, g, SB, st, c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[uin],
-                        cs.buf[vin], cs.buf[rout], cs.buf[eout], cs.buf[uout], cs.buf[vout], cs.fix);
+            launch_step(ks_advec_x<2>, g, SB, st, c, cs.tm_x2, cs.buf[rout], cs.buf[eout],
+                        cs.buf[uout], cs.buf[vout], cs.fix);
             STEP_LAUNCH_CHECK();
-            launch_step(kf_advec_x<2>, FIX_BLOCKS, SB, st, c, cs.buf[rin], cs.buf[ein], fx, fy,
-                        cs.buf[uin], cs.buf[vin], cs.buf[rout], cs.buf[eout], cs.buf[uout],
-                        cs.buf[vout], cs.fix);
+            launch_step(kf_advec_x<2>, FIX_BLOCKS, SB, st, c, cs.tm_x2, cs.buf[rout], cs.buf[eout],
+                        cs.buf[uout], cs.buf[vout], cs.fix);
             FIX_LAUNCH_CHECK();
           }
         }
@@ -1034,7 +1043,12 @@ int clover_init(const clover_grid* grid, const clover_state* states, int32_t nst
       const double* base = cs.buf[B_D0] - (int64_t)ROW0 * c.pitch - COL0;
       const int rows = c.ny + 2 + 2 * HALO;
       int rc = encode_rows_map(&cs.tm_lag, base, c.pitch, rows, align_up(fe * 8, kAlign), LNF, LRW);
-      if (!rc) rc = encode_rows_map(&cs.tm_visc, base, c.pitch, rows, align_up(fe * 8, kAlign), VNF, VRW);
+      const int64_t fs = align_up(fe * 8, kAlign);
+      if (!rc) rc = encode_rows_map(&cs.tm_visc, base, c.pitch, rows, fs, VNF, VRW);
+      if (!rc) rc = encode_rows_map(&cs.tm_x1, base + (B_D1 - B_D0) * (fs / 8), c.pitch, rows, fs,
+                                    XF<1>::NF, XRW);
+      if (!rc) rc = encode_rows_map(&cs.tm_x2, base + (B_FX - B_D0) * (fs / 8), c.pitch, rows, fs,
+                                    XF<2>::NF, XRW);
       if (rc) return bail(rc);
     }
     cs.ntx = (c.nx + ST - 1) / ST; cs.nty = (c.ny + ST - 1) / ST;

@@ -825,28 +825,43 @@ kf_advec_mom_x(Chunk c, const double* __restrict__ rho, const double* __restrict
 // depth-2 input halos (bitwise what the neighbour computes).
 constexpr int XW = 28;
 #ifndef CLOVER_XKS
-#define CLOVER_XKS 8
+#define CLOVER_XKS 16
 #endif
 constexpr int XKS = CLOVER_XKS;
 
+// Rows of the inputs stream through a per-warp XSTG-row shared-memory ring,
+// one 3D TMA tensor copy per row.  The engine keeps the inputs of each sweep
+// as consecutive equally spaced buffers: sweep 1 reads d1 e1 u1 v1 fy fx,
+// sweep 2 reads fx d2 e2 u2 v2 (it never reads fy).  Smem column t of a slot
+// holds memory column COL0 + J0 - 4 + t (even: 16-B aligned); lane l reads
+// its column j = J0 - 2 + l at t = l + 2 and reaches t = l .. l+4.
+template <int SWEEP> struct XF;
+template <> struct XF<1> { enum { R = 0, E = 1, U = 2, V = 3, FY = 4, FX = 5, NF = 6 }; };
+template <> struct XF<2> { enum { FX = 0, R = 1, E = 2, U = 3, V = 4, NF = 5, FY = -1 }; };
+constexpr int XRW = 36;
+#ifndef CLOVER_XSTG
+#define CLOVER_XSTG 4
+#endif
+constexpr int XSTG = CLOVER_XSTG;
+template <int SWEEP>
+__host__ __device__ constexpr int xslot() { return (XF<SWEEP>::NF * XRW + 15) / 16 * 16; }  // 128-B multiple
+static_assert((COL0 + 1 - 4) % 2 == 0 && XW % 2 == 0, "fused x ring box starts on an even column");
+
 template <int SWEEP, class D>
-__device__ __forceinline__ bool advec_x_body(const Chunk& c, const double* __restrict__ rho,
-                                             const double* __restrict__ en,
-                                             const double* __restrict__ fx,
-                                             const double* __restrict__ fy,
-                                             const double* __restrict__ uin,
-                                             const double* __restrict__ vin,
+__device__ __forceinline__ bool advec_x_body(const Chunk& c, const CUtensorMap* __restrict__ tm,
                                              double* __restrict__ rho_out,
                                              double* __restrict__ en_out,
                                              double* __restrict__ uout,
                                              double* __restrict__ vout, int gw, int k0, int k1,
-                                             int lane) {
+                                             int lane, double* ring, unsigned long long* bars) {
+  using F = XF<SWEEP>;
+  constexpr int SL = xslot<SWEEP>();
+  constexpr unsigned BYTES = F::NF * XRW * 8;
   D dv;
   const int J0 = 1 + XW * gw;
   if (J0 > c.nx + 1) return false;
   const int j = J0 - 2 + lane;
   const double vol = c.dx * c.dy;
-  const int P = c.pitch;
   const int nx = c.nx;
   const bool faceok = j >= 1 && j <= nx + 1;  // faces computed here (others mirrored)
   const bool cellok = j >= 0 && j <= nx + 2;  // pre_vol inputs exist
@@ -862,140 +877,188 @@ __device__ __forceinline__ bool advec_x_body(const Chunk& c, const double* __res
   if (src_m < 0 || src_m > 31) src_m = lane;
   if (src_r < 0 || src_r > 31) src_r = lane;
   const bool xwall_warp = __any_sync(FULL, src_m != lane || src_r != lane);
-  auto pv_mom = [&](int i) -> double { return (SWEEP == 1) ? vol + fy[i + P] - fy[i] : vol; };
+
+  const int r_first = k0 - 1, r_last = k1;  // staged rows (fy of row r+1 is read at row r)
+  const int xcol = COL0 + J0 - 4;
+  auto slot_of = [&](int r) { return (unsigned)(r - r_first) % (unsigned)XSTG; };
+  auto issue = [&](int r) {
+    const unsigned sl = slot_of(r);
+    mbar_arrive_expect_tx(&bars[sl], BYTES);
+    tma_load_3d(ring + sl * SL, tm, xcol, ROW0 + r, 0, &bars[sl]);
+  };
+  auto wait_row = [&](int r) {
+    const unsigned rel = (unsigned)(r - r_first);
+    mbar_wait(&bars[rel % XSTG], (rel / XSTG) & 1u);
+  };
+  auto row = [&](int r) -> const double* { return ring + slot_of(r) * SL + lane + 2; };
+  // post-sweep cell volume of the node-mass term
+  auto pv_mom = [&](const double* rc, const double* rn) -> double {
+    if constexpr (SWEEP == 1) return vol + rn[F::FY * XRW] - rc[F::FY * XRW];
+    else return vol;
+  };
+  if (lane == 0) {
+    for (int t = 0; t < XSTG; ++t) mbar_init(&bars[t], 1);
+    fence_mbar_init();
+    fence_proxy_async();
+    for (int r = r_first; r < r_first + XSTG && r <= r_last; ++r) issue(r);
+  }
+  __syncwarp();
+  wait_row(r_first);
 
   double mA_m = 0.0, mp_m = 0.0, mB_m = 0.0, mpl_m = 0.0, ro_m = 0.0;
   for (int r = k0 - 1; r < k1; ++r) {
-    const int i = idx(c, j, r);
-    const bool mir_bot = c.wb && r == 0;
-    const bool mir_top = c.wt && r == c.ny + 1;
-    if (mir_bot) continue;  // synthesised from row 1 below
-    double mA = 0.0, ro = 0.0;
-    if (mir_top) {
-      // row ny+1 = mirror of row ny (already mirrored along x)
-      mA = mA_m; ro = ro_m;
-    } else {
-      // ---- advec_cell x, row r
-      double pv = 0.0, F = 0.0, m = 0.0, ef = 0.0, rr = 0.0, ee = 0.0, flo = 0.0, fhi = 0.0;
-      if (cellok) {
-        flo = fx[i]; fhi = fx[i + 1];
-        F = flo;
-        pv = (SWEEP == 1) ? vol + (fhi - flo + fy[i + P] - fy[i]) : vol + fhi - flo;
-        rr = rho[i]; ee = en[i];
-      }
-      double pvl = __shfl_up_sync(FULL, pv, 1);
-      if (faceok) {
-        if (lane == 0) {
-          const double fl = fx[i - 1];
-          pvl = (SWEEP == 1) ? vol + (flo - fl + fy[i - 1 + P] - fy[i - 1]) : vol + flo - fl;
+    wait_row(r + 1);
+    const bool mir_bot = c.wb && r == 0;  // synthesised from row 1 below
+    if (!mir_bot) {
+      const double* rc = row(r);
+      const double* rn = row(r + 1);
+      const int i = idx(c, j, r);
+      const bool mir_top = c.wt && r == c.ny + 1;
+      double mA = 0.0, ro = 0.0;
+      if (mir_top) {
+        // row ny+1 = mirror of row ny (already mirrored along x)
+        mA = mA_m; ro = ro_m;
+      } else {
+        // ---- advec_cell x, row r
+        double pv = 0.0, F = 0.0, m = 0.0, ef = 0.0, rr = 0.0, ee = 0.0, flo = 0.0, fhi = 0.0;
+        if (cellok) {
+          flo = rc[F::FX * XRW]; fhi = rc[F::FX * XRW + 1];
+          F = flo;
+          if constexpr (SWEEP == 1)
+            pv = vol + (fhi - flo + rn[F::FY * XRW] - rc[F::FY * XRW]);
+          else
+            pv = vol + fhi - flo;
+          rr = rc[F::R * XRW]; ee = rc[F::E * XRW];
         }
-        double ru, rd, rw, eu, ed, ew, pvd;
-        if (F > 0.0) {
-          ru = rho[i - 2]; rd = rho[i - 1]; rw = rr;
-          eu = en[i - 2]; ed = en[i - 1]; ew = ee;
-          pvd = pvl;
-        } else {
-          const int up = min(j + 1, nx + 2) - j;
-          ru = rho[i + up]; rd = rr; rw = rho[i - 1];
-          eu = en[i + up]; ed = ee; ew = en[i - 1];
-          pvd = pv;
+        double pvl = __shfl_up_sync(FULL, pv, 1);
+        if (faceok) {
+          if (lane == 0) {
+            const double fl = rc[F::FX * XRW - 1];
+            if constexpr (SWEEP == 1)
+              pvl = vol + (flo - fl + rn[F::FY * XRW - 1] - rc[F::FY * XRW - 1]);
+            else
+              pvl = vol + flo - fl;
+          }
+          double ru, rd, rw, eu, ed, ew, pvd;
+          if (F > 0.0) {
+            ru = rc[F::R * XRW - 2]; rd = rc[F::R * XRW - 1]; rw = rr;
+            eu = rc[F::E * XRW - 2]; ed = rc[F::E * XRW - 1]; ew = ee;
+            pvd = pvl;
+          } else {
+            const int up = min(j + 1, nx + 2) - j;
+            ru = rc[F::R * XRW + up]; rd = rr; rw = rc[F::R * XRW - 1];
+            eu = rc[F::E * XRW + up]; ed = ee; ew = rc[F::E * XRW - 1];
+            pvd = pv;
+          }
+          cell_face_flux(dv, F, pvd, ru, rd, rw, eu, ed, ew, m, ef);
         }
-        cell_face_flux(dv, F, pvd, ru, rd, rw, eu, ed, ew, m, ef);
+        const double mh = __shfl_down_sync(FULL, m, 1);
+        const double efh = __shfl_down_sync(FULL, ef, 1);
+        double eo = 0.0;
+        if (j >= 1 && j <= nx && lane < 31) {
+          cell_update(dv, rr, ee, pv, m, mh, ef, efh, flo, fhi, ro, eo);
+          if (own && r >= k0 && r <= c.ny) {
+            const bool near = ncol || near_wall_row(c, r);
+            store_at(c, rho_out, K_CELL, j, r, i, near, ro);
+            store_at(c, en_out, K_CELL, j, r, i, near, eo);
+          }
+        }
+        mA = m;
+        if (xwall_warp) {
+          const double ms = __shfl_sync(FULL, m, src_m);
+          const double rs = __shfl_sync(FULL, ro, src_r);
+          if (src_m != lane) mA = sgn_m * ms;
+          if (src_r != lane) ro = rs;
+        }
       }
-      const double mh = __shfl_down_sync(FULL, m, 1);
-      const double efh = __shfl_down_sync(FULL, ef, 1);
-      double eo = 0.0;
-      if (j >= 1 && j <= nx && lane < 31) {
-        cell_update(dv, rr, ee, pv, m, mh, ef, efh, flo, fhi, ro, eo);
-        if (own && r >= k0 && r <= c.ny) {
+      const double mB = __shfl_down_sync(FULL, mA, 1);
+      double mp = 0.0;
+      if (mpok) mp = ro * pv_mom(rc, rn);
+      const double mpl = __shfl_up_sync(FULL, mp, 1);
+      if (c.wb && r == 1) {
+        // row 0 = mirror of row 1: same mass fluxes and density, row-0 volumes
+        mA_m = mA; mB_m = mB;
+        mp_m = mpok ? ro * pv_mom(row(0), rc) : 0.0;
+        mpl_m = __shfl_up_sync(FULL, mp_m, 1);
+      }
+      if (r >= k0) {
+        // ---- advec_mom x, node row r
+        const double nf = 0.25 * (mA_m + mA + mB_m + mB);
+        const double post = 0.25 * (mp_m + mp + mpl_m + mpl);
+        const double nfl = __shfl_up_sync(FULL, nf, 1);
+        const double pre = post - nfl + nf;
+        const double prer = __shfl_down_sync(FULL, pre, 1);
+        double mu = 0.0, mv = 0.0;
+        if (lane >= 1 && lane <= 29 && j <= nx + 1) {
+          int up, don, dw;
+          double nmp;
+          if (nf < 0.0) {
+            up = 2; don = 1; dw = 0; nmp = prer;
+          } else {
+            up = -1; don = 0; dw = 1; nmp = pre;
+          }
+          const double uu[3] = {rc[F::U * XRW + up], rc[F::U * XRW + don], rc[F::U * XRW + dw]};
+          const double vv[3] = {rc[F::V * XRW + up], rc[F::V * XRW + don], rc[F::V * XRW + dw]};
+          mom_flux2(dv, nf, nmp, uu, vv, c.dx, c.rdx, mu, mv);
+        }
+        const double mul = __shfl_up_sync(FULL, mu, 1);
+        const double mvl = __shfl_up_sync(FULL, mv, 1);
+        if (own && j >= 1 && j <= nx + 1) {
+          const double u = rc[F::U * XRW], v = rc[F::V * XRW];
+          double un, vn;
+          mom_update(dv, u, v, pre, post, mul, mu, mvl, mv, un, vn);
           const bool near = ncol || near_wall_row(c, r);
-          store_at(c, rho_out, K_CELL, j, r, i, near, ro);
-          store_at(c, en_out, K_CELL, j, r, i, near, eo);
+          store_at(c, uout, K_XVEL, j, r, i, near, un);
+          store_at(c, vout, K_YVEL, j, r, i, near, vn);
         }
       }
-      mA = m;
-      if (xwall_warp) {
-        const double ms = __shfl_sync(FULL, m, src_m);
-        const double rs = __shfl_sync(FULL, ro, src_r);
-        if (src_m != lane) mA = sgn_m * ms;
-        if (src_r != lane) ro = rs;
-      }
+      mA_m = mA; mB_m = mB; mp_m = mp; mpl_m = mpl; ro_m = ro;
     }
-    const double mB = __shfl_down_sync(FULL, mA, 1);
-    double mp = 0.0;
-    if (mpok) mp = ro * pv_mom(i);
-    const double mpl = __shfl_up_sync(FULL, mp, 1);
-    if (c.wb && r == 1) {
-      // row 0 = mirror of row 1: same mass fluxes and density, row-0 volumes
-      mA_m = mA; mB_m = mB;
-      mp_m = mpok ? ro * pv_mom(i - P) : 0.0;
-      mpl_m = __shfl_up_sync(FULL, mp_m, 1);
+    // row r-1 is consumed (row 0 is read at r = 1): refill its slot
+    if (r > r_first) {
+#if CLOVER_TMA_RELEASE_FENCE
+      fence_proxy_async();
+#endif
+      __syncwarp();
+      if (lane == 0 && r - 1 + XSTG <= r_last) issue(r - 1 + XSTG);
     }
-    if (r >= k0) {
-      // ---- advec_mom x, node row r
-      const double nf = 0.25 * (mA_m + mA + mB_m + mB);
-      const double post = 0.25 * (mp_m + mp + mpl_m + mpl);
-      const double nfl = __shfl_up_sync(FULL, nf, 1);
-      const double pre = post - nfl + nf;
-      const double prer = __shfl_down_sync(FULL, pre, 1);
-      double mu = 0.0, mv = 0.0;
-      if (lane >= 1 && lane <= 29 && j <= nx + 1) {
-        int up, don, dw;
-        double nmp;
-        if (nf < 0.0) {
-          up = 2; don = 1; dw = 0; nmp = prer;
-        } else {
-          up = -1; don = 0; dw = 1; nmp = pre;
-        }
-        const double uu[3] = {uin[i + up], uin[i + don], uin[i + dw]};
-        const double vv[3] = {vin[i + up], vin[i + don], vin[i + dw]};
-        mom_flux2(dv, nf, nmp, uu, vv, c.dx, c.rdx, mu, mv);
-      }
-      const double mul = __shfl_up_sync(FULL, mu, 1);
-      const double mvl = __shfl_up_sync(FULL, mv, 1);
-      if (own && j >= 1 && j <= nx + 1) {
-        const double u = uin[i], v = vin[i];
-        double un, vn;
-        mom_update(dv, u, v, pre, post, mul, mu, mvl, mv, un, vn);
-        const bool near = ncol || near_wall_row(c, r);
-        store_at(c, uout, K_XVEL, j, r, i, near, un);
-        store_at(c, vout, K_YVEL, j, r, i, near, vn);
-      }
-    }
-    mA_m = mA; mB_m = mB; mp_m = mp; mpl_m = mpl; ro_m = ro;
   }
+  __syncwarp();
+  if (lane == 0)
+    for (int t = 0; t < XSTG; ++t) mbar_inval(&bars[t]);  // the ring may be reused (fixup)
+  __syncwarp();
   return __any_sync(FULL, dv.bad);
 }
 
 template <int SWEEP>
 __global__ void LB_ADVX
-ks_advec_x(Chunk c, const double* __restrict__ rho, const double* __restrict__ en,
-           const double* __restrict__ fx, const double* __restrict__ fy,
-           const double* __restrict__ uin, const double* __restrict__ vin,
-           double* __restrict__ rho_out, double* __restrict__ en_out, double* __restrict__ uout,
-           double* __restrict__ vout, FixSlot fix) {
+ks_advec_x(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__ rho_out,
+           double* __restrict__ en_out, double* __restrict__ uout, double* __restrict__ vout,
+           FixSlot fix) {
   pdl_trigger();
   pdl_wait();
-  const int lane = threadIdx.x & 31;
-  const int gw = blockIdx.x * (SB / 32) + (threadIdx.x >> 5);
+  __shared__ __align__(128) double ring[SB / 32][XSTG * xslot<SWEEP>()];
+  __shared__ __align__(8) unsigned long long bars[SB / 32][XSTG];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const int gw = blockIdx.x * (SB / 32) + w;
   const int k0 = blockIdx.y * XKS + 1, k1 = min(k0 + XKS, c.ny + 2);
-  if (advec_x_body<SWEEP, DivFast>(c, rho, en, fx, fy, uin, vin, rho_out, en_out, uout, vout, gw,
-                                   k0, k1, lane))
+  if (advec_x_body<SWEEP, DivFast>(c, &tm, rho_out, en_out, uout, vout, gw, k0, k1, lane, ring[w],
+                                   bars[w]))
     fix_push(fix, lane, gw, blockIdx.y);
 }
 
 template <int SWEEP>
 __global__ void __launch_bounds__(SB)
-kf_advec_x(Chunk c, const double* __restrict__ rho, const double* __restrict__ en,
-           const double* __restrict__ fx, const double* __restrict__ fy,
-           const double* __restrict__ uin, const double* __restrict__ vin,
-           double* __restrict__ rho_out, double* __restrict__ en_out, double* __restrict__ uout,
-           double* __restrict__ vout, FixSlot fix) {
+kf_advec_x(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__ rho_out,
+           double* __restrict__ en_out, double* __restrict__ uout, double* __restrict__ vout,
+           FixSlot fix) {
   pdl_trigger();
   pdl_wait();
-  fix_loop(fix, XKS, c.ny + 2, [&](int gw, int k0, int k1, int lane, int) {
-    advec_x_body<SWEEP, DivIEEE>(c, rho, en, fx, fy, uin, vin, rho_out, en_out, uout, vout, gw,
-                                 k0, k1, lane);
+  __shared__ __align__(128) double ring[SB / 32][XSTG * xslot<SWEEP>()];
+  __shared__ __align__(8) unsigned long long bars[SB / 32][XSTG];
+  fix_loop(fix, XKS, c.ny + 2, [&](int gw, int k0, int k1, int lane, int w) {
+    advec_x_body<SWEEP, DivIEEE>(c, &tm, rho_out, en_out, uout, vout, gw, k0, k1, lane, ring[w],
+                                 bars[w]);
   });
 }
 
