@@ -847,7 +847,10 @@ template <int SWEEP>
 __host__ __device__ constexpr int xslot() { return (XF<SWEEP>::NF * XRW + 15) / 16 * 16; }  // 128-B multiple
 static_assert((COL0 + 1 - 4) % 2 == 0 && XW % 2 == 0, "fused x ring box starts on an even column");
 
-template <int SWEEP, class D>
+// EDGE = false: a warp segment whose columns and rows are all at least
+// HALO+2 away from any wall or chunk edge (see x_interior): every lane
+// predicate is constant and no mirror logic runs.
+template <int SWEEP, class D, bool EDGE>
 __device__ __forceinline__ bool advec_x_body(const Chunk& c, const CUtensorMap* __restrict__ tm,
                                              double* __restrict__ rho_out,
                                              double* __restrict__ en_out,
@@ -863,20 +866,22 @@ __device__ __forceinline__ bool advec_x_body(const Chunk& c, const CUtensorMap* 
   const int j = J0 - 2 + lane;
   const double vol = c.dx * c.dy;
   const int nx = c.nx;
-  const bool faceok = j >= 1 && j <= nx + 1;  // faces computed here (others mirrored)
-  const bool cellok = j >= 0 && j <= nx + 2;  // pre_vol inputs exist
-  const bool mpok = j >= -1 && j <= nx + 2;   // node-mass columns
-  const bool ncol = near_wall_col(c, j);
+  const bool faceok = !EDGE || (j >= 1 && j <= nx + 1);  // faces computed here (others mirrored)
+  const bool cellok = !EDGE || (j >= 0 && j <= nx + 2);  // pre_vol inputs exist
+  const bool mpok = !EDGE || (j >= -1 && j <= nx + 2);   // node-mass columns
+  const bool ncol = EDGE && near_wall_col(c, j);
   const bool own = lane >= 2 && lane < 2 + XW;
   // mirror sources at the x walls (lanes of this warp, see header)
   int src_m = lane, src_r = lane;
   double sgn_m = 1.0;
-  if (j <= 0) { src_m = lane + 2 - 2 * j; src_r = lane + 1 - 2 * j; sgn_m = -1.0; }
-  if (j >= nx + 2) { src_m = lane + 2 * nx + 2 - 2 * j; sgn_m = -1.0; }
-  if (j >= nx + 1) src_r = lane + 2 * nx + 1 - 2 * j;
-  if (src_m < 0 || src_m > 31) src_m = lane;
-  if (src_r < 0 || src_r > 31) src_r = lane;
-  const bool xwall_warp = __any_sync(FULL, src_m != lane || src_r != lane);
+  if (EDGE) {
+    if (j <= 0) { src_m = lane + 2 - 2 * j; src_r = lane + 1 - 2 * j; sgn_m = -1.0; }
+    if (j >= nx + 2) { src_m = lane + 2 * nx + 2 - 2 * j; sgn_m = -1.0; }
+    if (j >= nx + 1) src_r = lane + 2 * nx + 1 - 2 * j;
+    if (src_m < 0 || src_m > 31) src_m = lane;
+    if (src_r < 0 || src_r > 31) src_r = lane;
+  }
+  const bool xwall_warp = EDGE && __any_sync(FULL, src_m != lane || src_r != lane);
 
   const int r_first = k0 - 1, r_last = k1;  // staged rows (fy of row r+1 is read at row r)
   const int xcol = COL0 + J0 - 4;
@@ -908,12 +913,12 @@ __device__ __forceinline__ bool advec_x_body(const Chunk& c, const CUtensorMap* 
   double mA_m = 0.0, mp_m = 0.0, mB_m = 0.0, mpl_m = 0.0, ro_m = 0.0;
   for (int r = k0 - 1; r < k1; ++r) {
     wait_row(r + 1);
-    const bool mir_bot = c.wb && r == 0;  // synthesised from row 1 below
+    const bool mir_bot = EDGE && c.wb && r == 0;  // synthesised from row 1 below
     if (!mir_bot) {
       const double* rc = row(r);
       const double* rn = row(r + 1);
       const int i = idx(c, j, r);
-      const bool mir_top = c.wt && r == c.ny + 1;
+      const bool mir_top = EDGE && c.wt && r == c.ny + 1;
       double mA = 0.0, ro = 0.0;
       if (mir_top) {
         // row ny+1 = mirror of row ny (already mirrored along x)
@@ -945,7 +950,7 @@ __device__ __forceinline__ bool advec_x_body(const Chunk& c, const CUtensorMap* 
             eu = rc[F::E * XRW - 2]; ed = rc[F::E * XRW - 1]; ew = ee;
             pvd = pvl;
           } else {
-            const int up = min(j + 1, nx + 2) - j;
+            const int up = EDGE ? min(j + 1, nx + 2) - j : 1;
             ru = rc[F::R * XRW + up]; rd = rr; rw = rc[F::R * XRW - 1];
             eu = rc[F::E * XRW + up]; ed = ee; ew = rc[F::E * XRW - 1];
             pvd = pv;
@@ -955,10 +960,10 @@ __device__ __forceinline__ bool advec_x_body(const Chunk& c, const CUtensorMap* 
         const double mh = __shfl_down_sync(FULL, m, 1);
         const double efh = __shfl_down_sync(FULL, ef, 1);
         double eo = 0.0;
-        if (j >= 1 && j <= nx && lane < 31) {
+        if ((!EDGE || (j >= 1 && j <= nx)) && lane < 31) {
           cell_update(dv, rr, ee, pv, m, mh, ef, efh, flo, fhi, ro, eo);
-          if (own && r >= k0 && r <= c.ny) {
-            const bool near = ncol || near_wall_row(c, r);
+          if (own && r >= k0 && (!EDGE || r <= c.ny)) {
+            const bool near = EDGE && (ncol || near_wall_row(c, r));
             store_at(c, rho_out, K_CELL, j, r, i, near, ro);
             store_at(c, en_out, K_CELL, j, r, i, near, eo);
           }
@@ -975,7 +980,7 @@ __device__ __forceinline__ bool advec_x_body(const Chunk& c, const CUtensorMap* 
       double mp = 0.0;
       if (mpok) mp = ro * pv_mom(rc, rn);
       const double mpl = __shfl_up_sync(FULL, mp, 1);
-      if (c.wb && r == 1) {
+      if (EDGE && c.wb && r == 1) {
         // row 0 = mirror of row 1: same mass fluxes and density, row-0 volumes
         mA_m = mA; mB_m = mB;
         mp_m = mpok ? ro * pv_mom(row(0), rc) : 0.0;
@@ -989,7 +994,7 @@ __device__ __forceinline__ bool advec_x_body(const Chunk& c, const CUtensorMap* 
         const double pre = post - nfl + nf;
         const double prer = __shfl_down_sync(FULL, pre, 1);
         double mu = 0.0, mv = 0.0;
-        if (lane >= 1 && lane <= 29 && j <= nx + 1) {
+        if (lane >= 1 && lane <= 29 && (!EDGE || j <= nx + 1)) {
           int up, don, dw;
           double nmp;
           if (nf < 0.0) {
@@ -1003,11 +1008,11 @@ __device__ __forceinline__ bool advec_x_body(const Chunk& c, const CUtensorMap* 
         }
         const double mul = __shfl_up_sync(FULL, mu, 1);
         const double mvl = __shfl_up_sync(FULL, mv, 1);
-        if (own && j >= 1 && j <= nx + 1) {
+        if (own && (!EDGE || (j >= 1 && j <= nx + 1))) {
           const double u = rc[F::U * XRW], v = rc[F::V * XRW];
           double un, vn;
           mom_update(dv, u, v, pre, post, mul, mu, mvl, mv, un, vn);
-          const bool near = ncol || near_wall_row(c, r);
+          const bool near = EDGE && (ncol || near_wall_row(c, r));
           store_at(c, uout, K_XVEL, j, r, i, near, un);
           store_at(c, vout, K_YVEL, j, r, i, near, vn);
         }
@@ -1030,6 +1035,30 @@ __device__ __forceinline__ bool advec_x_body(const Chunk& c, const CUtensorMap* 
   return __any_sync(FULL, dv.bad);
 }
 
+// A warp segment is interior when every lane column j = J0-2 .. J0+29 and
+// its stencil reach (j-2 .. j+2) lie in [HALO+2, nx-HALO-1] and every row
+// r = k0-1 .. k1 in [HALO+2, ny-HALO-1]: no wall mirror, halo row or
+// near-wall store can occur.
+__device__ __forceinline__ bool x_interior(const Chunk& c, int gw, int k0, int k1) {
+  const int J0 = 1 + XW * gw;
+  return J0 - 4 >= HALO + 2 && J0 + 31 <= c.nx - HALO - 1 && k0 - 1 >= HALO + 2 &&
+         k1 <= c.ny - HALO - 1;
+}
+
+template <int SWEEP, class D>
+__device__ __forceinline__ bool advec_x_seg(const Chunk& c, const CUtensorMap* __restrict__ tm,
+                                            double* __restrict__ rho_out,
+                                            double* __restrict__ en_out,
+                                            double* __restrict__ uout, double* __restrict__ vout,
+                                            int gw, int k0, int k1, int lane, double* ring,
+                                            unsigned long long* bars) {
+  if (x_interior(c, gw, k0, k1))
+    return advec_x_body<SWEEP, D, false>(c, tm, rho_out, en_out, uout, vout, gw, k0, k1, lane,
+                                         ring, bars);
+  return advec_x_body<SWEEP, D, true>(c, tm, rho_out, en_out, uout, vout, gw, k0, k1, lane, ring,
+                                      bars);
+}
+
 template <int SWEEP>
 __global__ void LB_ADVX
 ks_advec_x(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__ rho_out,
@@ -1042,7 +1071,7 @@ ks_advec_x(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const int gw = blockIdx.x * (SB / 32) + w;
   const int k0 = blockIdx.y * XKS + 1, k1 = min(k0 + XKS, c.ny + 2);
-  if (advec_x_body<SWEEP, DivFast>(c, &tm, rho_out, en_out, uout, vout, gw, k0, k1, lane, ring[w],
+  if (advec_x_seg<SWEEP, DivFast>(c, &tm, rho_out, en_out, uout, vout, gw, k0, k1, lane, ring[w],
                                    bars[w]))
     fix_push(fix, lane, gw, blockIdx.y);
 }
@@ -1057,7 +1086,7 @@ kf_advec_x(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__
   __shared__ __align__(128) double ring[SB / 32][XSTG * xslot<SWEEP>()];
   __shared__ __align__(8) unsigned long long bars[SB / 32][XSTG];
   fix_loop(fix, XKS, c.ny + 2, [&](int gw, int k0, int k1, int lane, int w) {
-    advec_x_body<SWEEP, DivIEEE>(c, &tm, rho_out, en_out, uout, vout, gw, k0, k1, lane, ring[w],
+    advec_x_seg<SWEEP, DivIEEE>(c, &tm, rho_out, en_out, uout, vout, gw, k0, k1, lane, ring[w],
                                  bars[w]);
   });
 }
