@@ -173,7 +173,9 @@ static_assert(COL0 % 2 == 1, "visc ring box starts on an even (16-B aligned) col
 
 // Warp segment: columns j = 32*gw + lane + 1, rows [k0, k1).
 // Returns whether any lane flagged; dtw = the warp's dt minimum (all lanes).
-template <class D>
+// EDGE = false: columns, their x neighbours and rows k0-1 .. k1 are at least
+// HALO+2 away from every wall and chunk edge (visc_interior).
+template <class D, bool EDGE>
 __device__ __forceinline__ bool visc_body(const Chunk& c, const CUtensorMap* __restrict__ tm,
                                           double* __restrict__ q, const DtParams& prm, int gw,
                                           int k0, int k1, int lane, double* ring,
@@ -201,7 +203,7 @@ __device__ __forceinline__ bool visc_body(const Chunk& c, const CUtensorMap* __r
     for (int r = r_first; r < r_first + VSTG && r <= r_last; ++r) issue(r);
   }
   __syncwarp();
-  const bool ncol = near_wall_col(c, j);
+  const bool ncol = EDGE && near_wall_col(c, j);
   wait_row(r_first);
   wait_row(k0);
   double pcm = eos_pressure(row(r_first)[VF_R * VRW], row(r_first)[VF_E * VRW]);  // p(k-1)
@@ -217,7 +219,7 @@ __device__ __forceinline__ bool visc_body(const Chunk& c, const CUtensorMap* __r
     wait_row(k + 1);
     const double* rc = row(k);
     const double* rn = row(k + 1);
-    if (j <= c.nx) {
+    if (!EDGE || j <= c.nx) {
       ViscIn I;
       I.rho = rc[VF_R * VRW]; I.e = rc[VF_E * VRW];
       I.pb = pcm;
@@ -231,7 +233,7 @@ __device__ __forceinline__ bool visc_body(const Chunk& c, const CUtensorMap* __r
       double qv, cc;
       visc_cell(dv, I, c, qv, cc);
       acc.add(I, c, cc);
-      store_at(c, q, K_CELL, j, k, i, ncol || near_wall_row(c, k), qv);
+      store_at(c, q, K_CELL, j, k, i, EDGE && (ncol || near_wall_row(c, k)), qv);
       pcm = pc;
       pc = I.pt;
     }
@@ -246,10 +248,25 @@ __device__ __forceinline__ bool visc_body(const Chunk& c, const CUtensorMap* __r
   if (lane == 0)
     for (int t = 0; t < VSTG; ++t) mbar_inval(&bars[t]);  // the ring may be reused (fixup)
   __syncwarp();
-  if (j <= c.nx && k1 > k0) dtl = acc.dt(c, prm);
+  if ((!EDGE || j <= c.nx) && k1 > k0) dtl = acc.dt(c, prm);
   for (int o = 16; o > 0; o >>= 1) dtl = fmin(dtl, __shfl_xor_sync(FULL, dtl, o));
   dtw = dtl;
   return __any_sync(FULL, dv.bad);
+}
+
+__device__ __forceinline__ bool visc_interior(const Chunk& c, int gw, int k0, int k1) {
+  return gw * 32 >= HALO + 2 && gw * 32 + 34 <= c.nx - HALO - 1 && k0 - 1 >= HALO + 2 &&
+         k1 <= c.ny - HALO - 1;
+}
+
+template <class D>
+__device__ __forceinline__ bool visc_seg(const Chunk& c, const CUtensorMap* __restrict__ tm,
+                                         double* __restrict__ q, const DtParams& prm, int gw,
+                                         int k0, int k1, int lane, double* ring,
+                                         unsigned long long* bars, double& dtw) {
+  if (visc_interior(c, gw, k0, k1))
+    return visc_body<D, false>(c, tm, q, prm, gw, k0, k1, lane, ring, bars, dtw);
+  return visc_body<D, true>(c, tm, q, prm, gw, k0, k1, lane, ring, bars, dtw);
 }
 
 __global__ void LB_VISC
@@ -264,7 +281,7 @@ ks_visc_dt(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__
   double dtw = G_BIG;
   const int k0 = blockIdx.y * VKS + 1, k1 = min(k0 + VKS, c.ny + 1);
   if (gw * 32 < c.nx) {
-    if (visc_body<DivFast>(c, &tm, q, prm, gw, k0, k1, lane, ring[warp], bars[warp], dtw)) {
+    if (visc_seg<DivFast>(c, &tm, q, prm, gw, k0, k1, lane, ring[warp], bars[warp], dtw)) {
       fix_push(fix, lane, gw, blockIdx.y);
       dtw = G_BIG;  // this warp's dt comes from the fixup
     }
@@ -288,7 +305,7 @@ kf_visc_dt(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__
   __shared__ __align__(8) unsigned long long bars[SB / 32][VSTG];
   fix_loop(fix, VKS, c.ny + 1, [&](int gw, int k0, int k1, int lane, int w) {
     double dtw;
-    visc_body<DivIEEE>(c, &tm, q, prm, gw, k0, k1, lane, ring[w], bars[w], dtw);
+    visc_seg<DivIEEE>(c, &tm, q, prm, gw, k0, k1, lane, ring[w], bars[w], dtw);
     if (lane == 0) atomicMin(&s->dt_slot, (unsigned long long)__double_as_longlong(dtw));
   });
 }
@@ -326,7 +343,10 @@ constexpr unsigned LBYTES = LNF * LRW * 8;
 static_assert(LSLOT >= LNF * LRW && (LSLOT * 8) % 128 == 0, "slot");
 static_assert(LSTG >= 3, "ring");
 
-template <class D>
+// EDGE = false: a warp segment whose stencil reach is at least HALO+2 away
+// from every wall and chunk edge (lagr_interior): constant lane predicates,
+// no wall rows, no mirrored or extra stores.
+template <class D, bool EDGE>
 __device__ __forceinline__ bool lagr_body(const Chunk& c, const CUtensorMap* __restrict__ tm,
                                           double* __restrict__ d1, double* __restrict__ e1,
                                           double* __restrict__ u1, double* __restrict__ v1,
@@ -339,12 +359,12 @@ __device__ __forceinline__ bool lagr_body(const Chunk& c, const CUtensorMap* __r
   if (J0 > c.nx) return false;  // whole warp beyond the chunk (rings are per warp)
   D dv;
   const double dt = s->dt, dx = c.dx, dy = c.dy;
-  const bool colok = j <= c.nx + 1;
-  const bool ncol = near_wall_col(c, j);
+  const bool colok = !EDGE || j <= c.nx + 1;
+  const bool ncol = EDGE && near_wall_col(c, j);
   int src = lane;
-  if (c.wl && j == 0) src = lane + 1;
-  if (c.wr && j == c.nx + 1) src = lane - 1;
-  const bool xwall_warp = __any_sync(FULL, src != lane);
+  if (EDGE && c.wl && j == 0) src = lane + 1;
+  if (EDGE && c.wr && j == c.nx + 1) src = lane - 1;
+  const bool xwall_warp = EDGE && __any_sync(FULL, src != lane);
 
   const int r_first = k0 - 1, r_last = k1 + 1;  // staged rows
   const int xcol = COL0 + J0 - 2;  // = 14 + 30*gw: even, 16-B aligned (see visc_body)
@@ -379,7 +399,7 @@ __device__ __forceinline__ bool lagr_body(const Chunk& c, const CUtensorMap* __r
   // the predictor evaluated on row 1's inputs.
   double ph_m, phl_m;
   {
-    const int kp = (c.wb && k0 == 1) ? 1 : k0 - 1;
+    const int kp = (EDGE && c.wb && k0 == 1) ? 1 : k0 - 1;
     for (int r = r_first; r <= kp + 1; ++r) wait_row(r);
     double ph = 0.0;
     if (colok) ph = predict(row(kp), row(kp + 1));
@@ -393,7 +413,7 @@ __device__ __forceinline__ bool lagr_body(const Chunk& c, const CUtensorMap* __r
     const double* rm = row(k - 1);
     const double* rc = row(k);
     double ph = 0.0;
-    if (c.wt && k == c.ny + 1)
+    if (EDGE && c.wt && k == c.ny + 1)
       ph = ph_m;  // reflective top: mirror of row ny
     else if (colok)
       ph = predict(rc, row(k + 1));
@@ -413,7 +433,7 @@ __device__ __forceinline__ bool lagr_body(const Chunk& c, const CUtensorMap* __r
 
     // PdV corrector + flux_calc of cell (j,k-1)
     const int kc = k - 1;
-    if (kc >= k0 && lane >= 1 && lane <= LW && j <= c.nx) {
+    if (kc >= k0 && lane >= 1 && lane <= LW && (!EDGE || j <= c.nx)) {
       const double u0_m = rm[LF_U * LRW], u0r_m = rm[LF_U * LRW + 1];
       const double v0_m = rm[LF_V * LRW], v0r_m = rm[LF_V * LRW + 1];
       const double u0_c = rc[LF_U * LRW], u0r_c = rc[LF_U * LRW + 1];
@@ -427,7 +447,7 @@ __device__ __forceinline__ bool lagr_body(const Chunk& c, const CUtensorMap* __r
                   dx, dy, c.rvol, dt, ev, dvv);
       const int ic = idx(c, j, kc);
       const double cx = 0.25 * dt * dy, cy = 0.25 * dt * dx;
-      if (!(ncol || near_wall_row(c, kc))) {
+      if (!EDGE || !(ncol || near_wall_row(c, kc))) {
         e1[ic] = ev;
         d1[ic] = dvv;
         fx[ic] = cx * lsum;
@@ -442,7 +462,7 @@ __device__ __forceinline__ bool lagr_body(const Chunk& c, const CUtensorMap* __r
         store_mirrored(c, u1, K_XVEL, j, kc, u1_m);
         store_mirrored(c, v1, K_YVEL, j, kc, v1_m);
       }
-      if (j == c.nx || kc == c.ny) {
+      if (EDGE && (j == c.nx || kc == c.ny)) {
         if (j == c.nx) {
           store_field(c, fx, K_XFACE, j + 1, kc, cx * rsum);
           store_field(c, u1, K_XVEL, j + 1, kc, u1r_m);
@@ -476,6 +496,24 @@ __device__ __forceinline__ bool lagr_body(const Chunk& c, const CUtensorMap* __r
   return __any_sync(FULL, dv.bad);
 }
 
+__device__ __forceinline__ bool lagr_interior(const Chunk& c, int gw, int k0, int k1) {
+  const int J0 = 1 + LW * gw;
+  return J0 - 2 >= HALO + 2 && J0 + 31 <= c.nx - HALO - 1 && k0 - 1 >= HALO + 2 &&
+         k1 + 1 <= c.ny - HALO - 1;
+}
+
+template <class D>
+__device__ __forceinline__ bool lagr_seg(const Chunk& c, const CUtensorMap* __restrict__ tm,
+                                         double* __restrict__ d1, double* __restrict__ e1,
+                                         double* __restrict__ u1, double* __restrict__ v1,
+                                         double* __restrict__ fx, double* __restrict__ fy,
+                                         const StepScalars* __restrict__ s, int gw, int k0, int k1,
+                                         int lane, double* ring, unsigned long long* bars) {
+  if (lagr_interior(c, gw, k0, k1))
+    return lagr_body<D, false>(c, tm, d1, e1, u1, v1, fx, fy, s, gw, k0, k1, lane, ring, bars);
+  return lagr_body<D, true>(c, tm, d1, e1, u1, v1, fx, fy, s, gw, k0, k1, lane, ring, bars);
+}
+
 __global__ void LB_HEAVY
 ks_lagrangian(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__ d1,
               double* __restrict__ e1, double* __restrict__ u1, double* __restrict__ v1,
@@ -488,7 +526,7 @@ ks_lagrangian(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restric
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const int gw = blockIdx.x * (SB / 32) + w;
   const int k0 = blockIdx.y * LKS + 1, k1 = min(k0 + LKS, c.ny + 1);
-  if (lagr_body<DivFast>(c, &tm, d1, e1, u1, v1, fx, fy, s, gw, k0, k1, lane, ring[w], bars[w]))
+  if (lagr_seg<DivFast>(c, &tm, d1, e1, u1, v1, fx, fy, s, gw, k0, k1, lane, ring[w], bars[w]))
     fix_push(fix, lane, gw, blockIdx.y);
 }
 
@@ -502,7 +540,7 @@ kf_lagrangian(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restric
   __shared__ __align__(128) double ring[SB / 32][LSTG * LSLOT];
   __shared__ __align__(8) unsigned long long bars[SB / 32][LSTG];
   fix_loop(fix, LKS, c.ny + 1, [&](int gw, int k0, int k1, int lane, int w) {
-    lagr_body<DivIEEE>(c, &tm, d1, e1, u1, v1, fx, fy, s, gw, k0, k1, lane, ring[w], bars[w]);
+    lagr_seg<DivIEEE>(c, &tm, d1, e1, u1, v1, fx, fy, s, gw, k0, k1, lane, ring[w], bars[w]);
   });
 }
 // (a register-only Lagrangian variant was measured 3% slower; see git history)
