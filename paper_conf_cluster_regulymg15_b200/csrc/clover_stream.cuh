@@ -646,7 +646,9 @@ kf_advec_cell_x(Chunk c, const double* __restrict__ rho, const double* __restric
 // pre-sweep volume of rows k, k+1.
 constexpr int CKS_Y = CLOVER_CKS_Y;
 
-template <int SWEEP, class D>
+// EDGE = false: columns and rows k0-2 .. k1+1 at least HALO+2 away from
+// every wall and chunk edge (y_interior).
+template <int SWEEP, class D, bool EDGE>
 __device__ __forceinline__ bool advec_cell_y_body(const Chunk& c, const double* __restrict__ rho, const double* __restrict__ en,
                 const double* __restrict__ fx, const double* __restrict__ fy,
                 double* __restrict__ rho_out, double* __restrict__ en_out,
@@ -654,14 +656,14 @@ __device__ __forceinline__ bool advec_cell_y_body(const Chunk& c, const double* 
     int gw, int k0, int k1, int lane) {
   D dv;
   const int j = gw * 32 + lane + 1;
-  if (j <= c.nx) {
+  if (!EDGE || j <= c.nx) {
     const double vol = c.dx * c.dy;
     const int P = c.pitch;
     auto pre_vol = [&](int i) -> double {
       if (SWEEP == 1) return vol + (fy[i + P] - fy[i] + fx[i + 1] - fx[i]);
       return vol + fy[i + P] - fy[i];
     };
-    const bool ncol = near_wall_col(c, j);
+    const bool ncol = EDGE && near_wall_col(c, j);
     int i = idx(c, j, k0);
     // rows k0-2 .. k0+1
     double R0 = rho[i - 2 * P], R1 = rho[i - P], R2 = rho[i], R3 = rho[i + P];
@@ -701,11 +703,11 @@ __device__ __forceinline__ bool advec_cell_y_body(const Chunk& c, const double* 
         const double flo = fy[i], fhi = fy[i + P];
         cell_update(dv, R2, E2, pv0, m0, m1, ef0, ef1, flo, fhi, ro, eo);
       }
-      const bool near = ncol || near_wall_row(c, k);
+      const bool near = EDGE && (ncol || near_wall_row(c, k));
       store_at(c, rho_out, K_CELL, j, k, i, near, ro);
       store_at(c, en_out, K_CELL, j, k, i, near, eo);
       store_at(c, mfy, K_YFACE, j, k, i, near, m0);
-      if (k == c.ny) store_field(c, mfy, K_YFACE, j, k + 1, m1);
+      if (EDGE && k == c.ny) store_field(c, mfy, K_YFACE, j, k + 1, m1);
       R0 = R1; R1 = R2; R2 = R3; R3 = R4;
       E0 = E1; E1 = E2; E2 = E3; E3 = E4;
       pvm = pv0; pv0 = pv1;
@@ -713,6 +715,12 @@ __device__ __forceinline__ bool advec_cell_y_body(const Chunk& c, const double* 
     }
   }
   return __any_sync(FULL, dv.bad);
+}
+
+// columns j = 32*gw+1 .. 32*gw+32 with reach j-1 .. j+2, rows k0-2 .. k1+1
+__device__ __forceinline__ bool y_interior(const Chunk& c, int gw, int k0, int k1) {
+  return gw * 32 >= HALO + 2 && gw * 32 + 34 <= c.nx - HALO - 1 && k0 - 2 >= HALO + 2 &&
+         k1 + 1 <= c.ny - HALO - 1;
 }
 
 template <int SWEEP>
@@ -726,7 +734,8 @@ ks_advec_cell_y(Chunk c, const double* __restrict__ rho, const double* __restric
   const int lane = threadIdx.x & 31;
   const int gw = blockIdx.x * (SB / 32) + (threadIdx.x >> 5);
   const int k0 = blockIdx.y * CKS_Y + 1, k1 = min(k0 + CKS_Y, c.ny + 1);
-  if (advec_cell_y_body<SWEEP, DivFast>(c, rho, en, fx, fy, rho_out, en_out, mfy, gw, k0, k1, lane)) {
+  if (y_interior(c, gw, k0, k1) ? advec_cell_y_body<SWEEP, DivFast, false>(c, rho, en, fx, fy, rho_out, en_out, mfy, gw, k0, k1, lane)
+                                : advec_cell_y_body<SWEEP, DivFast, true>(c, rho, en, fx, fy, rho_out, en_out, mfy, gw, k0, k1, lane)) {
     fix_push(fix, lane, gw, blockIdx.y);
   }
 }
@@ -740,7 +749,7 @@ kf_advec_cell_y(Chunk c, const double* __restrict__ rho, const double* __restric
   pdl_trigger();
   pdl_wait();
   fix_loop(fix, CKS_Y, c.ny + 1, [&](int gw, int k0, int k1, int lane, int) {
-    advec_cell_y_body<SWEEP, DivIEEE>(c, rho, en, fx, fy, rho_out, en_out, mfy, gw, k0, k1, lane);
+    advec_cell_y_body<SWEEP, DivIEEE, true>(c, rho, en, fx, fy, rho_out, en_out, mfy, gw, k0, k1, lane);
   });
 }
 
@@ -1135,7 +1144,8 @@ kf_advec_x(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__
 // flux of row k and updates node k.
 constexpr int MKS_Y = CLOVER_MKS_Y;
 
-template <int SWEEP, class D>
+// EDGE = false: see y_interior.
+template <int SWEEP, class D, bool EDGE>
 __device__ __forceinline__ bool advec_mom_y_body(const Chunk& c, const double* __restrict__ rho, const double* __restrict__ mfy,
                const double* __restrict__ fx, const double* __restrict__ uin,
                const double* __restrict__ vin, double* __restrict__ uout,
@@ -1143,14 +1153,14 @@ __device__ __forceinline__ bool advec_mom_y_body(const Chunk& c, const double* _
     int gw, int k0, int k1, int lane) {
   D dv;
   const int j = gw * 32 + lane + 1;
-  if (j <= c.nx + 1) {
+  if (!EDGE || j <= c.nx + 1) {
     const double vol = c.dx * c.dy;
     const int P = c.pitch;
     auto mass_post = [&](int i) -> double {  // rho * post_vol of the cell at offset i
       const double pv = (SWEEP == 1) ? vol + fx[i + 1] - fx[i] : vol;
       return rho[i] * pv;
     };
-    const bool ncol = near_wall_col(c, j);
+    const bool ncol = EDGE && near_wall_col(c, j);
     // node flux of row r uses My(j-1,r), My(j,r), My(j-1,r+1), My(j,r+1)
     auto node_flux = [&](int i) -> double {
       return 0.25 * (mfy[i - 1] + mfy[i] + mfy[i - 1 + P] + mfy[i + P]);
@@ -1201,7 +1211,7 @@ __device__ __forceinline__ bool advec_mom_y_body(const Chunk& c, const double* _
       {
         mom_update(dv, U2, V2, pre_0, post_0, mu_m, mu, mv_m, mv, un, vn);
       }
-      const bool near = ncol || near_wall_row(c, k);
+      const bool near = EDGE && (ncol || near_wall_row(c, k));
       store_at(c, uout, K_XVEL, j, k, i, near, un);
       store_at(c, vout, K_YVEL, j, k, i, near, vn);
       U1 = U2; U2 = U3; U3 = U4;
@@ -1225,7 +1235,8 @@ ks_advec_mom_y(Chunk c, const double* __restrict__ rho, const double* __restrict
   const int lane = threadIdx.x & 31;
   const int gw = blockIdx.x * (SB / 32) + (threadIdx.x >> 5);
   const int k0 = blockIdx.y * MKS_Y + 1, k1 = min(k0 + MKS_Y, c.ny + 2);
-  if (advec_mom_y_body<SWEEP, DivFast>(c, rho, mfy, fx, uin, vin, uout, vout, gw, k0, k1, lane)) {
+  if (y_interior(c, gw, k0, k1) ? advec_mom_y_body<SWEEP, DivFast, false>(c, rho, mfy, fx, uin, vin, uout, vout, gw, k0, k1, lane)
+                                : advec_mom_y_body<SWEEP, DivFast, true>(c, rho, mfy, fx, uin, vin, uout, vout, gw, k0, k1, lane)) {
     fix_push(fix, lane, gw, blockIdx.y);
   }
 }
@@ -1239,7 +1250,7 @@ kf_advec_mom_y(Chunk c, const double* __restrict__ rho, const double* __restrict
   pdl_trigger();
   pdl_wait();
   fix_loop(fix, MKS_Y, c.ny + 2, [&](int gw, int k0, int k1, int lane, int) {
-    advec_mom_y_body<SWEEP, DivIEEE>(c, rho, mfy, fx, uin, vin, uout, vout, gw, k0, k1, lane);
+    advec_mom_y_body<SWEEP, DivIEEE, true>(c, rho, mfy, fx, uin, vin, uout, vout, gw, k0, k1, lane);
   });
 }
 
