@@ -56,10 +56,12 @@ struct ViscIn {
   double u00, u10, u01, u11, v00, v10, v01, v11;
 };
 
-// c.3 viscosity of one cell (writes q) and the c.4 sound-speed term cc.
+// c.3 viscosity of one cell (writes q) and the square of the c.4 sound-speed
+// term, cc2 = cs*cs + 2q/rho; the reading takes cc = max(sqrt(cc2), g_small)
+// per cell, which only enters calc_dt through its maximum (DtAcc).
 template <class D>
 __device__ __forceinline__ void visc_cell(D& dv, const ViscIn& I, const Chunk& C, double& qv,
-                                          double& cc) {
+                                          double& cc2) {
   const double dx = C.dx, dy = C.dy;
   const double u00 = I.u00, u10 = I.u10, u01 = I.u01, u11 = I.u11;
   const double v00 = I.v00, v10 = I.v10, v01 = I.v01, v11 = I.v11;
@@ -87,9 +89,8 @@ __device__ __forceinline__ void visc_cell(D& dv, const ViscIn& I, const Chunk& C
     qv = 2.0 * I.rho * grad2 * limiter * limiter;
   }
   double cs = eos_soundspeed(dv, I.rho, I.e);
-  cc = cs * cs;
-  cc = cc + dv(2.0 * qv, I.rho);
-  cc = fmax(sqrt(cc), G_SMALL);
+  cc2 = cs * cs;
+  cc2 = cc2 + dv(2.0 * qv, I.rho);
 }
 
 // c.4 calc_dt, reduced over a set of cells without per-cell divisions.
@@ -102,9 +103,12 @@ __device__ __forceinline__ void visc_cell(D& dv, const ViscIn& I, const Chunk& C
 // RN(min w / 2vol), and -1/x grows with x < 0: the minimum of the per-cell
 // dt over the set equals the dt computed once from the four extremes below,
 // bit for bit.  The kernel keeps the extremes per thread and divides once.
+// Likewise correctly rounded sqrt and fmax(., g_small) are monotone, so the
+// maximum over cells of cc = fmax(sqrt(cc2), g_small) is fmax(sqrt(max cc2),
+// g_small): one square root per thread instead of one per cell.
 struct DtAcc {
-  double ccmax = 0.0, dumax = 0.0, dvmax = 0.0, wmin = G_BIG;
-  __device__ __forceinline__ void add(const ViscIn& I, const Chunk& C, double cc) {
+  double cc2max = 0.0, dumax = 0.0, dvmax = 0.0, wmin = G_BIG;
+  __device__ __forceinline__ void add(const ViscIn& I, const Chunk& C, double cc2) {
     const double dx = C.dx, dy = C.dy, vol = dx * dy;
     double dvv = 0.0;
     double dv1 = (I.u00 + I.u01) * dy;
@@ -116,11 +120,12 @@ struct DtAcc {
     dvv = dvv + dv2 - dv1;
     dvmax = fmax(dvmax, fmax(fmax(fabs(dv1), fabs(dv2)), G_SMALL * vol));
     wmin = fmin(wmin, dvv);
-    ccmax = fmax(ccmax, cc);
+    cc2max = fmax(cc2max, cc2);
   }
   // dt of the set (call only if at least one cell was added)
   __device__ __forceinline__ double dt(const Chunk& C, const DtParams& prm) const {
     const double dx = C.dx, dy = C.dy, vol = dx * dy;
+    const double ccmax = fmax(sqrt(cc2max), G_SMALL);
     double dtct = div_fast_nz(prm.dtc_safe * fmin(dx, dy), ccmax);
     double dtut = div_fast_nz(prm.dtu_safe * 2.0 * vol, dumax);
     double dtvt = div_fast_nz(prm.dtv_safe * 2.0 * vol, dvmax);

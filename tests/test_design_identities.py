@@ -40,3 +40,21 @@ def test_min_of_divergence_term_is_term_of_min():
         m = np.min(w) / vol2
         once = s * (-1.0 / m) if m < -g_small else g_big
         assert np.float64(np.min(cell)).tobytes() == np.float64(once).tobytes()
+
+
+def test_max_of_rounded_sqrt_is_sqrt_of_max():
+    # DtAcc: max_i fmax(RN(sqrt(a_i)), g) == fmax(RN(sqrt(max_i a_i)), g)
+    rng = np.random.default_rng(13)
+    g = 1.0e-16
+    for trial in range(300):
+        n = int(rng.integers(1, 64))
+        if trial % 3 == 0:  # near-ties in the last ulps
+            a = np.full(n, float(_logu(rng, 1e-40, 1e6, 1)[0]))
+            a = a * (1 + rng.integers(0, 8, n) * 2.0**-52)
+        else:
+            a = _logu(rng, 1e-40, 1e6, n)
+        if trial % 5 == 0:
+            a[rng.integers(0, n)] = 0.0
+        per_cell = np.max(np.fmax(np.sqrt(a), g))
+        once = np.fmax(np.sqrt(np.max(a)), g)
+        assert np.float64(per_cell).tobytes() == np.float64(once).tobytes()
