@@ -49,6 +49,8 @@ ALGO_BYTES_PER_CELL = {
     "k_advec_mom_y<2>": 8 * (4 + 2),
     "k_advec_x<1>": 8 * (6 + 4),         # fused x sweep: rho e Fx Fy u v -> rho' e' u v
     "k_advec_x<2>": 8 * (5 + 4),         # rho e Fx u v -> rho' e' u v
+    "k_advec_y<1>": 8 * (6 + 4),         # fused y sweep: rho e Fx Fy u v -> rho' e' u v
+    "k_advec_y<2>": 8 * (5 + 4),         # rho e Fy u v -> rho' e' u v
 }
 # sum over one step of the kernels actually launched (the profile pass
 # below); with the fused x sweep 304/312 B for the x-first/y-first step,

@@ -186,7 +186,7 @@ int clover_kernels_per_step(clover_ctx* ctx, int32_t* out);
  * after every kernel on the context's work stream; ms_out[i] / launches_out[i]
  * receive the summed duration and launch count of kernel type i
  * (clover_profile_name(i)); nslots must be >= CLOVER_PROFILE_SLOTS. */
-#define CLOVER_PROFILE_SLOTS 13
+#define CLOVER_PROFILE_SLOTS 15
 int clover_profile_steps(clover_ctx* ctx, int32_t nsteps, double* ms_out, int64_t* launches_out,
                          int32_t nslots);
 const char* clover_profile_name(int32_t i);

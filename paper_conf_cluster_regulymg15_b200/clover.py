@@ -22,7 +22,7 @@ c_void_p = ctypes.c_void_p
 dptr = ctypes.POINTER(c_double)
 
 CLOVER_OK = 0
-PROFILE_SLOTS = 13
+PROFILE_SLOTS = 15
 ERRORS = {-1: "ARG", -2: "CUDA", -3: "NCCL", -4: "WORKSPACE", -5: "SMALL_DT", -7: "STATE"}
 
 FIELDS = {"density0": 0, "energy0": 1, "pressure": 2, "viscosity": 3, "soundspeed": 4,

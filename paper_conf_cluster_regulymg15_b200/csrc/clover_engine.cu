@@ -73,6 +73,11 @@ enum Buf {
 static_assert(B_E1 == B_D1 + XF<1>::E && B_U1 == B_D1 + XF<1>::U && B_V1 == B_D1 + XF<1>::V &&
                   B_FY == B_D1 + XF<1>::FY && B_FX == B_D1 + XF<1>::FX,
               "fused x sweep 1 tensor order");
+static_assert(YRW == XRW && (int)YL<1>::E == XF<1>::E * YRW && (int)YL<1>::U == XF<1>::U * YRW &&
+                  (int)YL<1>::V == XF<1>::V * YRW && (int)YL<1>::FY == XF<1>::FY * YRW &&
+                  (int)YL<1>::FX == XF<1>::FX * YRW && B_E2 == B_D2 + 1 && B_U2 == B_D2 + 2 &&
+                  B_V2 == B_D2 + 3,
+              "fused y sweep tensors (sweep 1 shares the fused x sweep 1 map)");
 static_assert(B_D2 == B_FX + XF<2>::R && B_E2 == B_FX + XF<2>::E && B_U2 == B_FX + XF<2>::U &&
                   B_V2 == B_FX + XF<2>::V,
               "fused x sweep 2 tensor order");
@@ -100,6 +105,8 @@ struct ChunkState {
   CUtensorMap tm_visc;  // d0 e0 u0 v0 as {pitch, rows, 4}, box {VRW, 1, 4}
   CUtensorMap tm_x1;    // d1 e1 u1 v1 fy fx, box {XRW, 1, 6} (fused x sweep 1)
   CUtensorMap tm_x2;    // fx d2 e2 u2 v2, box {XRW, 1, 5} (fused x sweep 2)
+  CUtensorMap tm_fy;    // fy, box {YRW, 1, 1} (fused y sweep 2)
+  CUtensorMap tm_c4;    // d2 e2 u2 v2, box {YRW, 1, 4} (fused y sweep 2)
 };
 
 struct Layout {
@@ -142,10 +149,10 @@ dim3 grid_strip(int ncols, int width, int nrows, int ks) {
   return dim3(cdiv(cdiv(ncols, width), SB / 32), cdiv(nrows, ks));
 }
 int64_t fix_capacity(int nx, int ny) {
-  const dim3 g[7] = {grid_cols(nx, ny, VKS),          grid_strip(nx, LW, ny, LKS),
+  const dim3 g[8] = {grid_cols(nx, ny, VKS),          grid_strip(nx, LW, ny, LKS),
                      grid_strip(nx, CW_X, ny, CKS),    grid_cols(nx, ny, CKS_Y),
                      grid_strip(nx + 1, MW_X, ny + 1, MKS), grid_cols(nx + 1, ny + 1, MKS_Y),
-                     grid_strip(nx + 1, XW, ny + 1, XKS)};
+                     grid_strip(nx + 1, XW, ny + 1, XKS), grid_strip(nx + 1, YW, ny + 1, YKS)};
   int64_t m = 0;
   for (const dim3& d : g) m = std::max<int64_t>(m, (int64_t)d.x * d.y * (SB / 32));
   return m;
@@ -209,6 +216,7 @@ struct clover_ctx {
   bool advect_x = true;
   bool use_graphs = true;
   bool fuse_x = true;  // fused x sweep where every chunk has both x walls (see fuse_x_ok)
+  bool fuse_y = true;  // fused y sweep where every chunk has both y walls (see fuse_y_ok)
   cudaGraphExec_t gexec[2] = {nullptr, nullptr};
   int64_t ws_bytes = 0;
   bool prof = false;
@@ -476,12 +484,12 @@ constexpr int PROF_FIXUP = 0x100;
 
 // Kernel types for clover_profile (names in kProfNames).
 enum { P_VISC_DT, P_DT_FINAL, P_LAGR, P_CELL_X1, P_CELL_X2, P_CELL_Y1, P_CELL_Y2,
-       P_MOM_X1, P_MOM_X2, P_MOM_Y1, P_MOM_Y2, P_ADV_X1, P_ADV_X2, NPROF };
+       P_MOM_X1, P_MOM_X2, P_MOM_Y1, P_MOM_Y2, P_ADV_X1, P_ADV_X2, P_ADV_Y1, P_ADV_Y2, NPROF };
 const char* kProfNames[NPROF] = {"k_visc_dt", "k_dt_finalize", "k_lagrangian",
                                  "k_advec_cell_x<1>", "k_advec_cell_x<2>", "k_advec_cell_y<1>",
                                  "k_advec_cell_y<2>", "k_advec_mom_x<1>", "k_advec_mom_x<2>",
                                  "k_advec_mom_y<1>", "k_advec_mom_y<2>", "k_advec_x<1>",
-                                 "k_advec_x<2>"};
+                                 "k_advec_x<2>", "k_advec_y<1>", "k_advec_y<2>"};
 static_assert(NPROF == CLOVER_PROFILE_SLOTS, "profile slots");
 
 // Record an event after each profiled kernel; (prev event, this event)
@@ -525,6 +533,16 @@ bool fuse_x_ok(const clover_ctx* ctx) {
   if (!ctx->fuse_x || ctx->g.face_mirror == CLOVER_MIRROR_CELLCENTRE) return false;
   for (const auto& cs : ctx->chunks)
     if (!cs.c.wl || !cs.c.wr) return false;
+  return true;
+}
+
+// The fused y sweep needs reflective walls at both y ends of every chunk
+// (its reach along y is 4 rows: a chunk boundary would need depth-4 halos)
+// and the geometric face mirror.
+bool fuse_y_ok(const clover_ctx* ctx) {
+  if (!ctx->fuse_y || ctx->g.face_mirror == CLOVER_MIRROR_CELLCENTRE) return false;
+  for (const auto& cs : ctx->chunks)
+    if (!cs.c.wb || !cs.c.wt) return false;
   return true;
 }
 
@@ -606,6 +624,45 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
             STEP_LAUNCH_CHECK();
             launch_step(kf_advec_x<2>, FIX_BLOCKS, SB, st, c, cs.tm_x2, cs.buf[rout], cs.buf[eout],
                         cs.buf[uout], cs.buf[vout], cs.fix);
+            FIX_LAUNCH_CHECK();
+          }
+        }
+        int rc = exchange(ctx, {rout, eout, uout, vout});
+        if (rc) return rc;
+        if (ctx->prof) prof_mark(ctx, -1);
+      }
+      continue;
+    }
+    if (!xdir && fuse_y_ok(ctx)) {
+      // wall bands of advec_cell y, then advec_cell y + advec_mom y in one
+      // kernel (ks_advec_y): phase ph_cell runs all, phase ph_cell + 1 is empty
+      if (nphase >= ph_cell) {
+        cur_prof_id = sweep == 1 ? P_ADV_Y1 : P_ADV_Y2;
+        for (auto& cs : ctx->chunks) {
+          const Chunk& c = cs.c;
+          const dim3 gw(cdiv(c.nx + 2, SB), 2);
+          const dim3 g = grid_strip(c.nx + 1, YW, c.ny + 1, YKS);
+          const CUtensorMap& ta = sweep == 1 ? cs.tm_x1 : cs.tm_fy;
+          const CUtensorMap& tb = sweep == 1 ? cs.tm_x1 : cs.tm_c4;
+          if (sweep == 1) {
+            launch_step(ks_cell_y_walls<1>, gw, SB, st, c, cs.buf[rin], cs.buf[ein], cs.buf[B_FX],
+                        cs.buf[B_FY], cs.buf[rout], cs.buf[eout], cs.buf[B_MY]);
+            FIX_LAUNCH_CHECK();
+            launch_step(ks_advec_y<1>, g, SB, st, c, ta, tb, cs.buf[rout], cs.buf[eout], cs.buf[B_MY],
+                        cs.buf[uout], cs.buf[vout], cs.fix);
+            STEP_LAUNCH_CHECK();
+            launch_step(kf_advec_y<1>, FIX_BLOCKS, SB, st, c, ta, tb, cs.buf[rout], cs.buf[eout],
+                        cs.buf[B_MY], cs.buf[uout], cs.buf[vout], cs.fix);
+            FIX_LAUNCH_CHECK();
+          } else {
+            launch_step(ks_cell_y_walls<2>, gw, SB, st, c, cs.buf[rin], cs.buf[ein], cs.buf[B_FX],
+                        cs.buf[B_FY], cs.buf[rout], cs.buf[eout], cs.buf[B_MY]);
+            FIX_LAUNCH_CHECK();
+            launch_step(ks_advec_y<2>, g, SB, st, c, ta, tb, cs.buf[rout], cs.buf[eout], cs.buf[B_MY],
+                        cs.buf[uout], cs.buf[vout], cs.fix);
+            STEP_LAUNCH_CHECK();
+            launch_step(kf_advec_y<2>, FIX_BLOCKS, SB, st, c, ta, tb, cs.buf[rout], cs.buf[eout],
+                        cs.buf[B_MY], cs.buf[uout], cs.buf[vout], cs.fix);
             FIX_LAUNCH_CHECK();
           }
         }
@@ -1049,6 +1106,10 @@ int clover_init(const clover_grid* grid, const clover_state* states, int32_t nst
                                     XF<1>::NF, XRW);
       if (!rc) rc = encode_rows_map(&cs.tm_x2, base + (B_FX - B_D0) * (fs / 8), c.pitch, rows, fs,
                                     XF<2>::NF, XRW);
+      if (!rc) rc = encode_rows_map(&cs.tm_fy, base + (B_FY - B_D0) * (fs / 8), c.pitch, rows, fs,
+                                    1, YRW);
+      if (!rc) rc = encode_rows_map(&cs.tm_c4, base + (B_D2 - B_D0) * (fs / 8), c.pitch, rows, fs,
+                                    4, YRW);
       if (rc) return bail(rc);
     }
     cs.ntx = (c.nx + ST - 1) / ST; cs.nty = (c.ny + ST - 1) / ST;
@@ -1151,6 +1212,7 @@ int clover_debug_set_virtual_remote(clover_ctx* ctx, int32_t enable) {
 int clover_debug_set_fusion(clover_ctx* ctx, int32_t enable) {
   if (!ctx) return fail(CLOVER_ERR_ARG, "ctx is NULL");
   ctx->fuse_x = enable != 0;
+  ctx->fuse_y = enable != 0;
   for (int i = 0; i < 2; ++i)
     if (ctx->gexec[i]) {
       cudaGraphExecDestroy(ctx->gexec[i]);
@@ -1174,7 +1236,11 @@ int clover_debug_fix_count(clover_ctx* ctx, int64_t* out) {
 
 int clover_kernels_per_step(clover_ctx* ctx, int32_t* out) {
   if (!ctx || !out) return fail(CLOVER_ERR_ARG, "NULL argument");
-  *out = (int32_t)(ctx->chunks.size() * 12 + 1);  // 6 step kernels + 6 fixups per chunk
+  // per chunk: visc_dt + fixup, Lagrangian + fixup, the x sweep (fused:
+  // kernel + fixup; else cell, mom + 2 fixups), the y sweep (fused: wall
+  // bands, kernel + fixup; else 4); plus k_dt_finalize once
+  const int x = fuse_x_ok(ctx) ? 2 : 4, y = fuse_y_ok(ctx) ? 3 : 4;
+  *out = (int32_t)(ctx->chunks.size() * (4 + x + y) + 1);
   return CLOVER_OK;
 }
 

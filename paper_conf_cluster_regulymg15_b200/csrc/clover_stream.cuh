@@ -653,10 +653,12 @@ __device__ __forceinline__ bool advec_cell_y_body(const Chunk& c, const double* 
                 const double* __restrict__ fx, const double* __restrict__ fy,
                 double* __restrict__ rho_out, double* __restrict__ en_out,
                 double* __restrict__ mfy,
-    int gw, int k0, int k1, int lane) {
+    int gw, int k0, int k1, int lane, int jlo = 1, int jhi = 0x7fffffff) {
+  // columns jlo + 32*gw + lane <= min(jhi, nx) (ks_cell_y_walls also
+  // computes the halo columns 0 / nx+1 at x chunk boundaries)
   D dv;
-  const int j = gw * 32 + lane + 1;
-  if (!EDGE || j <= c.nx) {
+  const int j = gw * 32 + lane + jlo;
+  if (!EDGE || j <= min(jhi, c.nx)) {
     const double vol = c.dx * c.dy;
     const int P = c.pitch;
     auto pre_vol = [&](int i) -> double {
@@ -1252,6 +1254,324 @@ kf_advec_mom_y(Chunk c, const double* __restrict__ rho, const double* __restrict
   fix_loop(fix, MKS_Y, c.ny + 2, [&](int gw, int k0, int k1, int lane, int) {
     advec_mom_y_body<SWEEP, DivIEEE, true>(c, rho, mfy, fx, uin, vin, uout, vout, gw, k0, k1, lane);
   });
+}
+
+// ================================================================ fused y sweep
+// advec_cell (y) and advec_mom (y) of one sweep in one pass, for chunks with
+// reflective walls at both y ends (py == 1) and the geometric face mirror.
+// Warp strip: lane l <-> column j = J0 - 1 + l, J0 = 1 + 31*gw; lanes 1..31
+// own cells and nodes, lane 0 is a halo lane whose post-sweep density and
+// y-face mass flux the node at J0 reads by shuffle.  Rows stream along the
+// sweep: iteration s computes the flux of face s+1 and the update of cell s
+// (as ks_advec_cell_y), then node flux / masses of row s, the momentum flux of
+// node s-1 and the update of node s-2 (as ks_advec_mom_y); the mass flux and
+// post-sweep density never travel through memory.  A segment of node rows
+// [k0, k1) computes faces [k0-2, k1+1] and cells [k0-2, k1].
+// Halo rows at the y walls (faces <= 0 or >= ny+2, cells <= 0 or >= ny+1)
+// are the mirrors written by ks_cell_y_walls (advec_cell_y on rows 1..3 and
+// ny-1..ny, launched first); halo columns at x walls take the mirror of the
+// adjacent lane (density +, y-face mass flux +); at x chunk boundaries they
+// are recomputed from the depth-2 input halos.
+// Inputs stream through a per-warp YRING-row ring: sweep 1 reads d1 e1 u1 v1
+// fy fx (one 3D tensor copy per row), sweep 2 reads fy and d2 e2 u2 v2 (two).
+constexpr int YW = 31;
+#ifndef CLOVER_YKS
+#define CLOVER_YKS 32
+#endif
+constexpr int YKS = CLOVER_YKS;
+#ifndef CLOVER_YRING
+#define CLOVER_YRING 6
+#endif
+constexpr int YRING = CLOVER_YRING;
+constexpr int YRW = 36;
+template <int SWEEP> struct YL;
+template <> struct YL<1> {  // tensor d1 e1 u1 v1 fy fx
+  enum { R = 0, E = YRW, U = 2 * YRW, V = 3 * YRW, FY = 4 * YRW, FX = 5 * YRW, B = 0,
+         SLOT = (6 * YRW + 15) / 16 * 16 };
+  static constexpr unsigned BYTES = 6 * YRW * 8;
+};
+template <> struct YL<2> {  // tensors fy | d2 e2 u2 v2
+  enum { FY = 0, B = (YRW + 15) / 16 * 16, R = B, E = B + YRW, U = B + 2 * YRW, V = B + 3 * YRW,
+         FX = -1, SLOT = (B + 4 * YRW + 15) / 16 * 16 };
+  static constexpr unsigned BYTES = 5 * YRW * 8;
+};
+
+template <int SWEEP, class D, bool EDGE>
+__device__ __forceinline__ bool advec_y_body(const Chunk& c, const CUtensorMap* __restrict__ ta,
+                                             const CUtensorMap* __restrict__ tb,
+                                             double* __restrict__ rho_out,
+                                             double* __restrict__ en_out,
+                                             const double* __restrict__ mfy,
+                                             double* __restrict__ uout,
+                                             double* __restrict__ vout, int gw, int k0, int k1,
+                                             int lane, double* ring, unsigned long long* bars) {
+  using L = YL<SWEEP>;
+  D dv;
+  const int J0 = 1 + YW * gw;
+  if (J0 > c.nx + 1) return false;
+  const int j = J0 - 1 + lane;
+  const int nx = c.nx, ny = c.ny;
+  const double vol = c.dx * c.dy;
+  // halo columns: mirror at an x wall, recomputed at a chunk boundary
+  int src = lane;
+  if (EDGE && c.wl && j == 0) src = lane + 1;
+  if (EDGE && c.wr && j == nx + 1) src = lane - 1;
+  const bool xwall_warp = EDGE && __any_sync(FULL, src != lane);
+  const bool comp = !EDGE || (j >= 0 && j <= nx + 1 && src == lane);  // computes its cells/faces
+  const bool own_cell = lane >= 1 && (!EDGE || j <= nx);
+  const bool own_node = lane >= 1 && (!EDGE || j <= nx + 1);
+  const bool ncol = EDGE && near_wall_col(c, j);
+
+  const int r_first = k0 - 4, r_last = k1 + 2;
+  const int x0 = COL0 + J0 - 2;
+  const int xcol = x0 & ~1;           // 16-B aligned box start
+  const int t0 = 1 + (x0 & 1);        // smem column of lane 0
+  auto issue = [&](int r) {
+    const unsigned sl = (unsigned)(r - r_first) % (unsigned)YRING;
+    double* d = ring + sl * L::SLOT;
+    mbar_arrive_expect_tx(&bars[sl], L::BYTES);
+    tma_load_3d(d, ta, xcol, ROW0 + r, 0, &bars[sl]);
+    if constexpr (SWEEP == 2) tma_load_3d(d + L::B, tb, xcol, ROW0 + r, 0, &bars[sl]);
+  };
+  auto row = [&](int r) -> const double* {
+    return ring + ((unsigned)(r - r_first) % (unsigned)YRING) * L::SLOT + lane + t0;
+  };
+  auto wait_row = [&](int r) {
+    const unsigned rel = (unsigned)(r - r_first);
+    mbar_wait(&bars[rel % YRING], (rel / YRING) & 1u);
+  };
+  if (lane == 0) {
+    for (int t = 0; t < YRING; ++t) mbar_init(&bars[t], 1);
+    fence_mbar_init();
+    fence_proxy_async();
+    for (int r = r_first; r < r_first + YRING && r <= r_last; ++r) issue(r);
+  }
+  __syncwarp();
+
+  auto pre_vol = [&](int r) -> double {  // advec_cell pre-sweep volume of cell row r
+    const double* q = row(r);
+    const double* qn = row(r + 1);
+    if constexpr (SWEEP == 1) return vol + (qn[L::FY] - q[L::FY] + q[L::FX + 1] - q[L::FX]);
+    else return vol + qn[L::FY] - q[L::FY];
+  };
+  auto pv_mom = [&](int r) -> double {  // advec_mom post-sweep volume of cell row r
+    if constexpr (SWEEP == 1) {
+      const double* q = row(r);
+      return vol + q[L::FX + 1] - q[L::FX];
+    } else {
+      return vol;
+    }
+  };
+  auto face_computed = [&](int f) { return !EDGE || (f >= 1 && f <= ny + 1); };
+  auto cell_computed = [&](int r) { return !EDGE || (r >= 1 && r <= ny); };
+  // flux of face f (between cells f-1 and f); pvlo = pre_vol(f-1), pvhi = pre_vol(f)
+  auto face_flux = [&](int f, double pvlo, double pvhi, double& m, double& ef) {
+    const double F = row(f)[L::FY];
+    double ru, rd, rw, eu, ed, ew, pvd;
+    if (F > 0.0) {
+      ru = row(f - 2)[L::R]; rd = row(f - 1)[L::R]; rw = row(f)[L::R];
+      eu = row(f - 2)[L::E]; ed = row(f - 1)[L::E]; ew = row(f)[L::E];
+      pvd = pvlo;
+    } else {
+      ru = row(f + 1)[L::R]; rd = row(f)[L::R]; rw = row(f - 1)[L::R];
+      eu = row(f + 1)[L::E]; ed = row(f)[L::E]; ew = row(f - 1)[L::E];
+      pvd = pvhi;
+    }
+    cell_face_flux(dv, F, pvd, ru, rd, rw, eu, ed, ew, m, ef);
+  };
+
+  // ---- prologue: face k0-2
+  for (int r = r_first; r <= k0 - 1; ++r) wait_row(r);
+  double m_s = 0.0, ef_s = 0.0, pv_s = 0.0;
+  {
+    const int f = k0 - 2;
+    if (face_computed(f)) {
+      pv_s = pre_vol(f);
+      if (comp) face_flux(f, pre_vol(f - 1), pv_s, m_s, ef_s);
+    } else {
+      m_s = mfy[idx(c, j, f)];
+    }
+    if (xwall_warp) {
+      const double ms = __shfl_sync(FULL, m_s, src);
+      if (src != lane) m_s = ms;
+    }
+  }
+  double myl_s = __shfl_up_sync(FULL, m_s, 1);
+  double mp_p = 0.0, mpl_p = 0.0, nf_p = 0.0, pre_p = 0.0, pre_pp = 0.0, post_p = 0.0,
+         post_pp = 0.0;
+  double mu_a = 0.0, mu_b = 0.0, mv_a = 0.0, mv_b = 0.0;
+
+  for (int s = k0 - 2; s <= k1 + 1; ++s) {
+    if (s + 2 <= r_last) wait_row(s + 2);
+    if (s <= k1) {
+      // ---- advec_cell y: face s+1, cell s
+      double m1 = 0.0, ef1 = 0.0, pv1 = 0.0, ro = 0.0;
+      if (face_computed(s + 1)) {
+        pv1 = pre_vol(s + 1);
+        if (comp) face_flux(s + 1, pv_s, pv1, m1, ef1);
+      } else {
+        m1 = mfy[idx(c, j, s + 1)];
+      }
+      if (cell_computed(s)) {
+        if (comp) {
+          double eo;
+          const double* q = row(s);
+          cell_update(dv, q[L::R], q[L::E], pv_s, m_s, m1, ef_s, ef1, q[L::FY], row(s + 1)[L::FY],
+                      ro, eo);
+          if (own_cell && s >= k0 && s < k1) {
+            const int i = idx(c, j, s);
+            const bool near = EDGE && (ncol || near_wall_row(c, s));
+            store_at(c, rho_out, K_CELL, j, s, i, near, ro);
+            store_at(c, en_out, K_CELL, j, s, i, near, eo);
+          }
+        }
+      } else {
+        ro = rho_out[idx(c, j, s)];
+      }
+      if (xwall_warp) {
+        const double ms = __shfl_sync(FULL, m1, src);
+        const double rs = __shfl_sync(FULL, ro, src);
+        if (src != lane) { m1 = ms; ro = rs; }
+      }
+      // ---- advec_mom y: node flux / masses of row s
+      const double mp = ro * pv_mom(s);
+      const double mpl = __shfl_up_sync(FULL, mp, 1);
+      const double myl1 = __shfl_up_sync(FULL, m1, 1);
+      const double nf = 0.25 * (myl_s + m_s + myl1 + m1);   // My(j-1,s) My(j,s) My(j-1,s+1) My(j,s+1)
+      const double post = 0.25 * (mp_p + mp + mpl_p + mpl);  // cells (j,s-1) (j,s) (j-1,s-1) (j-1,s)
+      const double pre = post - nf_p + nf;
+      // momentum flux of node s-1
+      double mu_c = 0.0, mv_c = 0.0;
+      if (s >= k0 && own_node) {
+        const double nfn = nf_p;
+        const double nmp = (nfn < 0.0) ? pre : pre_p;
+        const double* qm2 = row(s - 2);
+        const double* qm1 = row(s - 1);
+        const double* q0 = row(s);
+        const double* qp1 = row(s + 1);
+        const double uu[3] = {nfn < 0.0 ? qp1[L::U] : qm2[L::U], nfn < 0.0 ? q0[L::U] : qm1[L::U],
+                              nfn < 0.0 ? qm1[L::U] : q0[L::U]};
+        const double vv[3] = {nfn < 0.0 ? qp1[L::V] : qm2[L::V], nfn < 0.0 ? q0[L::V] : qm1[L::V],
+                              nfn < 0.0 ? qm1[L::V] : q0[L::V]};
+        mom_flux2(dv, nfn, nmp, uu, vv, c.dy, c.rdy, mu_c, mv_c);
+      }
+      // update of node s-2
+      if (s >= k0 + 2 && own_node) {
+        const int kn = s - 2;
+        const double* qn = row(kn);
+        double un, vn;
+        mom_update(dv, qn[L::U], qn[L::V], pre_pp, post_pp, mu_a, mu_b, mv_a, mv_b, un, vn);
+        const int i = idx(c, j, kn);
+        const bool near = EDGE && (ncol || near_wall_row(c, kn));
+        store_at(c, uout, K_XVEL, j, kn, i, near, un);
+        store_at(c, vout, K_YVEL, j, kn, i, near, vn);
+      }
+      m_s = m1; ef_s = ef1; pv_s = pv1; myl_s = myl1;
+      mp_p = mp; mpl_p = mpl; nf_p = nf;
+      pre_pp = pre_p; pre_p = pre; post_pp = post_p; post_p = post;
+      mu_a = mu_b; mu_b = mu_c; mv_a = mv_b; mv_b = mv_c;
+    } else if (own_node) {
+      // s = k1+1: update of node k1-1 only
+      const int kn = s - 2;
+      const double* qn = row(kn);
+      double un, vn;
+      mom_update(dv, qn[L::U], qn[L::V], pre_pp, post_pp, mu_a, mu_b, mv_a, mv_b, un, vn);
+      const int i = idx(c, j, kn);
+      const bool near = EDGE && (ncol || near_wall_row(c, kn));
+      store_at(c, uout, K_XVEL, j, kn, i, near, un);
+      store_at(c, vout, K_YVEL, j, kn, i, near, vn);
+    }
+    // row s-2 is consumed: refill its slot
+    if (s - 2 >= r_first) {
+#if CLOVER_TMA_RELEASE_FENCE
+      fence_proxy_async();
+#endif
+      __syncwarp();
+      if (lane == 0 && s - 2 + YRING <= r_last) issue(s - 2 + YRING);
+    }
+  }
+  __syncwarp();
+  if (lane == 0)
+    for (int t = 0; t < YRING; ++t) mbar_inval(&bars[t]);  // the ring may be reused (fixup)
+  __syncwarp();
+  return __any_sync(FULL, dv.bad);
+}
+
+// interior: columns J0-1 .. J0+31 and rows k0-4 .. k1+2 at least HALO+2 from
+// every edge (no halo column, loaded halo row or near-wall store)
+__device__ __forceinline__ bool y_fused_interior(const Chunk& c, int gw, int k0, int k1) {
+  const int J0 = 1 + YW * gw;
+  return J0 - 1 >= HALO + 2 && J0 + 31 <= c.nx - HALO - 1 && k0 - 4 >= HALO + 2 &&
+         k1 + 2 <= c.ny - HALO - 1;
+}
+
+template <int SWEEP, class D>
+__device__ __forceinline__ bool advec_y_seg(const Chunk& c, const CUtensorMap* ta,
+                                            const CUtensorMap* tb, double* rho_out, double* en_out,
+                                            const double* mfy, double* uout, double* vout, int gw,
+                                            int k0, int k1, int lane, double* ring,
+                                            unsigned long long* bars) {
+  if (y_fused_interior(c, gw, k0, k1))
+    return advec_y_body<SWEEP, D, false>(c, ta, tb, rho_out, en_out, mfy, uout, vout, gw, k0, k1,
+                                         lane, ring, bars);
+  return advec_y_body<SWEEP, D, true>(c, ta, tb, rho_out, en_out, mfy, uout, vout, gw, k0, k1,
+                                      lane, ring, bars);
+}
+
+template <int SWEEP>
+__global__ void __launch_bounds__(SB)
+ks_advec_y(Chunk c, const __grid_constant__ CUtensorMap ta, const __grid_constant__ CUtensorMap tb,
+           double* __restrict__ rho_out, double* __restrict__ en_out, const double* __restrict__ mfy,
+           double* __restrict__ uout, double* __restrict__ vout, FixSlot fix) {
+  pdl_trigger();
+  pdl_wait();
+  __shared__ __align__(128) double ring[SB / 32][YRING * YL<SWEEP>::SLOT];
+  __shared__ __align__(8) unsigned long long bars[SB / 32][YRING];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const int gw = blockIdx.x * (SB / 32) + w;
+  const int k0 = blockIdx.y * YKS + 1, k1 = min(k0 + YKS, c.ny + 2);
+  if (advec_y_seg<SWEEP, DivFast>(c, &ta, &tb, rho_out, en_out, mfy, uout, vout, gw, k0, k1, lane,
+                                  ring[w], bars[w]))
+    fix_push(fix, lane, gw, blockIdx.y);
+}
+
+template <int SWEEP>
+__global__ void __launch_bounds__(SB)
+kf_advec_y(Chunk c, const __grid_constant__ CUtensorMap ta, const __grid_constant__ CUtensorMap tb,
+           double* __restrict__ rho_out, double* __restrict__ en_out, const double* __restrict__ mfy,
+           double* __restrict__ uout, double* __restrict__ vout, FixSlot fix) {
+  pdl_trigger();
+  pdl_wait();
+  __shared__ __align__(128) double ring[SB / 32][YRING * YL<SWEEP>::SLOT];
+  __shared__ __align__(8) unsigned long long bars[SB / 32][YRING];
+  fix_loop(fix, YKS, c.ny + 2, [&](int gw, int k0, int k1, int lane, int w) {
+    advec_y_seg<SWEEP, DivIEEE>(c, &ta, &tb, rho_out, en_out, mfy, uout, vout, gw, k0, k1, lane,
+                                ring[w], bars[w]);
+  });
+}
+
+// advec_cell y on the wall bands (cell rows 1..3 and ny-1..ny, IEEE
+// division: bitwise the fast path's results) so the fused y sweep finds
+// the mirrored halo rows of the post-sweep density and the y-face mass flux.
+template <int SWEEP>
+__global__ void __launch_bounds__(SB)
+ks_cell_y_walls(Chunk c, const double* __restrict__ rho, const double* __restrict__ en,
+                const double* __restrict__ fx, const double* __restrict__ fy,
+                double* __restrict__ rho_out, double* __restrict__ en_out,
+                double* __restrict__ mfy) {
+  pdl_trigger();
+  pdl_wait();
+  const int lane = threadIdx.x & 31;
+  const int gw = blockIdx.x * (SB / 32) + (threadIdx.x >> 5);
+  const int k0 = blockIdx.y == 0 ? 1 : c.ny - 1;
+  const int k1 = blockIdx.y == 0 ? min(4, c.ny + 1) : c.ny + 1;
+  // halo columns at x chunk boundaries too: the fused y sweep's halo lanes
+  // recompute their interior rows but read these wall rows
+  const int jlo = c.wl ? 1 : 0;
+  Chunk cw = c;
+  cw.nx = c.wr ? c.nx : c.nx + 1;
+  advec_cell_y_body<SWEEP, DivIEEE, true>(cw, rho, en, fx, fy, rho_out, en_out, mfy, gw, k0, k1,
+                                          lane, jlo);
 }
 
 }  // namespace clover
