@@ -609,8 +609,6 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
         for (auto& cs : ctx->chunks) {
           const Chunk& c = cs.c;
           const dim3 g = grid_strip(c.nx + 1, XW, c.ny + 1, XKS);
-          const double* fx = cs.buf[B_FX];
-          const double* fy = cs.buf[B_FY];
           if (sweep == 1) {
             launch_step(ks_advec_x<1>, g, SB, st, c, cs.tm_x1, cs.buf[rout], cs.buf[eout],
                         cs.buf[uout], cs.buf[vout], cs.fix);
