@@ -124,10 +124,32 @@ def test_fused_x_sweep_stage_parity(torch_cuda):
             assert np.array_equal(a, b), (name, rel_cell(a, b))
 
 
-@pytest.mark.parametrize("case", ["bm", "fuzz", "random", "tiny", "ragged", "chunks_1x3"])
+def test_fused_y_sweep_stage_parity(torch_cuda):
+    """The fused y sweep (wall bands + advec_cell y + advec_mom y in one
+    kernel) against the oracle's adv_cell1 + adv_mom1 stages of step 2
+    (y first), single chunk and 2x1 chunks (x chunk boundary: halo columns
+    recomputed)."""
+    for deck, kw in ((bm_deck(64), {}), (fuzz_deck(3), {}), (fuzz_deck(5), dict(px=2, py=1))):
+        deck["max_timestep"] = 1.0
+        g, o = make_gpu(deck, **kw), Oracle(deck)
+        g.step(1)
+        o.step(1)
+        g.debug_partial_step(5)
+        for st in ("timestep", "pdv_predict", "accelerate", "pdv_correct", "flux_calc",
+                   "adv_cell1", "adv_mom1"):
+            o.run_stage(st)
+        for buf, kind, name in (("d2", "cell", "density1"), ("e2", "cell", "energy1"),
+                                ("u2", "xvel", "xvel1"), ("v2", "yvel", "yvel1")):
+            a, b = g.debug_read(buf, kind), o.read(name)
+            assert np.array_equal(a, b), (name, rel_cell(a, b))
+
+
+@pytest.mark.parametrize("case", ["bm", "fuzz", "random", "tiny", "ragged", "chunks_1x3",
+                                  "chunks_3x1"])
 def test_fused_and_separate_x_sweep_identical(torch_cuda, case):
-    """Fused and separate x sweeps give bit-identical states (halo included:
-    the next kernels read the mirrors/exchanged halos both paths produce)."""
+    """Fused and separate x and y sweeps give bit-identical states (halo
+    included: the next kernels read the mirrors/exchanged halos both paths
+    produce)."""
     kw = {}
     fields = None
     if case == "bm":
@@ -139,6 +161,9 @@ def test_fused_and_separate_x_sweep_identical(torch_cuda, case):
     elif case == "chunks_1x3":
         deck = fuzz_deck(11)
         kw = dict(px=1, py=3)
+    elif case == "chunks_3x1":  # fused y with x chunk boundaries
+        deck = fuzz_deck(12)
+        kw = dict(px=3, py=1)
     else:
         deck = bm_deck(70, 50)
         deck["max_timestep"] = 1.0
