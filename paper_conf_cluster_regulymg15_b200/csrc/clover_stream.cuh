@@ -1280,7 +1280,7 @@ constexpr int YW = 31;
 #endif
 constexpr int YKS = CLOVER_YKS;
 #ifndef CLOVER_YRING
-#define CLOVER_YRING 6
+#define CLOVER_YRING 8
 #endif
 constexpr int YRING = CLOVER_YRING;
 constexpr int YRW = 36;
@@ -1367,17 +1367,14 @@ __device__ __forceinline__ bool advec_y_body(const Chunk& c, const CUtensorMap* 
   // flux of face f (between cells f-1 and f); pvlo = pre_vol(f-1), pvhi = pre_vol(f)
   auto face_flux = [&](int f, double pvlo, double pvhi, double& m, double& ef) {
     const double F = row(f)[L::FY];
-    double ru, rd, rw, eu, ed, ew, pvd;
-    if (F > 0.0) {
-      ru = row(f - 2)[L::R]; rd = row(f - 1)[L::R]; rw = row(f)[L::R];
-      eu = row(f - 2)[L::E]; ed = row(f - 1)[L::E]; ew = row(f)[L::E];
-      pvd = pvlo;
-    } else {
-      ru = row(f + 1)[L::R]; rd = row(f)[L::R]; rw = row(f - 1)[L::R];
-      eu = row(f + 1)[L::E]; ed = row(f)[L::E]; ew = row(f - 1)[L::E];
-      pvd = pvhi;
-    }
-    cell_face_flux(dv, F, pvd, ru, rd, rw, eu, ed, ew, m, ef);
+    // upwind / donor / downwind rows picked by address (one select per row
+    // instead of one per loaded value)
+    const bool pos = F > 0.0;
+    const double* pu = pos ? row(f - 2) : row(f + 1);
+    const double* pd = pos ? row(f - 1) : row(f);
+    const double* pw = pos ? row(f) : row(f - 1);
+    cell_face_flux(dv, F, pos ? pvlo : pvhi, pu[L::R], pd[L::R], pw[L::R], pu[L::E], pd[L::E],
+                   pw[L::E], m, ef);
   };
 
   // ---- prologue: face k0-2
@@ -1397,13 +1394,12 @@ __device__ __forceinline__ bool advec_y_body(const Chunk& c, const CUtensorMap* 
     }
   }
   double myl_s = __shfl_up_sync(FULL, m_s, 1);
-  double mp_p = 0.0, mpl_p = 0.0, nf_p = 0.0, pre_p = 0.0, pre_pp = 0.0, post_p = 0.0,
-         post_pp = 0.0;
-  double mu_a = 0.0, mu_b = 0.0, mv_a = 0.0, mv_b = 0.0;
+  double mp_p = 0.0, mpl_p = 0.0, nf_p = 0.0, pre_p = 0.0, post_p = 0.0;
+  double mu_b = 0.0, mv_b = 0.0;  // momentum flux of node s-2
 
-  for (int s = k0 - 2; s <= k1 + 1; ++s) {
+  for (int s = k0 - 2; s <= k1; ++s) {
     if (s + 2 <= r_last) wait_row(s + 2);
-    if (s <= k1) {
+    {
       // ---- advec_cell y: face s+1, cell s
       double m1 = 0.0, ef1 = 0.0, pv1 = 0.0, ro = 0.0;
       if (face_computed(s + 1)) {
@@ -1440,46 +1436,35 @@ __device__ __forceinline__ bool advec_y_body(const Chunk& c, const CUtensorMap* 
       const double nf = 0.25 * (myl_s + m_s + myl1 + m1);   // My(j-1,s) My(j,s) My(j-1,s+1) My(j,s+1)
       const double post = 0.25 * (mp_p + mp + mpl_p + mpl);  // cells (j,s-1) (j,s) (j-1,s-1) (j-1,s)
       const double pre = post - nf_p + nf;
-      // momentum flux of node s-1
-      double mu_c = 0.0, mv_c = 0.0;
+      // momentum flux of node s-1, then the update of node s-1 (fluxes of
+      // nodes s-2 and s-1; node masses of row s-1)
       if (s >= k0 && own_node) {
         const double nfn = nf_p;
         const double nmp = (nfn < 0.0) ? pre : pre_p;
-        const double* qm2 = row(s - 2);
         const double* qm1 = row(s - 1);
         const double* q0 = row(s);
-        const double* qp1 = row(s + 1);
-        const double uu[3] = {nfn < 0.0 ? qp1[L::U] : qm2[L::U], nfn < 0.0 ? q0[L::U] : qm1[L::U],
-                              nfn < 0.0 ? qm1[L::U] : q0[L::U]};
-        const double vv[3] = {nfn < 0.0 ? qp1[L::V] : qm2[L::V], nfn < 0.0 ? q0[L::V] : qm1[L::V],
-                              nfn < 0.0 ? qm1[L::V] : q0[L::V]};
+        const bool neg = nfn < 0.0;
+        const double* pa = neg ? row(s + 1) : row(s - 2);  // upwind
+        const double* pb = neg ? q0 : qm1;                 // donor
+        const double* pc = neg ? qm1 : q0;                 // downwind
+        const double uu[3] = {pa[L::U], pb[L::U], pc[L::U]};
+        const double vv[3] = {pa[L::V], pb[L::V], pc[L::V]};
+        double mu_c, mv_c;
         mom_flux2(dv, nfn, nmp, uu, vv, c.dy, c.rdy, mu_c, mv_c);
-      }
-      // update of node s-2
-      if (s >= k0 + 2 && own_node) {
-        const int kn = s - 2;
-        const double* qn = row(kn);
-        double un, vn;
-        mom_update(dv, qn[L::U], qn[L::V], pre_pp, post_pp, mu_a, mu_b, mv_a, mv_b, un, vn);
-        const int i = idx(c, j, kn);
-        const bool near = EDGE && (ncol || near_wall_row(c, kn));
-        store_at(c, uout, K_XVEL, j, kn, i, near, un);
-        store_at(c, vout, K_YVEL, j, kn, i, near, vn);
+        if (s >= k0 + 1) {
+          const int kn = s - 1;
+          double un, vn;
+          mom_update(dv, qm1[L::U], qm1[L::V], pre_p, post_p, mu_b, mu_c, mv_b, mv_c, un, vn);
+          const int i = idx(c, j, kn);
+          const bool near = EDGE && (ncol || near_wall_row(c, kn));
+          store_at(c, uout, K_XVEL, j, kn, i, near, un);
+          store_at(c, vout, K_YVEL, j, kn, i, near, vn);
+        }
+        mu_b = mu_c; mv_b = mv_c;
       }
       m_s = m1; ef_s = ef1; pv_s = pv1; myl_s = myl1;
       mp_p = mp; mpl_p = mpl; nf_p = nf;
-      pre_pp = pre_p; pre_p = pre; post_pp = post_p; post_p = post;
-      mu_a = mu_b; mu_b = mu_c; mv_a = mv_b; mv_b = mv_c;
-    } else if (own_node) {
-      // s = k1+1: update of node k1-1 only
-      const int kn = s - 2;
-      const double* qn = row(kn);
-      double un, vn;
-      mom_update(dv, qn[L::U], qn[L::V], pre_pp, post_pp, mu_a, mu_b, mv_a, mv_b, un, vn);
-      const int i = idx(c, j, kn);
-      const bool near = EDGE && (ncol || near_wall_row(c, kn));
-      store_at(c, uout, K_XVEL, j, kn, i, near, un);
-      store_at(c, vout, K_YVEL, j, kn, i, near, vn);
+      pre_p = pre; post_p = post;
     }
     // row s-2 is consumed: refill its slot
     if (s - 2 >= r_first) {

@@ -23,7 +23,9 @@ def short(name):
                  ("ks_advec_cell_y<1>", "k_advec_cell_y<1>"), ("ks_advec_cell_y<2>", "k_advec_cell_y<2>"),
                  ("ks_advec_mom_x<1>", "k_advec_mom_x<1>"), ("ks_advec_mom_x<2>", "k_advec_mom_x<2>"),
                  ("ks_advec_mom_y<1>", "k_advec_mom_y<1>"), ("ks_advec_mom_y<2>", "k_advec_mom_y<2>"),
-                 ("ks_advec_x<1>", "k_advec_x<1>"), ("ks_advec_x<2>", "k_advec_x<2>")):
+                 ("ks_advec_x<1>", "k_advec_x<1>"), ("ks_advec_x<2>", "k_advec_x<2>"),
+                 ("ks_advec_y<1>", "k_advec_y<1>"), ("ks_advec_y<2>", "k_advec_y<2>"),
+                 ("ks_cell_y_walls<1>", "k_cell_y_walls<1>"), ("ks_cell_y_walls<2>", "k_cell_y_walls<2>")):
         if n.startswith(a):
             return b
     return NAMES.get(n, n)
