@@ -106,29 +106,49 @@ __device__ __forceinline__ void visc_cell(D& dv, const ViscIn& I, const Chunk& C
 // Likewise correctly rounded sqrt and fmax(., g_small) are monotone, so the
 // maximum over cells of cc = fmax(sqrt(cc2), g_small) is fmax(sqrt(max cc2),
 // g_small): one square root per thread instead of one per cell.
+//
+// Faces: |dv1| / |dv2| of a cell are the magnitudes of its left/right (u) and
+// bottom/top (v) face volume terms; the left face of cell j is bitwise the
+// right face of cell j-1 (same expression of the same node velocities), and
+// the bottom face of row k the top face of row k-1.  The maximum over a set
+// of cells is therefore the maximum over the set's faces, each taken once:
+// add() takes the right and top faces of every cell, plus the left face
+// when the caller's column has no left neighbour in the reduction (chunk
+// column 1); the bottom face of a segment's first row comes from bottom().
+// The g_small*vol floor of every per-cell term is applied once in dt()
+// (max is associative).  Non-negative, non-NaN operands: the compare-select
+// max equals fmax bit for bit.
+__device__ __forceinline__ double dmax_nn(double a, double b) { return b > a ? b : a; }
+
 struct DtAcc {
   double cc2max = 0.0, dumax = 0.0, dvmax = 0.0, wmin = G_BIG;
-  __device__ __forceinline__ void add(const ViscIn& I, const Chunk& C, double cc2) {
-    const double dx = C.dx, dy = C.dy, vol = dx * dy;
+  __device__ __forceinline__ void add(const ViscIn& I, const Chunk& C, double cc2, bool left) {
+    const double dx = C.dx, dy = C.dy;
     double dvv = 0.0;
     double dv1 = (I.u00 + I.u01) * dy;
     double dv2 = (I.u10 + I.u11) * dy;
     dvv = dvv + dv2 - dv1;
-    dumax = fmax(dumax, fmax(fmax(fabs(dv1), fabs(dv2)), G_SMALL * vol));
+    dumax = dmax_nn(dumax, fabs(dv2));
+    if (left) dumax = dmax_nn(dumax, fabs(dv1));
     dv1 = (I.v00 + I.v10) * dx;
     dv2 = (I.v01 + I.v11) * dx;
     dvv = dvv + dv2 - dv1;
-    dvmax = fmax(dvmax, fmax(fmax(fabs(dv1), fabs(dv2)), G_SMALL * vol));
-    wmin = fmin(wmin, dvv);
-    cc2max = fmax(cc2max, cc2);
+    dvmax = dmax_nn(dvmax, fabs(dv2));
+    wmin = dvv < wmin ? dvv : wmin;
+    cc2max = dmax_nn(cc2max, cc2);
+  }
+  // bottom face of the first row: v at nodes (j, k0) and (j+1, k0)
+  __device__ __forceinline__ void bottom(double v00, double v10, const Chunk& C) {
+    dvmax = dmax_nn(dvmax, fabs((v00 + v10) * C.dx));
   }
   // dt of the set (call only if at least one cell was added)
   __device__ __forceinline__ double dt(const Chunk& C, const DtParams& prm) const {
     const double dx = C.dx, dy = C.dy, vol = dx * dy;
     const double ccmax = fmax(sqrt(cc2max), G_SMALL);
+    const double dum = fmax(dumax, G_SMALL * vol), dvm = fmax(dvmax, G_SMALL * vol);
     double dtct = div_fast_nz(prm.dtc_safe * fmin(dx, dy), ccmax);
-    double dtut = div_fast_nz(prm.dtu_safe * 2.0 * vol, dumax);
-    double dtvt = div_fast_nz(prm.dtv_safe * 2.0 * vol, dvmax);
+    double dtut = div_fast_nz(prm.dtu_safe * 2.0 * vol, dum);
+    double dtvt = div_fast_nz(prm.dtv_safe * 2.0 * vol, dvm);
     double dvv = wmin / (2.0 * vol);
     double dtdivt = (dvv < -G_SMALL) ? prm.dtdiv_safe * div_fast_nz(-1.0, dvv) : G_BIG;
     return fmin(fmin(dtct, dtut), fmin(dtvt, dtdivt));

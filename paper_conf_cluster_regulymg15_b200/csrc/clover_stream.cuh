@@ -61,6 +61,14 @@ constexpr int SB = CLOVER_SB;  // threads per block
 #else
 #define LB_ADVX __launch_bounds__(SB)
 #endif
+#ifndef CLOVER_MINB_ADVY
+#define CLOVER_MINB_ADVY 0
+#endif
+#if CLOVER_MINB_ADVY > 0
+#define LB_ADVY __launch_bounds__(SB, CLOVER_MINB_ADVY)
+#else
+#define LB_ADVY __launch_bounds__(SB)
+#endif
 #ifndef CLOVER_MINB_MOMY
 #define CLOVER_MINB_MOMY 14
 #endif
@@ -214,6 +222,8 @@ __device__ __forceinline__ bool visc_body(const Chunk& c, const CUtensorMap* __r
   __syncwarp();
   if (lane == 0 && r_first + VSTG <= r_last) issue(r_first + VSTG);  // row k0-1 is consumed
   DtAcc acc;
+  if ((!EDGE || j <= c.nx) && k1 > k0) acc.bottom(row(k0)[VF_V * VRW], row(k0)[VF_V * VRW + 1], c);
+  const bool left = EDGE && j == 1;  // column 1: no left neighbour takes this face
   int i = idx(c, j, k0);
   for (int k = k0; k < k1; ++k, i += c.pitch) {
     wait_row(k + 1);
@@ -232,7 +242,7 @@ __device__ __forceinline__ bool visc_body(const Chunk& c, const CUtensorMap* __r
       I.v01 = rn[VF_V * VRW]; I.v11 = rn[VF_V * VRW + 1];
       double qv, cc2;
       visc_cell(dv, I, c, qv, cc2);
-      acc.add(I, c, cc2);
+      acc.add(I, c, cc2, left);
       store_at(c, q, K_CELL, j, k, i, EDGE && (ncol || near_wall_row(c, k)), qv);
       pcm = pc;
       pc = I.pt;
@@ -993,18 +1003,14 @@ __device__ __forceinline__ bool advec_x_body(const Chunk& c, const CUtensorMap* 
             else
               pvl = vol + flo - fl;
           }
-          double ru, rd, rw, eu, ed, ew, pvd;
-          if (F > 0.0) {
-            ru = rc[F::R * XRW - 2]; rd = rc[F::R * XRW - 1]; rw = rr;
-            eu = rc[F::E * XRW - 2]; ed = rc[F::E * XRW - 1]; ew = ee;
-            pvd = pvl;
-          } else {
-            const int up = EDGE ? min(j + 1, nx + 2) - j : 1;
-            ru = rc[F::R * XRW + up]; rd = rr; rw = rc[F::R * XRW - 1];
-            eu = rc[F::E * XRW + up]; ed = ee; ew = rc[F::E * XRW - 1];
-            pvd = pv;
-          }
-          cell_face_flux(dv, F, pvd, ru, rd, rw, eu, ed, ew, m, ef);
+          // upwind / donor / downwind columns picked by address (one select
+          // per column instead of one per loaded value)
+          const bool pos = F > 0.0;
+          const double* pu = pos ? rc - 2 : rc + (EDGE ? min(j + 1, nx + 2) - j : 1);
+          const double* pd = pos ? rc - 1 : rc;
+          const double* pw = pos ? rc : rc - 1;
+          cell_face_flux(dv, F, pos ? pvl : pv, pu[F::R * XRW], pd[F::R * XRW], pw[F::R * XRW],
+                         pu[F::E * XRW], pd[F::E * XRW], pw[F::E * XRW], m, ef);
         }
         const double mh = __shfl_down_sync(FULL, m, 1);
         const double efh = __shfl_down_sync(FULL, ef, 1);
@@ -1504,7 +1510,7 @@ __device__ __forceinline__ bool advec_y_seg(const Chunk& c, const CUtensorMap* t
 }
 
 template <int SWEEP>
-__global__ void __launch_bounds__(SB)
+__global__ void LB_ADVY
 ks_advec_y(Chunk c, const __grid_constant__ CUtensorMap ta, const __grid_constant__ CUtensorMap tb,
            double* __restrict__ rho_out, double* __restrict__ en_out, const double* __restrict__ mfy,
            double* __restrict__ uout, double* __restrict__ vout, FixSlot fix) {
