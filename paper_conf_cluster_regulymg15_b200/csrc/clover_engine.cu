@@ -551,6 +551,9 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
   cudaStream_t st = ctx->work;
   int cur_prof_id = P_VISC_DT;
   if (ctx->prof) prof_mark(ctx, -1);
+  // one chunk on one rank: the visc fixup's last block finalises dt (no
+  // k_dt_finalize launch); else the slot is combined first (NCCL MIN)
+  const int fold_fin = (nphase >= 2 && ctx->chunks.size() == 1 && ctx->nranks == 1) ? 1 : 0;
   if (nphase >= 1) {
     for (auto& cs : ctx->chunks) {
       const Chunk& c = cs.c;
@@ -558,7 +561,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
                   ctx->scal, ctx->dtp, cs.fix);
       STEP_LAUNCH_CHECK();
       launch_step(kf_visc_dt, FIX_BLOCKS, SB, st, c, cs.tm_visc, cs.buf[B_Q], ctx->scal, ctx->dtp,
-                  cs.fix);
+                  cs.fix, ctx->hist, fold_fin);
       FIX_LAUNCH_CHECK();
     }
     int rc = exchange(ctx, {B_Q});
@@ -572,8 +575,10 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
       NK(ncclAllReduce(&ctx->scal->dt_slot, &ctx->scal->dt_slot, 1, ncclUint64, ncclMin, ctx->comm, st));
 #endif
     if (ctx->prof) prof_mark(ctx, -1);
-    launch_step(k_dt_finalize, 1, 1, st, ctx->scal, ctx->hist, ctx->dtp);
-    STEP_LAUNCH_CHECK();
+    if (!fold_fin) {
+      launch_step(k_dt_finalize, 1, 1, st, ctx->scal, ctx->hist, ctx->dtp);
+      STEP_LAUNCH_CHECK();
+    }
   }
   if (nphase >= 3) {
     cur_prof_id = P_LAGR;
@@ -1236,9 +1241,11 @@ int clover_kernels_per_step(clover_ctx* ctx, int32_t* out) {
   if (!ctx || !out) return fail(CLOVER_ERR_ARG, "NULL argument");
   // per chunk: visc_dt + fixup, Lagrangian + fixup, the x sweep (fused:
   // kernel + fixup; else cell, mom + 2 fixups), the y sweep (fused: wall
-  // bands, kernel + fixup; else 4); plus k_dt_finalize once
+  // bands, kernel + fixup; else 4); plus k_dt_finalize once unless the
+  // visc fixup finalises dt (one chunk on one rank)
   const int x = fuse_x_ok(ctx) ? 2 : 4, y = fuse_y_ok(ctx) ? 3 : 4;
-  *out = (int32_t)(ctx->chunks.size() * (4 + x + y) + 1);
+  const int fin = (ctx->chunks.size() == 1 && ctx->nranks == 1) ? 0 : 1;
+  *out = (int32_t)(ctx->chunks.size() * (4 + x + y) + fin);
   return CLOVER_OK;
 }
 

@@ -156,11 +156,11 @@ struct DtAcc {
 };
 
 // ------------------------------------------------ k_dt_finalize (c.4 tail)
-__global__ void k_dt_finalize(StepScalars* __restrict__ s, double* __restrict__ hist,
-                              DtParams prm) {
-  pdl_trigger();
-  pdl_wait();
-  double dtc = __longlong_as_double((long long)s->dt_slot);
+// dt = min(cells, dtold*dtrise, dtmax), small-dt check, clock, history and
+// slot reset: one thread, after every contribution to dt_slot is visible.
+__device__ __forceinline__ void dt_finalize(StepScalars* __restrict__ s, double* __restrict__ hist,
+                                            const DtParams& prm) {
+  double dtc = __longlong_as_double((long long)*(volatile unsigned long long*)&s->dt_slot);
   double dt = fmin(fmin(dtc, (s->dtold * prm.dtrise)), prm.dtmax);
   s->dt = dt;
   if (dt < prm.dtmin) {
@@ -172,6 +172,14 @@ __global__ void k_dt_finalize(StepScalars* __restrict__ s, double* __restrict__ 
   s->step = s->step + 1;
   hist[(s->step - 1) % DT_HIST] = dt;
   s->dt_slot = (unsigned long long)__double_as_longlong(G_BIG);
+}
+
+// separate launch: multi-chunk / multi-rank steps (after the NCCL MIN)
+__global__ void k_dt_finalize(StepScalars* __restrict__ s, double* __restrict__ hist,
+                              DtParams prm) {
+  pdl_trigger();
+  pdl_wait();
+  dt_finalize(s, hist, prm);
 }
 
 // ------------------------------------------------ Lagrangian phase (c.5-c.7)

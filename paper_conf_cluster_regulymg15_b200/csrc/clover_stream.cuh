@@ -134,8 +134,11 @@ __device__ __forceinline__ void fix_push(FixSlot f, int lane, unsigned gw, unsig
 // (row-parallel, so the fixup's latency is one row, not one segment); the
 // last block to finish resets the list.  run(gw, k0, k1, lane, w) with
 // k1 = k0 + 1; rows at or beyond `lim` are skipped.
-template <class Run>
-__device__ __forceinline__ void fix_loop(FixSlot f, int ks, int lim, Run&& run) {
+struct NoLast {
+  __device__ void operator()() const {}
+};
+template <class Run, class Last = NoLast>
+__device__ __forceinline__ void fix_loop(FixSlot f, int ks, int lim, Run&& run, Last last = {}) {
   const unsigned n = *(volatile unsigned*)f.hdr;
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const unsigned items = n * (unsigned)ks;
@@ -151,6 +154,8 @@ __device__ __forceinline__ void fix_loop(FixSlot f, int ks, int lim, Run&& run) 
       f.hdr[2] += n;  // cumulative (clover_debug_fix_count)
       f.hdr[0] = 0u;
       f.hdr[1] = 0u;
+      __threadfence();
+      last();  // runs after every block's work (and atomics) of this launch
     }
   }
 }
@@ -308,16 +313,24 @@ ks_visc_dt(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__
 
 __global__ void __launch_bounds__(SB)
 kf_visc_dt(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__ q,
-           StepScalars* __restrict__ s, DtParams prm, FixSlot fix) {
+           StepScalars* __restrict__ s, DtParams prm, FixSlot fix, double* __restrict__ hist,
+           int fin) {
   pdl_trigger();
   pdl_wait();
   __shared__ __align__(128) double ring[SB / 32][VSTG * VSLOT];
   __shared__ __align__(8) unsigned long long bars[SB / 32][VSTG];
-  fix_loop(fix, VKS, c.ny + 1, [&](int gw, int k0, int k1, int lane, int w) {
-    double dtw;
-    visc_seg<DivIEEE>(c, &tm, q, prm, gw, k0, k1, lane, ring[w], bars[w], dtw);
-    if (lane == 0) atomicMin(&s->dt_slot, (unsigned long long)__double_as_longlong(dtw));
-  });
+  // fin: single chunk on one rank -- the last block also finalises dt
+  // (k_dt_finalize's work, once every contribution to the slot is in)
+  fix_loop(
+      fix, VKS, c.ny + 1,
+      [&](int gw, int k0, int k1, int lane, int w) {
+        double dtw;
+        visc_seg<DivIEEE>(c, &tm, q, prm, gw, k0, k1, lane, ring[w], bars[w], dtw);
+        if (lane == 0) atomicMin(&s->dt_slot, (unsigned long long)__double_as_longlong(dtw));
+      },
+      [&]() {
+        if (fin) dt_finalize(s, hist, prm);
+      });
 }
 
 // ================================================================ Lagrangian
