@@ -68,29 +68,34 @@ __device__ __forceinline__ void visc_cell(D& dv, const ViscIn& I, const Chunk& C
   double ugrad = (u10 + u11) - (u00 + u01);
   double vgrad = (v01 + v11) - (v00 + v10);
   double div = (dx * (ugrad) + dy * (vgrad));
-  double strain2 = dv.c(0.5 * (u01 + u11 - u00 - u10), dy, C.rdy) + dv.c(0.5 * (v10 + v11 - v00 - v01), dx, C.rdx);
-  double pgradx = dv.c(I.pr - I.pl, dx + dx, C.r2dx);
-  double pgrady = dv.c(I.pt - I.pb, dy + dy, C.r2dy);
-  double pgradx2 = pgradx * pgradx;
-  double pgrady2 = pgrady * pgrady;
-  double limiter = dv(dv.c(0.5 * (ugrad), dx, C.rdx) * pgradx2 + dv.c(0.5 * (vgrad), dy, C.rdy) * pgrady2 +
-                          strain2 * pgradx * pgrady,
-                      fmax(pgradx2 + pgrady2, 1.0e-16));
-  if ((limiter > 0.0) || (div >= 0.0)) {
-    qv = 0.0;
-  } else {
-    pgradx = copysign(fmax(1.0e-16, fabs(pgradx)), pgradx);
-    pgrady = copysign(fmax(1.0e-16, fabs(pgrady)), pgrady);
-    double pgrad = sqrt(pgradx * pgradx + pgrady * pgrady);
-    double xgrad = fabs(dv(dx * pgrad, pgradx));
-    double ygrad = fabs(dv(dy * pgrad, pgrady));
-    double grad = fmin(xgrad, ygrad);
-    double grad2 = grad * grad;
-    qv = 2.0 * I.rho * grad2 * limiter * limiter;
+  // The reading sets q = 0 when limiter > 0 or div >= 0; the limiter (and
+  // the pressure gradients it needs) is only evaluated when div >= 0 does not
+  // already decide it (same results; no work in non-compressing cells).
+  qv = 0.0;
+  if (!(div >= 0.0)) {
+    double strain2 = dv.c(0.5 * (u01 + u11 - u00 - u10), dy, C.rdy) + dv.c(0.5 * (v10 + v11 - v00 - v01), dx, C.rdx);
+    double pgradx = dv.c(I.pr - I.pl, dx + dx, C.r2dx);
+    double pgrady = dv.c(I.pt - I.pb, dy + dy, C.r2dy);
+    double pgradx2 = pgradx * pgradx;
+    double pgrady2 = pgrady * pgrady;
+    double limiter = dv(dv.c(0.5 * (ugrad), dx, C.rdx) * pgradx2 + dv.c(0.5 * (vgrad), dy, C.rdy) * pgrady2 +
+                            strain2 * pgradx * pgrady,
+                        fmax(pgradx2 + pgrady2, 1.0e-16));
+    if (!(limiter > 0.0)) {
+      pgradx = copysign(fmax(1.0e-16, fabs(pgradx)), pgradx);
+      pgrady = copysign(fmax(1.0e-16, fabs(pgrady)), pgrady);
+      double pgrad = sqrt(pgradx * pgradx + pgrady * pgrady);
+      double xgrad = fabs(dv(dx * pgrad, pgradx));
+      double ygrad = fabs(dv(dy * pgrad, pgrady));
+      double grad = fmin(xgrad, ygrad);
+      double grad2 = grad * grad;
+      qv = 2.0 * I.rho * grad2 * limiter * limiter;
+    }
   }
   double cs = eos_soundspeed(dv, I.rho, I.e);
   cc2 = cs * cs;
-  cc2 = cc2 + dv(2.0 * qv, I.rho);
+  // cc2 + RN(2q/rho) with q = +0 is cc2 (cs*cs >= +0): skip the division
+  if (qv != 0.0) cc2 = cc2 + dv(2.0 * qv, I.rho);
 }
 
 // c.4 calc_dt, reduced over a set of cells without per-cell divisions.
@@ -243,6 +248,14 @@ __device__ __forceinline__ void pdv_correct(D& dv, double r, double e, double ph
 }
 
 // ------------------------------------------------ advec_cell (c.8)
+// a / b for b > 0: a zero numerator (the common case in quiescent regions)
+// is its own quotient (+0/b = +0, -0/b = -0), skipping the division.
+template <class D>
+__device__ __forceinline__ double div_pos(D& dv, double a, double b) {
+  double q = a;
+  if (a != 0.0) q = dv(a, b);
+  return q;
+}
 constexpr double ONE_BY_SIX = 1.0 / 6.0;
 
 // Donor-cell flux with the limiter of c.8 for one face.  pv_don = pre_vol of
@@ -251,7 +264,7 @@ template <class D>
 __device__ __forceinline__ void cell_face_flux(D& dv, double F, double pv_don, double ru, double rd,
                                                double rw, double eu, double ed, double ew,
                                                double& mflux, double& eflux) {
-  double sigmat = dv(fabs(F), pv_don);
+  double sigmat = div_pos(dv, fabs(F), pv_don);
   double sigma3 = (1.0 + sigmat);  // * (vertexdx(j)/vertexdx(dif)) == 1 exactly (uniform mesh)
   double sigma4 = 2.0 - sigmat;
   double diffuw = rd - ru;
@@ -266,7 +279,7 @@ __device__ __forceinline__ void cell_face_flux(D& dv, double F, double pv_don, d
   else
     limiter = 0.0;
   mflux = F * (rd + limiter);
-  double sigmam = dv(fabs(mflux), rd * pv_don);
+  double sigmam = div_pos(dv, fabs(mflux), rd * pv_don);
   diffuw = ed - eu;
   diffdw = ew - ed;
   wind = 1.0;
@@ -299,7 +312,7 @@ template <class D>
 __device__ __forceinline__ double mom_flux(D& dv, double nf, double nmp_don, double vup,
                                            double vdon, double vdw, double width, double rwidth) {
   // width = celldx(j) and celldx(dif) are the same constant on the uniform mesh
-  double sigma = dv(fabs(nf), nmp_don);
+  double sigma = div_pos(dv, fabs(nf), nmp_don);
   double vdiffuw = vdon - vup;
   double vdiffdw = vdw - vdon;
   double limiter = 0.0;
@@ -330,8 +343,8 @@ template <class D>
 __device__ __forceinline__ void mom_update(D& dv, double u, double v, double pre, double post,
                                            double mulo, double muhi, double mvlo, double mvhi,
                                            double& un, double& vn) {
-  un = dv(u * pre + mulo - muhi, post);
-  vn = dv(v * pre + mvlo - mvhi, post);
+  un = div_pos(dv, u * pre + mulo - muhi, post);
+  vn = div_pos(dv, v * pre + mvlo - mvhi, post);
 }
 
 }  // namespace clover
