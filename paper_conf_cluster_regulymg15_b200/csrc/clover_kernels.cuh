@@ -40,6 +40,17 @@ __device__ __forceinline__ double eos_soundspeed(D& dv, double rho, double e) {
   return sqrt(c2);
 }
 
+// the square of the ideal_gas sound speed (eos_soundspeed = sqrt of this)
+template <class D>
+__device__ __forceinline__ double eos_c2(D& dv, double rho, double e) {
+  const double gm1 = 1.4 - 1.0;
+  double v = dv.nz(1.0, rho);
+  double p = gm1 * rho * e;
+  double pbe = gm1 * rho;
+  double pbv = -rho * p;
+  return v * v * (p * pbe - pbv);
+}
+
 __device__ __forceinline__ double eos_soundspeed_ieee(double rho, double e) {
   DivIEEE d;
   return eos_soundspeed(d, rho, e);
@@ -61,7 +72,7 @@ struct ViscIn {
 // per cell, which only enters calc_dt through its maximum (DtAcc).
 template <class D>
 __device__ __forceinline__ void visc_cell(D& dv, const ViscIn& I, const Chunk& C, double& qv,
-                                          double& cc2) {
+                                          double& cc2, double& c2) {
   const double dx = C.dx, dy = C.dy;
   const double u00 = I.u00, u10 = I.u10, u01 = I.u01, u11 = I.u11;
   const double v00 = I.v00, v10 = I.v10, v01 = I.v01, v11 = I.v11;
@@ -92,10 +103,16 @@ __device__ __forceinline__ void visc_cell(D& dv, const ViscIn& I, const Chunk& C
       qv = 2.0 * I.rho * grad2 * limiter * limiter;
     }
   }
-  double cs = eos_soundspeed(dv, I.rho, I.e);
-  cc2 = cs * cs;
-  // cc2 + RN(2q/rho) with q = +0 is cc2 (cs*cs >= +0): skip the division
-  if (qv != 0.0) cc2 = cc2 + dv(2.0 * qv, I.rho);
+  // c2 = cs^2 before the square root (ideal_gas).  Where q = 0 the reading's
+  // cc2 = RN(RN(sqrt(c2))^2) + RN(2q/rho) is f(c2) = RN(RN(sqrt(c2))^2), a
+  // monotone function of c2, so DtAcc keeps max c2 over those cells and
+  // applies f once; cells with q != 0 evaluate cc2 here.
+  c2 = eos_c2(dv, I.rho, I.e);
+  cc2 = 0.0;
+  if (qv != 0.0) {
+    const double cs = sqrt(c2);
+    cc2 = cs * cs + dv(2.0 * qv, I.rho);
+  }
 }
 
 // c.4 calc_dt, reduced over a set of cells without per-cell divisions.
@@ -126,8 +143,9 @@ __device__ __forceinline__ void visc_cell(D& dv, const ViscIn& I, const Chunk& C
 __device__ __forceinline__ double dmax_nn(double a, double b) { return b > a ? b : a; }
 
 struct DtAcc {
-  double cc2max = 0.0, dumax = 0.0, dvmax = 0.0, wmin = G_BIG;
-  __device__ __forceinline__ void add(const ViscIn& I, const Chunk& C, double cc2, bool left) {
+  double c2max = 0.0, ccqmax = 0.0, dumax = 0.0, dvmax = 0.0, wmin = G_BIG;
+  __device__ __forceinline__ void add(const ViscIn& I, const Chunk& C, double qv, double cc2,
+                                      double c2, bool left) {
     const double dx = C.dx, dy = C.dy;
     double dvv = 0.0;
     double dv1 = (I.u00 + I.u01) * dy;
@@ -140,7 +158,8 @@ struct DtAcc {
     dvv = dvv + dv2 - dv1;
     dvmax = dmax_nn(dvmax, fabs(dv2));
     wmin = dvv < wmin ? dvv : wmin;
-    cc2max = dmax_nn(cc2max, cc2);
+    if (qv != 0.0) ccqmax = dmax_nn(ccqmax, cc2);
+    else c2max = dmax_nn(c2max, c2);
   }
   // bottom face of the first row: v at nodes (j, k0) and (j+1, k0)
   __device__ __forceinline__ void bottom(double v00, double v10, const Chunk& C) {
@@ -149,7 +168,8 @@ struct DtAcc {
   // dt of the set (call only if at least one cell was added)
   __device__ __forceinline__ double dt(const Chunk& C, const DtParams& prm) const {
     const double dx = C.dx, dy = C.dy, vol = dx * dy;
-    const double ccmax = fmax(sqrt(cc2max), G_SMALL);
+    const double cs = sqrt(c2max);
+    const double ccmax = fmax(sqrt(dmax_nn(cs * cs, ccqmax)), G_SMALL);
     const double dum = fmax(dumax, G_SMALL * vol), dvm = fmax(dvmax, G_SMALL * vol);
     double dtct = div_fast_nz(prm.dtc_safe * fmin(dx, dy), ccmax);
     double dtut = div_fast_nz(prm.dtu_safe * 2.0 * vol, dum);
@@ -249,12 +269,22 @@ __device__ __forceinline__ void pdv_correct(D& dv, double r, double e, double ph
 
 // ------------------------------------------------ advec_cell (c.8)
 // a / b for b > 0: a zero numerator (the common case in quiescent regions)
-// is its own quotient (+0/b = +0, -0/b = -0), skipping the division.
+// is its own quotient (+0/b = +0, -0/b = -0), so the division may be
+// skipped.  Off by default: measured at 3840^2 the per-division branch
+// saves 0.018 ms/step on the bm deck but costs 0.10 ms/step on a fully
+// active flow (compare + branch per division, bench.py active_flow).
+#ifndef CLOVER_DIV_SKIP
+#define CLOVER_DIV_SKIP 0
+#endif
 template <class D>
 __device__ __forceinline__ double div_pos(D& dv, double a, double b) {
+#if CLOVER_DIV_SKIP
   double q = a;
   if (a != 0.0) q = dv(a, b);
   return q;
+#else
+  return dv(a, b);
+#endif
 }
 constexpr double ONE_BY_SIX = 1.0 / 6.0;
 

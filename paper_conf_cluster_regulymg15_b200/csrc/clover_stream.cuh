@@ -245,9 +245,9 @@ __device__ __forceinline__ bool visc_body(const Chunk& c, const CUtensorMap* __r
       I.u01 = rn[VF_U * VRW]; I.u11 = rn[VF_U * VRW + 1];
       I.v00 = rc[VF_V * VRW]; I.v10 = rc[VF_V * VRW + 1];
       I.v01 = rn[VF_V * VRW]; I.v11 = rn[VF_V * VRW + 1];
-      double qv, cc2;
-      visc_cell(dv, I, c, qv, cc2);
-      acc.add(I, c, cc2, left);
+      double qv, cc2, c2;
+      visc_cell(dv, I, c, qv, cc2, c2);
+      acc.add(I, c, qv, cc2, c2, left);
       store_at(c, q, K_CELL, j, k, i, EDGE && (ncol || near_wall_row(c, k)), qv);
       pcm = pc;
       pc = I.pt;

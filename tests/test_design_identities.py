@@ -58,3 +58,27 @@ def test_max_of_rounded_sqrt_is_sqrt_of_max():
         per_cell = np.max(np.fmax(np.sqrt(a), g))
         once = np.fmax(np.sqrt(np.max(a)), g)
         assert np.float64(per_cell).tobytes() == np.float64(once).tobytes()
+
+
+def test_max_of_rounded_square_of_sqrt_is_that_of_max():
+    # DtAcc: cells with q = 0 contribute cc2 = RN(RN(sqrt(c2))^2), a monotone
+    # function of c2, so max_i f(c2_i) == f(max_i c2_i); cells with q != 0
+    # keep their own cc2 and the two maxima combine exactly.
+    rng = np.random.default_rng(14)
+    for trial in range(300):
+        n = int(rng.integers(1, 64))
+        if trial % 3 == 0:  # near-ties in the last ulps
+            c2 = np.full(n, float(_logu(rng, 1e-30, 1e4, 1)[0]))
+            c2 = c2 * (1 + rng.integers(0, 16, n) * 2.0**-52)
+        else:
+            c2 = _logu(rng, 1e-30, 1e4, n)
+        q = np.where(rng.uniform(size=n) < 0.3, _logu(rng, 1e-12, 1.0, n), 0.0)
+        rho = _logu(rng, 1e-2, 1e2, n)
+        cs = np.sqrt(c2)
+        per_cell = np.max(cs * cs + 2.0 * q / rho)
+        z = q == 0.0
+        m1 = np.max(c2[z]) if z.any() else 0.0
+        s1 = np.sqrt(m1)
+        m2 = np.max((cs * cs + 2.0 * q / rho)[~z]) if (~z).any() else 0.0
+        once = max(s1 * s1, m2)
+        assert np.float64(per_cell).tobytes() == np.float64(once).tobytes()
