@@ -547,6 +547,19 @@ bool fuse_y_ok(const clover_ctx* ctx) {
 }
 
 // Enqueue kernel phases [0, nphase) of one step (7 = full step).
+// Serpentine segment order: each step kernel reads what the previous one
+// wrote, so alternate kernels run their row segments top-down (seg_y) and
+// start on the rows still in L2: visc_dt and sweep 1 reversed, the
+// Lagrangian phase and sweep 2 forward.  Measured at 3840^2: no gain
+// (visc_dt +0.004 ms, Lagrangian -0.002 ms), so off by default.
+#ifndef CLOVER_SERP
+#define CLOVER_SERP 0
+#endif
+static Chunk with_rev(Chunk c, int rev) {
+  c.rev = rev;
+  return c;
+}
+
 int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
   cudaStream_t st = ctx->work;
   int cur_prof_id = P_VISC_DT;
@@ -556,7 +569,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
   const int fold_fin = (nphase >= 2 && ctx->chunks.size() == 1 && ctx->nranks == 1) ? 1 : 0;
   if (nphase >= 1) {
     for (auto& cs : ctx->chunks) {
-      const Chunk& c = cs.c;
+      const Chunk c = with_rev(cs.c, CLOVER_SERP);  // top-down: sweep 2 wrote these rows last
       launch_step(ks_visc_dt, grid_cols(c.nx, c.ny, VKS), SB, st, c, cs.tm_visc, cs.buf[B_Q],
                   ctx->scal, ctx->dtp, cs.fix);
       STEP_LAUNCH_CHECK();
@@ -583,7 +596,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
   if (nphase >= 3) {
     cur_prof_id = P_LAGR;
     for (auto& cs : ctx->chunks) {
-      const Chunk& c = cs.c;
+      const Chunk c = with_rev(cs.c, 0);
       launch_step(ks_lagrangian, grid_strip(c.nx, LW, c.ny, LKS), SB, st, c, cs.tm_lag,
           cs.buf[B_D1], cs.buf[B_E1], cs.buf[B_U1], cs.buf[B_V1], cs.buf[B_FX], cs.buf[B_FY],
           ctx->scal, cs.fix);
@@ -612,7 +625,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
       if (nphase >= ph_cell) {
         cur_prof_id = sweep == 1 ? P_ADV_X1 : P_ADV_X2;
         for (auto& cs : ctx->chunks) {
-          const Chunk& c = cs.c;
+          const Chunk c = with_rev(cs.c, sweep == 1 ? CLOVER_SERP : 0);
           const dim3 g = grid_strip(c.nx + 1, XW, c.ny + 1, XKS);
           if (sweep == 1) {
             launch_step(ks_advec_x<1>, g, SB, st, c, cs.tm_x1, cs.buf[rout], cs.buf[eout],
@@ -642,7 +655,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
       if (nphase >= ph_cell) {
         cur_prof_id = sweep == 1 ? P_ADV_Y1 : P_ADV_Y2;
         for (auto& cs : ctx->chunks) {
-          const Chunk& c = cs.c;
+          const Chunk c = with_rev(cs.c, sweep == 1 ? CLOVER_SERP : 0);
           const dim3 gw(cdiv(c.nx + 2, SB), 2);
           const dim3 g = grid_strip(c.nx + 1, YW, c.ny + 1, YKS);
           const CUtensorMap& ta = sweep == 1 ? cs.tm_x1 : cs.tm_fy;
@@ -678,7 +691,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
     if (nphase >= ph_cell) {
       cur_prof_id = xdir ? (sweep == 1 ? P_CELL_X1 : P_CELL_X2) : (sweep == 1 ? P_CELL_Y1 : P_CELL_Y2);
       for (auto& cs : ctx->chunks) {
-        const Chunk& c = cs.c;
+        const Chunk c = with_rev(cs.c, sweep == 1 ? CLOVER_SERP : 0);
         const double* fx = cs.buf[B_FX];
         const double* fy = cs.buf[B_FY];
         if (xdir) {
@@ -716,7 +729,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
     if (nphase >= ph_cell + 1) {
       cur_prof_id = xdir ? (sweep == 1 ? P_MOM_X1 : P_MOM_X2) : (sweep == 1 ? P_MOM_Y1 : P_MOM_Y2);
       for (auto& cs : ctx->chunks) {
-        const Chunk& c = cs.c;
+        const Chunk c = with_rev(cs.c, sweep == 1 ? CLOVER_SERP : 0);
         if (xdir) {
           const dim3 g = grid_strip(c.nx + 1, MW_X, c.ny + 1, MKS);
           if (sweep == 1) {
@@ -1090,6 +1103,7 @@ int clover_init(const clover_grid* grid, const clover_state* states, int32_t nst
     const int64_t fe = field_elems(c.nx, c.ny, &c.pitch);
     c.wl = cs.cx == 0; c.wr = cs.cx == px - 1; c.wb = cs.cy == 0; c.wt = cs.cy == py - 1;
     c.face_cc = ctx->g.face_mirror == CLOVER_MIRROR_CELLCENTRE;
+    c.rev = 0;
     c.dx = dx; c.dy = dy; c.xmin = ctx->g.xmin; c.ymin = ctx->g.ymin;
     // correctly rounded reciprocals of the constant divisors (IEEE host division)
     c.rdx = 1.0 / dx; c.rdy = 1.0 / dy;

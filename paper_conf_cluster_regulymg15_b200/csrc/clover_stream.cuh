@@ -294,10 +294,10 @@ ks_visc_dt(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const int gw = blockIdx.x * (SB / 32) + warp;
   double dtw = G_BIG;
-  const int k0 = blockIdx.y * VKS + 1, k1 = min(k0 + VKS, c.ny + 1);
+  const int k0 = seg_y(c) * VKS + 1, k1 = min(k0 + VKS, c.ny + 1);
   if (gw * 32 < c.nx) {
     if (visc_seg<DivFast>(c, &tm, q, prm, gw, k0, k1, lane, ring[warp], bars[warp], dtw)) {
-      fix_push(fix, lane, gw, blockIdx.y);
+      fix_push(fix, lane, gw, (unsigned)seg_y(c));
       dtw = G_BIG;  // this warp's dt comes from the fixup
     }
   }
@@ -548,9 +548,9 @@ ks_lagrangian(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restric
   __shared__ __align__(8) unsigned long long bars[SB / 32][LSTG];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const int gw = blockIdx.x * (SB / 32) + w;
-  const int k0 = blockIdx.y * LKS + 1, k1 = min(k0 + LKS, c.ny + 1);
+  const int k0 = seg_y(c) * LKS + 1, k1 = min(k0 + LKS, c.ny + 1);
   if (lagr_seg<DivFast>(c, &tm, d1, e1, u1, v1, fx, fy, s, gw, k0, k1, lane, ring[w], bars[w]))
-    fix_push(fix, lane, gw, blockIdx.y);
+    fix_push(fix, lane, gw, (unsigned)seg_y(c));
 }
 
 __global__ void __launch_bounds__(SB)
@@ -643,9 +643,9 @@ ks_advec_cell_x(Chunk c, const double* __restrict__ rho, const double* __restric
   pdl_wait();
   const int lane = threadIdx.x & 31;
   const int gw = blockIdx.x * (SB / 32) + (threadIdx.x >> 5);
-  const int k0 = blockIdx.y * CKS + 1, k1 = min(k0 + CKS, c.ny + 1);
+  const int k0 = seg_y(c) * CKS + 1, k1 = min(k0 + CKS, c.ny + 1);
   if (advec_cell_x_body<SWEEP, DivFast>(c, rho, en, fx, fy, rho_out, en_out, mfx, gw, k0, k1, lane)) {
-    fix_push(fix, lane, gw, blockIdx.y);
+    fix_push(fix, lane, gw, (unsigned)seg_y(c));
   }
 }
 
@@ -758,10 +758,10 @@ ks_advec_cell_y(Chunk c, const double* __restrict__ rho, const double* __restric
   pdl_wait();
   const int lane = threadIdx.x & 31;
   const int gw = blockIdx.x * (SB / 32) + (threadIdx.x >> 5);
-  const int k0 = blockIdx.y * CKS_Y + 1, k1 = min(k0 + CKS_Y, c.ny + 1);
+  const int k0 = seg_y(c) * CKS_Y + 1, k1 = min(k0 + CKS_Y, c.ny + 1);
   if (y_interior(c, gw, k0, k1) ? advec_cell_y_body<SWEEP, DivFast, false>(c, rho, en, fx, fy, rho_out, en_out, mfy, gw, k0, k1, lane)
                                 : advec_cell_y_body<SWEEP, DivFast, true>(c, rho, en, fx, fy, rho_out, en_out, mfy, gw, k0, k1, lane)) {
-    fix_push(fix, lane, gw, blockIdx.y);
+    fix_push(fix, lane, gw, (unsigned)seg_y(c));
   }
 }
 
@@ -861,9 +861,9 @@ ks_advec_mom_x(Chunk c, const double* __restrict__ rho, const double* __restrict
   pdl_wait();
   const int lane = threadIdx.x & 31;
   const int gw = blockIdx.x * (SB / 32) + (threadIdx.x >> 5);
-  const int k0 = blockIdx.y * MKS + 1, k1 = min(k0 + MKS, c.ny + 2);
+  const int k0 = seg_y(c) * MKS + 1, k1 = min(k0 + MKS, c.ny + 2);
   if (advec_mom_x_body<SWEEP, DivFast>(c, rho, mfx, fy, uin, vin, uout, vout, gw, k0, k1, lane)) {
-    fix_push(fix, lane, gw, blockIdx.y);
+    fix_push(fix, lane, gw, (unsigned)seg_y(c));
   }
 }
 
@@ -1138,10 +1138,10 @@ ks_advec_x(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__
   __shared__ __align__(8) unsigned long long bars[SB / 32][XSTG];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const int gw = blockIdx.x * (SB / 32) + w;
-  const int k0 = blockIdx.y * XKS + 1, k1 = min(k0 + XKS, c.ny + 2);
+  const int k0 = seg_y(c) * XKS + 1, k1 = min(k0 + XKS, c.ny + 2);
   if (advec_x_seg<SWEEP, DivFast>(c, &tm, rho_out, en_out, uout, vout, gw, k0, k1, lane, ring[w],
                                    bars[w]))
-    fix_push(fix, lane, gw, blockIdx.y);
+    fix_push(fix, lane, gw, (unsigned)seg_y(c));
 }
 
 template <int SWEEP>
@@ -1255,10 +1255,10 @@ ks_advec_mom_y(Chunk c, const double* __restrict__ rho, const double* __restrict
   pdl_wait();
   const int lane = threadIdx.x & 31;
   const int gw = blockIdx.x * (SB / 32) + (threadIdx.x >> 5);
-  const int k0 = blockIdx.y * MKS_Y + 1, k1 = min(k0 + MKS_Y, c.ny + 2);
+  const int k0 = seg_y(c) * MKS_Y + 1, k1 = min(k0 + MKS_Y, c.ny + 2);
   if (y_interior(c, gw, k0, k1) ? advec_mom_y_body<SWEEP, DivFast, false>(c, rho, mfy, fx, uin, vin, uout, vout, gw, k0, k1, lane)
                                 : advec_mom_y_body<SWEEP, DivFast, true>(c, rho, mfy, fx, uin, vin, uout, vout, gw, k0, k1, lane)) {
-    fix_push(fix, lane, gw, blockIdx.y);
+    fix_push(fix, lane, gw, (unsigned)seg_y(c));
   }
 }
 
@@ -1533,10 +1533,10 @@ ks_advec_y(Chunk c, const __grid_constant__ CUtensorMap ta, const __grid_constan
   __shared__ __align__(8) unsigned long long bars[SB / 32][YRING];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const int gw = blockIdx.x * (SB / 32) + w;
-  const int k0 = blockIdx.y * YKS + 1, k1 = min(k0 + YKS, c.ny + 2);
+  const int k0 = seg_y(c) * YKS + 1, k1 = min(k0 + YKS, c.ny + 2);
   if (advec_y_seg<SWEEP, DivFast>(c, &ta, &tb, rho_out, en_out, mfy, uout, vout, gw, k0, k1, lane,
                                   ring[w], bars[w]))
-    fix_push(fix, lane, gw, blockIdx.y);
+    fix_push(fix, lane, gw, (unsigned)seg_y(c));
 }
 
 template <int SWEEP>
