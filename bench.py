@@ -331,9 +331,9 @@ def main():
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         cdeck = bm_deck(nx, ny)
-        rate, t = oracle_rate(cdeck, 2)
+        rate, t = oracle_rate(cdeck, 6)
         cpu = {"value": rate, "unit": UNIT, "cores": 1, "kind": "oracle",
-               "sample": f"first 2 steps of the same {nx}x{ny} bm workload, single-threaded "
+               "sample": f"first 6 steps of the same {nx}x{ny} bm workload, single-threaded "
                          f"C++ oracle (-O2), {t:.1f} s"}
 
     summ = sim.field_summary()
