@@ -148,11 +148,23 @@ dim3 grid_cols(int ncols, int nrows, int ks) { return dim3(cdiv(ncols, SB), cdiv
 dim3 grid_strip(int ncols, int width, int nrows, int ks) {
   return dim3(cdiv(cdiv(ncols, width), SB / 32), cdiv(nrows, ks));
 }
+// Rows per segment: the compile-time default, halved (down to MIN_KS) while
+// the grid would not fill the GPU once (148 SMs x SEG_FILL blocks): on small
+// meshes shorter segments halve each block's row chain, the latency that
+// bounds the step there.  Never below MIN_KS (fix-list capacity).
+constexpr int MIN_KS = 8;
+#ifndef CLOVER_SEG_FILL
+#define CLOVER_SEG_FILL 8
+#endif
+int seg_rows(int ks, int64_t colblocks, int nrows) {
+  while (ks > MIN_KS && colblocks * cdiv(nrows, ks) < 148 * CLOVER_SEG_FILL) ks /= 2;
+  return ks;
+}
 int64_t fix_capacity(int nx, int ny) {
-  const dim3 g[8] = {grid_cols(nx, ny, VKS),          grid_strip(nx, LW, ny, LKS),
+  const dim3 g[8] = {grid_cols(nx, ny, MIN_KS),          grid_strip(nx, LW, ny, MIN_KS),
                      grid_strip(nx, CW_X, ny, CKS),    grid_cols(nx, ny, CKS_Y),
                      grid_strip(nx + 1, MW_X, ny + 1, MKS), grid_cols(nx + 1, ny + 1, MKS_Y),
-                     grid_strip(nx + 1, XW, ny + 1, XKS), grid_strip(nx + 1, YW, ny + 1, YKS)};
+                     grid_strip(nx + 1, XW, ny + 1, MIN_KS), grid_strip(nx + 1, YW, ny + 1, MIN_KS)};
   int64_t m = 0;
   for (const dim3& d : g) m = std::max<int64_t>(m, (int64_t)d.x * d.y * (SB / 32));
   return m;
@@ -570,7 +582,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
   if (nphase >= 1) {
     for (auto& cs : ctx->chunks) {
       const Chunk c = with_rev(cs.c, CLOVER_SERP);  // top-down: sweep 2 wrote these rows last
-      launch_step(ks_visc_dt, grid_cols(c.nx, c.ny, VKS), SB, st, c, cs.tm_visc, cs.buf[B_Q],
+      launch_step(ks_visc_dt, grid_cols(c.nx, c.ny, c.vks), SB, st, c, cs.tm_visc, cs.buf[B_Q],
                   ctx->scal, ctx->dtp, cs.fix);
       STEP_LAUNCH_CHECK();
       launch_step(kf_visc_dt, FIX_BLOCKS, SB, st, c, cs.tm_visc, cs.buf[B_Q], ctx->scal, ctx->dtp,
@@ -597,7 +609,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
     cur_prof_id = P_LAGR;
     for (auto& cs : ctx->chunks) {
       const Chunk c = with_rev(cs.c, 0);
-      launch_step(ks_lagrangian, grid_strip(c.nx, LW, c.ny, LKS), SB, st, c, cs.tm_lag,
+      launch_step(ks_lagrangian, grid_strip(c.nx, LW, c.ny, c.lks), SB, st, c, cs.tm_lag,
           cs.buf[B_D1], cs.buf[B_E1], cs.buf[B_U1], cs.buf[B_V1], cs.buf[B_FX], cs.buf[B_FY],
           ctx->scal, cs.fix);
       STEP_LAUNCH_CHECK();
@@ -626,7 +638,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
         cur_prof_id = sweep == 1 ? P_ADV_X1 : P_ADV_X2;
         for (auto& cs : ctx->chunks) {
           const Chunk c = with_rev(cs.c, sweep == 1 ? CLOVER_SERP : 0);
-          const dim3 g = grid_strip(c.nx + 1, XW, c.ny + 1, XKS);
+          const dim3 g = grid_strip(c.nx + 1, XW, c.ny + 1, c.xks);
           if (sweep == 1) {
             launch_step(ks_advec_x<1>, g, SB, st, c, cs.tm_x1, cs.buf[rout], cs.buf[eout],
                         cs.buf[uout], cs.buf[vout], cs.fix);
@@ -657,7 +669,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
         for (auto& cs : ctx->chunks) {
           const Chunk c = with_rev(cs.c, sweep == 1 ? CLOVER_SERP : 0);
           const dim3 gw(cdiv(c.nx + 2, SB), 2);
-          const dim3 g = grid_strip(c.nx + 1, YW, c.ny + 1, YKS);
+          const dim3 g = grid_strip(c.nx + 1, YW, c.ny + 1, c.yks);
           const CUtensorMap& ta = sweep == 1 ? cs.tm_x1 : cs.tm_fy;
           const CUtensorMap& tb = sweep == 1 ? cs.tm_x1 : cs.tm_c4;
           if (sweep == 1) {
@@ -1104,6 +1116,10 @@ int clover_init(const clover_grid* grid, const clover_state* states, int32_t nst
     c.wl = cs.cx == 0; c.wr = cs.cx == px - 1; c.wb = cs.cy == 0; c.wt = cs.cy == py - 1;
     c.face_cc = ctx->g.face_mirror == CLOVER_MIRROR_CELLCENTRE;
     c.rev = 0;
+    c.vks = seg_rows(VKS, grid_cols(c.nx, c.ny, VKS).x, c.ny);
+    c.lks = seg_rows(LKS, grid_strip(c.nx, LW, c.ny, LKS).x, c.ny);
+    c.xks = seg_rows(XKS, grid_strip(c.nx + 1, XW, c.ny + 1, XKS).x, c.ny + 1);
+    c.yks = seg_rows(YKS, grid_strip(c.nx + 1, YW, c.ny + 1, YKS).x, c.ny + 1);
     c.dx = dx; c.dy = dy; c.xmin = ctx->g.xmin; c.ymin = ctx->g.ymin;
     // correctly rounded reciprocals of the constant divisors (IEEE host division)
     c.rdx = 1.0 / dx; c.rdy = 1.0 / dy;

@@ -294,7 +294,7 @@ ks_visc_dt(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const int gw = blockIdx.x * (SB / 32) + warp;
   double dtw = G_BIG;
-  const int k0 = seg_y(c) * VKS + 1, k1 = min(k0 + VKS, c.ny + 1);
+  const int k0 = seg_y(c) * c.vks + 1, k1 = min(k0 + c.vks, c.ny + 1);
   if (gw * 32 < c.nx) {
     if (visc_seg<DivFast>(c, &tm, q, prm, gw, k0, k1, lane, ring[warp], bars[warp], dtw)) {
       fix_push(fix, lane, gw, (unsigned)seg_y(c));
@@ -322,7 +322,7 @@ kf_visc_dt(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__
   // fin: single chunk on one rank -- the last block also finalises dt
   // (k_dt_finalize's work, once every contribution to the slot is in)
   fix_loop(
-      fix, VKS, c.ny + 1,
+      fix, c.vks, c.ny + 1,
       [&](int gw, int k0, int k1, int lane, int w) {
         double dtw;
         visc_seg<DivIEEE>(c, &tm, q, prm, gw, k0, k1, lane, ring[w], bars[w], dtw);
@@ -548,7 +548,7 @@ ks_lagrangian(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restric
   __shared__ __align__(8) unsigned long long bars[SB / 32][LSTG];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const int gw = blockIdx.x * (SB / 32) + w;
-  const int k0 = seg_y(c) * LKS + 1, k1 = min(k0 + LKS, c.ny + 1);
+  const int k0 = seg_y(c) * c.lks + 1, k1 = min(k0 + c.lks, c.ny + 1);
   if (lagr_seg<DivFast>(c, &tm, d1, e1, u1, v1, fx, fy, s, gw, k0, k1, lane, ring[w], bars[w]))
     fix_push(fix, lane, gw, (unsigned)seg_y(c));
 }
@@ -562,7 +562,7 @@ kf_lagrangian(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restric
   pdl_wait();
   __shared__ __align__(128) double ring[SB / 32][LSTG * LSLOT];
   __shared__ __align__(8) unsigned long long bars[SB / 32][LSTG];
-  fix_loop(fix, LKS, c.ny + 1, [&](int gw, int k0, int k1, int lane, int w) {
+  fix_loop(fix, c.lks, c.ny + 1, [&](int gw, int k0, int k1, int lane, int w) {
     lagr_seg<DivIEEE>(c, &tm, d1, e1, u1, v1, fx, fy, s, gw, k0, k1, lane, ring[w], bars[w]);
   });
 }
@@ -1138,7 +1138,7 @@ ks_advec_x(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__
   __shared__ __align__(8) unsigned long long bars[SB / 32][XSTG];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const int gw = blockIdx.x * (SB / 32) + w;
-  const int k0 = seg_y(c) * XKS + 1, k1 = min(k0 + XKS, c.ny + 2);
+  const int k0 = seg_y(c) * c.xks + 1, k1 = min(k0 + c.xks, c.ny + 2);
   if (advec_x_seg<SWEEP, DivFast>(c, &tm, rho_out, en_out, uout, vout, gw, k0, k1, lane, ring[w],
                                    bars[w]))
     fix_push(fix, lane, gw, (unsigned)seg_y(c));
@@ -1153,7 +1153,7 @@ kf_advec_x(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__
   pdl_wait();
   __shared__ __align__(128) double ring[SB / 32][XSTG * xslot<SWEEP>()];
   __shared__ __align__(8) unsigned long long bars[SB / 32][XSTG];
-  fix_loop(fix, XKS, c.ny + 2, [&](int gw, int k0, int k1, int lane, int w) {
+  fix_loop(fix, c.xks, c.ny + 2, [&](int gw, int k0, int k1, int lane, int w) {
     advec_x_seg<SWEEP, DivIEEE>(c, &tm, rho_out, en_out, uout, vout, gw, k0, k1, lane, ring[w],
                                  bars[w]);
   });
@@ -1533,7 +1533,7 @@ ks_advec_y(Chunk c, const __grid_constant__ CUtensorMap ta, const __grid_constan
   __shared__ __align__(8) unsigned long long bars[SB / 32][YRING];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const int gw = blockIdx.x * (SB / 32) + w;
-  const int k0 = seg_y(c) * YKS + 1, k1 = min(k0 + YKS, c.ny + 2);
+  const int k0 = seg_y(c) * c.yks + 1, k1 = min(k0 + c.yks, c.ny + 2);
   if (advec_y_seg<SWEEP, DivFast>(c, &ta, &tb, rho_out, en_out, mfy, uout, vout, gw, k0, k1, lane,
                                   ring[w], bars[w]))
     fix_push(fix, lane, gw, (unsigned)seg_y(c));
@@ -1548,7 +1548,7 @@ kf_advec_y(Chunk c, const __grid_constant__ CUtensorMap ta, const __grid_constan
   pdl_wait();
   __shared__ __align__(128) double ring[SB / 32][YRING * YL<SWEEP>::SLOT];
   __shared__ __align__(8) unsigned long long bars[SB / 32][YRING];
-  fix_loop(fix, YKS, c.ny + 2, [&](int gw, int k0, int k1, int lane, int w) {
+  fix_loop(fix, c.yks, c.ny + 2, [&](int gw, int k0, int k1, int lane, int w) {
     advec_y_seg<SWEEP, DivIEEE>(c, &ta, &tb, rho_out, en_out, mfy, uout, vout, gw, k0, k1, lane,
                                 ring[w], bars[w]);
   });
