@@ -10,8 +10,8 @@ import numpy as np
 import pytest
 
 from oracle import Oracle
-from workloads import (bm_deck, contact_deck, fuzz_deck, quiescent_deck, random_state_fields,
-                       symmetric_deck)
+from workloads import (bm_deck, contact_deck, fuzz_deck, point_deck, quiescent_deck,
+                       random_state_fields, symmetric_deck)
 
 pytestmark = pytest.mark.gpu
 
@@ -219,6 +219,23 @@ def test_ragged_meshes_bitwise(torch_cuda, shape):
     dts = o.step(6)
     assert np.array_equal(g.dt_history(1, 6), dts)
     assert_fields_equal(g, o, ctx=str(shape))
+
+
+@pytest.mark.parametrize("case", [(64, 64, None, None, 1, 1), (72, 56, 30, 21, 1, 1),
+                                  (96, 80, None, None, 2, 2)])
+def test_point_and_circle_decks_bitwise(torch_cuda, case):
+    """Point and circle state shapes: a point blast next to
+    a resting and a moving circle, on a dyadic and a ragged mesh and on 2x2
+    local chunks; fields, dt history and summary against the oracle."""
+    nx, ny, jp, kp, px, py = case
+    deck = point_deck(nx, ny, 25, jp=jp, kp=kp)
+    g, o = make_gpu(deck, px=px, py=py), Oracle(deck)
+    assert_fields_equal(g, o, ctx=f"point{case} init")
+    g.step(25)
+    dts = o.step(25)
+    assert np.array_equal(g.dt_history(1, 25), dts)
+    assert_fields_equal(g, o, ctx=f"point{case}")
+    assert_summary_close(g.field_summary(), o.field_summary())
 
 
 @pytest.mark.parametrize("smooth", [False, True])

@@ -19,7 +19,7 @@ import pytest
 
 import riemann
 from oracle import Oracle
-from workloads import (bm_deck, contact_deck, doubled_deck, fuzz_deck, quiescent_deck,
+from workloads import (bm_deck, contact_deck, doubled_deck, fuzz_deck, point_deck, quiescent_deck,
                        random_state_fields, sod_slab_deck, symmetric_deck, transpose_deck)
 
 GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
@@ -90,7 +90,8 @@ def test_p2_dt_rise_clamp():
 
 
 # ---------------------------------------------------------------- P3
-@pytest.mark.parametrize("deck", [bm_deck(64, end_step=20), fuzz_deck(3), fuzz_deck(7)])
+@pytest.mark.parametrize("deck", [bm_deck(64, end_step=20), fuzz_deck(3), fuzz_deck(7),
+                                  point_deck(64)])
 def test_p3_conservation(deck):
     """Volume exact, mass conserved to round-off (flux form, reflective walls),
     press = (gamma-1)*ie to round-off (EOS identity)."""
@@ -105,6 +106,40 @@ def test_p3_conservation(deck):
         assert _rel(s["mass"], s0["mass"]) < 1e-12
         # two sequential sums of ncell terms + 3 roundings per cell
         assert _rel(s["press"], GM1 * s["ie"]) < (ncell + 4) * eps
+
+
+def test_p1_point_and_circle_painting():
+    """generate_chunk's point and circle shapes: the point
+    state covers exactly the one cell whose lower-left vertex is the point;
+    a circle covers the cells whose centre lies within its radius (counted
+    here from the cell-centre coordinates (j - 1/2) dx in closed form); a
+    moving circle's velocity sits on exactly the corner nodes of its cells;
+    the step-0 mass is the closed-form sum over the painted areas."""
+    n = 64
+    d = point_deck(n)
+    o = Oracle(d)
+    rho, e = o.read("density0"), o.read("energy0")
+    u, v = o.read("xvel0"), o.read("yvel0")
+    hot = np.argwhere(e == 20.0)
+    assert hot.tolist() == [[n // 2, n // 2]]  # 0-based (k, j) of cell (33, 33)
+    dx = 10.0 / n
+    xc = (np.arange(1, n + 1) - 0.5) * dx  # exact on this dyadic mesh
+    X, Y = np.meshgrid(xc, xc)
+    dense = (X - 2.6) ** 2 + (Y - 7.3) ** 2 <= 1.1 ** 2
+    light = (X - 7.2) ** 2 + (Y - 3.1) ** 2 <= 0.9 ** 2
+    # no cell centre sits within rounding of either circle's edge
+    for cx, cy, r in ((2.6, 7.3, 1.1), (7.2, 3.1, 0.9)):
+        assert np.abs(np.hypot(X - cx, Y - cy) - r).min() > 1e-9
+    assert np.array_equal(rho == 2.5, dense)
+    assert np.array_equal(rho == 0.5, light)
+    node = np.zeros((n + 1, n + 1), bool)
+    for k, j in np.argwhere(light):
+        node[k:k + 2, j:j + 2] = True
+    assert np.array_equal(u == 0.3, node) and np.array_equal(v == -0.2, node)
+    area = dx * dx
+    n_dense, n_light = int(dense.sum()), int(light.sum())
+    mass = (1.0 * (n * n - n_dense - n_light) + 2.5 * n_dense + 0.5 * n_light) * area
+    assert _rel(o.field_summary()["mass"], mass) < 1e-14
 
 
 def test_p3_total_energy_drift_small():

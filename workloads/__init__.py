@@ -59,6 +59,30 @@ def symmetric_deck(n: int = 64, end_step: int = 20, **kw):
     return d
 
 
+def point_deck(nx: int = 64, ny: int | None = None, end_step: int = 20, jp: int | None = None,
+               kp: int | None = None):
+    """Geometry deck (the reference's circle and point state
+    shapes): background rho=1 e=1; a point state (rho=1, e=20) painted on the
+    one cell whose lower-left vertex is the point, placed on vertex (jp, kp)
+    (1-based; default the domain centre) with the vertex coordinate computed
+    as generate_chunk does, xmin + dx*(jp-1); a resting dense circle
+    (rho=2.5, e=0.5, r=1.1 about (2.6, 7.3)) and a moving light circle
+    (rho=0.5, e=1.5, u=0.3, v=-0.2, r=0.9 about (7.2, 3.1)), both clear of the
+    walls (reading A16)."""
+    ny = nx if ny is None else ny
+    d = bm_deck(nx, ny, end_step)
+    d["max_timestep"] = 0.04
+    jp = nx // 2 + 1 if jp is None else jp
+    kp = ny // 2 + 1 if kp is None else kp
+    dx, dy = (10.0 - 0.0) / float(nx), (10.0 - 0.0) / float(ny)
+    px, py = 0.0 + dx * float(jp - 1), 0.0 + dy * float(kp - 1)
+    d["states"] = [_state(1.0, 1.0),
+                   _state(2.5, 0.5, geometry="circle", xmin=2.6, ymin=7.3, radius=1.1),
+                   _state(0.5, 1.5, 0.3, -0.2, geometry="circle", xmin=7.2, ymin=3.1, radius=0.9),
+                   _state(1.0, 20.0, geometry="point", xmin=px, ymin=py)]
+    return d
+
+
 def quiescent_deck(n: int = 64, density=1.0, energy=2.5, end_step: int = 20):
     """One uniform state at rest."""
     d = bm_deck(n, n, end_step)
