@@ -160,11 +160,30 @@ int seg_rows(int ks, int64_t colblocks, int nrows) {
   while (ks > MIN_KS && colblocks * cdiv(nrows, ks) < 148 * CLOVER_SEG_FILL) ks /= 2;
   return ks;
 }
+// Segment rows of a kernel grid whose first nb segments have ks rows and
+// the rest ks/2 (seg_rows_of).
+int seg_count(int ks, int nb, int rows) {
+  if ((int64_t)nb * ks >= rows) return cdiv(rows, ks);
+  return nb + cdiv(rows - nb * ks, ks / 2);
+}
+// Full-height segments: all but about one wave of blocks (slots resident
+// blocks on the GPU, colblocks blocks per segment row), which run at half
+// height so the kernel's tail is half a segment.  CLOVER_TAIL=0: all full.
+#ifndef CLOVER_TAIL
+#define CLOVER_TAIL 1
+#endif
+int tail_nb(int ks, int64_t colblocks, int rows, int64_t slots) {
+  if (!CLOVER_TAIL || ks < 8 || slots <= 0) return 0x3fffffff;
+  const int64_t tail_rows = cdiv((int)std::min<int64_t>(slots, 1 << 30), (int)colblocks) * (int64_t)(ks / 2);
+  if (rows <= tail_rows) return 0;
+  return (int)((rows - tail_rows) / ks);
+}
 int64_t fix_capacity(int nx, int ny) {
-  const dim3 g[8] = {grid_cols(nx, ny, MIN_KS),          grid_strip(nx, LW, ny, MIN_KS),
+  // (adaptive segments: at least MIN_KS rows, half that in the tail)
+  const dim3 g[8] = {grid_cols(nx, ny, MIN_KS / 2),          grid_strip(nx, LW, ny, MIN_KS / 2),
                      grid_strip(nx, CW_X, ny, CKS),    grid_cols(nx, ny, CKS_Y),
                      grid_strip(nx + 1, MW_X, ny + 1, MKS), grid_cols(nx + 1, ny + 1, MKS_Y),
-                     grid_strip(nx + 1, XW, ny + 1, MIN_KS), grid_strip(nx + 1, YW, ny + 1, MIN_KS)};
+                     grid_strip(nx + 1, XW, ny + 1, MIN_KS / 2), grid_strip(nx + 1, YW, ny + 1, MIN_KS / 2)};
   int64_t m = 0;
   for (const dim3& d : g) m = std::max<int64_t>(m, (int64_t)d.x * d.y * (SB / 32));
   return m;
@@ -582,7 +601,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
   if (nphase >= 1) {
     for (auto& cs : ctx->chunks) {
       const Chunk c = with_rev(cs.c, CLOVER_SERP);  // top-down: sweep 2 wrote these rows last
-      launch_step(ks_visc_dt, grid_cols(c.nx, c.ny, c.vks), SB, st, c, cs.tm_visc, cs.buf[B_Q],
+      launch_step(ks_visc_dt, dim3(grid_cols(c.nx, c.ny, c.vks).x, seg_count(c.vks, c.vnb, c.ny)), SB, st, c, cs.tm_visc, cs.buf[B_Q],
                   ctx->scal, ctx->dtp, cs.fix);
       STEP_LAUNCH_CHECK();
       launch_step(kf_visc_dt, FIX_BLOCKS, SB, st, c, cs.tm_visc, cs.buf[B_Q], ctx->scal, ctx->dtp,
@@ -609,7 +628,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
     cur_prof_id = P_LAGR;
     for (auto& cs : ctx->chunks) {
       const Chunk c = with_rev(cs.c, 0);
-      launch_step(ks_lagrangian, grid_strip(c.nx, LW, c.ny, c.lks), SB, st, c, cs.tm_lag,
+      launch_step(ks_lagrangian, dim3(grid_strip(c.nx, LW, c.ny, c.lks).x, seg_count(c.lks, c.lnb, c.ny)), SB, st, c, cs.tm_lag,
           cs.buf[B_D1], cs.buf[B_E1], cs.buf[B_U1], cs.buf[B_V1], cs.buf[B_FX], cs.buf[B_FY],
           ctx->scal, cs.fix);
       STEP_LAUNCH_CHECK();
@@ -638,7 +657,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
         cur_prof_id = sweep == 1 ? P_ADV_X1 : P_ADV_X2;
         for (auto& cs : ctx->chunks) {
           const Chunk c = with_rev(cs.c, sweep == 1 ? CLOVER_SERP : 0);
-          const dim3 g = grid_strip(c.nx + 1, XW, c.ny + 1, c.xks);
+          const dim3 g(grid_strip(c.nx + 1, XW, c.ny + 1, c.xks).x, seg_count(c.xks, c.xnb, c.ny + 1));
           if (sweep == 1) {
             launch_step(ks_advec_x<1>, g, SB, st, c, cs.tm_x1, cs.buf[rout], cs.buf[eout],
                         cs.buf[uout], cs.buf[vout], cs.fix);
@@ -669,7 +688,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
         for (auto& cs : ctx->chunks) {
           const Chunk c = with_rev(cs.c, sweep == 1 ? CLOVER_SERP : 0);
           const dim3 gw(cdiv(c.nx + 2, SB), 2);
-          const dim3 g = grid_strip(c.nx + 1, YW, c.ny + 1, c.yks);
+          const dim3 g(grid_strip(c.nx + 1, YW, c.ny + 1, c.yks).x, seg_count(c.yks, c.ynb, c.ny + 1));
           const CUtensorMap& ta = sweep == 1 ? cs.tm_x1 : cs.tm_fy;
           const CUtensorMap& tb = sweep == 1 ? cs.tm_x1 : cs.tm_c4;
           if (sweep == 1) {
@@ -1120,6 +1139,20 @@ int clover_init(const clover_grid* grid, const clover_state* states, int32_t nst
     c.lks = seg_rows(LKS, grid_strip(c.nx, LW, c.ny, LKS).x, c.ny);
     c.xks = seg_rows(XKS, grid_strip(c.nx + 1, XW, c.ny + 1, XKS).x, c.ny + 1);
     c.yks = seg_rows(YKS, grid_strip(c.nx + 1, YW, c.ny + 1, YKS).x, c.ny + 1);
+    {
+      int nsm = 148, b[4] = {0, 0, 0, 0}, dev = 0;
+      cudaGetDevice(&dev);
+      cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b[0], ks_visc_dt, SB, 0);
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b[1], ks_lagrangian, SB, 0);
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b[2], ks_advec_x<1>, SB, 0);
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b[3], ks_advec_y<1>, SB, 0);
+      c.vnb = tail_nb(c.vks, grid_cols(c.nx, c.ny, c.vks).x, c.ny, (int64_t)nsm * b[0]);
+      c.lnb = tail_nb(c.lks, grid_strip(c.nx, LW, c.ny, c.lks).x, c.ny, (int64_t)nsm * b[1]);
+      c.xnb = tail_nb(c.xks, grid_strip(c.nx + 1, XW, c.ny + 1, c.xks).x, c.ny + 1, (int64_t)nsm * b[2]);
+      c.ynb = tail_nb(c.yks, grid_strip(c.nx + 1, YW, c.ny + 1, c.yks).x, c.ny + 1, (int64_t)nsm * b[3]);
+      cudaGetLastError();
+    }
     c.dx = dx; c.dy = dy; c.xmin = ctx->g.xmin; c.ymin = ctx->g.ymin;
     // correctly rounded reciprocals of the constant divisors (IEEE host division)
     c.rdx = 1.0 / dx; c.rdy = 1.0 / dy;

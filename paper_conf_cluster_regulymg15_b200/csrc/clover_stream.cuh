@@ -130,7 +130,7 @@ __device__ __forceinline__ void fix_push(FixSlot f, int lane, unsigned gw, unsig
     f.e[n] = make_uint2(gw, seg);
   }
 }
-// Fixup driver: every flagged segment of ks rows is redone one row per warp
+// Fixup driver: every flagged segment (seg_rows_of) is redone one row per warp
 // (row-parallel, so the fixup's latency is one row, not one segment); the
 // last block to finish resets the list.  run(gw, k0, k1, lane, w) with
 // k1 = k0 + 1; rows at or beyond `lim` are skipped.
@@ -138,14 +138,18 @@ struct NoLast {
   __device__ void operator()() const {}
 };
 template <class Run, class Last = NoLast>
-__device__ __forceinline__ void fix_loop(FixSlot f, int ks, int lim, Run&& run, Last last = {}) {
+__device__ __forceinline__ void fix_loop(FixSlot f, int ks, int nb, int lim, Run&& run,
+                                         Last last = {}) {
   const unsigned n = *(volatile unsigned*)f.hdr;
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const unsigned items = n * (unsigned)ks;
   for (unsigned it = blockIdx.x * (SB / 32) + w; it < items; it += gridDim.x * (SB / 32)) {
     const uint2 t = f.e[it / ks];
-    const int k0 = (int)t.y * ks + 1 + (int)(it % ks);
-    if (k0 < lim) run((int)t.x, k0, k0 + 1, lane, w);
+    int ks0, len;
+    seg_rows_of((int)t.y, ks, nb, ks0, len);
+    const int r = (int)(it % ks);
+    const int k0 = ks0 + r;
+    if (r < len && k0 < lim) run((int)t.x, k0, k0 + 1, lane, w);
   }
   __syncthreads();
   if (threadIdx.x == 0) {
@@ -294,7 +298,9 @@ ks_visc_dt(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const int gw = blockIdx.x * (SB / 32) + warp;
   double dtw = G_BIG;
-  const int k0 = seg_y(c) * c.vks + 1, k1 = min(k0 + c.vks, c.ny + 1);
+  int k0, len;
+  seg_rows_of(seg_y(c), c.vks, c.vnb, k0, len);
+  const int k1 = min(k0 + len, c.ny + 1);
   if (gw * 32 < c.nx) {
     if (visc_seg<DivFast>(c, &tm, q, prm, gw, k0, k1, lane, ring[warp], bars[warp], dtw)) {
       fix_push(fix, lane, gw, (unsigned)seg_y(c));
@@ -322,7 +328,7 @@ kf_visc_dt(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__
   // fin: single chunk on one rank -- the last block also finalises dt
   // (k_dt_finalize's work, once every contribution to the slot is in)
   fix_loop(
-      fix, c.vks, c.ny + 1,
+      fix, c.vks, c.vnb, c.ny + 1,
       [&](int gw, int k0, int k1, int lane, int w) {
         double dtw;
         visc_seg<DivIEEE>(c, &tm, q, prm, gw, k0, k1, lane, ring[w], bars[w], dtw);
@@ -548,7 +554,9 @@ ks_lagrangian(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restric
   __shared__ __align__(8) unsigned long long bars[SB / 32][LSTG];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const int gw = blockIdx.x * (SB / 32) + w;
-  const int k0 = seg_y(c) * c.lks + 1, k1 = min(k0 + c.lks, c.ny + 1);
+  int k0, len;
+  seg_rows_of(seg_y(c), c.lks, c.lnb, k0, len);
+  const int k1 = min(k0 + len, c.ny + 1);
   if (lagr_seg<DivFast>(c, &tm, d1, e1, u1, v1, fx, fy, s, gw, k0, k1, lane, ring[w], bars[w]))
     fix_push(fix, lane, gw, (unsigned)seg_y(c));
 }
@@ -562,7 +570,7 @@ kf_lagrangian(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restric
   pdl_wait();
   __shared__ __align__(128) double ring[SB / 32][LSTG * LSLOT];
   __shared__ __align__(8) unsigned long long bars[SB / 32][LSTG];
-  fix_loop(fix, c.lks, c.ny + 1, [&](int gw, int k0, int k1, int lane, int w) {
+  fix_loop(fix, c.lks, c.lnb, c.ny + 1, [&](int gw, int k0, int k1, int lane, int w) {
     lagr_seg<DivIEEE>(c, &tm, d1, e1, u1, v1, fx, fy, s, gw, k0, k1, lane, ring[w], bars[w]);
   });
 }
@@ -657,7 +665,7 @@ kf_advec_cell_x(Chunk c, const double* __restrict__ rho, const double* __restric
                 double* __restrict__ mfx, FixSlot fix) {
   pdl_trigger();
   pdl_wait();
-  fix_loop(fix, CKS, c.ny + 1, [&](int gw, int k0, int k1, int lane, int) {
+  fix_loop(fix, CKS, 0x7fffffff, c.ny + 1, [&](int gw, int k0, int k1, int lane, int) {
     advec_cell_x_body<SWEEP, DivIEEE>(c, rho, en, fx, fy, rho_out, en_out, mfx, gw, k0, k1, lane);
   });
 }
@@ -773,7 +781,7 @@ kf_advec_cell_y(Chunk c, const double* __restrict__ rho, const double* __restric
                 double* __restrict__ mfy, FixSlot fix) {
   pdl_trigger();
   pdl_wait();
-  fix_loop(fix, CKS_Y, c.ny + 1, [&](int gw, int k0, int k1, int lane, int) {
+  fix_loop(fix, CKS_Y, 0x7fffffff, c.ny + 1, [&](int gw, int k0, int k1, int lane, int) {
     advec_cell_y_body<SWEEP, DivIEEE, true>(c, rho, en, fx, fy, rho_out, en_out, mfy, gw, k0, k1, lane);
   });
 }
@@ -875,7 +883,7 @@ kf_advec_mom_x(Chunk c, const double* __restrict__ rho, const double* __restrict
                double* __restrict__ vout, FixSlot fix) {
   pdl_trigger();
   pdl_wait();
-  fix_loop(fix, MKS, c.ny + 2, [&](int gw, int k0, int k1, int lane, int) {
+  fix_loop(fix, MKS, 0x7fffffff, c.ny + 2, [&](int gw, int k0, int k1, int lane, int) {
     advec_mom_x_body<SWEEP, DivIEEE>(c, rho, mfx, fy, uin, vin, uout, vout, gw, k0, k1, lane);
   });
 }
@@ -1138,7 +1146,9 @@ ks_advec_x(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__
   __shared__ __align__(8) unsigned long long bars[SB / 32][XSTG];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const int gw = blockIdx.x * (SB / 32) + w;
-  const int k0 = seg_y(c) * c.xks + 1, k1 = min(k0 + c.xks, c.ny + 2);
+  int k0, len;
+  seg_rows_of(seg_y(c), c.xks, c.xnb, k0, len);
+  const int k1 = min(k0 + len, c.ny + 2);
   if (advec_x_seg<SWEEP, DivFast>(c, &tm, rho_out, en_out, uout, vout, gw, k0, k1, lane, ring[w],
                                    bars[w]))
     fix_push(fix, lane, gw, (unsigned)seg_y(c));
@@ -1153,7 +1163,7 @@ kf_advec_x(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__
   pdl_wait();
   __shared__ __align__(128) double ring[SB / 32][XSTG * xslot<SWEEP>()];
   __shared__ __align__(8) unsigned long long bars[SB / 32][XSTG];
-  fix_loop(fix, c.xks, c.ny + 2, [&](int gw, int k0, int k1, int lane, int w) {
+  fix_loop(fix, c.xks, c.xnb, c.ny + 2, [&](int gw, int k0, int k1, int lane, int w) {
     advec_x_seg<SWEEP, DivIEEE>(c, &tm, rho_out, en_out, uout, vout, gw, k0, k1, lane, ring[w],
                                  bars[w]);
   });
@@ -1270,7 +1280,7 @@ kf_advec_mom_y(Chunk c, const double* __restrict__ rho, const double* __restrict
                double* __restrict__ vout, FixSlot fix) {
   pdl_trigger();
   pdl_wait();
-  fix_loop(fix, MKS_Y, c.ny + 2, [&](int gw, int k0, int k1, int lane, int) {
+  fix_loop(fix, MKS_Y, 0x7fffffff, c.ny + 2, [&](int gw, int k0, int k1, int lane, int) {
     advec_mom_y_body<SWEEP, DivIEEE, true>(c, rho, mfy, fx, uin, vin, uout, vout, gw, k0, k1, lane);
   });
 }
@@ -1533,7 +1543,9 @@ ks_advec_y(Chunk c, const __grid_constant__ CUtensorMap ta, const __grid_constan
   __shared__ __align__(8) unsigned long long bars[SB / 32][YRING];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const int gw = blockIdx.x * (SB / 32) + w;
-  const int k0 = seg_y(c) * c.yks + 1, k1 = min(k0 + c.yks, c.ny + 2);
+  int k0, len;
+  seg_rows_of(seg_y(c), c.yks, c.ynb, k0, len);
+  const int k1 = min(k0 + len, c.ny + 2);
   if (advec_y_seg<SWEEP, DivFast>(c, &ta, &tb, rho_out, en_out, mfy, uout, vout, gw, k0, k1, lane,
                                   ring[w], bars[w]))
     fix_push(fix, lane, gw, (unsigned)seg_y(c));
@@ -1548,7 +1560,7 @@ kf_advec_y(Chunk c, const __grid_constant__ CUtensorMap ta, const __grid_constan
   pdl_wait();
   __shared__ __align__(128) double ring[SB / 32][YRING * YL<SWEEP>::SLOT];
   __shared__ __align__(8) unsigned long long bars[SB / 32][YRING];
-  fix_loop(fix, c.yks, c.ny + 2, [&](int gw, int k0, int k1, int lane, int w) {
+  fix_loop(fix, c.yks, c.ynb, c.ny + 2, [&](int gw, int k0, int k1, int lane, int w) {
     advec_y_seg<SWEEP, DivIEEE>(c, &ta, &tb, rho_out, en_out, mfy, uout, vout, gw, k0, k1, lane,
                                 ring[w], bars[w]);
   });
