@@ -164,26 +164,34 @@ int seg_rows(int ks, int64_t colblocks, int nrows) {
 // the rest ks/2 (seg_rows_of).
 int seg_count(int ks, int nb, int rows) {
   if ((int64_t)nb * ks >= rows) return cdiv(rows, ks);
-  return nb + cdiv(rows - nb * ks, ks / 2);
+  return nb + cdiv(rows - nb * ks, ks / CLOVER_TAIL_DIV);
 }
-// Full-height segments: all but about one wave of blocks (slots resident
-// blocks on the GPU, colblocks blocks per segment row), which run at half
-// height so the kernel's tail is half a segment.  CLOVER_TAIL=0: all full.
+// Full-height segments: all but about CLOVER_TAIL_WAVES waves of blocks
+// (slots resident blocks on the GPU, colblocks blocks per segment row),
+// which run at 1/CLOVER_TAIL_DIV height so the kernel's tail shrinks.
+// Measured at 3840^2 (step ms, one box): none 0.965, 1 wave at 1/2 0.931,
+// 2 waves at 1/2 0.925, 1 wave at 1/4 0.948, 2 waves at 1/4 0.938.
+// CLOVER_TAIL=0: all full height.
 #ifndef CLOVER_TAIL
 #define CLOVER_TAIL 1
 #endif
+#ifndef CLOVER_TAIL_WAVES
+#define CLOVER_TAIL_WAVES 2
+#endif
 int tail_nb(int ks, int64_t colblocks, int rows, int64_t slots) {
-  if (!CLOVER_TAIL || ks < 8 || slots <= 0) return 0x3fffffff;
-  const int64_t tail_rows = cdiv((int)std::min<int64_t>(slots, 1 << 30), (int)colblocks) * (int64_t)(ks / 2);
+  if (!CLOVER_TAIL || ks < 4 * CLOVER_TAIL_DIV || slots <= 0) return 0x3fffffff;
+  const int64_t tail_rows = (int64_t)CLOVER_TAIL_WAVES *
+                            cdiv((int)std::min<int64_t>(slots, 1 << 30), (int)colblocks) *
+                            (int64_t)(ks / CLOVER_TAIL_DIV);
   if (rows <= tail_rows) return 0;
   return (int)((rows - tail_rows) / ks);
 }
 int64_t fix_capacity(int nx, int ny) {
-  // (adaptive segments: at least MIN_KS rows, half that in the tail)
-  const dim3 g[8] = {grid_cols(nx, ny, MIN_KS / 2),          grid_strip(nx, LW, ny, MIN_KS / 2),
+  // (adaptive segments: tail segments have at least 4 rows, see tail_nb)
+  const dim3 g[8] = {grid_cols(nx, ny, 4),          grid_strip(nx, LW, ny, 4),
                      grid_strip(nx, CW_X, ny, CKS),    grid_cols(nx, ny, CKS_Y),
                      grid_strip(nx + 1, MW_X, ny + 1, MKS), grid_cols(nx + 1, ny + 1, MKS_Y),
-                     grid_strip(nx + 1, XW, ny + 1, MIN_KS / 2), grid_strip(nx + 1, YW, ny + 1, MIN_KS / 2)};
+                     grid_strip(nx + 1, XW, ny + 1, 4), grid_strip(nx + 1, YW, ny + 1, 4)};
   int64_t m = 0;
   for (const dim3& d : g) m = std::max<int64_t>(m, (int64_t)d.x * d.y * (SB / 32));
   return m;
