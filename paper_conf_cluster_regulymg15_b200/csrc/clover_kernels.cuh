@@ -211,16 +211,21 @@ __global__ void k_dt_finalize(StepScalars* __restrict__ s, double* __restrict__ 
 // PdV predictor (predict=T) + ideal_gas(predict): half-step pressure of one
 // cell from its 4 node velocities (a,b = left face nodes bottom/top;
 // c,d = right face; va,vb = bottom face nodes left/right; vc,vd = top face).
+// The y-face flux terms of the predictor: the top face of row k is the
+// bottom face of row k+1, the same expression of the same two node
+// velocities, so the row-streaming kernel carries it (pdv_face_pred).
+__device__ __forceinline__ double pdv_face_pred(double a, double b, double d, double dt) {
+  return (d * (a + b + a + b)) * 0.25 * dt * 0.5;
+}
 template <class D>
-__device__ __forceinline__ double pdv_predict_pressure(D& dv, double r, double e, double q,
-                                                       double ua, double ub, double uc, double ud,
-                                                       double va, double vb, double vc, double vd,
-                                                       double dx, double dy, double rvol, double dt) {
+__device__ __forceinline__ double pdv_predict_pressure_bt(D& dv, double r, double e, double q,
+                                                          double ua, double ub, double uc,
+                                                          double ud, double bottom_flux,
+                                                          double top_flux, double dx, double dy,
+                                                          double rvol, double dt) {
   const double vol = dx * dy;
-  double left_flux = (dy * (ua + ub + ua + ub)) * 0.25 * dt * 0.5;
-  double right_flux = (dy * (uc + ud + uc + ud)) * 0.25 * dt * 0.5;
-  double bottom_flux = (dx * (va + vb + va + vb)) * 0.25 * dt * 0.5;
-  double top_flux = (dx * (vc + vd + vc + vd)) * 0.25 * dt * 0.5;
+  double left_flux = pdv_face_pred(ua, ub, dy, dt);
+  double right_flux = pdv_face_pred(uc, ud, dy, dt);
   double total_flux = right_flux - left_flux + top_flux - bottom_flux;
   double volume_change = dv.nz(vol, vol + total_flux);
   double recip_volume = rvol;  // = RN(1.0/vol), precomputed
@@ -229,6 +234,14 @@ __device__ __forceinline__ double pdv_predict_pressure(D& dv, double r, double e
   double e1p = e - energy_change;
   double d1p = r * volume_change;
   return eos_pressure(d1p, e1p);
+}
+template <class D>
+__device__ __forceinline__ double pdv_predict_pressure(D& dv, double r, double e, double q,
+                                                       double ua, double ub, double uc, double ud,
+                                                       double va, double vb, double vc, double vd,
+                                                       double dx, double dy, double rvol, double dt) {
+  return pdv_predict_pressure_bt(dv, r, e, q, ua, ub, uc, ud, pdv_face_pred(va, vb, dx, dt),
+                                 pdv_face_pred(vc, vd, dx, dt), dx, dy, rvol, dt);
 }
 
 // accelerate (c.6) at one node: cells ordered (j-1,k-1), (j,k-1), (j,k), (j-1,k).
@@ -249,22 +262,33 @@ __device__ __forceinline__ void accelerate_node(D& dv, const double* rr, const d
 }
 
 // PdV corrector (predict=F) for one cell; returns energy1, density1.
+// corrector face flux from a face's summed velocities (the top face of row
+// k is the bottom face of row k+1: carried by the kernel)
+__device__ __forceinline__ double pdv_face_corr(double sum, double d, double dt) {
+  return (d * sum) * 0.25 * dt;
+}
 template <class D>
-__device__ __forceinline__ void pdv_correct(D& dv, double r, double e, double ph, double q,
-                                            double lsum, double rsum, double bsum, double tsum,
-                                            double dx, double dy, double rvol, double dt, double& e1v,
-                                            double& d1v) {
+__device__ __forceinline__ void pdv_correct_bt(D& dv, double r, double e, double ph, double q,
+                                               double lsum, double rsum, double bottom_flux,
+                                               double top_flux, double dx, double dy, double rvol,
+                                               double dt, double& e1v, double& d1v) {
   const double vol = dx * dy;
-  double left_flux = (dy * lsum) * 0.25 * dt;
-  double right_flux = (dy * rsum) * 0.25 * dt;
-  double bottom_flux = (dx * bsum) * 0.25 * dt;
-  double top_flux = (dx * tsum) * 0.25 * dt;
+  double left_flux = pdv_face_corr(lsum, dy, dt);
+  double right_flux = pdv_face_corr(rsum, dy, dt);
   double total_flux = right_flux - left_flux + top_flux - bottom_flux;
   double volume_change = dv.nz(vol, vol + total_flux);
   double recip_volume = rvol;  // = RN(1.0/vol), precomputed
   double energy_change = (dv(ph, r) + dv(q, r)) * total_flux * recip_volume;
   e1v = e - energy_change;
   d1v = r * volume_change;
+}
+template <class D>
+__device__ __forceinline__ void pdv_correct(D& dv, double r, double e, double ph, double q,
+                                            double lsum, double rsum, double bsum, double tsum,
+                                            double dx, double dy, double rvol, double dt, double& e1v,
+                                            double& d1v) {
+  pdv_correct_bt(dv, r, e, ph, q, lsum, rsum, pdv_face_corr(bsum, dx, dt),
+                 pdv_face_corr(tsum, dx, dt), dx, dy, rvol, dt, e1v, d1v);
 }
 
 // ------------------------------------------------ advec_cell (c.8)

@@ -427,25 +427,48 @@ __device__ __forceinline__ bool lagr_body(const Chunk& c, const CUtensorMap* __r
   // ring row 0 takes the mirror of row 1 (update_halo{pressure}), which is
   // the predictor evaluated on row 1's inputs.
   double ph_m, phl_m;
+  // interior body: the predictor's top y-face flux of row k is the bottom
+  // one of row k+1 (same expression, same node velocities): carried
+  double tfp = 0.0;
   {
     const int kp = (EDGE && c.wb && k0 == 1) ? 1 : k0 - 1;
     for (int r = r_first; r <= kp + 1; ++r) wait_row(r);
     double ph = 0.0;
-    if (colok) ph = predict(row(kp), row(kp + 1));
+    if constexpr (EDGE) {
+      if (colok) ph = predict(row(kp), row(kp + 1));
+    } else {
+      const double* a = row(kp);
+      const double* b = row(kp + 1);
+      tfp = pdv_face_pred(b[LF_V * LRW], b[LF_V * LRW + 1], dx, dt);
+      ph = pdv_predict_pressure_bt(dv, a[LF_R * LRW], a[LF_E * LRW], a[LF_Q * LRW], a[LF_U * LRW],
+                                   b[LF_U * LRW], a[LF_U * LRW + 1], b[LF_U * LRW + 1],
+                                   pdv_face_pred(a[LF_V * LRW], a[LF_V * LRW + 1], dx, dt), tfp,
+                                   dx, dy, c.rvol, dt);
+    }
     if (xwall_warp) ph = __shfl_sync(FULL, ph, src);
     ph_m = ph;
     phl_m = __shfl_up_sync(FULL, ph, 1);
   }
+  double tsum_m = 0.0, tfc_m = 0.0;  // corrector: top-face sum / flux of the previous row
   double u1_m = 0.0, v1_m = 0.0, u1r_m = 0.0, v1r_m = 0.0;
   for (int k = k0; k <= k1; ++k) {
     wait_row(k + 1);
     const double* rm = row(k - 1);
     const double* rc = row(k);
     double ph = 0.0;
-    if (EDGE && c.wt && k == c.ny + 1)
-      ph = ph_m;  // reflective top: mirror of row ny
-    else if (colok)
-      ph = predict(rc, row(k + 1));
+    if constexpr (EDGE) {
+      if (c.wt && k == c.ny + 1)
+        ph = ph_m;  // reflective top: mirror of row ny
+      else if (colok)
+        ph = predict(rc, row(k + 1));
+    } else {
+      const double* rn = row(k + 1);
+      const double tf = pdv_face_pred(rn[LF_V * LRW], rn[LF_V * LRW + 1], dx, dt);
+      ph = pdv_predict_pressure_bt(dv, rc[LF_R * LRW], rc[LF_E * LRW], rc[LF_Q * LRW],
+                                   rc[LF_U * LRW], rn[LF_U * LRW], rc[LF_U * LRW + 1],
+                                   rn[LF_U * LRW + 1], tfp, tf, dx, dy, c.rvol, dt);
+      tfp = tf;
+    }
     if (xwall_warp) ph = __shfl_sync(FULL, ph, src);
     const double phl = __shfl_up_sync(FULL, ph, 1);
 
@@ -462,18 +485,32 @@ __device__ __forceinline__ bool lagr_body(const Chunk& c, const CUtensorMap* __r
 
     // PdV corrector + flux_calc of cell (j,k-1)
     const int kc = k - 1;
+    double tsum_c = 0.0, tfc_c = 0.0;
+    if constexpr (!EDGE) {
+      // top face of cell row k-1 = bottom face of row k (carried to k+1)
+      tsum_c = rc[LF_V * LRW] + rc[LF_V * LRW + 1] + v1_c + v1r_c;
+      tfc_c = pdv_face_corr(tsum_c, dx, dt);
+    }
     if (kc >= k0 && lane >= 1 && lane <= LW && (!EDGE || j <= c.nx)) {
       const double u0_m = rm[LF_U * LRW], u0r_m = rm[LF_U * LRW + 1];
-      const double v0_m = rm[LF_V * LRW], v0r_m = rm[LF_V * LRW + 1];
       const double u0_c = rc[LF_U * LRW], u0r_c = rc[LF_U * LRW + 1];
-      const double v0_c = rc[LF_V * LRW], v0r_c = rc[LF_V * LRW + 1];
       const double lsum = u0_m + u0_c + u1_m + u1_c;
       const double rsum = u0r_m + u0r_c + u1r_m + u1r_c;
-      const double bsum = v0_m + v0r_m + v1_m + v1r_m;
-      const double tsum = v0_c + v0r_c + v1_c + v1r_c;
+      double bsum, tsum, bfc, tfc;
+      if constexpr (EDGE) {
+        const double v0_m = rm[LF_V * LRW], v0r_m = rm[LF_V * LRW + 1];
+        const double v0_c = rc[LF_V * LRW], v0r_c = rc[LF_V * LRW + 1];
+        bsum = v0_m + v0r_m + v1_m + v1r_m;
+        tsum = v0_c + v0r_c + v1_c + v1r_c;
+        bfc = pdv_face_corr(bsum, dx, dt);
+        tfc = pdv_face_corr(tsum, dx, dt);
+      } else {
+        bsum = tsum_m; tsum = tsum_c;
+        bfc = tfc_m; tfc = tfc_c;
+      }
       double ev, dvv;
-      pdv_correct(dv, rm[LF_R * LRW], rm[LF_E * LRW], ph_m, rm[LF_Q * LRW], lsum, rsum, bsum, tsum,
-                  dx, dy, c.rvol, dt, ev, dvv);
+      pdv_correct_bt(dv, rm[LF_R * LRW], rm[LF_E * LRW], ph_m, rm[LF_Q * LRW], lsum, rsum, bfc, tfc,
+                     dx, dy, c.rvol, dt, ev, dvv);
       const int ic = idx(c, j, kc);
       const double cx = 0.25 * dt * dy, cy = 0.25 * dt * dx;
       if (!EDGE || !(ncol || near_wall_row(c, kc))) {
@@ -510,6 +547,7 @@ __device__ __forceinline__ bool lagr_body(const Chunk& c, const CUtensorMap* __r
     }
     ph_m = ph; phl_m = phl;
     u1_m = u1_c; v1_m = v1_c; u1r_m = u1r_c; v1r_m = v1r_c;
+    tsum_m = tsum_c; tfc_m = tfc_c;
     // row k-1 is consumed (rows k, k+1 are still read next iteration):
     // refill its slot with row k-1+LSTG
 #if CLOVER_TMA_RELEASE_FENCE
