@@ -1339,25 +1339,35 @@ kf_advec_mom_y(Chunk c, const double* __restrict__ rho, const double* __restrict
 // ny-1..ny, launched first); halo columns at x walls take the mirror of the
 // adjacent lane (density +, y-face mass flux +); at x chunk boundaries they
 // are recomputed from the depth-2 input halos.
-// Inputs stream through a per-warp YRING-row ring: sweep 1 reads d1 e1 u1 v1
+// Inputs stream through a per-warp ring of YL<SWEEP>::RING rows: sweep 1 reads d1 e1 u1 v1
 // fy fx (one 3D tensor copy per row), sweep 2 reads fy and d2 e2 u2 v2 (two).
 constexpr int YW = 31;
 #ifndef CLOVER_YKS
 #define CLOVER_YKS 32
 #endif
 constexpr int YKS = CLOVER_YKS;
-#ifndef CLOVER_YRING
-#define CLOVER_YRING 8
+// Ring depth per sweep (rows): sweep 1 (6 fields per row) runs at 6 rows
+// and a register cap of 10 blocks/SM for occupancy, sweep 2 (5 fields) at
+// 8 rows uncapped -- measured best each (ncu: 281 vs 286 us for sweep 1).
+#ifndef CLOVER_YRING1
+#define CLOVER_YRING1 6
 #endif
-constexpr int YRING = CLOVER_YRING;
+#ifndef CLOVER_YRING2
+#define CLOVER_YRING2 8
+#endif
+#ifndef CLOVER_YMINB1
+#define CLOVER_YMINB1 10
+#endif
 constexpr int YRW = 36;
 template <int SWEEP> struct YL;
 template <> struct YL<1> {  // tensor d1 e1 u1 v1 fy fx
+  static constexpr int RING = CLOVER_YRING1, MINB = CLOVER_YMINB1;
   enum { R = 0, E = YRW, U = 2 * YRW, V = 3 * YRW, FY = 4 * YRW, FX = 5 * YRW, B = 0,
          SLOT = (6 * YRW + 15) / 16 * 16 };
   static constexpr unsigned BYTES = 6 * YRW * 8;
 };
 template <> struct YL<2> {  // tensors fy | d2 e2 u2 v2
+  static constexpr int RING = CLOVER_YRING2, MINB = 0;  // 0: no cap
   enum { FY = 0, B = (YRW + 15) / 16 * 16, R = B, E = B + YRW, U = B + 2 * YRW, V = B + 3 * YRW,
          FX = -1, SLOT = (B + 4 * YRW + 15) / 16 * 16 };
   static constexpr unsigned BYTES = 5 * YRW * 8;
@@ -1394,24 +1404,24 @@ __device__ __forceinline__ bool advec_y_body(const Chunk& c, const CUtensorMap* 
   const int xcol = x0 & ~1;           // 16-B aligned box start
   const int t0 = 1 + (x0 & 1);        // smem column of lane 0
   auto issue = [&](int r) {
-    const unsigned sl = (unsigned)(r - r_first) % (unsigned)YRING;
+    const unsigned sl = (unsigned)(r - r_first) % (unsigned)L::RING;
     double* d = ring + sl * L::SLOT;
     mbar_arrive_expect_tx(&bars[sl], L::BYTES);
     tma_load_3d(d, ta, xcol, ROW0 + r, 0, &bars[sl]);
     if constexpr (SWEEP == 2) tma_load_3d(d + L::B, tb, xcol, ROW0 + r, 0, &bars[sl]);
   };
   auto row = [&](int r) -> const double* {
-    return ring + ((unsigned)(r - r_first) % (unsigned)YRING) * L::SLOT + lane + t0;
+    return ring + ((unsigned)(r - r_first) % (unsigned)L::RING) * L::SLOT + lane + t0;
   };
   auto wait_row = [&](int r) {
     const unsigned rel = (unsigned)(r - r_first);
-    mbar_wait(&bars[rel % YRING], (rel / YRING) & 1u);
+    mbar_wait(&bars[rel % L::RING], (rel / L::RING) & 1u);
   };
   if (lane == 0) {
-    for (int t = 0; t < YRING; ++t) mbar_init(&bars[t], 1);
+    for (int t = 0; t < L::RING; ++t) mbar_init(&bars[t], 1);
     fence_mbar_init();
     fence_proxy_async();
-    for (int r = r_first; r < r_first + YRING && r <= r_last; ++r) issue(r);
+    for (int r = r_first; r < r_first + L::RING && r <= r_last; ++r) issue(r);
   }
   __syncwarp();
 
@@ -1539,12 +1549,12 @@ __device__ __forceinline__ bool advec_y_body(const Chunk& c, const CUtensorMap* 
       fence_proxy_async();
 #endif
       __syncwarp();
-      if (lane == 0 && s - 2 + YRING <= r_last) issue(s - 2 + YRING);
+      if (lane == 0 && s - 2 + L::RING <= r_last) issue(s - 2 + L::RING);
     }
   }
   __syncwarp();
   if (lane == 0)
-    for (int t = 0; t < YRING; ++t) mbar_inval(&bars[t]);  // the ring may be reused (fixup)
+    for (int t = 0; t < L::RING; ++t) mbar_inval(&bars[t]);  // the ring may be reused (fixup)
   __syncwarp();
   return __any_sync(FULL, dv.bad);
 }
@@ -1571,14 +1581,14 @@ __device__ __forceinline__ bool advec_y_seg(const Chunk& c, const CUtensorMap* t
 }
 
 template <int SWEEP>
-__global__ void LB_ADVY
+__global__ void __launch_bounds__(SB, YL<SWEEP>::MINB)
 ks_advec_y(Chunk c, const __grid_constant__ CUtensorMap ta, const __grid_constant__ CUtensorMap tb,
            double* __restrict__ rho_out, double* __restrict__ en_out, const double* __restrict__ mfy,
            double* __restrict__ uout, double* __restrict__ vout, FixSlot fix) {
   pdl_trigger();
   pdl_wait();
-  __shared__ __align__(128) double ring[SB / 32][YRING * YL<SWEEP>::SLOT];
-  __shared__ __align__(8) unsigned long long bars[SB / 32][YRING];
+  __shared__ __align__(128) double ring[SB / 32][YL<SWEEP>::RING * YL<SWEEP>::SLOT];
+  __shared__ __align__(8) unsigned long long bars[SB / 32][YL<SWEEP>::RING];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const int gw = blockIdx.x * (SB / 32) + w;
   int k0, len;
@@ -1596,8 +1606,8 @@ kf_advec_y(Chunk c, const __grid_constant__ CUtensorMap ta, const __grid_constan
            double* __restrict__ uout, double* __restrict__ vout, FixSlot fix) {
   pdl_trigger();
   pdl_wait();
-  __shared__ __align__(128) double ring[SB / 32][YRING * YL<SWEEP>::SLOT];
-  __shared__ __align__(8) unsigned long long bars[SB / 32][YRING];
+  __shared__ __align__(128) double ring[SB / 32][YL<SWEEP>::RING * YL<SWEEP>::SLOT];
+  __shared__ __align__(8) unsigned long long bars[SB / 32][YL<SWEEP>::RING];
   fix_loop(fix, c.yks, c.ynb, c.ny + 2, [&](int gw, int k0, int k1, int lane, int w) {
     advec_y_seg<SWEEP, DivIEEE>(c, &ta, &tb, rho_out, en_out, mfy, uout, vout, gw, k0, k1, lane,
                                 ring[w], bars[w]);
