@@ -140,7 +140,12 @@ struct NoLast {
 template <class Run, class Last = NoLast>
 __device__ __forceinline__ void fix_loop(FixSlot f, int ks, int nb, int lim, Run&& run,
                                          Last last = {}) {
-  const unsigned n = *(volatile unsigned*)f.hdr;
+  const unsigned n = *(volatile unsigned*)f.hdr;  // the same value in every thread
+  if (n == 0u) {
+    // nothing flagged (the common case): no list to reset, no counting
+    if (blockIdx.x == 0 && threadIdx.x == 0) last();
+    return;
+  }
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const unsigned items = n * (unsigned)ks;
   for (unsigned it = blockIdx.x * (SB / 32) + w; it < items; it += gridDim.x * (SB / 32)) {
