@@ -186,6 +186,9 @@ def main():
                     help="skip the fully-active-flow side measurement")
     ap.add_argument("--strong", action="store_true",
                     help="configs[3]: 7680^2 strong-scaled over the ranks (default: configs[4] weak)")
+    ap.add_argument("--transport", default="nccl", choices=["nccl", "host"],
+                    help="host: gloo host transport, ranks may share a GPU (validates the "
+                         "multi-rank path on a one-GPU box; its timing is not a bench value)")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
@@ -200,6 +203,9 @@ def main():
     rank, world, local = env_int("RANK", 0), env_int("WORLD_SIZE", 1), env_int("LOCAL_RANK", 0)
     if world != args.gpus:
         args.gpus = world
+    host_tp = args.transport == "host"
+    if host_tp:
+        local = local % max(torch.cuda.device_count(), 1)
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     from paper_conf_cluster_regulymg15_b200 import Clover, nccl_unique_id
@@ -207,7 +213,10 @@ def main():
     from workloads import bm_deck
 
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if host_tp:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=dev)
     if args.strong:
         nx, ny = 7680, 7680
         px, py = cdist.chunk_grid(world, nx, ny)
@@ -219,9 +228,11 @@ def main():
     # square cells: the domain grows with the mesh (weak scaling stacks
     # per-rank 3840^2 blocks along y)
     deck = bm_deck(nx, ny, end_step=args.steps, ymax=10.0 * ny / nx)
-    uid = cdist.share_unique_id(nccl_unique_id) if world > 1 else None
+    uid = cdist.share_unique_id(nccl_unique_id) if world > 1 and not host_tp else None
+    ht = cdist.GlooHostTransport() if world > 1 and host_tp else None
     stream = torch.cuda.Stream(dev)
-    sim = Clover(deck, px=px, py=py, rank=rank, nranks=world, unique_id=uid, stream=stream)
+    sim = Clover(deck, px=px, py=py, rank=rank, nranks=world, unique_id=uid, stream=stream,
+                 host_transport=ht)
     cells = nx * ny
 
     # warm-up (also builds the CUDA graphs)
@@ -242,7 +253,7 @@ def main():
     ms = e0.elapsed_time(e1)
     clk = clocks.stop()
     sim.sync()
-    ms = cdist.max_over_ranks(ms, dev)
+    ms = cdist.max_over_ranks(ms, None if host_tp else dev)
     value = cells * args.steps / (ms / 1000.0)
     kps = sim.kernels_per_step()
 
@@ -325,7 +336,8 @@ def main():
         active = {"ms_per_step": ams, "value": cells / (ams / 1e3), "unit": UNIT,
                   "state": "workloads.random_state_fields(7, smooth=True): every cell moving, limiters active"}
         act.close()
-        sim = Clover(deck, px=px, py=py, rank=rank, nranks=world, unique_id=uid, stream=stream)
+        sim = Clover(deck, px=px, py=py, rank=rank, nranks=world, unique_id=uid, stream=stream,
+                     host_transport=ht)
         sim.step(args.steps + args.warmup)
 
     cpu = None
@@ -349,6 +361,8 @@ def main():
                                         "1 GPU bandwidth-roofline run" if world == 1 else
                                         f"configs[4]: weak scaling, 3840^2 cells per GPU, global {nx}x{ny}"),
                            "mesh": [nx, ny], "decomposition": f"{px}x{py}",
+                           "transport": ("nccl" if not host_tp else "host (gloo; not a bench value)")
+                           if world > 1 else None,
                            "l2": "inputs larger than L2 (18 fp64 fields of the mesh, >2 GB vs 126 MB L2)",
                            "graphs": True},
                 "gpu_launches": kps * args.steps,

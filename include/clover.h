@@ -47,7 +47,7 @@
 extern "C" {
 #endif
 
-#define CLOVER_ABI_VERSION 1
+#define CLOVER_ABI_VERSION 2  /* 2: clover_dist.host_transport */
 
 enum {
   CLOVER_OK = 0,
@@ -86,15 +86,36 @@ typedef struct {
   double xmin, xmax, ymin, ymax, radius;
 } clover_state;
 
+/* Host transport (S:8(e), "standard halo exchanges"): the three
+ * collectives of a multi-rank step carried by caller callbacks on HOST
+ * buffers instead of NCCL -- for several ranks without NCCL (e.g. processes
+ * sharing one GPU, which NCCL refuses).  Every callback returns 0 on
+ * success; the library copies device data to host before a call and back
+ * after it, synchronously (CUDA graphs are off in this mode).
+ *  sendrecv: for i in [0, n): send send[i] (nsend[i] doubles) to rank
+ *    peer[i] and receive recv[i] (nrecv[i] doubles) from rank peer[i];
+ *    several messages to one peer are matched in list order.
+ *  allreduce_min_u64: *value = min over ranks (dt bit pattern, in place).
+ *  allgather_f64: recv[r*count .. ] = rank r's send (count doubles each). */
+typedef struct {
+  void* user;
+  int (*sendrecv)(void* user, int32_t n, const int32_t* peer, const double* const* send,
+                  const int64_t* nsend, double* const* recv, const int64_t* nrecv);
+  int (*allreduce_min_u64)(void* user, uint64_t* value);
+  int (*allgather_f64)(void* user, const double* send, int64_t count, double* recv);
+} clover_host_transport;
+
 /* Decomposition.  nranks processes, each owning chunks_x*chunks_y/nranks
  * chunks of a px*py chunk grid (px = chunks in x).  nranks==1 with
  * px*py>1 runs all chunks on one GPU.  nccl_unique_id: 128 bytes from
  * clover_nccl_unique_id() on rank 0, broadcast by the caller; NULL when
- * nranks == 1. */
+ * nranks == 1 or when host_transport is given (then NCCL is not used;
+ * the struct is copied, its callbacks must outlive the context). */
 typedef struct {
   int32_t rank, nranks;
   int32_t px, py;
   const void* nccl_unique_id;
+  const clover_host_transport* host_transport; /* NULL = NCCL */
 } clover_dist;
 
 /* field_summary totals: density = mass/vol,

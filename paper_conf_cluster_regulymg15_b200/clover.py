@@ -57,9 +57,22 @@ class CloverState(ctypes.Structure):
                 ("ymax", c_double), ("radius", c_double)]
 
 
+SENDRECV_FN = ctypes.CFUNCTYPE(ctypes.c_int, c_void_p, c_int32, ctypes.POINTER(c_int32),
+                               ctypes.POINTER(ctypes.POINTER(c_double)), ctypes.POINTER(c_int64),
+                               ctypes.POINTER(ctypes.POINTER(c_double)), ctypes.POINTER(c_int64))
+ALLREDUCE_FN = ctypes.CFUNCTYPE(ctypes.c_int, c_void_p, ctypes.POINTER(ctypes.c_uint64))
+ALLGATHER_FN = ctypes.CFUNCTYPE(ctypes.c_int, c_void_p, ctypes.POINTER(c_double), c_int64,
+                                ctypes.POINTER(c_double))
+
+
+class CloverHostTransport(ctypes.Structure):
+    _fields_ = [("user", c_void_p), ("sendrecv", SENDRECV_FN), ("allreduce_min_u64", ALLREDUCE_FN),
+                ("allgather_f64", ALLGATHER_FN)]
+
+
 class CloverDist(ctypes.Structure):
     _fields_ = [("rank", c_int32), ("nranks", c_int32), ("px", c_int32), ("py", c_int32),
-                ("nccl_unique_id", c_void_p)]
+                ("nccl_unique_id", c_void_p), ("host_transport", ctypes.POINTER(CloverHostTransport))]
 
 
 class CloverSummary(ctypes.Structure):
@@ -212,15 +225,20 @@ class Clover:
     None = torch's current stream)."""
 
     def __init__(self, deck: dict, px: int = 1, py: int = 1, rank: int = 0, nranks: int = 1,
-                 unique_id: bytes | None = None, stream=None, device=None):
+                 unique_id: bytes | None = None, stream=None, device=None, host_transport=None):
         import torch  # device memory + streams only
         L = load()
         self.nx, self.ny = deck["x_cells"], deck["y_cells"]
         self._grid = grid_from_deck(deck)
         self._states = states_from_deck(deck)
         self._uid = ctypes.create_string_buffer(unique_id, 128) if unique_id else None
+        # host_transport: an object with the three clover_host_transport
+        # collectives (paper_conf_cluster_regulymg15_b200.dist.GlooHostTransport);
+        # the ctypes callbacks are kept alive with the context
+        self._ht = host_transport.c_struct() if host_transport is not None else None
         self._dist = CloverDist(rank=rank, nranks=nranks, px=px, py=py,
-                                nccl_unique_id=ctypes.cast(self._uid, c_void_p) if self._uid else None)
+                                nccl_unique_id=ctypes.cast(self._uid, c_void_p) if self._uid else None,
+                                host_transport=ctypes.pointer(self._ht) if self._ht is not None else None)
         nbytes = c_int64()
         _check(L.clover_workspace_bytes(ctypes.byref(self._grid), ctypes.byref(self._dist),
                                         ctypes.byref(nbytes)), "clover_workspace_bytes")

@@ -264,6 +264,8 @@ struct clover_ctx {
 #ifdef CLOVER_WITH_NCCL
   ncclComm_t comm = nullptr;
 #endif
+  bool use_ht = false;            // collectives through the caller's host transport
+  clover_host_transport ht = {};
 };
 
 namespace {
@@ -290,7 +292,11 @@ int validate(const clover_grid* g, const clover_dist* d, int* px, int* py, int* 
     if (*px < 1 || *py < 1) return fail(CLOVER_ERR_ARG, "px, py must be >= 1");
     if (*nranks < 1 || *rank < 0 || *rank >= *nranks) return fail(CLOVER_ERR_ARG, "bad rank/nranks");
     if ((*px * *py) % *nranks != 0) return fail(CLOVER_ERR_ARG, "px*py must be a multiple of nranks");
-    if (*nranks > 1 && !d->nccl_unique_id) return fail(CLOVER_ERR_ARG, "nccl_unique_id required for nranks > 1");
+    if (*nranks > 1 && !d->nccl_unique_id && !d->host_transport)
+      return fail(CLOVER_ERR_ARG, "nccl_unique_id or host_transport required for nranks > 1");
+    if (d->host_transport && (!d->host_transport->sendrecv || !d->host_transport->allreduce_min_u64 ||
+                              !d->host_transport->allgather_f64))
+      return fail(CLOVER_ERR_ARG, "host_transport needs all three callbacks");
   }
   Layout L = decompose(g->x_cells, g->y_cells, *px, *py);
   for (int i = 0; i < *px; ++i)
@@ -463,6 +469,26 @@ int exchange_axis(clover_ctx* ctx, const std::vector<int>& bufs, int axis) {
         CK(cudaMemcpyAsync(ctx->xbuf_recv + m.off, ctx->xbuf_send + partner->off, (size_t)m.n * 8,
                            cudaMemcpyDeviceToDevice, ctx->work));
       }
+    } else if (ctx->use_ht) {
+      // host transport: staging to host, the caller's sendrecv, back
+      std::vector<double> hs((size_t)off), hr((size_t)off);
+      CK(cudaMemcpyAsync(hs.data(), ctx->xbuf_send, (size_t)off * 8, cudaMemcpyDeviceToHost, ctx->work));
+      CK(cudaStreamSynchronize(ctx->work));
+      std::vector<int32_t> peer;
+      std::vector<const double*> sp;
+      std::vector<double*> rp;
+      std::vector<int64_t> cnt;
+      for (auto& m : msgs) {
+        peer.push_back(m.peer);
+        sp.push_back(hs.data() + m.off);
+        rp.push_back(hr.data() + m.off);
+        cnt.push_back(m.n);
+      }
+      if (ctx->ht.sendrecv(ctx->ht.user, (int32_t)msgs.size(), peer.data(), sp.data(), cnt.data(),
+                           rp.data(), cnt.data()) != 0)
+        return fail(CLOVER_ERR_NCCL, "host transport sendrecv failed");
+      CK(cudaMemcpyAsync(ctx->xbuf_recv, hr.data(), (size_t)off * 8, cudaMemcpyHostToDevice, ctx->work));
+      CK(cudaStreamSynchronize(ctx->work));
     } else {
 #ifdef CLOVER_WITH_NCCL
       NK(ncclGroupStart());
@@ -622,8 +648,17 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
   }
   if (nphase >= 2) {
     cur_prof_id = P_DT_FINAL;
+    if (ctx->nranks > 1 && ctx->use_ht) {
+      uint64_t v = 0;
+      CK(cudaMemcpyAsync(&v, &ctx->scal->dt_slot, 8, cudaMemcpyDeviceToHost, st));
+      CK(cudaStreamSynchronize(st));
+      if (ctx->ht.allreduce_min_u64(ctx->ht.user, &v) != 0)
+        return fail(CLOVER_ERR_NCCL, "host transport allreduce failed");
+      CK(cudaMemcpyAsync(&ctx->scal->dt_slot, &v, 8, cudaMemcpyHostToDevice, st));
+      CK(cudaStreamSynchronize(st));
+    }
 #ifdef CLOVER_WITH_NCCL
-    if (ctx->nranks > 1)
+    else if (ctx->nranks > 1)
       NK(ncclAllReduce(&ctx->scal->dt_slot, &ctx->scal->dt_slot, 1, ncclUint64, ncclMin, ctx->comm, st));
 #endif
     if (ctx->prof) prof_mark(ctx, -1);
@@ -916,6 +951,14 @@ int scatter_local(clover_ctx* ctx, int buf, int kind, const double* host, int64_
 // (nranks*count, rank-major).  Uses a temporary device buffer: this is the
 // debug / I/O path (field readback, summaries, checkpoints), not the step.
 int allgather_to_host(clover_ctx* ctx, const double* send, int64_t count, double* out) {
+  if (ctx->use_ht) {
+    std::vector<double> h((size_t)count);
+    CK(cudaMemcpyAsync(h.data(), send, (size_t)count * 8, cudaMemcpyDeviceToHost, ctx->work));
+    CK(cudaStreamSynchronize(ctx->work));
+    if (ctx->ht.allgather_f64(ctx->ht.user, h.data(), count, out) != 0)
+      return fail(CLOVER_ERR_NCCL, "host transport allgather failed");
+    return CLOVER_OK;
+  }
 #ifdef CLOVER_WITH_NCCL
   double* recv = nullptr;
   CK(cudaMallocAsync((void**)&recv, (size_t)count * ctx->nranks * 8, ctx->work));
@@ -1093,7 +1136,7 @@ int clover_init(const clover_grid* grid, const clover_state* states, int32_t nst
   if (!states || nstates < 1) return fail(CLOVER_ERR_ARG, "need at least one state");
   if (nstates > MAX_STATES) return fail(CLOVER_ERR_ARG, "too many states");
 #ifndef CLOVER_WITH_NCCL
-  if (nranks > 1) return fail(CLOVER_ERR_NCCL, "libclover built without NCCL");
+  if (nranks > 1 && !dist->host_transport) return fail(CLOVER_ERR_NCCL, "libclover built without NCCL");
 #endif
   const int64_t need = compute_workspace(grid, px, py, rank, nranks);
   if (!workspace || workspace_bytes < need || ((uintptr_t)workspace % kAlign) != 0)
@@ -1204,8 +1247,13 @@ int clover_init(const clover_grid* grid, const clover_state* states, int32_t nst
     ctx->xbuf_recv = (double*)p;
     p += align_up(ctx->xbuf_elems * 8, kAlign);
   }
+  if (nranks > 1 && dist->host_transport) {
+    ctx->use_ht = true;
+    ctx->ht = *dist->host_transport;
+    ctx->use_graphs = false;  // host callbacks inside the step
+  }
 #ifdef CLOVER_WITH_NCCL
-  if (nranks > 1) {
+  if (nranks > 1 && !ctx->use_ht) {
     ncclUniqueId id;
     std::memcpy(&id, dist->nccl_unique_id, sizeof(id));
     if (ncclCommInitRank(&ctx->comm, nranks, id, rank) != ncclSuccess)
@@ -1266,7 +1314,7 @@ int clover_init(const clover_grid* grid, const clover_state* states, int32_t nst
 
 int clover_set_graphs(clover_ctx* ctx, int32_t enable) {
   if (!ctx) return fail(CLOVER_ERR_ARG, "ctx is NULL");
-  ctx->use_graphs = enable != 0;
+  ctx->use_graphs = enable != 0 && !ctx->use_ht;  // host callbacks cannot be captured
   return CLOVER_OK;
 }
 

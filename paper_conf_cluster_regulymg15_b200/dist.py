@@ -1,7 +1,10 @@
 """Multi-process plumbing for one-process-per-GPU runs (torch.distributed):
 chunk-grid choice, NCCL unique-id broadcast and max-over-ranks timing.
 The halo exchange and the dt MIN all-reduce themselves run inside
-libclover.so over NCCL; this module only sets them up.
+libclover.so over NCCL; this module only sets them up.  GlooHostTransport
+carries the same three collectives over a gloo process group on host
+buffers (clover_host_transport): ranks without NCCL, e.g. several processes
+sharing one GPU, which NCCL refuses.
 """
 from __future__ import annotations
 
@@ -55,3 +58,59 @@ def max_over_ranks(value: float, device=None) -> float:
     t = torch.tensor([float(value)], dtype=torch.float64, device=device)
     dist.all_reduce(t, op=dist.ReduceOp.MAX)
     return float(t.item())
+
+
+class GlooHostTransport:
+    """clover_host_transport over torch.distributed (gloo, CPU tensors).
+    The library hands host buffers; these callbacks only move them (halo
+    messages point to point, the dt bit pattern MIN, summary/readback
+    all-gather) -- no arithmetic of the method."""
+
+    def __init__(self, group=None):
+        self.group = group
+
+    def _sendrecv(self, user, n, peer, send, nsend, recv, nrecv):
+        import numpy as np
+        try:
+            reqs = []
+            for i in range(n):
+                a = np.ctypeslib.as_array(send[i], shape=(int(nsend[i]),))
+                reqs.append(dist.isend(torch.from_numpy(a), int(peer[i]), group=self.group))
+            for i in range(n):
+                b = np.ctypeslib.as_array(recv[i], shape=(int(nrecv[i]),))
+                reqs.append(dist.irecv(torch.from_numpy(b), int(peer[i]), group=self.group))
+            for r in reqs:
+                r.wait()
+            return 0
+        except Exception:  # noqa: BLE001 -- reported to the library as a failed call
+            return 1
+
+    def _allreduce(self, user, value):
+        try:
+            # positive doubles' bit patterns fit int64 and order like the values
+            t = torch.tensor([int(value[0])], dtype=torch.int64)
+            dist.all_reduce(t, op=dist.ReduceOp.MIN, group=self.group)
+            value[0] = int(t.item())
+            return 0
+        except Exception:  # noqa: BLE001
+            return 1
+
+    def _allgather(self, user, send, count, recv):
+        import numpy as np
+        try:
+            world = dist.get_world_size(self.group)
+            a = torch.from_numpy(np.ctypeslib.as_array(send, shape=(int(count),)).copy())
+            outs = [torch.empty(int(count), dtype=torch.float64) for _ in range(world)]
+            dist.all_gather(outs, a, group=self.group)
+            r = np.ctypeslib.as_array(recv, shape=(world * int(count),))
+            for i, o in enumerate(outs):
+                r[i * int(count):(i + 1) * int(count)] = o.numpy()
+            return 0
+        except Exception:  # noqa: BLE001
+            return 1
+
+    def c_struct(self):
+        from .clover import (ALLGATHER_FN, ALLREDUCE_FN, SENDRECV_FN, CloverHostTransport)
+        self._cb = (SENDRECV_FN(self._sendrecv), ALLREDUCE_FN(self._allreduce),
+                    ALLGATHER_FN(self._allgather))
+        return CloverHostTransport(None, *self._cb)

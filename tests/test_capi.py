@@ -32,7 +32,7 @@ def test_library_exports_every_declared_symbol():
     missing = [n for n in declared_functions() if not hasattr(L, n)]
     assert not missing, missing
     assert set(declared_functions()) <= set(cb.EXPORTS)
-    assert L.clover_abi_version() == 1
+    assert L.clover_abi_version() == 2
 
 
 def test_error_strings_and_validation_without_gpu():
