@@ -355,11 +355,47 @@ struct XferDesc {  // one rectangular strip of one field
 
 inline double* strip_ptr(const XferDesc& d) { return d.base + (int64_t)d.k0 * d.pitch + d.j0; }
 
-int copy_strip(clover_ctx* ctx, const XferDesc& dst, const XferDesc& src) {
-  CK(cudaMemcpy2DAsync(strip_ptr(dst), (size_t)dst.pitch * 8, strip_ptr(src), (size_t)src.pitch * 8,
-                       (size_t)src.w * 8, src.h, cudaMemcpyDeviceToDevice, ctx->work));
-  return CLOVER_OK;
+// Halo strips are many small rectangles (per phase: fields x sides x
+// chunks, plus pack/unpack of the multi-GPU staging buffer); one
+// cudaMemcpy2DAsync each cost ~2 us of launch per strip.  A batch collects
+// the strips of one ordering stage and copies them in one kernel launch
+// (elements enumerated strip by strip, rows contiguous for coalescing).
+constexpr int MAX_STRIPS = 48;
+struct StripCopy {
+  double* dst;
+  const double* src;
+  int dpitch, spitch, w, h;
+};
+struct StripBatch {
+  int n;
+  long long start[MAX_STRIPS + 1];  // element offset of each strip; start[n] = total
+  StripCopy s[MAX_STRIPS];
+};
+__global__ void __launch_bounds__(256) k_copy_strips(const __grid_constant__ StripBatch b) {
+  const long long total = b.start[b.n];
+  for (long long e = (long long)blockIdx.x * blockDim.x + threadIdx.x; e < total;
+       e += (long long)gridDim.x * blockDim.x) {
+    int lo = 0, hi = b.n - 1;  // last strip with start <= e
+    while (lo < hi) {
+      const int mid = (lo + hi + 1) >> 1;
+      if (b.start[mid] <= e) lo = mid; else hi = mid - 1;
+    }
+    const StripCopy& c = b.s[lo];
+    const long long off = e - b.start[lo];
+    const int r = (int)(off / c.w), col = (int)(off - (long long)r * c.w);
+    c.dst[(long long)r * c.dpitch + col] = c.src[(long long)r * c.spitch + col];
+  }
 }
+struct StripQueue {
+  clover_ctx* ctx;
+  StripBatch b{};
+  explicit StripQueue(clover_ctx* c) : ctx(c) { b.n = 0; b.start[0] = 0; }
+  int add(double* dst, int dpitch, const double* src, int spitch, int w, int h);
+  int add(const XferDesc& dst, const XferDesc& src) {
+    return add(strip_ptr(dst), dst.pitch, strip_ptr(src), src.pitch, src.w, src.h);
+  }
+  int flush();
+};
 
 // strips for side `side` (0 left, 1 right, 2 bottom, 3 top) of chunk cs:
 // send = owned points next to that side, recv = halo points of that side.
@@ -409,9 +445,33 @@ ChunkState* local_chunk(clover_ctx* ctx, int id) {
   return nullptr;
 }
 
+int StripQueue::add(double* dst, int dpitch, const double* src, int spitch, int w, int h) {
+  if (w <= 0 || h <= 0) return CLOVER_OK;
+  if (b.n == MAX_STRIPS) {
+    int rc = flush();
+    if (rc) return rc;
+  }
+  b.s[b.n] = {dst, src, dpitch, spitch, w, h};
+  b.start[b.n + 1] = b.start[b.n] + (long long)w * h;
+  ++b.n;
+  return CLOVER_OK;
+}
+int StripQueue::flush() {
+  if (b.n == 0) return CLOVER_OK;
+  const long long total = b.start[b.n];
+  const int blocks = (int)std::min<long long>((total + 255) / 256, 148 * 8);
+  k_copy_strips<<<blocks, 256, 0, ctx->work>>>(b);
+  CK(cudaGetLastError());
+  b.n = 0;
+  b.start[0] = 0;
+  return CLOVER_OK;
+}
+
 int exchange_axis(clover_ctx* ctx, const std::vector<int>& bufs, int axis) {
   const int s_lo = axis == 0 ? 0 : 2, s_hi = axis == 0 ? 1 : 3;
-  // local pairs
+  // stage 1 (one batch): local pairs' halo strips and the packing of the
+  // remote sides (owned points in, halo points / staging out: disjoint)
+  StripQueue q(ctx);
   for (auto& cs : ctx->chunks) {
     if (ctx->virtual_remote) break;
     int nb = neighbour(ctx, cs, s_hi);
@@ -422,9 +482,9 @@ int exchange_axis(clover_ctx* ctx, const std::vector<int>& bufs, int axis) {
       XferDesc sA, rA, sB, rB;
       side_strips(cs, b, s_hi, sA, rA);
       side_strips(*other, b, s_lo, sB, rB);
-      int rc = copy_strip(ctx, rB, sA);  // my high side -> neighbour's low halo
+      int rc = q.add(rB, sA);  // my high side -> neighbour's low halo
       if (rc) return rc;
-      rc = copy_strip(ctx, rA, sB);      // neighbour's low side -> my high halo
+      rc = q.add(rA, sB);      // neighbour's low side -> my high halo
       if (rc) return rc;
     }
   }
@@ -453,22 +513,26 @@ int exchange_axis(clover_ctx* ctx, const std::vector<int>& bufs, int axis) {
           XferDesc s, r;
           side_strips(cs, b, side, s, r);
           XferDesc dst{ctx->xbuf_send + off + n, s.w, 0, 0, s.w, s.h};
-          int rc = copy_strip(ctx, dst, s);
+          int rc = q.add(dst, s);
           if (rc) return rc;
           n += (int64_t)s.w * s.h;
         }
         msgs.push_back({ctx->owner[nb], nb, off, n, &cs, side});
         off += n;
       }
+    int rc = q.flush();  // the staging buffer is complete before it is sent
+    if (rc) return rc;
     if (ctx->virtual_remote) {
       for (auto& m : msgs) {
         const Msg* partner = nullptr;
-        for (auto& q : msgs)
-          if (q.cs->id == m.nb && q.side == (m.side ^ 1)) partner = &q;
+        for (auto& pm : msgs)
+          if (pm.cs->id == m.nb && pm.side == (m.side ^ 1)) partner = &pm;
         if (!partner || partner->n != m.n) return fail(CLOVER_ERR_STATE, "virtual remote: unmatched message");
-        CK(cudaMemcpyAsync(ctx->xbuf_recv + m.off, ctx->xbuf_send + partner->off, (size_t)m.n * 8,
-                           cudaMemcpyDeviceToDevice, ctx->work));
+        rc = q.add(ctx->xbuf_recv + m.off, (int)m.n, ctx->xbuf_send + partner->off, (int)m.n, (int)m.n, 1);
+        if (rc) return rc;
       }
+      rc = q.flush();
+      if (rc) return rc;
     } else if (ctx->use_ht) {
       // host transport: staging to host, the caller's sendrecv, back
       std::vector<double> hs((size_t)off), hr((size_t)off);
@@ -507,13 +571,13 @@ int exchange_axis(clover_ctx* ctx, const std::vector<int>& bufs, int axis) {
         XferDesc s, r;
         side_strips(*m.cs, b, m.side, s, r);
         XferDesc src{ctx->xbuf_recv + m.off + n, r.w, 0, 0, r.w, r.h};
-        int rc = copy_strip(ctx, r, src);
+        rc = q.add(r, src);
         if (rc) return rc;
         n += (int64_t)r.w * r.h;
       }
     }
   }
-  return CLOVER_OK;
+  return q.flush();
 }
 
 bool needs_exchange(const clover_ctx* ctx) { return ctx->L.px * ctx->L.py > 1; }
