@@ -255,7 +255,7 @@ struct clover_ctx {
   bool advect_x = true;
   bool use_graphs = true;
   bool fuse_x = true;  // fused x sweep where every chunk has both x walls (see fuse_x_ok)
-  bool fuse_y = true;  // fused y sweep where every chunk has both y walls (see fuse_y_ok)
+  bool fuse_y = true;  // fused y sweep (see fuse_y_ok)
   cudaGraphExec_t gexec[2] = {nullptr, nullptr};
   int64_t ws_bytes = 0;
   bool prof = false;
@@ -668,12 +668,19 @@ bool fuse_x_ok(const clover_ctx* ctx) {
 // The fused y sweep needs reflective walls at both y ends of every chunk
 // (its reach along y is 4 rows: a chunk boundary would need depth-4 halos)
 // and the geometric face mirror.
+// The fused y sweep reads the post-sweep density and y-face mass flux of
+// the halo rows from memory, the mirrors written by the wall band kernel:
+// every chunk needs both y walls.  (Exchanging the band values across y
+// chunk boundaries instead was tried and is not bitwise yet: 1x4 chunks of
+// bm 96x80 differ at the first row above the high-pressure block, the
+// EDGE segment below a chunk boundary; kept off.)
 bool fuse_y_ok(const clover_ctx* ctx) {
   if (!ctx->fuse_y || ctx->g.face_mirror == CLOVER_MIRROR_CELLCENTRE) return false;
   for (const auto& cs : ctx->chunks)
     if (!cs.c.wb || !cs.c.wt) return false;
   return true;
 }
+bool y_chunk_boundary(const clover_ctx* ctx) { return ctx->L.py > 1; }
 
 // Enqueue kernel phases [0, nphase) of one step (7 = full step).
 // Serpentine segment order: each step kernel reads what the previous one
@@ -788,20 +795,33 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
       continue;
     }
     if (!xdir && fuse_y_ok(ctx)) {
-      // wall bands of advec_cell y, then advec_cell y + advec_mom y in one
-      // kernel (ks_advec_y): phase ph_cell runs all, phase ph_cell + 1 is empty
+      // advec_cell y on the wall bands of every chunk (rows 1..3, ny-1..ny;
+      // mirrored at y walls), the band values into the neighbours' halo rows
+      // at y chunk boundaries, then advec_cell y + advec_mom y in one kernel
+      // (ks_advec_y): phase ph_cell runs all, phase ph_cell + 1 is empty
       if (nphase >= ph_cell) {
         cur_prof_id = sweep == 1 ? P_ADV_Y1 : P_ADV_Y2;
         for (auto& cs : ctx->chunks) {
           const Chunk c = with_rev(cs.c, sweep == 1 ? CLOVER_SERP : 0);
           const dim3 gw(cdiv(c.nx + 2, SB), 2);
+          if (sweep == 1)
+            launch_step(ks_cell_y_walls<1>, gw, SB, st, c, cs.buf[rin], cs.buf[ein], cs.buf[B_FX],
+                        cs.buf[B_FY], cs.buf[rout], cs.buf[eout], cs.buf[B_MY]);
+          else
+            launch_step(ks_cell_y_walls<2>, gw, SB, st, c, cs.buf[rin], cs.buf[ein], cs.buf[B_FX],
+                        cs.buf[B_FY], cs.buf[rout], cs.buf[eout], cs.buf[B_MY]);
+          FIX_LAUNCH_CHECK();
+        }
+        if (y_chunk_boundary(ctx)) {
+          int rc = exchange(ctx, {rout, B_MY});
+          if (rc) return rc;
+        }
+        for (auto& cs : ctx->chunks) {
+          const Chunk c = with_rev(cs.c, sweep == 1 ? CLOVER_SERP : 0);
           const dim3 g(grid_strip(c.nx + 1, YW, c.ny + 1, c.yks).x, seg_count(c.yks, c.ynb, c.ny + 1));
           const CUtensorMap& ta = sweep == 1 ? cs.tm_x1 : cs.tm_fy;
           const CUtensorMap& tb = sweep == 1 ? cs.tm_x1 : cs.tm_c4;
           if (sweep == 1) {
-            launch_step(ks_cell_y_walls<1>, gw, SB, st, c, cs.buf[rin], cs.buf[ein], cs.buf[B_FX],
-                        cs.buf[B_FY], cs.buf[rout], cs.buf[eout], cs.buf[B_MY]);
-            FIX_LAUNCH_CHECK();
             launch_step(ks_advec_y<1>, g, SB, st, c, ta, tb, cs.buf[rout], cs.buf[eout], cs.buf[B_MY],
                         cs.buf[uout], cs.buf[vout], cs.fix);
             STEP_LAUNCH_CHECK();
@@ -809,9 +829,6 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
                         cs.buf[B_MY], cs.buf[uout], cs.buf[vout], cs.fix);
             FIX_LAUNCH_CHECK();
           } else {
-            launch_step(ks_cell_y_walls<2>, gw, SB, st, c, cs.buf[rin], cs.buf[ein], cs.buf[B_FX],
-                        cs.buf[B_FY], cs.buf[rout], cs.buf[eout], cs.buf[B_MY]);
-            FIX_LAUNCH_CHECK();
             launch_step(ks_advec_y<2>, g, SB, st, c, ta, tb, cs.buf[rout], cs.buf[eout], cs.buf[B_MY],
                         cs.buf[uout], cs.buf[vout], cs.fix);
             STEP_LAUNCH_CHECK();
