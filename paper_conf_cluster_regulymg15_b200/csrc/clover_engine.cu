@@ -680,7 +680,6 @@ bool fuse_y_ok(const clover_ctx* ctx) {
     if (!cs.c.wb || !cs.c.wt) return false;
   return true;
 }
-bool y_chunk_boundary(const clover_ctx* ctx) { return ctx->L.py > 1; }
 
 // Enqueue kernel phases [0, nphase) of one step (7 = full step).
 // Serpentine segment order: each step kernel reads what the previous one
@@ -795,9 +794,8 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
       continue;
     }
     if (!xdir && fuse_y_ok(ctx)) {
-      // advec_cell y on the wall bands of every chunk (rows 1..3, ny-1..ny;
-      // mirrored at y walls), the band values into the neighbours' halo rows
-      // at y chunk boundaries, then advec_cell y + advec_mom y in one kernel
+      // advec_cell y on the wall bands of every chunk (rows 1..3, ny-1..ny,
+      // mirrored), then advec_cell y + advec_mom y in one kernel
       // (ks_advec_y): phase ph_cell runs all, phase ph_cell + 1 is empty
       if (nphase >= ph_cell) {
         cur_prof_id = sweep == 1 ? P_ADV_Y1 : P_ADV_Y2;
@@ -811,10 +809,6 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
             launch_step(ks_cell_y_walls<2>, gw, SB, st, c, cs.buf[rin], cs.buf[ein], cs.buf[B_FX],
                         cs.buf[B_FY], cs.buf[rout], cs.buf[eout], cs.buf[B_MY]);
           FIX_LAUNCH_CHECK();
-        }
-        if (y_chunk_boundary(ctx)) {
-          int rc = exchange(ctx, {rout, B_MY});
-          if (rc) return rc;
         }
         for (auto& cs : ctx->chunks) {
           const Chunk c = with_rev(cs.c, sweep == 1 ? CLOVER_SERP : 0);
