@@ -245,6 +245,22 @@ __device__ __forceinline__ double pdv_predict_pressure(D& dv, double r, double e
 }
 
 // accelerate (c.6) at one node: cells ordered (j-1,k-1), (j,k-1), (j,k), (j-1,k).
+// mm[i] = rr[i] * vol: the cell masses; the row-streaming kernel carries the
+// two of row k-1 from the previous node row (same products, same bits).
+template <class D>
+__device__ __forceinline__ void accelerate_node_m(D& dv, const double* mm, const double* pp,
+                                                  const double* qq, double u0v, double v0v,
+                                                  double dx, double dy, double dt, double& uu,
+                                                  double& vv) {
+  const double halfdt = 0.5 * dt;
+  double nodal_mass = (mm[0] + mm[1] + mm[2] + mm[3]) * 0.25;
+  double stepbymass = dv.nz(halfdt, nodal_mass);
+  uu = u0v - stepbymass * (dy * (pp[2] - pp[3]) + dy * (pp[1] - pp[0]));
+  vv = v0v - stepbymass * (dx * (pp[2] - pp[1]) + dx * (pp[3] - pp[0]));
+  uu = uu - stepbymass * (dy * (qq[2] - qq[3]) + dy * (qq[1] - qq[0]));
+  vv = vv - stepbymass * (dx * (qq[2] - qq[1]) + dx * (qq[3] - qq[0]));
+}
+
 template <class D>
 __device__ __forceinline__ void accelerate_node(D& dv, const double* rr, const double* pp,
                                                 const double* qq, double u0v, double v0v,

@@ -455,6 +455,14 @@ __device__ __forceinline__ bool lagr_body(const Chunk& c, const CUtensorMap* __r
     phl_m = __shfl_up_sync(FULL, ph, 1);
   }
   double tsum_m = 0.0, tfc_m = 0.0;  // corrector: top-face sum / flux of the previous row
+  // interior body: cell masses rho*vol of columns j and j-1, previous row
+  const double vol = dx * dy;
+  double mass_m = 0.0, massl_m = 0.0, mass_c = 0.0, massl_c = 0.0;
+  if constexpr (!EDGE) {
+    const double* a = row(k0 - 1);
+    mass_m = a[LF_R * LRW] * vol;
+    massl_m = a[LF_R * LRW - 1] * vol;
+  }
   double u1_m = 0.0, v1_m = 0.0, u1r_m = 0.0, v1r_m = 0.0;
   for (int k = k0; k <= k1; ++k) {
     wait_row(k + 1);
@@ -480,10 +488,18 @@ __device__ __forceinline__ bool lagr_body(const Chunk& c, const CUtensorMap* __r
     // accelerate at node (j,k): cells (j-1,k-1), (j,k-1), (j,k), (j-1,k)
     double u1_c = 0.0, v1_c = 0.0;
     if (colok) {
-      const double rr[4] = {rm[LF_R * LRW - 1], rm[LF_R * LRW], rc[LF_R * LRW], rc[LF_R * LRW - 1]};
       const double pp[4] = {phl_m, ph_m, ph, phl};
       const double qv[4] = {rm[LF_Q * LRW - 1], rm[LF_Q * LRW], rc[LF_Q * LRW], rc[LF_Q * LRW - 1]};
-      accelerate_node(dv, rr, pp, qv, rc[LF_U * LRW], rc[LF_V * LRW], dx, dy, dt, u1_c, v1_c);
+      if constexpr (EDGE) {
+        const double rr[4] = {rm[LF_R * LRW - 1], rm[LF_R * LRW], rc[LF_R * LRW], rc[LF_R * LRW - 1]};
+        accelerate_node(dv, rr, pp, qv, rc[LF_U * LRW], rc[LF_V * LRW], dx, dy, dt, u1_c, v1_c);
+      } else {
+        // cell masses of row k; those of row k-1 are carried from the last row
+        mass_c = rc[LF_R * LRW] * vol;
+        massl_c = rc[LF_R * LRW - 1] * vol;
+        const double mm[4] = {massl_m, mass_m, mass_c, massl_c};
+        accelerate_node_m(dv, mm, pp, qv, rc[LF_U * LRW], rc[LF_V * LRW], dx, dy, dt, u1_c, v1_c);
+      }
     }
     const double u1r_c = __shfl_down_sync(FULL, u1_c, 1);
     const double v1r_c = __shfl_down_sync(FULL, v1_c, 1);
@@ -553,6 +569,7 @@ __device__ __forceinline__ bool lagr_body(const Chunk& c, const CUtensorMap* __r
     ph_m = ph; phl_m = phl;
     u1_m = u1_c; v1_m = v1_c; u1r_m = u1r_c; v1r_m = v1r_c;
     tsum_m = tsum_c; tfc_m = tfc_c;
+    mass_m = mass_c; massl_m = massl_c;
     // row k-1 is consumed (rows k, k+1 are still read next iteration):
     // refill its slot with row k-1+LSTG
 #if CLOVER_TMA_RELEASE_FENCE
