@@ -93,7 +93,7 @@ constexpr int SB = CLOVER_SB;  // threads per block
 #define LB_ADV __launch_bounds__(SB)
 #endif
 #ifndef CLOVER_VKS
-#define CLOVER_VKS 16
+#define CLOVER_VKS 32
 #endif
 #ifndef CLOVER_LKS
 #define CLOVER_LKS 16
@@ -111,8 +111,14 @@ constexpr int SB = CLOVER_SB;  // threads per block
 #define CLOVER_MKS_Y 8
 #endif
 
-#ifndef CLOVER_TMA_RELEASE_FENCE  // proxy fence before refilling a slot (A/B: no measurable cost)
-#define CLOVER_TMA_RELEASE_FENCE 1
+// Proxy fence before a ring slot is refilled.  The slot's shared-memory
+// reads (generic proxy) are all consumed by arithmetic earlier in the same
+// iteration and the warp is converged (__syncwarp) before lane 0 issues the
+// TMA write, the same execution ordering CUTLASS's TMA pipelines rely on
+// for the consumer release (mbarrier arrive, no proxy fence); the fence is
+// kept as an option.  Measured at 3840^2: 0.5 % per step without it.
+#ifndef CLOVER_TMA_RELEASE_FENCE
+#define CLOVER_TMA_RELEASE_FENCE 0
 #endif
 
 // ---------------------------------------------------------------- fix lists
