@@ -801,7 +801,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
         cur_prof_id = sweep == 1 ? P_ADV_Y1 : P_ADV_Y2;
         for (auto& cs : ctx->chunks) {
           const Chunk c = with_rev(cs.c, sweep == 1 ? CLOVER_SERP : 0);
-          const dim3 gw(cdiv(c.nx + 2, SB), 2);
+          const dim3 gw(cdiv(c.nx + 2, SB), CLOVER_YWALLS_ROWS ? 5 : 2);
           if (sweep == 1)
             launch_step(ks_cell_y_walls<1>, gw, SB, st, c, cs.buf[rin], cs.buf[ein], cs.buf[B_FX],
                         cs.buf[B_FY], cs.buf[rout], cs.buf[eout], cs.buf[B_MY]);

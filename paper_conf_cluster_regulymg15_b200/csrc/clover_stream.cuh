@@ -1386,6 +1386,9 @@ constexpr int YKS = CLOVER_YKS;
 #ifndef CLOVER_YMINB1
 #define CLOVER_YMINB1 10
 #endif
+#ifndef CLOVER_YWALLS_ROWS  // ks_cell_y_walls: one thread per (column, band row)
+#define CLOVER_YWALLS_ROWS 1
+#endif
 constexpr int YRW = 36;
 template <int SWEEP> struct YL;
 template <> struct YL<1> {  // tensor d1 e1 u1 v1 fy fx
@@ -1653,6 +1656,50 @@ ks_cell_y_walls(Chunk c, const double* __restrict__ rho, const double* __restric
                 double* __restrict__ mfy) {
   pdl_trigger();
   pdl_wait();
+#if CLOVER_YWALLS_ROWS
+  // one thread per (column, band row): the five band rows (1..3, ny-1, ny)
+  // are independent -- each thread evaluates the two faces of its cell
+  // with the expressions the row-streaming body uses (-fmad=false: same
+  // bits), so the band's latency is one row's division chain, not three.
+  const int b = blockIdx.y;
+  const int k = b < 3 ? 1 + b : c.ny - 4 + b;
+  if (b < 3 && k > c.ny) return;
+  const int jlo = c.wl ? 1 : 0;
+  Chunk cw = c;
+  cw.nx = c.wr ? c.nx : c.nx + 1;
+  const int j = blockIdx.x * SB + threadIdx.x + jlo;
+  if (j > cw.nx) return;
+  DivIEEE dv;
+  const double vol = cw.dx * cw.dy;
+  const int P = cw.pitch;
+  auto pre_vol = [&](int i) -> double {
+    if (SWEEP == 1) return vol + (fy[i + P] - fy[i] + fx[i + 1] - fx[i]);
+    return vol + fy[i + P] - fy[i];
+  };
+  const int i = idx(cw, j, k);
+  const double R0 = rho[i - 2 * P], R1 = rho[i - P], R2 = rho[i], R3 = rho[i + P],
+               R4 = rho[i + 2 * P];
+  const double E0 = en[i - 2 * P], E1 = en[i - P], E2 = en[i], E3 = en[i + P], E4 = en[i + 2 * P];
+  const double pvm = pre_vol(i - P), pv0 = pre_vol(i), pv1 = pre_vol(i + P);
+  double m0, ef0, m1, ef1;
+  {  // face k
+    const double F = fy[i];
+    if (F > 0.0) cell_face_flux(dv, F, pvm, R0, R1, R2, E0, E1, E2, m0, ef0);
+    else cell_face_flux(dv, F, pv0, R3, R2, R1, E3, E2, E1, m0, ef0);
+  }
+  {  // face k+1
+    const double F = fy[i + P];
+    if (F > 0.0) cell_face_flux(dv, F, pv0, R1, R2, R3, E1, E2, E3, m1, ef1);
+    else cell_face_flux(dv, F, pv1, R4, R3, R2, E4, E3, E2, m1, ef1);
+  }
+  double ro, eo;
+  cell_update(dv, R2, E2, pv0, m0, m1, ef0, ef1, fy[i], fy[i + P], ro, eo);
+  const bool near = near_wall_col(cw, j) || near_wall_row(cw, k);
+  store_at(cw, rho_out, K_CELL, j, k, i, near, ro);
+  store_at(cw, en_out, K_CELL, j, k, i, near, eo);
+  store_at(cw, mfy, K_YFACE, j, k, i, near, m0);
+  if (k == cw.ny) store_field(cw, mfy, K_YFACE, j, k + 1, m1);
+#else
   const int lane = threadIdx.x & 31;
   const int gw = blockIdx.x * (SB / 32) + (threadIdx.x >> 5);
   const int k0 = blockIdx.y == 0 ? 1 : c.ny - 1;
@@ -1664,6 +1711,7 @@ ks_cell_y_walls(Chunk c, const double* __restrict__ rho, const double* __restric
   cw.nx = c.wr ? c.nx : c.nx + 1;
   advec_cell_y_body<SWEEP, DivIEEE, true>(cw, rho, en, fx, fy, rho_out, en_out, mfy, gw, k0, k1,
                                           lane, jlo);
+#endif
 }
 
 }  // namespace clover
