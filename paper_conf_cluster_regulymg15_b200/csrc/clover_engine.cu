@@ -695,8 +695,30 @@ static Chunk with_rev(Chunk c, int rev) {
   return c;
 }
 
+// The y-wall band work (YWalls) of advection sweep `sweep`, reading that
+// sweep's inputs and writing its outputs.
+static YWalls ywalls_of(const ChunkState& cs, int sweep) {
+  YWalls y;
+  y.nbx = cdiv(cs.c.nx + 2, SB);
+  y.rho = cs.buf[sweep == 1 ? B_D1 : B_D2];
+  y.en = cs.buf[sweep == 1 ? B_E1 : B_E2];
+  y.fx = cs.buf[B_FX];
+  y.fy = cs.buf[B_FY];
+  y.rho_out = cs.buf[sweep == 1 ? B_D2 : B_D0];
+  y.en_out = cs.buf[sweep == 1 ? B_E2 : B_E0];
+  y.mfy = cs.buf[B_MY];
+  return y;
+}
+static const YWalls kNoWalls = {0, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
+
 int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
   cudaStream_t st = ctx->work;
+  // one chunk on one rank: the y-wall bands ride on the fixup launch before
+  // the y sweep (kf_lagrangian when sweep 1 is y, kf_advec_x<1> when sweep 2
+  // is y), when that sweep is enqueued and fused
+  const bool fold1 = ctx->chunks.size() == 1 && ctx->nranks == 1 && fuse_y_ok(ctx);
+  const bool walls_in_lagr = CLOVER_YWALLS_FOLD && fold1 && !advect_x && nphase >= 4;
+  const bool walls_in_x1 = CLOVER_YWALLS_FOLD && fold1 && advect_x && fuse_x_ok(ctx) && nphase >= 6;
   int cur_prof_id = P_VISC_DT;
   if (ctx->prof) prof_mark(ctx, -1);
   // one chunk on one rank: the visc fixup's last block finalises dt (no
@@ -745,9 +767,10 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
           cs.buf[B_D1], cs.buf[B_E1], cs.buf[B_U1], cs.buf[B_V1], cs.buf[B_FX], cs.buf[B_FY],
           ctx->scal, cs.fix);
       STEP_LAUNCH_CHECK();
-      launch_step(kf_lagrangian, FIX_BLOCKS, SB, st, c, cs.tm_lag,
+      const YWalls yw = walls_in_lagr ? ywalls_of(cs, 1) : kNoWalls;
+      launch_step(kf_lagrangian, FIX_BLOCKS + 5 * yw.nbx, SB, st, c, cs.tm_lag,
           cs.buf[B_D1], cs.buf[B_E1], cs.buf[B_U1], cs.buf[B_V1], cs.buf[B_FX], cs.buf[B_FY],
-          ctx->scal, cs.fix);
+          ctx->scal, cs.fix, yw);
       FIX_LAUNCH_CHECK();
     }
     int rc = exchange(ctx, {B_D1, B_E1, B_U1, B_V1, B_FX, B_FY});
@@ -775,15 +798,16 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
             launch_step(ks_advec_x<1>, g, SB, st, c, cs.tm_x1, cs.buf[rout], cs.buf[eout],
                         cs.buf[uout], cs.buf[vout], cs.fix);
             STEP_LAUNCH_CHECK();
-            launch_step(kf_advec_x<1>, FIX_BLOCKS, SB, st, c, cs.tm_x1, cs.buf[rout], cs.buf[eout],
-                        cs.buf[uout], cs.buf[vout], cs.fix);
+            const YWalls yw = walls_in_x1 ? ywalls_of(cs, 2) : kNoWalls;
+            launch_step(kf_advec_x<1>, FIX_BLOCKS + 5 * yw.nbx, SB, st, c, cs.tm_x1, cs.buf[rout],
+                        cs.buf[eout], cs.buf[uout], cs.buf[vout], cs.fix, yw);
             FIX_LAUNCH_CHECK();
           } else {
             launch_step(ks_advec_x<2>, g, SB, st, c, cs.tm_x2, cs.buf[rout], cs.buf[eout],
                         cs.buf[uout], cs.buf[vout], cs.fix);
             STEP_LAUNCH_CHECK();
             launch_step(kf_advec_x<2>, FIX_BLOCKS, SB, st, c, cs.tm_x2, cs.buf[rout], cs.buf[eout],
-                        cs.buf[uout], cs.buf[vout], cs.fix);
+                        cs.buf[uout], cs.buf[vout], cs.fix, kNoWalls);
             FIX_LAUNCH_CHECK();
           }
         }
@@ -799,15 +823,16 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
       // (ks_advec_y): phase ph_cell runs all, phase ph_cell + 1 is empty
       if (nphase >= ph_cell) {
         cur_prof_id = sweep == 1 ? P_ADV_Y1 : P_ADV_Y2;
+        const bool folded = sweep == 1 ? walls_in_lagr : walls_in_x1;
         for (auto& cs : ctx->chunks) {
+          if (folded) break;
           const Chunk c = with_rev(cs.c, sweep == 1 ? CLOVER_SERP : 0);
-          const dim3 gw(cdiv(c.nx + 2, SB), CLOVER_YWALLS_ROWS ? 5 : 2);
+          const YWalls yw = ywalls_of(cs, sweep);
+          const dim3 gw(yw.nbx, 5);
           if (sweep == 1)
-            launch_step(ks_cell_y_walls<1>, gw, SB, st, c, cs.buf[rin], cs.buf[ein], cs.buf[B_FX],
-                        cs.buf[B_FY], cs.buf[rout], cs.buf[eout], cs.buf[B_MY]);
+            launch_step(ks_cell_y_walls<1>, gw, SB, st, c, yw);
           else
-            launch_step(ks_cell_y_walls<2>, gw, SB, st, c, cs.buf[rin], cs.buf[ein], cs.buf[B_FX],
-                        cs.buf[B_FY], cs.buf[rout], cs.buf[eout], cs.buf[B_MY]);
+            launch_step(ks_cell_y_walls<2>, gw, SB, st, c, yw);
           FIX_LAUNCH_CHECK();
         }
         for (auto& cs : ctx->chunks) {
@@ -1435,10 +1460,13 @@ int clover_kernels_per_step(clover_ctx* ctx, int32_t* out) {
   if (!ctx || !out) return fail(CLOVER_ERR_ARG, "NULL argument");
   // per chunk: visc_dt + fixup, Lagrangian + fixup, the x sweep (fused:
   // kernel + fixup; else cell, mom + 2 fixups), the y sweep (fused: wall
-  // bands, kernel + fixup; else 4); plus k_dt_finalize once unless the
-  // visc fixup finalises dt (one chunk on one rank)
-  const int x = fuse_x_ok(ctx) ? 2 : 4, y = fuse_y_ok(ctx) ? 3 : 4;
-  const int fin = (ctx->chunks.size() == 1 && ctx->nranks == 1) ? 0 : 1;
+  // bands, kernel + fixup; else 4; the bands ride on the previous fixup
+  // launch at one chunk on one rank, enqueue_step); plus k_dt_finalize once
+  // unless the visc fixup finalises dt (one chunk on one rank)
+  const bool one = ctx->chunks.size() == 1 && ctx->nranks == 1;
+  const int x = fuse_x_ok(ctx) ? 2 : 4;
+  const int y = fuse_y_ok(ctx) ? ((CLOVER_YWALLS_FOLD && one && fuse_x_ok(ctx)) ? 2 : 3) : 4;
+  const int fin = one ? 0 : 1;
   *out = (int32_t)(ctx->chunks.size() * (4 + x + y) + fin);
   return CLOVER_OK;
 }

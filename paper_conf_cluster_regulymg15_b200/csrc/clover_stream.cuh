@@ -143,6 +143,7 @@ __device__ __forceinline__ void fix_push(FixSlot f, int lane, unsigned gw, unsig
 struct NoLast {
   __device__ void operator()() const {}
 };
+constexpr int FIX_BLOCKS = 148;  // fixup blocks (one per SM); a launch may add y-wall blocks
 template <class Run, class Last = NoLast>
 __device__ __forceinline__ void fix_loop(FixSlot f, int ks, int nb, int lim, Run&& run,
                                          Last last = {}) {
@@ -154,7 +155,7 @@ __device__ __forceinline__ void fix_loop(FixSlot f, int ks, int nb, int lim, Run
   }
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const unsigned items = n * (unsigned)ks;
-  for (unsigned it = blockIdx.x * (SB / 32) + w; it < items; it += gridDim.x * (SB / 32)) {
+  for (unsigned it = blockIdx.x * (SB / 32) + w; it < items; it += FIX_BLOCKS * (SB / 32)) {
     const uint2 t = f.e[it / ks];
     int ks0, len;
     seg_rows_of((int)t.y, ks, nb, ks0, len);
@@ -165,8 +166,9 @@ __device__ __forceinline__ void fix_loop(FixSlot f, int ks, int nb, int lim, Run
   __syncthreads();
   if (threadIdx.x == 0) {
     __threadfence();
-    if (atomicAdd(f.hdr + 1, 1u) == gridDim.x - 1) {
+    if (atomicAdd(f.hdr + 1, 1u) == FIX_BLOCKS - 1) {
       f.hdr[2] += n;  // cumulative (clover_debug_fix_count)
+      __threadfence();  // every block's fixes before the reset (y_walls_after_fix waits on it)
       f.hdr[0] = 0u;
       f.hdr[1] = 0u;
       __threadfence();
@@ -174,7 +176,88 @@ __device__ __forceinline__ void fix_loop(FixSlot f, int ks, int nb, int lim, Run
     }
   }
 }
-constexpr int FIX_BLOCKS = 148;  // fixup grid (one block per SM)
+
+// ---------------------------------------------------------------- y-wall bands
+// advec_cell y on the wall bands (cell rows 1..3 and ny-1..ny, IEEE
+// division: bitwise the fast path's results) so the fused y sweep finds
+// the mirrored halo rows of the post-sweep density and the y-face mass flux.
+// One thread per (column, band row): the five band rows are independent --
+// each thread evaluates the two faces of its cell with the expressions the
+// row-streaming body (advec_cell_y_body) uses, -fmad=false: same bits -- so
+// the band's latency is one row's division chain.  Halo columns at x chunk
+// boundaries too: the fused y sweep's halo lanes recompute their interior
+// rows but read these wall rows.
+struct YWalls {
+  int nbx;  // blocks per band row (0: no wall work in this launch)
+  const double *rho, *en, *fx, *fy;
+  double *rho_out, *en_out, *mfy;
+};
+template <int SWEEP>
+__device__ __forceinline__ void y_walls_block(const Chunk& c, const YWalls& y, int bx, int b) {
+  const int k = b < 3 ? 1 + b : c.ny - 4 + b;
+  if (b < 3 && k > c.ny) return;
+  const int jlo = c.wl ? 1 : 0;
+  Chunk cw = c;
+  cw.nx = c.wr ? c.nx : c.nx + 1;
+  const int j = bx * SB + threadIdx.x + jlo;
+  if (j > cw.nx) return;
+  const double* __restrict__ rho = y.rho;
+  const double* __restrict__ en = y.en;
+  const double* __restrict__ fx = y.fx;
+  const double* __restrict__ fy = y.fy;
+  DivIEEE dv;
+  const double vol = cw.dx * cw.dy;
+  const int P = cw.pitch;
+  auto pre_vol = [&](int i) -> double {
+    if (SWEEP == 1) return vol + (fy[i + P] - fy[i] + fx[i + 1] - fx[i]);
+    return vol + fy[i + P] - fy[i];
+  };
+  const int i = idx(cw, j, k);
+  const double R0 = rho[i - 2 * P], R1 = rho[i - P], R2 = rho[i], R3 = rho[i + P],
+               R4 = rho[i + 2 * P];
+  const double E0 = en[i - 2 * P], E1 = en[i - P], E2 = en[i], E3 = en[i + P], E4 = en[i + 2 * P];
+  const double pvm = pre_vol(i - P), pv0 = pre_vol(i), pv1 = pre_vol(i + P);
+  double m0, ef0, m1, ef1;
+  {  // face k
+    const double F = fy[i];
+    if (F > 0.0) cell_face_flux(dv, F, pvm, R0, R1, R2, E0, E1, E2, m0, ef0);
+    else cell_face_flux(dv, F, pv0, R3, R2, R1, E3, E2, E1, m0, ef0);
+  }
+  {  // face k+1
+    const double F = fy[i + P];
+    if (F > 0.0) cell_face_flux(dv, F, pv0, R1, R2, R3, E1, E2, E3, m1, ef1);
+    else cell_face_flux(dv, F, pv1, R4, R3, R2, E4, E3, E2, m1, ef1);
+  }
+  double ro, eo;
+  cell_update(dv, R2, E2, pv0, m0, m1, ef0, ef1, fy[i], fy[i + P], ro, eo);
+  const bool near = near_wall_col(cw, j) || near_wall_row(cw, k);
+  store_at(cw, y.rho_out, K_CELL, j, k, i, near, ro);
+  store_at(cw, y.en_out, K_CELL, j, k, i, near, eo);
+  store_at(cw, y.mfy, K_YFACE, j, k, i, near, m0);
+  if (k == cw.ny) store_field(cw, y.mfy, K_YFACE, j, k + 1, m1);
+}
+// The wall bands carried by the fixup launch that precedes the y sweep (one
+// chunk on one rank: one launch hop fewer per step).  Blocks FIX_BLOCKS..
+// wait until the fixups of the previous kernel are done (fix_loop's last
+// block resets hdr[0] after a fence; 0 from the start when nothing was
+// flagged, the common case), then compute the bands.  Every block of the
+// launch is co-resident (small blocks), so the wait cannot starve the fixups.
+template <int SWEEP>
+__device__ __forceinline__ bool y_walls_after_fix(const Chunk& c, FixSlot f, const YWalls& y) {
+  if ((int)blockIdx.x < FIX_BLOCKS) return false;
+  if (threadIdx.x == 0) {
+    unsigned v;
+    for (;;) {
+      asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(f.hdr) : "memory");
+      if (v == 0u) break;
+      __nanosleep(64);
+    }
+  }
+  __syncthreads();
+  const int b = (int)blockIdx.x - FIX_BLOCKS;
+  y_walls_block<SWEEP>(c, y, b % y.nbx, b / y.nbx);
+  return true;
+}
 
 // ================================================================ visc_dt
 // Warp w of the grid owns columns j = 32*w + lane + 1 over rows [k0, k0+VKS).
@@ -631,9 +714,10 @@ __global__ void __launch_bounds__(SB)
 kf_lagrangian(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__ d1,
               double* __restrict__ e1, double* __restrict__ u1, double* __restrict__ v1,
               double* __restrict__ fx, double* __restrict__ fy, const StepScalars* __restrict__ s,
-              FixSlot fix) {
+              FixSlot fix, YWalls yw) {
   pdl_trigger();
   pdl_wait();
+  if (y_walls_after_fix<1>(c, fix, yw)) return;
   __shared__ __align__(128) double ring[SB / 32][LSTG * LSLOT];
   __shared__ __align__(8) unsigned long long bars[SB / 32][LSTG];
   fix_loop(fix, c.lks, c.lnb, c.ny + 1, [&](int gw, int k0, int k1, int lane, int w) {
@@ -1224,9 +1308,11 @@ template <int SWEEP>
 __global__ void __launch_bounds__(SB)
 kf_advec_x(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__ rho_out,
            double* __restrict__ en_out, double* __restrict__ uout, double* __restrict__ vout,
-           FixSlot fix) {
+           FixSlot fix, YWalls yw) {
   pdl_trigger();
   pdl_wait();
+  if constexpr (SWEEP == 1)  // sweep 2 is y
+    if (y_walls_after_fix<2>(c, fix, yw)) return;
   __shared__ __align__(128) double ring[SB / 32][XSTG * xslot<SWEEP>()];
   __shared__ __align__(8) unsigned long long bars[SB / 32][XSTG];
   fix_loop(fix, c.xks, c.xnb, c.ny + 2, [&](int gw, int k0, int k1, int lane, int w) {
@@ -1386,8 +1472,8 @@ constexpr int YKS = CLOVER_YKS;
 #ifndef CLOVER_YMINB1
 #define CLOVER_YMINB1 10
 #endif
-#ifndef CLOVER_YWALLS_ROWS  // ks_cell_y_walls: one thread per (column, band row)
-#define CLOVER_YWALLS_ROWS 1
+#ifndef CLOVER_YWALLS_FOLD  // y-wall bands carried by the preceding fixup launch
+#define CLOVER_YWALLS_FOLD 1
 #endif
 constexpr int YRW = 36;
 template <int SWEEP> struct YL;
@@ -1645,73 +1731,13 @@ kf_advec_y(Chunk c, const __grid_constant__ CUtensorMap ta, const __grid_constan
   });
 }
 
-// advec_cell y on the wall bands (cell rows 1..3 and ny-1..ny, IEEE
-// division: bitwise the fast path's results) so the fused y sweep finds
-// the mirrored halo rows of the post-sweep density and the y-face mass flux.
+// the y-wall bands as their own launch (several chunks or ranks; see YWalls)
 template <int SWEEP>
 __global__ void __launch_bounds__(SB)
-ks_cell_y_walls(Chunk c, const double* __restrict__ rho, const double* __restrict__ en,
-                const double* __restrict__ fx, const double* __restrict__ fy,
-                double* __restrict__ rho_out, double* __restrict__ en_out,
-                double* __restrict__ mfy) {
+ks_cell_y_walls(Chunk c, YWalls y) {
   pdl_trigger();
   pdl_wait();
-#if CLOVER_YWALLS_ROWS
-  // one thread per (column, band row): the five band rows (1..3, ny-1, ny)
-  // are independent -- each thread evaluates the two faces of its cell
-  // with the expressions the row-streaming body uses (-fmad=false: same
-  // bits), so the band's latency is one row's division chain, not three.
-  const int b = blockIdx.y;
-  const int k = b < 3 ? 1 + b : c.ny - 4 + b;
-  if (b < 3 && k > c.ny) return;
-  const int jlo = c.wl ? 1 : 0;
-  Chunk cw = c;
-  cw.nx = c.wr ? c.nx : c.nx + 1;
-  const int j = blockIdx.x * SB + threadIdx.x + jlo;
-  if (j > cw.nx) return;
-  DivIEEE dv;
-  const double vol = cw.dx * cw.dy;
-  const int P = cw.pitch;
-  auto pre_vol = [&](int i) -> double {
-    if (SWEEP == 1) return vol + (fy[i + P] - fy[i] + fx[i + 1] - fx[i]);
-    return vol + fy[i + P] - fy[i];
-  };
-  const int i = idx(cw, j, k);
-  const double R0 = rho[i - 2 * P], R1 = rho[i - P], R2 = rho[i], R3 = rho[i + P],
-               R4 = rho[i + 2 * P];
-  const double E0 = en[i - 2 * P], E1 = en[i - P], E2 = en[i], E3 = en[i + P], E4 = en[i + 2 * P];
-  const double pvm = pre_vol(i - P), pv0 = pre_vol(i), pv1 = pre_vol(i + P);
-  double m0, ef0, m1, ef1;
-  {  // face k
-    const double F = fy[i];
-    if (F > 0.0) cell_face_flux(dv, F, pvm, R0, R1, R2, E0, E1, E2, m0, ef0);
-    else cell_face_flux(dv, F, pv0, R3, R2, R1, E3, E2, E1, m0, ef0);
-  }
-  {  // face k+1
-    const double F = fy[i + P];
-    if (F > 0.0) cell_face_flux(dv, F, pv0, R1, R2, R3, E1, E2, E3, m1, ef1);
-    else cell_face_flux(dv, F, pv1, R4, R3, R2, E4, E3, E2, m1, ef1);
-  }
-  double ro, eo;
-  cell_update(dv, R2, E2, pv0, m0, m1, ef0, ef1, fy[i], fy[i + P], ro, eo);
-  const bool near = near_wall_col(cw, j) || near_wall_row(cw, k);
-  store_at(cw, rho_out, K_CELL, j, k, i, near, ro);
-  store_at(cw, en_out, K_CELL, j, k, i, near, eo);
-  store_at(cw, mfy, K_YFACE, j, k, i, near, m0);
-  if (k == cw.ny) store_field(cw, mfy, K_YFACE, j, k + 1, m1);
-#else
-  const int lane = threadIdx.x & 31;
-  const int gw = blockIdx.x * (SB / 32) + (threadIdx.x >> 5);
-  const int k0 = blockIdx.y == 0 ? 1 : c.ny - 1;
-  const int k1 = blockIdx.y == 0 ? min(4, c.ny + 1) : c.ny + 1;
-  // halo columns at x chunk boundaries too: the fused y sweep's halo lanes
-  // recompute their interior rows but read these wall rows
-  const int jlo = c.wl ? 1 : 0;
-  Chunk cw = c;
-  cw.nx = c.wr ? c.nx : c.nx + 1;
-  advec_cell_y_body<SWEEP, DivIEEE, true>(cw, rho, en, fx, fy, rho_out, en_out, mfy, gw, k0, k1,
-                                          lane, jlo);
-#endif
+  y_walls_block<SWEEP>(c, y, blockIdx.x, blockIdx.y);
 }
 
 }  // namespace clover
