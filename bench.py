@@ -87,7 +87,40 @@ class ClockSampler:
         self._stop = threading.Event()
         self._t = None
 
+    def _nvml_handle(self):
+        """NVML handle of the CUDA device (by UUID, else by index), or None."""
+        try:
+            import pynvml
+            import torch
+            pynvml.nvmlInit()
+            try:
+                u = str(torch.cuda.get_device_properties(self.idx).uuid)
+                return pynvml, pynvml.nvmlDeviceGetHandleByUUID(u if u.startswith("GPU-") else "GPU-" + u)
+            except Exception:
+                return pynvml, pynvml.nvmlDeviceGetHandleByIndex(self.idx)
+        except Exception:
+            return None
+
     def _run(self):
+        nv = self._nvml_handle()
+        if nv is not None:
+            # NVML directly: ~1 ms per sample, so a timed region of tens of
+            # milliseconds still gets many samples (nvidia-smi takes ~0.1 s)
+            p, h = nv
+            bits = (p.nvmlClocksThrottleReasonHwSlowdown, p.nvmlClocksThrottleReasonHwThermalSlowdown,
+                    p.nvmlClocksThrottleReasonSwThermalSlowdown, p.nvmlClocksThrottleReasonSwPowerCap)
+            while not self._stop.is_set():
+                try:
+                    sm = p.nvmlDeviceGetClockInfo(h, p.NVML_CLOCK_SM)
+                    smax = p.nvmlDeviceGetMaxClockInfo(h, p.NVML_CLOCK_SM)
+                    r = p.nvmlDeviceGetCurrentClocksThrottleReasons(h)
+                    self.rows.append([str(self.idx), str(sm), str(smax), "", ""] +
+                                     ["Active" if r & b else "Not Active" for b in bits])
+                except Exception:
+                    break
+                self._stop.wait(0.001)
+            if self.rows:
+                return
         while not self._stop.is_set():
             try:
                 out = subprocess.run(["nvidia-smi", "-i", str(self.idx), f"--query-gpu={self.Q}",
@@ -119,7 +152,8 @@ class ClockSampler:
                     reasons.add(n)
         return {"sm_mhz": statistics.median(sm) if sm else None,
                 "sm_max_mhz": max(smax) if smax else None,
-                "reasons": sorted(reasons), "samples": len(self.rows)}
+                "reasons": sorted(reasons), "samples": len(self.rows),
+                "source": "nvml" if self.rows and self.rows[0][3] == "" else "nvidia-smi"}
 
 
 def oracle_rate(deck, steps, warmup=0):
