@@ -1472,6 +1472,9 @@ constexpr int YKS = CLOVER_YKS;
 #ifndef CLOVER_YMINB1
 #define CLOVER_YMINB1 10
 #endif
+#ifndef CLOVER_L2HINT  // y sweep: L2 policy for the ring rows shared with the segment below
+#define CLOVER_L2HINT 0
+#endif
 #ifndef CLOVER_YWALLS_FOLD  // y-wall bands carried by the preceding fixup launch
 #define CLOVER_YWALLS_FOLD 1
 #endif
@@ -1520,10 +1523,30 @@ __device__ __forceinline__ bool advec_y_body(const Chunk& c, const CUtensorMap* 
   const int x0 = COL0 + J0 - 2;
   const int xcol = x0 & ~1;           // 16-B aligned box start
   const int t0 = 1 + (x0 & 1);        // smem column of lane 0
+#if CLOVER_L2HINT
+  // rows r_first..k0+2 are read again by the segment below at its end, tens
+  // of microseconds later: keep them in L2
+  const unsigned long long pol_keep = l2_policy_evict_last();
+#if CLOVER_L2HINT > 1
+  const unsigned long long pol_once = l2_policy_evict_first();
+#endif
+#endif
   auto issue = [&](int r) {
     const unsigned sl = (unsigned)(r - r_first) % (unsigned)L::RING;
     double* d = ring + sl * L::SLOT;
     mbar_arrive_expect_tx(&bars[sl], L::BYTES);
+#if CLOVER_L2HINT
+    if (r <= k0 + 2) {
+      tma_load_3d_hint(d, ta, xcol, ROW0 + r, 0, &bars[sl], pol_keep);
+      if constexpr (SWEEP == 2) tma_load_3d_hint(d + L::B, tb, xcol, ROW0 + r, 0, &bars[sl], pol_keep);
+      return;
+    }
+#if CLOVER_L2HINT > 1
+    tma_load_3d_hint(d, ta, xcol, ROW0 + r, 0, &bars[sl], pol_once);
+    if constexpr (SWEEP == 2) tma_load_3d_hint(d + L::B, tb, xcol, ROW0 + r, 0, &bars[sl], pol_once);
+    return;
+#endif
+#endif
     tma_load_3d(d, ta, xcol, ROW0 + r, 0, &bars[sl]);
     if constexpr (SWEEP == 2) tma_load_3d(d + L::B, tb, xcol, ROW0 + r, 0, &bars[sl]);
   };
