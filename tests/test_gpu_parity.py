@@ -398,3 +398,16 @@ def test_full_size_first_steps(torch_cuda, n):
     # the sequential oracle sum carries up to n*eps (3e-9) of its own
     # rounding at this size; compare with its compensated twin
     assert_summary_close(g.field_summary(), o.field_summary(compensated=True))
+
+
+@pytest.mark.parametrize("pxy,expected", [((1, 1), 8), ((3, 1), 34), ((1, 3), 31)])
+def test_kernels_per_step(torch_cuda, pxy, expected):
+    """Launches per step (bench.py's gpu_launches): one chunk runs visc_dt,
+    Lagrangian and both fused sweeps with a fixup each, the y-wall bands
+    riding on the fixup before the y sweep (8); several chunks launch the
+    bands separately (+1 per chunk) and finalise dt in k_dt_finalize (+1);
+    x (y) chunk boundaries use the separate x (y) kernels, 4 launches per
+    chunk: 3x1 = 3 * (4 + 4 + 3) + 1, 1x3 = 3 * (4 + 2 + 4) + 1."""
+    px, py = pxy
+    g = make_gpu(fuzz_deck(11), px=px, py=py)
+    assert g.kernels_per_step() == expected
