@@ -86,6 +86,7 @@ class ClockSampler:
         self.rows = []
         self._stop = threading.Event()
         self._t = None
+        self._nv = self._nvml_handle()  # NVML init (~tens of ms) before the timed region
 
     def _nvml_handle(self):
         """NVML handle of the CUDA device (by UUID, else by index), or None."""
@@ -102,7 +103,7 @@ class ClockSampler:
             return None
 
     def _run(self):
-        nv = self._nvml_handle()
+        nv = self._nv
         if nv is not None:
             # NVML directly: ~1 ms per sample, so a timed region of tens of
             # milliseconds still gets many samples (nvidia-smi takes ~0.1 s)
