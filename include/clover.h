@@ -68,7 +68,7 @@ enum { CLOVER_MIRROR_GEOMETRIC = 0, CLOVER_MIRROR_CELLCENTRE = 1 };
  * dtinit/dtmax/dtmin/dtrise/dt*_safe selects the CloverLeaf default
  * 0.1 / 1.0 / 1e-7 / 1.5 / (0.7, 0.5, 0.5, 0.7). */
 typedef struct {
-  int32_t x_cells, y_cells;         /* global mesh, >= 2 each */
+  int32_t x_cells, y_cells;         /* global mesh, >= 4 each */
   double xmin, ymin, xmax, ymax;    /* domain, xmax > xmin, ymax > ymin */
   double dtinit, dtmax, dtmin, dtrise;
   double dtc_safe, dtu_safe, dtv_safe, dtdiv_safe;
@@ -150,7 +150,7 @@ int clover_nccl_unique_id(void* out128);
 
 /* Create a context: carve fields from `workspace`, paint the states
  * (generate_chunk), compute the EOS and prime all halos (start of run,
- * SURVEY 8(c) c.1).  Validation: x_cells,y_cells >= 2; nstates >= 1;
+ * SURVEY 8(c) c.1).  Validation: x_cells,y_cells >= 4; nstates >= 1;
  * xmax > xmin; ymax > ymin; px*py >= nranks and divisible by nranks; every
  * chunk at least 4x4 cells.  On error *out is NULL. */
 int clover_init(const clover_grid* grid, const clover_state* states, int32_t nstates,
