@@ -256,7 +256,7 @@ struct clover_ctx {
   bool use_graphs = true;
   bool fuse_x = true;  // fused x sweep where every chunk has both x walls (see fuse_x_ok)
   bool fuse_y = true;  // fused y sweep (see fuse_y_ok)
-  cudaGraphExec_t gexec[2] = {nullptr, nullptr};
+  cudaGraphExec_t gexec[4] = {nullptr, nullptr, nullptr, nullptr};  // [parity + 2 * multi-step]
   int64_t ws_bytes = 0;
   bool prof = false;
   bool virtual_remote = false;  // test mode: every chunk boundary takes the NCCL packing path
@@ -951,17 +951,26 @@ int join_out(clover_ctx* ctx) {
   return CLOVER_OK;
 }
 
-int build_graph(clover_ctx* ctx, int parity) {
+// Steps per multi-step graph: consecutive steps in one graph keep the
+// programmatic (PDL) edges across the step boundary, which a graph launch
+// per step breaks.
+#ifndef CLOVER_GRAPH_STEPS
+#define CLOVER_GRAPH_STEPS 1
+#endif
+// Graph of `nst` consecutive steps starting with sweep order `parity`
+// (0: x first), instantiated into gexec[slot].
+int build_graph(clover_ctx* ctx, int parity, int nst, int slot) {
   cudaGraph_t graph = nullptr;
   CK(cudaStreamBeginCapture(ctx->work, cudaStreamCaptureModeThreadLocal));
-  int rc = enqueue_step(ctx, parity == 0, 7);
+  int rc = 0;
+  for (int i = 0; i < nst && !rc; ++i) rc = enqueue_step(ctx, (parity == 0) != (i % 2 == 1), 7);
   cudaError_t e = cudaStreamEndCapture(ctx->work, &graph);
   if (rc) {
     if (graph) cudaGraphDestroy(graph);
     return rc;
   }
   if (e != cudaSuccess) return fail(CLOVER_ERR_CUDA, std::string("capture: ") + cudaGetErrorString(e));
-  e = cudaGraphInstantiate(&ctx->gexec[parity], graph, 0);
+  e = cudaGraphInstantiate(&ctx->gexec[slot], graph, 0);
   cudaGraphDestroy(graph);
   if (e != cudaSuccess) return fail(CLOVER_ERR_CUDA, std::string("instantiate: ") + cudaGetErrorString(e));
   return CLOVER_OK;
@@ -1423,7 +1432,7 @@ int clover_debug_set_virtual_remote(clover_ctx* ctx, int32_t enable) {
   if (ctx->nranks > 1) return fail(CLOVER_ERR_STATE, "virtual remote is a single-process test mode");
   if (enable && ctx->L.px * ctx->L.py < 2) return fail(CLOVER_ERR_STATE, "virtual remote needs px*py > 1");
   ctx->virtual_remote = enable != 0;
-  for (int i = 0; i < 2; ++i)
+  for (int i = 0; i < 4; ++i)
     if (ctx->gexec[i]) {
       cudaGraphExecDestroy(ctx->gexec[i]);
       ctx->gexec[i] = nullptr;
@@ -1435,7 +1444,7 @@ int clover_debug_set_fusion(clover_ctx* ctx, int32_t enable) {
   if (!ctx) return fail(CLOVER_ERR_ARG, "ctx is NULL");
   ctx->fuse_x = enable != 0;
   ctx->fuse_y = enable != 0;
-  for (int i = 0; i < 2; ++i)
+  for (int i = 0; i < 4; ++i)
     if (ctx->gexec[i]) {
       cudaGraphExecDestroy(ctx->gexec[i]);
       ctx->gexec[i] = nullptr;
@@ -1479,9 +1488,20 @@ int clover_step(clover_ctx* ctx, int32_t nsteps) {
   if (rc) return rc;
   for (int i = 0; i < nsteps; ++i) {
     const int parity = ctx->advect_x ? 0 : 1;
+    if (ctx->use_graphs && CLOVER_GRAPH_STEPS > 1 && nsteps - i >= CLOVER_GRAPH_STEPS) {
+      const int slot = parity + 2;
+      if (!ctx->gexec[slot]) {
+        rc = build_graph(ctx, parity, CLOVER_GRAPH_STEPS, slot);
+        if (rc) return rc;
+      }
+      CK(cudaGraphLaunch(ctx->gexec[slot], ctx->work));
+      i += CLOVER_GRAPH_STEPS - 1;
+      if (CLOVER_GRAPH_STEPS % 2) ctx->advect_x = !ctx->advect_x;
+      continue;
+    }
     if (ctx->use_graphs) {
       if (!ctx->gexec[parity]) {
-        rc = build_graph(ctx, parity);
+        rc = build_graph(ctx, parity, 1, parity);
         if (rc) return rc;
       }
       CK(cudaGraphLaunch(ctx->gexec[parity], ctx->work));
@@ -1884,7 +1904,7 @@ int clover_finalize(clover_ctx* ctx) {
   if (ctx->work) {
     rc = check_err(ctx);
   }
-  for (int i = 0; i < 2; ++i)
+  for (int i = 0; i < 4; ++i)
     if (ctx->gexec[i]) cudaGraphExecDestroy(ctx->gexec[i]);
 #ifdef CLOVER_WITH_NCCL
   if (ctx->comm) ncclCommDestroy(ctx->comm);
