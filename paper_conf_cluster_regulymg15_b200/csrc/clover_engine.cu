@@ -631,16 +631,22 @@ void prof_mark(clover_ctx* ctx, int id) {
 }
 
 
+// Programmatic dependent launch (the kernels call pdl_trigger/pdl_wait,
+// clover_common.cuh): launch latency and the next grid's block scheduling
+// overlap the previous grid's tail; graph capture keeps the edges.  Used
+// for the IEEE-fixup launches only (CLOVER_PDL_FIX): a streaming kernel
+// launched early behind a fixup measured slower (same box, ms/step, PDL on
+// streaming/fixup launches: on/on 0.8925, off/off 0.8905, off/on 0.8903 at
+// 3840^2; 960^2 0.1495 / 0.1453 / 0.1435; 7680^2 3.26 / 3.24 / 3.24).
 #ifndef CLOVER_PDL
-#define CLOVER_PDL 1
+#define CLOVER_PDL 0
 #endif
-// Launch a step kernel with programmatic dependent launch (the kernels call
-// pdl_trigger/pdl_wait, clover_common.cuh), so launch latency and the next
-// grid's block scheduling overlap the previous grid's tail.  Graph capture
-// keeps the programmatic edges.
+#ifndef CLOVER_PDL_FIX
+#define CLOVER_PDL_FIX 1
+#endif
 template <typename... KArgs, typename... Args>
-cudaError_t launch_step(void (*kernel)(KArgs...), dim3 grid, dim3 block, cudaStream_t st,
-                        Args&&... args) {
+cudaError_t launch_pdl(int pdl, void (*kernel)(KArgs...), dim3 grid, dim3 block, cudaStream_t st,
+                       Args&&... args) {
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = grid;
   cfg.blockDim = block;
@@ -648,10 +654,22 @@ cudaError_t launch_step(void (*kernel)(KArgs...), dim3 grid, dim3 block, cudaStr
   cfg.stream = st;
   cudaLaunchAttribute at[1];
   at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-  at[0].val.programmaticStreamSerializationAllowed = CLOVER_PDL;
+  at[0].val.programmaticStreamSerializationAllowed = pdl;
   cfg.attrs = at;
   cfg.numAttrs = 1;
   return cudaLaunchKernelEx(&cfg, kernel, std::forward<Args>(args)...);
+}
+template <typename... KArgs, typename... Args>
+cudaError_t launch_step(void (*kernel)(KArgs...), dim3 grid, dim3 block, cudaStream_t st,
+                        Args&&... args) {
+  return launch_pdl(CLOVER_PDL, kernel, grid, block, st, std::forward<Args>(args)...);
+}
+// IEEE-fixup launches (kf_*): their programmatic edge to the streaming
+// kernel before them is set separately (CLOVER_PDL_FIX)
+template <typename... KArgs, typename... Args>
+cudaError_t launch_fix(void (*kernel)(KArgs...), dim3 grid, dim3 block, cudaStream_t st,
+                       Args&&... args) {
+  return launch_pdl(CLOVER_PDL_FIX, kernel, grid, block, st, std::forward<Args>(args)...);
 }
 
 // The fused x sweep needs every chunk to have reflective walls on both x
@@ -730,7 +748,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
       launch_step(ks_visc_dt, dim3(grid_cols(c.nx, c.ny, c.vks).x, seg_count(c.vks, c.vnb, c.ny)), SB, st, c, cs.tm_visc, cs.buf[B_Q],
                   ctx->scal, ctx->dtp, cs.fix);
       STEP_LAUNCH_CHECK();
-      launch_step(kf_visc_dt, FIX_BLOCKS, SB, st, c, cs.tm_visc, cs.buf[B_Q], ctx->scal, ctx->dtp,
+      launch_fix(kf_visc_dt, FIX_BLOCKS, SB, st, c, cs.tm_visc, cs.buf[B_Q], ctx->scal, ctx->dtp,
                   cs.fix, ctx->hist, fold_fin);
       FIX_LAUNCH_CHECK();
     }
@@ -768,7 +786,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
           ctx->scal, cs.fix);
       STEP_LAUNCH_CHECK();
       const YWalls yw = walls_in_lagr ? ywalls_of(cs, 1) : kNoWalls;
-      launch_step(kf_lagrangian, FIX_BLOCKS + 5 * yw.nbx, SB, st, c, cs.tm_lag,
+      launch_fix(kf_lagrangian, FIX_BLOCKS + 5 * yw.nbx, SB, st, c, cs.tm_lag,
           cs.buf[B_D1], cs.buf[B_E1], cs.buf[B_U1], cs.buf[B_V1], cs.buf[B_FX], cs.buf[B_FY],
           ctx->scal, cs.fix, yw);
       FIX_LAUNCH_CHECK();
@@ -799,14 +817,14 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
                         cs.buf[uout], cs.buf[vout], cs.fix);
             STEP_LAUNCH_CHECK();
             const YWalls yw = walls_in_x1 ? ywalls_of(cs, 2) : kNoWalls;
-            launch_step(kf_advec_x<1>, FIX_BLOCKS + 5 * yw.nbx, SB, st, c, cs.tm_x1, cs.buf[rout],
+            launch_fix(kf_advec_x<1>, FIX_BLOCKS + 5 * yw.nbx, SB, st, c, cs.tm_x1, cs.buf[rout],
                         cs.buf[eout], cs.buf[uout], cs.buf[vout], cs.fix, yw);
             FIX_LAUNCH_CHECK();
           } else {
             launch_step(ks_advec_x<2>, g, SB, st, c, cs.tm_x2, cs.buf[rout], cs.buf[eout],
                         cs.buf[uout], cs.buf[vout], cs.fix);
             STEP_LAUNCH_CHECK();
-            launch_step(kf_advec_x<2>, FIX_BLOCKS, SB, st, c, cs.tm_x2, cs.buf[rout], cs.buf[eout],
+            launch_fix(kf_advec_x<2>, FIX_BLOCKS, SB, st, c, cs.tm_x2, cs.buf[rout], cs.buf[eout],
                         cs.buf[uout], cs.buf[vout], cs.fix, kNoWalls);
             FIX_LAUNCH_CHECK();
           }
@@ -844,14 +862,14 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
             launch_step(ks_advec_y<1>, g, SB, st, c, ta, tb, cs.buf[rout], cs.buf[eout], cs.buf[B_MY],
                         cs.buf[uout], cs.buf[vout], cs.fix);
             STEP_LAUNCH_CHECK();
-            launch_step(kf_advec_y<1>, FIX_BLOCKS, SB, st, c, ta, tb, cs.buf[rout], cs.buf[eout],
+            launch_fix(kf_advec_y<1>, FIX_BLOCKS, SB, st, c, ta, tb, cs.buf[rout], cs.buf[eout],
                         cs.buf[B_MY], cs.buf[uout], cs.buf[vout], cs.fix);
             FIX_LAUNCH_CHECK();
           } else {
             launch_step(ks_advec_y<2>, g, SB, st, c, ta, tb, cs.buf[rout], cs.buf[eout], cs.buf[B_MY],
                         cs.buf[uout], cs.buf[vout], cs.fix);
             STEP_LAUNCH_CHECK();
-            launch_step(kf_advec_y<2>, FIX_BLOCKS, SB, st, c, ta, tb, cs.buf[rout], cs.buf[eout],
+            launch_fix(kf_advec_y<2>, FIX_BLOCKS, SB, st, c, ta, tb, cs.buf[rout], cs.buf[eout],
                         cs.buf[B_MY], cs.buf[uout], cs.buf[vout], cs.fix);
             FIX_LAUNCH_CHECK();
           }
@@ -873,12 +891,12 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
           if (sweep == 1) {
             launch_step(ks_advec_cell_x<1>, g, SB, st, c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf], cs.fix);
             STEP_LAUNCH_CHECK();
-            launch_step(kf_advec_cell_x<1>, FIX_BLOCKS, SB, st, c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf], cs.fix);
+            launch_fix(kf_advec_cell_x<1>, FIX_BLOCKS, SB, st, c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf], cs.fix);
             FIX_LAUNCH_CHECK();
           } else {
             launch_step(ks_advec_cell_x<2>, g, SB, st, c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf], cs.fix);
             STEP_LAUNCH_CHECK();
-            launch_step(kf_advec_cell_x<2>, FIX_BLOCKS, SB, st, c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf], cs.fix);
+            launch_fix(kf_advec_cell_x<2>, FIX_BLOCKS, SB, st, c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf], cs.fix);
             FIX_LAUNCH_CHECK();
           }
         } else {
@@ -886,12 +904,12 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
           if (sweep == 1) {
             launch_step(ks_advec_cell_y<1>, g, SB, st, c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf], cs.fix);
             STEP_LAUNCH_CHECK();
-            launch_step(kf_advec_cell_y<1>, FIX_BLOCKS, SB, st, c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf], cs.fix);
+            launch_fix(kf_advec_cell_y<1>, FIX_BLOCKS, SB, st, c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf], cs.fix);
             FIX_LAUNCH_CHECK();
           } else {
             launch_step(ks_advec_cell_y<2>, g, SB, st, c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf], cs.fix);
             STEP_LAUNCH_CHECK();
-            launch_step(kf_advec_cell_y<2>, FIX_BLOCKS, SB, st, c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf], cs.fix);
+            launch_fix(kf_advec_cell_y<2>, FIX_BLOCKS, SB, st, c, cs.buf[rin], cs.buf[ein], fx, fy, cs.buf[rout], cs.buf[eout], cs.buf[mbuf], cs.fix);
             FIX_LAUNCH_CHECK();
           }
         }
@@ -909,12 +927,12 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
           if (sweep == 1) {
             launch_step(ks_advec_mom_x<1>, g, SB, st, c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FY], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout], cs.fix);
             STEP_LAUNCH_CHECK();
-            launch_step(kf_advec_mom_x<1>, FIX_BLOCKS, SB, st, c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FY], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout], cs.fix);
+            launch_fix(kf_advec_mom_x<1>, FIX_BLOCKS, SB, st, c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FY], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout], cs.fix);
             FIX_LAUNCH_CHECK();
           } else {
             launch_step(ks_advec_mom_x<2>, g, SB, st, c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FY], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout], cs.fix);
             STEP_LAUNCH_CHECK();
-            launch_step(kf_advec_mom_x<2>, FIX_BLOCKS, SB, st, c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FY], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout], cs.fix);
+            launch_fix(kf_advec_mom_x<2>, FIX_BLOCKS, SB, st, c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FY], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout], cs.fix);
             FIX_LAUNCH_CHECK();
           }
         } else {
@@ -922,12 +940,12 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
           if (sweep == 1) {
             launch_step(ks_advec_mom_y<1>, g, SB, st, c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FX], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout], cs.fix);
             STEP_LAUNCH_CHECK();
-            launch_step(kf_advec_mom_y<1>, FIX_BLOCKS, SB, st, c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FX], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout], cs.fix);
+            launch_fix(kf_advec_mom_y<1>, FIX_BLOCKS, SB, st, c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FX], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout], cs.fix);
             FIX_LAUNCH_CHECK();
           } else {
             launch_step(ks_advec_mom_y<2>, g, SB, st, c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FX], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout], cs.fix);
             STEP_LAUNCH_CHECK();
-            launch_step(kf_advec_mom_y<2>, FIX_BLOCKS, SB, st, c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FX], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout], cs.fix);
+            launch_fix(kf_advec_mom_y<2>, FIX_BLOCKS, SB, st, c, cs.buf[rout], cs.buf[mbuf], cs.buf[B_FX], cs.buf[uin], cs.buf[vin], cs.buf[uout], cs.buf[vout], cs.fix);
             FIX_LAUNCH_CHECK();
           }
         }
