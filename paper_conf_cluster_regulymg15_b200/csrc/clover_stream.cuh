@@ -143,7 +143,10 @@ __device__ __forceinline__ void fix_push(FixSlot f, int lane, unsigned gw, unsig
 struct NoLast {
   __device__ void operator()() const {}
 };
-constexpr int FIX_BLOCKS = 148;  // fixup blocks (one per SM); a launch may add y-wall blocks
+#ifndef CLOVER_FIX_BLOCKS
+#define CLOVER_FIX_BLOCKS 148
+#endif
+constexpr int FIX_BLOCKS = CLOVER_FIX_BLOCKS;  // fixup blocks (one per SM); a launch may add y-wall blocks
 template <class Run, class Last = NoLast>
 __device__ __forceinline__ void fix_loop(FixSlot f, int ks, int nb, int lim, Run&& run,
                                          Last last = {}) {
