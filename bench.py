@@ -52,10 +52,12 @@ ALGO_BYTES_PER_CELL = {
     "k_advec_y<1>": 8 * (6 + 4),         # fused y sweep: rho e Fx Fy u v -> rho' e' u v
     "k_advec_y<2>": 8 * (5 + 4),         # rho e Fy u v -> rho' e' u v
 }
-# sum over one step of the kernels actually launched (the profile pass
-# below); with the fused x sweep 304/312 B for the x-first/y-first step,
-# 336 with separate kernels
-STEP_ALGO_BYTES_PER_CELL = 336
+# (the step total is summed over the kernels actually launched in the
+# profile pass below: 280 B/cell-step with the fused sweeps)
+
+# Issue roofline: every SM sub-partition issues at most one
+# warp instruction per cycle, 4 per SM.
+ISSUE_PER_SM_PER_CLK = 4
 
 
 def env_int(name, default):
@@ -157,6 +159,55 @@ class ClockSampler:
                 "source": "nvml" if self.rows and self.rows[0][3] == "" else "nvidia-smi"}
 
 
+def host_cpu():
+    """CPU model and logical core count of this host (for cpu_baseline)."""
+    model = None
+    try:
+        with open("/proc/cpuinfo") as fh:
+            for line in fh:
+                if line.startswith("model name"):
+                    model = line.split(":", 1)[1].strip()
+                    break
+    except OSError:
+        pass
+    sockets = None
+    try:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=5).stdout
+        for line in out.splitlines():
+            if line.startswith("Socket(s):"):
+                sockets = int(line.split(":", 1)[1])
+    except Exception:
+        pass
+    return {"cpu_model": model, "nproc": os.cpu_count(), "sockets": sockets}
+
+
+def issue_roofline(kernels, top, sm_mhz, nsm):
+    """Second roofline: warp instructions per
+    launch of the dominant kernel (ncu, profiles/ncu_instr.json, same mesh)
+    over its live CUDA-event duration, against the issue peak of nsm SMs x
+    4 sub-partitions x 1 warp instruction per cycle at the SM clock sampled
+    during the timed region; plus the kernel's fp64-pipe utilisation from the
+    same capture."""
+    p = os.path.join(ROOT, "profiles", "ncu_instr.json")
+    if not os.path.exists(p) or not sm_mhz:
+        return None
+    with open(p) as fh:
+        d = json.load(fh)
+    ent = d.get("kernels", {}).get(top)
+    if not ent:
+        return None
+    avg_s = kernels[top]["avg_ms"] / 1e3
+    ach = ent["warp_inst_per_launch"] / avg_s / 1e12
+    peak = nsm * ISSUE_PER_SM_PER_CLK * sm_mhz * 1e6 / 1e12
+    return {"bound": "issue", "kernel": top, "achieved": ach, "peak": peak, "unit": "T warp-inst/s",
+            "frac": ach / peak, "thread_inst_per_cell": ent.get("thread_inst_per_cell"),
+            "fp64_pipe_pct_active": ent.get("fp64_pipe_pct"),
+            "issue_active_pct_ncu": ent.get("issue_active_pct"),
+            "peak_source": f"{nsm} SMs x {ISSUE_PER_SM_PER_CLK} warp-inst/clk x median SM clock "
+                           f"{sm_mhz:.0f} MHz under load (B200_PROFILING.md unit counts)",
+            "inst_source": d.get("source")}
+
+
 def oracle_rate(deck, steps, warmup=0):
     """Time the CPU oracle (as it stands, single-threaded) on `deck`."""
     from oracle import Oracle
@@ -194,6 +245,7 @@ def run_reference(args):
     t = time.perf_counter() - t0
     cells = deck["x_cells"] * deck["y_cells"]
     v = cells * args.steps / t
+    hc = host_cpu()
     sample = (f"oracle (single-threaded C++ -O2) on a bounded sample of configs[2]: the bottom "
               f"{deck['y_cells']} rows of the 3840^2 bm mesh at the same cell size "
               f"({cells} cells) per step, {args.steps} timed steps after {args.warmup} warm-up")
@@ -203,7 +255,8 @@ def run_reference(args):
             "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": "configs[2] sample: CloverLeaf 2D bm deck, 3840 x 240 band",
                        "mesh": [deck["x_cells"], deck["y_cells"]]},
-            "cpu_baseline": {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
+            "cpu_baseline": {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample,
+                             **hc},
             "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
@@ -217,6 +270,7 @@ def main():
     ap.add_argument("--mesh", type=int, nargs=2, default=None, help="override global mesh (nx ny)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-full", action="store_true", help="skip the full 300-step configs[2] run")
     ap.add_argument("--no-active", action="store_true",
                     help="skip the fully-active-flow side measurement")
     ap.add_argument("--strong", action="store_true",
@@ -326,6 +380,8 @@ def main():
                 "frac": ach / peak if ach else None, "traffic": traffic, "peak_source": peak_src,
                 "step_achieved": step_gbs, "step_frac": step_gbs / peak,
                 "algo_bytes_per_cell_step": step_bpc}
+    nsm = torch.cuda.get_device_properties(dev).multi_processor_count
+    roofline["alu"] = issue_roofline(kernels, top, clk.get("sm_mhz"), nsm)
 
     # end-to-end through the host-buffer C-ABI entry (pinned host memory)
     e2e = None
@@ -375,6 +431,36 @@ def main():
                      host_transport=ht)
         sim.step(args.steps + args.warmup)
 
+    # full configs[2] run: all 300 steps from step 0, each on a
+    # freshly initialised context (median of 3, after one warm-up context);
+    # covers the late, fully developed flow as well as the cheap early steps
+    full = None
+    if world == 1 and not args.no_full and not args.mesh and not args.strong:
+        sim.close()
+        nfull = 300
+        times = []
+        for rep in range(4):
+            f = Clover(deck, stream=stream)
+            f.sync()
+            f0, f1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            torch.cuda.synchronize()
+            f0.record(stream)
+            f.step(nfull)
+            f1.record(stream)
+            torch.cuda.synchronize()
+            f.sync()
+            if rep:
+                times.append(f0.elapsed_time(f1))
+            f.close()
+        fms = statistics.median(times)
+        full = {"steps": nfull, "ms": fms, "ms_per_step": fms / nfull,
+                "value": cells * nfull / (fms / 1e3), "unit": UNIT, "repeats_ms": times,
+                "how": "clover_step(ctx, 300) from step 0 on a fresh context, CUDA events, "
+                       "median of 3 after one warm-up context (graphs on)"}
+        sim = Clover(deck, px=px, py=py, rank=rank, nranks=world, unique_id=uid, stream=stream,
+                     host_transport=ht)
+        sim.step(args.steps + args.warmup)
+
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         cdeck = bm_deck(nx, ny)
@@ -382,6 +468,7 @@ def main():
         cpu = {"value": rate, "unit": UNIT, "cores": 1, "kind": "oracle",
                "sample": f"first 6 steps of the same {nx}x{ny} bm workload, single-threaded "
                          f"C++ oracle (-O2), {t:.1f} s"}
+        cpu.update(host_cpu())
 
     summ = sim.field_summary()
     if rank == 0:
@@ -404,6 +491,7 @@ def main():
                 "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "clocks": clk,
                 "kernels": kernels,
                 "active_flow": active,
+                "full_run": full,
                 "summary_after": summ}
         print(json.dumps(line), flush=True)
     sim.close()

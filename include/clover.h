@@ -27,7 +27,8 @@
  *    caller keeps ownership.
  *  - Streams: all device work is enqueued on the cudaStream_t passed to
  *    clover_init (NULL = legacy default stream).  clover_step is
- *    asynchronous; errors detected on the device (small dt) are latched and
+ *    asynchronous; errors detected on the device (small dt, negative
+ *    volume in PdV) are latched (the first one wins) and
  *    returned by the next synchronising call (clover_field_summary,
  *    clover_get_clock, clover_read_field, clover_sync, clover_finalize).
  *  - Multi-GPU: one process per GPU; the mesh is 2D-block decomposed into
@@ -56,7 +57,11 @@ enum {
   CLOVER_ERR_NCCL = -3,       /* an NCCL call failed or NCCL is unavailable */
   CLOVER_ERR_WORKSPACE = -4,  /* workspace too small or misaligned */
   CLOVER_ERR_SMALL_DT = -5,   /* dt < dtmin: the reference's "small timestep" abort */
-  CLOVER_ERR_STATE = -7       /* call not valid in the current state */
+  CLOVER_ERR_NEG_VOLUME = -6, /* PdV corrector: volume + total_flux is not
+                                 > 0 in some cell (negative volume, or NaN in the fluxes);
+                                 latched on the device, the step's results are invalid */
+  CLOVER_ERR_STATE = -7,      /* call not valid in the current state */
+  CLOVER_ERR_NAN = -8         /* clover_field_summary: a total is NaN */
 };
 
 enum { CLOVER_GEOM_RECT = 1, CLOVER_GEOM_CIRCLE = 2, CLOVER_GEOM_POINT = 3 };
@@ -173,15 +178,22 @@ int clover_step_host(clover_ctx* ctx, int32_t nsteps,
                      double* xvel0_out, double* yvel0_out);
 
 /* Global field_summary over all chunks and ranks; synchronises.  The
- * reduction is deterministic: fixed 16x16-cell tiles aligned to the global
- * index, summed in global tile order, so every decomposition gives the same
- * bits. */
+ * reduction is deterministic: each 16x16-cell tile aligned to the global
+ * index is reduced in a fixed order on the device (row sums by warp
+ * shuffles, then a fixed tree), and the tile partials are summed in global
+ * tile order on the host, so every decomposition gives the same bits.
+ * Returns CLOVER_ERR_NAN (the totals are still written) if a total is NaN,
+ * else a latched device error if any.  Multi-rank contexts all-gather the
+ * tile partials through a temporary device buffer (an I/O path, like
+ * clover_read_field). */
 int clover_field_summary(clover_ctx* ctx, clover_summary* out);
 
 /* Step counter, simulated time and the last dt; synchronises. */
 int clover_get_clock(clover_ctx* ctx, int32_t* step, double* time, double* dt_last);
 
-/* dt of steps [first, first+n) (1-based step numbers, last 4096 kept). */
+/* dt of steps [first, first+n) (1-based step numbers, last 4096 kept).
+ * After clover_restart only steps after the checkpoint's step are known:
+ * earlier ones are rejected with CLOVER_ERR_ARG. */
 int clover_dt_history(clover_ctx* ctx, int32_t first, int32_t n, double* host_out);
 
 /* Gather a field's global interior into host memory (n = element count of

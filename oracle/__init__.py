@@ -105,7 +105,8 @@ class Oracle:
                        xmin=deck["xmin"], ymin=deck["ymin"], xmax=deck["xmax"], ymax=deck["ymax"],
                        dtinit=deck.get("initial_timestep", 0.04), dtmax=deck.get("max_timestep", 0.04),
                        dtmin=deck.get("dtmin", 0.0), dtrise=deck.get("timestep_rise", 1.5),
-                       dtc_safe=0.0, dtu_safe=0.0, dtv_safe=0.0, dtdiv_safe=0.0,
+                       dtc_safe=deck.get("dtc_safe", 0.0), dtu_safe=deck.get("dtu_safe", 0.0),
+                       dtv_safe=deck.get("dtv_safe", 0.0), dtdiv_safe=deck.get("dtdiv_safe", 0.0),
                        advect_x_first=int(deck.get("advect_x_first", 1)),
                        face_mirror=int(deck.get("face_mirror", 0)))
         sts = deck["states"]

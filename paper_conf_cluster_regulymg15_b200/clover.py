@@ -23,7 +23,8 @@ dptr = ctypes.POINTER(c_double)
 
 CLOVER_OK = 0
 PROFILE_SLOTS = 15
-ERRORS = {-1: "ARG", -2: "CUDA", -3: "NCCL", -4: "WORKSPACE", -5: "SMALL_DT", -7: "STATE"}
+ERRORS = {-1: "ARG", -2: "CUDA", -3: "NCCL", -4: "WORKSPACE", -5: "SMALL_DT", -6: "NEG_VOLUME",
+          -7: "STATE", -8: "NAN"}
 
 FIELDS = {"density0": 0, "energy0": 1, "pressure": 2, "viscosity": 3, "soundspeed": 4,
           "xvel0": 5, "yvel0": 6, "vol_flux_x": 11, "vol_flux_y": 12,
@@ -161,7 +162,8 @@ def grid_from_deck(deck: dict) -> CloverGrid:
                       ymin=deck["ymin"], xmax=deck["xmax"], ymax=deck["ymax"],
                       dtinit=deck.get("initial_timestep", 0.04), dtmax=deck.get("max_timestep", 0.04),
                       dtmin=deck.get("dtmin", 0.0), dtrise=deck.get("timestep_rise", 1.5),
-                      dtc_safe=0.0, dtu_safe=0.0, dtv_safe=0.0, dtdiv_safe=0.0,
+                      dtc_safe=deck.get("dtc_safe", 0.0), dtu_safe=deck.get("dtu_safe", 0.0),
+                      dtv_safe=deck.get("dtv_safe", 0.0), dtdiv_safe=deck.get("dtdiv_safe", 0.0),
                       advect_x_first=int(deck.get("advect_x_first", 1)),
                       face_mirror=int(deck.get("face_mirror", 0)))
 

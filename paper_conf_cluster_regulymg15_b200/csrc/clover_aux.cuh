@@ -125,18 +125,22 @@ __global__ void k_eos_field(Chunk c, const double* __restrict__ d0, const double
   out[i] = soundspeed ? eos_soundspeed_ieee(d0[i], e0[i]) : eos_pressure(d0[i], e0[i]);
 }
 
-// field_summary (c.12): one 16x16 tile of cells per CTA; per-cell terms
-// reduced in a fixed binary tree, written as 5 partials per tile.
+// field_summary (c.12): one 16x16 tile of cells per CTA (8 warps of two
+// tile rows each).  Per-cell terms are reduced in a fixed order: a warp
+// butterfly (__shfl_xor_sync, offsets 16..1; a+b and b+a round alike, so
+// every lane holds the same bits), then the 8 warp sums in warp order by
+// one thread; 5 partials per tile.  The tiles are aligned to the global
+// index, so the bits do not depend on the decomposition.
 constexpr int ST = 16;
 __global__ void __launch_bounds__(ST * ST)
 k_summary(Chunk c, const double* __restrict__ d0, const double* __restrict__ e0,
           const double* __restrict__ u0, const double* __restrict__ v0,
           double* __restrict__ partials) {
-  __shared__ double red[5][ST * ST];
+  __shared__ double red[5][ST * ST / 32];
   const int j = blockIdx.x * ST + threadIdx.x + 1;
   const int k = blockIdx.y * ST + threadIdx.y + 1;
   const int t = threadIdx.y * ST + threadIdx.x;
-  double a0 = 0.0, a1 = 0.0, a2 = 0.0, a3 = 0.0, a4 = 0.0;
+  double a[5] = {0.0, 0.0, 0.0, 0.0, 0.0};
   if (j <= c.nx && k <= c.ny) {
     const int i = idx(c, j, k);
     const int P = c.pitch;
@@ -147,20 +151,25 @@ k_summary(Chunk c, const double* __restrict__ d0, const double* __restrict__ e0,
     vsqrd = vsqrd + 0.25 * (u0[i + P + 1] * u0[i + P + 1] + v0[i + P + 1] * v0[i + P + 1]);
     const double cell_vol = c.dx * c.dy;
     const double cell_mass = cell_vol * d0[i];
-    a0 = cell_vol;
-    a1 = cell_mass;
-    a2 = cell_mass * e0[i];
-    a3 = cell_mass * 0.5 * vsqrd;
-    a4 = cell_vol * eos_pressure(d0[i], e0[i]);
+    a[0] = cell_vol;
+    a[1] = cell_mass;
+    a[2] = cell_mass * e0[i];
+    a[3] = cell_mass * 0.5 * vsqrd;
+    a[4] = cell_vol * eos_pressure(d0[i], e0[i]);
   }
-  red[0][t] = a0; red[1][t] = a1; red[2][t] = a2; red[3][t] = a3; red[4][t] = a4;
+#pragma unroll
+  for (int q = 0; q < 5; ++q) {
+    double x = a[q];
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) x = x + __shfl_xor_sync(0xffffffffu, x, o);
+    if ((t & 31) == 0) red[q][t >> 5] = x;
+  }
   __syncthreads();
-  for (int s = ST * ST / 2; s > 0; s >>= 1) {
-    if (t < s)
-      for (int q = 0; q < 5; ++q) red[q][t] = red[q][t] + red[q][t + s];
-    __syncthreads();
+  if (t < 5) {
+    double x = red[t][0];
+    for (int w = 1; w < ST * ST / 32; ++w) x = x + red[t][w];
+    partials[((int64_t)blockIdx.y * gridDim.x + blockIdx.x) * 5 + t] = x;
   }
-  if (t < 5) partials[((int64_t)blockIdx.y * gridDim.x + blockIdx.x) * 5 + t] = red[t][0];
 }
 
 }  // namespace clover

@@ -12,6 +12,7 @@
 #include <algorithm>
 #include <cmath>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 #include <utility>
@@ -256,6 +257,10 @@ struct clover_ctx {
   bool use_graphs = true;
   bool fuse_x = true;  // fused x sweep where every chunk has both x walls (see fuse_x_ok)
   bool fuse_y = true;  // fused y sweep (see fuse_y_ok)
+  // the y-wall band blocks may ride on a fixup launch (y_walls_after_fix)
+  // only if every block of that launch is co-resident: the band blocks spin
+  // until the fixup blocks are done (clover_init checks the occupancy)
+  bool walls_fold_fits = false;
   cudaGraphExec_t gexec[4] = {nullptr, nullptr, nullptr, nullptr};  // [parity + 2 * multi-step]
   int64_t ws_bytes = 0;
   bool prof = false;
@@ -264,6 +269,7 @@ struct clover_ctx {
 #ifdef CLOVER_WITH_NCCL
   ncclComm_t comm = nullptr;
 #endif
+  int hist_first = 1;             // first step whose dt is in the history (after a restart: ckpt step + 1)
   bool use_ht = false;            // collectives through the caller's host transport
   clover_host_transport ht = {};
 };
@@ -734,7 +740,8 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
   // one chunk on one rank: the y-wall bands ride on the fixup launch before
   // the y sweep (kf_lagrangian when sweep 1 is y, kf_advec_x<1> when sweep 2
   // is y), when that sweep is enqueued and fused
-  const bool fold1 = ctx->chunks.size() == 1 && ctx->nranks == 1 && fuse_y_ok(ctx);
+  const bool fold1 = ctx->chunks.size() == 1 && ctx->nranks == 1 && fuse_y_ok(ctx) &&
+                     ctx->walls_fold_fits;
   const bool walls_in_lagr = CLOVER_YWALLS_FOLD && fold1 && !advect_x && nphase >= 4;
   const bool walls_in_x1 = CLOVER_YWALLS_FOLD && fold1 && advect_x && fuse_x_ok(ctx) && nphase >= 6;
   int cur_prof_id = P_VISC_DT;
@@ -1009,7 +1016,9 @@ int check_err(clover_ctx* ctx) {
   CK(cudaStreamSynchronize(ctx->work));
   StepScalars h;
   CK(cudaMemcpy(&h, ctx->scal, sizeof(h), cudaMemcpyDeviceToHost));
-  if (h.err) return fail(h.err, "small timestep: dt < dtmin");
+  if (h.err == CLOVER_ERR_SMALL_DT) return fail(h.err, "small timestep: dt < dtmin");
+  if (h.err == CLOVER_ERR_NEG_VOLUME) return fail(h.err, "negative volume (or NaN) in PdV");
+  if (h.err) return fail(h.err, "latched device error");
   return CLOVER_OK;
 }
 
@@ -1224,7 +1233,9 @@ const char* clover_error_string(int code) {
     case CLOVER_ERR_NCCL: return "NCCL error";
     case CLOVER_ERR_WORKSPACE: return "workspace too small or misaligned";
     case CLOVER_ERR_SMALL_DT: return "small timestep (dt < dtmin)";
+    case CLOVER_ERR_NEG_VOLUME: return "negative volume in PdV";
     case CLOVER_ERR_STATE: return "invalid state";
+    case CLOVER_ERR_NAN: return "NaN in field_summary";
   }
   return "unknown error";
 }
@@ -1366,6 +1377,21 @@ int clover_init(const clover_grid* grid, const clover_state* states, int32_t nst
     maxcols = std::max<int64_t>(maxcols, c.nx + 2 + 2 * HALO);
     ctx->chunks.push_back(cs);
   }
+  {
+    // co-residency of the folded y-wall launches (kf_lagrangian, kf_advec_x<1>
+    // with FIX_BLOCKS + 5 * nbx blocks): all blocks must fit at once
+    int nsm = 148, dev = 0, b1 = 0, b2 = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b1, kf_lagrangian, SB, 0);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b2, kf_advec_x<1>, SB, 0);
+    cudaGetLastError();
+    const int64_t resident = (int64_t)nsm * std::min(b1, b2);
+    ctx->walls_fold_fits = ctx->chunks.size() == 1 &&
+                           (int64_t)FIX_BLOCKS + 5 * ywalls_of(ctx->chunks[0], 1).nbx <= resident;
+    if (const char* e = std::getenv("CLOVER_WALLS_FOLD_LIMIT"))  // test hook: force the unfolded path
+      ctx->walls_fold_fits = ctx->walls_fold_fits && std::atoi(e) != 0;
+  }
   if (px * py > 1) {
     int64_t line = std::max(maxrows, maxcols);
     ctx->xbuf_elems = (int64_t)ctx->chunks.size() * 4 * 6 * HALO * line;
@@ -1492,7 +1518,7 @@ int clover_kernels_per_step(clover_ctx* ctx, int32_t* out) {
   // unless the visc fixup finalises dt (one chunk on one rank)
   const bool one = ctx->chunks.size() == 1 && ctx->nranks == 1;
   const int x = fuse_x_ok(ctx) ? 2 : 4;
-  const int y = fuse_y_ok(ctx) ? ((CLOVER_YWALLS_FOLD && one && fuse_x_ok(ctx)) ? 2 : 3) : 4;
+  const int y = fuse_y_ok(ctx) ? ((CLOVER_YWALLS_FOLD && one && fuse_x_ok(ctx) && ctx->walls_fold_fits) ? 2 : 3) : 4;
   const int fin = one ? 0 : 1;
   *out = (int32_t)(ctx->chunks.size() * (4 + x + y) + fin);
   return CLOVER_OK;
@@ -1504,15 +1530,22 @@ int clover_step(clover_ctx* ctx, int32_t nsteps) {
   if (nsteps == 0) return CLOVER_OK;
   int rc = join_in(ctx);
   if (rc) return rc;
+  // on an error after join_in, whatever was enqueued is still ordered before
+  // later work on the caller's stream (join_out's own error is ignored)
+  auto bail = [&](int code) {
+    join_out(ctx);
+    return code;
+  };
   for (int i = 0; i < nsteps; ++i) {
     const int parity = ctx->advect_x ? 0 : 1;
     if (ctx->use_graphs && CLOVER_GRAPH_STEPS > 1 && nsteps - i >= CLOVER_GRAPH_STEPS) {
       const int slot = parity + 2;
       if (!ctx->gexec[slot]) {
         rc = build_graph(ctx, parity, CLOVER_GRAPH_STEPS, slot);
-        if (rc) return rc;
+        if (rc) return bail(rc);
       }
-      CK(cudaGraphLaunch(ctx->gexec[slot], ctx->work));
+      if (cudaGraphLaunch(ctx->gexec[slot], ctx->work) != cudaSuccess)
+        return bail(fail(CLOVER_ERR_CUDA, "cudaGraphLaunch failed"));
       i += CLOVER_GRAPH_STEPS - 1;
       if (CLOVER_GRAPH_STEPS % 2) ctx->advect_x = !ctx->advect_x;
       continue;
@@ -1520,12 +1553,13 @@ int clover_step(clover_ctx* ctx, int32_t nsteps) {
     if (ctx->use_graphs) {
       if (!ctx->gexec[parity]) {
         rc = build_graph(ctx, parity, 1, parity);
-        if (rc) return rc;
+        if (rc) return bail(rc);
       }
-      CK(cudaGraphLaunch(ctx->gexec[parity], ctx->work));
+      if (cudaGraphLaunch(ctx->gexec[parity], ctx->work) != cudaSuccess)
+        return bail(fail(CLOVER_ERR_CUDA, "cudaGraphLaunch failed"));
     } else {
       rc = enqueue_step(ctx, ctx->advect_x, 7);
-      if (rc) return rc;
+      if (rc) return bail(rc);
     }
     ctx->advect_x = !ctx->advect_x;
   }
@@ -1661,6 +1695,8 @@ int clover_dt_history(clover_ctx* ctx, int32_t first, int32_t n, double* host_ou
   StepScalars h;
   CK(cudaMemcpy(&h, ctx->scal, sizeof(h), cudaMemcpyDeviceToHost));
   if (first + n - 1 > h.step || h.step - first >= DT_HIST) return fail(CLOVER_ERR_ARG, "steps outside the kept history");
+  if (n > 0 && first < ctx->hist_first)
+    return fail(CLOVER_ERR_ARG, "steps before the restart point are not in the history");
   std::vector<double> all(DT_HIST);
   CK(cudaMemcpy(all.data(), ctx->hist, DT_HIST * 8, cudaMemcpyDeviceToHost));
   for (int i = 0; i < n; ++i) host_out[i] = all[(first - 1 + i) % DT_HIST];
@@ -1743,6 +1779,9 @@ int clover_field_summary(clover_ctx* ctx, clover_summary* out) {
   }
   out->vol = acc[0]; out->mass = acc[1]; out->ie = acc[2]; out->ke = acc[3]; out->press = acc[4];
   int rc2 = join_out(ctx);
+  if (!rc && (std::isnan(acc[0]) || std::isnan(acc[1]) || std::isnan(acc[2]) || std::isnan(acc[3]) ||
+              std::isnan(acc[4])))
+    rc = fail(CLOVER_ERR_NAN, "field_summary: a total is NaN");
   return rc ? rc : rc2;
 }
 
@@ -1906,6 +1945,7 @@ int clover_restart(clover_ctx* ctx, const void* host, int64_t bytes) {
   CK(cudaStreamSynchronize(ctx->work));
   CK(cudaMemcpy(&h, ctx->scal, sizeof(h), cudaMemcpyDeviceToHost));
   h.step = hd.step; h.time = hd.time; h.dt = hd.dt; h.dtold = hd.dtold; h.err = 0;
+  ctx->hist_first = hd.step + 1;
   {
     double big = G_BIG;
     std::memcpy(&h.dt_slot, &big, 8);

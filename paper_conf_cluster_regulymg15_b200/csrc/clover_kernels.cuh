@@ -189,7 +189,7 @@ __device__ __forceinline__ void dt_finalize(StepScalars* __restrict__ s, double*
   double dt = fmin(fmin(dtc, (s->dtold * prm.dtrise)), prm.dtmax);
   s->dt = dt;
   if (dt < prm.dtmin) {
-    if (s->err == 0) s->err = -5;
+    if (s->err == 0) s->err = -5;  // CLOVER_ERR_SMALL_DT
   } else {
     s->dtold = dt;
   }
@@ -292,7 +292,9 @@ __device__ __forceinline__ void pdv_correct_bt(D& dv, double r, double e, double
   double left_flux = pdv_face_corr(lsum, dy, dt);
   double right_flux = pdv_face_corr(rsum, dy, dt);
   double total_flux = right_flux - left_flux + top_flux - bottom_flux;
-  double volume_change = dv.nz(vol, vol + total_flux);
+  const double new_vol = vol + total_flux;
+  double volume_change = dv.nz(vol, new_vol);
+  dv.vol_check(new_vol);  // CLOVER_ERR_NEG_VOLUME (kf_lagrangian latches it)
   double recip_volume = rvol;  // = RN(1.0/vol), precomputed
   double energy_change = (dv(ph, r) + dv(q, r)) * total_flux * recip_volume;
   e1v = e - energy_change;

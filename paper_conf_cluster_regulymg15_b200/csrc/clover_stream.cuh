@@ -716,7 +716,7 @@ ks_lagrangian(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restric
 __global__ void __launch_bounds__(SB)
 kf_lagrangian(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__ d1,
               double* __restrict__ e1, double* __restrict__ u1, double* __restrict__ v1,
-              double* __restrict__ fx, double* __restrict__ fy, const StepScalars* __restrict__ s,
+              double* __restrict__ fx, double* __restrict__ fy, StepScalars* __restrict__ s,
               FixSlot fix, YWalls yw) {
   pdl_trigger();
   pdl_wait();
@@ -724,7 +724,10 @@ kf_lagrangian(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restric
   __shared__ __align__(128) double ring[SB / 32][LSTG * LSLOT];
   __shared__ __align__(8) unsigned long long bars[SB / 32][LSTG];
   fix_loop(fix, c.lks, c.lnb, c.ny + 1, [&](int gw, int k0, int k1, int lane, int w) {
-    lagr_seg<DivIEEE>(c, &tm, d1, e1, u1, v1, fx, fy, s, gw, k0, k1, lane, ring[w], bars[w]);
+    // the IEEE redo's flag is the exact PdV volume test (DivIEEE::vol_check)
+    if (lagr_seg<DivIEEE>(c, &tm, d1, e1, u1, v1, fx, fy, s, gw, k0, k1, lane, ring[w], bars[w]) &&
+        lane == 0)
+      atomicCAS(&s->err, 0, -6);  // CLOVER_ERR_NEG_VOLUME
   });
 }
 // (a register-only Lagrangian variant was measured 3% slower; see git history)

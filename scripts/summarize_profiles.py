@@ -89,7 +89,9 @@ if os.path.exists(rep):
                   f"{g(r, 'sm__pipe_fp64_cycles_active.avg.pct_of_peak_sustained_active'):.1f} | "
                   f"{g(r, 'sm__warps_active.avg.pct_of_peak_sustained_active'):.1f} | "
                   f"{g(r, 'launch__registers_per_thread'):.0f} | {inst * 32 / cells:.0f} |")
-        kern.setdefault(n, []).append({"dram_bytes": (rd + wr) * scale, "time_ns": t})
+        kern.setdefault(n, []).append({"dram_bytes": (rd + wr) * scale, "time_ns": t, "inst": inst,
+                                       "issue": g(r, 'smsp__issue_active.avg.pct_of_peak_sustained_active'),
+                                       "fp64": g(r, 'sm__pipe_fp64_cycles_active.avg.pct_of_peak_sustained_active')})
     with open(os.path.join(P, f"{tag}_kernels.md"), "w") as fh:
         fh.write("\n".join(md) + "\n")
     out = {"mesh": [3840, 3840], "source": f"profiles/{tag}_kernels.md (ncu --set full)",
@@ -97,6 +99,14 @@ if os.path.exists(rep):
                            "launches": len(v)} for k, v in kern.items()}}
     with open(os.path.join(P, "ncu_traffic.json"), "w") as fh:
         json.dump(out, fh, indent=1)
+    avg = lambda v, k: sum(x[k] for x in v) / len(v)
+    ins = {"mesh": [3840, 3840], "source": f"profiles/{tag}_kernels.md (ncu --set full, smsp__inst_executed.sum)",
+           "kernels": {k: {"warp_inst_per_launch": avg(v, "inst"),
+                           "thread_inst_per_cell": avg(v, "inst") * 32 / cells,
+                           "issue_active_pct": avg(v, "issue"), "fp64_pipe_pct": avg(v, "fp64"),
+                           "launches": len(v)} for k, v in kern.items()}}
+    with open(os.path.join(P, "ncu_instr.json"), "w") as fh:
+        json.dump(ins, fh, indent=1)
     print("wrote kernels", len(kern))
 b = os.path.join(G, "bench.json")
 if os.path.exists(b):

@@ -82,6 +82,10 @@ def test_gpu_checkpoint_restart_bitwise():
         assert np.array_equal(a.read(f), b.read(f)), f
     assert a.clock() == b.clock()
     assert np.array_equal(a.dt_history(8, 9), b.dt_history(8, 9))
+    # steps before the restart point are not in b's history
+    from paper_conf_cluster_regulymg15_b200 import CloverError
+    with pytest.raises(CloverError):
+        b.dt_history(7, 2)
     # restart into a context that has already run a different history
     c = Clover(deck)
     c.step(3)

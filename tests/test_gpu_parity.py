@@ -10,7 +10,7 @@ import numpy as np
 import pytest
 
 from oracle import Oracle
-from workloads import (bm_deck, contact_deck, fuzz_deck, point_deck, quiescent_deck,
+from workloads import (bm_deck, colliding_slab_deck, contact_deck, fuzz_deck, point_deck, quiescent_deck,
                        random_state_fields, symmetric_deck)
 
 pytestmark = pytest.mark.gpu
@@ -278,6 +278,26 @@ def test_tiny_numerators_take_the_ieee_fixup_bitwise(torch_cuda, scale):
     assert g.debug_fix_count() > 0
 
 
+@pytest.mark.parametrize("axis", ["x", "y", "xy"])
+@pytest.mark.parametrize("pxy", [(1, 1), (2, 2), (1, 3)])
+def test_divergence_limit_decks_bitwise(torch_cuda, axis, pxy):
+    """calc_dt's divergence term (c.4 dtdivt) decides dt on steps 1-2 of the
+    colliding-slab decks (oracle pin test_p2c_*): the kernel's min-w path
+    must give the same dt history, fields and summary bit for bit, on one
+    chunk and across chunk boundaries (the collision column sits on the
+    x = 5 chunk edge of the 2x2 layout)."""
+    n = 72
+    deck = colliding_slab_deck(n, axis, 1.0, end_step=12)
+    g, o = make_gpu(deck, px=pxy[0], py=pxy[1]), Oracle(deck)
+    g.step(12)
+    dts = o.step(12)
+    factor = 0.175 if axis == "xy" else 0.35
+    assert abs(dts[0] / (factor * 10.0 / n) - 1.0) < 1e-15  # dtdivt binds (closed form)
+    assert np.array_equal(g.dt_history(1, 12), dts)
+    assert_fields_equal(g, o, ctx=f"slab {axis} {pxy}")
+    assert_summary_close(g.field_summary(), o.field_summary())
+
+
 def test_invariant_decks(torch_cuda):
     for deck in (quiescent_deck(64), contact_deck(64), symmetric_deck(64)):
         g, o = make_gpu(deck), Oracle(deck)
@@ -371,6 +391,53 @@ def test_small_dt_error_is_latched(torch_cuda):
     assert ei.value.code == -5
 
 
+def test_negative_volume_is_latched(torch_cuda):
+    """SURVEY 8(b) CLOVER_ERR_NEG_VOLUME: with the CFL safety factors raised
+    20x the step is far beyond stability and PdV produces negative volumes
+    by step 2 (the oracle's density goes negative there); the library
+    latches the error and returns it from the next synchronising call.  Step
+    1 is still bitwise the oracle's."""
+    from paper_conf_cluster_regulymg15_b200 import CloverError
+    deck = bm_deck(64)
+    deck.update(max_timestep=10.0, initial_timestep=2.0, dtc_safe=14.0, dtu_safe=10.0,
+                dtv_safe=10.0, dtdiv_safe=14.0)
+    g, o = make_gpu(deck), Oracle(deck)
+    g.step(1)
+    o.step(1)
+    assert_fields_equal(g, o, ctx="unstable step 1")
+    g.step(1)
+    with pytest.raises(CloverError) as ei:
+        g.sync()
+    assert ei.value.code == -6
+    # a NaN in the state: the summary reports it, and the next step latches it
+    g2 = make_gpu(bm_deck(64))
+    rho = g2.read("density0")
+    rho[20, 30] = np.nan
+    g2.write("density0", rho)
+    with pytest.raises(CloverError) as ei:
+        g2.field_summary()
+    assert ei.value.code == -8
+    g2.step(1)
+    with pytest.raises(CloverError) as ei:
+        g2.sync()
+    assert ei.value.code == -6
+
+
+def test_y_wall_fold_guard(torch_cuda, monkeypatch):
+    """the y-wall bands ride on a fixup launch only when all its
+    blocks are co-resident.  Forcing the separate band launch gives the same
+    bits (one launch more per step)."""
+    deck = fuzz_deck(6, nx=96, ny=80)
+    a = make_gpu(deck)
+    monkeypatch.setenv("CLOVER_WALLS_FOLD_LIMIT", "0")
+    b = make_gpu(deck)
+    assert b.kernels_per_step() == a.kernels_per_step() + 1
+    a.step(6)
+    b.step(6)
+    for f in STATE:
+        assert np.array_equal(a.read(f), b.read(f)), f
+
+
 def test_c2_960_87_steps(torch_cuda):
     """configs[1]: clover_bm_short shape, full run; also the QA constant."""
     deck = bm_deck(960, end_step=87)
@@ -385,15 +452,17 @@ def test_c2_960_87_steps(torch_cuda):
     print("C2 IEEE fixup warp segments:", g.debug_fix_count())
 
 
-@pytest.mark.parametrize("n", [3840])
-def test_full_size_first_steps(torch_cuda, n):
-    """configs[2] size in the bench's launch configuration: full-field
-    comparison over the first 2 steps (the oracle needs ~3 s per step)."""
+@pytest.mark.parametrize("n,steps", [(3840, 20), (7680, 2)])
+def test_full_size_first_steps(torch_cuda, n, steps):
+    """configs[2] (bm 3840^2) over its first 20 steps and configs[3]'s 7680^2
+    strong-scaling base over 2 steps, one chunk, graphs, in the bench's launch
+    configuration: every state field and the dt history bitwise (the oracle
+    needs ~1.8 s per step at 3840^2, ~8 s at 7680^2)."""
     deck = bm_deck(n, end_step=300)
     g, o = make_gpu(deck), Oracle(deck)
-    g.step(2)
-    dts = o.step(2)
-    assert np.array_equal(g.dt_history(1, 2), dts)
+    g.step(steps)
+    dts = o.step(steps)
+    assert np.array_equal(g.dt_history(1, steps), dts)
     assert_fields_equal(g, o, ctx=f"{n}")
     # the sequential oracle sum carries up to n*eps (3e-9) of its own
     # rounding at this size; compare with its compensated twin

@@ -19,7 +19,7 @@ import pytest
 
 import riemann
 from oracle import Oracle
-from workloads import (bm_deck, contact_deck, doubled_deck, fuzz_deck, point_deck, quiescent_deck,
+from workloads import (bm_deck, colliding_slab_deck, contact_deck, doubled_deck, fuzz_deck, point_deck, quiescent_deck,
                        random_state_fields, sod_slab_deck, symmetric_deck, transpose_deck)
 
 GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
@@ -87,6 +87,32 @@ def test_p2_dt_rise_clamp():
     assert dts[0] == 1e-3 * 1.5
     for a, b in zip(dts[:-1], dts[1:]):
         assert b <= a * 1.5
+
+
+# ---------------------------------------------------------------- P2c
+@pytest.mark.parametrize("axis,factor", [("x", 0.35), ("y", 0.35), ("xy", 0.175)])
+@pytest.mark.parametrize("n", [64, 72, 200])
+def test_p2c_divergence_limit_binds_colliding_slabs(axis, factor, n):
+    """c.4's divergence limit dtdivt = dtdiv_safe * (-1/div), div = net face
+    volume flow / (2*volume), pinned in closed form.
+    Colliding slabs at uniform pressure (q = 0 at step 1): the one column of
+    cells whose left nodes move +U and right nodes -U has net outflow
+    -4*U*dy per unit time, so div = -2U/dx and dtdivt = 0.7*dx/(2U) =
+    0.35*dx/U; in the converging quadrants (xy) the centre cell adds the same
+    from v: div = -4U/dx, dtdivt = 0.175*dx/U.  Every other limit is larger:
+    the face-speed limit dtu = 0.5*dx/U, the sound-speed CFL 0.7*dx/c with
+    c = sqrt(gamma*(gamma-1)*e) = sqrt(1.4) (U=1 > c/2), 1.5*dtinit = 0.06,
+    dtmax = 1.  A dropped factor 2, a missing v (or u) term or a wrong sign
+    of the divergence test changes the first dt by 2x or makes it negative."""
+    U = 1.0
+    o = Oracle(colliding_slab_deck(n, axis, U))
+    dt = o.step(1)[0]
+    dx = 10.0 / n
+    c = math.sqrt(1.4 * GM1 * 2.5)
+    expect = factor * dx / U
+    others = (0.5 * dx / U, 0.7 * dx / c, 1.5 * 0.04, 1.0)
+    assert expect < min(others) * 0.95  # the divergence term is the binding one
+    assert _rel(dt, expect) < 1e-15
 
 
 # ---------------------------------------------------------------- P3

@@ -112,6 +112,34 @@ def sod_slab_deck(nx: int = 256, ny: int = 4, end_step: int = 100, max_timestep=
     return d
 
 
+def colliding_slab_deck(n: int = 64, axis: str = "x", U: float = 1.0, end_step: int = 10):
+    """Colliding slabs (pins calc_dt's divergence term,
+    SURVEY 8(c) c.4): uniform rho=1, e=2.5 (so p is uniform and q = 0 at
+    step 1); along `axis`, a slab on [3,5] moves with +U and a slab on [5,7]
+    with -U across the whole other axis.  axis="xy": four quadrants of
+    [3,7]^2 converge on (5,5) (u = +-U and v = +-U).  dtinit 0.04 (x1.5 =
+    0.06), dtmax 1.0, so the first dt is min(dtdiv, dtu, dtc), with U > c/2
+    making the divergence limit the binding one."""
+    d = bm_deck(n, n, end_step)
+    d["max_timestep"] = 1.0
+    bg = _state(1.0, 2.5)
+    if axis == "x":
+        d["states"] = [bg, _state(1.0, 2.5, U, 0.0, xmin=3.0, xmax=5.0, ymin=0.0, ymax=10.0),
+                       _state(1.0, 2.5, -U, 0.0, xmin=5.0, xmax=7.0, ymin=0.0, ymax=10.0)]
+    elif axis == "y":
+        d["states"] = [bg, _state(1.0, 2.5, 0.0, U, xmin=0.0, xmax=10.0, ymin=3.0, ymax=5.0),
+                       _state(1.0, 2.5, 0.0, -U, xmin=0.0, xmax=10.0, ymin=5.0, ymax=7.0)]
+    elif axis == "xy":
+        d["states"] = [bg,
+                       _state(1.0, 2.5, U, U, xmin=3.0, xmax=5.0, ymin=3.0, ymax=5.0),
+                       _state(1.0, 2.5, -U, U, xmin=5.0, xmax=7.0, ymin=3.0, ymax=5.0),
+                       _state(1.0, 2.5, U, -U, xmin=3.0, xmax=5.0, ymin=5.0, ymax=7.0),
+                       _state(1.0, 2.5, -U, -U, xmin=5.0, xmax=7.0, ymin=5.0, ymax=7.0)]
+    else:
+        raise ValueError(axis)
+    return d
+
+
 def doubled_deck(nx_half: int = 64, ny: int = 64, end_step: int = 20, **kw):
     """bm mirrored about x=0: domain [-10,10]x[0,10] on
     (2*nx_half) x ny, state 2 on [-5,5]x[0,2]."""
