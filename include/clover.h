@@ -226,8 +226,12 @@ const char* clover_profile_name(int32_t i);
 
 /* Test: route every chunk boundary of a single-process multi-chunk context
  * through the remote-neighbour path (pack -> staging -> unpack, exactly the
- * code around the NCCL send/recv pair, which a device copy replaces), so the
- * multi-GPU message layout is exercised on one GPU. */
+ * code around the NCCL send/recv pair), so the multi-GPU message layout is
+ * exercised on one GPU.  enable = 1: a device copy replaces the NCCL pair;
+ * enable = 2: the messages travel through a one-rank NCCL communicator
+ * (ncclSend/ncclRecv to self inside one group, created here) and dt through a
+ * one-rank ncclAllReduce(MIN), captured in the step's CUDA graph like the
+ * multi-rank path; CLOVER_ERR_NCCL if the library was built without NCCL. */
 int clover_debug_set_virtual_remote(clover_ctx* ctx, int32_t enable);
 
 /* Debug: run only the first `nkernels` kernel phases of the next step
@@ -240,11 +244,13 @@ int clover_debug_partial_step(clover_ctx* ctx, int32_t nkernels);
 int clover_debug_read_buffer(clover_ctx* ctx, int32_t buffer_id, int32_t kind,
                              double* host, int64_t n);
 
-/* Debug: enable (default) or disable the fused x-sweep kernel (advec_cell x
- * + advec_mom x in one pass, used when every local chunk has reflective
- * walls on both x sides and the geometric face mirror).  Disabled, the
- * x sweep runs the separate cell and momentum kernels.  Both paths are
- * bitwise identical; tests compare them.  Test only. */
+/* Debug: the fused advection sweeps (advec_cell + advec_mom of one
+ * direction in one pass).  enable = 1 (default): fused x sweep where every
+ * local chunk has reflective walls on both x sides, fused y sweep everywhere
+ * (at y chunk boundaries from depth-4 input halos); 2: fused y sweep only
+ * where every chunk has both y walls (the separate kernels elsewhere); 0:
+ * separate cell and momentum kernels throughout.  Geometric face mirror
+ * only.  All settings are bitwise identical; tests compare them.  Test only. */
 int clover_debug_set_fusion(clover_ctx* ctx, int32_t enable);
 
 /* Debug: total number of warp segments the IEEE-division fixup launches

@@ -335,16 +335,22 @@ class Clover:
         buf = ctypes.create_string_buffer(blob, len(blob))
         _check(load().clover_restart(self._ctx, buf, len(blob)), "clover_restart")
 
-    def debug_set_virtual_remote(self, on: bool):
-        _check(load().clover_debug_set_virtual_remote(self._ctx, 1 if on else 0),
+    def debug_set_virtual_remote(self, on, nccl: bool = False):
+        """on: chunk boundaries through the remote (pack/staging/unpack) path;
+        nccl: the messages through a one-rank NCCL communicator (send/recv to
+        self) and dt through a one-rank NCCL all-reduce."""
+        _check(load().clover_debug_set_virtual_remote(self._ctx, (2 if nccl else 1) if on else 0),
                "clover_debug_set_virtual_remote")
 
     def debug_partial_step(self, nkernels: int):
         _check(load().clover_debug_partial_step(self._ctx, nkernels), "clover_debug_partial_step")
 
-    def debug_set_fusion(self, enable: bool):
-        """Fused x sweep on (default) or off (separate cell / momentum kernels)."""
-        _check(load().clover_debug_set_fusion(self._ctx, 1 if enable else 0), "clover_debug_set_fusion")
+    def debug_set_fusion(self, enable, walls_only: bool = False):
+        """Fused sweeps on (default), off (separate cell / momentum kernels),
+        or with walls_only the fused y sweep only where every chunk has both
+        y walls (round-1 behaviour: separate y kernels at y chunk boundaries)."""
+        v = (2 if walls_only else 1) if enable else 0
+        _check(load().clover_debug_set_fusion(self._ctx, v), "clover_debug_set_fusion")
 
     def debug_fix_count(self) -> int:
         """Warp segments recomputed so far by the IEEE-division fixup launches."""

@@ -135,10 +135,11 @@ Layout decompose(int NX, int NY, int px, int py) {
 }
 
 int64_t field_elems(int nx, int ny, int* pitch_out) {
-  // columns: j in [-HALO, nx+1+HALO] with j=0 at COL0; rows k in [-HALO, ny+1+HALO]
+  // columns: j in [-HALO, nx+1+HALO] with j=0 at COL0; rows k in
+  // [-HALO_ROWS, ny+1+HALO_ROWS]
   int pitch = (int)align_up(COL0 + nx + 2 + HALO, 32);
   if (pitch_out) *pitch_out = pitch;
-  int rows = ny + 2 + 2 * HALO;
+  int rows = ny + 2 + 2 * HALO_ROWS;
   return (int64_t)pitch * rows;
 }
 
@@ -257,6 +258,7 @@ struct clover_ctx {
   bool use_graphs = true;
   bool fuse_x = true;  // fused x sweep where every chunk has both x walls (see fuse_x_ok)
   bool fuse_y = true;  // fused y sweep (see fuse_y_ok)
+  bool fuse_y_chunks = true;  // ... also at y chunk boundaries (depth-4 row exchange)
   // the y-wall band blocks may ride on a fixup launch (y_walls_after_fix)
   // only if every block of that launch is co-resident: the band blocks spin
   // until the fixup blocks are done (clover_init checks the occupancy)
@@ -265,6 +267,7 @@ struct clover_ctx {
   int64_t ws_bytes = 0;
   bool prof = false;
   bool virtual_remote = false;  // test mode: every chunk boundary takes the NCCL packing path
+  bool virtual_nccl = false;    // ... and the messages travel through a 1-rank NCCL communicator
   std::vector<std::pair<int, cudaEvent_t>> prof_events;
 #ifdef CLOVER_WITH_NCCL
   ncclComm_t comm = nullptr;
@@ -335,14 +338,14 @@ int64_t compute_workspace(const clover_grid* g, int px, int py, int rank, int nr
     int ntx = (nx + ST - 1) / ST, nty = (ny + ST - 1) / ST;
     bytes += align_up((int64_t)ntx * nty * 5 * 8, kAlign);
     bytes += fix_bytes(nx, ny);
-    maxrows = std::max<int64_t>(maxrows, ny + 2 + 2 * HALO);
+    maxrows = std::max<int64_t>(maxrows, ny + 2 + 2 * HALO_ROWS);
     maxcols = std::max<int64_t>(maxcols, nx + 2 + 2 * HALO);
   }
   if (px * py > 1) {
     // staging for the remote-neighbour path: every local chunk x 4 sides x
-    // 6 fields x HALO lines (also used by the virtual-remote test mode)
+    // 6 fields x HALO_ROWS lines (also used by the virtual-remote test mode)
     int64_t line = std::max(maxrows, maxcols);
-    int64_t el = (int64_t)local_chunk_ids(px, py, rank, nranks).size() * 4 * 6 * HALO * line;
+    int64_t el = (int64_t)local_chunk_ids(px, py, rank, nranks).size() * 4 * 6 * HALO_ROWS * line;
     bytes += 2 * align_up(el * 8, kAlign);
   }
   return bytes;
@@ -405,32 +408,35 @@ struct StripQueue {
 
 // strips for side `side` (0 left, 1 right, 2 bottom, 3 top) of chunk cs:
 // send = owned points next to that side, recv = halo points of that side.
-void side_strips(const ChunkState& cs, int buf, int side, XferDesc& send, XferDesc& recv) {
+// x sides are HALO columns deep; y sides `ydepth` rows (HALO, or HALO_ROWS
+// for the inputs of a fused y sweep).
+void side_strips(const ChunkState& cs, int buf, int side, XferDesc& send, XferDesc& recv,
+                 int ydepth = HALO) {
   const Chunk& c = cs.c;
   const int kind = kBufKind[buf];
   const int ox = (kind == K_XVEL || kind == K_YVEL || kind == K_XFACE) ? 1 : 0;
   const int oy = (kind == K_XVEL || kind == K_YVEL || kind == K_YFACE) ? 1 : 0;
   send.base = recv.base = cs.buf[buf];
   send.pitch = recv.pitch = c.pitch;
-  // full extent of this kind including both halos: rows [-HALO, ny+oy+HALO],
-  // columns [-HALO, nx+ox+HALO] (x strips carry every row, y strips every
-  // column, so 4-chunk corners are refreshed by the second axis)
-  const int full_h = c.ny + oy + 1 + 2 * HALO, full_w = c.nx + ox + 1 + 2 * HALO;
+  // full extent of this kind including both halos: rows [-HALO_ROWS,
+  // ny+oy+HALO_ROWS], columns [-HALO, nx+ox+HALO] (x strips carry every row,
+  // y strips every column, so 4-chunk corners are refreshed by the second axis)
+  const int full_h = c.ny + oy + 1 + 2 * HALO_ROWS, full_w = c.nx + ox + 1 + 2 * HALO;
   if (side == 0) {          // left: send [1+ox, HALO+ox], recv [1-HALO, 0]
     send.j0 = 1 + ox; recv.j0 = 1 - HALO;
     send.w = recv.w = HALO;
-    send.k0 = recv.k0 = -HALO; send.h = recv.h = full_h;
+    send.k0 = recv.k0 = -HALO_ROWS; send.h = recv.h = full_h;
   } else if (side == 1) {   // right: send [nx+1-HALO, nx], recv [nx+ox+1, nx+ox+HALO]
     send.j0 = c.nx + 1 - HALO; recv.j0 = c.nx + ox + 1;
     send.w = recv.w = HALO;
-    send.k0 = recv.k0 = -HALO; send.h = recv.h = full_h;
-  } else if (side == 2) {   // bottom
-    send.k0 = 1 + oy; recv.k0 = 1 - HALO;
-    send.h = recv.h = HALO;
+    send.k0 = recv.k0 = -HALO_ROWS; send.h = recv.h = full_h;
+  } else if (side == 2) {   // bottom: send [1+oy, d+oy], recv [1-d, 0]
+    send.k0 = 1 + oy; recv.k0 = 1 - ydepth;
+    send.h = recv.h = ydepth;
     send.j0 = recv.j0 = -HALO; send.w = recv.w = full_w;
-  } else {                  // top
-    send.k0 = c.ny + 1 - HALO; recv.k0 = c.ny + oy + 1;
-    send.h = recv.h = HALO;
+  } else {                  // top: send [ny+1-d, ny], recv [ny+oy+1, ny+oy+d]
+    send.k0 = c.ny + 1 - ydepth; recv.k0 = c.ny + oy + 1;
+    send.h = recv.h = ydepth;
     send.j0 = recv.j0 = -HALO; send.w = recv.w = full_w;
   }
 }
@@ -473,7 +479,7 @@ int StripQueue::flush() {
   return CLOVER_OK;
 }
 
-int exchange_axis(clover_ctx* ctx, const std::vector<int>& bufs, int axis) {
+int exchange_axis(clover_ctx* ctx, const std::vector<int>& bufs, int axis, int ydepth = HALO) {
   const int s_lo = axis == 0 ? 0 : 2, s_hi = axis == 0 ? 1 : 3;
   // stage 1 (one batch): local pairs' halo strips and the packing of the
   // remote sides (owned points in, halo points / staging out: disjoint)
@@ -486,8 +492,8 @@ int exchange_axis(clover_ctx* ctx, const std::vector<int>& bufs, int axis) {
     if (!other) continue;
     for (int b : bufs) {
       XferDesc sA, rA, sB, rB;
-      side_strips(cs, b, s_hi, sA, rA);
-      side_strips(*other, b, s_lo, sB, rB);
+      side_strips(cs, b, s_hi, sA, rA, ydepth);
+      side_strips(*other, b, s_lo, sB, rB, ydepth);
       int rc = q.add(rB, sA);  // my high side -> neighbour's low halo
       if (rc) return rc;
       rc = q.add(rA, sB);      // neighbour's low side -> my high halo
@@ -510,14 +516,14 @@ int exchange_axis(clover_ctx* ctx, const std::vector<int>& bufs, int axis) {
         int64_t n = 0;
         for (int b : bufs) {
           XferDesc s, r;
-          side_strips(cs, b, side, s, r);
+          side_strips(cs, b, side, s, r, ydepth);
           n += (int64_t)s.w * s.h;
         }
         if (off + n > ctx->xbuf_elems) return fail(CLOVER_ERR_STATE, "halo staging buffer too small");
         n = 0;
         for (int b : bufs) {
           XferDesc s, r;
-          side_strips(cs, b, side, s, r);
+          side_strips(cs, b, side, s, r, ydepth);
           XferDesc dst{ctx->xbuf_send + off + n, s.w, 0, 0, s.w, s.h};
           int rc = q.add(dst, s);
           if (rc) return rc;
@@ -528,7 +534,26 @@ int exchange_axis(clover_ctx* ctx, const std::vector<int>& bufs, int axis) {
       }
     int rc = q.flush();  // the staging buffer is complete before it is sent
     if (rc) return rc;
-    if (ctx->virtual_remote) {
+    if (ctx->virtual_remote && ctx->virtual_nccl) {
+#ifdef CLOVER_WITH_NCCL
+      // one rank talks to itself: the i-th send to peer 0 matches the i-th
+      // receive from peer 0, so each message's send is paired with the
+      // receive slot of its partner (the neighbour's message on the facing
+      // side), exactly as the two ranks' lists pair up in a real exchange
+      NK(ncclGroupStart());
+      for (auto& m : msgs) {
+        const Msg* partner = nullptr;
+        for (auto& pm : msgs)
+          if (pm.cs->id == m.nb && pm.side == (m.side ^ 1)) partner = &pm;
+        if (!partner || partner->n != m.n) return fail(CLOVER_ERR_STATE, "virtual remote: unmatched message");
+        NK(ncclSend(ctx->xbuf_send + m.off, (size_t)m.n, ncclFloat64, 0, ctx->comm, ctx->work));
+        NK(ncclRecv(ctx->xbuf_recv + partner->off, (size_t)m.n, ncclFloat64, 0, ctx->comm, ctx->work));
+      }
+      NK(ncclGroupEnd());
+#else
+      return fail(CLOVER_ERR_NCCL, "libclover built without NCCL");
+#endif
+    } else if (ctx->virtual_remote) {
       for (auto& m : msgs) {
         const Msg* partner = nullptr;
         for (auto& pm : msgs)
@@ -575,7 +600,7 @@ int exchange_axis(clover_ctx* ctx, const std::vector<int>& bufs, int axis) {
       int64_t n = 0;
       for (int b : bufs) {
         XferDesc s, r;
-        side_strips(*m.cs, b, m.side, s, r);
+        side_strips(*m.cs, b, m.side, s, r, ydepth);
         XferDesc src{ctx->xbuf_recv + m.off + n, r.w, 0, 0, r.w, r.h};
         rc = q.add(r, src);
         if (rc) return rc;
@@ -588,11 +613,11 @@ int exchange_axis(clover_ctx* ctx, const std::vector<int>& bufs, int axis) {
 
 bool needs_exchange(const clover_ctx* ctx) { return ctx->L.px * ctx->L.py > 1; }
 
-int exchange(clover_ctx* ctx, const std::vector<int>& bufs) {
+int exchange(clover_ctx* ctx, const std::vector<int>& bufs, int ydepth = HALO) {
   if (!needs_exchange(ctx)) return CLOVER_OK;
   int rc = exchange_axis(ctx, bufs, 0);
   if (rc) return rc;
-  return exchange_axis(ctx, bufs, 1);
+  return exchange_axis(ctx, bufs, 1, ydepth);
 }
 
 // ---------------------------------------------------------------- schedule
@@ -689,17 +714,15 @@ bool fuse_x_ok(const clover_ctx* ctx) {
   return true;
 }
 
-// The fused y sweep needs reflective walls at both y ends of every chunk
-// (its reach along y is 4 rows: a chunk boundary would need depth-4 halos)
-// and the geometric face mirror.
-// The fused y sweep reads the post-sweep density and y-face mass flux of
-// the halo rows from memory, the mirrors written by the wall band kernel:
-// every chunk needs both y walls.  (Exchanging the band values across y
-// chunk boundaries instead was tried and is not bitwise yet: 1x4 chunks of
-// bm 96x80 differ at the first row above the high-pressure block, the
-// EDGE segment below a chunk boundary; kept off.)
+// The fused y sweep (reach 4 rows along y) runs at y walls (the mirrored
+// halo rows come from the band kernel) and at y chunk boundaries (its inputs
+// exchanged HALO_ROWS deep, the neighbour's first rows recomputed: SURVEY
+// 8(e) H1/H2); it needs the geometric face mirror.  fuse_y_chunks = false
+// keeps the separate cell / momentum kernels at y chunk boundaries (A/B and
+// tests).
 bool fuse_y_ok(const clover_ctx* ctx) {
   if (!ctx->fuse_y || ctx->g.face_mirror == CLOVER_MIRROR_CELLCENTRE) return false;
+  if (ctx->fuse_y_chunks) return true;
   for (const auto& cs : ctx->chunks)
     if (!cs.c.wb || !cs.c.wt) return false;
   return true;
@@ -759,8 +782,12 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
                   cs.fix, ctx->hist, fold_fin);
       FIX_LAUNCH_CHECK();
     }
-    int rc = exchange(ctx, {B_Q});
-    if (rc) return rc;
+    // q on ring 1: visc_dt computes rows 0 / ny+1 at y chunk boundaries
+    // itself (visc_ring_rows); only x chunk boundaries exchange q
+    if (needs_exchange(ctx)) {
+      int rc = exchange_axis(ctx, {B_Q}, 0);
+      if (rc) return rc;
+    }
     if (ctx->prof) prof_mark(ctx, -1);
   }
   if (nphase >= 2) {
@@ -775,7 +802,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
       CK(cudaStreamSynchronize(st));
     }
 #ifdef CLOVER_WITH_NCCL
-    else if (ctx->nranks > 1)
+    else if (ctx->nranks > 1 || ctx->virtual_nccl)
       NK(ncclAllReduce(&ctx->scal->dt_slot, &ctx->scal->dt_slot, 1, ncclUint64, ncclMin, ctx->comm, st));
 #endif
     if (ctx->prof) prof_mark(ctx, -1);
@@ -798,7 +825,8 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
           ctx->scal, cs.fix, yw);
       FIX_LAUNCH_CHECK();
     }
-    int rc = exchange(ctx, {B_D1, B_E1, B_U1, B_V1, B_FX, B_FY});
+    // a fused y sweep (either sweep) reads these HALO_ROWS deep in y
+    int rc = exchange(ctx, {B_D1, B_E1, B_U1, B_V1, B_FX, B_FY}, fuse_y_ok(ctx) ? HALO_ROWS : HALO);
     if (rc) return rc;
     if (ctx->prof) prof_mark(ctx, -1);
   }
@@ -836,7 +864,9 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
             FIX_LAUNCH_CHECK();
           }
         }
-        int rc = exchange(ctx, {rout, eout, uout, vout});
+        // sweep 1 feeds a fused y sweep 2: HALO_ROWS deep in y
+        int rc = exchange(ctx, {rout, eout, uout, vout},
+                          (sweep == 1 && fuse_y_ok(ctx)) ? HALO_ROWS : HALO);
         if (rc) return rc;
         if (ctx->prof) prof_mark(ctx, -1);
       }
@@ -851,6 +881,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
         const bool folded = sweep == 1 ? walls_in_lagr : walls_in_x1;
         for (auto& cs : ctx->chunks) {
           if (folded) break;
+          if (!cs.c.wb && !cs.c.wt) continue;  // no y wall band in this chunk
           const Chunk c = with_rev(cs.c, sweep == 1 ? CLOVER_SERP : 0);
           const YWalls yw = ywalls_of(cs, sweep);
           const dim3 gw(yw.nbx, 5);
@@ -1353,7 +1384,7 @@ int clover_init(const clover_grid* grid, const clover_state* states, int32_t nst
     }
     {
       const double* base = cs.buf[B_D0] - (int64_t)ROW0 * c.pitch - COL0;
-      const int rows = c.ny + 2 + 2 * HALO;
+      const int rows = c.ny + 2 + 2 * HALO_ROWS;
       int rc = encode_rows_map(&cs.tm_lag, base, c.pitch, rows, align_up(fe * 8, kAlign), LNF, LRW);
       const int64_t fs = align_up(fe * 8, kAlign);
       if (!rc) rc = encode_rows_map(&cs.tm_visc, base, c.pitch, rows, fs, VNF, VRW);
@@ -1373,7 +1404,7 @@ int clover_init(const clover_grid* grid, const clover_state* states, int32_t nst
     cs.fix.hdr = (unsigned*)p;
     cs.fix.e = (uint2*)(p + kAlign);
     p += fix_bytes(c.nx, c.ny);
-    maxrows = std::max<int64_t>(maxrows, c.ny + 2 + 2 * HALO);
+    maxrows = std::max<int64_t>(maxrows, c.ny + 2 + 2 * HALO_ROWS);
     maxcols = std::max<int64_t>(maxcols, c.nx + 2 + 2 * HALO);
     ctx->chunks.push_back(cs);
   }
@@ -1394,7 +1425,7 @@ int clover_init(const clover_grid* grid, const clover_state* states, int32_t nst
   }
   if (px * py > 1) {
     int64_t line = std::max(maxrows, maxcols);
-    ctx->xbuf_elems = (int64_t)ctx->chunks.size() * 4 * 6 * HALO * line;
+    ctx->xbuf_elems = (int64_t)ctx->chunks.size() * 4 * 6 * HALO_ROWS * line;
     ctx->xbuf_send = (double*)p;
     p += align_up(ctx->xbuf_elems * 8, kAlign);
     ctx->xbuf_recv = (double*)p;
@@ -1475,7 +1506,23 @@ int clover_debug_set_virtual_remote(clover_ctx* ctx, int32_t enable) {
   if (!ctx) return fail(CLOVER_ERR_ARG, "ctx is NULL");
   if (ctx->nranks > 1) return fail(CLOVER_ERR_STATE, "virtual remote is a single-process test mode");
   if (enable && ctx->L.px * ctx->L.py < 2) return fail(CLOVER_ERR_STATE, "virtual remote needs px*py > 1");
+  if (enable < 0 || enable > 2) return fail(CLOVER_ERR_ARG, "enable must be 0, 1 or 2");
+  if (enable == 2) {
+#ifdef CLOVER_WITH_NCCL
+    if (!ctx->comm) {
+      // a one-rank communicator on this GPU: every halo message becomes an
+      // ncclSend/ncclRecv pair to self, the dt MIN a 1-rank ncclAllReduce
+      CK(cudaStreamSynchronize(ctx->work));
+      ncclUniqueId id;
+      NK(ncclGetUniqueId(&id));
+      NK(ncclCommInitRank(&ctx->comm, 1, id, 0));
+    }
+#else
+    return fail(CLOVER_ERR_NCCL, "libclover built without NCCL");
+#endif
+  }
   ctx->virtual_remote = enable != 0;
+  ctx->virtual_nccl = enable == 2;
   for (int i = 0; i < 4; ++i)
     if (ctx->gexec[i]) {
       cudaGraphExecDestroy(ctx->gexec[i]);
@@ -1486,8 +1533,10 @@ int clover_debug_set_virtual_remote(clover_ctx* ctx, int32_t enable) {
 
 int clover_debug_set_fusion(clover_ctx* ctx, int32_t enable) {
   if (!ctx) return fail(CLOVER_ERR_ARG, "ctx is NULL");
+  if (enable < 0 || enable > 2) return fail(CLOVER_ERR_ARG, "enable must be 0, 1 or 2");
   ctx->fuse_x = enable != 0;
   ctx->fuse_y = enable != 0;
+  ctx->fuse_y_chunks = enable == 1;
   for (int i = 0; i < 4; ++i)
     if (ctx->gexec[i]) {
       cudaGraphExecDestroy(ctx->gexec[i]);
@@ -1516,11 +1565,17 @@ int clover_kernels_per_step(clover_ctx* ctx, int32_t* out) {
   // bands, kernel + fixup; else 4; the bands ride on the previous fixup
   // launch at one chunk on one rank, enqueue_step); plus k_dt_finalize once
   // unless the visc fixup finalises dt (one chunk on one rank)
+  // (chunks without a y wall launch no band kernel; the halo strip copies
+  // between phases, k_copy_strips, are not counted)
   const bool one = ctx->chunks.size() == 1 && ctx->nranks == 1;
   const int x = fuse_x_ok(ctx) ? 2 : 4;
-  const int y = fuse_y_ok(ctx) ? ((CLOVER_YWALLS_FOLD && one && fuse_x_ok(ctx) && ctx->walls_fold_fits) ? 2 : 3) : 4;
-  const int fin = one ? 0 : 1;
-  *out = (int32_t)(ctx->chunks.size() * (4 + x + y) + fin);
+  const bool folded = CLOVER_YWALLS_FOLD && one && fuse_x_ok(ctx) && ctx->walls_fold_fits;
+  int n = one ? 0 : 1;
+  for (const auto& cs : ctx->chunks) {
+    const int y = fuse_y_ok(ctx) ? (2 + ((!folded && (cs.c.wb || cs.c.wt)) ? 1 : 0)) : 4;
+    n += 4 + x + y;
+  }
+  *out = (int32_t)n;
   return CLOVER_OK;
 }
 

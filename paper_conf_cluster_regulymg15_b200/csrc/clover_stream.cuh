@@ -199,6 +199,7 @@ template <int SWEEP>
 __device__ __forceinline__ void y_walls_block(const Chunk& c, const YWalls& y, int bx, int b) {
   const int k = b < 3 ? 1 + b : c.ny - 4 + b;
   if (b < 3 && k > c.ny) return;
+  if (b < 3 ? !c.wb : !c.wt) return;  // a chunk boundary: the y sweep recomputes these rows
   const int jlo = c.wl ? 1 : 0;
   Chunk cw = c;
   cw.nx = c.wr ? c.nx : c.nx + 1;
@@ -328,13 +329,17 @@ __device__ __forceinline__ bool visc_body(const Chunk& c, const CUtensorMap* __r
   __syncwarp();
   if (lane == 0 && r_first + VSTG <= r_last) issue(r_first + VSTG);  // row k0-1 is consumed
   DtAcc acc;
-  if ((!EDGE || j <= c.nx) && k1 > k0) acc.bottom(row(k0)[VF_V * VRW], row(k0)[VF_V * VRW + 1], c);
+  // rows 0 / ny+1 at a y chunk boundary are ring rows (q only, no dt): the
+  // Lagrangian phase reads q on ring 1, so no q exchange is needed in y
+  if ((!EDGE || j <= c.nx) && k1 > k0 && (!EDGE || k0 >= 1))
+    acc.bottom(row(k0)[VF_V * VRW], row(k0)[VF_V * VRW + 1], c);
   const bool left = EDGE && j == 1;  // column 1: no left neighbour takes this face
   int i = idx(c, j, k0);
   for (int k = k0; k < k1; ++k, i += c.pitch) {
     wait_row(k + 1);
     const double* rc = row(k);
     const double* rn = row(k + 1);
+    const bool owned_row = !EDGE || (k >= 1 && k <= c.ny);
     if (!EDGE || j <= c.nx) {
       ViscIn I;
       I.rho = rc[VF_R * VRW]; I.e = rc[VF_E * VRW];
@@ -348,7 +353,10 @@ __device__ __forceinline__ bool visc_body(const Chunk& c, const CUtensorMap* __r
       I.v01 = rn[VF_V * VRW]; I.v11 = rn[VF_V * VRW + 1];
       double qv, cc2, c2;
       visc_cell(dv, I, c, qv, cc2, c2);
-      acc.add(I, c, qv, cc2, c2, left);
+      if (owned_row) {
+        if (EDGE && k == 1 && k0 == 0) acc.bottom(I.v00, I.v10, c);  // after ring row 0
+        acc.add(I, c, qv, cc2, c2, left);
+      }
       store_at(c, q, K_CELL, j, k, i, EDGE && (ncol || near_wall_row(c, k)), qv);
       pcm = pc;
       pc = I.pt;
@@ -385,6 +393,13 @@ __device__ __forceinline__ bool visc_seg(const Chunk& c, const CUtensorMap* __re
   return visc_body<D, true>(c, tm, q, prm, gw, k0, k1, lane, ring, bars, dtw);
 }
 
+// Rows [k0, k1) of a visc segment extended by the ring row 0 (ny+1) when the
+// segment starts at row 1 (ends at row ny) next to a y chunk boundary.
+__device__ __forceinline__ void visc_ring_rows(const Chunk& c, int& k0, int& k1) {
+  if (k0 == 1 && !c.wb) k0 = 0;
+  if (k1 == c.ny + 1 && !c.wt) k1 = c.ny + 2;
+}
+
 __global__ void LB_VISC
 ks_visc_dt(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__ q,
            StepScalars* __restrict__ s, DtParams prm, FixSlot fix) {
@@ -397,7 +412,8 @@ ks_visc_dt(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__
   double dtw = G_BIG;
   int k0, len;
   seg_rows_of(seg_y(c), c.vks, c.vnb, k0, len);
-  const int k1 = min(k0 + len, c.ny + 1);
+  int k1 = min(k0 + len, c.ny + 1);
+  visc_ring_rows(c, k0, k1);
   if (gw * 32 < c.nx) {
     if (visc_seg<DivFast>(c, &tm, q, prm, gw, k0, k1, lane, ring[warp], bars[warp], dtw)) {
       fix_push(fix, lane, gw, (unsigned)seg_y(c));
@@ -428,6 +444,7 @@ kf_visc_dt(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__
       fix, c.vks, c.vnb, c.ny + 1,
       [&](int gw, int k0, int k1, int lane, int w) {
         double dtw;
+        visc_ring_rows(c, k0, k1);  // rows 1 / ny redo their ring row too
         visc_seg<DivIEEE>(c, &tm, q, prm, gw, k0, k1, lane, ring[w], bars[w], dtw);
         if (lane == 0) atomicMin(&s->dt_slot, (unsigned long long)__double_as_longlong(dtw));
       },
@@ -1585,8 +1602,14 @@ __device__ __forceinline__ bool advec_y_body(const Chunk& c, const CUtensorMap* 
       return vol;
     }
   };
-  auto face_computed = [&](int f) { return !EDGE || (f >= 1 && f <= ny + 1); };
-  auto cell_computed = [&](int r) { return !EDGE || (r >= 1 && r <= ny); };
+  // at a y wall the faces / cells beyond it are the mirrors ks_cell_y_walls
+  // wrote; at a y chunk boundary they are recomputed from the depth-4 input
+  // halos (the neighbour computes the same rows from the same inputs: same
+  // bits), so no exchange is needed between advec_cell and advec_mom
+  auto face_computed = [&](int f) {
+    return !EDGE || ((!c.wb || f >= 1) && (!c.wt || f <= ny + 1));
+  };
+  auto cell_computed = [&](int r) { return !EDGE || ((!c.wb || r >= 1) && (!c.wt || r <= ny)); };
   // flux of face f (between cells f-1 and f); pvlo = pre_vol(f-1), pvhi = pre_vol(f)
   auto face_flux = [&](int f, double pvlo, double pvhi, double& m, double& ef) {
     const double F = row(f)[L::FY];

@@ -1,7 +1,12 @@
 """Cost of the halo-exchange machinery on one GPU: the same bm mesh as one
-chunk and as px x py local chunks (device-to-device exchange phases), and
+chunk and as px x py local chunks (device-to-device exchange phases), with
+the fused y sweep across y chunk boundaries (default) or only at walls
+(round-1 schedule: separate y kernels + an extra exchange phase), and
 through the virtual-remote packing path (pack -> staging -> unpack, the
-multi-GPU message layout).  usage: chunk_overhead.py NX NY PX PY [STEPS]"""
+multi-GPU message layout), by device copy and through a one-rank NCCL
+communicator.  Prints one JSON line.
+usage: chunk_overhead.py NX NY PX PY [STEPS]"""
+import json
 import os
 import sys
 
@@ -9,7 +14,6 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import torch  # noqa: E402
 
 from paper_conf_cluster_regulymg15_b200 import Clover  # noqa: E402
-from paper_conf_cluster_regulymg15_b200.clover import load  # noqa: E402
 from workloads import bm_deck  # noqa: E402
 
 nx, ny, px, py = (int(a) for a in sys.argv[1:5])
@@ -18,10 +22,12 @@ torch.cuda.set_device(0)
 deck = bm_deck(nx, ny, end_step=steps, ymax=10.0 * ny / nx)
 
 
-def run(p, q, vr=False):
+def run(p, q, vr=0, walls_only=False):
     sim = Clover(deck, px=p, py=q)
+    if walls_only:
+        sim.debug_set_fusion(True, walls_only=True)
     if vr:
-        load().clover_debug_set_virtual_remote(sim._ctx, 1)
+        sim.debug_set_virtual_remote(True, nccl=vr == 2)
     sim.step(3)
     sim.sync()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -31,12 +37,15 @@ def run(p, q, vr=False):
     e1.record(sim.stream)
     torch.cuda.synchronize()
     ms = e0.elapsed_time(e1) / steps
+    kps = sim.kernels_per_step()
     sim.close()
-    return ms
+    return ms, kps
 
 
-one = run(1, 1)
-many = run(px, py)
-vr = run(px, py, True)
-print(f"{nx}x{ny}: 1 chunk {one:.4f} ms/step; {px}x{py} local chunks {many:.4f} ms/step "
-      f"(+{many - one:.4f}); virtual remote {vr:.4f} (+{vr - one:.4f})")
+one, k1 = run(1, 1)
+res = {"mesh": [nx, ny], "chunks": [px, py], "steps": steps, "one_chunk_ms": one, "one_chunk_kernels": k1}
+for name, kw in (("local_fused", {}), ("local_walls_only", dict(walls_only=True)),
+                 ("virtual_remote", dict(vr=1)), ("virtual_nccl", dict(vr=2))):
+    ms, k = run(px, py, **kw)
+    res[name] = {"ms": ms, "overhead": ms / one - 1.0, "kernels": k}
+print(json.dumps(res), flush=True)

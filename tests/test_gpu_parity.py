@@ -340,6 +340,51 @@ def test_virtual_remote_exchange_bitwise(torch_cuda, pxy):
     assert np.array_equal(many.dt_history(1, 10), one.dt_history(1, 10))
 
 
+@pytest.mark.parametrize("pxy", [(2, 2), (1, 3), (2, 4)])
+def test_virtual_remote_through_nccl_bitwise(torch_cuda, pxy):
+    """the multi-GPU exchange code with NCCL itself executing.
+    A one-rank NCCL communicator carries every chunk-boundary message as an
+    ncclSend/ncclRecv pair to self (paired exactly as two ranks' lists pair
+    up) and dt through a one-rank ncclAllReduce(MIN), all captured in the
+    step's CUDA graph: same bits as one chunk, dt history included."""
+    deck = fuzz_deck(9, nx=96, ny=80)
+    one = make_gpu(deck)
+    many = make_gpu(deck, px=pxy[0], py=pxy[1])
+    many.debug_set_virtual_remote(True, nccl=True)
+    one.step(10)
+    many.step(10)
+    for f in STATE:
+        assert np.array_equal(many.read(f), one.read(f)), f
+    assert np.array_equal(many.dt_history(1, 10), one.dt_history(1, 10))
+    assert many.field_summary() == one.field_summary()
+
+
+@pytest.mark.parametrize("seed,pxy", [(8, (1, 2)), (9, (1, 4)), (10, (2, 3)), (11, (1, 5))])
+def test_fused_y_sweep_across_chunk_boundaries(torch_cuda, seed, pxy):
+    """at y chunk boundaries the
+    fused y sweep recomputes the neighbour's first post-sweep rows from
+    depth-4 input halos.  Same bits as the separate cell / momentum kernels
+    with their extra exchange (fusion walls_only) and as one chunk, on
+    fuzz decks (flow across the boundaries) for 12 steps (both sweep
+    orders), local and virtual-remote exchange."""
+    deck = fuzz_deck(seed, nx=72, ny=96)
+    deck["max_timestep"] = 1.0
+    one = make_gpu(deck)
+    fused = make_gpu(deck, px=pxy[0], py=pxy[1])
+    split = make_gpu(deck, px=pxy[0], py=pxy[1])
+    split.debug_set_fusion(True, walls_only=True)
+    remote = make_gpu(deck, px=pxy[0], py=pxy[1])
+    remote.debug_set_virtual_remote(True)
+    assert fused.kernels_per_step() < split.kernels_per_step()
+    for g in (one, fused, split, remote):
+        g.step(12)
+    for f in STATE:
+        a = one.read(f)
+        for g in (fused, split, remote):
+            assert np.array_equal(g.read(f), a), f
+    assert np.array_equal(fused.dt_history(1, 12), one.dt_history(1, 12))
+
+
 @pytest.mark.parametrize("seed,pxy", [(8, (2, 3)), (9, (3, 2)), (9, (2, 4)), (12, (4, 4)),
                                       (13, (3, 3))])
 def test_local_chunks_fuzz(torch_cuda, seed, pxy):
@@ -468,14 +513,15 @@ def test_full_size_first_steps(torch_cuda, n, steps):
     assert_summary_close(g.field_summary(), o.field_summary(compensated=True))
 
 
-@pytest.mark.parametrize("pxy,expected", [((1, 1), 8), ((3, 1), 34), ((1, 3), 31)])
+@pytest.mark.parametrize("pxy,expected", [((1, 1), 8), ((3, 1), 34), ((1, 3), 27)])
 def test_kernels_per_step(torch_cuda, pxy, expected):
     """Launches per step (bench.py's gpu_launches): one chunk runs visc_dt,
     Lagrangian and both fused sweeps with a fixup each, the y-wall bands
     riding on the fixup before the y sweep (8); several chunks launch the
-    bands separately (+1 per chunk) and finalise dt in k_dt_finalize (+1);
-    x (y) chunk boundaries use the separate x (y) kernels, 4 launches per
-    chunk: 3x1 = 3 * (4 + 4 + 3) + 1, 1x3 = 3 * (4 + 2 + 4) + 1."""
+    bands separately (+1 per chunk with a y wall) and finalise dt in
+    k_dt_finalize (+1); x chunk boundaries use the separate x kernels, 4
+    launches per chunk: 3x1 = 3 * (4 + 4 + 3) + 1; y chunk boundaries keep
+    the fused y sweep: 1x3 = (4 + 2 + 3) + (4 + 2 + 2) + (4 + 2 + 3) + 1."""
     px, py = pxy
     g = make_gpu(fuzz_deck(11), px=px, py=py)
     assert g.kernels_per_step() == expected
