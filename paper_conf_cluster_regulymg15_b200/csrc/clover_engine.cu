@@ -952,7 +952,10 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
           }
         }
       }
-      int rc = exchange(ctx, {rout, eout, mbuf});
+      // x sweep 1 feeding a fused y sweep 2: the post-sweep density and
+      // energy HALO_ROWS deep in y
+      const int yd = (sweep == 1 && xdir && fuse_y_ok(ctx)) ? HALO_ROWS : HALO;
+      int rc = exchange(ctx, {rout, eout, mbuf}, yd);
       if (rc) return rc;
       if (ctx->prof) prof_mark(ctx, -1);
     }
@@ -988,7 +991,8 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
           }
         }
       }
-      int rc = exchange(ctx, {uout, vout});
+      const int yd = (sweep == 1 && xdir && fuse_y_ok(ctx)) ? HALO_ROWS : HALO;
+      int rc = exchange(ctx, {uout, vout}, yd);
       if (rc) return rc;
       if (ctx->prof) prof_mark(ctx, -1);
     }
