@@ -50,11 +50,19 @@ class OracleState(ctypes.Structure):
                 ("radius", ctypes.c_double)]
 
 
+CLI_PATH = os.path.join(_HERE, "clover_oracle")  # c.15 command-line driver
+
+
 def build(force: bool = False) -> str:
-    src = os.path.join(_HERE, "clover_oracle.cpp")
-    if force or not os.path.exists(_LIB_PATH) or \
-            os.path.getmtime(_LIB_PATH) < os.path.getmtime(src):
-        subprocess.check_call(["make", "-s", "-C", _HERE, "liboracle.so"])
+    srcs = [os.path.join(_HERE, f) for f in ("clover_oracle.cpp", "clover_oracle.h",
+                                             "clover_oracle_main.cpp")]
+    newest = max(os.path.getmtime(s) for s in srcs)
+    for target in (_LIB_PATH, CLI_PATH):
+        if force or not os.path.exists(target) or os.path.getmtime(target) < newest:
+            if force:
+                subprocess.check_call(["make", "-s", "-B", "-C", _HERE, os.path.basename(target)])
+            else:
+                subprocess.check_call(["make", "-s", "-C", _HERE, os.path.basename(target)])
     return _LIB_PATH
 
 

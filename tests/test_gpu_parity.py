@@ -298,6 +298,30 @@ def test_divergence_limit_decks_bitwise(torch_cuda, axis, pxy):
     assert_summary_close(g.field_summary(), o.field_summary())
 
 
+@pytest.mark.parametrize("mirror", [0, 1])
+def test_byte_equal_to_oracle_cli_dump(torch_cuda, tmp_path, mirror):
+    """the oracle's command-line driver (text deck in,
+    raw fp64 dumps out) and clover_read_field share one layout, so parity is
+    a byte compare of the files: state, EOS fields, viscosity and the volume
+    fluxes (the fused sweeps never store the mass fluxes)."""
+    import subprocess
+
+    import oracle
+    from oracle.deck import deck_to_text
+    deck = fuzz_deck(6, nx=45, ny=38)
+    deck["face_mirror"] = mirror
+    oracle.build()
+    (tmp_path / "clover.in").write_text(deck_to_text(deck))
+    r = subprocess.run([oracle.CLI_PATH, "--steps", "8", "--dump", str(tmp_path),
+                        str(tmp_path / "clover.in")], capture_output=True, text=True, timeout=300)
+    assert r.returncode == 0, r.stderr
+    g = make_gpu(deck)
+    g.step(8)
+    for f in ("density0", "energy0", "pressure", "soundspeed", "viscosity", "xvel0", "yvel0",
+              "vol_flux_x", "vol_flux_y"):
+        assert g.read(f).astype("<f8").tobytes() == (tmp_path / f"{f}.f64").read_bytes(), f
+
+
 def test_invariant_decks(torch_cuda):
     for deck in (quiescent_deck(64), contact_deck(64), symmetric_deck(64)):
         g, o = make_gpu(deck), Oracle(deck)
