@@ -159,6 +159,22 @@ class ClockSampler:
                 "source": "nvml" if self.rows and self.rows[0][3] == "" else "nvidia-smi"}
 
 
+# The paper's own CloverLeaf numbers (PAPER.md:177-205 Fig. 5, :209, :259
+# Fig. 6): context only -- whole-application runtimes whose
+# mesh, step count and single-node hardware the paper does not state.
+PAPER_CONTEXT = {
+    "fig5_runtime_s": {"CUDA original": 14.14, "CUDA OPS": 15.01, "OpenCL GPU original": 16.19,
+                       "OpenCL GPU OPS": 16.27, "OpenACC original": 21.67, "OpenACC OPS": 19.82,
+                       "32 MPI CPU original": 44.60, "32 MPI CPU OPS": 45.55},
+    "fig5_hardware": "not stated (the paper's other single-node runs: Xeon E5-2697 v2 + Tesla K40, "
+                     "PAPER.md:93,109); workload not stated",
+    "fig6": "ORNL Titan (Cray XK7, K20X GPUs): weak scaling -6% from 1 to 8192 GPUs, -1% from 16 to "
+            "65k CPU cores; GPU strong scaling 'does not strong scale very well' (PAPER.md:259)",
+    "note": "context only, not a target: no cell-updates/s or GB/s are published (BASELINE.json "
+            "published = {})",
+}
+
+
 def host_cpu():
     """CPU model and logical core count of this host (for cpu_baseline)."""
     model = None
@@ -492,6 +508,7 @@ def main():
                 "kernels": kernels,
                 "active_flow": active,
                 "full_run": full,
+                "paper_context": PAPER_CONTEXT,
                 "summary_after": summ}
         print(json.dumps(line), flush=True)
     sim.close()

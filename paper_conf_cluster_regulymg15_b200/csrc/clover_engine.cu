@@ -263,6 +263,7 @@ struct clover_ctx {
   // only if every block of that launch is co-resident: the band blocks spin
   // until the fixup blocks are done (clover_init checks the occupancy)
   bool walls_fold_fits = false;
+  bool f2_probe = false;  // CLOVER_F2_PROBE=1 at init: sweep-2 y kernel with the visc epilogue (A/B only)
   cudaGraphExec_t gexec[4] = {nullptr, nullptr, nullptr, nullptr};  // [parity + 2 * multi-step]
   int64_t ws_bytes = 0;
   bool prof = false;
@@ -903,6 +904,20 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
             launch_fix(kf_advec_y<1>, FIX_BLOCKS, SB, st, c, ta, tb, cs.buf[rout], cs.buf[eout],
                         cs.buf[B_MY], cs.buf[uout], cs.buf[vout], cs.fix);
             FIX_LAUNCH_CHECK();
+          } else if (ctx->f2_probe) {
+            // DESIGN.md 9 f2 probe: sweep 2 with the next step's viscosity
+            // and calc_dt terms folded in (q written, dt to a scratch slot;
+            // visc_dt still runs, so results are unchanged)
+            ViscProbe vp;
+            vp.q = cs.buf[B_Q];
+            vp.dt = (unsigned long long*)cs.partials;
+            vp.prm = ctx->dtp;
+            launch_step(ks_advec_y2_probe, g, SB, st, c, ta, tb, cs.buf[rout], cs.buf[eout],
+                        cs.buf[B_MY], cs.buf[uout], cs.buf[vout], cs.fix, vp);
+            STEP_LAUNCH_CHECK();
+            launch_fix(kf_advec_y<2>, FIX_BLOCKS, SB, st, c, ta, tb, cs.buf[rout], cs.buf[eout],
+                        cs.buf[B_MY], cs.buf[uout], cs.buf[vout], cs.fix);
+            FIX_LAUNCH_CHECK();
           } else {
             launch_step(ks_advec_y<2>, g, SB, st, c, ta, tb, cs.buf[rout], cs.buf[eout], cs.buf[B_MY],
                         cs.buf[uout], cs.buf[vout], cs.fix);
@@ -1424,6 +1439,7 @@ int clover_init(const clover_grid* grid, const clover_state* states, int32_t nst
     const int64_t resident = (int64_t)nsm * std::min(b1, b2);
     ctx->walls_fold_fits = ctx->chunks.size() == 1 &&
                            (int64_t)FIX_BLOCKS + 5 * ywalls_of(ctx->chunks[0], 1).nbx <= resident;
+    if (const char* e = std::getenv("CLOVER_F2_PROBE")) ctx->f2_probe = std::atoi(e) != 0;
     if (const char* e = std::getenv("CLOVER_WALLS_FOLD_LIMIT"))  // test hook: force the unfolded path
       ctx->walls_fold_fits = ctx->walls_fold_fits && std::atoi(e) != 0;
   }
