@@ -54,6 +54,20 @@ if os.path.exists(src):
                      f"{m.get('dram__bytes_read.sum', 0):.0f},{m.get('dram__bytes_write.sum', 0):.0f}\n")
     print("wrote launches", len(order))
 
+# NCCL virtual-remote launch list (kernel name, duration): NCCL's own kernels
+src = os.path.join(G, "launches_nccl.csv")
+if os.path.exists(src):
+    lines = [l for l in open(src) if l.startswith('"')]
+    rows = list(csv.reader(io.StringIO("".join(lines))))
+    hdr, data = rows[0], rows[1:]
+    ki, mi, vi = hdr.index("Kernel Name"), hdr.index("Metric Name"), hdr.index("Metric Value")
+    with open(os.path.join(P, f"{tag}_launches_nccl.csv"), "w") as fh:
+        fh.write("launch,kernel,gpu_time_ns\n")
+        for r in data:
+            if r[mi] == "gpu__time_duration.sum":
+                fh.write(f"{r[0]},{r[ki].split('(')[0]},{r[vi].replace(',', '')}\n")
+    print("wrote nccl launches")
+
 # full capture
 rep = os.path.join(G, "prof_full.ncu-rep")
 if os.path.exists(rep):
@@ -71,7 +85,7 @@ if os.path.exists(rep):
     kern = {}
     md = [f"# ncu --set full summary ({tag}): bm 3840x3840, one launch per kernel type\n",
           "Captured with `ncu --set full --clock-control none --import-source on -k regex:ks_` on "
-          "`scripts/prof_run.py 3840 3840 8` (scripts/profile_round.sh). DRAM bytes in MB "
+          "`scripts/prof_run.py 3840 3840 53` with `-s 200 -c 8`: steps 51-52, x-first then y-first (scripts/profile_round.sh). DRAM bytes in MB "
           "(units as reported: " + units[hdr.index('dram__bytes_read.sum')] + ").\n",
           "| kernel | time us | DRAM read | DRAM write | DRAM GB/s | issue % | fp64 pipe % | warps active % | regs | thread inst/cell |",
           "|---|---|---|---|---|---|---|---|---|---|"]
