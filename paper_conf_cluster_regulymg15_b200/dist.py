@@ -34,9 +34,16 @@ def chunk_grid(nranks: int, nx: int, ny: int, strips: bool = True) -> tuple[int,
 
 
 def weak_mesh(nranks: int, per: int = 3840) -> tuple[int, int, int, int]:
-    """Reading A4: per-rank per^2 cells, stacked along y (1 x nranks chunk
-    grid): global mesh per x (per * nranks) and the chunk grid."""
-    return per, per * nranks, 1, nranks
+    """Reading A4: per^2 cells per rank on the fixed [0,10]^2
+    domain, the global mesh growing in both axes -- 1: per^2, 2: 2per x per,
+    4: (2per)^2, 8: 4per x 2per (nranks = a*b, b the largest power of two
+    with b*b <= nranks, a = nranks/b); y strips (1 x nranks chunk grid), so
+    every rank owns per^2 cells and both sweeps stay fused."""
+    b = 1
+    while (2 * b) * (2 * b) <= nranks and nranks % (2 * b) == 0:
+        b *= 2
+    a = nranks // b
+    return per * a, per * b, 1, nranks
 
 
 def share_unique_id(make_id) -> bytes:

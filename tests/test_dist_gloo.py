@@ -63,7 +63,7 @@ def test_two_ranks_gloo(world):
     sizes = res[0][3]
     assert all(rc == 0 for rc, _ in sizes)
     assert sizes[0][1] == sizes[1][1] > 0  # equal chunks -> equal workspaces
-    assert res[0][4] == (64, 128, 1, 2)
+    assert res[0][4] == (128, 64, 1, 2)
 
 
 def test_chunk_grid_and_weak_series():
@@ -74,5 +74,12 @@ def test_chunk_grid_and_weak_series():
     assert cdist.chunk_grid(8, 7680, 7680, strips=False) in ((2, 4), (4, 2))
     assert cdist.chunk_grid(2, 1000, 100, strips=False) == (2, 1)
     assert cdist.chunk_grid(8, 100, 64)[0] > 1  # strips would be < 16 rows
-    assert cdist.weak_mesh(8) == (3840, 30720, 1, 8)
-    assert cdist.weak_mesh(2) == (3840, 7680, 1, 2)
+    # SURVEY reading A4: per-GPU 3840^2 on [0,10]^2: 1: 3840^2, 2: 7680x3840,
+    # 4: 7680^2, 8: 15360x7680, y strips
+    assert cdist.weak_mesh(1) == (3840, 3840, 1, 1)
+    assert cdist.weak_mesh(2) == (7680, 3840, 1, 2)
+    assert cdist.weak_mesh(4) == (7680, 7680, 1, 4)
+    assert cdist.weak_mesh(8) == (15360, 7680, 1, 8)
+    for n in (1, 2, 4, 8, 3, 6):
+        nx, ny, px, py = cdist.weak_mesh(n)
+        assert nx * ny == n * 3840 * 3840 and px * py == n
