@@ -135,9 +135,9 @@ Layout decompose(int NX, int NY, int px, int py) {
 }
 
 int64_t field_elems(int nx, int ny, int* pitch_out) {
-  // columns: j in [-HALO, nx+1+HALO] with j=0 at COL0; rows k in
-  // [-HALO_ROWS, ny+1+HALO_ROWS]
-  int pitch = (int)align_up(COL0 + nx + 2 + HALO, 32);
+  // columns: j in [-COL0, nx+1+HALO_COLS] (at least) with j=0 at COL0;
+  // rows k in [-HALO_ROWS, ny+1+HALO_ROWS]
+  int pitch = (int)align_up(COL0 + nx + 2 + HALO_COLS, 32);
   if (pitch_out) *pitch_out = pitch;
   int rows = ny + 2 + 2 * HALO_ROWS;
   return (int64_t)pitch * rows;
@@ -259,6 +259,7 @@ struct clover_ctx {
   bool fuse_x = true;  // fused x sweep where every chunk has both x walls (see fuse_x_ok)
   bool fuse_y = true;  // fused y sweep (see fuse_y_ok)
   bool fuse_y_chunks = true;  // ... also at y chunk boundaries (depth-4 row exchange)
+  bool fuse_x_chunks = true;  // fused x sweep also at x chunk boundaries (depth-4 column exchange)
   // the y-wall band blocks may ride on a fixup launch (y_walls_after_fix)
   // only if every block of that launch is co-resident: the band blocks spin
   // until the fixup blocks are done (clover_init checks the occupancy)
@@ -340,7 +341,7 @@ int64_t compute_workspace(const clover_grid* g, int px, int py, int rank, int nr
     bytes += align_up((int64_t)ntx * nty * 5 * 8, kAlign);
     bytes += fix_bytes(nx, ny);
     maxrows = std::max<int64_t>(maxrows, ny + 2 + 2 * HALO_ROWS);
-    maxcols = std::max<int64_t>(maxcols, nx + 2 + 2 * HALO);
+    maxcols = std::max<int64_t>(maxcols, nx + 2 + 2 * HALO_COLS);
   }
   if (px * py > 1) {
     // staging for the remote-neighbour path: every local chunk x 4 sides x
@@ -409,10 +410,11 @@ struct StripQueue {
 
 // strips for side `side` (0 left, 1 right, 2 bottom, 3 top) of chunk cs:
 // send = owned points next to that side, recv = halo points of that side.
-// x sides are HALO columns deep; y sides `ydepth` rows (HALO, or HALO_ROWS
-// for the inputs of a fused y sweep).
+// x sides are `xdepth` columns deep, y sides `ydepth` rows: HALO, or 4
+// (HALO_COLS / HALO_ROWS) for the inputs of a fused sweep across a chunk
+// boundary.
 void side_strips(const ChunkState& cs, int buf, int side, XferDesc& send, XferDesc& recv,
-                 int ydepth = HALO) {
+                 int ydepth = HALO, int xdepth = HALO) {
   const Chunk& c = cs.c;
   const int kind = kBufKind[buf];
   const int ox = (kind == K_XVEL || kind == K_YVEL || kind == K_XFACE) ? 1 : 0;
@@ -420,25 +422,26 @@ void side_strips(const ChunkState& cs, int buf, int side, XferDesc& send, XferDe
   send.base = recv.base = cs.buf[buf];
   send.pitch = recv.pitch = c.pitch;
   // full extent of this kind including both halos: rows [-HALO_ROWS,
-  // ny+oy+HALO_ROWS], columns [-HALO, nx+ox+HALO] (x strips carry every row,
-  // y strips every column, so 4-chunk corners are refreshed by the second axis)
-  const int full_h = c.ny + oy + 1 + 2 * HALO_ROWS, full_w = c.nx + ox + 1 + 2 * HALO;
-  if (side == 0) {          // left: send [1+ox, HALO+ox], recv [1-HALO, 0]
-    send.j0 = 1 + ox; recv.j0 = 1 - HALO;
-    send.w = recv.w = HALO;
+  // ny+oy+HALO_ROWS], columns [-HALO_COLS, nx+ox+HALO_COLS] (x strips carry
+  // every row, y strips every column, so 4-chunk corners are refreshed by
+  // the second axis)
+  const int full_h = c.ny + oy + 1 + 2 * HALO_ROWS, full_w = c.nx + ox + 1 + 2 * HALO_COLS;
+  if (side == 0) {          // left: send [1+ox, d+ox], recv [1-d, 0]
+    send.j0 = 1 + ox; recv.j0 = 1 - xdepth;
+    send.w = recv.w = xdepth;
     send.k0 = recv.k0 = -HALO_ROWS; send.h = recv.h = full_h;
-  } else if (side == 1) {   // right: send [nx+1-HALO, nx], recv [nx+ox+1, nx+ox+HALO]
-    send.j0 = c.nx + 1 - HALO; recv.j0 = c.nx + ox + 1;
-    send.w = recv.w = HALO;
+  } else if (side == 1) {   // right: send [nx+1-d, nx], recv [nx+ox+1, nx+ox+d]
+    send.j0 = c.nx + 1 - xdepth; recv.j0 = c.nx + ox + 1;
+    send.w = recv.w = xdepth;
     send.k0 = recv.k0 = -HALO_ROWS; send.h = recv.h = full_h;
   } else if (side == 2) {   // bottom: send [1+oy, d+oy], recv [1-d, 0]
     send.k0 = 1 + oy; recv.k0 = 1 - ydepth;
     send.h = recv.h = ydepth;
-    send.j0 = recv.j0 = -HALO; send.w = recv.w = full_w;
+    send.j0 = recv.j0 = -HALO_COLS; send.w = recv.w = full_w;
   } else {                  // top: send [ny+1-d, ny], recv [ny+oy+1, ny+oy+d]
     send.k0 = c.ny + 1 - ydepth; recv.k0 = c.ny + oy + 1;
     send.h = recv.h = ydepth;
-    send.j0 = recv.j0 = -HALO; send.w = recv.w = full_w;
+    send.j0 = recv.j0 = -HALO_COLS; send.w = recv.w = full_w;
   }
 }
 
@@ -480,7 +483,8 @@ int StripQueue::flush() {
   return CLOVER_OK;
 }
 
-int exchange_axis(clover_ctx* ctx, const std::vector<int>& bufs, int axis, int ydepth = HALO) {
+int exchange_axis(clover_ctx* ctx, const std::vector<int>& bufs, int axis, int ydepth = HALO,
+                  int xdepth = HALO) {
   const int s_lo = axis == 0 ? 0 : 2, s_hi = axis == 0 ? 1 : 3;
   // stage 1 (one batch): local pairs' halo strips and the packing of the
   // remote sides (owned points in, halo points / staging out: disjoint)
@@ -493,8 +497,8 @@ int exchange_axis(clover_ctx* ctx, const std::vector<int>& bufs, int axis, int y
     if (!other) continue;
     for (int b : bufs) {
       XferDesc sA, rA, sB, rB;
-      side_strips(cs, b, s_hi, sA, rA, ydepth);
-      side_strips(*other, b, s_lo, sB, rB, ydepth);
+      side_strips(cs, b, s_hi, sA, rA, ydepth, xdepth);
+      side_strips(*other, b, s_lo, sB, rB, ydepth, xdepth);
       int rc = q.add(rB, sA);  // my high side -> neighbour's low halo
       if (rc) return rc;
       rc = q.add(rA, sB);      // neighbour's low side -> my high halo
@@ -517,14 +521,14 @@ int exchange_axis(clover_ctx* ctx, const std::vector<int>& bufs, int axis, int y
         int64_t n = 0;
         for (int b : bufs) {
           XferDesc s, r;
-          side_strips(cs, b, side, s, r, ydepth);
+          side_strips(cs, b, side, s, r, ydepth, xdepth);
           n += (int64_t)s.w * s.h;
         }
         if (off + n > ctx->xbuf_elems) return fail(CLOVER_ERR_STATE, "halo staging buffer too small");
         n = 0;
         for (int b : bufs) {
           XferDesc s, r;
-          side_strips(cs, b, side, s, r, ydepth);
+          side_strips(cs, b, side, s, r, ydepth, xdepth);
           XferDesc dst{ctx->xbuf_send + off + n, s.w, 0, 0, s.w, s.h};
           int rc = q.add(dst, s);
           if (rc) return rc;
@@ -601,7 +605,7 @@ int exchange_axis(clover_ctx* ctx, const std::vector<int>& bufs, int axis, int y
       int64_t n = 0;
       for (int b : bufs) {
         XferDesc s, r;
-        side_strips(*m.cs, b, m.side, s, r, ydepth);
+        side_strips(*m.cs, b, m.side, s, r, ydepth, xdepth);
         XferDesc src{ctx->xbuf_recv + m.off + n, r.w, 0, 0, r.w, r.h};
         rc = q.add(r, src);
         if (rc) return rc;
@@ -614,11 +618,11 @@ int exchange_axis(clover_ctx* ctx, const std::vector<int>& bufs, int axis, int y
 
 bool needs_exchange(const clover_ctx* ctx) { return ctx->L.px * ctx->L.py > 1; }
 
-int exchange(clover_ctx* ctx, const std::vector<int>& bufs, int ydepth = HALO) {
+int exchange(clover_ctx* ctx, const std::vector<int>& bufs, int ydepth = HALO, int xdepth = HALO) {
   if (!needs_exchange(ctx)) return CLOVER_OK;
-  int rc = exchange_axis(ctx, bufs, 0);
+  int rc = exchange_axis(ctx, bufs, 0, ydepth, xdepth);
   if (rc) return rc;
-  return exchange_axis(ctx, bufs, 1, ydepth);
+  return exchange_axis(ctx, bufs, 1, ydepth, xdepth);
 }
 
 // ---------------------------------------------------------------- schedule
@@ -704,12 +708,14 @@ cudaError_t launch_fix(void (*kernel)(KArgs...), dim3 grid, dim3 block, cudaStre
   return launch_pdl(CLOVER_PDL_FIX, kernel, grid, block, st, std::forward<Args>(args)...);
 }
 
-// The fused x sweep needs every chunk to have reflective walls on both x
-// sides (its wall halo columns are mirrors of lanes in the same warp; at a
-// chunk boundary the x stencil would need depth-3 halos) and the geometric
-// face mirror.
+// The fused x sweep (reach 4 columns along x) runs at x walls (mirrors of
+// lanes of the same warp) and at x chunk boundaries (its inputs exchanged
+// HALO_COLS deep, the neighbour's first columns recomputed); it needs the
+// geometric face mirror.  fuse_x_chunks = false keeps the separate cell /
+// momentum kernels at x chunk boundaries (A/B and tests).
 bool fuse_x_ok(const clover_ctx* ctx) {
   if (!ctx->fuse_x || ctx->g.face_mirror == CLOVER_MIRROR_CELLCENTRE) return false;
+  if (ctx->fuse_x_chunks) return true;
   for (const auto& cs : ctx->chunks)
     if (!cs.c.wl || !cs.c.wr) return false;
   return true;
@@ -827,7 +833,8 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
       FIX_LAUNCH_CHECK();
     }
     // a fused y sweep (either sweep) reads these HALO_ROWS deep in y
-    int rc = exchange(ctx, {B_D1, B_E1, B_U1, B_V1, B_FX, B_FY}, fuse_y_ok(ctx) ? HALO_ROWS : HALO);
+    int rc = exchange(ctx, {B_D1, B_E1, B_U1, B_V1, B_FX, B_FY}, fuse_y_ok(ctx) ? HALO_ROWS : HALO,
+                      fuse_x_ok(ctx) ? HALO_COLS : HALO);
     if (rc) return rc;
     if (ctx->prof) prof_mark(ctx, -1);
   }
@@ -927,7 +934,9 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
             FIX_LAUNCH_CHECK();
           }
         }
-        int rc = exchange(ctx, {rout, eout, uout, vout});
+        // y sweep 1 feeds a fused x sweep 2: HALO_COLS deep in x
+        int rc = exchange(ctx, {rout, eout, uout, vout}, HALO,
+                          (sweep == 1 && fuse_x_ok(ctx)) ? HALO_COLS : HALO);
         if (rc) return rc;
         if (ctx->prof) prof_mark(ctx, -1);
       }
@@ -968,9 +977,11 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
         }
       }
       // x sweep 1 feeding a fused y sweep 2: the post-sweep density and
-      // energy HALO_ROWS deep in y
+      // energy HALO_ROWS deep in y; y sweep 1 feeding a fused x sweep 2:
+      // HALO_COLS deep in x
       const int yd = (sweep == 1 && xdir && fuse_y_ok(ctx)) ? HALO_ROWS : HALO;
-      int rc = exchange(ctx, {rout, eout, mbuf}, yd);
+      const int xd = (sweep == 1 && !xdir && fuse_x_ok(ctx)) ? HALO_COLS : HALO;
+      int rc = exchange(ctx, {rout, eout, mbuf}, yd, xd);
       if (rc) return rc;
       if (ctx->prof) prof_mark(ctx, -1);
     }
@@ -1007,7 +1018,8 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
         }
       }
       const int yd = (sweep == 1 && xdir && fuse_y_ok(ctx)) ? HALO_ROWS : HALO;
-      int rc = exchange(ctx, {uout, vout}, yd);
+      const int xd = (sweep == 1 && !xdir && fuse_x_ok(ctx)) ? HALO_COLS : HALO;
+      int rc = exchange(ctx, {uout, vout}, yd, xd);
       if (rc) return rc;
       if (ctx->prof) prof_mark(ctx, -1);
     }
@@ -1424,7 +1436,7 @@ int clover_init(const clover_grid* grid, const clover_state* states, int32_t nst
     cs.fix.e = (uint2*)(p + kAlign);
     p += fix_bytes(c.nx, c.ny);
     maxrows = std::max<int64_t>(maxrows, c.ny + 2 + 2 * HALO_ROWS);
-    maxcols = std::max<int64_t>(maxcols, c.nx + 2 + 2 * HALO);
+    maxcols = std::max<int64_t>(maxcols, c.nx + 2 + 2 * HALO_COLS);
     ctx->chunks.push_back(cs);
   }
   {
@@ -1557,6 +1569,7 @@ int clover_debug_set_fusion(clover_ctx* ctx, int32_t enable) {
   ctx->fuse_x = enable != 0;
   ctx->fuse_y = enable != 0;
   ctx->fuse_y_chunks = enable == 1;
+  ctx->fuse_x_chunks = enable == 1;
   for (int i = 0; i < 4; ++i)
     if (ctx->gexec[i]) {
       cudaGraphExecDestroy(ctx->gexec[i]);

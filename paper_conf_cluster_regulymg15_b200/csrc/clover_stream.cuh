@@ -1062,8 +1062,10 @@ kf_advec_mom_x(Chunk c, const double* __restrict__ rho, const double* __restrict
 }
 
 // ================================================================ fused x sweep
-// advec_cell (x) and advec_mom (x) of one sweep in one pass, for chunks with
-// reflective walls on both x sides (px == 1) and the geometric face mirror.
+// advec_cell (x) and advec_mom (x) of one sweep in one pass (geometric face
+// mirror).  At x walls the halo columns are mirrors of lanes of the same
+// warp; at x chunk boundaries they are recomputed from inputs exchanged
+// HALO_COLS deep (reach: cells j-3 .. j+3, x-faces depth 3).
 // Warp strip: lane l <-> column j = J0 - 2 + l, J0 = 1 + 28*(warp).  At cell
 // row r every lane computes the x-face flux of face j and (lanes 0..30) the
 // cell update of cell j; lanes on wall halo columns take the mirror image of
@@ -1119,18 +1121,22 @@ __device__ __forceinline__ bool advec_x_body(const Chunk& c, const CUtensorMap* 
   const int j = J0 - 2 + lane;
   const double vol = c.dx * c.dy;
   const int nx = c.nx;
-  const bool faceok = !EDGE || (j >= 1 && j <= nx + 1);  // faces computed here (others mirrored)
-  const bool cellok = !EDGE || (j >= 0 && j <= nx + 2);  // pre_vol inputs exist
-  const bool mpok = !EDGE || (j >= -1 && j <= nx + 2);   // node-mass columns
+  // at an x wall the halo faces / cells are mirrors of lanes of this warp;
+  // at an x chunk boundary (no wall) they are computed from the HALO_COLS
+  // deep input halos, bitwise what the neighbour computes
+  const bool faceok = !EDGE || ((!c.wl || j >= 1) && (!c.wr || j <= nx + 1));  // faces computed here
+  const bool cellok = !EDGE || ((!c.wl || j >= 0) && (!c.wr || j <= nx + 2));  // pre_vol inputs exist
+  const bool mpok = !EDGE || ((!c.wl || j >= -1) && (!c.wr || j <= nx + 2));   // node-mass columns
+  const bool cellup = !EDGE || ((!c.wl || j >= 1) && (!c.wr || j <= nx));      // cell updates
   const bool ncol = EDGE && near_wall_col(c, j);
   const bool own = lane >= 2 && lane < 2 + XW;
   // mirror sources at the x walls (lanes of this warp, see header)
   int src_m = lane, src_r = lane;
   double sgn_m = 1.0;
   if (EDGE) {
-    if (j <= 0) { src_m = lane + 2 - 2 * j; src_r = lane + 1 - 2 * j; sgn_m = -1.0; }
-    if (j >= nx + 2) { src_m = lane + 2 * nx + 2 - 2 * j; sgn_m = -1.0; }
-    if (j >= nx + 1) src_r = lane + 2 * nx + 1 - 2 * j;
+    if (c.wl && j <= 0) { src_m = lane + 2 - 2 * j; src_r = lane + 1 - 2 * j; sgn_m = -1.0; }
+    if (c.wr && j >= nx + 2) { src_m = lane + 2 * nx + 2 - 2 * j; sgn_m = -1.0; }
+    if (c.wr && j >= nx + 1) src_r = lane + 2 * nx + 1 - 2 * j;
     if (src_m < 0 || src_m > 31) src_m = lane;
     if (src_r < 0 || src_r > 31) src_r = lane;
   }
@@ -1200,7 +1206,8 @@ __device__ __forceinline__ bool advec_x_body(const Chunk& c, const CUtensorMap* 
           // upwind / donor / downwind columns picked by address (one select
           // per column instead of one per loaded value)
           const bool pos = F > 0.0;
-          const double* pu = pos ? rc - 2 : rc + (EDGE ? min(j + 1, nx + 2) - j : 1);
+          // (the reading's MIN(j+1, x_max+2) upwind clamp only acts at a wall)
+          const double* pu = pos ? rc - 2 : rc + ((EDGE && c.wr) ? min(j + 1, nx + 2) - j : 1);
           const double* pd = pos ? rc - 1 : rc;
           const double* pw = pos ? rc : rc - 1;
           cell_face_flux(dv, F, pos ? pvl : pv, pu[F::R * XRW], pd[F::R * XRW], pw[F::R * XRW],
@@ -1209,7 +1216,7 @@ __device__ __forceinline__ bool advec_x_body(const Chunk& c, const CUtensorMap* 
         const double mh = __shfl_down_sync(FULL, m, 1);
         const double efh = __shfl_down_sync(FULL, ef, 1);
         double eo = 0.0;
-        if ((!EDGE || (j >= 1 && j <= nx)) && lane < 31) {
+        if (cellup && lane < 31) {
           cell_update(dv, rr, ee, pv, m, mh, ef, efh, flo, fhi, ro, eo);
           if (own && r >= k0 && (!EDGE || r <= c.ny)) {
             const bool near = EDGE && (ncol || near_wall_row(c, r));

@@ -20,6 +20,7 @@ nx, ny, px, py = (int(a) for a in sys.argv[1:5])
 steps = int(sys.argv[5]) if len(sys.argv) > 5 else 20
 torch.cuda.set_device(0)
 deck = bm_deck(nx, ny, end_step=steps, ymax=10.0 * ny / nx)
+# (square cells: the domain grows with the mesh)
 
 
 def run(p, q, vr=0, walls_only=False):
@@ -44,8 +45,21 @@ def run(p, q, vr=0, walls_only=False):
 
 one, k1 = run(1, 1)
 res = {"mesh": [nx, ny], "chunks": [px, py], "steps": steps, "one_chunk_ms": one, "one_chunk_kernels": k1}
+# one rank's share alone: a single chunk of the per-rank size (walls on all
+# sides, same cell size) -- what a rank of a real px*py run computes per
+# step minus the exchange; nchunks x this = the serialised one-GPU ideal
+cx, cy = nx // px, ny // py
+deck_full = deck
+deck = bm_deck(cx, cy, end_step=steps, xmax=10.0 * cx / nx, ymax=10.0 * cy / ny)
+alone, _ = run(1, 1)
+deck = deck_full
+res["rank_chunk"] = [cx, cy]
+res["rank_chunk_alone_ms"] = alone
+res["serial_ideal_ms"] = alone * px * py
+res["strong_scaling_efficiency_bound"] = one / (px * py * alone)
 for name, kw in (("local_fused", {}), ("local_walls_only", dict(walls_only=True)),
                  ("virtual_remote", dict(vr=1)), ("virtual_nccl", dict(vr=2))):
     ms, k = run(px, py, **kw)
-    res[name] = {"ms": ms, "overhead": ms / one - 1.0, "kernels": k}
+    res[name] = {"ms": ms, "overhead": ms / one - 1.0, "kernels": k,
+                 "over_serial_ideal": ms / (alone * px * py) - 1.0}
 print(json.dumps(res), flush=True)

@@ -383,13 +383,14 @@ def test_virtual_remote_through_nccl_bitwise(torch_cuda, pxy):
     assert many.field_summary() == one.field_summary()
 
 
-@pytest.mark.parametrize("seed,pxy", [(8, (1, 2)), (9, (1, 4)), (10, (2, 3)), (11, (1, 5))])
-def test_fused_y_sweep_across_chunk_boundaries(torch_cuda, seed, pxy):
-    """at y chunk boundaries the
-    fused y sweep recomputes the neighbour's first post-sweep rows from
-    depth-4 input halos.  Same bits as the separate cell / momentum kernels
-    with their extra exchange (fusion walls_only) and as one chunk, on
-    fuzz decks (flow across the boundaries) for 12 steps (both sweep
+@pytest.mark.parametrize("seed,pxy", [(8, (1, 2)), (9, (1, 4)), (10, (2, 3)), (11, (1, 5)),
+                                      (12, (2, 1)), (13, (3, 1)), (14, (4, 2)), (15, (3, 3))])
+def test_fused_sweeps_across_chunk_boundaries(torch_cuda, seed, pxy):
+    """at chunk boundaries the fused
+    sweeps recompute the neighbour's first post-sweep rows (y) / columns (x)
+    from depth-4 input halos.  Same bits as the separate cell / momentum
+    kernels with their extra exchanges (fusion walls_only) and as one chunk,
+    on fuzz decks (flow across the boundaries) for 12 steps (both sweep
     orders), local and virtual-remote exchange."""
     deck = fuzz_deck(seed, nx=72, ny=96)
     deck["max_timestep"] = 1.0
@@ -537,15 +538,14 @@ def test_full_size_first_steps(torch_cuda, n, steps):
     assert_summary_close(g.field_summary(), o.field_summary(compensated=True))
 
 
-@pytest.mark.parametrize("pxy,expected", [((1, 1), 8), ((3, 1), 34), ((1, 3), 27)])
+@pytest.mark.parametrize("pxy,expected", [((1, 1), 8), ((3, 1), 28), ((1, 3), 27)])
 def test_kernels_per_step(torch_cuda, pxy, expected):
     """Launches per step (bench.py's gpu_launches): one chunk runs visc_dt,
     Lagrangian and both fused sweeps with a fixup each, the y-wall bands
     riding on the fixup before the y sweep (8); several chunks launch the
     bands separately (+1 per chunk with a y wall) and finalise dt in
-    k_dt_finalize (+1); x chunk boundaries use the separate x kernels, 4
-    launches per chunk: 3x1 = 3 * (4 + 4 + 3) + 1; y chunk boundaries keep
-    the fused y sweep: 1x3 = (4 + 2 + 3) + (4 + 2 + 2) + (4 + 2 + 3) + 1."""
+    k_dt_finalize (+1); chunk boundaries keep both fused sweeps: 3x1 =
+    3 * (4 + 2 + 3) + 1, 1x3 = (4 + 2 + 3) + (4 + 2 + 2) + (4 + 2 + 3) + 1."""
     px, py = pxy
     g = make_gpu(fuzz_deck(11), px=px, py=py)
     assert g.kernels_per_step() == expected
