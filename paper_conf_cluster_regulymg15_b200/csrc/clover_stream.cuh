@@ -335,6 +335,8 @@ __device__ __forceinline__ bool visc_body(const Chunk& c, const CUtensorMap* __r
     acc.bottom(row(k0)[VF_V * VRW], row(k0)[VF_V * VRW + 1], c);
   const bool left = EDGE && j == 1;  // column 1: no left neighbour takes this face
   int i = idx(c, j, k0);
+  // (ring slots by mask: VSTG is a power of two; rotating the row pointers
+  // as the Lagrangian and y-sweep bodies do measured neutral here, +2 regs)
   for (int k = k0; k < k1; ++k, i += c.pitch) {
     wait_row(k + 1);
     const double* rc = row(k);
@@ -573,18 +575,24 @@ __device__ __forceinline__ bool lagr_body(const Chunk& c, const CUtensorMap* __r
     massl_m = a[LF_R * LRW - 1] * vol;
   }
   double u1_m = 0.0, v1_m = 0.0, u1r_m = 0.0, v1r_m = 0.0;
+  // ring rows k-1, k, k+1 of the iteration, rotated at its end (one slot
+  // address per row instead of a modulo per access); slot / phase of row k+1
+  const double* Pm = row(k0 - 1);
+  const double* Pc = row(k0);
+  const double* Pn = row(k0 + 1);
+  unsigned wsl = 2u % (unsigned)LSTG, wph = 0u;
   for (int k = k0; k <= k1; ++k) {
-    wait_row(k + 1);
-    const double* rm = row(k - 1);
-    const double* rc = row(k);
+    mbar_wait(&bars[wsl], wph);  // row k+1
+    const double* rm = Pm;
+    const double* rc = Pc;
     double ph = 0.0;
     if constexpr (EDGE) {
       if (c.wt && k == c.ny + 1)
         ph = ph_m;  // reflective top: mirror of row ny
       else if (colok)
-        ph = predict(rc, row(k + 1));
+        ph = predict(rc, Pn);
     } else {
-      const double* rn = row(k + 1);
+      const double* rn = Pn;
       const double tf = pdv_face_pred(rn[LF_V * LRW], rn[LF_V * LRW + 1], dx, dt);
       ph = pdv_predict_pressure_bt(dv, rc[LF_R * LRW], rc[LF_E * LRW], rc[LF_Q * LRW],
                                    rc[LF_U * LRW], rn[LF_U * LRW], rc[LF_U * LRW + 1],
@@ -686,6 +694,9 @@ __device__ __forceinline__ bool lagr_body(const Chunk& c, const CUtensorMap* __r
 #endif
     __syncwarp();
     if (lane == 0 && k - 1 + LSTG <= r_last) issue(k - 1 + LSTG);
+    Pm = Pc; Pc = Pn;
+    if (++wsl == (unsigned)LSTG) { wsl = 0u; wph ^= 1u; }
+    Pn = ring + wsl * LSLOT + lane + 1;
   }
   __syncwarp();
   if (lane == 0)
@@ -1170,6 +1181,9 @@ __device__ __forceinline__ bool advec_x_body(const Chunk& c, const CUtensorMap* 
   wait_row(r_first);
 
   double mA_m = 0.0, mp_m = 0.0, mB_m = 0.0, mpl_m = 0.0, ro_m = 0.0;
+  // (ring slots by mask: XSTG is a power of two; rotating the row pointers
+  // as the Lagrangian and y-sweep bodies do cost 8 registers and 2.7 % on
+  // sweep 1 here)
   for (int r = k0 - 1; r < k1; ++r) {
     wait_row(r + 1);
     const bool mir_bot = EDGE && c.wb && r == 0;  // synthesised from row 1 below
@@ -1606,19 +1620,15 @@ __device__ __forceinline__ bool advec_y_body(const Chunk& c, const CUtensorMap* 
   }
   __syncwarp();
 
-  auto pre_vol = [&](int r) -> double {  // advec_cell pre-sweep volume of cell row r
-    const double* q = row(r);
-    const double* qn = row(r + 1);
+  // advec_cell pre-sweep volume of a cell row (q) given the next row (qn)
+  auto pre_vol_p = [&](const double* q, const double* qn) -> double {
     if constexpr (SWEEP == 1) return vol + (qn[L::FY] - q[L::FY] + q[L::FX + 1] - q[L::FX]);
     else return vol + qn[L::FY] - q[L::FY];
   };
-  auto pv_mom = [&](int r) -> double {  // advec_mom post-sweep volume of cell row r
-    if constexpr (SWEEP == 1) {
-      const double* q = row(r);
-      return vol + q[L::FX + 1] - q[L::FX];
-    } else {
-      return vol;
-    }
+  auto pre_vol = [&](int r) -> double { return pre_vol_p(row(r), row(r + 1)); };
+  auto pv_mom_p = [&](const double* q) -> double {  // advec_mom post-sweep volume
+    if constexpr (SWEEP == 1) return vol + q[L::FX + 1] - q[L::FX];
+    else return vol;
   };
   // at a y wall the faces / cells beyond it are the mirrors ks_cell_y_walls
   // wrote; at a y chunk boundary they are recomputed from the depth-4 input
@@ -1628,17 +1638,22 @@ __device__ __forceinline__ bool advec_y_body(const Chunk& c, const CUtensorMap* 
     return !EDGE || ((!c.wb || f >= 1) && (!c.wt || f <= ny + 1));
   };
   auto cell_computed = [&](int r) { return !EDGE || ((!c.wb || r >= 1) && (!c.wt || r <= ny)); };
-  // flux of face f (between cells f-1 and f); pvlo = pre_vol(f-1), pvhi = pre_vol(f)
-  auto face_flux = [&](int f, double pvlo, double pvhi, double& m, double& ef) {
-    const double F = row(f)[L::FY];
+  // flux of face f (between cells f-1 and f) from the ring rows f-2 .. f+1;
+  // pvlo = pre_vol(f-1), pvhi = pre_vol(f)
+  auto face_flux_p = [&](const double* r2, const double* r1, const double* r0, const double* rp,
+                         double pvlo, double pvhi, double& m, double& ef) {
+    const double F = r0[L::FY];
     // upwind / donor / downwind rows picked by address (one select per row
     // instead of one per loaded value)
     const bool pos = F > 0.0;
-    const double* pu = pos ? row(f - 2) : row(f + 1);
-    const double* pd = pos ? row(f - 1) : row(f);
-    const double* pw = pos ? row(f) : row(f - 1);
+    const double* pu = pos ? r2 : rp;
+    const double* pd = pos ? r1 : r0;
+    const double* pw = pos ? r0 : r1;
     cell_face_flux(dv, F, pos ? pvlo : pvhi, pu[L::R], pd[L::R], pw[L::R], pu[L::E], pd[L::E],
                    pw[L::E], m, ef);
+  };
+  auto face_flux = [&](int f, double pvlo, double pvhi, double& m, double& ef) {
+    face_flux_p(row(f - 2), row(f - 1), row(f), row(f + 1), pvlo, pvhi, m, ef);
   };
 
   // ---- prologue: face k0-2
@@ -1664,23 +1679,32 @@ __device__ __forceinline__ bool advec_y_body(const Chunk& c, const CUtensorMap* 
   double vp1 = 0.0, vp2 = 0.0, vp3 = 0.0, vr1 = 0.0, vr2 = 0.0, ve1 = 0.0, ve2 = 0.0;
   double vu2 = 0.0, vv2 = 0.0;
   DtAcc vacc;
+  // ring rows s-2 .. s+2 of the iteration, rotated at its end (one slot
+  // address per row instead of one per access); slot / phase of row s+2
+  // for its mbarrier wait (rows k0-4 .. k0 are slots 0 .. 4 at s = k0-2)
+  static_assert(L::RING >= 5, "the y sweep reads rows s-2 .. s+2");
+  const double* Rm2 = row(k0 - 4);
+  const double* Rm1 = row(k0 - 3);
+  const double* R0 = row(k0 - 2);
+  const double* Rp1 = row(k0 - 1);
+  const double* Rp2 = row(k0);
+  unsigned wsl = 4u % (unsigned)L::RING, wph = 0u;
 
   for (int s = k0 - 2; s <= k1; ++s) {
-    if (s + 2 <= r_last) wait_row(s + 2);
+    if (s + 2 <= r_last) mbar_wait(&bars[wsl], wph);
     {
       // ---- advec_cell y: face s+1, cell s
       double m1 = 0.0, ef1 = 0.0, pv1 = 0.0, ro = 0.0, eo_s = 0.0;
       if (face_computed(s + 1)) {
-        pv1 = pre_vol(s + 1);
-        if (comp) face_flux(s + 1, pv_s, pv1, m1, ef1);
+        pv1 = pre_vol_p(Rp1, Rp2);
+        if (comp) face_flux_p(Rm1, R0, Rp1, Rp2, pv_s, pv1, m1, ef1);
       } else {
         m1 = mfy[idx(c, j, s + 1)];
       }
       if (cell_computed(s)) {
         if (comp) {
           double eo;
-          const double* q = row(s);
-          cell_update(dv, q[L::R], q[L::E], pv_s, m_s, m1, ef_s, ef1, q[L::FY], row(s + 1)[L::FY],
+          cell_update(dv, R0[L::R], R0[L::E], pv_s, m_s, m1, ef_s, ef1, R0[L::FY], Rp1[L::FY],
                       ro, eo);
           eo_s = eo;
           if (own_cell && s >= k0 && s < k1) {
@@ -1699,7 +1723,7 @@ __device__ __forceinline__ bool advec_y_body(const Chunk& c, const CUtensorMap* 
         if (src != lane) { m1 = ms; ro = rs; }
       }
       // ---- advec_mom y: node flux / masses of row s
-      const double mp = ro * pv_mom(s);
+      const double mp = ro * pv_mom_p(R0);
       const double mpl = __shfl_up_sync(FULL, mp, 1);
       const double myl1 = __shfl_up_sync(FULL, m1, 1);
       const double nf = 0.25 * (myl_s + m_s + myl1 + m1);   // My(j-1,s) My(j,s) My(j-1,s+1) My(j,s+1)
@@ -1711,10 +1735,10 @@ __device__ __forceinline__ bool advec_y_body(const Chunk& c, const CUtensorMap* 
       if (s >= k0 && own_node) {
         const double nfn = nf_p;
         const double nmp = (nfn < 0.0) ? pre : pre_p;
-        const double* qm1 = row(s - 1);
-        const double* q0 = row(s);
+        const double* qm1 = Rm1;
+        const double* q0 = R0;
         const bool neg = nfn < 0.0;
-        const double* pa = neg ? row(s + 1) : row(s - 2);  // upwind
+        const double* pa = neg ? Rp1 : Rm2;  // upwind
         const double* pb = neg ? q0 : qm1;                 // donor
         const double* pc = neg ? qm1 : q0;                 // downwind
         const double uu[3] = {pa[L::U], pb[L::U], pc[L::U]};
@@ -1771,6 +1795,9 @@ __device__ __forceinline__ bool advec_y_body(const Chunk& c, const CUtensorMap* 
       __syncwarp();
       if (lane == 0 && s - 2 + L::RING <= r_last) issue(s - 2 + L::RING);
     }
+    Rm2 = Rm1; Rm1 = R0; R0 = Rp1; Rp1 = Rp2;
+    if (++wsl == (unsigned)L::RING) { wsl = 0u; wph ^= 1u; }
+    Rp2 = ring + wsl * L::SLOT + lane + t0;
   }
   __syncwarp();
   if (lane == 0)
