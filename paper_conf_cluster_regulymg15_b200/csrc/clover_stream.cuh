@@ -514,11 +514,11 @@ __device__ __forceinline__ bool lagr_body(const Chunk& c, const CUtensorMap* __r
   const int r_first = k0 - 1, r_last = k1 + 1;  // staged rows
   const int xcol = COL0 + J0 - 2;  // = 14 + 30*gw: even, 16-B aligned (see visc_body)
   auto slot_of = [&](int r) { return (unsigned)(r - r_first) % (unsigned)LSTG; };
-  auto issue = [&](int r) {
-    const unsigned sl = slot_of(r);
+  auto issue_at = [&](unsigned sl, int r) {  // row r into slot sl
     mbar_arrive_expect_tx(&bars[sl], LBYTES);
     tma_load_3d(ring + sl * LSLOT, tm, xcol, ROW0 + r, 0, &bars[sl]);
   };
+  auto issue = [&](int r) { issue_at(slot_of(r), r); };
   auto wait_row = [&](int r) {
     const unsigned rel = (unsigned)(r - r_first);
     mbar_wait(&bars[rel % LSTG], (rel / LSTG) & 1u);
@@ -581,6 +581,7 @@ __device__ __forceinline__ bool lagr_body(const Chunk& c, const CUtensorMap* __r
   const double* Pc = row(k0);
   const double* Pn = row(k0 + 1);
   unsigned wsl = 2u % (unsigned)LSTG, wph = 0u;
+  unsigned isl = 0u;  // slot of row k-1, refilled at the end of iteration k
   for (int k = k0; k <= k1; ++k) {
     mbar_wait(&bars[wsl], wph);  // row k+1
     const double* rm = Pm;
@@ -693,7 +694,8 @@ __device__ __forceinline__ bool lagr_body(const Chunk& c, const CUtensorMap* __r
     fence_proxy_async();
 #endif
     __syncwarp();
-    if (lane == 0 && k - 1 + LSTG <= r_last) issue(k - 1 + LSTG);
+    if (lane == 0 && k - 1 + LSTG <= r_last) issue_at(isl, k - 1 + LSTG);
+    if (++isl == (unsigned)LSTG) isl = 0u;
     Pm = Pc; Pc = Pn;
     if (++wsl == (unsigned)LSTG) { wsl = 0u; wph ^= 1u; }
     Pn = ring + wsl * LSLOT + lane + 1;
@@ -1586,8 +1588,7 @@ __device__ __forceinline__ bool advec_y_body(const Chunk& c, const CUtensorMap* 
   const unsigned long long pol_once = l2_policy_evict_first();
 #endif
 #endif
-  auto issue = [&](int r) {
-    const unsigned sl = (unsigned)(r - r_first) % (unsigned)L::RING;
+  auto issue_at = [&](unsigned sl, int r) {  // row r into slot sl
     double* d = ring + sl * L::SLOT;
     mbar_arrive_expect_tx(&bars[sl], L::BYTES);
 #if CLOVER_L2HINT
@@ -1605,6 +1606,7 @@ __device__ __forceinline__ bool advec_y_body(const Chunk& c, const CUtensorMap* 
     tma_load_3d(d, ta, xcol, ROW0 + r, 0, &bars[sl]);
     if constexpr (SWEEP == 2) tma_load_3d(d + L::B, tb, xcol, ROW0 + r, 0, &bars[sl]);
   };
+  auto issue = [&](int r) { issue_at((unsigned)(r - r_first) % (unsigned)L::RING, r); };
   auto row = [&](int r) -> const double* {
     return ring + ((unsigned)(r - r_first) % (unsigned)L::RING) * L::SLOT + lane + t0;
   };
@@ -1689,6 +1691,7 @@ __device__ __forceinline__ bool advec_y_body(const Chunk& c, const CUtensorMap* 
   const double* Rp1 = row(k0 - 1);
   const double* Rp2 = row(k0);
   unsigned wsl = 4u % (unsigned)L::RING, wph = 0u;
+  unsigned isl = 0u;  // slot of row s-2, refilled at the end of iteration s
 
   for (int s = k0 - 2; s <= k1; ++s) {
     if (s + 2 <= r_last) mbar_wait(&bars[wsl], wph);
@@ -1793,8 +1796,9 @@ __device__ __forceinline__ bool advec_y_body(const Chunk& c, const CUtensorMap* 
       fence_proxy_async();
 #endif
       __syncwarp();
-      if (lane == 0 && s - 2 + L::RING <= r_last) issue(s - 2 + L::RING);
+      if (lane == 0 && s - 2 + L::RING <= r_last) issue_at(isl, s - 2 + L::RING);
     }
+    if (++isl == (unsigned)L::RING) isl = 0u;
     Rm2 = Rm1; Rm1 = R0; R0 = Rp1; Rp1 = Rp2;
     if (++wsl == (unsigned)L::RING) { wsl = 0u; wph ^= 1u; }
     Rp2 = ring + wsl * L::SLOT + lane + t0;
