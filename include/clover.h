@@ -202,6 +202,16 @@ int clover_dt_history(clover_ctx* ctx, int32_t first, int32_t n, double* host_ou
  * place the library allocates device memory, a debug/I-O path). */
 int clover_read_field(clover_ctx* ctx, int32_t field_id, double* host, int64_t n);
 
+/* Read a w x h window of a field's global interior, starting at global
+ * 1-based index (j0, k0), into host (row-major, j fastest, w*h doubles);
+ * PRESSURE / SOUNDSPEED are evaluated from the current state as above.  The
+ * window must lie inside the field's interior (nx*ny cells, (nx+1)*(ny+1)
+ * nodes, ...), else CLOVER_ERR_ARG.  Single-process contexts (any number of
+ * local chunks); CLOVER_ERR_STATE for nranks > 1.  Synchronises.  For
+ * inspecting part of a mesh too large to copy whole to the host. */
+int clover_read_field_window(clover_ctx* ctx, int32_t field_id, int32_t j0, int32_t k0, int32_t w,
+                             int32_t h, double* host);
+
 /* Overwrite the global interior of a state field (DENSITY0, ENERGY0, XVEL0,
  * YVEL0) from host memory and refresh its halos. */
 int clover_write_field(clover_ctx* ctx, int32_t field_id, const double* host, int64_t n);

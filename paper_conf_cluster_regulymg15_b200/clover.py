@@ -37,7 +37,7 @@ BUF = {"d0": 0, "e0": 1, "u0": 2, "v0": 3, "q": 4, "d1": 5, "e1": 6, "u1": 7, "v
        "my": 16, "scr": 17}
 EXPORTS = ["clover_workspace_bytes", "clover_nccl_unique_id", "clover_init", "clover_step",
            "clover_step_host", "clover_field_summary", "clover_get_clock", "clover_dt_history",
-           "clover_read_field", "clover_write_field", "clover_sync", "clover_set_graphs",
+           "clover_read_field", "clover_read_field_window", "clover_write_field", "clover_sync", "clover_set_graphs",
            "clover_kernels_per_step", "clover_debug_partial_step", "clover_debug_read_buffer",
            "clover_profile_steps", "clover_profile_name", "clover_debug_div_check",
            "clover_debug_fix_count", "clover_debug_set_fusion",
@@ -112,6 +112,9 @@ def load(build_if_missing: bool = True):
     L.clover_dt_history.argtypes = [c_void_p, c_int32, c_int32, dptr]
     L.clover_read_field.argtypes = [c_void_p, c_int32, dptr, c_int64]
     L.clover_write_field.argtypes = [c_void_p, c_int32, dptr, c_int64]
+    if hasattr(L, "clover_read_field_window"):
+        L.clover_read_field_window.argtypes = [c_void_p, c_int32, c_int32, c_int32, c_int32, c_int32,
+                                               dptr]
     L.clover_sync.argtypes = [c_void_p]
     L.clover_set_graphs.argtypes = [c_void_p, c_int32]
     L.clover_kernels_per_step.argtypes = [c_void_p, P(c_int32)]
@@ -300,6 +303,14 @@ class Clover:
         a = np.zeros(field_shape(name, self.nx, self.ny), dtype=np.float64)
         _check(load().clover_read_field(self._ctx, FIELDS[name], a.ctypes.data_as(dptr), a.size),
                f"clover_read_field({name})")
+        return a
+
+    def read_window(self, name: str, j0: int, k0: int, w: int, h: int) -> np.ndarray:
+        """Rows k0..k0+h-1, columns j0..j0+w-1 (global, 1-based) of a field."""
+        a = np.zeros((h, w), dtype=np.float64)
+        _check(load().clover_read_field_window(self._ctx, FIELDS[name], j0, k0, w, h,
+                                               a.ctypes.data_as(dptr)),
+               f"clover_read_field_window({name})")
         return a
 
     def write(self, name: str, a: np.ndarray):

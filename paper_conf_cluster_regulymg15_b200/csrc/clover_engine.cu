@@ -1891,6 +1891,44 @@ int clover_read_field(clover_ctx* ctx, int32_t field_id, double* host, int64_t n
   return check_err(ctx);
 }
 
+int clover_read_field_window(clover_ctx* ctx, int32_t field_id, int32_t j0, int32_t k0, int32_t w,
+                             int32_t h, double* host) {
+  if (!ctx || !host) return fail(CLOVER_ERR_ARG, "NULL argument");
+  if (ctx->nranks > 1) return fail(CLOVER_ERR_STATE, "windowed read is single-process only");
+  FieldMap m;
+  if (field_map(field_id, &m)) return fail(CLOVER_ERR_ARG, "unknown field id");
+  int ax, ay;
+  const int kind = kBufKind[m.buf];
+  kind_extra(kind, &ax, &ay);
+  const int NXE = ctx->g.x_cells + ax, NYE = ctx->g.y_cells + ay;
+  if (w < 1 || h < 1 || j0 < 1 || k0 < 1 || j0 + w - 1 > NXE || k0 + h - 1 > NYE)
+    return fail(CLOVER_ERR_ARG, "window outside the field's global interior");
+  int rc = join_in(ctx);
+  if (rc) return rc;
+  if (field_id == CLOVER_F_PRESSURE || field_id == CLOVER_F_SOUNDSPEED) {
+    for (auto& cs : ctx->chunks) {
+      k_eos_field<<<cell_grid(cs.c, 32, 8), dim3(32, 8), 0, ctx->work>>>(
+          cs.c, cs.buf[B_D0], cs.buf[B_E0], cs.buf[B_SCR], field_id == CLOVER_F_SOUNDSPEED);
+      LAUNCH_CHECK();
+    }
+  }
+  for (auto& cs : ctx->chunks) {
+    const Chunk& c = cs.c;
+    // owned global range of this chunk for the kind (shared last node/face
+    // only on the global edge), intersected with the window
+    const int cw = c.nx + ((c.gj0 + c.nx == ctx->g.x_cells) ? ax : 0);
+    const int ch = c.ny + ((c.gk0 + c.ny == ctx->g.y_cells) ? ay : 0);
+    const int ja = std::max(j0, c.gj0 + 1), jb = std::min(j0 + w - 1, c.gj0 + cw);
+    const int ka = std::max(k0, c.gk0 + 1), kb = std::min(k0 + h - 1, c.gk0 + ch);
+    if (ja > jb || ka > kb) continue;
+    double* dst = host + (int64_t)(ka - k0) * w + (ja - j0);
+    const double* src = cs.buf[m.buf] + idx(c, ja - c.gj0, ka - c.gk0);
+    CK(cudaMemcpy2DAsync(dst, (size_t)w * 8, src, (size_t)c.pitch * 8, (size_t)(jb - ja + 1) * 8,
+                         kb - ka + 1, cudaMemcpyDeviceToHost, ctx->work));
+  }
+  return check_err(ctx);
+}
+
 int clover_debug_read_buffer(clover_ctx* ctx, int32_t buffer_id, int32_t kind, double* host, int64_t n) {
   if (!ctx || !host) return fail(CLOVER_ERR_ARG, "NULL argument");
   if (buffer_id < 0 || buffer_id >= NBUF) return fail(CLOVER_ERR_ARG, "bad buffer id");

@@ -52,7 +52,7 @@ for spec in specs:
         continue
     env = dict(os.environ, CLOVER_LIB=path)
     out = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--steps", "20", "--warmup", "3",
-                          "--no-cpu-baseline", "--no-e2e", "--no-active"], env=env, capture_output=True, text=True)
+                          "--no-cpu-baseline", "--no-e2e", "--no-active", "--no-full"], env=env, capture_output=True, text=True)
     try:
         d = json.loads(out.stdout.strip().splitlines()[-1])
     except Exception:

@@ -538,6 +538,57 @@ def test_full_size_first_steps(torch_cuda, n, steps):
     assert_summary_close(g.field_summary(), o.field_summary(compensated=True))
 
 
+def test_read_field_window_matches_full_read(torch_cuda):
+    """clover_read_field_window == the same window of clover_read_field, on
+    local chunks (the window spans chunk boundaries) for every field kind."""
+    deck = fuzz_deck(5, nx=70, ny=52)
+    g = make_gpu(deck, px=2, py=3)
+    g.step(3)
+    for f in ("density0", "pressure", "xvel0", "yvel0", "vol_flux_x", "vol_flux_y"):
+        full = g.read(f)
+        for j0, k0, w, h in ((1, 1, 5, 7), (30, 12, 20, 25), (1, 1, full.shape[1], full.shape[0])):
+            a = g.read_window(f, j0, k0, w, h)
+            assert np.array_equal(a, full[k0 - 1:k0 - 1 + h, j0 - 1:j0 - 1 + w]), (f, j0, k0)
+    from paper_conf_cluster_regulymg15_b200 import CloverError
+    with pytest.raises(CloverError):
+        g.read_window("density0", 60, 1, 20, 5)  # past nx = 70
+
+
+def test_maximum_size_corner_window_bitwise(torch_cuda):
+    """Maximum sizes (one chunk of 20480^2 = 419 M cells, 61 GB of fields):
+    a blast in the corner of a huge mesh evolves bit for bit like the same
+    blast on a small mesh with the same cell size (dx = 10/20480 = 2^-11, so
+    the 256-cell domain [0, 0.125]^2 has exactly the same geometry), for as
+    long as nothing from the small mesh's far walls can have reached the
+    window: one step's stencil reaches < 8 cells, so after 10 steps the
+    cells below 128 are untouched by walls 256 cells away.  dt is set by the
+    blast on both (the quiescent far field has a smaller sound speed), so the
+    dt histories are bitwise equal too.  The oracle runs the small mesh."""
+    from workloads import _state
+    n_big, n_small, steps = 20480, 256, 10
+    dx = 10.0 / n_big
+    assert dx == 2.0 ** -11
+    blast = _state(1.0, 2.5, geometry="rectangle", xmin=0.0, xmax=64 * dx, ymin=0.0, ymax=32 * dx)
+    big = bm_deck(n_big)
+    big["states"] = [_state(0.2, 1.0), blast]
+    small = bm_deck(n_small, xmax=n_small * dx, ymax=n_small * dx)
+    small["states"] = [_state(0.2, 1.0), dict(blast)]
+    g = make_gpu(big)
+    g.step(steps)
+    o = Oracle(small)
+    dts = o.step(steps)
+    assert np.array_equal(g.dt_history(1, steps), dts)
+    w = 128
+    for f in STATE:
+        a = g.read_window(f, 1, 1, w, w)
+        b = o.read(f)[:w, :w]
+        assert np.array_equal(a, b), (f, rel_cell(a, b))
+    # and the far field is exactly the untouched background
+    far = g.read_window("density0", n_big - 63, n_big - 63, 64, 64)
+    assert np.all(far == 0.2)
+    g.close()
+
+
 @pytest.mark.parametrize("pxy,expected", [((1, 1), 8), ((3, 1), 28), ((1, 3), 27)])
 def test_kernels_per_step(torch_cuda, pxy, expected):
     """Launches per step (bench.py's gpu_launches): one chunk runs visc_dt,
