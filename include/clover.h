@@ -254,6 +254,14 @@ int clover_debug_partial_step(clover_ctx* ctx, int32_t nkernels);
 int clover_debug_read_buffer(clover_ctx* ctx, int32_t buffer_id, int32_t kind,
                              double* host, int64_t n);
 
+/* Boundary-first overlap (S:8(e)): for y-strip layouts (px == 1) whose
+ * exchanges take the remote path (several ranks, or virtual-remote mode),
+ * each fused kernel runs the row segments next to a y chunk boundary first,
+ * then the halo exchange on a second stream while the interior segments run;
+ * the next kernel waits for both.  enable = 1 (default) / 0.  Results are
+ * bitwise identical either way; tests compare them. */
+int clover_debug_set_overlap(clover_ctx* ctx, int32_t enable);
+
 /* Debug: the fused advection sweeps (advec_cell + advec_mom of one
  * direction in one pass).  enable = 1 (default): fused x sweep where every
  * local chunk has reflective walls on both x sides, fused y sweep everywhere

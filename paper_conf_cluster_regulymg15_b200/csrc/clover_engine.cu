@@ -246,6 +246,11 @@ struct clover_ctx {
   std::vector<ChunkState> chunks;  // local chunks
   std::vector<int> owner;          // chunk id -> rank
   cudaStream_t user = nullptr, work = nullptr;
+  // halo exchanges run on `xs`: the work stream, or -- boundary segments
+  // first, the interior overlapped with the exchange -- the comm stream
+  cudaStream_t comm_stream = nullptr, xs = nullptr;
+  cudaEvent_t ev_b = nullptr, ev_x = nullptr;
+  bool overlap = false;  // see overlap_ok
   cudaEvent_t ev_in = nullptr, ev_out = nullptr;
   StepScalars* scal = nullptr;
   double* hist = nullptr;
@@ -476,7 +481,7 @@ int StripQueue::flush() {
   if (b.n == 0) return CLOVER_OK;
   const long long total = b.start[b.n];
   const int blocks = (int)std::min<long long>((total + 255) / 256, 148 * 8);
-  k_copy_strips<<<blocks, 256, 0, ctx->work>>>(b);
+  k_copy_strips<<<blocks, 256, 0, ctx->xs>>>(b);
   CK(cudaGetLastError());
   b.n = 0;
   b.start[0] = 0;
@@ -551,8 +556,8 @@ int exchange_axis(clover_ctx* ctx, const std::vector<int>& bufs, int axis, int y
         for (auto& pm : msgs)
           if (pm.cs->id == m.nb && pm.side == (m.side ^ 1)) partner = &pm;
         if (!partner || partner->n != m.n) return fail(CLOVER_ERR_STATE, "virtual remote: unmatched message");
-        NK(ncclSend(ctx->xbuf_send + m.off, (size_t)m.n, ncclFloat64, 0, ctx->comm, ctx->work));
-        NK(ncclRecv(ctx->xbuf_recv + partner->off, (size_t)m.n, ncclFloat64, 0, ctx->comm, ctx->work));
+        NK(ncclSend(ctx->xbuf_send + m.off, (size_t)m.n, ncclFloat64, 0, ctx->comm, ctx->xs));
+        NK(ncclRecv(ctx->xbuf_recv + partner->off, (size_t)m.n, ncclFloat64, 0, ctx->comm, ctx->xs));
       }
       NK(ncclGroupEnd());
 #else
@@ -572,8 +577,8 @@ int exchange_axis(clover_ctx* ctx, const std::vector<int>& bufs, int axis, int y
     } else if (ctx->use_ht) {
       // host transport: staging to host, the caller's sendrecv, back
       std::vector<double> hs((size_t)off), hr((size_t)off);
-      CK(cudaMemcpyAsync(hs.data(), ctx->xbuf_send, (size_t)off * 8, cudaMemcpyDeviceToHost, ctx->work));
-      CK(cudaStreamSynchronize(ctx->work));
+      CK(cudaMemcpyAsync(hs.data(), ctx->xbuf_send, (size_t)off * 8, cudaMemcpyDeviceToHost, ctx->xs));
+      CK(cudaStreamSynchronize(ctx->xs));
       std::vector<int32_t> peer;
       std::vector<const double*> sp;
       std::vector<double*> rp;
@@ -587,14 +592,14 @@ int exchange_axis(clover_ctx* ctx, const std::vector<int>& bufs, int axis, int y
       if (ctx->ht.sendrecv(ctx->ht.user, (int32_t)msgs.size(), peer.data(), sp.data(), cnt.data(),
                            rp.data(), cnt.data()) != 0)
         return fail(CLOVER_ERR_NCCL, "host transport sendrecv failed");
-      CK(cudaMemcpyAsync(ctx->xbuf_recv, hr.data(), (size_t)off * 8, cudaMemcpyHostToDevice, ctx->work));
-      CK(cudaStreamSynchronize(ctx->work));
+      CK(cudaMemcpyAsync(ctx->xbuf_recv, hr.data(), (size_t)off * 8, cudaMemcpyHostToDevice, ctx->xs));
+      CK(cudaStreamSynchronize(ctx->xs));
     } else {
 #ifdef CLOVER_WITH_NCCL
       NK(ncclGroupStart());
       for (auto& m : msgs) {
-        NK(ncclSend(ctx->xbuf_send + m.off, (size_t)m.n, ncclFloat64, m.peer, ctx->comm, ctx->work));
-        NK(ncclRecv(ctx->xbuf_recv + m.off, (size_t)m.n, ncclFloat64, m.peer, ctx->comm, ctx->work));
+        NK(ncclSend(ctx->xbuf_send + m.off, (size_t)m.n, ncclFloat64, m.peer, ctx->comm, ctx->xs));
+        NK(ncclRecv(ctx->xbuf_recv + m.off, (size_t)m.n, ncclFloat64, m.peer, ctx->comm, ctx->xs));
       }
       NK(ncclGroupEnd());
 #else
@@ -735,6 +740,42 @@ bool fuse_y_ok(const clover_ctx* ctx) {
   return true;
 }
 
+// ---------------------------------------------------------------- overlap
+// Boundary segments first, the exchange overlapped with the interior
+// (S:8(e) "boundary-strip-first + interior overlap"): for y-strip layouts
+// (px == 1; x strips would need every row) whose exchanges leave the GPU
+// (several ranks over NCCL) or take the remote path in virtual-remote mode.
+// The host transport is synchronous, so it gains nothing there.
+bool overlap_ok(const clover_ctx* ctx) {
+  return ctx->overlap && ctx->L.px == 1 && ctx->L.py > 1 && !ctx->use_ht &&
+         (ctx->nranks > 1 || ctx->virtual_remote);
+}
+
+// Row-segment geometry of a streaming kernel kind on a chunk: rows per
+// segment, full-height segments, rows covered (seg_rows_of).
+enum { SEG_LAGR, SEG_X, SEG_Y };
+void seg_geom(const Chunk& c, int kind, int* ks, int* nb, int* rows) {
+  if (kind == SEG_LAGR) { *ks = c.lks; *nb = c.lnb; *rows = c.ny; }
+  else if (kind == SEG_X) { *ks = c.xks; *nb = c.xnb; *rows = c.ny + 1; }
+  else { *ks = c.yks; *nb = c.ynb; *rows = c.ny + 1; }
+}
+// the segment holding row r (1-based), inverse of seg_rows_of
+int seg_of_row(int r, int ks, int nb) {
+  if (r < 1) r = 1;
+  if ((int64_t)(r - 1) < (int64_t)nb * ks) return (r - 1) / ks;
+  return nb + (int)(((int64_t)(r - 1) - (int64_t)nb * ks) / (ks / CLOVER_TAIL_DIV));
+}
+// Boundary / interior split of a chunk's segments [0, n) for an exchange of
+// depth yd: [0, lo) holds the rows sent to the neighbour below (1 .. yd+1),
+// [hi, n) those sent up (ny+1-yd .. ny); [lo, hi) is the interior.
+void phase_ranges(const Chunk& c, int kind, int yd, int* lo, int* hi, int* n) {
+  int ks, nb, rows;
+  seg_geom(c, kind, &ks, &nb, &rows);
+  *n = seg_count(ks, nb, rows);
+  *lo = c.wb ? 0 : std::min(*n, seg_of_row(yd + 1, ks, nb) + 1);
+  *hi = c.wt ? *n : std::min(*n, std::max(*lo, seg_of_row(std::max(1, c.ny + 1 - yd), ks, nb)));
+}
+
 // Enqueue kernel phases [0, nphase) of one step (7 = full step).
 // Serpentine segment order: each step kernel reads what the previous one
 // wrote, so alternate kernels run their row segments top-down (seg_y) and
@@ -779,6 +820,57 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
   // one chunk on one rank: the visc fixup's last block finalises dt (no
   // k_dt_finalize launch); else the slot is combined first (NCCL MIN)
   const int fold_fin = (nphase >= 2 && ctx->chunks.size() == 1 && ctx->nranks == 1) ? 1 : 0;
+  // A streaming kernel on every chunk, then the exchange of `bufs`.
+  // launch(cs, c, n) runs the kernel over row segments [c.seg0, c.seg0+n),
+  // fixup(cs, c) its IEEE fixup.  With overlap_ok the segments next to a y
+  // chunk boundary (the rows the exchange sends) run first, then the
+  // exchange on the comm stream while the interior segments run on the work
+  // stream; the next phase waits for both.
+  auto run_phase = [&](int kind, auto&& launch, auto&& fixup, const std::vector<int>& bufs, int yd,
+                       int xd) -> int {
+    if (!overlap_ok(ctx)) {
+      for (auto& cs : ctx->chunks) {
+        int lo, hi, n;
+        phase_ranges(cs.c, kind, yd, &lo, &hi, &n);
+        Chunk c = cs.c;
+        c.seg0 = 0;
+        int rc = launch(cs, c, n);
+        if (!rc) rc = fixup(cs, c);
+        if (rc) return rc;
+      }
+      return exchange(ctx, bufs, yd, xd);
+    }
+    std::vector<int> ilo(ctx->chunks.size()), ihi(ctx->chunks.size());
+    for (size_t t = 0; t < ctx->chunks.size(); ++t) {
+      auto& cs = ctx->chunks[t];
+      int n;
+      phase_ranges(cs.c, kind, yd, &ilo[t], &ihi[t], &n);
+      Chunk c = cs.c;
+      int rc = 0;
+      if (ilo[t] > 0) { c.seg0 = 0; rc = launch(cs, c, ilo[t]); }
+      if (!rc && ihi[t] < n) { c.seg0 = ihi[t]; rc = launch(cs, c, n - ihi[t]); }
+      if (!rc) rc = fixup(cs, c);
+      if (rc) return rc;
+    }
+    CK(cudaEventRecord(ctx->ev_b, ctx->work));
+    CK(cudaStreamWaitEvent(ctx->comm_stream, ctx->ev_b, 0));
+    ctx->xs = ctx->comm_stream;
+    int rc = exchange(ctx, bufs, yd, xd);
+    ctx->xs = ctx->work;
+    if (rc) return rc;
+    CK(cudaEventRecord(ctx->ev_x, ctx->comm_stream));
+    for (size_t t = 0; t < ctx->chunks.size(); ++t) {
+      if (ilo[t] >= ihi[t]) continue;
+      auto& cs = ctx->chunks[t];
+      Chunk c = cs.c;
+      c.seg0 = ilo[t];
+      rc = launch(cs, c, ihi[t] - ilo[t]);
+      if (!rc) rc = fixup(cs, c);
+      if (rc) return rc;
+    }
+    CK(cudaStreamWaitEvent(ctx->work, ctx->ev_x, 0));
+    return CLOVER_OK;
+  };
   if (nphase >= 1) {
     for (auto& cs : ctx->chunks) {
       const Chunk c = with_rev(cs.c, CLOVER_SERP);  // top-down: sweep 2 wrote these rows last
@@ -820,21 +912,26 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
   }
   if (nphase >= 3) {
     cur_prof_id = P_LAGR;
-    for (auto& cs : ctx->chunks) {
-      const Chunk c = with_rev(cs.c, 0);
-      launch_step(ks_lagrangian, dim3(grid_strip(c.nx, LW, c.ny, c.lks).x, seg_count(c.lks, c.lnb, c.ny)), SB, st, c, cs.tm_lag,
+    auto launch = [&](ChunkState& cs, Chunk c, int n) -> int {
+      c = with_rev(c, 0);
+      launch_step(ks_lagrangian, dim3(grid_strip(c.nx, LW, c.ny, c.lks).x, n), SB, st, c, cs.tm_lag,
           cs.buf[B_D1], cs.buf[B_E1], cs.buf[B_U1], cs.buf[B_V1], cs.buf[B_FX], cs.buf[B_FY],
           ctx->scal, cs.fix);
       STEP_LAUNCH_CHECK();
+      return CLOVER_OK;
+    };
+    auto fixup = [&](ChunkState& cs, Chunk c) -> int {
+      c = with_rev(c, 0);
       const YWalls yw = walls_in_lagr ? ywalls_of(cs, 1) : kNoWalls;
       launch_fix(kf_lagrangian, FIX_BLOCKS + 5 * yw.nbx, SB, st, c, cs.tm_lag,
           cs.buf[B_D1], cs.buf[B_E1], cs.buf[B_U1], cs.buf[B_V1], cs.buf[B_FX], cs.buf[B_FY],
           ctx->scal, cs.fix, yw);
       FIX_LAUNCH_CHECK();
-    }
+      return CLOVER_OK;
+    };
     // a fused y sweep (either sweep) reads these HALO_ROWS deep in y
-    int rc = exchange(ctx, {B_D1, B_E1, B_U1, B_V1, B_FX, B_FY}, fuse_y_ok(ctx) ? HALO_ROWS : HALO,
-                      fuse_x_ok(ctx) ? HALO_COLS : HALO);
+    int rc = run_phase(SEG_LAGR, launch, fixup, {B_D1, B_E1, B_U1, B_V1, B_FX, B_FY},
+                       fuse_y_ok(ctx) ? HALO_ROWS : HALO, fuse_x_ok(ctx) ? HALO_COLS : HALO);
     if (rc) return rc;
     if (ctx->prof) prof_mark(ctx, -1);
   }
@@ -852,29 +949,35 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
       // runs both, phase ph_cell + 1 is empty
       if (nphase >= ph_cell) {
         cur_prof_id = sweep == 1 ? P_ADV_X1 : P_ADV_X2;
-        for (auto& cs : ctx->chunks) {
-          const Chunk c = with_rev(cs.c, sweep == 1 ? CLOVER_SERP : 0);
-          const dim3 g(grid_strip(c.nx + 1, XW, c.ny + 1, c.xks).x, seg_count(c.xks, c.xnb, c.ny + 1));
-          if (sweep == 1) {
+        const int serp = sweep == 1 ? CLOVER_SERP : 0;
+        auto launch = [&](ChunkState& cs, Chunk c, int n) -> int {
+          c = with_rev(c, serp);
+          const dim3 g(grid_strip(c.nx + 1, XW, c.ny + 1, c.xks).x, n);
+          if (sweep == 1)
             launch_step(ks_advec_x<1>, g, SB, st, c, cs.tm_x1, cs.buf[rout], cs.buf[eout],
                         cs.buf[uout], cs.buf[vout], cs.fix);
-            STEP_LAUNCH_CHECK();
+          else
+            launch_step(ks_advec_x<2>, g, SB, st, c, cs.tm_x2, cs.buf[rout], cs.buf[eout],
+                        cs.buf[uout], cs.buf[vout], cs.fix);
+          STEP_LAUNCH_CHECK();
+          return CLOVER_OK;
+        };
+        auto fixup = [&](ChunkState& cs, Chunk c) -> int {
+          c = with_rev(c, serp);
+          if (sweep == 1) {
             const YWalls yw = walls_in_x1 ? ywalls_of(cs, 2) : kNoWalls;
             launch_fix(kf_advec_x<1>, FIX_BLOCKS + 5 * yw.nbx, SB, st, c, cs.tm_x1, cs.buf[rout],
                         cs.buf[eout], cs.buf[uout], cs.buf[vout], cs.fix, yw);
-            FIX_LAUNCH_CHECK();
           } else {
-            launch_step(ks_advec_x<2>, g, SB, st, c, cs.tm_x2, cs.buf[rout], cs.buf[eout],
-                        cs.buf[uout], cs.buf[vout], cs.fix);
-            STEP_LAUNCH_CHECK();
             launch_fix(kf_advec_x<2>, FIX_BLOCKS, SB, st, c, cs.tm_x2, cs.buf[rout], cs.buf[eout],
                         cs.buf[uout], cs.buf[vout], cs.fix, kNoWalls);
-            FIX_LAUNCH_CHECK();
           }
-        }
+          FIX_LAUNCH_CHECK();
+          return CLOVER_OK;
+        };
         // sweep 1 feeds a fused y sweep 2: HALO_ROWS deep in y
-        int rc = exchange(ctx, {rout, eout, uout, vout},
-                          (sweep == 1 && fuse_y_ok(ctx)) ? HALO_ROWS : HALO);
+        int rc = run_phase(SEG_X, launch, fixup, {rout, eout, uout, vout},
+                           (sweep == 1 && fuse_y_ok(ctx)) ? HALO_ROWS : HALO, HALO);
         if (rc) return rc;
         if (ctx->prof) prof_mark(ctx, -1);
       }
@@ -899,20 +1002,17 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
             launch_step(ks_cell_y_walls<2>, gw, SB, st, c, yw);
           FIX_LAUNCH_CHECK();
         }
-        for (auto& cs : ctx->chunks) {
-          const Chunk c = with_rev(cs.c, sweep == 1 ? CLOVER_SERP : 0);
-          const dim3 g(grid_strip(c.nx + 1, YW, c.ny + 1, c.yks).x, seg_count(c.yks, c.ynb, c.ny + 1));
+        const int serp = sweep == 1 ? CLOVER_SERP : 0;
+        auto launch = [&](ChunkState& cs, Chunk c, int n) -> int {
+          c = with_rev(c, serp);
+          const dim3 g(grid_strip(c.nx + 1, YW, c.ny + 1, c.yks).x, n);
           const CUtensorMap& ta = sweep == 1 ? cs.tm_x1 : cs.tm_fy;
           const CUtensorMap& tb = sweep == 1 ? cs.tm_x1 : cs.tm_c4;
           if (sweep == 1) {
             launch_step(ks_advec_y<1>, g, SB, st, c, ta, tb, cs.buf[rout], cs.buf[eout], cs.buf[B_MY],
                         cs.buf[uout], cs.buf[vout], cs.fix);
-            STEP_LAUNCH_CHECK();
-            launch_fix(kf_advec_y<1>, FIX_BLOCKS, SB, st, c, ta, tb, cs.buf[rout], cs.buf[eout],
-                        cs.buf[B_MY], cs.buf[uout], cs.buf[vout], cs.fix);
-            FIX_LAUNCH_CHECK();
           } else if (ctx->f2_probe) {
-            // DESIGN.md 9 f2 probe: sweep 2 with the next step's viscosity
+            // DESIGN.md 4.5 f2 probe: sweep 2 with the next step's viscosity
             // and calc_dt terms folded in (q written, dt to a scratch slot;
             // visc_dt still runs, so results are unchanged)
             ViscProbe vp;
@@ -921,22 +1021,29 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
             vp.prm = ctx->dtp;
             launch_step(ks_advec_y2_probe, g, SB, st, c, ta, tb, cs.buf[rout], cs.buf[eout],
                         cs.buf[B_MY], cs.buf[uout], cs.buf[vout], cs.fix, vp);
-            STEP_LAUNCH_CHECK();
-            launch_fix(kf_advec_y<2>, FIX_BLOCKS, SB, st, c, ta, tb, cs.buf[rout], cs.buf[eout],
-                        cs.buf[B_MY], cs.buf[uout], cs.buf[vout], cs.fix);
-            FIX_LAUNCH_CHECK();
           } else {
             launch_step(ks_advec_y<2>, g, SB, st, c, ta, tb, cs.buf[rout], cs.buf[eout], cs.buf[B_MY],
                         cs.buf[uout], cs.buf[vout], cs.fix);
-            STEP_LAUNCH_CHECK();
+          }
+          STEP_LAUNCH_CHECK();
+          return CLOVER_OK;
+        };
+        auto fixup = [&](ChunkState& cs, Chunk c) -> int {
+          c = with_rev(c, serp);
+          const CUtensorMap& ta = sweep == 1 ? cs.tm_x1 : cs.tm_fy;
+          const CUtensorMap& tb = sweep == 1 ? cs.tm_x1 : cs.tm_c4;
+          if (sweep == 1)
+            launch_fix(kf_advec_y<1>, FIX_BLOCKS, SB, st, c, ta, tb, cs.buf[rout], cs.buf[eout],
+                        cs.buf[B_MY], cs.buf[uout], cs.buf[vout], cs.fix);
+          else
             launch_fix(kf_advec_y<2>, FIX_BLOCKS, SB, st, c, ta, tb, cs.buf[rout], cs.buf[eout],
                         cs.buf[B_MY], cs.buf[uout], cs.buf[vout], cs.fix);
-            FIX_LAUNCH_CHECK();
-          }
-        }
+          FIX_LAUNCH_CHECK();
+          return CLOVER_OK;
+        };
         // y sweep 1 feeds a fused x sweep 2: HALO_COLS deep in x
-        int rc = exchange(ctx, {rout, eout, uout, vout}, HALO,
-                          (sweep == 1 && fuse_x_ok(ctx)) ? HALO_COLS : HALO);
+        int rc = run_phase(SEG_Y, launch, fixup, {rout, eout, uout, vout}, HALO,
+                           (sweep == 1 && fuse_x_ok(ctx)) ? HALO_COLS : HALO);
         if (rc) return rc;
         if (ctx->prof) prof_mark(ctx, -1);
       }
@@ -1359,11 +1466,16 @@ int clover_init(const clover_grid* grid, const clover_state* states, int32_t nst
   ctx->gg = GlobalGeom{ctx->g.x_cells, ctx->g.y_cells, ctx->g.xmin, ctx->g.ymin, dx, dy};
 
   auto bail = [&](int code) { clover_finalize(ctx); return code; };
+  ctx->overlap = true;  // used where overlap_ok
   if (cudaStreamCreateWithFlags(&ctx->work, cudaStreamNonBlocking) != cudaSuccess ||
+      cudaStreamCreateWithFlags(&ctx->comm_stream, cudaStreamNonBlocking) != cudaSuccess ||
+      cudaEventCreateWithFlags(&ctx->ev_b, cudaEventDisableTiming) != cudaSuccess ||
+      cudaEventCreateWithFlags(&ctx->ev_x, cudaEventDisableTiming) != cudaSuccess ||
       cudaEventCreateWithFlags(&ctx->ev_in, cudaEventDisableTiming) != cudaSuccess ||
       cudaEventCreateWithFlags(&ctx->ev_out, cudaEventDisableTiming) != cudaSuccess)
     return bail(fail(CLOVER_ERR_CUDA, "stream/event creation failed"));
 
+  ctx->xs = ctx->work;
   // carve the workspace
   char* p = (char*)workspace;
   ctx->scal = (StepScalars*)p;
@@ -1386,6 +1498,7 @@ int clover_init(const clover_grid* grid, const clover_state* states, int32_t nst
     c.wl = cs.cx == 0; c.wr = cs.cx == px - 1; c.wb = cs.cy == 0; c.wt = cs.cy == py - 1;
     c.face_cc = ctx->g.face_mirror == CLOVER_MIRROR_CELLCENTRE;
     c.rev = 0;
+    c.seg0 = 0;
     c.vks = seg_rows(VKS, grid_cols(c.nx, c.ny, VKS).x, c.ny);
     c.lks = seg_rows(LKS, grid_strip(c.nx, LW, c.ny, LKS).x, c.ny);
     c.xks = seg_rows(XKS, grid_strip(c.nx + 1, XW, c.ny + 1, XKS).x, c.ny + 1);
@@ -1563,6 +1676,17 @@ int clover_debug_set_virtual_remote(clover_ctx* ctx, int32_t enable) {
   return CLOVER_OK;
 }
 
+int clover_debug_set_overlap(clover_ctx* ctx, int32_t enable) {
+  if (!ctx) return fail(CLOVER_ERR_ARG, "ctx is NULL");
+  ctx->overlap = enable != 0;
+  for (int i = 0; i < 4; ++i)
+    if (ctx->gexec[i]) {
+      cudaGraphExecDestroy(ctx->gexec[i]);
+      ctx->gexec[i] = nullptr;
+    }
+  return CLOVER_OK;
+}
+
 int clover_debug_set_fusion(clover_ctx* ctx, int32_t enable) {
   if (!ctx) return fail(CLOVER_ERR_ARG, "ctx is NULL");
   if (enable < 0 || enable > 2) return fail(CLOVER_ERR_ARG, "enable must be 0, 1 or 2");
@@ -1607,6 +1731,22 @@ int clover_kernels_per_step(clover_ctx* ctx, int32_t* out) {
   for (const auto& cs : ctx->chunks) {
     const int y = fuse_y_ok(ctx) ? (2 + ((!folded && (cs.c.wb || cs.c.wt)) ? 1 : 0)) : 4;
     n += 4 + x + y;
+    if (overlap_ok(ctx)) {
+      // boundary ranges + interior as separate launches, a fixup after each
+      // part (run_phase); for the current sweep order
+      auto extra = [&](int kind, int yd) {
+        int lo, hi, ns;
+        phase_ranges(cs.c, kind, yd, &lo, &hi, &ns);
+        return (lo > 0) + (hi < ns) + 2 * (lo < hi) - 1;
+      };
+      const bool ax = ctx->advect_x;
+      n += extra(SEG_LAGR, fuse_y_ok(ctx) ? HALO_ROWS : HALO);
+      for (int sweep = 1; sweep <= 2; ++sweep) {
+        const bool xdir = (sweep == 1) ? ax : !ax;
+        if (xdir && fuse_x_ok(ctx)) n += extra(SEG_X, (sweep == 1 && fuse_y_ok(ctx)) ? HALO_ROWS : HALO);
+        if (!xdir && fuse_y_ok(ctx)) n += extra(SEG_Y, HALO);
+      }
+    }
   }
   *out = (int32_t)n;
   return CLOVER_OK;
@@ -2094,6 +2234,9 @@ int clover_finalize(clover_ctx* ctx) {
   if (ctx->comm) ncclCommDestroy(ctx->comm);
 #endif
   if (ctx->ev_in) cudaEventDestroy(ctx->ev_in);
+  if (ctx->ev_b) cudaEventDestroy(ctx->ev_b);
+  if (ctx->ev_x) cudaEventDestroy(ctx->ev_x);
+  if (ctx->comm_stream) cudaStreamDestroy(ctx->comm_stream);
   if (ctx->ev_out) cudaEventDestroy(ctx->ev_out);
   if (ctx->work) cudaStreamDestroy(ctx->work);
   delete ctx;

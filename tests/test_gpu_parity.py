@@ -383,6 +383,33 @@ def test_virtual_remote_through_nccl_bitwise(torch_cuda, pxy):
     assert many.field_summary() == one.field_summary()
 
 
+@pytest.mark.parametrize("nccl", [False, True])
+@pytest.mark.parametrize("py", [2, 3, 5])
+def test_boundary_first_overlap_bitwise(torch_cuda, nccl, py):
+    """S:8(e) boundary-strip-first + interior overlap: with y strips whose
+    exchanges take the remote path, each fused kernel runs the segments next
+    to a chunk boundary first, then the exchange (device copy or one-rank
+    NCCL) on a second stream while the interior segments run.  Same bits as
+    without the overlap and as one chunk (fields, dt history), both sweep
+    orders, graphs on; more launches per step than without."""
+    deck = fuzz_deck(16, nx=64, ny=40 * py)
+    deck["max_timestep"] = 1.0
+    one = make_gpu(deck)
+    ov = make_gpu(deck, px=1, py=py)
+    ov.debug_set_virtual_remote(True, nccl=nccl)
+    plain = make_gpu(deck, px=1, py=py)
+    plain.debug_set_virtual_remote(True, nccl=nccl)
+    plain.debug_set_overlap(False)
+    assert ov.kernels_per_step() > plain.kernels_per_step()
+    for g in (one, ov, plain):
+        g.step(9)
+    for f in STATE:
+        a = one.read(f)
+        assert np.array_equal(ov.read(f), a), f
+        assert np.array_equal(plain.read(f), a), f
+    assert np.array_equal(ov.dt_history(1, 9), one.dt_history(1, 9))
+
+
 @pytest.mark.parametrize("seed,pxy", [(8, (1, 2)), (9, (1, 4)), (10, (2, 3)), (11, (1, 5)),
                                       (12, (2, 1)), (13, (3, 1)), (14, (4, 2)), (15, (3, 3))])
 def test_fused_sweeps_across_chunk_boundaries(torch_cuda, seed, pxy):
