@@ -102,6 +102,7 @@ struct ChunkState {
   double* partials;  // summary partials, ntx*nty*5
   int ntx, nty;
   FixSlot fix;       // warps to redo with IEEE division (clover_stream.cuh)
+  FixSlot fix_b;     // the same for boundary segments running beside the interior (run_phase)
   CUtensorMap tm_lag;   // d0 e0 u0 v0 q as one {pitch, rows, 5} fp64 tensor, box {LRW, 1, 5}
   CUtensorMap tm_visc;  // d0 e0 u0 v0 as {pitch, rows, 4}, box {VRW, 1, 4}
   CUtensorMap tm_x1;    // d1 e1 u1 v1 fy fx, box {XRW, 1, 6} (fused x sweep 1)
@@ -344,7 +345,7 @@ int64_t compute_workspace(const clover_grid* g, int px, int py, int rank, int nr
     bytes += NBUF * align_up(fe * 8, kAlign);
     int ntx = (nx + ST - 1) / ST, nty = (ny + ST - 1) / ST;
     bytes += align_up((int64_t)ntx * nty * 5 * 8, kAlign);
-    bytes += fix_bytes(nx, ny);
+    bytes += 2 * fix_bytes(nx, ny);
     maxrows = std::max<int64_t>(maxrows, ny + 2 + 2 * HALO_ROWS);
     maxcols = std::max<int64_t>(maxcols, nx + 2 + 2 * HALO_COLS);
   }
@@ -821,11 +822,13 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
   // k_dt_finalize launch); else the slot is combined first (NCCL MIN)
   const int fold_fin = (nphase >= 2 && ctx->chunks.size() == 1 && ctx->nranks == 1) ? 1 : 0;
   // A streaming kernel on every chunk, then the exchange of `bufs`.
-  // launch(cs, c, n) runs the kernel over row segments [c.seg0, c.seg0+n),
-  // fixup(cs, c) its IEEE fixup.  With overlap_ok the segments next to a y
-  // chunk boundary (the rows the exchange sends) run first, then the
-  // exchange on the comm stream while the interior segments run on the work
-  // stream; the next phase waits for both.
+  // launch(cs, c, n, stream, fix) runs the kernel over row segments
+  // [c.seg0, c.seg0+n) on `stream`, pushing IEEE redos to `fix`;
+  // fixup(cs, c, stream, fix) is its IEEE fixup.  With overlap_ok the
+  // segments next to a y chunk boundary (the rows the exchange sends) run on
+  // the comm stream, followed there by their fixup and the exchange, while
+  // the interior segments run beside them on the work stream (own fix list);
+  // the next phase waits for both.
   auto run_phase = [&](int kind, auto&& launch, auto&& fixup, const std::vector<int>& bufs, int yd,
                        int xd) -> int {
     if (!overlap_ok(ctx)) {
@@ -834,12 +837,15 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
         phase_ranges(cs.c, kind, yd, &lo, &hi, &n);
         Chunk c = cs.c;
         c.seg0 = 0;
-        int rc = launch(cs, c, n);
-        if (!rc) rc = fixup(cs, c);
+        int rc = launch(cs, c, n, st, cs.fix);
+        if (!rc) rc = fixup(cs, c, st, cs.fix);
         if (rc) return rc;
       }
       return exchange(ctx, bufs, yd, xd);
     }
+    cudaStream_t cm = ctx->comm_stream;
+    CK(cudaEventRecord(ctx->ev_b, st));  // the previous phase is complete on st
+    CK(cudaStreamWaitEvent(cm, ctx->ev_b, 0));
     std::vector<int> ilo(ctx->chunks.size()), ihi(ctx->chunks.size());
     for (size_t t = 0; t < ctx->chunks.size(); ++t) {
       auto& cs = ctx->chunks[t];
@@ -847,28 +853,27 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
       phase_ranges(cs.c, kind, yd, &ilo[t], &ihi[t], &n);
       Chunk c = cs.c;
       int rc = 0;
-      if (ilo[t] > 0) { c.seg0 = 0; rc = launch(cs, c, ilo[t]); }
-      if (!rc && ihi[t] < n) { c.seg0 = ihi[t]; rc = launch(cs, c, n - ihi[t]); }
-      if (!rc) rc = fixup(cs, c);
+      bool any = false;
+      if (ilo[t] > 0) { c.seg0 = 0; rc = launch(cs, c, ilo[t], cm, cs.fix_b); any = true; }
+      if (!rc && ihi[t] < n) { c.seg0 = ihi[t]; rc = launch(cs, c, n - ihi[t], cm, cs.fix_b); any = true; }
+      if (!rc && any) rc = fixup(cs, c, cm, cs.fix_b);
       if (rc) return rc;
     }
-    CK(cudaEventRecord(ctx->ev_b, ctx->work));
-    CK(cudaStreamWaitEvent(ctx->comm_stream, ctx->ev_b, 0));
-    ctx->xs = ctx->comm_stream;
+    ctx->xs = cm;
     int rc = exchange(ctx, bufs, yd, xd);
     ctx->xs = ctx->work;
     if (rc) return rc;
-    CK(cudaEventRecord(ctx->ev_x, ctx->comm_stream));
+    CK(cudaEventRecord(ctx->ev_x, cm));
     for (size_t t = 0; t < ctx->chunks.size(); ++t) {
       if (ilo[t] >= ihi[t]) continue;
       auto& cs = ctx->chunks[t];
       Chunk c = cs.c;
       c.seg0 = ilo[t];
-      rc = launch(cs, c, ihi[t] - ilo[t]);
-      if (!rc) rc = fixup(cs, c);
+      rc = launch(cs, c, ihi[t] - ilo[t], st, cs.fix);
+      if (!rc) rc = fixup(cs, c, st, cs.fix);
       if (rc) return rc;
     }
-    CK(cudaStreamWaitEvent(ctx->work, ctx->ev_x, 0));
+    CK(cudaStreamWaitEvent(st, ctx->ev_x, 0));
     return CLOVER_OK;
   };
   if (nphase >= 1) {
@@ -912,20 +917,20 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
   }
   if (nphase >= 3) {
     cur_prof_id = P_LAGR;
-    auto launch = [&](ChunkState& cs, Chunk c, int n) -> int {
+    auto launch = [&](ChunkState& cs, Chunk c, int n, cudaStream_t sm, FixSlot fx) -> int {
       c = with_rev(c, 0);
-      launch_step(ks_lagrangian, dim3(grid_strip(c.nx, LW, c.ny, c.lks).x, n), SB, st, c, cs.tm_lag,
+      launch_step(ks_lagrangian, dim3(grid_strip(c.nx, LW, c.ny, c.lks).x, n), SB, sm, c, cs.tm_lag,
           cs.buf[B_D1], cs.buf[B_E1], cs.buf[B_U1], cs.buf[B_V1], cs.buf[B_FX], cs.buf[B_FY],
-          ctx->scal, cs.fix);
+          ctx->scal, fx);
       STEP_LAUNCH_CHECK();
       return CLOVER_OK;
     };
-    auto fixup = [&](ChunkState& cs, Chunk c) -> int {
+    auto fixup = [&](ChunkState& cs, Chunk c, cudaStream_t sm, FixSlot fx) -> int {
       c = with_rev(c, 0);
       const YWalls yw = walls_in_lagr ? ywalls_of(cs, 1) : kNoWalls;
-      launch_fix(kf_lagrangian, FIX_BLOCKS + 5 * yw.nbx, SB, st, c, cs.tm_lag,
+      launch_fix(kf_lagrangian, FIX_BLOCKS + 5 * yw.nbx, SB, sm, c, cs.tm_lag,
           cs.buf[B_D1], cs.buf[B_E1], cs.buf[B_U1], cs.buf[B_V1], cs.buf[B_FX], cs.buf[B_FY],
-          ctx->scal, cs.fix, yw);
+          ctx->scal, fx, yw);
       FIX_LAUNCH_CHECK();
       return CLOVER_OK;
     };
@@ -950,27 +955,27 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
       if (nphase >= ph_cell) {
         cur_prof_id = sweep == 1 ? P_ADV_X1 : P_ADV_X2;
         const int serp = sweep == 1 ? CLOVER_SERP : 0;
-        auto launch = [&](ChunkState& cs, Chunk c, int n) -> int {
+        auto launch = [&](ChunkState& cs, Chunk c, int n, cudaStream_t sm, FixSlot fx) -> int {
           c = with_rev(c, serp);
           const dim3 g(grid_strip(c.nx + 1, XW, c.ny + 1, c.xks).x, n);
           if (sweep == 1)
-            launch_step(ks_advec_x<1>, g, SB, st, c, cs.tm_x1, cs.buf[rout], cs.buf[eout],
-                        cs.buf[uout], cs.buf[vout], cs.fix);
+            launch_step(ks_advec_x<1>, g, SB, sm, c, cs.tm_x1, cs.buf[rout], cs.buf[eout],
+                        cs.buf[uout], cs.buf[vout], fx);
           else
-            launch_step(ks_advec_x<2>, g, SB, st, c, cs.tm_x2, cs.buf[rout], cs.buf[eout],
-                        cs.buf[uout], cs.buf[vout], cs.fix);
+            launch_step(ks_advec_x<2>, g, SB, sm, c, cs.tm_x2, cs.buf[rout], cs.buf[eout],
+                        cs.buf[uout], cs.buf[vout], fx);
           STEP_LAUNCH_CHECK();
           return CLOVER_OK;
         };
-        auto fixup = [&](ChunkState& cs, Chunk c) -> int {
+        auto fixup = [&](ChunkState& cs, Chunk c, cudaStream_t sm, FixSlot fx) -> int {
           c = with_rev(c, serp);
           if (sweep == 1) {
             const YWalls yw = walls_in_x1 ? ywalls_of(cs, 2) : kNoWalls;
-            launch_fix(kf_advec_x<1>, FIX_BLOCKS + 5 * yw.nbx, SB, st, c, cs.tm_x1, cs.buf[rout],
-                        cs.buf[eout], cs.buf[uout], cs.buf[vout], cs.fix, yw);
+            launch_fix(kf_advec_x<1>, FIX_BLOCKS + 5 * yw.nbx, SB, sm, c, cs.tm_x1, cs.buf[rout],
+                        cs.buf[eout], cs.buf[uout], cs.buf[vout], fx, yw);
           } else {
-            launch_fix(kf_advec_x<2>, FIX_BLOCKS, SB, st, c, cs.tm_x2, cs.buf[rout], cs.buf[eout],
-                        cs.buf[uout], cs.buf[vout], cs.fix, kNoWalls);
+            launch_fix(kf_advec_x<2>, FIX_BLOCKS, SB, sm, c, cs.tm_x2, cs.buf[rout], cs.buf[eout],
+                        cs.buf[uout], cs.buf[vout], fx, kNoWalls);
           }
           FIX_LAUNCH_CHECK();
           return CLOVER_OK;
@@ -1003,14 +1008,14 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
           FIX_LAUNCH_CHECK();
         }
         const int serp = sweep == 1 ? CLOVER_SERP : 0;
-        auto launch = [&](ChunkState& cs, Chunk c, int n) -> int {
+        auto launch = [&](ChunkState& cs, Chunk c, int n, cudaStream_t sm, FixSlot fx) -> int {
           c = with_rev(c, serp);
           const dim3 g(grid_strip(c.nx + 1, YW, c.ny + 1, c.yks).x, n);
           const CUtensorMap& ta = sweep == 1 ? cs.tm_x1 : cs.tm_fy;
           const CUtensorMap& tb = sweep == 1 ? cs.tm_x1 : cs.tm_c4;
           if (sweep == 1) {
-            launch_step(ks_advec_y<1>, g, SB, st, c, ta, tb, cs.buf[rout], cs.buf[eout], cs.buf[B_MY],
-                        cs.buf[uout], cs.buf[vout], cs.fix);
+            launch_step(ks_advec_y<1>, g, SB, sm, c, ta, tb, cs.buf[rout], cs.buf[eout], cs.buf[B_MY],
+                        cs.buf[uout], cs.buf[vout], fx);
           } else if (ctx->f2_probe) {
             // DESIGN.md 4.5 f2 probe: sweep 2 with the next step's viscosity
             // and calc_dt terms folded in (q written, dt to a scratch slot;
@@ -1019,25 +1024,25 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
             vp.q = cs.buf[B_Q];
             vp.dt = (unsigned long long*)cs.partials;
             vp.prm = ctx->dtp;
-            launch_step(ks_advec_y2_probe, g, SB, st, c, ta, tb, cs.buf[rout], cs.buf[eout],
-                        cs.buf[B_MY], cs.buf[uout], cs.buf[vout], cs.fix, vp);
+            launch_step(ks_advec_y2_probe, g, SB, sm, c, ta, tb, cs.buf[rout], cs.buf[eout],
+                        cs.buf[B_MY], cs.buf[uout], cs.buf[vout], fx, vp);
           } else {
-            launch_step(ks_advec_y<2>, g, SB, st, c, ta, tb, cs.buf[rout], cs.buf[eout], cs.buf[B_MY],
-                        cs.buf[uout], cs.buf[vout], cs.fix);
+            launch_step(ks_advec_y<2>, g, SB, sm, c, ta, tb, cs.buf[rout], cs.buf[eout], cs.buf[B_MY],
+                        cs.buf[uout], cs.buf[vout], fx);
           }
           STEP_LAUNCH_CHECK();
           return CLOVER_OK;
         };
-        auto fixup = [&](ChunkState& cs, Chunk c) -> int {
+        auto fixup = [&](ChunkState& cs, Chunk c, cudaStream_t sm, FixSlot fx) -> int {
           c = with_rev(c, serp);
           const CUtensorMap& ta = sweep == 1 ? cs.tm_x1 : cs.tm_fy;
           const CUtensorMap& tb = sweep == 1 ? cs.tm_x1 : cs.tm_c4;
           if (sweep == 1)
-            launch_fix(kf_advec_y<1>, FIX_BLOCKS, SB, st, c, ta, tb, cs.buf[rout], cs.buf[eout],
-                        cs.buf[B_MY], cs.buf[uout], cs.buf[vout], cs.fix);
+            launch_fix(kf_advec_y<1>, FIX_BLOCKS, SB, sm, c, ta, tb, cs.buf[rout], cs.buf[eout],
+                        cs.buf[B_MY], cs.buf[uout], cs.buf[vout], fx);
           else
-            launch_fix(kf_advec_y<2>, FIX_BLOCKS, SB, st, c, ta, tb, cs.buf[rout], cs.buf[eout],
-                        cs.buf[B_MY], cs.buf[uout], cs.buf[vout], cs.fix);
+            launch_fix(kf_advec_y<2>, FIX_BLOCKS, SB, sm, c, ta, tb, cs.buf[rout], cs.buf[eout],
+                        cs.buf[B_MY], cs.buf[uout], cs.buf[vout], fx);
           FIX_LAUNCH_CHECK();
           return CLOVER_OK;
         };
@@ -1548,6 +1553,9 @@ int clover_init(const clover_grid* grid, const clover_state* states, int32_t nst
     cs.fix.hdr = (unsigned*)p;
     cs.fix.e = (uint2*)(p + kAlign);
     p += fix_bytes(c.nx, c.ny);
+    cs.fix_b.hdr = (unsigned*)p;
+    cs.fix_b.e = (uint2*)(p + kAlign);
+    p += fix_bytes(c.nx, c.ny);
     maxrows = std::max<int64_t>(maxrows, c.ny + 2 + 2 * HALO_ROWS);
     maxcols = std::max<int64_t>(maxcols, c.nx + 2 + 2 * HALO_COLS);
     ctx->chunks.push_back(cs);
@@ -1710,6 +1718,8 @@ int clover_debug_fix_count(clover_ctx* ctx, int64_t* out) {
     unsigned h[3];
     CK(cudaMemcpy(h, cs.fix.hdr, sizeof(h), cudaMemcpyDeviceToHost));
     t += h[2];
+    CK(cudaMemcpy(h, cs.fix_b.hdr, sizeof(h), cudaMemcpyDeviceToHost));
+    t += h[2];
   }
   *out = t;
   return CLOVER_OK;
@@ -1737,7 +1747,8 @@ int clover_kernels_per_step(clover_ctx* ctx, int32_t* out) {
       auto extra = [&](int kind, int yd) {
         int lo, hi, ns;
         phase_ranges(cs.c, kind, yd, &lo, &hi, &ns);
-        return (lo > 0) + (hi < ns) + 2 * (lo < hi) - 1;
+        const int b = (lo > 0) + (hi < ns);
+        return b + (b > 0) + 2 * (lo < hi) - 2;
       };
       const bool ax = ctx->advect_x;
       n += extra(SEG_LAGR, fuse_y_ok(ctx) ? HALO_ROWS : HALO);
