@@ -258,8 +258,9 @@ int clover_debug_read_buffer(clover_ctx* ctx, int32_t buffer_id, int32_t kind,
  * exchanges take the remote path (several ranks, or virtual-remote mode),
  * each fused kernel runs the row segments next to a y chunk boundary first,
  * then the halo exchange on a second stream while the interior segments run;
- * the next kernel waits for both.  enable = 1 (default) / 0.  Results are
- * bitwise identical either way; tests compare them. */
+ * the next kernel waits for both.  enable = 1 / 0 (default 0, or the
+ * environment's CLOVER_OVERLAP at clover_init).  Results are bitwise
+ * identical either way; tests compare them. */
 int clover_debug_set_overlap(clover_ctx* ctx, int32_t enable);
 
 /* Debug: the fused advection sweeps (advec_cell + advec_mom of one

@@ -367,7 +367,7 @@ class Clover:
 
     def debug_set_overlap(self, enable: bool):
         """Boundary segments first + the exchange overlapped with the interior
-        (y strips with remote / virtual-remote exchanges; default on)."""
+        (y strips with remote / virtual-remote exchanges; default off)."""
         _check(load().clover_debug_set_overlap(self._ctx, 1 if enable else 0), "clover_debug_set_overlap")
 
     def debug_fix_count(self) -> int:

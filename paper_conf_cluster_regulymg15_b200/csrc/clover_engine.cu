@@ -1471,7 +1471,11 @@ int clover_init(const clover_grid* grid, const clover_state* states, int32_t nst
   ctx->gg = GlobalGeom{ctx->g.x_cells, ctx->g.y_cells, ctx->g.xmin, ctx->g.ymin, dx, dy};
 
   auto bail = [&](int code) { clover_finalize(ctx); return code; };
-  ctx->overlap = true;  // used where overlap_ok
+  // boundary-first overlap: off by default (measured on one GPU, where all
+  // chunks share the SMs, it only pays for 2-chunk layouts);
+  // clover_debug_set_overlap or CLOVER_OVERLAP=1 turn it on
+  ctx->overlap = false;
+  if (const char* e = std::getenv("CLOVER_OVERLAP")) ctx->overlap = std::atoi(e) != 0;
   if (cudaStreamCreateWithFlags(&ctx->work, cudaStreamNonBlocking) != cudaSuccess ||
       cudaStreamCreateWithFlags(&ctx->comm_stream, cudaStreamNonBlocking) != cudaSuccess ||
       cudaEventCreateWithFlags(&ctx->ev_b, cudaEventDisableTiming) != cudaSuccess ||

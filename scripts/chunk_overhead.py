@@ -23,14 +23,13 @@ deck = bm_deck(nx, ny, end_step=steps, ymax=10.0 * ny / nx)
 # (square cells: the domain grows with the mesh)
 
 
-def run(p, q, vr=0, walls_only=False, overlap=True):
+def run(p, q, vr=0, walls_only=False, overlap=False):
     sim = Clover(deck, px=p, py=q)
     if walls_only:
         sim.debug_set_fusion(True, walls_only=True)
     if vr:
         sim.debug_set_virtual_remote(True, nccl=vr == 2)
-    if not overlap:
-        sim.debug_set_overlap(False)
+    sim.debug_set_overlap(overlap)
     sim.step(3)
     sim.sync()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -61,8 +60,8 @@ res["serial_ideal_ms"] = alone * px * py
 res["strong_scaling_efficiency_bound"] = one / (px * py * alone)
 for name, kw in (("local_fused", {}), ("local_walls_only", dict(walls_only=True)),
                  ("virtual_remote", dict(vr=1)), ("virtual_nccl", dict(vr=2)),
-                 ("virtual_remote_no_overlap", dict(vr=1, overlap=False)),
-                 ("virtual_nccl_no_overlap", dict(vr=2, overlap=False))):
+                 ("virtual_remote_overlap", dict(vr=1, overlap=True)),
+                 ("virtual_nccl_overlap", dict(vr=2, overlap=True))):
     ms, k = run(px, py, **kw)
     res[name] = {"ms": ms, "overhead": ms / one - 1.0, "kernels": k,
                  "over_serial_ideal": ms / (alone * px * py) - 1.0}

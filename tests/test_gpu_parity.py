@@ -397,6 +397,7 @@ def test_boundary_first_overlap_bitwise(torch_cuda, nccl, py):
     one = make_gpu(deck)
     ov = make_gpu(deck, px=1, py=py)
     ov.debug_set_virtual_remote(True, nccl=nccl)
+    ov.debug_set_overlap(True)
     plain = make_gpu(deck, px=1, py=py)
     plain.debug_set_virtual_remote(True, nccl=nccl)
     plain.debug_set_overlap(False)
