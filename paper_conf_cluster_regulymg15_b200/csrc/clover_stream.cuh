@@ -1506,17 +1506,20 @@ constexpr int YW = 31;
 #define CLOVER_YKS 32
 #endif
 constexpr int YKS = CLOVER_YKS;
-// Ring depth per sweep (rows): sweep 1 (6 fields per row) runs at 6 rows
-// and a register cap of 10 blocks/SM for occupancy, sweep 2 (5 fields) at
-// 8 rows uncapped -- measured best each (ncu: 281 vs 286 us for sweep 1).
+// Ring depth per sweep (rows): sweep 1 (6 fields per row) at 7 rows and a
+// register cap of 9 blocks/SM (what its 25 KB of ring per block allows),
+// sweep 2 (5 fields) at 7 rows uncapped (10 blocks/SM) -- measured best
+// after the ring-pointer rotation (round 2, same box, 3 repeats: step
+// 0.8737 -> 0.8693 ms against 6/10 and 8/uncapped; round 1's best were 6
+// and 8 rows).
 #ifndef CLOVER_YRING1
-#define CLOVER_YRING1 6
+#define CLOVER_YRING1 7
 #endif
 #ifndef CLOVER_YRING2
-#define CLOVER_YRING2 8
+#define CLOVER_YRING2 7
 #endif
 #ifndef CLOVER_YMINB1
-#define CLOVER_YMINB1 10
+#define CLOVER_YMINB1 9
 #endif
 #ifndef CLOVER_L2HINT  // y sweep: L2 policy for the ring rows shared with the segment below
 #define CLOVER_L2HINT 0
