@@ -254,14 +254,6 @@ int clover_debug_partial_step(clover_ctx* ctx, int32_t nkernels);
 int clover_debug_read_buffer(clover_ctx* ctx, int32_t buffer_id, int32_t kind,
                              double* host, int64_t n);
 
-/* Band flow (one chunk on one rank, both fused sweeps): each advection
- * sweep waits only for the row segments of the previous kernel (the
- * Lagrangian phase, or sweep 1) that its rows read -- per-segment counters
- * released by the producer warps, programmatic dependent launch -- instead
- * of for the whole previous grid, so it starts during that kernel's tail.
- * enable = 1 (default) / 0.  Bitwise identical either way. */
-int clover_debug_set_flow(clover_ctx* ctx, int32_t enable);
-
 /* Device-initiated halo stores (S:8(f) f1): for y strips of local chunks
  * (one process, px == 1) with both fused sweeps, the Lagrangian and the
  * fused advection kernels write the rows a y neighbour keeps as halo

@@ -102,11 +102,7 @@ struct ChunkState {
   double* partials;  // summary partials, ntx*nty*5
   int ntx, nty;
   FixSlot fix;       // warps to redo with IEEE division (clover_stream.cuh)
-  FixSlot fix_b;     // the same for boundary segments running beside the interior (run_phase),
-                     // and for sweep 1 under the band flow
-  FixSlot fix_c;     // sweep 2 under the band flow (flow_ok)
-  unsigned* flow = nullptr;  // band-flow counters: [Lagrangian segs | sweep-1 segs | done L, done S1,
-  int nflow = 0, maxseg = 0; //  bands L, bands S1] (clover_stream.cuh Flow)
+  FixSlot fix_b;     // the same for boundary segments running beside the interior (run_phase)
   PeerY peer{0, 0};  // device-initiated y-halo stores to local neighbours (peer_halos_ok)
   CUtensorMap tm_lag;   // d0 e0 u0 v0 q as one {pitch, rows, 5} fp64 tensor, box {LRW, 1, 5}
   CUtensorMap tm_visc;  // d0 e0 u0 v0 as {pitch, rows, 4}, box {VRW, 1, 4}
@@ -257,7 +253,6 @@ struct clover_ctx {
   cudaStream_t comm_stream = nullptr, xs = nullptr;
   cudaEvent_t ev_b = nullptr, ev_x = nullptr;
   bool overlap = false;  // see overlap_ok
-  bool flow = true;         // see flow_ok
   bool peer_halos = false;  // see peer_halos_ok (off by default: measured 0.3-1.6 % slower on one
                             // GPU than the batched strip copies)
   cudaEvent_t ev_in = nullptr, ev_out = nullptr;
@@ -346,12 +341,9 @@ std::vector<int> local_chunk_ids(int px, int py, int rank, int nranks) {
 // one common stride, then summary partials and the two fix lists), sized for
 // the largest chunk: the same field of two chunks is then a constant offset
 // apart, which the device-initiated halo stores use (PeerY).
-struct ChunkBlock { int64_t field, partials, fix, flow; };
-// segments of any streaming kernel of a chunk with ny rows (shortest tail
-// segment: MIN_KS / CLOVER_TAIL_DIV rows)
-inline int max_segs(int ny) { return (ny + 1) / (MIN_KS / CLOVER_TAIL_DIV) + 2; }
+struct ChunkBlock { int64_t field, partials, fix; };
 ChunkBlock chunk_block(const Layout& L, int px, int py, int rank, int nranks) {
-  ChunkBlock b{0, 0, 0, 0};
+  ChunkBlock b{0, 0, 0};
   for (int id : local_chunk_ids(px, py, rank, nranks)) {
     const int cx = id % px, cy = id / px;
     const int nx = L.xs[cx + 1] - L.xs[cx], ny = L.ys[cy + 1] - L.ys[cy];
@@ -359,7 +351,6 @@ ChunkBlock chunk_block(const Layout& L, int px, int py, int rank, int nranks) {
     const int ntx = (nx + ST - 1) / ST, nty = (ny + ST - 1) / ST;
     b.partials = std::max(b.partials, align_up((int64_t)ntx * nty * 5 * 8, kAlign));
     b.fix = std::max(b.fix, fix_bytes(nx, ny));
-    b.flow = std::max(b.flow, align_up((int64_t)(2 * max_segs(ny) + 8) * 4, kAlign));
   }
   return b;
 }
@@ -372,7 +363,7 @@ int64_t compute_workspace(const clover_grid* g, int px, int py, int rank, int nr
   for (int id : local_chunk_ids(px, py, rank, nranks)) {
     int cx = id % px, cy = id / px;
     int nx = L.xs[cx + 1] - L.xs[cx], ny = L.ys[cy + 1] - L.ys[cy];
-    bytes += NBUF * blk.field + blk.partials + 3 * blk.fix + blk.flow;
+    bytes += NBUF * blk.field + blk.partials + 2 * blk.fix;
     maxrows = std::max<int64_t>(maxrows, ny + 2 + 2 * HALO_ROWS);
     maxcols = std::max<int64_t>(maxcols, nx + 2 + 2 * HALO_COLS);
   }
@@ -790,14 +781,6 @@ bool peer_halos_ok(const clover_ctx* ctx) {
          ctx->L.py > 1 && fuse_x_ok(ctx) && fuse_y_ok(ctx);
 }
 
-// Band flow (clover_stream.cuh Flow): one chunk on one rank, both fused
-// sweeps -- the sweeps start on the Lagrangian's / sweep 1's finished row
-// segments while that kernel's tail still runs.
-bool flow_ok(const clover_ctx* ctx) {
-  return ctx->flow && ctx->chunks.size() == 1 && ctx->nranks == 1 && !ctx->virtual_remote &&
-         fuse_x_ok(ctx) && fuse_y_ok(ctx);
-}
-
 // Row-segment geometry of a streaming kernel kind on a chunk: rows per
 // segment, full-height segments, rows covered (seg_rows_of).
 enum { SEG_LAGR, SEG_X, SEG_Y };
@@ -877,44 +860,6 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
   // the next phase waits for both.
   const bool peers = peer_halos_ok(ctx);
   auto peer_of = [&](const ChunkState& cs) { return peers ? cs.peer : PeerY{0, 0}; };
-  // band flow: counters of the Lagrangian (producer 0) and sweep 1 (1)
-  const bool flw = flow_ok(ctx);
-  auto fdone = [&](const ChunkState& cs, int prod, bool bands) {
-    FlowDone d{nullptr, nullptr};
-    if (!flw || prod > 1) return d;
-    d.done = cs.flow + 2 * cs.maxseg + prod;
-    if (bands) d.bands = cs.flow + 2 * cs.maxseg + 2 + prod;
-    return d;
-  };
-  // kind of the kernel that produced a phase's inputs, for a consumer flow
-  auto producer_geom = [&](const ChunkState& cs, int kind, Flow& f) {
-    int ks, nb, rows;
-    seg_geom(cs.c, kind, &ks, &nb, &rows);
-    f.wks = ks; f.wnb = nb; f.wnseg = seg_count(ks, nb, rows);
-    const int cols = kind == SEG_LAGR ? grid_strip(cs.c.nx, LW, cs.c.ny, ks).x
-                   : kind == SEG_X ? grid_strip(cs.c.nx + 1, XW, cs.c.ny + 1, ks).x
-                                   : grid_strip(cs.c.nx + 1, YW, cs.c.ny + 1, ks).x;
-    f.wtarget = (unsigned)cols * (SB / 32);
-  };
-  // prod: this launch's producer slot (0 L, 1 S1, -1 none); cons_of: the
-  // producer slot it waits for (-1 none) with that producer's kind
-  auto flow_of = [&](const ChunkState& cs, int prod, int cons_of, int prod_kind, int rlo, int rhi,
-                     bool bands) {
-    Flow f{};
-    if (!flw) return f;
-    if (prod >= 0) f.sig = cs.flow + prod * cs.maxseg;
-    if (cons_of >= 0) {
-      f.wcnt = cs.flow + cons_of * cs.maxseg;
-      f.wdone = cs.flow + 2 * cs.maxseg + cons_of;
-      if (bands) {
-        f.wbands = cs.flow + 2 * cs.maxseg + 2 + cons_of;
-        f.wbtarget = 5u * (unsigned)ywalls_of(cs, 1).nbx;
-      }
-      producer_geom(cs, prod_kind, f);
-      f.rlo = rlo; f.rhi = rhi;
-    }
-    return f;
-  };
   auto run_phase = [&](int kind, auto&& launch, auto&& fixup, const std::vector<int>& bufs, int yd,
                        int xd) -> int {
     if (!overlap_ok(ctx)) {
@@ -971,7 +916,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
                   ctx->scal, ctx->dtp, cs.fix);
       STEP_LAUNCH_CHECK();
       launch_fix(kf_visc_dt, FIX_BLOCKS, SB, st, c, cs.tm_visc, cs.buf[B_Q], ctx->scal, ctx->dtp,
-                  cs.fix, ctx->hist, fold_fin, cs.flow, cs.nflow);
+                  cs.fix, ctx->hist, fold_fin);
       FIX_LAUNCH_CHECK();
     }
     // q on ring 1: visc_dt computes rows 0 / ny+1 at y chunk boundaries
@@ -1009,7 +954,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
       c = with_rev(c, 0);
       launch_step(ks_lagrangian, dim3(grid_strip(c.nx, LW, c.ny, c.lks).x, n), SB, sm, c, cs.tm_lag,
           cs.buf[B_D1], cs.buf[B_E1], cs.buf[B_U1], cs.buf[B_V1], cs.buf[B_FX], cs.buf[B_FY],
-          ctx->scal, fx, peer_of(cs), flow_of(cs, 0, -1, 0, 0, 0, false));
+          ctx->scal, fx, peer_of(cs));
       STEP_LAUNCH_CHECK();
       return CLOVER_OK;
     };
@@ -1018,7 +963,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
       const YWalls yw = walls_in_lagr ? ywalls_of(cs, 1) : kNoWalls;
       launch_fix(kf_lagrangian, FIX_BLOCKS + 5 * yw.nbx, SB, sm, c, cs.tm_lag,
           cs.buf[B_D1], cs.buf[B_E1], cs.buf[B_U1], cs.buf[B_V1], cs.buf[B_FX], cs.buf[B_FY],
-          ctx->scal, fx, yw, peer_of(cs), fdone(cs, 0, walls_in_lagr));
+          ctx->scal, fx, yw, peer_of(cs));
       FIX_LAUNCH_CHECK();
       return CLOVER_OK;
     };
@@ -1046,31 +991,24 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
         auto launch = [&](ChunkState& cs, Chunk c, int n, cudaStream_t sm, FixSlot fx) -> int {
           c = with_rev(c, serp);
           const dim3 g(grid_strip(c.nx + 1, XW, c.ny + 1, c.xks).x, n);
-          // band flow: sweep 1 waits for the Lagrangian's segments, sweep 2
-          // for sweep 1's (a y sweep); own fix list per sweep
-          const Flow fl = sweep == 1 ? flow_of(cs, 1, 0, SEG_LAGR, -1, 1, false)
-                                     : flow_of(cs, -1, 1, SEG_Y, -1, 1, false);
-          if (flw) fx = sweep == 1 ? cs.fix_b : cs.fix_c;
           if (sweep == 1)
-            launch_pdl(flw ? 1 : CLOVER_PDL, ks_advec_x<1>, g, SB, sm, c, cs.tm_x1, cs.buf[rout],
-                       cs.buf[eout], cs.buf[uout], cs.buf[vout], fx, peer_of(cs), fl);
+            launch_step(ks_advec_x<1>, g, SB, sm, c, cs.tm_x1, cs.buf[rout], cs.buf[eout],
+                        cs.buf[uout], cs.buf[vout], fx, peer_of(cs));
           else
-            launch_pdl(flw ? 1 : CLOVER_PDL, ks_advec_x<2>, g, SB, sm, c, cs.tm_x2, cs.buf[rout],
-                       cs.buf[eout], cs.buf[uout], cs.buf[vout], fx, peer_of(cs), fl);
+            launch_step(ks_advec_x<2>, g, SB, sm, c, cs.tm_x2, cs.buf[rout], cs.buf[eout],
+                        cs.buf[uout], cs.buf[vout], fx, peer_of(cs));
           STEP_LAUNCH_CHECK();
           return CLOVER_OK;
         };
         auto fixup = [&](ChunkState& cs, Chunk c, cudaStream_t sm, FixSlot fx) -> int {
           c = with_rev(c, serp);
-          if (flw) fx = sweep == 1 ? cs.fix_b : cs.fix_c;
           if (sweep == 1) {
             const YWalls yw = walls_in_x1 ? ywalls_of(cs, 2) : kNoWalls;
             launch_fix(kf_advec_x<1>, FIX_BLOCKS + 5 * yw.nbx, SB, sm, c, cs.tm_x1, cs.buf[rout],
-                        cs.buf[eout], cs.buf[uout], cs.buf[vout], fx, yw, peer_of(cs),
-                        fdone(cs, 1, walls_in_x1));
+                        cs.buf[eout], cs.buf[uout], cs.buf[vout], fx, yw, peer_of(cs));
           } else {
             launch_fix(kf_advec_x<2>, FIX_BLOCKS, SB, sm, c, cs.tm_x2, cs.buf[rout], cs.buf[eout],
-                        cs.buf[uout], cs.buf[vout], fx, kNoWalls, peer_of(cs), fdone(cs, 2, false));
+                        cs.buf[uout], cs.buf[vout], fx, kNoWalls, peer_of(cs));
           }
           FIX_LAUNCH_CHECK();
           return CLOVER_OK;
@@ -1108,15 +1046,9 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
           const dim3 g(grid_strip(c.nx + 1, YW, c.ny + 1, c.yks).x, n);
           const CUtensorMap& ta = sweep == 1 ? cs.tm_x1 : cs.tm_fy;
           const CUtensorMap& tb = sweep == 1 ? cs.tm_x1 : cs.tm_c4;
-          // band flow: rows k0-4 .. k1+2 of the producer; the wall bands ride
-          // on the producer's fixup launch (walls_in_lagr / walls_in_x1)
-          const Flow fl = sweep == 1 ? flow_of(cs, 1, 0, SEG_LAGR, -4, 3, walls_in_lagr)
-                                     : flow_of(cs, -1, 1, SEG_X, -4, 3, walls_in_x1);
-          if (flw) fx = sweep == 1 ? cs.fix_b : cs.fix_c;
-          const int pdl = flw ? 1 : CLOVER_PDL;
           if (sweep == 1) {
-            launch_pdl(pdl, ks_advec_y<1>, g, SB, sm, c, ta, tb, cs.buf[rout], cs.buf[eout],
-                       cs.buf[B_MY], cs.buf[uout], cs.buf[vout], fx, peer_of(cs), fl);
+            launch_step(ks_advec_y<1>, g, SB, sm, c, ta, tb, cs.buf[rout], cs.buf[eout], cs.buf[B_MY],
+                        cs.buf[uout], cs.buf[vout], fx, peer_of(cs));
           } else if (ctx->f2_probe) {
             // DESIGN.md 4.5 f2 probe: sweep 2 with the next step's viscosity
             // and calc_dt terms folded in (q written, dt to a scratch slot;
@@ -1128,8 +1060,8 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
             launch_step(ks_advec_y2_probe, g, SB, sm, c, ta, tb, cs.buf[rout], cs.buf[eout],
                         cs.buf[B_MY], cs.buf[uout], cs.buf[vout], fx, vp);
           } else {
-            launch_pdl(pdl, ks_advec_y<2>, g, SB, sm, c, ta, tb, cs.buf[rout], cs.buf[eout],
-                       cs.buf[B_MY], cs.buf[uout], cs.buf[vout], fx, peer_of(cs), fl);
+            launch_step(ks_advec_y<2>, g, SB, sm, c, ta, tb, cs.buf[rout], cs.buf[eout], cs.buf[B_MY],
+                        cs.buf[uout], cs.buf[vout], fx, peer_of(cs));
           }
           STEP_LAUNCH_CHECK();
           return CLOVER_OK;
@@ -1138,13 +1070,12 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
           c = with_rev(c, serp);
           const CUtensorMap& ta = sweep == 1 ? cs.tm_x1 : cs.tm_fy;
           const CUtensorMap& tb = sweep == 1 ? cs.tm_x1 : cs.tm_c4;
-          if (flw) fx = sweep == 1 ? cs.fix_b : cs.fix_c;
           if (sweep == 1)
             launch_fix(kf_advec_y<1>, FIX_BLOCKS, SB, sm, c, ta, tb, cs.buf[rout], cs.buf[eout],
-                        cs.buf[B_MY], cs.buf[uout], cs.buf[vout], fx, peer_of(cs), fdone(cs, 1, false));
+                        cs.buf[B_MY], cs.buf[uout], cs.buf[vout], fx, peer_of(cs));
           else
             launch_fix(kf_advec_y<2>, FIX_BLOCKS, SB, sm, c, ta, tb, cs.buf[rout], cs.buf[eout],
-                        cs.buf[B_MY], cs.buf[uout], cs.buf[vout], fx, peer_of(cs), fdone(cs, 2, false));
+                        cs.buf[B_MY], cs.buf[uout], cs.buf[vout], fx, peer_of(cs));
           FIX_LAUNCH_CHECK();
           return CLOVER_OK;
         };
@@ -1664,13 +1595,6 @@ int clover_init(const clover_grid* grid, const clover_state* states, int32_t nst
     cs.fix_b.hdr = (unsigned*)p;
     cs.fix_b.e = (uint2*)(p + kAlign);
     p += blk.fix;
-    cs.fix_c.hdr = (unsigned*)p;
-    cs.fix_c.e = (uint2*)(p + kAlign);
-    p += blk.fix;
-    cs.flow = (unsigned*)p;
-    cs.maxseg = max_segs(c.ny);
-    cs.nflow = 2 * cs.maxseg + 8;
-    p += blk.flow;
     maxrows = std::max<int64_t>(maxrows, c.ny + 2 + 2 * HALO_ROWS);
     maxcols = std::max<int64_t>(maxcols, c.nx + 2 + 2 * HALO_COLS);
     ctx->chunks.push_back(cs);
@@ -1810,17 +1734,6 @@ int clover_debug_set_virtual_remote(clover_ctx* ctx, int32_t enable) {
   return CLOVER_OK;
 }
 
-int clover_debug_set_flow(clover_ctx* ctx, int32_t enable) {
-  if (!ctx) return fail(CLOVER_ERR_ARG, "ctx is NULL");
-  ctx->flow = enable != 0;
-  for (int i = 0; i < 4; ++i)
-    if (ctx->gexec[i]) {
-      cudaGraphExecDestroy(ctx->gexec[i]);
-      ctx->gexec[i] = nullptr;
-    }
-  return CLOVER_OK;
-}
-
 int clover_debug_set_peer_halos(clover_ctx* ctx, int32_t enable) {
   if (!ctx) return fail(CLOVER_ERR_ARG, "ctx is NULL");
   ctx->peer_halos = enable != 0;
@@ -1867,8 +1780,6 @@ int clover_debug_fix_count(clover_ctx* ctx, int64_t* out) {
     CK(cudaMemcpy(h, cs.fix.hdr, sizeof(h), cudaMemcpyDeviceToHost));
     t += h[2];
     CK(cudaMemcpy(h, cs.fix_b.hdr, sizeof(h), cudaMemcpyDeviceToHost));
-    t += h[2];
-    CK(cudaMemcpy(h, cs.fix_c.hdr, sizeof(h), cudaMemcpyDeviceToHost));
     t += h[2];
   }
   *out = t;

@@ -180,75 +180,6 @@ __device__ __forceinline__ void fix_loop(FixSlot f, int ks, int nb, int lim, Run
   }
 }
 
-// ---------------------------------------------------------------- band flow
-// Fine-grained producer -> consumer ordering between consecutive streaming
-// kernels (one chunk on one rank): instead of waiting for the whole previous
-// grid (griddepcontrol.wait), a consumer warp waits only for the producer's
-// row segments its rows depend on, so it starts while the producer's last
-// segments -- the kernel tail -- still run.  The consumer is launched with
-// programmatic dependent launch behind the producer's fixup launch, so every
-// producer and fixup block is resident or done before any consumer block
-// spins (no deadlock).  A producer warp adds 1 to its segment's counter
-// (release) unless it flagged an IEEE redo; the fixup launch raises `done`
-// (release) once every redo is written; a consumer proceeds when each needed
-// segment has all its warps or `done` is up (acquire), then orders its TMA
-// reads after that (proxy fence).  Wall-band blocks carried by the fixup
-// launch count themselves in `bands`.  Counters are reset by the visc fixup
-// at every step start (the Lagrangian waits for it: dt).
-struct FlowDone {          // a fixup launch's signals for the band flow (null: none)
-  unsigned* done;          // raised once every redo of the launch is written
-  unsigned* bands;         // +1 per wall-band block finished
-};
-struct Flow {
-  unsigned* sig;          // producer: this launch's per-segment counters (null: none)
-  const unsigned* wcnt;   // consumer: the producer's counters (null: griddepcontrol.wait)
-  const unsigned* wdone;  // consumer: the producer fixup's done flag
-  const unsigned* wbands; // consumer: wall-band blocks done (null: no bands to wait for)
-  int wks, wnb, wnseg;    // producer row segments (seg_rows_of)
-  unsigned wtarget;       // producer warps per segment row
-  unsigned wbtarget;      // band blocks
-  int rlo, rhi;           // consumer segment [k0, k1) reads producer rows [k0+rlo, k1-1+rhi]
-};
-__device__ __forceinline__ unsigned ld_acquire_u32(const unsigned* p) {
-  unsigned v;
-  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
-  return v;
-}
-__device__ __forceinline__ void red_release_add(unsigned* p, unsigned v) {
-  asm volatile("red.release.gpu.global.add.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
-}
-__device__ __forceinline__ void st_release_u32(unsigned* p, unsigned v) {
-  asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
-}
-__device__ __forceinline__ int seg_of_row_d(int r, int ks, int nb, int nseg) {
-  if (r < 1) r = 1;
-  int s;
-  if ((long long)(r - 1) < (long long)nb * ks) s = (r - 1) / ks;
-  else s = nb + (int)(((long long)(r - 1) - (long long)nb * ks) / (ks / CLOVER_TAIL_DIV));
-  return s < nseg ? s : nseg - 1;
-}
-// consumer: the warp's producer rows are final (call by the whole warp)
-__device__ __forceinline__ void flow_wait(const Flow& f, const Chunk& c, int k0, int k1, int lane) {
-  if (!f.wcnt) return;
-  if (lane == 0) {
-    const int s0 = seg_of_row_d(k0 + f.rlo, f.wks, f.wnb, f.wnseg);
-    const int s1 = seg_of_row_d(k1 - 1 + f.rhi, f.wks, f.wnb, f.wnseg);
-    for (int sg = s0; sg <= s1; ++sg)
-      while (ld_acquire_u32(f.wcnt + sg) < f.wtarget && ld_acquire_u32(f.wdone) == 0u)
-        __nanosleep(32);
-    if (f.wbands && ((c.wb && k0 + f.rlo <= 4) || (c.wt && k1 - 1 + f.rhi >= c.ny - 3)))
-      while (ld_acquire_u32(f.wbands) < f.wbtarget) __nanosleep(32);
-    asm volatile("fence.proxy.async.global;" ::: "memory");  // TMA reads after the acquire
-  }
-  __syncwarp();
-}
-// producer: this warp's rows of segment `seg` are final (whole warp)
-__device__ __forceinline__ void flow_signal(const Flow& f, int seg, bool redo, int lane) {
-  if (!f.sig) return;
-  __syncwarp();
-  if (lane == 0 && !redo) red_release_add(f.sig + seg, 1u);
-}
-
 // ---------------------------------------------------------------- y-wall bands
 // advec_cell y on the wall bands (cell rows 1..3 and ny-1..ny, IEEE
 // division: bitwise the fast path's results) so the fused y sweep finds
@@ -316,8 +247,7 @@ __device__ __forceinline__ void y_walls_block(const Chunk& c, const YWalls& y, i
 // flagged, the common case), then compute the bands.  Every block of the
 // launch is co-resident (small blocks), so the wait cannot starve the fixups.
 template <int SWEEP>
-__device__ __forceinline__ bool y_walls_after_fix(const Chunk& c, FixSlot f, const YWalls& y,
-                                                  unsigned* bands = nullptr) {
+__device__ __forceinline__ bool y_walls_after_fix(const Chunk& c, FixSlot f, const YWalls& y) {
   if ((int)blockIdx.x < FIX_BLOCKS) return false;
   if (threadIdx.x == 0) {
     unsigned v;
@@ -330,10 +260,6 @@ __device__ __forceinline__ bool y_walls_after_fix(const Chunk& c, FixSlot f, con
   __syncthreads();
   const int b = (int)blockIdx.x - FIX_BLOCKS;
   y_walls_block<SWEEP>(c, y, b % y.nbx, b / y.nbx);
-  if (bands) {  // band flow: this block's rows are final
-    __syncthreads();
-    if (threadIdx.x == 0) red_release_add(bands, 1u);
-  }
   return true;
 }
 
@@ -509,13 +435,9 @@ ks_visc_dt(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__
 __global__ void __launch_bounds__(SB)
 kf_visc_dt(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__ q,
            StepScalars* __restrict__ s, DtParams prm, FixSlot fix, double* __restrict__ hist,
-           int fin, unsigned* __restrict__ flow, int nflow) {
+           int fin) {
   pdl_trigger();
   pdl_wait();
-  // band-flow counters of this step start at zero (the Lagrangian launch
-  // waits for this grid: it needs dt)
-  for (int t = blockIdx.x * blockDim.x + threadIdx.x; t < nflow; t += gridDim.x * blockDim.x)
-    flow[t] = 0u;
   __shared__ __align__(128) double ring[SB / 32][VSTG * VSLOT];
   __shared__ __align__(8) unsigned long long bars[SB / 32][VSTG];
   // fin: single chunk on one rank -- the last block also finalises dt
@@ -822,7 +744,7 @@ __global__ void LB_HEAVY
 ks_lagrangian(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__ d1,
               double* __restrict__ e1, double* __restrict__ u1, double* __restrict__ v1,
               double* __restrict__ fx, double* __restrict__ fy, const StepScalars* __restrict__ s,
-              FixSlot fix, PeerY peer, Flow flow) {
+              FixSlot fix, PeerY peer) {
   pdl_trigger();
   pdl_wait();
   __shared__ __align__(128) double ring[SB / 32][LSTG * LSLOT];
@@ -832,34 +754,26 @@ ks_lagrangian(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restric
   int k0, len;
   seg_rows_of(seg_y(c), c.lks, c.lnb, k0, len);
   const int k1 = min(k0 + len, c.ny + 1);
-  const bool redo =
-      lagr_seg<DivFast>(c, &tm, d1, e1, u1, v1, fx, fy, s, gw, k0, k1, lane, ring[w], bars[w], peer);
-  if (redo) fix_push(fix, lane, gw, (unsigned)seg_y(c));
-  flow_signal(flow, seg_y(c), redo, lane);
+  if (lagr_seg<DivFast>(c, &tm, d1, e1, u1, v1, fx, fy, s, gw, k0, k1, lane, ring[w], bars[w], peer))
+    fix_push(fix, lane, gw, (unsigned)seg_y(c));
 }
 
 __global__ void __launch_bounds__(SB)
 kf_lagrangian(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__ d1,
               double* __restrict__ e1, double* __restrict__ u1, double* __restrict__ v1,
               double* __restrict__ fx, double* __restrict__ fy, StepScalars* __restrict__ s,
-              FixSlot fix, YWalls yw, PeerY peer, FlowDone fd) {
+              FixSlot fix, YWalls yw, PeerY peer) {
   pdl_trigger();
   pdl_wait();
-  if (y_walls_after_fix<1>(c, fix, yw, fd.bands)) return;
+  if (y_walls_after_fix<1>(c, fix, yw)) return;
   __shared__ __align__(128) double ring[SB / 32][LSTG * LSLOT];
   __shared__ __align__(8) unsigned long long bars[SB / 32][LSTG];
-  fix_loop(
-      fix, c.lks, c.lnb, c.ny + 1,
-      [&](int gw, int k0, int k1, int lane, int w) {
-        // the IEEE redo's flag is the exact PdV volume test (DivIEEE::vol_check)
-        if (lagr_seg<DivIEEE>(c, &tm, d1, e1, u1, v1, fx, fy, s, gw, k0, k1, lane, ring[w], bars[w],
-                              peer) &&
-            lane == 0)
-          atomicCAS(&s->err, 0, -6);  // CLOVER_ERR_NEG_VOLUME
-      },
-      [&]() {
-        if (fd.done) st_release_u32(fd.done, 1u);
-      });
+  fix_loop(fix, c.lks, c.lnb, c.ny + 1, [&](int gw, int k0, int k1, int lane, int w) {
+    // the IEEE redo's flag is the exact PdV volume test (DivIEEE::vol_check)
+    if (lagr_seg<DivIEEE>(c, &tm, d1, e1, u1, v1, fx, fy, s, gw, k0, k1, lane, ring[w], bars[w], peer) &&
+        lane == 0)
+      atomicCAS(&s->err, 0, -6);  // CLOVER_ERR_NEG_VOLUME
+  });
 }
 // (a register-only Lagrangian variant was measured 3% slower; see git history)
 
@@ -1445,9 +1359,9 @@ template <int SWEEP>
 __global__ void LB_ADVX
 ks_advec_x(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__ rho_out,
            double* __restrict__ en_out, double* __restrict__ uout, double* __restrict__ vout,
-           FixSlot fix, PeerY peer, Flow flow) {
+           FixSlot fix, PeerY peer) {
   pdl_trigger();
-  if (!flow.wcnt) pdl_wait();
+  pdl_wait();
   __shared__ __align__(128) double ring[SB / 32][XSTG * xslot<SWEEP>()];
   __shared__ __align__(8) unsigned long long bars[SB / 32][XSTG];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
@@ -1455,33 +1369,26 @@ ks_advec_x(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__
   int k0, len;
   seg_rows_of(seg_y(c), c.xks, c.xnb, k0, len);
   const int k1 = min(k0 + len, c.ny + 2);
-  flow_wait(flow, c, k0, k1, lane);
-  const bool redo = advec_x_seg<SWEEP, DivFast>(c, &tm, rho_out, en_out, uout, vout, gw, k0, k1,
-                                                lane, ring[w], bars[w], peer);
-  if (redo) fix_push(fix, lane, gw, (unsigned)seg_y(c));
-  flow_signal(flow, seg_y(c), redo, lane);
+  if (advec_x_seg<SWEEP, DivFast>(c, &tm, rho_out, en_out, uout, vout, gw, k0, k1, lane, ring[w],
+                                   bars[w], peer))
+    fix_push(fix, lane, gw, (unsigned)seg_y(c));
 }
 
 template <int SWEEP>
 __global__ void __launch_bounds__(SB)
 kf_advec_x(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__ rho_out,
            double* __restrict__ en_out, double* __restrict__ uout, double* __restrict__ vout,
-           FixSlot fix, YWalls yw, PeerY peer, FlowDone fd) {
+           FixSlot fix, YWalls yw, PeerY peer) {
   pdl_trigger();
   pdl_wait();
   if constexpr (SWEEP == 1)  // sweep 2 is y
-    if (y_walls_after_fix<2>(c, fix, yw, fd.bands)) return;
+    if (y_walls_after_fix<2>(c, fix, yw)) return;
   __shared__ __align__(128) double ring[SB / 32][XSTG * xslot<SWEEP>()];
   __shared__ __align__(8) unsigned long long bars[SB / 32][XSTG];
-  fix_loop(
-      fix, c.xks, c.xnb, c.ny + 2,
-      [&](int gw, int k0, int k1, int lane, int w) {
-        advec_x_seg<SWEEP, DivIEEE>(c, &tm, rho_out, en_out, uout, vout, gw, k0, k1, lane, ring[w],
-                                     bars[w], peer);
-      },
-      [&]() {
-        if (fd.done) st_release_u32(fd.done, 1u);
-      });
+  fix_loop(fix, c.xks, c.xnb, c.ny + 2, [&](int gw, int k0, int k1, int lane, int w) {
+    advec_x_seg<SWEEP, DivIEEE>(c, &tm, rho_out, en_out, uout, vout, gw, k0, k1, lane, ring[w],
+                                 bars[w], peer);
+  });
 }
 
 // ================================================================ advec_mom y
@@ -1968,10 +1875,9 @@ template <int SWEEP>
 __global__ void __launch_bounds__(SB, YL<SWEEP>::MINB)
 ks_advec_y(Chunk c, const __grid_constant__ CUtensorMap ta, const __grid_constant__ CUtensorMap tb,
            double* __restrict__ rho_out, double* __restrict__ en_out, const double* __restrict__ mfy,
-           double* __restrict__ uout, double* __restrict__ vout, FixSlot fix, PeerY peer,
-           Flow flow) {
+           double* __restrict__ uout, double* __restrict__ vout, FixSlot fix, PeerY peer) {
   pdl_trigger();
-  if (!flow.wcnt) pdl_wait();
+  pdl_wait();
   __shared__ __align__(128) double ring[SB / 32][YL<SWEEP>::RING * YL<SWEEP>::SLOT];
   __shared__ __align__(8) unsigned long long bars[SB / 32][YL<SWEEP>::RING];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
@@ -1979,11 +1885,9 @@ ks_advec_y(Chunk c, const __grid_constant__ CUtensorMap ta, const __grid_constan
   int k0, len;
   seg_rows_of(seg_y(c), c.yks, c.ynb, k0, len);
   const int k1 = min(k0 + len, c.ny + 2);
-  flow_wait(flow, c, k0, k1, lane);
-  const bool redo = advec_y_seg<SWEEP, DivFast>(c, &ta, &tb, rho_out, en_out, mfy, uout, vout, gw,
-                                                k0, k1, lane, ring[w], bars[w], peer);
-  if (redo) fix_push(fix, lane, gw, (unsigned)seg_y(c));
-  flow_signal(flow, seg_y(c), redo, lane);
+  if (advec_y_seg<SWEEP, DivFast>(c, &ta, &tb, rho_out, en_out, mfy, uout, vout, gw, k0, k1, lane,
+                                  ring[w], bars[w], peer))
+    fix_push(fix, lane, gw, (unsigned)seg_y(c));
 }
 
 // the f2 probe kernel: interior segments run advec_y_body<2, DivFast,
@@ -2017,21 +1921,15 @@ template <int SWEEP>
 __global__ void __launch_bounds__(SB)
 kf_advec_y(Chunk c, const __grid_constant__ CUtensorMap ta, const __grid_constant__ CUtensorMap tb,
            double* __restrict__ rho_out, double* __restrict__ en_out, const double* __restrict__ mfy,
-           double* __restrict__ uout, double* __restrict__ vout, FixSlot fix, PeerY peer,
-           FlowDone fd) {
+           double* __restrict__ uout, double* __restrict__ vout, FixSlot fix, PeerY peer) {
   pdl_trigger();
   pdl_wait();
   __shared__ __align__(128) double ring[SB / 32][YL<SWEEP>::RING * YL<SWEEP>::SLOT];
   __shared__ __align__(8) unsigned long long bars[SB / 32][YL<SWEEP>::RING];
-  fix_loop(
-      fix, c.yks, c.ynb, c.ny + 2,
-      [&](int gw, int k0, int k1, int lane, int w) {
-        advec_y_seg<SWEEP, DivIEEE>(c, &ta, &tb, rho_out, en_out, mfy, uout, vout, gw, k0, k1, lane,
-                                    ring[w], bars[w], peer);
-      },
-      [&]() {
-        if (fd.done) st_release_u32(fd.done, 1u);
-      });
+  fix_loop(fix, c.yks, c.ynb, c.ny + 2, [&](int gw, int k0, int k1, int lane, int w) {
+    advec_y_seg<SWEEP, DivIEEE>(c, &ta, &tb, rho_out, en_out, mfy, uout, vout, gw, k0, k1, lane,
+                                ring[w], bars[w], peer);
+  });
 }
 
 // the y-wall bands as their own launch (several chunks or ranks; see YWalls)
