@@ -258,8 +258,7 @@ int clover_debug_read_buffer(clover_ctx* ctx, int32_t buffer_id, int32_t kind,
  * (one process, px == 1) with both fused sweeps, the Lagrangian and the
  * fused advection kernels write the rows a y neighbour keeps as halo
  * straight into its buffers from their epilogues, and those phases run no
- * exchange.  enable = 1 / 0 (default: on one GPU the batched strip copies
- * measured cheaper); bitwise identical either way. */
+ * exchange.  enable = 1 (default) / 0; bitwise identical either way. */
 int clover_debug_set_peer_halos(clover_ctx* ctx, int32_t enable);
 
 /* Boundary-first overlap (S:8(e)): for y-strip layouts (px == 1) whose

@@ -373,7 +373,7 @@ class Clover:
         _check(load().clover_debug_set_overlap(self._ctx, 1 if enable else 0), "clover_debug_set_overlap")
 
     def debug_set_peer_halos(self, enable: bool):
-        """Device-initiated y-halo stores between local y-strip chunks (default off)."""
+        """Device-initiated y-halo stores between local y-strip chunks (default on)."""
         _check(load().clover_debug_set_peer_halos(self._ctx, 1 if enable else 0),
                "clover_debug_set_peer_halos")
 

@@ -253,8 +253,7 @@ struct clover_ctx {
   cudaStream_t comm_stream = nullptr, xs = nullptr;
   cudaEvent_t ev_b = nullptr, ev_x = nullptr;
   bool overlap = false;  // see overlap_ok
-  bool peer_halos = false;  // see peer_halos_ok (off by default: measured 0.3-1.6 % slower on one
-                            // GPU than the batched strip copies)
+  bool peer_halos = true;  // see peer_halos_ok
   cudaEvent_t ev_in = nullptr, ev_out = nullptr;
   StepScalars* scal = nullptr;
   double* hist = nullptr;

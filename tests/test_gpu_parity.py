@@ -395,7 +395,6 @@ def test_device_initiated_halo_stores_bitwise(torch_cuda, seed, py):
     deck["max_timestep"] = 1.0
     one = make_gpu(deck)
     peer = make_gpu(deck, px=1, py=py)
-    peer.debug_set_peer_halos(True)
     exch = make_gpu(deck, px=1, py=py)
     exch.debug_set_peer_halos(False)
     for g in (one, peer, exch):
