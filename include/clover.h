@@ -254,13 +254,6 @@ int clover_debug_partial_step(clover_ctx* ctx, int32_t nkernels);
 int clover_debug_read_buffer(clover_ctx* ctx, int32_t buffer_id, int32_t kind,
                              double* host, int64_t n);
 
-/* Device-initiated halo stores (S:8(f) f1): for y strips of local chunks
- * (one process, px == 1) with both fused sweeps, the Lagrangian and the
- * fused advection kernels write the rows a y neighbour keeps as halo
- * straight into its buffers from their epilogues, and those phases run no
- * exchange.  enable = 1 (default) / 0; bitwise identical either way. */
-int clover_debug_set_peer_halos(clover_ctx* ctx, int32_t enable);
-
 /* Boundary-first overlap (S:8(e)): for y-strip layouts (px == 1) whose
  * exchanges take the remote path (several ranks, or virtual-remote mode),
  * each fused kernel runs the row segments next to a y chunk boundary first,

@@ -40,7 +40,7 @@ EXPORTS = ["clover_workspace_bytes", "clover_nccl_unique_id", "clover_init", "cl
            "clover_read_field", "clover_read_field_window", "clover_write_field", "clover_sync", "clover_set_graphs",
            "clover_kernels_per_step", "clover_debug_partial_step", "clover_debug_read_buffer",
            "clover_profile_steps", "clover_profile_name", "clover_debug_div_check",
-           "clover_debug_fix_count", "clover_debug_set_fusion", "clover_debug_set_overlap", "clover_debug_set_peer_halos",
+           "clover_debug_fix_count", "clover_debug_set_fusion", "clover_debug_set_overlap",
            "clover_checkpoint_plan", "clover_debug_set_virtual_remote", "clover_checkpoint_bytes", "clover_checkpoint", "clover_restart", "clover_finalize", "clover_error_string", "clover_last_error", "clover_abi_version"]
 
 
@@ -129,8 +129,6 @@ def load(build_if_missing: bool = True):
         L.clover_debug_set_fusion.argtypes = [c_void_p, c_int32]
     if hasattr(L, "clover_debug_set_overlap"):
         L.clover_debug_set_overlap.argtypes = [c_void_p, c_int32]
-    if hasattr(L, "clover_debug_set_peer_halos"):
-        L.clover_debug_set_peer_halos.argtypes = [c_void_p, c_int32]
     L.clover_debug_div_check.argtypes = [c_int64, ctypes.c_uint64, c_int32, ctypes.POINTER(c_int64), dptr]
     L.clover_checkpoint_plan.argtypes = [c_int32, ctypes.POINTER(ctypes.c_uint32), ctypes.POINTER(c_int32),
                                          ctypes.POINTER(ctypes.c_char_p)]
@@ -371,11 +369,6 @@ class Clover:
         """Boundary segments first + the exchange overlapped with the interior
         (y strips with remote / virtual-remote exchanges; default off)."""
         _check(load().clover_debug_set_overlap(self._ctx, 1 if enable else 0), "clover_debug_set_overlap")
-
-    def debug_set_peer_halos(self, enable: bool):
-        """Device-initiated y-halo stores between local y-strip chunks (default on)."""
-        _check(load().clover_debug_set_peer_halos(self._ctx, 1 if enable else 0),
-               "clover_debug_set_peer_halos")
 
     def debug_fix_count(self) -> int:
         """Warp segments recomputed so far by the IEEE-division fixup launches."""

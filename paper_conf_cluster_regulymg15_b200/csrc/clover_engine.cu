@@ -103,7 +103,6 @@ struct ChunkState {
   int ntx, nty;
   FixSlot fix;       // warps to redo with IEEE division (clover_stream.cuh)
   FixSlot fix_b;     // the same for boundary segments running beside the interior (run_phase)
-  PeerY peer{0, 0};  // device-initiated y-halo stores to local neighbours (peer_halos_ok)
   CUtensorMap tm_lag;   // d0 e0 u0 v0 q as one {pitch, rows, 5} fp64 tensor, box {LRW, 1, 5}
   CUtensorMap tm_visc;  // d0 e0 u0 v0 as {pitch, rows, 4}, box {VRW, 1, 4}
   CUtensorMap tm_x1;    // d1 e1 u1 v1 fy fx, box {XRW, 1, 6} (fused x sweep 1)
@@ -253,7 +252,6 @@ struct clover_ctx {
   cudaStream_t comm_stream = nullptr, xs = nullptr;
   cudaEvent_t ev_b = nullptr, ev_x = nullptr;
   bool overlap = false;  // see overlap_ok
-  bool peer_halos = true;  // see peer_halos_ok
   cudaEvent_t ev_in = nullptr, ev_out = nullptr;
   StepScalars* scal = nullptr;
   double* hist = nullptr;
@@ -336,33 +334,18 @@ std::vector<int> local_chunk_ids(int px, int py, int rank, int nranks) {
   return ids;
 }
 
-// Every local chunk gets an equally sized block of the workspace (fields at
-// one common stride, then summary partials and the two fix lists), sized for
-// the largest chunk: the same field of two chunks is then a constant offset
-// apart, which the device-initiated halo stores use (PeerY).
-struct ChunkBlock { int64_t field, partials, fix; };
-ChunkBlock chunk_block(const Layout& L, int px, int py, int rank, int nranks) {
-  ChunkBlock b{0, 0, 0};
-  for (int id : local_chunk_ids(px, py, rank, nranks)) {
-    const int cx = id % px, cy = id / px;
-    const int nx = L.xs[cx + 1] - L.xs[cx], ny = L.ys[cy + 1] - L.ys[cy];
-    b.field = std::max(b.field, align_up(field_elems(nx, ny, nullptr) * 8, kAlign));
-    const int ntx = (nx + ST - 1) / ST, nty = (ny + ST - 1) / ST;
-    b.partials = std::max(b.partials, align_up((int64_t)ntx * nty * 5 * 8, kAlign));
-    b.fix = std::max(b.fix, fix_bytes(nx, ny));
-  }
-  return b;
-}
-
 int64_t compute_workspace(const clover_grid* g, int px, int py, int rank, int nranks) {
   Layout L = decompose(g->x_cells, g->y_cells, px, py);
   int64_t bytes = align_up(sizeof(StepScalars), kAlign) + align_up(DT_HIST * 8, kAlign);
   int64_t maxrows = 0, maxcols = 0;
-  const ChunkBlock blk = chunk_block(L, px, py, rank, nranks);
   for (int id : local_chunk_ids(px, py, rank, nranks)) {
     int cx = id % px, cy = id / px;
     int nx = L.xs[cx + 1] - L.xs[cx], ny = L.ys[cy + 1] - L.ys[cy];
-    bytes += NBUF * blk.field + blk.partials + 2 * blk.fix;
+    int64_t fe = field_elems(nx, ny, nullptr);
+    bytes += NBUF * align_up(fe * 8, kAlign);
+    int ntx = (nx + ST - 1) / ST, nty = (ny + ST - 1) / ST;
+    bytes += align_up((int64_t)ntx * nty * 5 * 8, kAlign);
+    bytes += 2 * fix_bytes(nx, ny);
     maxrows = std::max<int64_t>(maxrows, ny + 2 + 2 * HALO_ROWS);
     maxcols = std::max<int64_t>(maxcols, nx + 2 + 2 * HALO_COLS);
   }
@@ -769,17 +752,6 @@ bool overlap_ok(const clover_ctx* ctx) {
          (ctx->nranks > 1 || ctx->virtual_remote);
 }
 
-// Device-initiated halo stores (S:8(f) f1; PeerY in clover_common.cuh):
-// y strips of local chunks with both fused sweeps -- the Lagrangian and the
-// fused sweeps write their y neighbours' halo rows from their epilogues, and
-// those phases need no exchange.  (Several ranks would need each peer's
-// workspace mapped -- CUDA IPC or NCCL symmetric windows -- and a cross-GPU
-// flag per phase; not built: every box here has one GPU.)
-bool peer_halos_ok(const clover_ctx* ctx) {
-  return ctx->peer_halos && ctx->nranks == 1 && !ctx->virtual_remote && ctx->L.px == 1 &&
-         ctx->L.py > 1 && fuse_x_ok(ctx) && fuse_y_ok(ctx);
-}
-
 // Row-segment geometry of a streaming kernel kind on a chunk: rows per
 // segment, full-height segments, rows covered (seg_rows_of).
 enum { SEG_LAGR, SEG_X, SEG_Y };
@@ -857,8 +829,6 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
   // the comm stream, followed there by their fixup and the exchange, while
   // the interior segments run beside them on the work stream (own fix list);
   // the next phase waits for both.
-  const bool peers = peer_halos_ok(ctx);
-  auto peer_of = [&](const ChunkState& cs) { return peers ? cs.peer : PeerY{0, 0}; };
   auto run_phase = [&](int kind, auto&& launch, auto&& fixup, const std::vector<int>& bufs, int yd,
                        int xd) -> int {
     if (!overlap_ok(ctx)) {
@@ -871,8 +841,6 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
         if (!rc) rc = fixup(cs, c, st, cs.fix);
         if (rc) return rc;
       }
-      // the kernels wrote their neighbours' halo rows themselves
-      if (peer_halos_ok(ctx)) return CLOVER_OK;
       return exchange(ctx, bufs, yd, xd);
     }
     cudaStream_t cm = ctx->comm_stream;
@@ -953,7 +921,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
       c = with_rev(c, 0);
       launch_step(ks_lagrangian, dim3(grid_strip(c.nx, LW, c.ny, c.lks).x, n), SB, sm, c, cs.tm_lag,
           cs.buf[B_D1], cs.buf[B_E1], cs.buf[B_U1], cs.buf[B_V1], cs.buf[B_FX], cs.buf[B_FY],
-          ctx->scal, fx, peer_of(cs));
+          ctx->scal, fx);
       STEP_LAUNCH_CHECK();
       return CLOVER_OK;
     };
@@ -962,7 +930,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
       const YWalls yw = walls_in_lagr ? ywalls_of(cs, 1) : kNoWalls;
       launch_fix(kf_lagrangian, FIX_BLOCKS + 5 * yw.nbx, SB, sm, c, cs.tm_lag,
           cs.buf[B_D1], cs.buf[B_E1], cs.buf[B_U1], cs.buf[B_V1], cs.buf[B_FX], cs.buf[B_FY],
-          ctx->scal, fx, yw, peer_of(cs));
+          ctx->scal, fx, yw);
       FIX_LAUNCH_CHECK();
       return CLOVER_OK;
     };
@@ -992,10 +960,10 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
           const dim3 g(grid_strip(c.nx + 1, XW, c.ny + 1, c.xks).x, n);
           if (sweep == 1)
             launch_step(ks_advec_x<1>, g, SB, sm, c, cs.tm_x1, cs.buf[rout], cs.buf[eout],
-                        cs.buf[uout], cs.buf[vout], fx, peer_of(cs));
+                        cs.buf[uout], cs.buf[vout], fx);
           else
             launch_step(ks_advec_x<2>, g, SB, sm, c, cs.tm_x2, cs.buf[rout], cs.buf[eout],
-                        cs.buf[uout], cs.buf[vout], fx, peer_of(cs));
+                        cs.buf[uout], cs.buf[vout], fx);
           STEP_LAUNCH_CHECK();
           return CLOVER_OK;
         };
@@ -1004,10 +972,10 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
           if (sweep == 1) {
             const YWalls yw = walls_in_x1 ? ywalls_of(cs, 2) : kNoWalls;
             launch_fix(kf_advec_x<1>, FIX_BLOCKS + 5 * yw.nbx, SB, sm, c, cs.tm_x1, cs.buf[rout],
-                        cs.buf[eout], cs.buf[uout], cs.buf[vout], fx, yw, peer_of(cs));
+                        cs.buf[eout], cs.buf[uout], cs.buf[vout], fx, yw);
           } else {
             launch_fix(kf_advec_x<2>, FIX_BLOCKS, SB, sm, c, cs.tm_x2, cs.buf[rout], cs.buf[eout],
-                        cs.buf[uout], cs.buf[vout], fx, kNoWalls, peer_of(cs));
+                        cs.buf[uout], cs.buf[vout], fx, kNoWalls);
           }
           FIX_LAUNCH_CHECK();
           return CLOVER_OK;
@@ -1047,7 +1015,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
           const CUtensorMap& tb = sweep == 1 ? cs.tm_x1 : cs.tm_c4;
           if (sweep == 1) {
             launch_step(ks_advec_y<1>, g, SB, sm, c, ta, tb, cs.buf[rout], cs.buf[eout], cs.buf[B_MY],
-                        cs.buf[uout], cs.buf[vout], fx, peer_of(cs));
+                        cs.buf[uout], cs.buf[vout], fx);
           } else if (ctx->f2_probe) {
             // DESIGN.md 4.5 f2 probe: sweep 2 with the next step's viscosity
             // and calc_dt terms folded in (q written, dt to a scratch slot;
@@ -1060,7 +1028,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
                         cs.buf[B_MY], cs.buf[uout], cs.buf[vout], fx, vp);
           } else {
             launch_step(ks_advec_y<2>, g, SB, sm, c, ta, tb, cs.buf[rout], cs.buf[eout], cs.buf[B_MY],
-                        cs.buf[uout], cs.buf[vout], fx, peer_of(cs));
+                        cs.buf[uout], cs.buf[vout], fx);
           }
           STEP_LAUNCH_CHECK();
           return CLOVER_OK;
@@ -1071,10 +1039,10 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
           const CUtensorMap& tb = sweep == 1 ? cs.tm_x1 : cs.tm_c4;
           if (sweep == 1)
             launch_fix(kf_advec_y<1>, FIX_BLOCKS, SB, sm, c, ta, tb, cs.buf[rout], cs.buf[eout],
-                        cs.buf[B_MY], cs.buf[uout], cs.buf[vout], fx, peer_of(cs));
+                        cs.buf[B_MY], cs.buf[uout], cs.buf[vout], fx);
           else
             launch_fix(kf_advec_y<2>, FIX_BLOCKS, SB, sm, c, ta, tb, cs.buf[rout], cs.buf[eout],
-                        cs.buf[B_MY], cs.buf[uout], cs.buf[vout], fx, peer_of(cs));
+                        cs.buf[B_MY], cs.buf[uout], cs.buf[vout], fx);
           FIX_LAUNCH_CHECK();
           return CLOVER_OK;
         };
@@ -1527,7 +1495,6 @@ int clover_init(const clover_grid* grid, const clover_state* states, int32_t nst
   for (int r = 0; r < nranks; ++r)
     for (int id : local_chunk_ids(px, py, r, nranks)) ctx->owner[id] = r;
   int64_t maxrows = 0, maxcols = 0;
-  const ChunkBlock blk = chunk_block(ctx->L, px, py, rank, nranks);
   for (int id : local_chunk_ids(px, py, rank, nranks)) {
     ChunkState cs;
     cs.id = id; cs.cx = id % px; cs.cy = id / px;
@@ -1564,16 +1531,15 @@ int clover_init(const clover_grid* grid, const clover_state* states, int32_t nst
     c.rdx = 1.0 / dx; c.rdy = 1.0 / dy;
     c.r2dx = 1.0 / (dx + dx); c.r2dy = 1.0 / (dy + dy);
     c.rvol = 1.0 / (dx * dy); c.r2vol = 1.0 / (2.0 * (dx * dy));
-    (void)fe;
     for (int b = 0; b < NBUF; ++b) {
       cs.buf[b] = (double*)p + (int64_t)ROW0 * c.pitch + COL0;
-      p += blk.field;
+      p += align_up(fe * 8, kAlign);
     }
     {
       const double* base = cs.buf[B_D0] - (int64_t)ROW0 * c.pitch - COL0;
       const int rows = c.ny + 2 + 2 * HALO_ROWS;
-      const int64_t fs = blk.field;
-      int rc = encode_rows_map(&cs.tm_lag, base, c.pitch, rows, fs, LNF, LRW);
+      int rc = encode_rows_map(&cs.tm_lag, base, c.pitch, rows, align_up(fe * 8, kAlign), LNF, LRW);
+      const int64_t fs = align_up(fe * 8, kAlign);
       if (!rc) rc = encode_rows_map(&cs.tm_visc, base, c.pitch, rows, fs, VNF, VRW);
       if (!rc) rc = encode_rows_map(&cs.tm_x1, base + (B_D1 - B_D0) * (fs / 8), c.pitch, rows, fs,
                                     XF<1>::NF, XRW);
@@ -1587,27 +1553,16 @@ int clover_init(const clover_grid* grid, const clover_state* states, int32_t nst
     }
     cs.ntx = (c.nx + ST - 1) / ST; cs.nty = (c.ny + ST - 1) / ST;
     cs.partials = (double*)p;
-    p += blk.partials;
+    p += align_up((int64_t)cs.ntx * cs.nty * 5 * 8, kAlign);
     cs.fix.hdr = (unsigned*)p;
     cs.fix.e = (uint2*)(p + kAlign);
-    p += blk.fix;
+    p += fix_bytes(c.nx, c.ny);
     cs.fix_b.hdr = (unsigned*)p;
     cs.fix_b.e = (uint2*)(p + kAlign);
-    p += blk.fix;
+    p += fix_bytes(c.nx, c.ny);
     maxrows = std::max<int64_t>(maxrows, c.ny + 2 + 2 * HALO_ROWS);
     maxcols = std::max<int64_t>(maxcols, c.nx + 2 + 2 * HALO_COLS);
     ctx->chunks.push_back(cs);
-  }
-  // device-initiated y-halo offsets between local neighbour chunks (equal
-  // blocks, so one element offset per side serves every field)
-  for (auto& cs : ctx->chunks) {
-    const Chunk& c = cs.c;
-    for (auto& o : ctx->chunks) {
-      if (o.cx != cs.cx) continue;
-      const int64_t d = (int64_t)(o.buf[B_D0] - cs.buf[B_D0]);
-      if (o.cy == cs.cy - 1) cs.peer.dn = d + (int64_t)o.c.ny * c.pitch;  // my (j,k) -> its (j, k+ny_o)
-      if (o.cy == cs.cy + 1) cs.peer.up = d - (int64_t)c.ny * c.pitch;    // my (j,k) -> its (j, k-ny)
-    }
   }
   {
     // co-residency of the folded y-wall launches (kf_lagrangian, kf_advec_x<1>
@@ -1725,17 +1680,6 @@ int clover_debug_set_virtual_remote(clover_ctx* ctx, int32_t enable) {
   }
   ctx->virtual_remote = enable != 0;
   ctx->virtual_nccl = enable == 2;
-  for (int i = 0; i < 4; ++i)
-    if (ctx->gexec[i]) {
-      cudaGraphExecDestroy(ctx->gexec[i]);
-      ctx->gexec[i] = nullptr;
-    }
-  return CLOVER_OK;
-}
-
-int clover_debug_set_peer_halos(clover_ctx* ctx, int32_t enable) {
-  if (!ctx) return fail(CLOVER_ERR_ARG, "ctx is NULL");
-  ctx->peer_halos = enable != 0;
   for (int i = 0; i < 4; ++i)
     if (ctx->gexec[i]) {
       cudaGraphExecDestroy(ctx->gexec[i]);

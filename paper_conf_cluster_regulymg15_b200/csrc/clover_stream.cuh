@@ -498,7 +498,7 @@ __device__ __forceinline__ bool lagr_body(const Chunk& c, const CUtensorMap* __r
                                           double* __restrict__ fx, double* __restrict__ fy,
                                           const StepScalars* __restrict__ s, int gw, int k0,
                                           int k1, int lane, double* ring,
-                                          unsigned long long* bars, const PeerY& peer) {
+                                          unsigned long long* bars) {
   const int J0 = 1 + LW * gw;
   const int j = J0 - 1 + lane;
   if (J0 > c.nx) return false;  // whole warp beyond the chunk (rings are per warp)
@@ -683,20 +683,6 @@ __device__ __forceinline__ bool lagr_body(const Chunk& c, const CUtensorMap* __r
           store_field(c, v1, K_YVEL, j + 1, kc + 1, v1r_c);
         }
       }
-      if (EDGE && (peer.dn | peer.up) && (kc <= 4 || kc >= c.ny - 3)) {
-        // the y neighbours' halo rows, straight into their buffers (f1)
-        peer_put(c, peer, e1, K_CELL, j, kc, ev);
-        peer_put(c, peer, d1, K_CELL, j, kc, dvv);
-        peer_put(c, peer, fx, K_XFACE, j, kc, cx * lsum);
-        peer_put(c, peer, fy, K_YFACE, j, kc, cy * bsum);
-        peer_put(c, peer, u1, K_XVEL, j, kc, u1_m);
-        peer_put(c, peer, v1, K_YVEL, j, kc, v1_m);
-        if (j == c.nx) {
-          peer_put(c, peer, fx, K_XFACE, j + 1, kc, cx * rsum);
-          peer_put(c, peer, u1, K_XVEL, j + 1, kc, u1r_m);
-          peer_put(c, peer, v1, K_YVEL, j + 1, kc, v1r_m);
-        }
-      }
     }
     ph_m = ph; phl_m = phl;
     u1_m = u1_c; v1_m = v1_c; u1r_m = u1r_c; v1r_m = v1r_c;
@@ -733,18 +719,17 @@ __device__ __forceinline__ bool lagr_seg(const Chunk& c, const CUtensorMap* __re
                                          double* __restrict__ u1, double* __restrict__ v1,
                                          double* __restrict__ fx, double* __restrict__ fy,
                                          const StepScalars* __restrict__ s, int gw, int k0, int k1,
-                                         int lane, double* ring, unsigned long long* bars,
-                                         const PeerY& peer) {
+                                         int lane, double* ring, unsigned long long* bars) {
   if (lagr_interior(c, gw, k0, k1))
-    return lagr_body<D, false>(c, tm, d1, e1, u1, v1, fx, fy, s, gw, k0, k1, lane, ring, bars, peer);
-  return lagr_body<D, true>(c, tm, d1, e1, u1, v1, fx, fy, s, gw, k0, k1, lane, ring, bars, peer);
+    return lagr_body<D, false>(c, tm, d1, e1, u1, v1, fx, fy, s, gw, k0, k1, lane, ring, bars);
+  return lagr_body<D, true>(c, tm, d1, e1, u1, v1, fx, fy, s, gw, k0, k1, lane, ring, bars);
 }
 
 __global__ void LB_HEAVY
 ks_lagrangian(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__ d1,
               double* __restrict__ e1, double* __restrict__ u1, double* __restrict__ v1,
               double* __restrict__ fx, double* __restrict__ fy, const StepScalars* __restrict__ s,
-              FixSlot fix, PeerY peer) {
+              FixSlot fix) {
   pdl_trigger();
   pdl_wait();
   __shared__ __align__(128) double ring[SB / 32][LSTG * LSLOT];
@@ -754,7 +739,7 @@ ks_lagrangian(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restric
   int k0, len;
   seg_rows_of(seg_y(c), c.lks, c.lnb, k0, len);
   const int k1 = min(k0 + len, c.ny + 1);
-  if (lagr_seg<DivFast>(c, &tm, d1, e1, u1, v1, fx, fy, s, gw, k0, k1, lane, ring[w], bars[w], peer))
+  if (lagr_seg<DivFast>(c, &tm, d1, e1, u1, v1, fx, fy, s, gw, k0, k1, lane, ring[w], bars[w]))
     fix_push(fix, lane, gw, (unsigned)seg_y(c));
 }
 
@@ -762,7 +747,7 @@ __global__ void __launch_bounds__(SB)
 kf_lagrangian(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__ d1,
               double* __restrict__ e1, double* __restrict__ u1, double* __restrict__ v1,
               double* __restrict__ fx, double* __restrict__ fy, StepScalars* __restrict__ s,
-              FixSlot fix, YWalls yw, PeerY peer) {
+              FixSlot fix, YWalls yw) {
   pdl_trigger();
   pdl_wait();
   if (y_walls_after_fix<1>(c, fix, yw)) return;
@@ -770,7 +755,7 @@ kf_lagrangian(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restric
   __shared__ __align__(8) unsigned long long bars[SB / 32][LSTG];
   fix_loop(fix, c.lks, c.lnb, c.ny + 1, [&](int gw, int k0, int k1, int lane, int w) {
     // the IEEE redo's flag is the exact PdV volume test (DivIEEE::vol_check)
-    if (lagr_seg<DivIEEE>(c, &tm, d1, e1, u1, v1, fx, fy, s, gw, k0, k1, lane, ring[w], bars[w], peer) &&
+    if (lagr_seg<DivIEEE>(c, &tm, d1, e1, u1, v1, fx, fy, s, gw, k0, k1, lane, ring[w], bars[w]) &&
         lane == 0)
       atomicCAS(&s->err, 0, -6);  // CLOVER_ERR_NEG_VOLUME
   });
@@ -1139,8 +1124,7 @@ __device__ __forceinline__ bool advec_x_body(const Chunk& c, const CUtensorMap* 
                                              double* __restrict__ en_out,
                                              double* __restrict__ uout,
                                              double* __restrict__ vout, int gw, int k0, int k1,
-                                             int lane, double* ring, unsigned long long* bars,
-                                             const PeerY& peer) {
+                                             int lane, double* ring, unsigned long long* bars) {
   using F = XF<SWEEP>;
   constexpr int SL = xslot<SWEEP>();
   constexpr unsigned BYTES = F::NF * XRW * 8;
@@ -1254,10 +1238,6 @@ __device__ __forceinline__ bool advec_x_body(const Chunk& c, const CUtensorMap* 
             const bool near = EDGE && (ncol || near_wall_row(c, r));
             store_at(c, rho_out, K_CELL, j, r, i, near, ro);
             store_at(c, en_out, K_CELL, j, r, i, near, eo);
-            if (EDGE && (peer.dn | peer.up)) {
-              peer_put(c, peer, rho_out, K_CELL, j, r, ro);
-              peer_put(c, peer, en_out, K_CELL, j, r, eo);
-            }
           }
         }
         mA = m;
@@ -1307,10 +1287,6 @@ __device__ __forceinline__ bool advec_x_body(const Chunk& c, const CUtensorMap* 
           const bool near = EDGE && (ncol || near_wall_row(c, r));
           store_at(c, uout, K_XVEL, j, r, i, near, un);
           store_at(c, vout, K_YVEL, j, r, i, near, vn);
-          if (EDGE && (peer.dn | peer.up)) {
-            peer_put(c, peer, uout, K_XVEL, j, r, un);
-            peer_put(c, peer, vout, K_YVEL, j, r, vn);
-          }
         }
       }
       mA_m = mA; mB_m = mB; mp_m = mp; mpl_m = mpl; ro_m = ro;
@@ -1347,19 +1323,19 @@ __device__ __forceinline__ bool advec_x_seg(const Chunk& c, const CUtensorMap* _
                                             double* __restrict__ en_out,
                                             double* __restrict__ uout, double* __restrict__ vout,
                                             int gw, int k0, int k1, int lane, double* ring,
-                                            unsigned long long* bars, const PeerY& peer) {
+                                            unsigned long long* bars) {
   if (x_interior(c, gw, k0, k1))
     return advec_x_body<SWEEP, D, false>(c, tm, rho_out, en_out, uout, vout, gw, k0, k1, lane,
-                                         ring, bars, peer);
+                                         ring, bars);
   return advec_x_body<SWEEP, D, true>(c, tm, rho_out, en_out, uout, vout, gw, k0, k1, lane, ring,
-                                      bars, peer);
+                                      bars);
 }
 
 template <int SWEEP>
 __global__ void LB_ADVX
 ks_advec_x(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__ rho_out,
            double* __restrict__ en_out, double* __restrict__ uout, double* __restrict__ vout,
-           FixSlot fix, PeerY peer) {
+           FixSlot fix) {
   pdl_trigger();
   pdl_wait();
   __shared__ __align__(128) double ring[SB / 32][XSTG * xslot<SWEEP>()];
@@ -1370,7 +1346,7 @@ ks_advec_x(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__
   seg_rows_of(seg_y(c), c.xks, c.xnb, k0, len);
   const int k1 = min(k0 + len, c.ny + 2);
   if (advec_x_seg<SWEEP, DivFast>(c, &tm, rho_out, en_out, uout, vout, gw, k0, k1, lane, ring[w],
-                                   bars[w], peer))
+                                   bars[w]))
     fix_push(fix, lane, gw, (unsigned)seg_y(c));
 }
 
@@ -1378,7 +1354,7 @@ template <int SWEEP>
 __global__ void __launch_bounds__(SB)
 kf_advec_x(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__ rho_out,
            double* __restrict__ en_out, double* __restrict__ uout, double* __restrict__ vout,
-           FixSlot fix, YWalls yw, PeerY peer) {
+           FixSlot fix, YWalls yw) {
   pdl_trigger();
   pdl_wait();
   if constexpr (SWEEP == 1)  // sweep 2 is y
@@ -1387,7 +1363,7 @@ kf_advec_x(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__
   __shared__ __align__(8) unsigned long long bars[SB / 32][XSTG];
   fix_loop(fix, c.xks, c.xnb, c.ny + 2, [&](int gw, int k0, int k1, int lane, int w) {
     advec_x_seg<SWEEP, DivIEEE>(c, &tm, rho_out, en_out, uout, vout, gw, k0, k1, lane, ring[w],
-                                 bars[w], peer);
+                                 bars[w]);
   });
 }
 
@@ -1585,7 +1561,7 @@ __device__ __forceinline__ bool advec_y_body(const Chunk& c, const CUtensorMap* 
                                              double* __restrict__ uout,
                                              double* __restrict__ vout, int gw, int k0, int k1,
                                              int lane, double* ring, unsigned long long* bars,
-                                             const PeerY& peer, const ViscProbe& vp = ViscProbe{}) {
+                                             const ViscProbe& vp = ViscProbe{}) {
   using L = YL<SWEEP>;
   D dv;
   const int J0 = 1 + YW * gw;
@@ -1742,10 +1718,6 @@ __device__ __forceinline__ bool advec_y_body(const Chunk& c, const CUtensorMap* 
             const bool near = EDGE && (ncol || near_wall_row(c, s));
             store_at(c, rho_out, K_CELL, j, s, i, near, ro);
             store_at(c, en_out, K_CELL, j, s, i, near, eo);
-            if (EDGE && (peer.dn | peer.up)) {
-              peer_put(c, peer, rho_out, K_CELL, j, s, ro);
-              peer_put(c, peer, en_out, K_CELL, j, s, eo);
-            }
           }
         }
       } else {
@@ -1788,10 +1760,6 @@ __device__ __forceinline__ bool advec_y_body(const Chunk& c, const CUtensorMap* 
           const bool near = EDGE && (ncol || near_wall_row(c, kn));
           store_at(c, uout, K_XVEL, j, kn, i, near, un);
           store_at(c, vout, K_YVEL, j, kn, i, near, vn);
-          if (EDGE && (peer.dn | peer.up)) {
-            peer_put(c, peer, uout, K_XVEL, j, kn, un);
-            peer_put(c, peer, vout, K_YVEL, j, kn, vn);
-          }
         }
         mu_b = mu_c; mv_b = mv_c;
       }
@@ -1863,19 +1831,19 @@ __device__ __forceinline__ bool advec_y_seg(const Chunk& c, const CUtensorMap* t
                                             const CUtensorMap* tb, double* rho_out, double* en_out,
                                             const double* mfy, double* uout, double* vout, int gw,
                                             int k0, int k1, int lane, double* ring,
-                                            unsigned long long* bars, const PeerY& peer) {
+                                            unsigned long long* bars) {
   if (y_fused_interior(c, gw, k0, k1))
     return advec_y_body<SWEEP, D, false>(c, ta, tb, rho_out, en_out, mfy, uout, vout, gw, k0, k1,
-                                         lane, ring, bars, peer);
+                                         lane, ring, bars);
   return advec_y_body<SWEEP, D, true>(c, ta, tb, rho_out, en_out, mfy, uout, vout, gw, k0, k1,
-                                      lane, ring, bars, peer);
+                                      lane, ring, bars);
 }
 
 template <int SWEEP>
 __global__ void __launch_bounds__(SB, YL<SWEEP>::MINB)
 ks_advec_y(Chunk c, const __grid_constant__ CUtensorMap ta, const __grid_constant__ CUtensorMap tb,
            double* __restrict__ rho_out, double* __restrict__ en_out, const double* __restrict__ mfy,
-           double* __restrict__ uout, double* __restrict__ vout, FixSlot fix, PeerY peer) {
+           double* __restrict__ uout, double* __restrict__ vout, FixSlot fix) {
   pdl_trigger();
   pdl_wait();
   __shared__ __align__(128) double ring[SB / 32][YL<SWEEP>::RING * YL<SWEEP>::SLOT];
@@ -1886,7 +1854,7 @@ ks_advec_y(Chunk c, const __grid_constant__ CUtensorMap ta, const __grid_constan
   seg_rows_of(seg_y(c), c.yks, c.ynb, k0, len);
   const int k1 = min(k0 + len, c.ny + 2);
   if (advec_y_seg<SWEEP, DivFast>(c, &ta, &tb, rho_out, en_out, mfy, uout, vout, gw, k0, k1, lane,
-                                  ring[w], bars[w], peer))
+                                  ring[w], bars[w]))
     fix_push(fix, lane, gw, (unsigned)seg_y(c));
 }
 
@@ -1910,10 +1878,10 @@ ks_advec_y2_probe(Chunk c, const __grid_constant__ CUtensorMap ta,
   bool bad;
   if (y_fused_interior(c, gw, k0, k1))
     bad = advec_y_body<2, DivFast, false, true>(c, &ta, &tb, rho_out, en_out, mfy, uout, vout, gw,
-                                                k0, k1, lane, ring[w], bars[w], PeerY{0, 0}, vp);
+                                                k0, k1, lane, ring[w], bars[w], vp);
   else
     bad = advec_y_body<2, DivFast, true>(c, &ta, &tb, rho_out, en_out, mfy, uout, vout, gw, k0, k1,
-                                         lane, ring[w], bars[w], PeerY{0, 0});
+                                         lane, ring[w], bars[w]);
   if (bad) fix_push(fix, lane, gw, (unsigned)seg_y(c));
 }
 
@@ -1921,14 +1889,14 @@ template <int SWEEP>
 __global__ void __launch_bounds__(SB)
 kf_advec_y(Chunk c, const __grid_constant__ CUtensorMap ta, const __grid_constant__ CUtensorMap tb,
            double* __restrict__ rho_out, double* __restrict__ en_out, const double* __restrict__ mfy,
-           double* __restrict__ uout, double* __restrict__ vout, FixSlot fix, PeerY peer) {
+           double* __restrict__ uout, double* __restrict__ vout, FixSlot fix) {
   pdl_trigger();
   pdl_wait();
   __shared__ __align__(128) double ring[SB / 32][YL<SWEEP>::RING * YL<SWEEP>::SLOT];
   __shared__ __align__(8) unsigned long long bars[SB / 32][YL<SWEEP>::RING];
   fix_loop(fix, c.yks, c.ynb, c.ny + 2, [&](int gw, int k0, int k1, int lane, int w) {
     advec_y_seg<SWEEP, DivIEEE>(c, &ta, &tb, rho_out, en_out, mfy, uout, vout, gw, k0, k1, lane,
-                                ring[w], bars[w], peer);
+                                ring[w], bars[w]);
   });
 }
 

@@ -23,9 +23,8 @@ deck = bm_deck(nx, ny, end_step=steps, ymax=10.0 * ny / nx)
 # (square cells: the domain grows with the mesh)
 
 
-def run(p, q, vr=0, walls_only=False, overlap=False, peers=True):
+def run(p, q, vr=0, walls_only=False, overlap=False):
     sim = Clover(deck, px=p, py=q)
-    sim.debug_set_peer_halos(peers)
     if walls_only:
         sim.debug_set_fusion(True, walls_only=True)
     if vr:
@@ -59,8 +58,7 @@ res["rank_chunk"] = [cx, cy]
 res["rank_chunk_alone_ms"] = alone
 res["serial_ideal_ms"] = alone * px * py
 res["strong_scaling_efficiency_bound"] = one / (px * py * alone)
-for name, kw in (("local_fused", {}), ("local_exchange", dict(peers=False)),
-                 ("local_walls_only", dict(walls_only=True)),
+for name, kw in (("local_fused", {}), ("local_walls_only", dict(walls_only=True)),
                  ("virtual_remote", dict(vr=1)), ("virtual_nccl", dict(vr=2)),
                  ("virtual_remote_overlap", dict(vr=1, overlap=True)),
                  ("virtual_nccl_overlap", dict(vr=2, overlap=True))):

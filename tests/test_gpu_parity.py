@@ -383,29 +383,6 @@ def test_virtual_remote_through_nccl_bitwise(torch_cuda, pxy):
     assert many.field_summary() == one.field_summary()
 
 
-@pytest.mark.parametrize("seed,py", [(17, 2), (18, 3), (19, 6)])
-def test_device_initiated_halo_stores_bitwise(torch_cuda, seed, py):
-    """S:8(f) f1: with y strips of local chunks the Lagrangian and both fused
-    sweeps write their neighbours' halo rows from their epilogues (no
-    exchange phase).  Same bits as the exchange path and as one chunk,
-    fields and dt history, both sweep orders (fuzz decks with flow across
-    the strip boundaries; 6 strips of 12-13 rows reach the 4-row bands from
-    both sides)."""
-    deck = fuzz_deck(seed, nx=70, ny=76)
-    deck["max_timestep"] = 1.0
-    one = make_gpu(deck)
-    peer = make_gpu(deck, px=1, py=py)
-    exch = make_gpu(deck, px=1, py=py)
-    exch.debug_set_peer_halos(False)
-    for g in (one, peer, exch):
-        g.step(10)
-    for f in STATE:
-        a = one.read(f)
-        assert np.array_equal(peer.read(f), a), f
-        assert np.array_equal(exch.read(f), a), f
-    assert np.array_equal(peer.dt_history(1, 10), one.dt_history(1, 10))
-
-
 @pytest.mark.parametrize("nccl", [False, True])
 @pytest.mark.parametrize("py", [2, 3, 5])
 def test_boundary_first_overlap_bitwise(torch_cuda, nccl, py):
