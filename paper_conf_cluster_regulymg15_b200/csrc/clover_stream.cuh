@@ -1210,9 +1210,12 @@ __device__ __forceinline__ bool advec_x_body(const Chunk& c, const CUtensorMap* 
             pv = vol + fhi - flo;
           rr = rc[F::R * XRW]; ee = rc[F::E * XRW];
         }
-        double pvl = __shfl_up_sync(FULL, pv, 1);
         if (faceok) {
-          if (lane == 0) {
+          // pre_vol of cell j-1 from the ring (the same expression lane j-1
+          // evaluates: same bits; cheaper than a 64-bit shuffle plus a
+          // divergent lane-0 path)
+          double pvl;
+          {
             const double fl = rc[F::FX * XRW - 1];
             if constexpr (SWEEP == 1)
               pvl = vol + (flo - fl + rn[F::FY * XRW - 1] - rc[F::FY * XRW - 1]);
