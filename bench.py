@@ -350,6 +350,7 @@ def main():
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
+    nl0 = sim.launch_count()
     e0.record(stream)
     sim.step(args.steps)
     e1.record(stream)
@@ -361,7 +362,7 @@ def main():
     sim.sync()
     ms = cdist.max_over_ranks(ms, None if host_tp else dev)
     value = cells * args.steps / (ms / 1000.0)
-    kps = sim.kernels_per_step()
+    launches = sim.launch_count() - nl0  # counted by the engine, graph launches included
 
     # per-kernel CUDA-event durations over a second pass of K steps on the
     # same stream (direct launches, event after every kernel)
@@ -514,7 +515,7 @@ def main():
                            if world > 1 else None,
                            "l2": "inputs larger than L2 (18 fp64 fields of the mesh, >2 GB vs 126 MB L2)",
                            "graphs": True},
-                "gpu_launches": kps * args.steps,
+                "gpu_launches": launches,
                 "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "clocks": clk,
                 "kernels": kernels,
                 "active_flow": active,

@@ -225,6 +225,13 @@ int clover_set_graphs(clover_ctx* ctx, int32_t enable);
 /* Number of CUDA kernels one clover_step(ctx, 1) launches on this rank. */
 int clover_kernels_per_step(clover_ctx* ctx, int32_t* out);
 
+/* Step kernels (streaming kernels, IEEE fixups, wall bands; not the halo
+ * strip copies) launched on this context so far by clover_step,
+ * clover_profile_steps and clover_debug_partial_step; a graph launch counts
+ * the kernels captured in it.  The bench's gpu_launches is the difference
+ * across its timed region. */
+int clover_launch_count(clover_ctx* ctx, int64_t* out);
+
 /* Profiling: run nsteps full steps with direct launches and a CUDA event
  * after every kernel on the context's work stream; ms_out[i] / launches_out[i]
  * receive the summed duration and launch count of kernel type i

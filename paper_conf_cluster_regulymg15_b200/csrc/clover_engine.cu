@@ -272,6 +272,8 @@ struct clover_ctx {
   bool walls_fold_fits = false;
   bool f2_probe = false;  // CLOVER_F2_PROBE=1 at init: sweep-2 y kernel with the visc epilogue (A/B only)
   cudaGraphExec_t gexec[4] = {nullptr, nullptr, nullptr, nullptr};  // [parity + 2 * multi-step]
+  int graph_launches[4] = {0, 0, 0, 0};  // kernels captured in gexec[i]
+  int64_t launches = 0;  // step kernels launched so far (clover_launch_count)
   int64_t ws_bytes = 0;
   bool prof = false;
   bool virtual_remote = false;  // test mode: every chunk boundary takes the NCCL packing path
@@ -643,6 +645,7 @@ dim3 cell_grid(const Chunk& c, int bx, int by) { return dim3((c.nx + bx - 1) / b
 #define STEP_LAUNCH_CHECK()                                                       \
   do {                                                                            \
     LAUNCH_CHECK();                                                               \
+    ++ctx->launches;                                                              \
     if (ctx->prof) prof_mark(ctx, cur_prof_id);                                   \
   } while (0)
 // after a fixup launch: its time joins the phase, it is not counted as a launch
@@ -650,6 +653,7 @@ constexpr int PROF_FIXUP = 0x100;
 #define FIX_LAUNCH_CHECK()                                                        \
   do {                                                                            \
     LAUNCH_CHECK();                                                               \
+    ++ctx->launches;                                                              \
     if (ctx->prof) prof_mark(ctx, cur_prof_id | PROF_FIXUP);                      \
   } while (0)
 
@@ -1162,7 +1166,10 @@ int build_graph(clover_ctx* ctx, int parity, int nst, int slot) {
   cudaGraph_t graph = nullptr;
   CK(cudaStreamBeginCapture(ctx->work, cudaStreamCaptureModeThreadLocal));
   int rc = 0;
+  const int64_t n0 = ctx->launches;  // captured, not launched: counted per graph launch
   for (int i = 0; i < nst && !rc; ++i) rc = enqueue_step(ctx, (parity == 0) != (i % 2 == 1), 7);
+  ctx->graph_launches[slot] = (int)(ctx->launches - n0);
+  ctx->launches = n0;
   cudaError_t e = cudaStreamEndCapture(ctx->work, &graph);
   if (rc) {
     if (graph) cudaGraphDestroy(graph);
@@ -1789,6 +1796,7 @@ int clover_step(clover_ctx* ctx, int32_t nsteps) {
       }
       if (cudaGraphLaunch(ctx->gexec[slot], ctx->work) != cudaSuccess)
         return bail(fail(CLOVER_ERR_CUDA, "cudaGraphLaunch failed"));
+      ctx->launches += ctx->graph_launches[slot];
       i += CLOVER_GRAPH_STEPS - 1;
       if (CLOVER_GRAPH_STEPS % 2) ctx->advect_x = !ctx->advect_x;
       continue;
@@ -1800,6 +1808,7 @@ int clover_step(clover_ctx* ctx, int32_t nsteps) {
       }
       if (cudaGraphLaunch(ctx->gexec[parity], ctx->work) != cudaSuccess)
         return bail(fail(CLOVER_ERR_CUDA, "cudaGraphLaunch failed"));
+      ctx->launches += ctx->graph_launches[parity];
     } else {
       rc = enqueue_step(ctx, ctx->advect_x, 7);
       if (rc) return bail(rc);
@@ -1807,6 +1816,12 @@ int clover_step(clover_ctx* ctx, int32_t nsteps) {
     ctx->advect_x = !ctx->advect_x;
   }
   return join_out(ctx);
+}
+
+int clover_launch_count(clover_ctx* ctx, int64_t* out) {
+  if (!ctx || !out) return fail(CLOVER_ERR_ARG, "NULL argument");
+  *out = ctx->launches;
+  return CLOVER_OK;
 }
 
 int clover_profile_steps(clover_ctx* ctx, int32_t nsteps, double* ms_out, int64_t* launches_out,

@@ -628,3 +628,11 @@ def test_kernels_per_step(torch_cuda, pxy, expected):
     px, py = pxy
     g = make_gpu(fuzz_deck(11), px=px, py=py)
     assert g.kernels_per_step() == expected
+    # the engine's own launch counter (clover_launch_count, the bench's
+    # gpu_launches) agrees, through graph launches and direct launches
+    n0 = g.launch_count()
+    g.step(3)
+    assert g.launch_count() - n0 == 3 * expected
+    g.set_graphs(False)
+    g.step(2)
+    assert g.launch_count() - n0 == 5 * expected
