@@ -261,6 +261,19 @@ int clover_debug_partial_step(clover_ctx* ctx, int32_t nkernels);
 int clover_debug_read_buffer(clover_ctx* ctx, int32_t buffer_id, int32_t kind,
                              double* host, int64_t n);
 
+/* Deep halos (S:8(f) f1): on y-strip layouts (px == 1,
+ * py > 1, every chunk >= 16 rows, both fused sweeps) the state is exchanged
+ * once per step, 7 rows deep, and each kernel of the step also computes the
+ * rows of its y neighbours it would otherwise receive (visc_dt and the
+ * Lagrangian phase 5 rows beyond each non-wall y side, sweep 1 4 (x) or 1
+ * (y)), so a step has one halo exchange plus the dt MIN instead of three.
+ * Results are bitwise identical either way.  enable = 1 / 0 (default 1, or
+ * the environment's CLOVER_DEEP_HALO at clover_init); where the layout does
+ * not qualify the setting has no effect.  clover_deep_halo_active reports
+ * whether the next step uses it. */
+int clover_set_deep_halo(clover_ctx* ctx, int32_t enable);
+int clover_deep_halo_active(clover_ctx* ctx, int32_t* out);
+
 /* Boundary-first overlap (S:8(e)): for y-strip layouts (px == 1) whose
  * exchanges take the remote path (several ranks, or virtual-remote mode),
  * each fused kernel runs the row segments next to a y chunk boundary first,

@@ -41,6 +41,7 @@ EXPORTS = ["clover_workspace_bytes", "clover_nccl_unique_id", "clover_init", "cl
            "clover_kernels_per_step", "clover_launch_count", "clover_debug_partial_step", "clover_debug_read_buffer",
            "clover_profile_steps", "clover_profile_name", "clover_debug_div_check",
            "clover_debug_fix_count", "clover_debug_set_fusion", "clover_debug_set_overlap",
+           "clover_set_deep_halo", "clover_deep_halo_active",
            "clover_checkpoint_plan", "clover_debug_set_virtual_remote", "clover_checkpoint_bytes", "clover_checkpoint", "clover_restart", "clover_finalize", "clover_error_string", "clover_last_error", "clover_abi_version"]
 
 
@@ -118,7 +119,8 @@ def load(build_if_missing: bool = True):
     L.clover_sync.argtypes = [c_void_p]
     L.clover_set_graphs.argtypes = [c_void_p, c_int32]
     L.clover_kernels_per_step.argtypes = [c_void_p, P(c_int32)]
-    L.clover_launch_count.argtypes = [c_void_p, P(ctypes.c_int64)]
+    if hasattr(L, "clover_launch_count"):
+        L.clover_launch_count.argtypes = [c_void_p, P(ctypes.c_int64)]
     L.clover_debug_partial_step.argtypes = [c_void_p, c_int32]
     L.clover_debug_read_buffer.argtypes = [c_void_p, c_int32, c_int32, dptr, c_int64]
     L.clover_profile_steps.argtypes = [c_void_p, c_int32, dptr, ctypes.POINTER(c_int64), c_int32]
@@ -130,6 +132,9 @@ def load(build_if_missing: bool = True):
         L.clover_debug_set_fusion.argtypes = [c_void_p, c_int32]
     if hasattr(L, "clover_debug_set_overlap"):
         L.clover_debug_set_overlap.argtypes = [c_void_p, c_int32]
+    if hasattr(L, "clover_set_deep_halo"):  # (older A/B builds lack the newer calls)
+        L.clover_set_deep_halo.argtypes = [c_void_p, c_int32]
+        L.clover_deep_halo_active.argtypes = [c_void_p, P(c_int32)]
     L.clover_debug_div_check.argtypes = [c_int64, ctypes.c_uint64, c_int32, ctypes.POINTER(c_int64), dptr]
     L.clover_checkpoint_plan.argtypes = [c_int32, ctypes.POINTER(ctypes.c_uint32), ctypes.POINTER(c_int32),
                                          ctypes.POINTER(ctypes.c_char_p)]
@@ -376,6 +381,16 @@ class Clover:
         """Boundary segments first + the exchange overlapped with the interior
         (y strips with remote / virtual-remote exchanges; default off)."""
         _check(load().clover_debug_set_overlap(self._ctx, 1 if enable else 0), "clover_debug_set_overlap")
+
+    def set_deep_halo(self, enable: bool):
+        """Deep halos (one 7-row state exchange per step on y-strip layouts;
+        include/clover.h clover_set_deep_halo)."""
+        _check(load().clover_set_deep_halo(self._ctx, 1 if enable else 0), "clover_set_deep_halo")
+
+    def deep_halo_active(self) -> bool:
+        n = c_int32()
+        _check(load().clover_deep_halo_active(self._ctx, ctypes.byref(n)), "clover_deep_halo_active")
+        return bool(n.value)
 
     def debug_fix_count(self) -> int:
         """Warp segments recomputed so far by the IEEE-division fixup launches."""

@@ -189,6 +189,15 @@ int tail_nb(int ks, int64_t colblocks, int rows, int64_t slots) {
   if (rows <= tail_rows) return 0;
   return (int)((rows - tail_rows) / ks);
 }
+// Deep halos (deep_ok below): state exchange depth, row extension of each
+// phase's view beyond the chunk, minimum chunk height.
+constexpr int DEEP_ROWS = 7;
+constexpr int DEEP_EXT_VISC = 5, DEEP_EXT_LAGR = 5, DEEP_EXT_X1 = 4, DEEP_EXT_Y1 = 1;
+constexpr int DEEP_EXT_MAX = 5;
+constexpr int DEEP_MIN_NY = 16;
+static_assert(DEEP_ROWS + 1 <= HALO_ROWS, "deep state halo allocated");
+// (fix lists hold every warp segment of the largest kernel grid, views
+// included: callers pass ny + 2 * DEEP_EXT_MAX)
 int64_t fix_capacity(int nx, int ny) {
   // (adaptive segments: tail segments have at least 4 rows, see tail_nb)
   const dim3 g[8] = {grid_cols(nx, ny, 4),          grid_strip(nx, LW, ny, 4),
@@ -271,6 +280,9 @@ struct clover_ctx {
   // until the fixup blocks are done (clover_init checks the occupancy)
   bool walls_fold_fits = false;
   bool f2_probe = false;  // CLOVER_F2_PROBE=1 at init: sweep-2 y kernel with the visc epilogue (A/B only)
+  bool deep = true;       // deep halos where they apply (deep_ok; clover_set_deep_halo)
+  int nsm = 148, occ[4] = {1, 1, 1, 1};  // SMs, resident blocks/SM of the 4 segment kernels (set_segs)
+  int state_rows = 0;     // rows of the state's y halo known current (ensure_state_rows)
   cudaGraphExec_t gexec[4] = {nullptr, nullptr, nullptr, nullptr};  // [parity + 2 * multi-step]
   int graph_launches[4] = {0, 0, 0, 0};  // kernels captured in gexec[i]
   int64_t launches = 0;  // step kernels launched so far (clover_launch_count)
@@ -347,7 +359,7 @@ int64_t compute_workspace(const clover_grid* g, int px, int py, int rank, int nr
     bytes += NBUF * align_up(fe * 8, kAlign);
     int ntx = (nx + ST - 1) / ST, nty = (ny + ST - 1) / ST;
     bytes += align_up((int64_t)ntx * nty * 5 * 8, kAlign);
-    bytes += 2 * fix_bytes(nx, ny);
+    bytes += 2 * fix_bytes(nx, ny + 2 * DEEP_EXT_MAX);
     maxrows = std::max<int64_t>(maxrows, ny + 2 + 2 * HALO_ROWS);
     maxcols = std::max<int64_t>(maxcols, nx + 2 + 2 * HALO_COLS);
   }
@@ -418,9 +430,9 @@ struct StripQueue {
 
 // strips for side `side` (0 left, 1 right, 2 bottom, 3 top) of chunk cs:
 // send = owned points next to that side, recv = halo points of that side.
-// x sides are `xdepth` columns deep, y sides `ydepth` rows: HALO, or 4
-// (HALO_COLS / HALO_ROWS) for the inputs of a fused sweep across a chunk
-// boundary.
+// x sides are `xdepth` columns deep, y sides `ydepth` rows: HALO, 4
+// (HALO_COLS / FUSE_ROWS) for the inputs of a fused sweep across a chunk
+// boundary, or DEEP_ROWS for the state with deep halos.
 void side_strips(const ChunkState& cs, int buf, int side, XferDesc& send, XferDesc& recv,
                  int ydepth = HALO, int xdepth = HALO) {
   const Chunk& c = cs.c;
@@ -733,7 +745,7 @@ bool fuse_x_ok(const clover_ctx* ctx) {
 
 // The fused y sweep (reach 4 rows along y) runs at y walls (the mirrored
 // halo rows come from the band kernel) and at y chunk boundaries (its inputs
-// exchanged HALO_ROWS deep, the neighbour's first rows recomputed: SURVEY
+// exchanged FUSE_ROWS deep, the neighbour's first rows recomputed: SURVEY
 // 8(e) H1/H2); it needs the geometric face mirror.  fuse_y_chunks = false
 // keeps the separate cell / momentum kernels at y chunk boundaries (A/B and
 // tests).
@@ -751,9 +763,70 @@ bool fuse_y_ok(const clover_ctx* ctx) {
 // (px == 1; x strips would need every row) whose exchanges leave the GPU
 // (several ranks over NCCL) or take the remote path in virtual-remote mode.
 // The host transport is synchronous, so it gains nothing there.
+bool deep_ok(const clover_ctx* ctx);
 bool overlap_ok(const clover_ctx* ctx) {
   return ctx->overlap && ctx->L.px == 1 && ctx->L.py > 1 && !ctx->use_ht &&
-         (ctx->nranks > 1 || ctx->virtual_remote);
+         (ctx->nranks > 1 || ctx->virtual_remote) && !deep_ok(ctx);
+}
+
+// ---------------------------------------------------------------- deep halos
+// S:8(f) f1, communication-avoiding halos: the state (d0 e0 u0 v0) is
+// exchanged once per step, DEEP_ROWS deep, and every kernel of the step runs
+// over rows beyond its y chunk boundaries -- the rows of the neighbour it
+// would otherwise receive -- so no other phase exchanges (the dt MIN stays).
+// A kernel run on an extended view computes those rows with the same
+// expressions from the same inputs as the neighbour does for its own rows:
+// same bits, so the step stays bitwise equal to one chunk.  Extensions (rows
+// beyond each non-wall y side), from the last reader back:
+//   y sweep 2 (x-first step) reads its inputs rows -3 .. ny+4
+//     -> x sweep 1 on rows -3 .. ny+4 (cells; nodes to ny+5): DEEP_EXT_X1 = 4
+//   x sweep 2 (y-first step) reads rows 0 .. ny+1
+//     -> y sweep 1 on rows 0 .. ny+1 (nodes to ny+2): DEEP_EXT_Y1 = 1
+//   x sweep 1 on ext 4 reads rows -4 .. ny+6, y sweep 1 on ext 1 rows
+//     -4 .. ny+5 -> the Lagrangian phase on ext 5 (cells -4 .. ny+5, nodes
+//     and y faces to ny+6): DEEP_EXT_LAGR = 5
+//   the Lagrangian on ext 5 reads q and the state rows -5 .. ny+7
+//     -> visc_dt on ext 5 (q on its ring rows -5 and ny+6): DEEP_EXT_VISC = 5
+//   visc_dt on ext 5 reads the state rows -6 .. ny+7: DEEP_ROWS = 7.
+// The extra dt terms are the neighbours' own cells (the MIN is unchanged).
+// y strips only (px == 1: every chunk has both x walls), both fused sweeps,
+// chunks at least DEEP_MIN_NY rows (an extension never reaches past the
+// neighbour).
+bool deep_ok(const clover_ctx* ctx) {
+  if (!ctx->deep || ctx->L.px != 1 || ctx->L.py < 2 || !fuse_x_ok(ctx) || !fuse_y_ok(ctx))
+    return false;
+  for (int k = 0; k < ctx->L.py; ++k)
+    if (ctx->L.ys[k + 1] - ctx->L.ys[k] < DEEP_MIN_NY) return false;
+  return true;
+}
+
+// Row-segment parameters of a chunk (or view) of c.ny rows (see seg_rows,
+// tail_nb): occ = resident blocks per SM of visc_dt, the Lagrangian, the
+// fused x and y sweeps.
+void set_segs(Chunk& c, int nsm, const int occ[4]) {
+  c.vks = seg_rows(VKS, grid_cols(c.nx, c.ny, VKS).x, c.ny);
+  c.lks = seg_rows(LKS, grid_strip(c.nx, LW, c.ny, LKS).x, c.ny);
+  c.xks = seg_rows(XKS, grid_strip(c.nx + 1, XW, c.ny + 1, XKS).x, c.ny + 1);
+  c.yks = seg_rows(YKS, grid_strip(c.nx + 1, YW, c.ny + 1, YKS).x, c.ny + 1);
+  c.vnb = tail_nb(c.vks, grid_cols(c.nx, c.ny, c.vks).x, c.ny, (int64_t)nsm * occ[0]);
+  c.lnb = tail_nb(c.lks, grid_strip(c.nx, LW, c.ny, c.lks).x, c.ny, (int64_t)nsm * occ[1]);
+  c.xnb = tail_nb(c.xks, grid_strip(c.nx + 1, XW, c.ny + 1, c.xks).x, c.ny + 1, (int64_t)nsm * occ[2]);
+  c.ynb = tail_nb(c.yks, grid_strip(c.nx + 1, YW, c.ny + 1, c.yks).x, c.ny + 1, (int64_t)nsm * occ[3]);
+}
+
+// The chunk seen from `e` rows beyond each of its non-wall y sides: rows
+// 1 .. ny+eb+et of the view are rows 1-eb .. ny+et of the chunk (field
+// pointers and the TMA row origin shifted by eb rows).  Same fix lists.
+ChunkState deep_view(const clover_ctx* ctx, const ChunkState& cs, int e) {
+  ChunkState v = cs;
+  Chunk& c = v.c;
+  const int eb = c.wb ? 0 : e, et = c.wt ? 0 : e;
+  c.ny += eb + et;
+  c.gk0 -= eb;
+  c.row0 = ROW0 - eb;
+  for (int b = 0; b < NBUF; ++b) v.buf[b] = cs.buf[b] - (int64_t)eb * c.pitch;
+  set_segs(c, ctx->nsm, ctx->occ);
+  return v;
 }
 
 // Row-segment geometry of a streaming kernel kind on a chunk: rows per
@@ -821,6 +894,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
   const bool walls_in_lagr = CLOVER_YWALLS_FOLD && fold1 && !advect_x && nphase >= 4;
   const bool walls_in_x1 = CLOVER_YWALLS_FOLD && fold1 && advect_x && fuse_x_ok(ctx) && nphase >= 6;
   int cur_prof_id = P_VISC_DT;
+  const bool deep = deep_ok(ctx);
   if (ctx->prof) prof_mark(ctx, -1);
   // one chunk on one rank: the visc fixup's last block finalises dt (no
   // k_dt_finalize launch); else the slot is combined first (NCCL MIN)
@@ -833,10 +907,19 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
   // the comm stream, followed there by their fixup and the exchange, while
   // the interior segments run beside them on the work stream (own fix list);
   // the next phase waits for both.
+  // ext > 0 (deep halos): the kernels run on each chunk's view extended
+  // ext rows beyond its y chunk boundaries (deep_view); bufs may be empty.
   auto run_phase = [&](int kind, auto&& launch, auto&& fixup, const std::vector<int>& bufs, int yd,
-                       int xd) -> int {
-    if (!overlap_ok(ctx)) {
-      for (auto& cs : ctx->chunks) {
+                       int xd, int ext = 0) -> int {
+    if (ext > 0 || !overlap_ok(ctx)) {
+      for (auto& cs0 : ctx->chunks) {
+        ChunkState view;
+        ChunkState* csp = &cs0;
+        if (ext > 0) {
+          view = deep_view(ctx, cs0, ext);
+          csp = &view;
+        }
+        ChunkState& cs = *csp;
         int lo, hi, n;
         phase_ranges(cs.c, kind, yd, &lo, &hi, &n);
         Chunk c = cs.c;
@@ -845,7 +928,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
         if (!rc) rc = fixup(cs, c, st, cs.fix);
         if (rc) return rc;
       }
-      return exchange(ctx, bufs, yd, xd);
+      return bufs.empty() ? CLOVER_OK : exchange(ctx, bufs, yd, xd);
     }
     cudaStream_t cm = ctx->comm_stream;
     CK(cudaEventRecord(ctx->ev_b, st));  // the previous phase is complete on st
@@ -881,7 +964,12 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
     return CLOVER_OK;
   };
   if (nphase >= 1) {
-    for (auto& cs : ctx->chunks) {
+    for (auto& cs0 : ctx->chunks) {
+      // deep halos: q (and the dt terms) of DEEP_EXT_VISC rows beyond the
+      // chunk, the rows the Lagrangian view reads (no q exchange)
+      ChunkState view;
+      if (deep) view = deep_view(ctx, cs0, DEEP_EXT_VISC);
+      const ChunkState& cs = deep ? view : cs0;
       const Chunk c = with_rev(cs.c, CLOVER_SERP);  // top-down: sweep 2 wrote these rows last
       launch_step(ks_visc_dt, dim3(grid_cols(c.nx, c.ny, c.vks).x, seg_count(c.vks, c.vnb, c.ny)), SB, st, c, cs.tm_visc, cs.buf[B_Q],
                   ctx->scal, ctx->dtp, cs.fix);
@@ -892,7 +980,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
     }
     // q on ring 1: visc_dt computes rows 0 / ny+1 at y chunk boundaries
     // itself (visc_ring_rows); only x chunk boundaries exchange q
-    if (needs_exchange(ctx)) {
+    if (needs_exchange(ctx) && !deep) {
       int rc = exchange_axis(ctx, {B_Q}, 0);
       if (rc) return rc;
     }
@@ -938,9 +1026,11 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
       FIX_LAUNCH_CHECK();
       return CLOVER_OK;
     };
-    // a fused y sweep (either sweep) reads these HALO_ROWS deep in y
-    int rc = run_phase(SEG_LAGR, launch, fixup, {B_D1, B_E1, B_U1, B_V1, B_FX, B_FY},
-                       fuse_y_ok(ctx) ? HALO_ROWS : HALO, fuse_x_ok(ctx) ? HALO_COLS : HALO);
+    // a fused y sweep (either sweep) reads these FUSE_ROWS deep in y; with
+    // deep halos the phase runs DEEP_EXT_LAGR rows beyond the chunk instead
+    int rc = deep ? run_phase(SEG_LAGR, launch, fixup, {}, 0, 0, DEEP_EXT_LAGR)
+                  : run_phase(SEG_LAGR, launch, fixup, {B_D1, B_E1, B_U1, B_V1, B_FX, B_FY},
+                              fuse_y_ok(ctx) ? FUSE_ROWS : HALO, fuse_x_ok(ctx) ? HALO_COLS : HALO);
     if (rc) return rc;
     if (ctx->prof) prof_mark(ctx, -1);
   }
@@ -984,9 +1074,14 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
           FIX_LAUNCH_CHECK();
           return CLOVER_OK;
         };
-        // sweep 1 feeds a fused y sweep 2: HALO_ROWS deep in y
-        int rc = run_phase(SEG_X, launch, fixup, {rout, eout, uout, vout},
-                           (sweep == 1 && fuse_y_ok(ctx)) ? HALO_ROWS : HALO, HALO);
+        // sweep 1 feeds a fused y sweep 2: FUSE_ROWS deep in y.  Deep
+        // halos: sweep 1 runs DEEP_EXT_X1 rows beyond the chunk (the rows the
+        // y sweep 2 reads), sweep 2 ends the step with the one exchange
+        int rc = !deep ? run_phase(SEG_X, launch, fixup, {rout, eout, uout, vout},
+                                   (sweep == 1 && fuse_y_ok(ctx)) ? FUSE_ROWS : HALO, HALO)
+                 : sweep == 1 ? run_phase(SEG_X, launch, fixup, {}, 0, 0, DEEP_EXT_X1)
+                              : run_phase(SEG_X, launch, fixup, {rout, eout, uout, vout},
+                                          DEEP_ROWS, HALO);
         if (rc) return rc;
         if (ctx->prof) prof_mark(ctx, -1);
       }
@@ -1050,9 +1145,14 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
           FIX_LAUNCH_CHECK();
           return CLOVER_OK;
         };
-        // y sweep 1 feeds a fused x sweep 2: HALO_COLS deep in x
-        int rc = run_phase(SEG_Y, launch, fixup, {rout, eout, uout, vout}, HALO,
-                           (sweep == 1 && fuse_x_ok(ctx)) ? HALO_COLS : HALO);
+        // y sweep 1 feeds a fused x sweep 2: HALO_COLS deep in x.  Deep
+        // halos: sweep 1 runs DEEP_EXT_Y1 rows beyond the chunk, sweep 2 ends
+        // the step with the one exchange
+        int rc = !deep ? run_phase(SEG_Y, launch, fixup, {rout, eout, uout, vout}, HALO,
+                                   (sweep == 1 && fuse_x_ok(ctx)) ? HALO_COLS : HALO)
+                 : sweep == 1 ? run_phase(SEG_Y, launch, fixup, {}, 0, 0, DEEP_EXT_Y1)
+                              : run_phase(SEG_Y, launch, fixup, {rout, eout, uout, vout},
+                                          DEEP_ROWS, HALO);
         if (rc) return rc;
         if (ctx->prof) prof_mark(ctx, -1);
       }
@@ -1093,9 +1193,9 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
         }
       }
       // x sweep 1 feeding a fused y sweep 2: the post-sweep density and
-      // energy HALO_ROWS deep in y; y sweep 1 feeding a fused x sweep 2:
+      // energy FUSE_ROWS deep in y; y sweep 1 feeding a fused x sweep 2:
       // HALO_COLS deep in x
-      const int yd = (sweep == 1 && xdir && fuse_y_ok(ctx)) ? HALO_ROWS : HALO;
+      const int yd = (sweep == 1 && xdir && fuse_y_ok(ctx)) ? FUSE_ROWS : HALO;
       const int xd = (sweep == 1 && !xdir && fuse_x_ok(ctx)) ? HALO_COLS : HALO;
       int rc = exchange(ctx, {rout, eout, mbuf}, yd, xd);
       if (rc) return rc;
@@ -1133,7 +1233,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
           }
         }
       }
-      const int yd = (sweep == 1 && xdir && fuse_y_ok(ctx)) ? HALO_ROWS : HALO;
+      const int yd = (sweep == 1 && xdir && fuse_y_ok(ctx)) ? FUSE_ROWS : HALO;
       const int xd = (sweep == 1 && !xdir && fuse_x_ok(ctx)) ? HALO_COLS : HALO;
       int rc = exchange(ctx, {uout, vout}, yd, xd);
       if (rc) return rc;
@@ -1182,6 +1282,8 @@ int build_graph(clover_ctx* ctx, int parity, int nst, int slot) {
   return CLOVER_OK;
 }
 
+// Wall mirrors and chunk halos of state fields written from outside a step
+// (init, write_field, restart): DEEP_ROWS deep in y with deep halos.
 int reflect_all(clover_ctx* ctx, const std::vector<int>& bufs) {
   for (auto& cs : ctx->chunks)
     for (int b : bufs) {
@@ -1190,8 +1292,26 @@ int reflect_all(clover_ctx* ctx, const std::vector<int>& bufs) {
       k_reflect<<<grd, blk, 0, ctx->work>>>(cs.c, cs.buf[b], kBufKind[b]);
       LAUNCH_CHECK();
     }
-  return exchange(ctx, bufs);
+  const int yd = deep_ok(ctx) ? DEEP_ROWS : HALO;
+  int rc = exchange(ctx, bufs, yd, HALO);
+  if (rc) return rc;
+  if (bufs.size() == 4) ctx->state_rows = yd;
+  else ctx->state_rows = std::min(ctx->state_rows, yd);
+  return CLOVER_OK;
 }
+
+// A deep-halo step reads the state DEEP_ROWS deep; a step without deep halos
+// (or a setting change since) left it HALO deep: refresh it first, outside
+// any graph.
+int ensure_state_rows(clover_ctx* ctx) {
+  if (!deep_ok(ctx) || ctx->state_rows >= DEEP_ROWS) return CLOVER_OK;
+  int rc = exchange(ctx, {B_D0, B_E0, B_U0, B_V0}, DEEP_ROWS, HALO);
+  if (rc) return rc;
+  ctx->state_rows = DEEP_ROWS;
+  return CLOVER_OK;
+}
+// the state's halo depth after a full step
+inline int step_state_rows(const clover_ctx* ctx) { return deep_ok(ctx) ? DEEP_ROWS : HALO; }
 
 int check_err(clover_ctx* ctx) {
   CK(cudaStreamSynchronize(ctx->work));
@@ -1483,6 +1603,20 @@ int clover_init(const clover_grid* grid, const clover_state* states, int32_t nst
   // clover_debug_set_overlap or CLOVER_OVERLAP=1 turn it on
   ctx->overlap = false;
   if (const char* e = std::getenv("CLOVER_OVERLAP")) ctx->overlap = std::atoi(e) != 0;
+  // deep halos where the layout allows (deep_ok; measured faster on every
+  // y-strip layout): clover_set_deep_halo or CLOVER_DEEP_HALO=0
+  ctx->deep = true;
+  if (const char* e = std::getenv("CLOVER_DEEP_HALO")) ctx->deep = std::atoi(e) != 0;
+  {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&ctx->nsm, cudaDevAttrMultiProcessorCount, dev);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&ctx->occ[0], ks_visc_dt, SB, 0);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&ctx->occ[1], ks_lagrangian, SB, 0);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&ctx->occ[2], ks_advec_x<1>, SB, 0);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&ctx->occ[3], ks_advec_y<1>, SB, 0);
+    cudaGetLastError();
+  }
   if (cudaStreamCreateWithFlags(&ctx->work, cudaStreamNonBlocking) != cudaSuccess ||
       cudaStreamCreateWithFlags(&ctx->comm_stream, cudaStreamNonBlocking) != cudaSuccess ||
       cudaEventCreateWithFlags(&ctx->ev_b, cudaEventDisableTiming) != cudaSuccess ||
@@ -1515,24 +1649,8 @@ int clover_init(const clover_grid* grid, const clover_state* states, int32_t nst
     c.face_cc = ctx->g.face_mirror == CLOVER_MIRROR_CELLCENTRE;
     c.rev = 0;
     c.seg0 = 0;
-    c.vks = seg_rows(VKS, grid_cols(c.nx, c.ny, VKS).x, c.ny);
-    c.lks = seg_rows(LKS, grid_strip(c.nx, LW, c.ny, LKS).x, c.ny);
-    c.xks = seg_rows(XKS, grid_strip(c.nx + 1, XW, c.ny + 1, XKS).x, c.ny + 1);
-    c.yks = seg_rows(YKS, grid_strip(c.nx + 1, YW, c.ny + 1, YKS).x, c.ny + 1);
-    {
-      int nsm = 148, b[4] = {0, 0, 0, 0}, dev = 0;
-      cudaGetDevice(&dev);
-      cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b[0], ks_visc_dt, SB, 0);
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b[1], ks_lagrangian, SB, 0);
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b[2], ks_advec_x<1>, SB, 0);
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b[3], ks_advec_y<1>, SB, 0);
-      c.vnb = tail_nb(c.vks, grid_cols(c.nx, c.ny, c.vks).x, c.ny, (int64_t)nsm * b[0]);
-      c.lnb = tail_nb(c.lks, grid_strip(c.nx, LW, c.ny, c.lks).x, c.ny, (int64_t)nsm * b[1]);
-      c.xnb = tail_nb(c.xks, grid_strip(c.nx + 1, XW, c.ny + 1, c.xks).x, c.ny + 1, (int64_t)nsm * b[2]);
-      c.ynb = tail_nb(c.yks, grid_strip(c.nx + 1, YW, c.ny + 1, c.yks).x, c.ny + 1, (int64_t)nsm * b[3]);
-      cudaGetLastError();
-    }
+    c.row0 = ROW0;
+    set_segs(c, ctx->nsm, ctx->occ);
     c.dx = dx; c.dy = dy; c.xmin = ctx->g.xmin; c.ymin = ctx->g.ymin;
     // correctly rounded reciprocals of the constant divisors (IEEE host division)
     c.rdx = 1.0 / dx; c.rdy = 1.0 / dy;
@@ -1563,10 +1681,10 @@ int clover_init(const clover_grid* grid, const clover_state* states, int32_t nst
     p += align_up((int64_t)cs.ntx * cs.nty * 5 * 8, kAlign);
     cs.fix.hdr = (unsigned*)p;
     cs.fix.e = (uint2*)(p + kAlign);
-    p += fix_bytes(c.nx, c.ny);
+    p += fix_bytes(c.nx, c.ny + 2 * DEEP_EXT_MAX);
     cs.fix_b.hdr = (unsigned*)p;
     cs.fix_b.e = (uint2*)(p + kAlign);
-    p += fix_bytes(c.nx, c.ny);
+    p += fix_bytes(c.nx, c.ny + 2 * DEEP_EXT_MAX);
     maxrows = std::max<int64_t>(maxrows, c.ny + 2 + 2 * HALO_ROWS);
     maxcols = std::max<int64_t>(maxcols, c.nx + 2 + 2 * HALO_COLS);
     ctx->chunks.push_back(cs);
@@ -1695,6 +1813,23 @@ int clover_debug_set_virtual_remote(clover_ctx* ctx, int32_t enable) {
   return CLOVER_OK;
 }
 
+int clover_set_deep_halo(clover_ctx* ctx, int32_t enable) {
+  if (!ctx) return fail(CLOVER_ERR_ARG, "ctx is NULL");
+  ctx->deep = enable != 0;
+  for (int i = 0; i < 4; ++i)
+    if (ctx->gexec[i]) {
+      cudaGraphExecDestroy(ctx->gexec[i]);
+      ctx->gexec[i] = nullptr;
+    }
+  return CLOVER_OK;  // the next step refreshes the state halo if needed (ensure_state_rows)
+}
+
+int clover_deep_halo_active(clover_ctx* ctx, int32_t* out) {
+  if (!ctx || !out) return fail(CLOVER_ERR_ARG, "NULL argument");
+  *out = deep_ok(ctx) ? 1 : 0;
+  return CLOVER_OK;
+}
+
 int clover_debug_set_overlap(clover_ctx* ctx, int32_t enable) {
   if (!ctx) return fail(CLOVER_ERR_ARG, "ctx is NULL");
   ctx->overlap = enable != 0;
@@ -1762,10 +1897,10 @@ int clover_kernels_per_step(clover_ctx* ctx, int32_t* out) {
         return b + (b > 0) + 2 * (lo < hi) - 2;
       };
       const bool ax = ctx->advect_x;
-      n += extra(SEG_LAGR, fuse_y_ok(ctx) ? HALO_ROWS : HALO);
+      n += extra(SEG_LAGR, fuse_y_ok(ctx) ? FUSE_ROWS : HALO);
       for (int sweep = 1; sweep <= 2; ++sweep) {
         const bool xdir = (sweep == 1) ? ax : !ax;
-        if (xdir && fuse_x_ok(ctx)) n += extra(SEG_X, (sweep == 1 && fuse_y_ok(ctx)) ? HALO_ROWS : HALO);
+        if (xdir && fuse_x_ok(ctx)) n += extra(SEG_X, (sweep == 1 && fuse_y_ok(ctx)) ? FUSE_ROWS : HALO);
         if (!xdir && fuse_y_ok(ctx)) n += extra(SEG_Y, HALO);
       }
     }
@@ -1786,8 +1921,11 @@ int clover_step(clover_ctx* ctx, int32_t nsteps) {
     join_out(ctx);
     return code;
   };
+  rc = ensure_state_rows(ctx);
+  if (rc) return bail(rc);
   for (int i = 0; i < nsteps; ++i) {
     const int parity = ctx->advect_x ? 0 : 1;
+    ctx->state_rows = step_state_rows(ctx);
     if (ctx->use_graphs && CLOVER_GRAPH_STEPS > 1 && nsteps - i >= CLOVER_GRAPH_STEPS) {
       const int slot = parity + 2;
       if (!ctx->gexec[slot]) {
@@ -1831,9 +1969,11 @@ int clover_profile_steps(clover_ctx* ctx, int32_t nsteps, double* ms_out, int64_
   for (int i = 0; i < NPROF; ++i) { ms_out[i] = 0.0; launches_out[i] = 0; }
   int rc = join_in(ctx);
   if (rc) return rc;
+  rc = ensure_state_rows(ctx);
   ctx->prof = true;
   for (int s = 0; s < nsteps && !rc; ++s) {
     rc = enqueue_step(ctx, ctx->advect_x, 7);
+    ctx->state_rows = step_state_rows(ctx);
     ctx->advect_x = !ctx->advect_x;
   }
   ctx->prof = false;
@@ -1926,8 +2066,10 @@ int clover_debug_partial_step(clover_ctx* ctx, int32_t nkernels) {
   if (!ctx) return fail(CLOVER_ERR_ARG, "ctx is NULL");
   int rc = join_in(ctx);
   if (rc) return rc;
-  rc = enqueue_step(ctx, ctx->advect_x, nkernels);
+  rc = ensure_state_rows(ctx);
+  if (!rc) rc = enqueue_step(ctx, ctx->advect_x, nkernels);
   if (rc) return rc;
+  if (nkernels >= 6) ctx->state_rows = step_state_rows(ctx);  // sweep 2 rewrote the state
   return join_out(ctx);
 }
 

@@ -304,7 +304,7 @@ __device__ __forceinline__ bool visc_body(const Chunk& c, const CUtensorMap* __r
   auto issue = [&](int r) {
     const unsigned sl = slot_of(r);
     mbar_arrive_expect_tx(&bars[sl], VBYTES);
-    tma_load_3d(ring + sl * VSLOT, tm, xcol, ROW0 + r, 0, &bars[sl]);
+    tma_load_3d(ring + sl * VSLOT, tm, xcol, c.row0 + r, 0, &bars[sl]);
   };
   auto wait_row = [&](int r) {
     const unsigned rel = (unsigned)(r - r_first);
@@ -516,7 +516,7 @@ __device__ __forceinline__ bool lagr_body(const Chunk& c, const CUtensorMap* __r
   auto slot_of = [&](int r) { return (unsigned)(r - r_first) % (unsigned)LSTG; };
   auto issue_at = [&](unsigned sl, int r) {  // row r into slot sl
     mbar_arrive_expect_tx(&bars[sl], LBYTES);
-    tma_load_3d(ring + sl * LSLOT, tm, xcol, ROW0 + r, 0, &bars[sl]);
+    tma_load_3d(ring + sl * LSLOT, tm, xcol, c.row0 + r, 0, &bars[sl]);
   };
   auto issue = [&](int r) { issue_at(slot_of(r), r); };
   auto wait_row = [&](int r) {
@@ -1161,7 +1161,7 @@ __device__ __forceinline__ bool advec_x_body(const Chunk& c, const CUtensorMap* 
   auto issue = [&](int r) {
     const unsigned sl = slot_of(r);
     mbar_arrive_expect_tx(&bars[sl], BYTES);
-    tma_load_3d(ring + sl * SL, tm, xcol, ROW0 + r, 0, &bars[sl]);
+    tma_load_3d(ring + sl * SL, tm, xcol, c.row0 + r, 0, &bars[sl]);
   };
   auto wait_row = [&](int r) {
     const unsigned rel = (unsigned)(r - r_first);
@@ -1599,18 +1599,18 @@ __device__ __forceinline__ bool advec_y_body(const Chunk& c, const CUtensorMap* 
     mbar_arrive_expect_tx(&bars[sl], L::BYTES);
 #if CLOVER_L2HINT
     if (r <= k0 + 2) {
-      tma_load_3d_hint(d, ta, xcol, ROW0 + r, 0, &bars[sl], pol_keep);
-      if constexpr (SWEEP == 2) tma_load_3d_hint(d + L::B, tb, xcol, ROW0 + r, 0, &bars[sl], pol_keep);
+      tma_load_3d_hint(d, ta, xcol, c.row0 + r, 0, &bars[sl], pol_keep);
+      if constexpr (SWEEP == 2) tma_load_3d_hint(d + L::B, tb, xcol, c.row0 + r, 0, &bars[sl], pol_keep);
       return;
     }
 #if CLOVER_L2HINT > 1
-    tma_load_3d_hint(d, ta, xcol, ROW0 + r, 0, &bars[sl], pol_once);
-    if constexpr (SWEEP == 2) tma_load_3d_hint(d + L::B, tb, xcol, ROW0 + r, 0, &bars[sl], pol_once);
+    tma_load_3d_hint(d, ta, xcol, c.row0 + r, 0, &bars[sl], pol_once);
+    if constexpr (SWEEP == 2) tma_load_3d_hint(d + L::B, tb, xcol, c.row0 + r, 0, &bars[sl], pol_once);
     return;
 #endif
 #endif
-    tma_load_3d(d, ta, xcol, ROW0 + r, 0, &bars[sl]);
-    if constexpr (SWEEP == 2) tma_load_3d(d + L::B, tb, xcol, ROW0 + r, 0, &bars[sl]);
+    tma_load_3d(d, ta, xcol, c.row0 + r, 0, &bars[sl]);
+    if constexpr (SWEEP == 2) tma_load_3d(d + L::B, tb, xcol, c.row0 + r, 0, &bars[sl]);
   };
   auto issue = [&](int r) { issue_at((unsigned)(r - r_first) % (unsigned)L::RING, r); };
   auto row = [&](int r) -> const double* {

@@ -4,7 +4,8 @@ the fused y sweep across y chunk boundaries (default) or only at walls
 (round-1 schedule: separate y kernels + an extra exchange phase), and
 through the virtual-remote packing path (pack -> staging -> unpack, the
 multi-GPU message layout), by device copy and through a one-rank NCCL
-communicator.  Prints one JSON line.
+communicator; each also with deep halos (one 7-row state exchange per
+step, *_deep).  Prints one JSON line.
 usage: chunk_overhead.py NX NY PX PY [STEPS]"""
 import json
 import os
@@ -23,8 +24,9 @@ deck = bm_deck(nx, ny, end_step=steps, ymax=10.0 * ny / nx)
 # (square cells: the domain grows with the mesh)
 
 
-def run(p, q, vr=0, walls_only=False, overlap=False):
+def run(p, q, vr=0, walls_only=False, overlap=False, deep=False):
     sim = Clover(deck, px=p, py=q)
+    sim.set_deep_halo(deep)
     if walls_only:
         sim.debug_set_fusion(True, walls_only=True)
     if vr:
@@ -61,7 +63,9 @@ res["strong_scaling_efficiency_bound"] = one / (px * py * alone)
 for name, kw in (("local_fused", {}), ("local_walls_only", dict(walls_only=True)),
                  ("virtual_remote", dict(vr=1)), ("virtual_nccl", dict(vr=2)),
                  ("virtual_remote_overlap", dict(vr=1, overlap=True)),
-                 ("virtual_nccl_overlap", dict(vr=2, overlap=True))):
+                 ("virtual_nccl_overlap", dict(vr=2, overlap=True)),
+                 ("local_deep", dict(deep=True)), ("virtual_remote_deep", dict(vr=1, deep=True)),
+                 ("virtual_nccl_deep", dict(vr=2, deep=True))):
     ms, k = run(px, py, **kw)
     res[name] = {"ms": ms, "overhead": ms / one - 1.0, "kernels": k,
                  "over_serial_ideal": ms / (alone * px * py) - 1.0}

@@ -31,7 +31,7 @@ def _free_port() -> int:
         return s.getsockname()[1]
 
 
-def _worker(rank, world, port, deck, px, py, steps, out):
+def _worker(rank, world, port, deck, px, py, steps, out, deep=False):
     import torch
     import torch.distributed as dist
 
@@ -43,6 +43,8 @@ def _worker(rank, world, port, deck, px, py, steps, out):
     dist.init_process_group("gloo", rank=rank, world_size=world)
     torch.cuda.set_device(0)
     sim = Clover(deck, px=px, py=py, rank=rank, nranks=world, host_transport=GlooHostTransport())
+    sim.set_deep_halo(deep)  # (on by default: the plain cases keep the per-phase schedule)
+    assert sim.deep_halo_active() == deep
     sim.step(steps)
     fields = {f: sim.read(f) for f in STATE}
     summ = sim.field_summary()
@@ -57,10 +59,10 @@ def _worker(rank, world, port, deck, px, py, steps, out):
     dist.destroy_process_group()
 
 
-def _run(world, deck, px, py, steps, tmp_path):
+def _run(world, deck, px, py, steps, tmp_path, deep=False):
     import torch.multiprocessing as mp
-    out = str(tmp_path / f"r0_{world}_{px}x{py}.npz")
-    ctx = mp.start_processes(_worker, args=(world, _free_port(), deck, px, py, steps, out),
+    out = str(tmp_path / f"r0_{world}_{px}x{py}_{int(deep)}.npz")
+    ctx = mp.start_processes(_worker, args=(world, _free_port(), deck, px, py, steps, out, deep),
                              nprocs=world, join=False, start_method="spawn")
     while not ctx.join(timeout=240):
         pass
@@ -76,16 +78,18 @@ def torch_cuda():
 
 
 @pytest.mark.timeout(600)
-@pytest.mark.parametrize("world,px,py,deck", [
-    (2, 1, 2, "fuzz"),   # y strips: the launcher's default decomposition
-    (2, 2, 1, "point"),  # x strips: separate x kernels, fused y
-    (4, 2, 2, "fuzz"),   # four ranks, 4-rank corners
+@pytest.mark.parametrize("world,px,py,deck,deep", [
+    (2, 1, 2, "fuzz", False),  # y strips: the launcher's default decomposition
+    (2, 2, 1, "point", False),  # x strips: separate x kernels, fused y
+    (4, 2, 2, "fuzz", False),  # four ranks, 4-rank corners
+    (2, 1, 2, "fuzz", True),   # deep halos: one 7-row state exchange per step
+    (4, 1, 4, "point", True),  # deep halos, 16-row strips (the minimum)
 ])
-def test_processes_match_one_chunk_and_oracle(torch_cuda, tmp_path, world, px, py, deck):
+def test_processes_match_one_chunk_and_oracle(torch_cuda, tmp_path, world, px, py, deck, deep):
     from paper_conf_cluster_regulymg15_b200 import Clover
     d = fuzz_deck(21, nx=72, ny=64) if deck == "fuzz" else point_deck(72, 64)
     steps = 12
-    got = _run(world, d, px, py, steps, tmp_path)
+    got = _run(world, d, px, py, steps, tmp_path, deep)
     one = Clover(d)
     one.step(steps)
     o = Oracle(d)

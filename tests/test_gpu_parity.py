@@ -397,9 +397,11 @@ def test_boundary_first_overlap_bitwise(torch_cuda, nccl, py):
     one = make_gpu(deck)
     ov = make_gpu(deck, px=1, py=py)
     ov.debug_set_virtual_remote(True, nccl=nccl)
+    ov.set_deep_halo(False)  # (overlap is for the per-phase exchange schedule)
     ov.debug_set_overlap(True)
     plain = make_gpu(deck, px=1, py=py)
     plain.debug_set_virtual_remote(True, nccl=nccl)
+    plain.set_deep_halo(False)
     plain.debug_set_overlap(False)
     assert ov.kernels_per_step() > plain.kernels_per_step()
     for g in (one, ov, plain):
@@ -436,6 +438,79 @@ def test_fused_sweeps_across_chunk_boundaries(torch_cuda, seed, pxy):
         for g in (fused, split, remote):
             assert np.array_equal(g.read(f), a), f
     assert np.array_equal(fused.dt_history(1, 12), one.dt_history(1, 12))
+
+
+@pytest.mark.parametrize("seed,py,mode", [(8, 2, "local"), (9, 3, "local"), (10, 5, "local"),
+                                           (11, 2, "remote"), (12, 4, "remote"), (13, 3, "nccl"),
+                                           (14, 6, "nccl")])
+def test_deep_halo_bitwise(torch_cuda, seed, py, mode):
+    """S:8(f) f1 deep halos: one 7-row state exchange per step, every kernel
+    run over the rows of its y neighbours it would otherwise receive.  Fuzz
+    decks (flow across the boundaries), 12 steps (both sweep orders): fields,
+    dt history and summary bitwise equal to one chunk and to the per-phase
+    exchange schedule; local chunks, virtual remote (device copy) and NCCL
+    messages."""
+    deck = fuzz_deck(seed, nx=72, ny=112)
+    deck["max_timestep"] = 1.0
+    one = make_gpu(deck)
+    deep = make_gpu(deck, px=1, py=py)
+    plain = make_gpu(deck, px=1, py=py)
+    if mode != "local":
+        for g in (deep, plain):
+            g.debug_set_virtual_remote(True, nccl=(mode == "nccl"))
+    deep.set_deep_halo(True)
+    plain.set_deep_halo(False)
+    assert deep.deep_halo_active() and not plain.deep_halo_active()
+    for g in (one, deep, plain):
+        g.step(12)
+    for f in STATE:
+        a = one.read(f)
+        assert np.array_equal(deep.read(f), a), f
+        assert np.array_equal(plain.read(f), a), f
+    assert np.array_equal(deep.dt_history(1, 12), one.dt_history(1, 12))
+    assert deep.field_summary() == one.field_summary()
+
+
+def test_deep_halo_bm_blast_and_toggles(torch_cuda):
+    """The bm blast crossing 1x4 strip boundaries for 40 steps with deep
+    halos switched on and off between steps (the state halo is refreshed 7
+    deep when a deep step follows a plain one), graphs on and off: bitwise
+    equal to one chunk and to the oracle."""
+    deck = bm_deck(128, end_step=40)
+    one, g = make_gpu(deck), make_gpu(deck, px=1, py=4)
+    g.set_deep_halo(True)
+    assert g.deep_halo_active()
+    g.step(10)
+    g.set_deep_halo(False)
+    g.step(5)
+    g.set_deep_halo(True)
+    g.set_graphs(False)
+    g.step(10)
+    g.set_graphs(True)
+    g.step(15)
+    one.step(40)
+    for f in STATE:
+        assert np.array_equal(g.read(f), one.read(f)), f
+    assert np.array_equal(g.dt_history(1, 40), one.dt_history(1, 40))
+    o = Oracle(deck)
+    o.step(40)
+    assert_fields_equal(g, o, ctx="deep bm 1x4")
+
+
+@pytest.mark.parametrize("pxy,ny", [((2, 2), 112), ((1, 8), 112), ((1, 1), 112)])
+def test_deep_halo_inactive_layouts(torch_cuda, pxy, ny):
+    """Deep halos need y strips (px == 1, py > 1) of at least 16 rows; other
+    layouts keep the per-phase schedule (the setting has no effect) and stay
+    bitwise."""
+    deck = fuzz_deck(15, nx=72, ny=ny)
+    deck["max_timestep"] = 1.0
+    one, g = make_gpu(deck), make_gpu(deck, px=pxy[0], py=pxy[1])
+    g.set_deep_halo(True)
+    assert not g.deep_halo_active()
+    one.step(6)
+    g.step(6)
+    for f in STATE:
+        assert np.array_equal(g.read(f), one.read(f)), f
 
 
 @pytest.mark.parametrize("seed,pxy", [(8, (2, 3)), (9, (3, 2)), (9, (2, 4)), (12, (4, 4)),
