@@ -363,6 +363,7 @@ def main():
     ms = cdist.max_over_ranks(ms, None if host_tp else dev)
     value = cells * args.steps / (ms / 1000.0)
     launches = sim.launch_count() - nl0  # counted by the engine, graph launches included
+    deep_halo = sim.deep_halo_active()
 
     # per-kernel CUDA-event durations over a second pass of K steps on the
     # same stream (direct launches, event after every kernel)
@@ -513,6 +514,8 @@ def main():
                            "mesh": [nx, ny], "decomposition": f"{px}x{py}",
                            "transport": ("nccl" if not host_tp else "host (gloo; not a bench value)")
                            if world > 1 else None,
+                           "halo_exchange": ("deep: 1 state exchange (7 rows) + dt MIN per step"
+                                             if deep_halo else "per phase") if world > 1 else None,
                            "l2": "inputs larger than L2 (18 fp64 fields of the mesh, >2 GB vs 126 MB L2)",
                            "graphs": True},
                 "gpu_launches": launches,

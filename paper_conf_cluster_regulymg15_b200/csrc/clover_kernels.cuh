@@ -379,12 +379,12 @@ __device__ __forceinline__ void cell_update(D& dv, double rho, double en, double
 }
 
 // ------------------------------------------------ advec_mom (c.9)
-// Momentum flux at one node for one velocity component (limited, c.9).
+// Momentum flux at one node for one velocity component (limited, c.9),
+// given sigma = |node_flux| / node_mass_pre(donor).
 template <class D>
-__device__ __forceinline__ double mom_flux(D& dv, double nf, double nmp_don, double vup,
+__device__ __forceinline__ double mom_flux(D& dv, double nf, double sigma, double vup,
                                            double vdon, double vdw, double width, double rwidth) {
   // width = celldx(j) and celldx(dif) are the same constant on the uniform mesh
-  double sigma = div_pos(dv, fabs(nf), nmp_don);
   double vdiffuw = vdon - vup;
   double vdiffdw = vdw - vdon;
   double limiter = 0.0;
@@ -402,13 +402,16 @@ __device__ __forceinline__ double mom_flux(D& dv, double nf, double nmp_don, dou
   return advec_vel * nf;
 }
 
-// both velocity components at one node (they share sigma's inputs)
+// both velocity components at one node: the reference evaluates sigma in
+// each component's loop from the same node flux and mass, so one division
+// serves both (same bits)
 template <class D>
 __device__ __forceinline__ void mom_flux2(D& dv, double nf, double nmp, const double* uu,
                                           const double* vv, double w, double rw, double& mu,
                                           double& mv) {
-  mu = mom_flux(dv, nf, nmp, uu[0], uu[1], uu[2], w, rw);
-  mv = mom_flux(dv, nf, nmp, vv[0], vv[1], vv[2], w, rw);
+  const double sigma = div_pos(dv, fabs(nf), nmp);
+  mu = mom_flux(dv, nf, sigma, uu[0], uu[1], uu[2], w, rw);
+  mv = mom_flux(dv, nf, sigma, vv[0], vv[1], vv[2], w, rw);
 }
 
 template <class D>
