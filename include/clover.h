@@ -157,7 +157,13 @@ int clover_nccl_unique_id(void* out128);
  * (generate_chunk), compute the EOS and prime all halos (start of run,
  * SURVEY 8(c) c.1).  Validation: x_cells,y_cells >= 4; nstates >= 1;
  * xmax > xmin; ymax > ymin; px*py >= nranks and divisible by nranks; every
- * chunk at least 4x4 cells.  On error *out is NULL. */
+ * chunk at least 4x4 cells.  On error *out is NULL.
+ * Multi-rank NCCL contexts with CLOVER_LSA=1 in every rank's environment
+ * exchange halos by device-initiated stores into the peers' NCCL symmetric
+ * windows (see clover_debug_set_virtual_remote, enable = 3); the library
+ * then allocates its mailbox with ncclMemAlloc (collective, freed by
+ * clover_finalize); CLOVER_ERR_NCCL if not every rank is load/store
+ * reachable. */
 int clover_init(const clover_grid* grid, const clover_state* states, int32_t nstates,
                 const clover_dist* dist, void* workspace, int64_t workspace_bytes,
                 void* cuda_stream, clover_ctx** out);
@@ -248,7 +254,13 @@ const char* clover_profile_name(int32_t i);
  * enable = 2: the messages travel through a one-rank NCCL communicator
  * (ncclSend/ncclRecv to self inside one group, created here) and dt through a
  * one-rank ncclAllReduce(MIN), captured in the step's CUDA graph like the
- * multi-rank path; CLOVER_ERR_NCCL if the library was built without NCCL. */
+ * multi-rank path; enable = 3: as 2, but the messages are device-initiated
+ * stores (S:8(f) f1): the pack kernel writes each message straight into its
+ * receiver's slot of a one-rank NCCL symmetric window (ncclMemAlloc +
+ * ncclCommWindowRegister, peer mapping from ncclGetPeerPointer), an LSA
+ * barrier (ncclDevComm) makes the stores visible, the receiver unpacks, a
+ * second barrier frees the mailbox -- the multi-rank path of CLOVER_LSA=1.
+ * CLOVER_ERR_NCCL if the library was built without NCCL. */
 int clover_debug_set_virtual_remote(clover_ctx* ctx, int32_t enable);
 
 /* Debug: run only the first `nkernels` kernel phases of the next step

@@ -360,12 +360,14 @@ class Clover:
         buf = ctypes.create_string_buffer(blob, len(blob))
         _check(load().clover_restart(self._ctx, buf, len(blob)), "clover_restart")
 
-    def debug_set_virtual_remote(self, on, nccl: bool = False):
+    def debug_set_virtual_remote(self, on, nccl: bool = False, lsa: bool = False):
         """on: chunk boundaries through the remote (pack/staging/unpack) path;
         nccl: the messages through a one-rank NCCL communicator (send/recv to
-        self) and dt through a one-rank NCCL all-reduce."""
-        _check(load().clover_debug_set_virtual_remote(self._ctx, (2 if nccl else 1) if on else 0),
-               "clover_debug_set_virtual_remote")
+        self) and dt through a one-rank NCCL all-reduce; lsa: the messages
+        as device-initiated stores into a one-rank NCCL symmetric window
+        (LSA barriers), dt as with nccl."""
+        mode = (3 if lsa else 2 if nccl else 1) if on else 0
+        _check(load().clover_debug_set_virtual_remote(self._ctx, mode), "clover_debug_set_virtual_remote")
 
     def debug_partial_step(self, nkernels: int):
         _check(load().clover_debug_partial_step(self._ctx, nkernels), "clover_debug_partial_step")

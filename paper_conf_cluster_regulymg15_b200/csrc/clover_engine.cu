@@ -26,6 +26,7 @@
 
 #ifdef CLOVER_WITH_NCCL
 #include <nccl.h>
+#include <nccl_device.h>  // symmetric windows + LSA barrier (device-initiated halo stores)
 #endif
 
 using namespace clover;
@@ -293,6 +294,17 @@ struct clover_ctx {
   std::vector<std::pair<int, cudaEvent_t>> prof_events;
 #ifdef CLOVER_WITH_NCCL
   ncclComm_t comm = nullptr;
+  // device-initiated halo stores (S:8(f) f1, lsa_setup): every rank's halo
+  // mailbox is a symmetric NCCL window; a sender packs its boundary strips
+  // straight into the receiver's mailbox through the peer mapping, then an
+  // LSA barrier, the unpack, and a second barrier
+  bool lsa = false;
+  double* lsa_recv = nullptr;         // this rank's mailbox (ncclMemAlloc)
+  size_t lsa_bytes = 0;
+  ncclWindow_t lsa_win = nullptr;
+  ncclDevComm lsa_dc{};
+  bool lsa_dc_ok = false;
+  std::vector<double*> lsa_peer;      // rank r's mailbox as mapped here
 #endif
   int hist_first = 1;             // first step whose dt is in the history (after a restart: ckpt step + 1)
   bool use_ht = false;            // collectives through the caller's host transport
@@ -346,6 +358,19 @@ std::vector<int> local_chunk_ids(int px, int py, int rank, int nranks) {
   std::vector<int> ids;
   for (int i = rank * per; i < (rank + 1) * per; ++i) ids.push_back(i);
   return ids;
+}
+
+// Halo staging of one rank (doubles per buffer): every local chunk x 4
+// sides x 6 fields x HALO_ROWS lines of the longest chunk extent.
+int64_t staging_elems(const Layout& L, int rank, int nranks) {
+  int64_t line = 0, n = 0;
+  for (int id : local_chunk_ids(L.px, L.py, rank, nranks)) {
+    const int cx = id % L.px, cy = id / L.px;
+    const int nx = L.xs[cx + 1] - L.xs[cx], ny = L.ys[cy + 1] - L.ys[cy];
+    line = std::max<int64_t>(line, std::max(ny + 2 + 2 * HALO_ROWS, nx + 2 + 2 * HALO_COLS));
+    ++n;
+  }
+  return n * 4 * 6 * HALO_ROWS * line;
 }
 
 int64_t compute_workspace(const clover_grid* g, int px, int py, int rank, int nranks) {
@@ -503,6 +528,117 @@ int StripQueue::flush() {
   return CLOVER_OK;
 }
 
+// Geometry-only view of chunk `id` of the layout (any rank's): enough for
+// neighbour() and the strip sizes of side_strips.
+ChunkState geom_chunk(const clover_ctx* ctx, int id) {
+  ChunkState g{};
+  g.id = id; g.cx = id % ctx->L.px; g.cy = id / ctx->L.px;
+  g.c.nx = ctx->L.xs[g.cx + 1] - ctx->L.xs[g.cx];
+  g.c.ny = ctx->L.ys[g.cy + 1] - ctx->L.ys[g.cy];
+  return g;
+}
+// Doubles of one side's message: the strips of every field in `bufs`.
+int64_t msg_elems(const ChunkState& cs, int side, const std::vector<int>& bufs, int yd, int xd) {
+  int64_t n = 0;
+  for (int b : bufs) {
+    XferDesc s, r;
+    side_strips(cs, b, side, s, r, yd, xd);
+    n += (int64_t)s.w * s.h;
+  }
+  return n;
+}
+// Where rank q receives the message of its chunk `id`, side `side`: the
+// offset q's own message list (exchange_axis) gives it, rebuilt from the
+// layout -- the address a sender stores into with device-initiated stores.
+int64_t peer_recv_off(const clover_ctx* ctx, int q, int id, int side, const std::vector<int>& bufs,
+                      int axis, int yd, int xd) {
+  const int s_lo = axis == 0 ? 0 : 2, s_hi = axis == 0 ? 1 : 3;
+  int64_t off = 0;
+  for (int cid : local_chunk_ids(ctx->L.px, ctx->L.py, q, ctx->nranks)) {
+    const ChunkState g = geom_chunk(ctx, cid);
+    for (int sd : {s_lo, s_hi}) {
+      const int nb = neighbour(ctx, g, sd);
+      if (nb < 0 || (!ctx->virtual_remote && ctx->owner[nb] == q)) continue;
+      if (cid == id && sd == side) return off;
+      off += msg_elems(g, sd, bufs, yd, xd);
+    }
+  }
+  return -1;
+}
+
+#ifdef CLOVER_WITH_NCCL
+// LSA barrier over every rank of the node (one CTA; release/acquire at
+// system scope): the device-initiated halo stores before it are visible to
+// their receivers after it.
+__global__ void k_lsa_barrier(ncclDevComm dc) {
+  ncclLsaBarrierSession<ncclCoopCta> bar(ncclCoopCta(), dc, ncclTeamTagLsa(), 0);
+  bar.sync(ncclCoopCta(), cuda::memory_order_acq_rel);
+}
+// rank r's window base as mapped into this process
+__global__ void k_lsa_bases(ncclWindow_t w, int n, void** out) {
+  for (int i = threadIdx.x; i < n; i += blockDim.x) out[i] = ncclGetPeerPointer(w, 0, i);
+}
+#endif
+bool lsa_active(const clover_ctx* ctx) {
+#ifdef CLOVER_WITH_NCCL
+  return ctx->lsa && !ctx->use_ht && (ctx->nranks > 1 || (ctx->virtual_remote && ctx->virtual_nccl));
+#else
+  (void)ctx;
+  return false;
+#endif
+}
+
+// Device-initiated halo stores (S:8(f) f1): a symmetric NCCL window per rank
+// as the halo mailbox (the same size on every rank: the largest rank's
+// staging need), an LSA barrier, and the peers' mailbox addresses as mapped
+// here.  Collective over the communicator: every rank calls it together.
+int lsa_setup(clover_ctx* ctx) {
+#ifdef CLOVER_WITH_NCCL
+  if (ctx->lsa_recv) return CLOVER_OK;
+  if (!ctx->comm) return fail(CLOVER_ERR_STATE, "LSA halo stores need an NCCL communicator");
+  int64_t el = 0;
+  for (int r = 0; r < ctx->nranks; ++r) el = std::max(el, staging_elems(ctx->L, r, ctx->nranks));
+  ctx->lsa_bytes = (size_t)align_up(std::max<int64_t>(el * 8, 1), NCCL_WIN_REQUIRED_ALIGNMENT);
+  NK(ncclMemAlloc((void**)&ctx->lsa_recv, ctx->lsa_bytes));
+  NK(ncclCommWindowRegister(ctx->comm, ctx->lsa_recv, ctx->lsa_bytes, &ctx->lsa_win,
+                            NCCL_WIN_COLL_SYMMETRIC));
+  ncclDevCommRequirements reqs;
+  std::memset(&reqs, 0, sizeof(reqs));
+  reqs.lsaBarrierCount = 1;
+  NK(ncclDevCommCreate(ctx->comm, &reqs, &ctx->lsa_dc));
+  ctx->lsa_dc_ok = true;
+  if (ncclTeamLsa(ctx->comm).nRanks != ctx->nranks)
+    return fail(CLOVER_ERR_NCCL, "LSA halo stores need every rank load/store reachable (one NVLink domain)");
+  void** d = nullptr;
+  CK(cudaMalloc((void**)&d, sizeof(void*) * ctx->nranks));
+  k_lsa_bases<<<1, 32, 0, ctx->work>>>(ctx->lsa_win, ctx->nranks, d);
+  std::vector<void*> h((size_t)ctx->nranks);
+  cudaError_t e = cudaMemcpyAsync(h.data(), d, sizeof(void*) * ctx->nranks, cudaMemcpyDeviceToHost,
+                                  ctx->work);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(ctx->work);
+  cudaFree(d);
+  if (e != cudaSuccess) return fail(CLOVER_ERR_CUDA, std::string("LSA bases: ") + cudaGetErrorString(e));
+  ctx->lsa_peer.assign((size_t)ctx->nranks, nullptr);
+  for (int r = 0; r < ctx->nranks; ++r) ctx->lsa_peer[r] = (double*)h[r];
+  return CLOVER_OK;
+#else
+  return fail(CLOVER_ERR_NCCL, "libclover built without NCCL");
+#endif
+}
+void lsa_teardown(clover_ctx* ctx) {
+#ifdef CLOVER_WITH_NCCL
+  if (ctx->lsa_dc_ok) ncclDevCommDestroy(ctx->comm, &ctx->lsa_dc);
+  if (ctx->lsa_win) ncclCommWindowDeregister(ctx->comm, ctx->lsa_win);
+  if (ctx->lsa_recv) ncclMemFree(ctx->lsa_recv);
+  ctx->lsa_dc_ok = false;
+  ctx->lsa_win = nullptr;
+  ctx->lsa_recv = nullptr;
+  ctx->lsa = false;
+#else
+  (void)ctx;
+#endif
+}
+
 int exchange_axis(clover_ctx* ctx, const std::vector<int>& bufs, int axis, int ydepth = HALO,
                   int xdepth = HALO) {
   const int s_lo = axis == 0 ? 0 : 2, s_hi = axis == 0 ? 1 : 3;
@@ -538,28 +674,43 @@ int exchange_axis(clover_ctx* ctx, const std::vector<int>& bufs, int axis, int y
       for (int side : {s_lo, s_hi}) {
         int nb = neighbour(ctx, cs, side);
         if (nb < 0 || (!ctx->virtual_remote && local_chunk(ctx, nb))) continue;
-        int64_t n = 0;
-        for (int b : bufs) {
-          XferDesc s, r;
-          side_strips(cs, b, side, s, r, ydepth, xdepth);
-          n += (int64_t)s.w * s.h;
-        }
+        const int64_t n = msg_elems(cs, side, bufs, ydepth, xdepth);
         if (off + n > ctx->xbuf_elems) return fail(CLOVER_ERR_STATE, "halo staging buffer too small");
-        n = 0;
-        for (int b : bufs) {
-          XferDesc s, r;
-          side_strips(cs, b, side, s, r, ydepth, xdepth);
-          XferDesc dst{ctx->xbuf_send + off + n, s.w, 0, 0, s.w, s.h};
-          int rc = q.add(dst, s);
-          if (rc) return rc;
-          n += (int64_t)s.w * s.h;
-        }
         msgs.push_back({ctx->owner[nb], nb, off, n, &cs, side});
         off += n;
       }
+    // pack: into the staging buffer, or -- device-initiated stores (LSA) --
+    // straight into the receiver's mailbox slot for this message
+    const bool lsa = lsa_active(ctx);
+    for (auto& m : msgs) {
+      double* dst0 = ctx->xbuf_send + m.off;
+#ifdef CLOVER_WITH_NCCL
+      if (lsa) {
+        const int64_t ro = peer_recv_off(ctx, m.peer, m.nb, m.side ^ 1, bufs, axis, ydepth, xdepth);
+        if (ro < 0 || (size_t)(ro + m.n) * 8 > ctx->lsa_bytes)
+          return fail(CLOVER_ERR_STATE, "LSA: no mailbox slot for a halo message");
+        dst0 = ctx->lsa_peer[m.peer] + ro;
+      }
+#endif
+      int64_t n = 0;
+      for (int b : bufs) {
+        XferDesc s, r;
+        side_strips(*m.cs, b, m.side, s, r, ydepth, xdepth);
+        XferDesc dst{dst0 + n, s.w, 0, 0, s.w, s.h};
+        int rc = q.add(dst, s);
+        if (rc) return rc;
+        n += (int64_t)s.w * s.h;
+      }
+    }
     int rc = q.flush();  // the staging buffer is complete before it is sent
     if (rc) return rc;
-    if (ctx->virtual_remote && ctx->virtual_nccl) {
+    if (lsa) {
+#ifdef CLOVER_WITH_NCCL
+      // every sender's stores into this rank's mailbox are complete
+      k_lsa_barrier<<<1, 128, 0, ctx->xs>>>(ctx->lsa_dc);
+      if (cudaGetLastError() != cudaSuccess) return fail(CLOVER_ERR_CUDA, "LSA barrier launch failed");
+#endif
+    } else if (ctx->virtual_remote && ctx->virtual_nccl) {
 #ifdef CLOVER_WITH_NCCL
       // one rank talks to itself: the i-th send to peer 0 matches the i-th
       // receive from peer 0, so each message's send is paired with the
@@ -621,17 +772,32 @@ int exchange_axis(clover_ctx* ctx, const std::vector<int>& bufs, int axis, int y
       return fail(CLOVER_ERR_NCCL, "libclover built without NCCL");
 #endif
     }
+    double* rbuf = ctx->xbuf_recv;
+#ifdef CLOVER_WITH_NCCL
+    if (lsa) rbuf = ctx->lsa_recv;
+#endif
     for (auto& m : msgs) {
       int64_t n = 0;
       for (int b : bufs) {
         XferDesc s, r;
         side_strips(*m.cs, b, m.side, s, r, ydepth, xdepth);
-        XferDesc src{ctx->xbuf_recv + m.off + n, r.w, 0, 0, r.w, r.h};
+        XferDesc src{rbuf + m.off + n, r.w, 0, 0, r.w, r.h};
         rc = q.add(r, src);
         if (rc) return rc;
         n += (int64_t)r.w * r.h;
       }
     }
+#ifdef CLOVER_WITH_NCCL
+    if (lsa) {
+      // every rank has unpacked its mailbox before any sender stores the
+      // next message into it
+      rc = q.flush();
+      if (rc) return rc;
+      k_lsa_barrier<<<1, 128, 0, ctx->xs>>>(ctx->lsa_dc);
+      if (cudaGetLastError() != cudaSuccess) return fail(CLOVER_ERR_CUDA, "LSA barrier launch failed");
+      return CLOVER_OK;
+    }
+#endif
   }
   return q.flush();
 }
@@ -1724,6 +1890,14 @@ int clover_init(const clover_grid* grid, const clover_state* states, int32_t nst
     std::memcpy(&id, dist->nccl_unique_id, sizeof(id));
     if (ncclCommInitRank(&ctx->comm, nranks, id, rank) != ncclSuccess)
       return bail(fail(CLOVER_ERR_NCCL, "ncclCommInitRank failed"));
+    // device-initiated halo stores over NVLink (CLOVER_LSA=1 on every rank)
+    if (const char* e = std::getenv("CLOVER_LSA")) {
+      if (std::atoi(e) != 0) {
+        int rc = lsa_setup(ctx);
+        if (rc) return bail(rc);
+        ctx->lsa = true;
+      }
+    }
   }
 #endif
 
@@ -1788,8 +1962,8 @@ int clover_debug_set_virtual_remote(clover_ctx* ctx, int32_t enable) {
   if (!ctx) return fail(CLOVER_ERR_ARG, "ctx is NULL");
   if (ctx->nranks > 1) return fail(CLOVER_ERR_STATE, "virtual remote is a single-process test mode");
   if (enable && ctx->L.px * ctx->L.py < 2) return fail(CLOVER_ERR_STATE, "virtual remote needs px*py > 1");
-  if (enable < 0 || enable > 2) return fail(CLOVER_ERR_ARG, "enable must be 0, 1 or 2");
-  if (enable == 2) {
+  if (enable < 0 || enable > 3) return fail(CLOVER_ERR_ARG, "enable must be 0, 1, 2 or 3");
+  if (enable >= 2) {
 #ifdef CLOVER_WITH_NCCL
     if (!ctx->comm) {
       // a one-rank communicator on this GPU: every halo message becomes an
@@ -1799,12 +1973,21 @@ int clover_debug_set_virtual_remote(clover_ctx* ctx, int32_t enable) {
       NK(ncclGetUniqueId(&id));
       NK(ncclCommInitRank(&ctx->comm, 1, id, 0));
     }
+    if (enable == 3) {
+      // device-initiated stores through a one-rank symmetric window: each
+      // message is stored into its receiver's mailbox slot via the peer
+      // mapping, LSA barriers around the unpack
+      CK(cudaStreamSynchronize(ctx->work));
+      int rc = lsa_setup(ctx);
+      if (rc) return rc;
+    }
+    ctx->lsa = enable == 3;
 #else
     return fail(CLOVER_ERR_NCCL, "libclover built without NCCL");
 #endif
   }
   ctx->virtual_remote = enable != 0;
-  ctx->virtual_nccl = enable == 2;
+  ctx->virtual_nccl = enable >= 2;
   for (int i = 0; i < 4; ++i)
     if (ctx->gexec[i]) {
       cudaGraphExecDestroy(ctx->gexec[i]);
@@ -2402,6 +2585,7 @@ int clover_finalize(clover_ctx* ctx) {
   }
   for (int i = 0; i < 4; ++i)
     if (ctx->gexec[i]) cudaGraphExecDestroy(ctx->gexec[i]);
+  lsa_teardown(ctx);
 #ifdef CLOVER_WITH_NCCL
   if (ctx->comm) ncclCommDestroy(ctx->comm);
 #endif

@@ -4,8 +4,9 @@ the fused y sweep across y chunk boundaries (default) or only at walls
 (round-1 schedule: separate y kernels + an extra exchange phase), and
 through the virtual-remote packing path (pack -> staging -> unpack, the
 multi-GPU message layout), by device copy and through a one-rank NCCL
-communicator; each also with deep halos (one 7-row state exchange per
-step, *_deep).  Prints one JSON line.
+communicator, and as device-initiated stores into a one-rank NCCL symmetric
+window (virtual_lsa*); each also with deep halos (one 7-row state exchange
+per step, *_deep).  Prints one JSON line.
 usage: chunk_overhead.py NX NY PX PY [STEPS]"""
 import json
 import os
@@ -30,7 +31,7 @@ def run(p, q, vr=0, walls_only=False, overlap=False, deep=False):
     if walls_only:
         sim.debug_set_fusion(True, walls_only=True)
     if vr:
-        sim.debug_set_virtual_remote(True, nccl=vr == 2)
+        sim.debug_set_virtual_remote(True, nccl=vr == 2, lsa=vr == 3)
     sim.debug_set_overlap(overlap)
     sim.step(3)
     sim.sync()
@@ -65,7 +66,8 @@ for name, kw in (("local_fused", {}), ("local_walls_only", dict(walls_only=True)
                  ("virtual_remote_overlap", dict(vr=1, overlap=True)),
                  ("virtual_nccl_overlap", dict(vr=2, overlap=True)),
                  ("local_deep", dict(deep=True)), ("virtual_remote_deep", dict(vr=1, deep=True)),
-                 ("virtual_nccl_deep", dict(vr=2, deep=True))):
+                 ("virtual_nccl_deep", dict(vr=2, deep=True)),
+                 ("virtual_lsa", dict(vr=3)), ("virtual_lsa_deep", dict(vr=3, deep=True))):
     ms, k = run(px, py, **kw)
     res[name] = {"ms": ms, "overhead": ms / one - 1.0, "kernels": k,
                  "over_serial_ideal": ms / (alone * px * py) - 1.0}

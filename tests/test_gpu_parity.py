@@ -471,6 +471,44 @@ def test_deep_halo_bitwise(torch_cuda, seed, py, mode):
     assert deep.field_summary() == one.field_summary()
 
 
+@pytest.mark.parametrize("py,deep", [(2, True), (3, True), (6, True), (3, False)])
+def test_lsa_device_initiated_halo_stores_bitwise(torch_cuda, py, deep):
+    """S:8(f) f1 device-initiated halo stores: every halo message is packed
+    straight into its receiver's slot of an NCCL symmetric window (one-rank
+    communicator, peer mapping from the window), LSA barriers around the
+    unpack; with deep halos (one 7-row state exchange per step) and the
+    per-phase schedule.  Fuzz decks, 12 steps: fields, dt history and summary
+    bitwise equal to one chunk."""
+    deck = fuzz_deck(17 + py, nx=72, ny=112)
+    deck["max_timestep"] = 1.0
+    one = make_gpu(deck)
+    g = make_gpu(deck, px=1, py=py)
+    g.debug_set_virtual_remote(True, lsa=True)
+    g.set_deep_halo(deep)
+    assert g.deep_halo_active() == deep
+    one.step(12)
+    g.step(12)
+    for f in STATE:
+        assert np.array_equal(g.read(f), one.read(f)), f
+    assert np.array_equal(g.dt_history(1, 12), one.dt_history(1, 12))
+    assert g.field_summary() == one.field_summary()
+
+
+@pytest.mark.parametrize("pxy", [(2, 2), (3, 2)])
+def test_lsa_halo_stores_2d_layouts(torch_cuda, pxy):
+    """Device-initiated stores on 2D chunk grids (x and y messages, the
+    4-chunk corners through the second axis): bitwise equal to one chunk."""
+    deck = fuzz_deck(23, nx=96, ny=80)
+    deck["max_timestep"] = 1.0
+    one, g = make_gpu(deck), make_gpu(deck, px=pxy[0], py=pxy[1])
+    g.debug_set_virtual_remote(True, lsa=True)
+    one.step(10)
+    g.step(10)
+    for f in STATE:
+        assert np.array_equal(g.read(f), one.read(f)), f
+    assert np.array_equal(g.dt_history(1, 10), one.dt_history(1, 10))
+
+
 def test_deep_halo_bm_blast_and_toggles(torch_cuda):
     """The bm blast crossing 1x4 strip boundaries for 40 steps with deep
     halos switched on and off between steps (the state halo is refreshed 7
