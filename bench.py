@@ -512,7 +512,9 @@ def main():
                                         f"configs[4]: weak scaling, 3840^2 cells per GPU, global {nx}x{ny} "
                                         f"on [0,10]^2 (reading A4)"),
                            "mesh": [nx, ny], "decomposition": f"{px}x{py}",
-                           "transport": ("nccl" if not host_tp else "host (gloo; not a bench value)")
+                           "transport": (("nccl, device-initiated LSA halo stores"
+                                          if os.environ.get("CLOVER_LSA", "0") != "0" else "nccl")
+                                         if not host_tp else "host (gloo; not a bench value)")
                            if world > 1 else None,
                            "halo_exchange": ("deep: 1 state exchange (7 rows) + dt MIN per step"
                                              if deep_halo else "per phase") if world > 1 else None,
