@@ -280,7 +280,6 @@ struct clover_ctx {
   // only if every block of that launch is co-resident: the band blocks spin
   // until the fixup blocks are done (clover_init checks the occupancy)
   bool walls_fold_fits = false;
-  bool f2_probe = false;  // CLOVER_F2_PROBE=1 at init: sweep-2 y kernel with the visc epilogue (A/B only)
   bool deep = true;       // deep halos where they apply (deep_ok; clover_set_deep_halo)
   int nsm = 148, occ[4] = {1, 1, 1, 1};  // SMs, resident blocks/SM of the 4 segment kernels (set_segs)
   int state_rows = 0;     // rows of the state's y halo known current (ensure_state_rows)
@@ -1281,16 +1280,6 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
           if (sweep == 1) {
             launch_step(ks_advec_y<1>, g, SB, sm, c, ta, tb, cs.buf[rout], cs.buf[eout], cs.buf[B_MY],
                         cs.buf[uout], cs.buf[vout], fx);
-          } else if (ctx->f2_probe) {
-            // DESIGN.md 4.5 f2 probe: sweep 2 with the next step's viscosity
-            // and calc_dt terms folded in (q written, dt to a scratch slot;
-            // visc_dt still runs, so results are unchanged)
-            ViscProbe vp;
-            vp.q = cs.buf[B_Q];
-            vp.dt = (unsigned long long*)cs.partials;
-            vp.prm = ctx->dtp;
-            launch_step(ks_advec_y2_probe, g, SB, sm, c, ta, tb, cs.buf[rout], cs.buf[eout],
-                        cs.buf[B_MY], cs.buf[uout], cs.buf[vout], fx, vp);
           } else {
             launch_step(ks_advec_y<2>, g, SB, sm, c, ta, tb, cs.buf[rout], cs.buf[eout], cs.buf[B_MY],
                         cs.buf[uout], cs.buf[vout], fx);
@@ -1867,7 +1856,6 @@ int clover_init(const clover_grid* grid, const clover_state* states, int32_t nst
     const int64_t resident = (int64_t)nsm * std::min(b1, b2);
     ctx->walls_fold_fits = ctx->chunks.size() == 1 &&
                            (int64_t)FIX_BLOCKS + 5 * ywalls_of(ctx->chunks[0], 1).nbx <= resident;
-    if (const char* e = std::getenv("CLOVER_F2_PROBE")) ctx->f2_probe = std::atoi(e) != 0;
     if (const char* e = std::getenv("CLOVER_WALLS_FOLD_LIMIT"))  // test hook: force the unfolded path
       ctx->walls_fold_fits = ctx->walls_fold_fits && std::atoi(e) != 0;
   }

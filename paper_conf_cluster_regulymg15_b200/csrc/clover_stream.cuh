@@ -1545,17 +1545,7 @@ template <> struct YL<2> {  // tensors fy | d2 e2 u2 v2
   static constexpr unsigned BYTES = 5 * YRW * 8;
 };
 
-// VISC (f2 probe; CLOVER_F2_PROBE): the interior body also
-// evaluates the NEXT step's viscosity and calc_dt terms of cell row s-2
-// from the post-sweep values it holds in registers (lanes 1..30; the last
-// row of each segment is skipped) and writes q -- an upper bound on what
-// folding visc_dt into sweep 2 would save, measured, not a production path.
-struct ViscProbe {
-  double* q = nullptr;
-  unsigned long long* dt = nullptr;
-  DtParams prm{};
-};
-template <int SWEEP, class D, bool EDGE, bool VISC = false>
+template <int SWEEP, class D, bool EDGE>
 __device__ __forceinline__ bool advec_y_body(const Chunk& c, const CUtensorMap* __restrict__ ta,
                                              const CUtensorMap* __restrict__ tb,
                                              double* __restrict__ rho_out,
@@ -1563,8 +1553,7 @@ __device__ __forceinline__ bool advec_y_body(const Chunk& c, const CUtensorMap* 
                                              const double* __restrict__ mfy,
                                              double* __restrict__ uout,
                                              double* __restrict__ vout, int gw, int k0, int k1,
-                                             int lane, double* ring, unsigned long long* bars,
-                                             const ViscProbe& vp = ViscProbe{}) {
+                                             int lane, double* ring, unsigned long long* bars) {
   using L = YL<SWEEP>;
   D dv;
   const int J0 = 1 + YW * gw;
@@ -1683,10 +1672,6 @@ __device__ __forceinline__ bool advec_y_body(const Chunk& c, const CUtensorMap* 
   double myl_s = __shfl_up_sync(FULL, m_s, 1);
   double mp_p = 0.0, mpl_p = 0.0, nf_p = 0.0, pre_p = 0.0, post_p = 0.0;
   double mu_b = 0.0, mv_b = 0.0;  // momentum flux of node s-2
-  // VISC: p of cells s-1..s-3, rho/e of cells s-1, s-2, u/v of node s-2
-  double vp1 = 0.0, vp2 = 0.0, vp3 = 0.0, vr1 = 0.0, vr2 = 0.0, ve1 = 0.0, ve2 = 0.0;
-  double vu2 = 0.0, vv2 = 0.0;
-  DtAcc vacc;
   // ring rows s-2 .. s+2 of the iteration, rotated at its end (one slot
   // address per row instead of one per access); slot / phase of row s+2
   // for its mbarrier wait (rows k0-4 .. k0 are slots 0 .. 4 at s = k0-2)
@@ -1703,7 +1688,7 @@ __device__ __forceinline__ bool advec_y_body(const Chunk& c, const CUtensorMap* 
     if (s + 2 <= r_last) mbar_wait(&bars[wsl], wph);
     {
       // ---- advec_cell y: face s+1, cell s
-      double m1 = 0.0, ef1 = 0.0, pv1 = 0.0, ro = 0.0, eo_s = 0.0;
+      double m1 = 0.0, ef1 = 0.0, pv1 = 0.0, ro = 0.0;
       if (face_computed(s + 1)) {
         pv1 = pre_vol_p(Rp1, Rp2);
         if (comp) face_flux_p(Rm1, R0, Rp1, Rp2, pv_s, pv1, m1, ef1);
@@ -1715,7 +1700,6 @@ __device__ __forceinline__ bool advec_y_body(const Chunk& c, const CUtensorMap* 
           double eo;
           cell_update(dv, R0[L::R], R0[L::E], pv_s, m_s, m1, ef_s, ef1, R0[L::FY], Rp1[L::FY],
                       ro, eo);
-          eo_s = eo;
           if (own_cell && s >= k0 && s < k1) {
             const int i = idx(c, j, s);
             const bool near = EDGE && (ncol || near_wall_row(c, s));
@@ -1740,7 +1724,6 @@ __device__ __forceinline__ bool advec_y_body(const Chunk& c, const CUtensorMap* 
       const double pre = post - nf_p + nf;
       // momentum flux of node s-1, then the update of node s-1 (fluxes of
       // nodes s-2 and s-1; node masses of row s-1)
-      double un_s = 0.0, vn_s = 0.0;
       if (s >= k0 && own_node) {
         const double nfn = nf_p;
         const double nmp = (nfn < 0.0) ? pre : pre_p;
@@ -1758,39 +1741,12 @@ __device__ __forceinline__ bool advec_y_body(const Chunk& c, const CUtensorMap* 
           const int kn = s - 1;
           double un, vn;
           mom_update(dv, qm1[L::U], qm1[L::V], pre_p, post_p, mu_b, mu_c, mv_b, mv_c, un, vn);
-          un_s = un; vn_s = vn;
           const int i = idx(c, j, kn);
           const bool near = EDGE && (ncol || near_wall_row(c, kn));
           store_at(c, uout, K_XVEL, j, kn, i, near, un);
           store_at(c, vout, K_YVEL, j, kn, i, near, vn);
         }
         mu_b = mu_c; mv_b = mv_c;
-      }
-      if constexpr (VISC) {
-        // viscosity + calc_dt terms of cell row s-2 (nodes s-2 and s-1 are done)
-        const double pcur = eos_pressure(ro, eo_s);
-        if (s >= k0 + 2) {
-          ViscIn I;
-          I.rho = vr2; I.e = ve2;
-          I.pb = vp3; I.pt = vp1;
-          I.pl = __shfl_up_sync(FULL, vp2, 1);
-          I.pr = __shfl_down_sync(FULL, vp2, 1);
-          I.u00 = vu2; I.v00 = vv2;
-          I.u10 = __shfl_down_sync(FULL, vu2, 1);
-          I.v10 = __shfl_down_sync(FULL, vv2, 1);
-          I.u01 = un_s; I.v01 = vn_s;
-          I.u11 = __shfl_down_sync(FULL, un_s, 1);
-          I.v11 = __shfl_down_sync(FULL, vn_s, 1);
-          if (lane >= 1 && lane <= 30) {
-            double qv, cc2, c2;
-            visc_cell(dv, I, c, qv, cc2, c2);
-            vacc.add(I, c, qv, cc2, c2, false);
-            vp.q[idx(c, j, s - 2)] = qv;
-          }
-        }
-        vp3 = vp2; vp2 = vp1; vp1 = pcur;
-        vr2 = vr1; vr1 = ro; ve2 = ve1; ve1 = eo_s;
-        vu2 = un_s; vv2 = vn_s;
       }
       m_s = m1; ef_s = ef1; pv_s = pv1; myl_s = myl1;
       mp_p = mp; mpl_p = mpl; nf_p = nf;
@@ -1813,11 +1769,6 @@ __device__ __forceinline__ bool advec_y_body(const Chunk& c, const CUtensorMap* 
   if (lane == 0)
     for (int t = 0; t < L::RING; ++t) mbar_inval(&bars[t]);  // the ring may be reused (fixup)
   __syncwarp();
-  if constexpr (VISC) {
-    double d = (lane >= 1 && lane <= 30 && k1 - k0 >= 3) ? vacc.dt(c, vp.prm) : G_BIG;
-    for (int o = 16; o > 0; o >>= 1) d = fmin(d, __shfl_xor_sync(FULL, d, o));
-    if (lane == 0) atomicMin(vp.dt, (unsigned long long)__double_as_longlong(d));
-  }
   return __any_sync(FULL, dv.bad);
 }
 
@@ -1859,33 +1810,6 @@ ks_advec_y(Chunk c, const __grid_constant__ CUtensorMap ta, const __grid_constan
   if (advec_y_seg<SWEEP, DivFast>(c, &ta, &tb, rho_out, en_out, mfy, uout, vout, gw, k0, k1, lane,
                                   ring[w], bars[w]))
     fix_push(fix, lane, gw, (unsigned)seg_y(c));
-}
-
-// the f2 probe kernel: interior segments run advec_y_body<2, DivFast,
-// false, true>, edge segments the production body
-__global__ void __launch_bounds__(SB, YL<2>::MINB)
-ks_advec_y2_probe(Chunk c, const __grid_constant__ CUtensorMap ta,
-                  const __grid_constant__ CUtensorMap tb, double* __restrict__ rho_out,
-                  double* __restrict__ en_out, const double* __restrict__ mfy,
-                  double* __restrict__ uout, double* __restrict__ vout, FixSlot fix,
-                  ViscProbe vp) {
-  pdl_trigger();
-  pdl_wait();
-  __shared__ __align__(128) double ring[SB / 32][YL<2>::RING * YL<2>::SLOT];
-  __shared__ __align__(8) unsigned long long bars[SB / 32][YL<2>::RING];
-  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-  const int gw = blockIdx.x * (SB / 32) + w;
-  int k0, len;
-  seg_rows_of(seg_y(c), c.yks, c.ynb, k0, len);
-  const int k1 = min(k0 + len, c.ny + 2);
-  bool bad;
-  if (y_fused_interior(c, gw, k0, k1))
-    bad = advec_y_body<2, DivFast, false, true>(c, &ta, &tb, rho_out, en_out, mfy, uout, vout, gw,
-                                                k0, k1, lane, ring[w], bars[w], vp);
-  else
-    bad = advec_y_body<2, DivFast, true>(c, &ta, &tb, rho_out, en_out, mfy, uout, vout, gw, k0, k1,
-                                         lane, ring[w], bars[w]);
-  if (bad) fix_push(fix, lane, gw, (unsigned)seg_y(c));
 }
 
 template <int SWEEP>
