@@ -101,6 +101,35 @@ def test_gpu_checkpoint_restart_bitwise():
 
 
 @pytest.mark.gpu
+def test_gpu_checkpoint_across_decompositions_with_deep_halos():
+    """A checkpoint is the global state: taken on one chunk, restarted on 1x4
+    y strips with deep halos (the restart refreshes the state halo 7 rows
+    deep), and back; the continued runs stay bitwise equal to one chunk."""
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_cluster_regulymg15_b200 import Clover
+    deck = bm_deck(96, 128)
+    one = Clover(deck)
+    one.step(6)
+    blob = one.checkpoint()
+    one.step(8)
+    strips = Clover(deck, px=1, py=4)
+    assert strips.deep_halo_active()
+    strips.restart(blob)
+    strips.step(5)
+    blob2 = strips.checkpoint()
+    strips.step(3)
+    back = Clover(deck)
+    back.restart(blob2)
+    back.step(3)
+    for f in STATE:
+        assert np.array_equal(strips.read(f), one.read(f)), f
+        assert np.array_equal(back.read(f), one.read(f)), f
+    assert np.array_equal(strips.dt_history(7, 8), one.dt_history(7, 8))
+
+
+@pytest.mark.gpu
 def test_gpu_restart_rejects_other_mesh():
     import torch
     if not torch.cuda.is_available():
