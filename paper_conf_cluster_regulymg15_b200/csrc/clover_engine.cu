@@ -166,10 +166,7 @@ int seg_rows(int ks, int64_t colblocks, int nrows) {
 }
 // Segment rows of a kernel grid whose first nb segments have ks rows and
 // the rest ks/2 (seg_rows_of).
-int seg_count(int ks, int nb, int rows) {
-  if ((int64_t)nb * ks >= rows) return cdiv(rows, ks);
-  return nb + cdiv(rows - nb * ks, ks / CLOVER_TAIL_DIV);
-}
+int seg_count(int ks, int nb, int rows) { return seg_count_of(ks, nb, rows); }
 // Full-height segments: all but about CLOVER_TAIL_WAVES waves of blocks
 // (slots resident blocks on the GPU, colblocks blocks per segment row),
 // which run at 1/CLOVER_TAIL_DIV height so the kernel's tail shrinks.
@@ -281,6 +278,7 @@ struct clover_ctx {
   // until the fixup blocks are done (clover_init checks the occupancy)
   bool walls_fold_fits = false;
   bool deep = true;       // deep halos where they apply (deep_ok; clover_set_deep_halo)
+  bool batch = true;      // several local chunks: one launch per kernel (KBatch; CLOVER_BATCH=0 off)
   int nsm = 148, occ[4] = {1, 1, 1, 1};  // SMs, resident blocks/SM of the 4 segment kernels (set_segs)
   int state_rows = 0;     // rows of the state's y halo known current (ensure_state_rows)
   cudaGraphExec_t gexec[4] = {nullptr, nullptr, nullptr, nullptr};  // [parity + 2 * multi-step]
@@ -1060,6 +1058,9 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
   const bool walls_in_x1 = CLOVER_YWALLS_FOLD && fold1 && advect_x && fuse_x_ok(ctx) && nphase >= 6;
   int cur_prof_id = P_VISC_DT;
   const bool deep = deep_ok(ctx);
+  // several local chunks: one launch per kernel for all of them (KBatch)
+  const bool batch = ctx->batch && CLOVER_SERP == 0 && ctx->chunks.size() > 1 &&
+                     ctx->chunks.size() <= (size_t)MAX_BATCH;
   if (ctx->prof) prof_mark(ctx, -1);
   // one chunk on one rank: the visc fixup's last block finalises dt (no
   // k_dt_finalize launch); else the slot is combined first (NCCL MIN)
@@ -1074,8 +1075,18 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
   // the next phase waits for both.
   // ext > 0 (deep halos): the kernels run on each chunk's view extended
   // ext rows beyond its y chunk boundaries (deep_view); bufs may be empty.
-  auto run_phase = [&](int kind, auto&& launch, auto&& fixup, const std::vector<int>& bufs, int yd,
-                       int xd, int ext = 0) -> int {
+  // batched (several local chunks, no overlap): launch_b(views) runs the
+  // streaming kernel and its fixup once for all chunks (blockIdx.z = chunk).
+  auto run_phase = [&](int kind, auto&& launch, auto&& fixup, auto&& launch_b,
+                       const std::vector<int>& bufs, int yd, int xd, int ext = 0) -> int {
+    if (batch && (ext > 0 || !overlap_ok(ctx))) {
+      std::vector<ChunkState> views;
+      views.reserve(ctx->chunks.size());
+      for (auto& cs0 : ctx->chunks) views.push_back(ext > 0 ? deep_view(ctx, cs0, ext) : cs0);
+      int rc = launch_b(views);
+      if (rc) return rc;
+      return bufs.empty() ? CLOVER_OK : exchange(ctx, bufs, yd, xd);
+    }
     if (ext > 0 || !overlap_ok(ctx)) {
       for (auto& cs0 : ctx->chunks) {
         ChunkState view;
@@ -1128,7 +1139,28 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
     CK(cudaStreamWaitEvent(st, ctx->ev_x, 0));
     return CLOVER_OK;
   };
-  if (nphase >= 1) {
+  if (nphase >= 1 && batch) {
+    KBatch<VArgs> vb;
+    dim3 g(1, 1, (unsigned)ctx->chunks.size());
+    for (size_t t = 0; t < ctx->chunks.size(); ++t) {
+      const ChunkState v = deep ? deep_view(ctx, ctx->chunks[t], DEEP_EXT_VISC) : ctx->chunks[t];
+      vb.a[t].c = v.c;
+      vb.a[t].tm = v.tm_visc;
+      vb.a[t].q = v.buf[B_Q];
+      vb.a[t].fix = v.fix;
+      g.x = std::max(g.x, grid_cols(v.c.nx, v.c.ny, v.c.vks).x);
+      g.y = std::max<unsigned>(g.y, (unsigned)seg_count(v.c.vks, v.c.vnb, v.c.ny));
+    }
+    launch_step(ks_visc_dt_b, g, SB, st, vb, ctx->scal, ctx->dtp);
+    STEP_LAUNCH_CHECK();
+    launch_fix(kf_visc_dt_b, dim3(FIX_BLOCKS, 1, g.z), SB, st, vb, ctx->scal, ctx->dtp);
+    FIX_LAUNCH_CHECK();
+    if (needs_exchange(ctx) && !deep) {
+      int rc = exchange_axis(ctx, {B_Q}, 0);
+      if (rc) return rc;
+    }
+    if (ctx->prof) prof_mark(ctx, -1);
+  } else if (nphase >= 1) {
     for (auto& cs0 : ctx->chunks) {
       // deep halos: q (and the dt terms) of DEEP_EXT_VISC rows beyond the
       // chunk, the rows the Lagrangian view reads (no q exchange)
@@ -1191,10 +1223,27 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
       FIX_LAUNCH_CHECK();
       return CLOVER_OK;
     };
+    auto launch_b = [&](std::vector<ChunkState>& vs) -> int {
+      KBatch<LArgs> lb;
+      dim3 g(1, 1, (unsigned)vs.size());
+      for (size_t t = 0; t < vs.size(); ++t) {
+        const ChunkState& v = vs[t];
+        lb.a[t] = LArgs{v.c, v.tm_lag, v.buf[B_D1], v.buf[B_E1], v.buf[B_U1], v.buf[B_V1],
+                        v.buf[B_FX], v.buf[B_FY], v.fix};
+        g.x = std::max(g.x, grid_strip(v.c.nx, LW, v.c.ny, v.c.lks).x);
+        g.y = std::max<unsigned>(g.y, (unsigned)seg_count(v.c.lks, v.c.lnb, v.c.ny));
+      }
+      launch_step(ks_lagrangian_b, g, SB, st, lb, ctx->scal);
+      STEP_LAUNCH_CHECK();
+      launch_fix(kf_lagrangian_b, dim3(FIX_BLOCKS, 1, g.z), SB, st, lb, ctx->scal);
+      FIX_LAUNCH_CHECK();
+      return CLOVER_OK;
+    };
     // a fused y sweep (either sweep) reads these FUSE_ROWS deep in y; with
     // deep halos the phase runs DEEP_EXT_LAGR rows beyond the chunk instead
-    int rc = deep ? run_phase(SEG_LAGR, launch, fixup, {}, 0, 0, DEEP_EXT_LAGR)
-                  : run_phase(SEG_LAGR, launch, fixup, {B_D1, B_E1, B_U1, B_V1, B_FX, B_FY},
+    int rc = deep ? run_phase(SEG_LAGR, launch, fixup, launch_b, {}, 0, 0, DEEP_EXT_LAGR)
+                  : run_phase(SEG_LAGR, launch, fixup, launch_b,
+                              {B_D1, B_E1, B_U1, B_V1, B_FX, B_FY},
                               fuse_y_ok(ctx) ? FUSE_ROWS : HALO, fuse_x_ok(ctx) ? HALO_COLS : HALO);
     if (rc) return rc;
     if (ctx->prof) prof_mark(ctx, -1);
@@ -1239,13 +1288,31 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
           FIX_LAUNCH_CHECK();
           return CLOVER_OK;
         };
+        auto launch_b = [&](std::vector<ChunkState>& vs) -> int {
+          KBatch<XArgs> xb;
+          dim3 g(1, 1, (unsigned)vs.size());
+          for (size_t t = 0; t < vs.size(); ++t) {
+            const ChunkState& v = vs[t];
+            xb.a[t] = XArgs{v.c, sweep == 1 ? v.tm_x1 : v.tm_x2, v.buf[rout], v.buf[eout],
+                            v.buf[uout], v.buf[vout], v.fix};
+            g.x = std::max(g.x, grid_strip(v.c.nx + 1, XW, v.c.ny + 1, v.c.xks).x);
+            g.y = std::max<unsigned>(g.y, (unsigned)seg_count(v.c.xks, v.c.xnb, v.c.ny + 1));
+          }
+          if (sweep == 1) launch_step(ks_advec_x_b<1>, g, SB, st, xb);
+          else launch_step(ks_advec_x_b<2>, g, SB, st, xb);
+          STEP_LAUNCH_CHECK();
+          if (sweep == 1) launch_fix(kf_advec_x_b<1>, dim3(FIX_BLOCKS, 1, g.z), SB, st, xb);
+          else launch_fix(kf_advec_x_b<2>, dim3(FIX_BLOCKS, 1, g.z), SB, st, xb);
+          FIX_LAUNCH_CHECK();
+          return CLOVER_OK;
+        };
         // sweep 1 feeds a fused y sweep 2: FUSE_ROWS deep in y.  Deep
         // halos: sweep 1 runs DEEP_EXT_X1 rows beyond the chunk (the rows the
         // y sweep 2 reads), sweep 2 ends the step with the one exchange
-        int rc = !deep ? run_phase(SEG_X, launch, fixup, {rout, eout, uout, vout},
+        int rc = !deep ? run_phase(SEG_X, launch, fixup, launch_b, {rout, eout, uout, vout},
                                    (sweep == 1 && fuse_y_ok(ctx)) ? FUSE_ROWS : HALO, HALO)
-                 : sweep == 1 ? run_phase(SEG_X, launch, fixup, {}, 0, 0, DEEP_EXT_X1)
-                              : run_phase(SEG_X, launch, fixup, {rout, eout, uout, vout},
+                 : sweep == 1 ? run_phase(SEG_X, launch, fixup, launch_b, {}, 0, 0, DEEP_EXT_X1)
+                              : run_phase(SEG_X, launch, fixup, launch_b, {rout, eout, uout, vout},
                                           DEEP_ROWS, HALO);
         if (rc) return rc;
         if (ctx->prof) prof_mark(ctx, -1);
@@ -1303,10 +1370,29 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
         // y sweep 1 feeds a fused x sweep 2: HALO_COLS deep in x.  Deep
         // halos: sweep 1 runs DEEP_EXT_Y1 rows beyond the chunk, sweep 2 ends
         // the step with the one exchange
-        int rc = !deep ? run_phase(SEG_Y, launch, fixup, {rout, eout, uout, vout}, HALO,
+        auto launch_b = [&](std::vector<ChunkState>& vs) -> int {
+          KBatch<YArgs> yb;
+          dim3 g(1, 1, (unsigned)vs.size());
+          for (size_t t = 0; t < vs.size(); ++t) {
+            const ChunkState& v = vs[t];
+            yb.a[t] = YArgs{v.c, sweep == 1 ? v.tm_x1 : v.tm_fy, sweep == 1 ? v.tm_x1 : v.tm_c4,
+                            v.buf[rout], v.buf[eout], v.buf[B_MY], v.buf[uout], v.buf[vout],
+                            v.fix};
+            g.x = std::max(g.x, grid_strip(v.c.nx + 1, YW, v.c.ny + 1, v.c.yks).x);
+            g.y = std::max<unsigned>(g.y, (unsigned)seg_count(v.c.yks, v.c.ynb, v.c.ny + 1));
+          }
+          if (sweep == 1) launch_step(ks_advec_y_b<1>, g, SB, st, yb);
+          else launch_step(ks_advec_y_b<2>, g, SB, st, yb);
+          STEP_LAUNCH_CHECK();
+          if (sweep == 1) launch_fix(kf_advec_y_b<1>, dim3(FIX_BLOCKS, 1, g.z), SB, st, yb);
+          else launch_fix(kf_advec_y_b<2>, dim3(FIX_BLOCKS, 1, g.z), SB, st, yb);
+          FIX_LAUNCH_CHECK();
+          return CLOVER_OK;
+        };
+        int rc = !deep ? run_phase(SEG_Y, launch, fixup, launch_b, {rout, eout, uout, vout}, HALO,
                                    (sweep == 1 && fuse_x_ok(ctx)) ? HALO_COLS : HALO)
-                 : sweep == 1 ? run_phase(SEG_Y, launch, fixup, {}, 0, 0, DEEP_EXT_Y1)
-                              : run_phase(SEG_Y, launch, fixup, {rout, eout, uout, vout},
+                 : sweep == 1 ? run_phase(SEG_Y, launch, fixup, launch_b, {}, 0, 0, DEEP_EXT_Y1)
+                              : run_phase(SEG_Y, launch, fixup, launch_b, {rout, eout, uout, vout},
                                           DEEP_ROWS, HALO);
         if (rc) return rc;
         if (ctx->prof) prof_mark(ctx, -1);
@@ -1762,6 +1848,7 @@ int clover_init(const clover_grid* grid, const clover_state* states, int32_t nst
   // y-strip layout): clover_set_deep_halo or CLOVER_DEEP_HALO=0
   ctx->deep = true;
   if (const char* e = std::getenv("CLOVER_DEEP_HALO")) ctx->deep = std::atoi(e) != 0;
+  if (const char* e = std::getenv("CLOVER_BATCH")) ctx->batch = std::atoi(e) != 0;
   {
     int dev = 0;
     cudaGetDevice(&dev);

@@ -1827,6 +1827,169 @@ kf_advec_y(Chunk c, const __grid_constant__ CUtensorMap ta, const __grid_constan
   });
 }
 
+// ================================================================ batched launches
+// Several chunks of one process in one launch (blockIdx.z = chunk): the
+// streaming kernels and their IEEE fixups above, with each chunk's view,
+// tensor maps, outputs and fix list taken from one __grid_constant__ array.
+// The grid is the largest chunk's; blocks beyond a chunk's strips or row
+// segments return at once.  Forward segment order only (Chunk.rev = 0).
+// (One chunk per GPU keeps the single-chunk kernels; this removes the
+// per-chunk launches and tails when a process owns several chunks.)
+constexpr int MAX_BATCH = 16;
+template <class A> struct KBatch { A a[MAX_BATCH]; };
+struct VArgs { Chunk c; CUtensorMap tm; double* q; FixSlot fix; };
+struct LArgs { Chunk c; CUtensorMap tm; double *d1, *e1, *u1, *v1, *fx, *fy; FixSlot fix; };
+struct XArgs { Chunk c; CUtensorMap tm; double *rho, *en, *u, *v; FixSlot fix; };
+struct YArgs {
+  Chunk c; CUtensorMap ta, tb; double *rho, *en; const double* mfy; double *u, *v; FixSlot fix;
+};
+
+__global__ void LB_VISC
+ks_visc_dt_b(const __grid_constant__ KBatch<VArgs> b, StepScalars* __restrict__ s, DtParams prm) {
+  pdl_trigger();
+  pdl_wait();
+  const VArgs& a = b.a[blockIdx.z];
+  const Chunk& c = a.c;
+  if ((int)blockIdx.y >= seg_count_of(c.vks, c.vnb, c.ny)) return;
+  __shared__ __align__(128) double ring[SB / 32][VSTG * VSLOT];
+  __shared__ __align__(8) unsigned long long bars[SB / 32][VSTG];
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int gw = blockIdx.x * (SB / 32) + warp;
+  double dtw = G_BIG;
+  int k0, len;
+  seg_rows_of((int)blockIdx.y, c.vks, c.vnb, k0, len);
+  int k1 = min(k0 + len, c.ny + 1);
+  visc_ring_rows(c, k0, k1);
+  if (gw * 32 < c.nx) {
+    if (visc_seg<DivFast>(c, &a.tm, a.q, prm, gw, k0, k1, lane, ring[warp], bars[warp], dtw)) {
+      fix_push(a.fix, lane, gw, blockIdx.y);
+      dtw = G_BIG;
+    }
+  }
+  __shared__ double wmin[SB / 32];
+  if (lane == 0) wmin[warp] = dtw;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    double m = wmin[0];
+    for (int w = 1; w < SB / 32; ++w) m = fmin(m, wmin[w]);
+    atomicMin(&s->dt_slot, (unsigned long long)__double_as_longlong(m));
+  }
+}
+__global__ void __launch_bounds__(SB)
+kf_visc_dt_b(const __grid_constant__ KBatch<VArgs> b, StepScalars* __restrict__ s, DtParams prm) {
+  pdl_trigger();
+  pdl_wait();
+  const VArgs& a = b.a[blockIdx.z];
+  const Chunk& c = a.c;
+  __shared__ __align__(128) double ring[SB / 32][VSTG * VSLOT];
+  __shared__ __align__(8) unsigned long long bars[SB / 32][VSTG];
+  fix_loop(a.fix, c.vks, c.vnb, c.ny + 1, [&](int gw, int k0, int k1, int lane, int w) {
+    double dtw;
+    visc_ring_rows(c, k0, k1);
+    visc_seg<DivIEEE>(c, &a.tm, a.q, prm, gw, k0, k1, lane, ring[w], bars[w], dtw);
+    if (lane == 0) atomicMin(&s->dt_slot, (unsigned long long)__double_as_longlong(dtw));
+  });
+}
+
+__global__ void LB_HEAVY
+ks_lagrangian_b(const __grid_constant__ KBatch<LArgs> b, const StepScalars* __restrict__ s) {
+  pdl_trigger();
+  pdl_wait();
+  const LArgs& a = b.a[blockIdx.z];
+  const Chunk& c = a.c;
+  if ((int)blockIdx.y >= seg_count_of(c.lks, c.lnb, c.ny)) return;
+  __shared__ __align__(128) double ring[SB / 32][LSTG * LSLOT];
+  __shared__ __align__(8) unsigned long long bars[SB / 32][LSTG];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const int gw = blockIdx.x * (SB / 32) + w;
+  int k0, len;
+  seg_rows_of((int)blockIdx.y, c.lks, c.lnb, k0, len);
+  const int k1 = min(k0 + len, c.ny + 1);
+  if (lagr_seg<DivFast>(c, &a.tm, a.d1, a.e1, a.u1, a.v1, a.fx, a.fy, s, gw, k0, k1, lane, ring[w],
+                        bars[w]))
+    fix_push(a.fix, lane, gw, blockIdx.y);
+}
+__global__ void __launch_bounds__(SB)
+kf_lagrangian_b(const __grid_constant__ KBatch<LArgs> b, StepScalars* __restrict__ s) {
+  pdl_trigger();
+  pdl_wait();
+  const LArgs& a = b.a[blockIdx.z];
+  const Chunk& c = a.c;
+  __shared__ __align__(128) double ring[SB / 32][LSTG * LSLOT];
+  __shared__ __align__(8) unsigned long long bars[SB / 32][LSTG];
+  fix_loop(a.fix, c.lks, c.lnb, c.ny + 1, [&](int gw, int k0, int k1, int lane, int w) {
+    if (lagr_seg<DivIEEE>(c, &a.tm, a.d1, a.e1, a.u1, a.v1, a.fx, a.fy, s, gw, k0, k1, lane,
+                          ring[w], bars[w]) &&
+        lane == 0)
+      atomicCAS(&s->err, 0, -6);  // CLOVER_ERR_NEG_VOLUME
+  });
+}
+
+template <int SWEEP>
+__global__ void LB_ADVX ks_advec_x_b(const __grid_constant__ KBatch<XArgs> b) {
+  pdl_trigger();
+  pdl_wait();
+  const XArgs& a = b.a[blockIdx.z];
+  const Chunk& c = a.c;
+  if ((int)blockIdx.y >= seg_count_of(c.xks, c.xnb, c.ny + 1)) return;
+  __shared__ __align__(128) double ring[SB / 32][XSTG * xslot<SWEEP>()];
+  __shared__ __align__(8) unsigned long long bars[SB / 32][XSTG];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const int gw = blockIdx.x * (SB / 32) + w;
+  int k0, len;
+  seg_rows_of((int)blockIdx.y, c.xks, c.xnb, k0, len);
+  const int k1 = min(k0 + len, c.ny + 2);
+  if (advec_x_seg<SWEEP, DivFast>(c, &a.tm, a.rho, a.en, a.u, a.v, gw, k0, k1, lane, ring[w],
+                                   bars[w]))
+    fix_push(a.fix, lane, gw, blockIdx.y);
+}
+template <int SWEEP>
+__global__ void __launch_bounds__(SB) kf_advec_x_b(const __grid_constant__ KBatch<XArgs> b) {
+  pdl_trigger();
+  pdl_wait();
+  const XArgs& a = b.a[blockIdx.z];
+  const Chunk& c = a.c;
+  __shared__ __align__(128) double ring[SB / 32][XSTG * xslot<SWEEP>()];
+  __shared__ __align__(8) unsigned long long bars[SB / 32][XSTG];
+  fix_loop(a.fix, c.xks, c.xnb, c.ny + 2, [&](int gw, int k0, int k1, int lane, int w) {
+    advec_x_seg<SWEEP, DivIEEE>(c, &a.tm, a.rho, a.en, a.u, a.v, gw, k0, k1, lane, ring[w],
+                                 bars[w]);
+  });
+}
+
+template <int SWEEP>
+__global__ void __launch_bounds__(SB, YL<SWEEP>::MINB)
+ks_advec_y_b(const __grid_constant__ KBatch<YArgs> b) {
+  pdl_trigger();
+  pdl_wait();
+  const YArgs& a = b.a[blockIdx.z];
+  const Chunk& c = a.c;
+  if ((int)blockIdx.y >= seg_count_of(c.yks, c.ynb, c.ny + 1)) return;
+  __shared__ __align__(128) double ring[SB / 32][YL<SWEEP>::RING * YL<SWEEP>::SLOT];
+  __shared__ __align__(8) unsigned long long bars[SB / 32][YL<SWEEP>::RING];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const int gw = blockIdx.x * (SB / 32) + w;
+  int k0, len;
+  seg_rows_of((int)blockIdx.y, c.yks, c.ynb, k0, len);
+  const int k1 = min(k0 + len, c.ny + 2);
+  if (advec_y_seg<SWEEP, DivFast>(c, &a.ta, &a.tb, a.rho, a.en, a.mfy, a.u, a.v, gw, k0, k1, lane,
+                                  ring[w], bars[w]))
+    fix_push(a.fix, lane, gw, blockIdx.y);
+}
+template <int SWEEP>
+__global__ void __launch_bounds__(SB) kf_advec_y_b(const __grid_constant__ KBatch<YArgs> b) {
+  pdl_trigger();
+  pdl_wait();
+  const YArgs& a = b.a[blockIdx.z];
+  const Chunk& c = a.c;
+  __shared__ __align__(128) double ring[SB / 32][YL<SWEEP>::RING * YL<SWEEP>::SLOT];
+  __shared__ __align__(8) unsigned long long bars[SB / 32][YL<SWEEP>::RING];
+  fix_loop(a.fix, c.yks, c.ynb, c.ny + 2, [&](int gw, int k0, int k1, int lane, int w) {
+    advec_y_seg<SWEEP, DivIEEE>(c, &a.ta, &a.tb, a.rho, a.en, a.mfy, a.u, a.v, gw, k0, k1, lane,
+                                ring[w], bars[w]);
+  });
+}
+
 // the y-wall bands as their own launch (several chunks or ranks; see YWalls)
 template <int SWEEP>
 __global__ void __launch_bounds__(SB)

@@ -511,6 +511,29 @@ def test_lsa_halo_stores_2d_layouts(torch_cuda, pxy):
     assert np.array_equal(g.dt_history(1, 10), one.dt_history(1, 10))
 
 
+@pytest.mark.parametrize("pxy,deep", [((1, 4), True), ((1, 4), False), ((2, 3), False),
+                                      ((1, 16), False)])
+def test_batched_chunk_launches_bitwise(torch_cuda, monkeypatch, pxy, deep):
+    """Several chunks in one process: every streaming kernel and its fixup is
+    one launch for all chunks (blockIdx.z = chunk, KBatch) -- the same bits
+    as one launch per chunk (CLOVER_BATCH=0) and as one chunk."""
+    deck = fuzz_deck(31, nx=80, ny=128)
+    deck["max_timestep"] = 1.0
+    one = make_gpu(deck)
+    b = make_gpu(deck, px=pxy[0], py=pxy[1])
+    monkeypatch.setenv("CLOVER_BATCH", "0")
+    per = make_gpu(deck, px=pxy[0], py=pxy[1])
+    for g in (b, per):
+        g.set_deep_halo(deep)
+    for g in (one, b, per):
+        g.step(11)
+    for f in STATE:
+        a = one.read(f)
+        assert np.array_equal(b.read(f), a), f
+        assert np.array_equal(per.read(f), a), f
+    assert np.array_equal(b.dt_history(1, 11), one.dt_history(1, 11))
+
+
 def test_deep_halo_bm_blast_and_toggles(torch_cuda):
     """The bm blast crossing 1x4 strip boundaries for 40 steps with deep
     halos switched on and off between steps (the state halo is refreshed 7
