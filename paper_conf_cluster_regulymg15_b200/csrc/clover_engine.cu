@@ -963,6 +963,21 @@ bool deep_ok(const clover_ctx* ctx) {
   return true;
 }
 
+// Serpentine segment order: each step kernel reads what the previous one
+// wrote, so alternate kernels run their row segments top-down (seg_y) and
+// start on the rows still in L2: visc_dt and sweep 1 reversed, the
+// Lagrangian phase and sweep 2 forward.  Measured at 3840^2: no gain
+// (visc_dt +0.004 ms, Lagrangian -0.002 ms), so off by default.
+#ifndef CLOVER_SERP
+#define CLOVER_SERP 0
+#endif
+// Several local chunks: each streaming kernel and its fixup is one launch
+// for all of them (KBatch, blockIdx.z = chunk; forward segment order).
+bool batch_ok(const clover_ctx* ctx) {
+  return ctx->batch && CLOVER_SERP == 0 && ctx->chunks.size() > 1 &&
+         ctx->chunks.size() <= (size_t)MAX_BATCH;
+}
+
 // Row-segment parameters of a chunk (or view) of c.ny rows (see seg_rows,
 // tail_nb): occ = resident blocks per SM of visc_dt, the Lagrangian, the
 // fused x and y sweeps.
@@ -1018,14 +1033,7 @@ void phase_ranges(const Chunk& c, int kind, int yd, int* lo, int* hi, int* n) {
 }
 
 // Enqueue kernel phases [0, nphase) of one step (7 = full step).
-// Serpentine segment order: each step kernel reads what the previous one
-// wrote, so alternate kernels run their row segments top-down (seg_y) and
-// start on the rows still in L2: visc_dt and sweep 1 reversed, the
-// Lagrangian phase and sweep 2 forward.  Measured at 3840^2: no gain
-// (visc_dt +0.004 ms, Lagrangian -0.002 ms), so off by default.
-#ifndef CLOVER_SERP
-#define CLOVER_SERP 0
-#endif
+// (Serpentine segment order, CLOVER_SERP: see batch_ok.)
 static Chunk with_rev(Chunk c, int rev) {
   c.rev = rev;
   return c;
@@ -1059,8 +1067,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
   int cur_prof_id = P_VISC_DT;
   const bool deep = deep_ok(ctx);
   // several local chunks: one launch per kernel for all of them (KBatch)
-  const bool batch = ctx->batch && CLOVER_SERP == 0 && ctx->chunks.size() > 1 &&
-                     ctx->chunks.size() <= (size_t)MAX_BATCH;
+  const bool batch = batch_ok(ctx);
   if (ctx->prof) prof_mark(ctx, -1);
   // one chunk on one rank: the visc fixup's last block finalises dt (no
   // k_dt_finalize launch); else the slot is combined first (NCCL MIN)
@@ -2131,36 +2138,46 @@ int clover_debug_fix_count(clover_ctx* ctx, int64_t* out) {
 
 int clover_kernels_per_step(clover_ctx* ctx, int32_t* out) {
   if (!ctx || !out) return fail(CLOVER_ERR_ARG, "NULL argument");
-  // per chunk: visc_dt + fixup, Lagrangian + fixup, the x sweep (fused:
-  // kernel + fixup; else cell, mom + 2 fixups), the y sweep (fused: wall
-  // bands, kernel + fixup; else 4; the bands ride on the previous fixup
-  // launch at one chunk on one rank, enqueue_step); plus k_dt_finalize once
-  // unless the visc fixup finalises dt (one chunk on one rank)
-  // (chunks without a y wall launch no band kernel; the halo strip copies
-  // between phases, k_copy_strips, are not counted)
+  // visc_dt + fixup, Lagrangian + fixup, the x sweep (fused: kernel + fixup;
+  // else cell, mom + 2 fixups), the y sweep (fused: wall bands, kernel +
+  // fixup; else 4; the bands ride on the previous fixup launch at one chunk
+  // on one rank, enqueue_step) -- per chunk, or once for all local chunks
+  // when batched (batch_ok; the unfused sweeps and the y-wall bands stay per
+  // chunk) -- plus k_dt_finalize once unless the visc fixup finalises dt (one
+  // chunk on one rank).  (Chunks without a y wall launch no band kernel; the
+  // halo strip copies, k_copy_strips, are not counted.)
   const bool one = ctx->chunks.size() == 1 && ctx->nranks == 1;
-  const int x = fuse_x_ok(ctx) ? 2 : 4;
   const bool folded = CLOVER_YWALLS_FOLD && one && fuse_x_ok(ctx) && ctx->walls_fold_fits;
+  const bool bat = batch_ok(ctx), ov = overlap_ok(ctx);
+  const int nch = (int)ctx->chunks.size();
+  // boundary ranges + interior as separate launches, a fixup after each part
+  // (run_phase with the boundary-first overlap)
+  auto extra = [&](const ChunkState& cs, int kind, int yd) {
+    int lo, hi, ns;
+    phase_ranges(cs.c, kind, yd, &lo, &hi, &ns);
+    const int b = (lo > 0) + (hi < ns);
+    return b + (b > 0) + 2 * (lo < hi) - 2;
+  };
+  // a fused phase: 2 launches, batched or per chunk (+ the overlap split)
+  auto fused = [&](int kind, int yd) {
+    if (bat && !ov) return 2;
+    int m = 0;
+    for (const auto& cs : ctx->chunks) m += 2 + (ov ? extra(cs, kind, yd) : 0);
+    return m;
+  };
   int n = one ? 0 : 1;
-  for (const auto& cs : ctx->chunks) {
-    const int y = fuse_y_ok(ctx) ? (2 + ((!folded && (cs.c.wb || cs.c.wt)) ? 1 : 0)) : 4;
-    n += 4 + x + y;
-    if (overlap_ok(ctx)) {
-      // boundary ranges + interior as separate launches, a fixup after each
-      // part (run_phase); for the current sweep order
-      auto extra = [&](int kind, int yd) {
-        int lo, hi, ns;
-        phase_ranges(cs.c, kind, yd, &lo, &hi, &ns);
-        const int b = (lo > 0) + (hi < ns);
-        return b + (b > 0) + 2 * (lo < hi) - 2;
-      };
-      const bool ax = ctx->advect_x;
-      n += extra(SEG_LAGR, fuse_y_ok(ctx) ? FUSE_ROWS : HALO);
-      for (int sweep = 1; sweep <= 2; ++sweep) {
-        const bool xdir = (sweep == 1) ? ax : !ax;
-        if (xdir && fuse_x_ok(ctx)) n += extra(SEG_X, (sweep == 1 && fuse_y_ok(ctx)) ? FUSE_ROWS : HALO);
-        if (!xdir && fuse_y_ok(ctx)) n += extra(SEG_Y, HALO);
-      }
+  n += bat ? 2 : 2 * nch;  // visc_dt
+  n += fused(SEG_LAGR, fuse_y_ok(ctx) ? FUSE_ROWS : HALO);
+  const bool ax = ctx->advect_x;
+  for (int sweep = 1; sweep <= 2; ++sweep) {
+    const bool xdir = (sweep == 1) ? ax : !ax;
+    if (xdir) {
+      n += fuse_x_ok(ctx) ? fused(SEG_X, (sweep == 1 && fuse_y_ok(ctx)) ? FUSE_ROWS : HALO) : 4 * nch;
+    } else if (fuse_y_ok(ctx)) {
+      for (const auto& cs : ctx->chunks) n += (!folded && (cs.c.wb || cs.c.wt)) ? 1 : 0;
+      n += fused(SEG_Y, HALO);
+    } else {
+      n += 4 * nch;
     }
   }
   *out = (int32_t)n;

@@ -755,15 +755,21 @@ def test_maximum_size_corner_window_bitwise(torch_cuda):
     g.close()
 
 
-@pytest.mark.parametrize("pxy,expected", [((1, 1), 8), ((3, 1), 28), ((1, 3), 27)])
-def test_kernels_per_step(torch_cuda, pxy, expected):
+@pytest.mark.parametrize("pxy,batch,expected", [((1, 1), True, 8), ((3, 1), False, 28),
+                                                ((1, 3), False, 27), ((3, 1), True, 12),
+                                                ((1, 3), True, 11)])
+def test_kernels_per_step(torch_cuda, monkeypatch, pxy, batch, expected):
     """Launches per step (bench.py's gpu_launches): one chunk runs visc_dt,
     Lagrangian and both fused sweeps with a fixup each, the y-wall bands
     riding on the fixup before the y sweep (8); several chunks launch the
     bands separately (+1 per chunk with a y wall) and finalise dt in
-    k_dt_finalize (+1); chunk boundaries keep both fused sweeps: 3x1 =
-    3 * (4 + 2 + 3) + 1, 1x3 = (4 + 2 + 3) + (4 + 2 + 2) + (4 + 2 + 3) + 1."""
+    k_dt_finalize (+1); chunk boundaries keep both fused sweeps.  One launch
+    per chunk (CLOVER_BATCH=0): 3x1 = 3 * (4 + 2 + 3) + 1, 1x3 = (4 + 2 + 3)
+    + (4 + 2 + 2) + (4 + 2 + 3) + 1; batched: 3x1 = 8 + 3 bands + 1, 1x3 =
+    8 + 2 bands + 1."""
     px, py = pxy
+    if not batch:
+        monkeypatch.setenv("CLOVER_BATCH", "0")
     g = make_gpu(fuzz_deck(11), px=px, py=py)
     assert g.kernels_per_step() == expected
     # the engine's own launch counter (clover_launch_count, the bench's
