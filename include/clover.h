@@ -176,7 +176,11 @@ int clover_step(clover_ctx* ctx, int32_t nsteps);
 /* End-to-end entry with HOST buffers: copy the state density0, energy0
  * (cells), xvel0, yvel0 (nodes) from host memory (pinned for speed) into the
  * mesh, advance nsteps, copy the four state fields back to host_out (may
- * alias host_in).  Synchronous.  Single-chunk contexts only. */
+ * alias host_in).  Synchronous.  The host arrays are the global interiors
+ * (row-major, j fastest); with several chunks each process moves the owned
+ * blocks of its own chunks (a multi-rank call is collective, and a rank's
+ * arrays outside its chunks are neither read nor written).  A NULL input
+ * keeps that field's current values; a NULL output is not copied back. */
 int clover_step_host(clover_ctx* ctx, int32_t nsteps,
                      const double* density0_in, const double* energy0_in,
                      const double* xvel0_in, const double* yvel0_in,

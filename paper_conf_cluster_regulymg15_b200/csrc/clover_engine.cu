@@ -2550,7 +2550,6 @@ int clover_step_host(clover_ctx* ctx, int32_t nsteps, const double* d_in, const 
                      const double* u_in, const double* v_in, double* d_out, double* e_out,
                      double* u_out, double* v_out) {
   if (!ctx) return fail(CLOVER_ERR_ARG, "ctx is NULL");
-  if (ctx->chunks.size() != 1 || ctx->nranks != 1) return fail(CLOVER_ERR_STATE, "clover_step_host needs a single-chunk context");
   const int64_t nc = (int64_t)ctx->g.x_cells * ctx->g.y_cells;
   const int64_t nn = (int64_t)(ctx->g.x_cells + 1) * (ctx->g.y_cells + 1);
   int rc = join_in(ctx);

@@ -616,6 +616,22 @@ def test_step_host_matches_device_path(torch_cuda):
         assert np.array_equal(outs[k], o.read(k)), k
 
 
+@pytest.mark.parametrize("pxy", [(1, 3), (2, 2)])
+def test_step_host_on_several_chunks(torch_cuda, pxy):
+    """clover_step_host on a multi-chunk context: every chunk takes its block
+    of the global host arrays in and out; same bits as one chunk."""
+    nx, ny = 64, 96
+    deck = bm_deck(nx, ny)
+    f = random_state_fields(5, nx, ny, smooth=True)
+    one, many = make_gpu(deck), make_gpu(deck, px=pxy[0], py=pxy[1])
+    o1 = {k: np.empty_like(v) for k, v in f.items()}
+    om = {k: np.full_like(v, np.nan) for k, v in f.items()}
+    one.step_host(4, f, o1)
+    many.step_host(4, f, om)
+    for k in STATE:
+        assert np.array_equal(om[k], o1[k]), k
+
+
 def test_small_dt_error_is_latched(torch_cuda):
     from paper_conf_cluster_regulymg15_b200 import CloverError
     deck = bm_deck(32)
