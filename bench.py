@@ -431,6 +431,39 @@ def main():
                       "d2h_bytes_per_step": 8 * (2 * nc + 2 * nn) / args.steps,
                       "api": f"clover_step_host (h2d state, {args.steps} steps, d2h state)"}
 
+    if not args.no_e2e and world > 1:
+        # every rank moves its own strip of the global host arrays through
+        # clover_step_host (collective): the arrays are allocated lazily
+        # (np.empty), only this rank's rows are touched and pinned
+        # (cudaHostRegister); wall clock per call, max over ranks
+        gj0, gk0, bw, bh = sim.local_block()
+        host, regs = {}, []
+        for name, shp in (("density0", (ny, nx)), ("energy0", (ny, nx)),
+                          ("xvel0", (ny + 1, nx + 1)), ("yvel0", (ny + 1, nx + 1))):
+            a = np.empty(shp, dtype=np.float64)
+            host[name] = a
+            r1 = min(shp[0], gk0 + bh + 1)
+            ptr = a.ctypes.data + gk0 * a.strides[0]
+            nbytes = (r1 - gk0) * a.strides[0]
+            if torch.cuda.cudart().cudaHostRegister(ptr, nbytes, 0) == 0:
+                regs.append(ptr)
+        sim.step_host(0, {}, host)  # this rank's rows <- the current state
+        ke = max(3, min(args.steps, 10))
+        sim.step_host(1, host, host)  # warm
+        dist.barrier()
+        t0 = time.perf_counter()
+        for _ in range(ke):
+            sim.step_host(1, host, host)
+        te = cdist.max_over_ranks(time.perf_counter() - t0, None if host_tp else dev)
+        for ptr in regs:
+            torch.cuda.cudart().cudaHostUnregister(ptr)
+        nc, nn = cells, (nx + 1) * (ny + 1)
+        e2e = {"value": cells * ke / te, "unit": UNIT, "h2d_bytes_per_step": 8 * (2 * nc + 2 * nn),
+               "d2h_bytes_per_step": 8 * (2 * nc + 2 * nn), "steps": ke,
+               "api": "clover_step_host (each rank: h2d its strip of the state, 1 step, d2h), "
+                      "bytes summed over ranks",
+               "pinned": len(regs) == 4}
+
     # side measurement: the same mesh with every cell moving (seeded smooth
     # random state + noise, workloads.random_state_fields), so the headline
     # is not an artifact of the bm deck's quiescent regions
@@ -519,7 +552,7 @@ def main():
                            "halo_exchange": ("deep: 1 state exchange (7 rows) + dt MIN per step"
                                              if deep_halo else "per phase") if world > 1 else None,
                            "l2": "inputs larger than L2 (18 fp64 fields of the mesh, >2 GB vs 126 MB L2)",
-                           "graphs": True},
+                           "graphs": not host_tp},
                 "gpu_launches": launches,
                 "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "clocks": clk,
                 "kernels": kernels,

@@ -242,6 +242,12 @@ int clover_kernels_per_step(clover_ctx* ctx, int32_t* out);
  * across its timed region. */
 int clover_launch_count(clover_ctx* ctx, int64_t* out);
 
+/* Bounding box of this process's chunks in global cell indices: out4 =
+ * {j0, k0, width, height} (0-based origin; cells [j0, j0+width) x
+ * [k0, k0+height)).  E.g. to pin only the rows of the global host arrays
+ * that clover_step_host moves on this rank. */
+int clover_local_block(clover_ctx* ctx, int32_t* out4);
+
 /* Profiling: run nsteps full steps with direct launches and a CUDA event
  * after every kernel on the context's work stream; ms_out[i] / launches_out[i]
  * receive the summed duration and launch count of kernel type i

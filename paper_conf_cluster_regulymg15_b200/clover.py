@@ -38,7 +38,7 @@ BUF = {"d0": 0, "e0": 1, "u0": 2, "v0": 3, "q": 4, "d1": 5, "e1": 6, "u1": 7, "v
 EXPORTS = ["clover_workspace_bytes", "clover_nccl_unique_id", "clover_init", "clover_step",
            "clover_step_host", "clover_field_summary", "clover_get_clock", "clover_dt_history",
            "clover_read_field", "clover_read_field_window", "clover_write_field", "clover_sync", "clover_set_graphs",
-           "clover_kernels_per_step", "clover_launch_count", "clover_debug_partial_step", "clover_debug_read_buffer",
+           "clover_kernels_per_step", "clover_launch_count", "clover_local_block", "clover_debug_partial_step", "clover_debug_read_buffer",
            "clover_profile_steps", "clover_profile_name", "clover_debug_div_check",
            "clover_debug_fix_count", "clover_debug_set_fusion", "clover_debug_set_overlap",
            "clover_set_deep_halo", "clover_deep_halo_active",
@@ -121,6 +121,8 @@ def load(build_if_missing: bool = True):
     L.clover_kernels_per_step.argtypes = [c_void_p, P(c_int32)]
     if hasattr(L, "clover_launch_count"):
         L.clover_launch_count.argtypes = [c_void_p, P(ctypes.c_int64)]
+    if hasattr(L, "clover_local_block"):
+        L.clover_local_block.argtypes = [c_void_p, P(c_int32)]
     L.clover_debug_partial_step.argtypes = [c_void_p, c_int32]
     L.clover_debug_read_buffer.argtypes = [c_void_p, c_int32, c_int32, dptr, c_int64]
     L.clover_profile_steps.argtypes = [c_void_p, c_int32, dptr, ctypes.POINTER(c_int64), c_int32]
@@ -290,6 +292,12 @@ class Clover:
         n = c_int32()
         _check(load().clover_kernels_per_step(self._ctx, ctypes.byref(n)), "clover_kernels_per_step")
         return n.value
+
+    def local_block(self):
+        """(j0, k0, width, height): this process's chunks in global cells."""
+        a = (c_int32 * 4)()
+        _check(load().clover_local_block(self._ctx, a), "clover_local_block")
+        return tuple(a)
 
     def launch_count(self) -> int:
         """Step kernels launched on this context so far (clover_launch_count)."""

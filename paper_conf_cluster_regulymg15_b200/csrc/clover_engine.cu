@@ -2231,6 +2231,17 @@ int clover_step(clover_ctx* ctx, int32_t nsteps) {
   return join_out(ctx);
 }
 
+int clover_local_block(clover_ctx* ctx, int32_t* out4) {
+  if (!ctx || !out4) return fail(CLOVER_ERR_ARG, "NULL argument");
+  int j0 = 1 << 30, k0 = 1 << 30, j1 = 0, k1 = 0;
+  for (const auto& cs : ctx->chunks) {
+    j0 = std::min(j0, cs.c.gj0); k0 = std::min(k0, cs.c.gk0);
+    j1 = std::max(j1, cs.c.gj0 + cs.c.nx); k1 = std::max(k1, cs.c.gk0 + cs.c.ny);
+  }
+  out4[0] = j0; out4[1] = k0; out4[2] = j1 - j0; out4[3] = k1 - k0;
+  return CLOVER_OK;
+}
+
 int clover_launch_count(clover_ctx* ctx, int64_t* out) {
   if (!ctx || !out) return fail(CLOVER_ERR_ARG, "NULL argument");
   *out = ctx->launches;
