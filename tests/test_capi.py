@@ -8,8 +8,6 @@ import os
 import re
 import subprocess
 
-import pytest
-
 from paper_conf_cluster_regulymg15_b200 import clover as cb
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
