@@ -68,6 +68,29 @@ def env_int(name, default):
         return default
 
 
+# BASELINE.json north_star: "achieved HBM GB/s against about 8 TB/s per B200"
+NOMINAL_HBM_GBS = 8000.0
+
+
+def ncu_window(cx, cy):
+    """S:8(d) hbm_gbs from the committed ncu capture (profiles/ncu_traffic.json,
+    written by scripts/summarize_profiles.py): the sum of DRAM bytes over the
+    sum of kernel time of the captured window's streaming kernels, when the
+    capture's mesh is this rank's chunk."""
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    try:
+        with open(p) as fh:
+            tr = json.load(fh)
+        w = tr.get("window")
+        if not w or tuple(tr.get("mesh", [])) != (cx, cy) or not w.get("hbm_gbs"):
+            return None
+        return {"hbm_gbs": w["hbm_gbs"], "launches": w["launches"], "source": tr.get("source"),
+                "how": "sum of ncu dram__bytes (read+write) / sum of gpu__time_duration, "
+                       "streaming kernels of the captured steps (cold-cache, serialised launches)"}
+    except (OSError, ValueError, KeyError):
+        return None
+
+
 def measured_peaks():
     p = os.path.join(ROOT, "MEASURED_PEAKS.json")
     if os.path.exists(p):
@@ -398,7 +421,15 @@ def main():
     roofline = {"bound": "hbm", "kernel": top, "achieved": ach, "peak": peak, "unit": "GB/s",
                 "frac": ach / peak if ach else None, "traffic": traffic, "peak_source": peak_src,
                 "step_achieved": step_gbs, "step_frac": step_gbs / peak,
-                "algo_bytes_per_cell_step": step_bpc}
+                "algo_bytes_per_cell_step": step_bpc,
+                # S:8(d): fractions also against the north_star's ~8 TB/s nominal
+                "nominal_peak": NOMINAL_HBM_GBS, "frac_nominal": ach / NOMINAL_HBM_GBS if ach else None,
+                "step_frac_nominal": step_gbs / NOMINAL_HBM_GBS}
+    win = ncu_window(nx // px, ny // py)
+    if win:
+        win["frac"] = win["hbm_gbs"] / peak
+        win["frac_nominal"] = win["hbm_gbs"] / NOMINAL_HBM_GBS
+        roofline["ncu_window"] = win
     nsm = torch.cuda.get_device_properties(dev).multi_processor_count
     roofline["alu"] = issue_roofline(kernels, top, clk.get("sm_mhz"), nsm)
 

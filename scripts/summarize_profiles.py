@@ -85,7 +85,7 @@ if os.path.exists(rep):
     kern = {}
     md = [f"# ncu --set full summary ({tag}): bm 3840x3840, one launch per kernel type\n",
           "Captured with `ncu --set full --clock-control none --import-source on -k regex:ks_` on "
-          "`scripts/prof_run.py 3840 3840 53` with `-s 200 -c 8`: steps 51-52, x-first then y-first (scripts/profile_round.sh). DRAM bytes in MB "
+          "`scripts/prof_run.py 3840 3840 54` with `-s 200 -c 12`: steps 51-53, x-first, y-first, x-first (scripts/profile_round.sh). DRAM bytes in MB "
           "(units as reported: " + units[hdr.index('dram__bytes_read.sum')] + ").\n",
           "| kernel | time us | DRAM read | DRAM write | DRAM GB/s | issue % | fp64 pipe % | warps active % | regs | thread inst/cell |",
           "|---|---|---|---|---|---|---|---|---|---|"]
@@ -108,9 +108,15 @@ if os.path.exists(rep):
                                        "fp64": g(r, 'sm__pipe_fp64_cycles_active.avg.pct_of_peak_sustained_active')})
     with open(os.path.join(P, f"{tag}_kernels.md"), "w") as fh:
         fh.write("\n".join(md) + "\n")
+    allx = [x for v in kern.values() for x in v]
+    tb, tt = sum(x["dram_bytes"] for x in allx), sum(x["time_ns"] for x in allx)
     out = {"mesh": [3840, 3840], "source": f"profiles/{tag}_kernels.md (ncu --set full)",
            "kernels": {k: {"dram_bytes_per_launch": sum(x["dram_bytes"] for x in v) / len(v),
-                           "launches": len(v)} for k, v in kern.items()}}
+                           "launches": len(v)} for k, v in kern.items()},
+           # S:8(d) hbm_gbs: sum of DRAM bytes over sum of kernel time, the
+           # streaming kernels of the captured window (cold-cache, serialised)
+           "window": {"launches": len(allx), "dram_bytes": tb, "time_ns": tt,
+                      "hbm_gbs": tb / (tt * 1e-9) / 1e9 if tt else None}}
     with open(os.path.join(P, "ncu_traffic.json"), "w") as fh:
         json.dump(out, fh, indent=1)
     avg = lambda v, k: sum(x[k] for x in v) / len(v)
