@@ -262,12 +262,28 @@ def oracle_rate(deck, steps, warmup=0):
     return cells * steps / t, t
 
 
-def band_deck(nx=3840, rows=240):
-    """Bounded sample of the 3840^2 bm workload: the bottom `rows` rows at
-    the same cell size (domain [0,10] x [0, 10*rows/nx])."""
+def arm_mesh(args, world):
+    """Global mesh and chunk grid of this run: configs[2] at N = 1,
+    configs[4]'s weak series (reading A4) or with --strong configs[3] at N > 1,
+    or --mesh."""
+    from paper_conf_cluster_regulymg15_b200 import dist as cdist
+    if args.strong:
+        nx, ny = 7680, 7680
+        px, py = cdist.chunk_grid(world, nx, ny)
+    else:
+        nx, ny, px, py = cdist.weak_mesh(world)
+    if args.mesh:
+        nx, ny = args.mesh
+        px, py = cdist.chunk_grid(world, nx, ny)
+    return nx, ny, px, py
+
+
+def band_deck(nx=3840, ny=3840, rows=240):
+    """Bounded sample of the nx x ny bm workload on [0,10]^2: its bottom
+    `rows` rows at the same cell size (domain [0,10] x [0, 10*rows/ny])."""
     from workloads import bm_deck
     d = bm_deck(nx, rows)
-    d["ymax"] = 10.0 * rows / nx
+    d["ymax"] = 10.0 * rows / ny
     return d
 
 
@@ -275,8 +291,11 @@ def run_reference(args):
     rank = env_int("RANK", 0)
     if rank != 0:
         return
-    from workloads import bm_deck  # noqa: F401
-    deck = band_deck()
+    # the arm's own workload (the same mesh and cell size as `bench.py
+    # --gpus N` with these flags), a band of about 0.9 M cells per step
+    nx, ny, _, _ = arm_mesh(args, max(args.gpus, env_int("WORLD_SIZE", 1)))
+    rows = max(16, min(240, 921600 // nx))
+    deck = band_deck(nx, ny, rows)
     from oracle import Oracle
     o = Oracle(deck)
     o.step(args.warmup)
@@ -286,15 +305,17 @@ def run_reference(args):
     cells = deck["x_cells"] * deck["y_cells"]
     v = cells * args.steps / t
     hc = host_cpu()
-    sample = (f"oracle (single-threaded C++ -O2) on a bounded sample of configs[2]: the bottom "
-              f"{deck['y_cells']} rows of the 3840^2 bm mesh at the same cell size "
+    sample = (f"oracle (single-threaded C++ -O2) on a bounded sample of the arm's workload: the "
+              f"bottom {deck['y_cells']} rows of the {nx}x{ny} bm mesh at the same cell size "
               f"({cells} cells) per step, {args.steps} timed steps after {args.warmup} warm-up")
     line = {"impl": "reference", "metric": METRIC, "value": v, "unit": UNIT,
             "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": 1000.0 * t / max(args.steps, 1), "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": {"workload": "configs[2] sample: CloverLeaf 2D bm deck, 3840 x 240 band",
-                       "mesh": [deck["x_cells"], deck["y_cells"]]},
+            "scaling": "strong" if args.strong else "weak", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic",
+            "config": {"workload": f"sample of the {nx}x{ny} CloverLeaf 2D bm deck: "
+                                   f"{nx} x {deck['y_cells']} band",
+                       "mesh": [deck["x_cells"], deck["y_cells"]], "full_mesh": [nx, ny]},
             "cpu_baseline": {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample,
                              **hc},
             "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
@@ -346,14 +367,7 @@ def main():
             dist.init_process_group("gloo")
         else:
             dist.init_process_group("nccl", device_id=dev)
-    if args.strong:
-        nx, ny = 7680, 7680
-        px, py = cdist.chunk_grid(world, nx, ny)
-    else:
-        nx, ny, px, py = cdist.weak_mesh(world)
-    if args.mesh:
-        nx, ny = args.mesh
-        px, py = cdist.chunk_grid(world, nx, ny)
+    nx, ny, px, py = arm_mesh(args, world)
     # the bm deck on [0,10]^2 for every mesh (reading A4: the weak-scaling
     # series grows the mesh in both axes on the fixed domain)
     deck = bm_deck(nx, ny, end_step=args.steps)
