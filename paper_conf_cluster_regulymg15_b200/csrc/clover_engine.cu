@@ -981,6 +981,23 @@ bool batch_ok(const clover_ctx* ctx) {
 // Row-segment parameters of a chunk (or view) of c.ny rows (see seg_rows,
 // tail_nb): occ = resident blocks per SM of visc_dt, the Lagrangian, the
 // fused x and y sweeps.
+// Segment chains (seg_chain): one chain per segment row of blocks resident
+// at a time (ceil(slots / column blocks)), so consecutive segments of a chain
+// run in consecutive waves and share their overlap rows through L2.
+// CLOVER_CHAIN=0: launch order = row order.  CLOVER_CHAIN_ADJ: chains added
+// to that count (A/B).
+#ifndef CLOVER_CHAIN
+#define CLOVER_CHAIN 1
+#endif
+#ifndef CLOVER_CHAIN_ADJ
+#define CLOVER_CHAIN_ADJ 0
+#endif
+int chain_count(int64_t colblocks, int nb, int64_t slots) {
+  if (!CLOVER_CHAIN || colblocks <= 0 || nb >= 0x3fffffff) return 0;
+  const int64_t ch = (slots + colblocks - 1) / colblocks + CLOVER_CHAIN_ADJ;
+  return (ch >= 1 && ch < nb) ? (int)ch : 0;
+}
+
 void set_segs(Chunk& c, int nsm, const int occ[4]) {
   c.vks = seg_rows(VKS, grid_cols(c.nx, c.ny, VKS).x, c.ny);
   c.lks = seg_rows(LKS, grid_strip(c.nx, LW, c.ny, LKS).x, c.ny);
@@ -990,6 +1007,10 @@ void set_segs(Chunk& c, int nsm, const int occ[4]) {
   c.lnb = tail_nb(c.lks, grid_strip(c.nx, LW, c.ny, c.lks).x, c.ny, (int64_t)nsm * occ[1]);
   c.xnb = tail_nb(c.xks, grid_strip(c.nx + 1, XW, c.ny + 1, c.xks).x, c.ny + 1, (int64_t)nsm * occ[2]);
   c.ynb = tail_nb(c.yks, grid_strip(c.nx + 1, YW, c.ny + 1, c.yks).x, c.ny + 1, (int64_t)nsm * occ[3]);
+  c.vch = chain_count(grid_cols(c.nx, c.ny, c.vks).x, c.vnb, (int64_t)nsm * occ[0]);
+  c.lch = chain_count(grid_strip(c.nx, LW, c.ny, c.lks).x, c.lnb, (int64_t)nsm * occ[1]);
+  c.xch = chain_count(grid_strip(c.nx + 1, XW, c.ny + 1, c.xks).x, c.xnb, (int64_t)nsm * occ[2]);
+  c.ych = chain_count(grid_strip(c.nx + 1, YW, c.ny + 1, c.yks).x, c.ynb, (int64_t)nsm * occ[3]);
 }
 
 // The chunk seen from `e` rows beyond each of its non-wall y sides: rows
@@ -1122,6 +1143,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
       int n;
       phase_ranges(cs.c, kind, yd, &ilo[t], &ihi[t], &n);
       Chunk c = cs.c;
+      c.vch = c.lch = c.xch = c.ych = 0;  // sub-range launches: row order
       int rc = 0;
       bool any = false;
       if (ilo[t] > 0) { c.seg0 = 0; rc = launch(cs, c, ilo[t], cm, cs.fix_b); any = true; }
@@ -1138,6 +1160,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
       if (ilo[t] >= ihi[t]) continue;
       auto& cs = ctx->chunks[t];
       Chunk c = cs.c;
+      c.vch = c.lch = c.xch = c.ych = 0;
       c.seg0 = ilo[t];
       rc = launch(cs, c, ihi[t] - ilo[t], st, cs.fix);
       if (!rc) rc = fixup(cs, c, st, cs.fix);

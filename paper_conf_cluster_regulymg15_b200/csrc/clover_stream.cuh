@@ -413,12 +413,13 @@ ks_visc_dt(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__
   const int gw = blockIdx.x * (SB / 32) + warp;
   double dtw = G_BIG;
   int k0, len;
-  seg_rows_of(seg_y(c), c.vks, c.vnb, k0, len);
+  const int sg = seg_y(c, c.vch, c.vnb);
+  seg_rows_of(sg, c.vks, c.vnb, k0, len);
   int k1 = min(k0 + len, c.ny + 1);
   visc_ring_rows(c, k0, k1);
   if (gw * 32 < c.nx) {
     if (visc_seg<DivFast>(c, &tm, q, prm, gw, k0, k1, lane, ring[warp], bars[warp], dtw)) {
-      fix_push(fix, lane, gw, (unsigned)seg_y(c));
+      fix_push(fix, lane, gw, (unsigned)sg);
       dtw = G_BIG;  // this warp's dt comes from the fixup
     }
   }
@@ -737,10 +738,11 @@ ks_lagrangian(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restric
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const int gw = blockIdx.x * (SB / 32) + w;
   int k0, len;
-  seg_rows_of(seg_y(c), c.lks, c.lnb, k0, len);
+  const int sg = seg_y(c, c.lch, c.lnb);
+  seg_rows_of(sg, c.lks, c.lnb, k0, len);
   const int k1 = min(k0 + len, c.ny + 1);
   if (lagr_seg<DivFast>(c, &tm, d1, e1, u1, v1, fx, fy, s, gw, k0, k1, lane, ring[w], bars[w]))
-    fix_push(fix, lane, gw, (unsigned)seg_y(c));
+    fix_push(fix, lane, gw, (unsigned)sg);
 }
 
 __global__ void __launch_bounds__(SB)
@@ -1346,11 +1348,12 @@ ks_advec_x(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const int gw = blockIdx.x * (SB / 32) + w;
   int k0, len;
-  seg_rows_of(seg_y(c), c.xks, c.xnb, k0, len);
+  const int sg = seg_y(c, c.xch, c.xnb);
+  seg_rows_of(sg, c.xks, c.xnb, k0, len);
   const int k1 = min(k0 + len, c.ny + 2);
   if (advec_x_seg<SWEEP, DivFast>(c, &tm, rho_out, en_out, uout, vout, gw, k0, k1, lane, ring[w],
                                    bars[w]))
-    fix_push(fix, lane, gw, (unsigned)seg_y(c));
+    fix_push(fix, lane, gw, (unsigned)sg);
 }
 
 template <int SWEEP>
@@ -1805,11 +1808,12 @@ ks_advec_y(Chunk c, const __grid_constant__ CUtensorMap ta, const __grid_constan
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const int gw = blockIdx.x * (SB / 32) + w;
   int k0, len;
-  seg_rows_of(seg_y(c), c.yks, c.ynb, k0, len);
+  const int sg = seg_y(c, c.ych, c.ynb);
+  seg_rows_of(sg, c.yks, c.ynb, k0, len);
   const int k1 = min(k0 + len, c.ny + 2);
   if (advec_y_seg<SWEEP, DivFast>(c, &ta, &tb, rho_out, en_out, mfy, uout, vout, gw, k0, k1, lane,
                                   ring[w], bars[w]))
-    fix_push(fix, lane, gw, (unsigned)seg_y(c));
+    fix_push(fix, lane, gw, (unsigned)sg);
 }
 
 template <int SWEEP>
@@ -1857,12 +1861,13 @@ ks_visc_dt_b(const __grid_constant__ KBatch<VArgs> b, StepScalars* __restrict__ 
   const int gw = blockIdx.x * (SB / 32) + warp;
   double dtw = G_BIG;
   int k0, len;
-  seg_rows_of((int)blockIdx.y, c.vks, c.vnb, k0, len);
+  const int sg = seg_chain((int)blockIdx.y, c.vch, c.vnb);
+  seg_rows_of(sg, c.vks, c.vnb, k0, len);
   int k1 = min(k0 + len, c.ny + 1);
   visc_ring_rows(c, k0, k1);
   if (gw * 32 < c.nx) {
     if (visc_seg<DivFast>(c, &a.tm, a.q, prm, gw, k0, k1, lane, ring[warp], bars[warp], dtw)) {
-      fix_push(a.fix, lane, gw, blockIdx.y);
+      fix_push(a.fix, lane, gw, (unsigned)sg);
       dtw = G_BIG;
     }
   }
@@ -1903,11 +1908,12 @@ ks_lagrangian_b(const __grid_constant__ KBatch<LArgs> b, const StepScalars* __re
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const int gw = blockIdx.x * (SB / 32) + w;
   int k0, len;
-  seg_rows_of((int)blockIdx.y, c.lks, c.lnb, k0, len);
+  const int sg = seg_chain((int)blockIdx.y, c.lch, c.lnb);
+  seg_rows_of(sg, c.lks, c.lnb, k0, len);
   const int k1 = min(k0 + len, c.ny + 1);
   if (lagr_seg<DivFast>(c, &a.tm, a.d1, a.e1, a.u1, a.v1, a.fx, a.fy, s, gw, k0, k1, lane, ring[w],
                         bars[w]))
-    fix_push(a.fix, lane, gw, blockIdx.y);
+    fix_push(a.fix, lane, gw, (unsigned)sg);
 }
 __global__ void __launch_bounds__(SB)
 kf_lagrangian_b(const __grid_constant__ KBatch<LArgs> b, StepScalars* __restrict__ s) {
@@ -1937,11 +1943,12 @@ __global__ void LB_ADVX ks_advec_x_b(const __grid_constant__ KBatch<XArgs> b) {
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const int gw = blockIdx.x * (SB / 32) + w;
   int k0, len;
-  seg_rows_of((int)blockIdx.y, c.xks, c.xnb, k0, len);
+  const int sg = seg_chain((int)blockIdx.y, c.xch, c.xnb);
+  seg_rows_of(sg, c.xks, c.xnb, k0, len);
   const int k1 = min(k0 + len, c.ny + 2);
   if (advec_x_seg<SWEEP, DivFast>(c, &a.tm, a.rho, a.en, a.u, a.v, gw, k0, k1, lane, ring[w],
                                    bars[w]))
-    fix_push(a.fix, lane, gw, blockIdx.y);
+    fix_push(a.fix, lane, gw, (unsigned)sg);
 }
 template <int SWEEP>
 __global__ void __launch_bounds__(SB) kf_advec_x_b(const __grid_constant__ KBatch<XArgs> b) {
@@ -1970,11 +1977,12 @@ ks_advec_y_b(const __grid_constant__ KBatch<YArgs> b) {
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const int gw = blockIdx.x * (SB / 32) + w;
   int k0, len;
-  seg_rows_of((int)blockIdx.y, c.yks, c.ynb, k0, len);
+  const int sg = seg_chain((int)blockIdx.y, c.ych, c.ynb);
+  seg_rows_of(sg, c.yks, c.ynb, k0, len);
   const int k1 = min(k0 + len, c.ny + 2);
   if (advec_y_seg<SWEEP, DivFast>(c, &a.ta, &a.tb, a.rho, a.en, a.mfy, a.u, a.v, gw, k0, k1, lane,
                                   ring[w], bars[w]))
-    fix_push(a.fix, lane, gw, blockIdx.y);
+    fix_push(a.fix, lane, gw, (unsigned)sg);
 }
 template <int SWEEP>
 __global__ void __launch_bounds__(SB) kf_advec_y_b(const __grid_constant__ KBatch<YArgs> b) {
