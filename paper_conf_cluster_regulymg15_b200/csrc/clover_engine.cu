@@ -166,7 +166,6 @@ int seg_rows(int ks, int64_t colblocks, int nrows) {
 }
 // Segment rows of a kernel grid whose first nb segments have ks rows and
 // the rest ks/2 (seg_rows_of).
-int seg_count(int ks, int nb, int rows) { return seg_count_of(ks, nb, rows); }
 // Full-height segments: all but about CLOVER_TAIL_WAVES waves of blocks
 // (slots resident blocks on the GPU, colblocks blocks per segment row),
 // which run at 1/CLOVER_TAIL_DIV height so the kernel's tail shrinks.
@@ -197,11 +196,13 @@ static_assert(DEEP_ROWS + 1 <= HALO_ROWS, "deep state halo allocated");
 // (fix lists hold every warp segment of the largest kernel grid, views
 // included: callers pass ny + 2 * DEEP_EXT_MAX)
 int64_t fix_capacity(int nx, int ny) {
-  // (adaptive segments: tail segments have at least 4 rows, see tail_nb)
-  const dim3 g[8] = {grid_cols(nx, ny, 4),          grid_strip(nx, LW, ny, 4),
+  // (adaptive segments: tail segments have at least 4 rows, see tail_nb;
+  // the band layout adds at most one shorter segment per band: bounded by
+  // counting segments of 2 rows)
+  const dim3 g[8] = {grid_cols(nx, ny, 2),          grid_strip(nx, LW, ny, 2),
                      grid_strip(nx, CW_X, ny, CKS),    grid_cols(nx, ny, CKS_Y),
                      grid_strip(nx + 1, MW_X, ny + 1, MKS), grid_cols(nx + 1, ny + 1, MKS_Y),
-                     grid_strip(nx + 1, XW, ny + 1, 4), grid_strip(nx + 1, YW, ny + 1, 4)};
+                     grid_strip(nx + 1, XW, ny + 1, 2), grid_strip(nx + 1, YW, ny + 1, 2)};
   int64_t m = 0;
   for (const dim3& d : g) m = std::max<int64_t>(m, (int64_t)d.x * d.y * (SB / 32));
   return m;
@@ -279,6 +280,7 @@ struct clover_ctx {
   bool walls_fold_fits = false;
   bool deep = true;       // deep halos where they apply (deep_ok; clover_set_deep_halo)
   bool batch = true;      // several local chunks: one launch per kernel (KBatch; CLOVER_BATCH=0 off)
+  bool chain = true;      // band layout of the row segments (seg_rows_lay; CLOVER_CHAIN=0 off)
   int nsm = 148, occ[4] = {1, 1, 1, 1};  // SMs, resident blocks/SM of the 4 segment kernels (set_segs)
   int state_rows = 0;     // rows of the state's y halo known current (ensure_state_rows)
   cudaGraphExec_t gexec[4] = {nullptr, nullptr, nullptr, nullptr};  // [parity + 2 * multi-step]
@@ -981,24 +983,30 @@ bool batch_ok(const clover_ctx* ctx) {
 // Row-segment parameters of a chunk (or view) of c.ny rows (see seg_rows,
 // tail_nb): occ = resident blocks per SM of visc_dt, the Lagrangian, the
 // fused x and y sweeps.
-// Segment chains (seg_chain): one chain per segment row of blocks resident
-// at a time (ceil(slots / column blocks)), so consecutive segments of a chain
-// run in consecutive waves and share their overlap rows through L2.
-// CLOVER_CHAIN=0: launch order = row order.  CLOVER_CHAIN_ADJ: chains added
-// to that count (A/B).
+// Band layout (seg_rows_lay): one band per segment row of blocks resident
+// at a time (ceil(slots / column blocks)), so a band's consecutive segments
+// run in consecutive waves and share their overlap rows through L2; each
+// band ends in CLOVER_TAIL_WAVES half-height segments (the kernel's last
+// waves).  Used when every band holds at least one full segment and the
+// tail; otherwise (small meshes, CLOVER_TAIL=0) the row layout (tail_nb).
+// Env CLOVER_CHAIN=0 (read at init; default CLOVER_CHAIN): row layout.
+// CLOVER_CHAIN_ADJ: bands added to that count (A/B builds).
 #ifndef CLOVER_CHAIN
 #define CLOVER_CHAIN 1
 #endif
 #ifndef CLOVER_CHAIN_ADJ
 #define CLOVER_CHAIN_ADJ 0
 #endif
-int chain_count(int64_t colblocks, int nb, int64_t slots) {
-  if (!CLOVER_CHAIN || colblocks <= 0 || nb >= 0x3fffffff) return 0;
-  const int64_t ch = (slots + colblocks - 1) / colblocks + CLOVER_CHAIN_ADJ;
-  return (ch >= 1 && ch < nb) ? (int)ch : 0;
+void band_layout(bool on, int ks, int64_t colblocks, int rows, int64_t slots, int* ch, int* cf) {
+  *ch = 0;
+  *cf = 0;
+  if (!on || !CLOVER_TAIL || ks < 4 * CLOVER_TAIL_DIV || colblocks <= 0 || slots <= 0) return;
+  const int64_t C = (slots + colblocks - 1) / colblocks + CLOVER_CHAIN_ADJ;
+  if (C < 2 || C > rows) return;
+  band_params(ks, (int)C, rows, ch, cf);
 }
 
-void set_segs(Chunk& c, int nsm, const int occ[4]) {
+void set_segs(Chunk& c, int nsm, const int occ[4], bool chain) {
   c.vks = seg_rows(VKS, grid_cols(c.nx, c.ny, VKS).x, c.ny);
   c.lks = seg_rows(LKS, grid_strip(c.nx, LW, c.ny, LKS).x, c.ny);
   c.xks = seg_rows(XKS, grid_strip(c.nx + 1, XW, c.ny + 1, XKS).x, c.ny + 1);
@@ -1007,10 +1015,12 @@ void set_segs(Chunk& c, int nsm, const int occ[4]) {
   c.lnb = tail_nb(c.lks, grid_strip(c.nx, LW, c.ny, c.lks).x, c.ny, (int64_t)nsm * occ[1]);
   c.xnb = tail_nb(c.xks, grid_strip(c.nx + 1, XW, c.ny + 1, c.xks).x, c.ny + 1, (int64_t)nsm * occ[2]);
   c.ynb = tail_nb(c.yks, grid_strip(c.nx + 1, YW, c.ny + 1, c.yks).x, c.ny + 1, (int64_t)nsm * occ[3]);
-  c.vch = chain_count(grid_cols(c.nx, c.ny, c.vks).x, c.vnb, (int64_t)nsm * occ[0]);
-  c.lch = chain_count(grid_strip(c.nx, LW, c.ny, c.lks).x, c.lnb, (int64_t)nsm * occ[1]);
-  c.xch = chain_count(grid_strip(c.nx + 1, XW, c.ny + 1, c.xks).x, c.xnb, (int64_t)nsm * occ[2]);
-  c.ych = chain_count(grid_strip(c.nx + 1, YW, c.ny + 1, c.yks).x, c.ynb, (int64_t)nsm * occ[3]);
+  band_layout(chain, c.vks, grid_cols(c.nx, c.ny, c.vks).x, c.ny, (int64_t)nsm * occ[0], &c.vch, &c.vcf);
+  band_layout(chain, c.lks, grid_strip(c.nx, LW, c.ny, c.lks).x, c.ny, (int64_t)nsm * occ[1], &c.lch, &c.lcf);
+  band_layout(chain, c.xks, grid_strip(c.nx + 1, XW, c.ny + 1, c.xks).x, c.ny + 1, (int64_t)nsm * occ[2],
+              &c.xch, &c.xcf);
+  band_layout(chain, c.yks, grid_strip(c.nx + 1, YW, c.ny + 1, c.yks).x, c.ny + 1, (int64_t)nsm * occ[3],
+              &c.ych, &c.ycf);
 }
 
 // The chunk seen from `e` rows beyond each of its non-wall y sides: rows
@@ -1024,17 +1034,17 @@ ChunkState deep_view(const clover_ctx* ctx, const ChunkState& cs, int e) {
   c.gk0 -= eb;
   c.row0 = ROW0 - eb;
   for (int b = 0; b < NBUF; ++b) v.buf[b] = cs.buf[b] - (int64_t)eb * c.pitch;
-  set_segs(c, ctx->nsm, ctx->occ);
+  set_segs(c, ctx->nsm, ctx->occ, ctx->chain);
   return v;
 }
 
 // Row-segment geometry of a streaming kernel kind on a chunk: rows per
 // segment, full-height segments, rows covered (seg_rows_of).
 enum { SEG_LAGR, SEG_X, SEG_Y };
-void seg_geom(const Chunk& c, int kind, int* ks, int* nb, int* rows) {
-  if (kind == SEG_LAGR) { *ks = c.lks; *nb = c.lnb; *rows = c.ny; }
-  else if (kind == SEG_X) { *ks = c.xks; *nb = c.xnb; *rows = c.ny + 1; }
-  else { *ks = c.yks; *nb = c.ynb; *rows = c.ny + 1; }
+void seg_geom(const Chunk& c, int kind, int* ks, int* nb, int* rows, int* ch, int* cf) {
+  if (kind == SEG_LAGR) { *ks = c.lks; *nb = c.lnb; *rows = c.ny; *ch = c.lch; *cf = c.lcf; }
+  else if (kind == SEG_X) { *ks = c.xks; *nb = c.xnb; *rows = c.ny + 1; *ch = c.xch; *cf = c.xcf; }
+  else { *ks = c.yks; *nb = c.ynb; *rows = c.ny + 1; *ch = c.ych; *cf = c.ycf; }
 }
 // the segment holding row r (1-based), inverse of seg_rows_of
 int seg_of_row(int r, int ks, int nb) {
@@ -1046,9 +1056,10 @@ int seg_of_row(int r, int ks, int nb) {
 // depth yd: [0, lo) holds the rows sent to the neighbour below (1 .. yd+1),
 // [hi, n) those sent up (ny+1-yd .. ny); [lo, hi) is the interior.
 void phase_ranges(const Chunk& c, int kind, int yd, int* lo, int* hi, int* n) {
-  int ks, nb, rows;
-  seg_geom(c, kind, &ks, &nb, &rows);
-  *n = seg_count(ks, nb, rows);
+  int ks, nb, rows, ch, cf;
+  seg_geom(c, kind, &ks, &nb, &rows, &ch, &cf);
+  *n = seg_count_lay(ks, nb, ch, cf, rows);
+  // (lo / hi: sub-range launches, row layout only -- callers pass ch = 0)
   *lo = c.wb ? 0 : std::min(*n, seg_of_row(yd + 1, ks, nb) + 1);
   *hi = c.wt ? *n : std::min(*n, std::max(*lo, seg_of_row(std::max(1, c.ny + 1 - yd), ks, nb)));
 }
@@ -1141,9 +1152,9 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
     for (size_t t = 0; t < ctx->chunks.size(); ++t) {
       auto& cs = ctx->chunks[t];
       int n;
-      phase_ranges(cs.c, kind, yd, &ilo[t], &ihi[t], &n);
       Chunk c = cs.c;
-      c.vch = c.lch = c.xch = c.ych = 0;  // sub-range launches: row order
+      c.vch = c.lch = c.xch = c.ych = 0;  // sub-range launches: row layout
+      phase_ranges(c, kind, yd, &ilo[t], &ihi[t], &n);
       int rc = 0;
       bool any = false;
       if (ilo[t] > 0) { c.seg0 = 0; rc = launch(cs, c, ilo[t], cm, cs.fix_b); any = true; }
@@ -1179,7 +1190,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
       vb.a[t].q = v.buf[B_Q];
       vb.a[t].fix = v.fix;
       g.x = std::max(g.x, grid_cols(v.c.nx, v.c.ny, v.c.vks).x);
-      g.y = std::max<unsigned>(g.y, (unsigned)seg_count(v.c.vks, v.c.vnb, v.c.ny));
+      g.y = std::max<unsigned>(g.y, (unsigned)seg_count_lay(v.c.vks, v.c.vnb, v.c.vch, v.c.vcf, v.c.ny));
     }
     launch_step(ks_visc_dt_b, g, SB, st, vb, ctx->scal, ctx->dtp);
     STEP_LAUNCH_CHECK();
@@ -1198,7 +1209,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
       if (deep) view = deep_view(ctx, cs0, DEEP_EXT_VISC);
       const ChunkState& cs = deep ? view : cs0;
       const Chunk c = with_rev(cs.c, CLOVER_SERP);  // top-down: sweep 2 wrote these rows last
-      launch_step(ks_visc_dt, dim3(grid_cols(c.nx, c.ny, c.vks).x, seg_count(c.vks, c.vnb, c.ny)), SB, st, c, cs.tm_visc, cs.buf[B_Q],
+      launch_step(ks_visc_dt, dim3(grid_cols(c.nx, c.ny, c.vks).x, seg_count_lay(c.vks, c.vnb, c.vch, c.vcf, c.ny)), SB, st, c, cs.tm_visc, cs.buf[B_Q],
                   ctx->scal, ctx->dtp, cs.fix);
       STEP_LAUNCH_CHECK();
       launch_fix(kf_visc_dt, FIX_BLOCKS, SB, st, c, cs.tm_visc, cs.buf[B_Q], ctx->scal, ctx->dtp,
@@ -1261,7 +1272,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
         lb.a[t] = LArgs{v.c, v.tm_lag, v.buf[B_D1], v.buf[B_E1], v.buf[B_U1], v.buf[B_V1],
                         v.buf[B_FX], v.buf[B_FY], v.fix};
         g.x = std::max(g.x, grid_strip(v.c.nx, LW, v.c.ny, v.c.lks).x);
-        g.y = std::max<unsigned>(g.y, (unsigned)seg_count(v.c.lks, v.c.lnb, v.c.ny));
+        g.y = std::max<unsigned>(g.y, (unsigned)seg_count_lay(v.c.lks, v.c.lnb, v.c.lch, v.c.lcf, v.c.ny));
       }
       launch_step(ks_lagrangian_b, g, SB, st, lb, ctx->scal);
       STEP_LAUNCH_CHECK();
@@ -1326,7 +1337,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
             xb.a[t] = XArgs{v.c, sweep == 1 ? v.tm_x1 : v.tm_x2, v.buf[rout], v.buf[eout],
                             v.buf[uout], v.buf[vout], v.fix};
             g.x = std::max(g.x, grid_strip(v.c.nx + 1, XW, v.c.ny + 1, v.c.xks).x);
-            g.y = std::max<unsigned>(g.y, (unsigned)seg_count(v.c.xks, v.c.xnb, v.c.ny + 1));
+            g.y = std::max<unsigned>(g.y, (unsigned)seg_count_lay(v.c.xks, v.c.xnb, v.c.xch, v.c.xcf, v.c.ny + 1));
           }
           if (sweep == 1) launch_step(ks_advec_x_b<1>, g, SB, st, xb);
           else launch_step(ks_advec_x_b<2>, g, SB, st, xb);
@@ -1409,7 +1420,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
                             v.buf[rout], v.buf[eout], v.buf[B_MY], v.buf[uout], v.buf[vout],
                             v.fix};
             g.x = std::max(g.x, grid_strip(v.c.nx + 1, YW, v.c.ny + 1, v.c.yks).x);
-            g.y = std::max<unsigned>(g.y, (unsigned)seg_count(v.c.yks, v.c.ynb, v.c.ny + 1));
+            g.y = std::max<unsigned>(g.y, (unsigned)seg_count_lay(v.c.yks, v.c.ynb, v.c.ych, v.c.ycf, v.c.ny + 1));
           }
           if (sweep == 1) launch_step(ks_advec_y_b<1>, g, SB, st, yb);
           else launch_step(ks_advec_y_b<2>, g, SB, st, yb);
@@ -1879,6 +1890,8 @@ int clover_init(const clover_grid* grid, const clover_state* states, int32_t nst
   ctx->deep = true;
   if (const char* e = std::getenv("CLOVER_DEEP_HALO")) ctx->deep = std::atoi(e) != 0;
   if (const char* e = std::getenv("CLOVER_BATCH")) ctx->batch = std::atoi(e) != 0;
+  ctx->chain = CLOVER_CHAIN != 0;  // band layout (band_layout; CLOVER_CHAIN=0 off)
+  if (const char* e = std::getenv("CLOVER_CHAIN")) ctx->chain = std::atoi(e) != 0;
   {
     int dev = 0;
     cudaGetDevice(&dev);
@@ -1922,7 +1935,7 @@ int clover_init(const clover_grid* grid, const clover_state* states, int32_t nst
     c.rev = 0;
     c.seg0 = 0;
     c.row0 = ROW0;
-    set_segs(c, ctx->nsm, ctx->occ);
+    set_segs(c, ctx->nsm, ctx->occ, ctx->chain);
     c.dx = dx; c.dy = dy; c.xmin = ctx->g.xmin; c.ymin = ctx->g.ymin;
     // correctly rounded reciprocals of the constant divisors (IEEE host division)
     c.rdx = 1.0 / dx; c.rdy = 1.0 / dy;
@@ -2177,7 +2190,9 @@ int clover_kernels_per_step(clover_ctx* ctx, int32_t* out) {
   // (run_phase with the boundary-first overlap)
   auto extra = [&](const ChunkState& cs, int kind, int yd) {
     int lo, hi, ns;
-    phase_ranges(cs.c, kind, yd, &lo, &hi, &ns);
+    Chunk c = cs.c;
+    c.vch = c.lch = c.xch = c.ych = 0;  // overlap launches use the row layout
+    phase_ranges(c, kind, yd, &lo, &hi, &ns);
     const int b = (lo > 0) + (hi < ns);
     return b + (b > 0) + 2 * (lo < hi) - 2;
   };

@@ -1,7 +1,7 @@
 # segment-chain A/B: kernel times (bm 3840^2 and active flow) per variant,
 # DRAM bytes per kernel under ncu for base and chain0, then the GPU suite
 mkdir -p gpurun_out
-VARIANTS="${VARIANTS:-base chain0 chainp2 chainm2}" bash scripts/gpu_ks_ab.sh
+VARIANTS="${VARIANTS:-base chain0 chainp1 chainm1}" bash scripts/gpu_ks_ab.sh
 cp gpurun_out/ks_ab.jsonl gpurun_out/chain_ab.jsonl
 for v in base chain0; do
   CLOVER_LIB=build_ab/libclover_$v.so timeout 600 ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum \

@@ -534,6 +534,26 @@ def test_batched_chunk_launches_bitwise(torch_cuda, monkeypatch, pxy, deep):
     assert np.array_equal(b.dt_history(1, 11), one.dt_history(1, 11))
 
 
+@pytest.mark.parametrize("pxy", [(1, 1), (1, 2)])
+def test_segment_chains_on_off_bitwise(torch_cuda, monkeypatch, pxy):
+    """Segment chains (seg_chain: the launch order walks consecutive row
+    segments in consecutive waves) change only which block runs which rows
+    when: a mesh large enough for several waves and chains on every kernel
+    (3840 x 4096; 1 x 2 batched chunks of 3840 x 2048 with deep halos) gives
+    the same bits with chains on and off (CLOVER_CHAIN=0).  The bm 3840^2
+    oracle comparison (test_full_size_first_steps) runs with chains on."""
+    deck = fuzz_deck(5, nx=3840, ny=4096)
+    deck["max_timestep"] = 1.0
+    on = make_gpu(deck, px=pxy[0], py=pxy[1])
+    monkeypatch.setenv("CLOVER_CHAIN", "0")
+    off = make_gpu(deck, px=pxy[0], py=pxy[1])
+    for g in (on, off):
+        g.step(4)
+    for f in STATE:
+        assert np.array_equal(on.read(f), off.read(f)), f
+    assert np.array_equal(on.dt_history(1, 4), off.dt_history(1, 4))
+
+
 def test_deep_halo_bm_blast_and_toggles(torch_cuda):
     """The bm blast crossing 1x4 strip boundaries for 40 steps with deep
     halos switched on and off between steps (the state halo is refreshed 7
