@@ -1690,6 +1690,9 @@ __device__ __forceinline__ bool advec_y_body(const Chunk& c, const CUtensorMap* 
   unsigned wsl = 4u % (unsigned)L::RING, wph = 0u;
   unsigned isl = 0u;  // slot of row s-2, refilled at the end of iteration s
 
+#ifdef CLOVER_YUNROLL
+  _Pragma(CLOVER_STR(unroll CLOVER_YUNROLL))
+#endif
   for (int s = k0 - 2; s <= k1; ++s) {
     if (s + 2 <= r_last) mbar_wait(&bars[wsl], wph);
     {

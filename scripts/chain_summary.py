@@ -3,8 +3,9 @@ ncu DRAM reads of gpurun_out/chain_ncu_{base,chain0}.csv."""
 import csv
 import json
 import re
+import sys
 
-txt = open("gpurun_out/chain_ab.jsonl").read()
+txt = open(sys.argv[1] if len(sys.argv) > 1 else "gpurun_out/chain_ab.jsonl").read()
 for m in re.finditer(r'\{"variant": "(\w+)", "mode": "(\w+)", "r": (\d), "t": (\{.*?\})\s*\n\}', txt, re.S):
     t = json.loads(m.group(4))
     k = t["kernels_ms"]
