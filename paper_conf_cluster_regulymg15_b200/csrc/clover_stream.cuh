@@ -709,156 +709,6 @@ __device__ __forceinline__ bool lagr_body(const Chunk& c, const CUtensorMap* __r
   return __any_sync(FULL, dv.bad);
 }
 
-// Interior body with the predictor skewed one row ahead (CLOVER_LSKEW):
-// iteration k evaluates the PdV predictor + EOS of cell row k+1 (rows k+1,
-// k+2) beside accelerate at node row k and the corrector of cell row k-1,
-// which use the half-step pressures of rows k-1 and k computed one
-// iteration earlier.  The two chains are independent, so the scheduler can
-// interleave them (the unskewed body is one serial chain per row:
-// predictor -> shuffle -> accelerate -> shuffle -> corrector).  Same
-// expressions on the same operands as lagr_body<D, false>: same bits.
-#ifndef CLOVER_LSKEW
-#define CLOVER_LSKEW 0
-#endif
-template <class D>
-__device__ __forceinline__ bool lagr_body_skew(const Chunk& c, const CUtensorMap* __restrict__ tm,
-                                               double* __restrict__ d1, double* __restrict__ e1,
-                                               double* __restrict__ u1, double* __restrict__ v1,
-                                               double* __restrict__ fx, double* __restrict__ fy,
-                                               const StepScalars* __restrict__ s, int gw, int k0,
-                                               int k1, int lane, double* ring,
-                                               unsigned long long* bars) {
-  static_assert(LSTG >= 5, "the skewed Lagrangian body holds rows k-1 .. k+2");
-  const int J0 = 1 + LW * gw;
-  const int j = J0 - 1 + lane;
-  D dv;
-  const double dt = s->dt, dx = c.dx, dy = c.dy;
-  const int r_first = k0 - 1, r_last = k1 + 1;  // staged rows
-  const int xcol = COL0 + J0 - 2;
-  auto slot_of = [&](int r) { return (unsigned)(r - r_first) % (unsigned)LSTG; };
-  auto issue_at = [&](unsigned sl, int r) {
-    mbar_arrive_expect_tx(&bars[sl], LBYTES);
-    tma_load_3d(ring + sl * LSLOT, tm, xcol, c.row0 + r, 0, &bars[sl]);
-  };
-  auto wait_row = [&](int r) {
-    const unsigned rel = (unsigned)(r - r_first);
-    mbar_wait(&bars[rel % LSTG], (rel / LSTG) & 1u);
-  };
-  auto row = [&](int r) -> const double* { return ring + slot_of(r) * LSLOT + lane + 1; };
-  if (lane == 0) {
-    for (int t = 0; t < LSTG; ++t) mbar_init(&bars[t], 1);
-    fence_mbar_init();
-    fence_proxy_async();
-    for (int r = r_first; r < r_first + LSTG && r <= r_last; ++r) issue_at(slot_of(r), r);
-  }
-  __syncwarp();
-  // half-step pressures of rows k0-1 (ph_m) and k0 (ph_c) before the loop
-  for (int r = r_first; r <= k0 + 1; ++r) wait_row(r);
-  double tfp;
-  double ph_m, phl_m, ph_c, phl_c;
-  {
-    const double* a = row(k0 - 1);
-    const double* b = row(k0);
-    const double* n = row(k0 + 1);
-    const double tfa = pdv_face_pred(b[LF_V * LRW], b[LF_V * LRW + 1], dx, dt);
-    ph_m = pdv_predict_pressure_bt(dv, a[LF_R * LRW], a[LF_E * LRW], a[LF_Q * LRW], a[LF_U * LRW],
-                                   b[LF_U * LRW], a[LF_U * LRW + 1], b[LF_U * LRW + 1],
-                                   pdv_face_pred(a[LF_V * LRW], a[LF_V * LRW + 1], dx, dt), tfa,
-                                   dx, dy, c.rvol, dt);
-    tfp = pdv_face_pred(n[LF_V * LRW], n[LF_V * LRW + 1], dx, dt);
-    ph_c = pdv_predict_pressure_bt(dv, b[LF_R * LRW], b[LF_E * LRW], b[LF_Q * LRW], b[LF_U * LRW],
-                                   n[LF_U * LRW], b[LF_U * LRW + 1], n[LF_U * LRW + 1], tfa, tfp,
-                                   dx, dy, c.rvol, dt);
-    phl_m = __shfl_up_sync(FULL, ph_m, 1);
-    phl_c = __shfl_up_sync(FULL, ph_c, 1);
-  }
-  double tsum_m = 0.0, tfc_m = 0.0;
-  const double vol = dx * dy;
-  double mass_m, massl_m;
-  {
-    const double* a = row(k0 - 1);
-    mass_m = a[LF_R * LRW] * vol;
-    massl_m = a[LF_R * LRW - 1] * vol;
-  }
-  double u1_m = 0.0, v1_m = 0.0, u1r_m = 0.0, v1r_m = 0.0;
-  // ring rows k-1 .. k+2 of the iteration, rotated at its end; slot / phase
-  // of row k+2 for its wait
-  const double* Pm = row(k0 - 1);
-  const double* Pc = row(k0);
-  const double* Pn = row(k0 + 1);
-  const double* Pnn = row(k0 + 2);
-  unsigned wsl = 3u % (unsigned)LSTG, wph = 0u;
-  unsigned isl = 0u;  // slot of row k-1, refilled at the end of iteration k
-  for (int k = k0; k <= k1; ++k) {
-    const double* rm = Pm;
-    const double* rc = Pc;
-    // predictor of row k+1 (rows k+1, k+2), independent of the rest
-    double ph_n = 0.0, phl_n = 0.0;
-    if (k + 2 <= r_last) {
-      mbar_wait(&bars[wsl], wph);  // row k+2
-      const double* rn = Pn;
-      const double* rnn = Pnn;
-      const double tf = pdv_face_pred(rnn[LF_V * LRW], rnn[LF_V * LRW + 1], dx, dt);
-      ph_n = pdv_predict_pressure_bt(dv, rn[LF_R * LRW], rn[LF_E * LRW], rn[LF_Q * LRW],
-                                     rn[LF_U * LRW], rnn[LF_U * LRW], rn[LF_U * LRW + 1],
-                                     rnn[LF_U * LRW + 1], tfp, tf, dx, dy, c.rvol, dt);
-      tfp = tf;
-      phl_n = __shfl_up_sync(FULL, ph_n, 1);
-    }
-    // accelerate at node (j,k): cells (j-1,k-1), (j,k-1), (j,k), (j-1,k)
-    double u1_c, v1_c;
-    const double mass_c = rc[LF_R * LRW] * vol;
-    const double massl_c = rc[LF_R * LRW - 1] * vol;
-    {
-      const double pp[4] = {phl_m, ph_m, ph_c, phl_c};
-      const double qv[4] = {rm[LF_Q * LRW - 1], rm[LF_Q * LRW], rc[LF_Q * LRW], rc[LF_Q * LRW - 1]};
-      const double mm[4] = {massl_m, mass_m, mass_c, massl_c};
-      accelerate_node_m(dv, mm, pp, qv, rc[LF_U * LRW], rc[LF_V * LRW], dx, dy, dt, u1_c, v1_c);
-    }
-    const double u1r_c = __shfl_down_sync(FULL, u1_c, 1);
-    const double v1r_c = __shfl_down_sync(FULL, v1_c, 1);
-    // PdV corrector + flux_calc of cell (j,k-1)
-    const int kc = k - 1;
-    const double tsum_c = rc[LF_V * LRW] + rc[LF_V * LRW + 1] + v1_c + v1r_c;
-    const double tfc_c = pdv_face_corr(tsum_c, dx, dt);
-    if (kc >= k0 && lane >= 1 && lane <= LW) {
-      const double lsum = rm[LF_U * LRW] + rc[LF_U * LRW] + u1_m + u1_c;
-      const double rsum = rm[LF_U * LRW + 1] + rc[LF_U * LRW + 1] + u1r_m + u1r_c;
-      double ev, dvv;
-      pdv_correct_bt(dv, rm[LF_R * LRW], rm[LF_E * LRW], ph_m, rm[LF_Q * LRW], lsum, rsum, tfc_m,
-                     tfc_c, dx, dy, c.rvol, dt, ev, dvv);
-      const int ic = idx(c, j, kc);
-      const double cx = 0.25 * dt * dy, cy = 0.25 * dt * dx;
-      e1[ic] = ev;
-      d1[ic] = dvv;
-      fx[ic] = cx * lsum;
-      fy[ic] = cy * tsum_m;
-      u1[ic] = u1_m;
-      v1[ic] = v1_m;
-    }
-    ph_m = ph_c; phl_m = phl_c;
-    ph_c = ph_n; phl_c = phl_n;
-    u1_m = u1_c; v1_m = v1_c; u1r_m = u1r_c; v1r_m = v1r_c;
-    tsum_m = tsum_c; tfc_m = tfc_c;
-    mass_m = mass_c; massl_m = massl_c;
-    // row k-1 is consumed (rows k .. k+2 are read next iteration)
-#if CLOVER_TMA_RELEASE_FENCE
-    fence_proxy_async();
-#endif
-    __syncwarp();
-    if (lane == 0 && k - 1 + LSTG <= r_last) issue_at(isl, k - 1 + LSTG);
-    if (++isl == (unsigned)LSTG) isl = 0u;
-    Pm = Pc; Pc = Pn; Pn = Pnn;
-    if (++wsl == (unsigned)LSTG) { wsl = 0u; wph ^= 1u; }
-    Pnn = ring + wsl * LSLOT + lane + 1;
-  }
-  __syncwarp();
-  if (lane == 0)
-    for (int t = 0; t < LSTG; ++t) mbar_inval(&bars[t]);
-  __syncwarp();
-  return __any_sync(FULL, dv.bad);
-}
-
 __device__ __forceinline__ bool lagr_interior(const Chunk& c, int gw, int k0, int k1) {
   const int J0 = 1 + LW * gw;
   return J0 - 2 >= HALO + 2 && J0 + 31 <= c.nx - HALO - 1 && k0 - 1 >= HALO + 2 &&
@@ -872,13 +722,8 @@ __device__ __forceinline__ bool lagr_seg(const Chunk& c, const CUtensorMap* __re
                                          double* __restrict__ fx, double* __restrict__ fy,
                                          const StepScalars* __restrict__ s, int gw, int k0, int k1,
                                          int lane, double* ring, unsigned long long* bars) {
-  if (lagr_interior(c, gw, k0, k1)) {
-#if CLOVER_LSKEW
-    return lagr_body_skew<D>(c, tm, d1, e1, u1, v1, fx, fy, s, gw, k0, k1, lane, ring, bars);
-#else
+  if (lagr_interior(c, gw, k0, k1))
     return lagr_body<D, false>(c, tm, d1, e1, u1, v1, fx, fy, s, gw, k0, k1, lane, ring, bars);
-#endif
-  }
   return lagr_body<D, true>(c, tm, d1, e1, u1, v1, fx, fy, s, gw, k0, k1, lane, ring, bars);
 }
 
