@@ -3,10 +3,7 @@ VERDICT r1 #8: bm 64^2 for 20 steps on one chunk, and a 2x2 local-chunk
 fuzz deck for 2 steps (halo exchange + separate sweep kernels), both
 checked against the oracle; 1x3 y strips with deep halos (deep), also
 through the device-initiated store transport (lsa).
-bands: meshes large enough for the band layout of the row segments on
-every kernel (3840 x 2048 on one chunk; 3840 x 3200 as 1 x 2 batched
-deep-halo strips), 1 step.
-usage: sanitize_run.py [bm|chunks|deep|lsa|bands|bands2]"""
+usage: sanitize_run.py [bm|chunks|deep|lsa]"""
 import os
 import sys
 
@@ -26,10 +23,6 @@ elif case in ("deep", "lsa"):
     # y strips with deep halos (row-shifted views), and the device-initiated
     # store transport (one-rank NCCL symmetric window)
     deck, kw, steps = fuzz_deck(9, nx=48, ny=64), dict(px=1, py=3), 3
-elif case == "bands":
-    deck, kw, steps = fuzz_deck(9, nx=3840, ny=2048), {}, 1
-elif case == "bands2":
-    deck, kw, steps = fuzz_deck(9, nx=3840, ny=3200), dict(px=1, py=2), 1
 else:
     deck, kw, steps = fuzz_deck(9, nx=48, ny=40), dict(px=2, py=2), 2
 g = Clover(deck, **kw)
