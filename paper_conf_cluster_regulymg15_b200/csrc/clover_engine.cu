@@ -149,6 +149,8 @@ int64_t field_elems(int nx, int ny, int* pitch_out) {
 // (grid shapes as in enqueue_step).
 inline int cdiv(int a, int b) { return (a + b - 1) / b; }
 dim3 grid_cols(int ncols, int nrows, int ks) { return dim3(cdiv(ncols, SB), cdiv(nrows, ks)); }
+// visc_dt's grid (blocks of SBV threads, one column per thread)
+dim3 grid_cols_v(int ncols, int nrows, int ks) { return dim3(cdiv(ncols, SBV), cdiv(nrows, ks)); }
 dim3 grid_strip(int ncols, int width, int nrows, int ks) {
   return dim3(cdiv(cdiv(ncols, width), SB / 32), cdiv(nrows, ks));
 }
@@ -199,11 +201,12 @@ int64_t fix_capacity(int nx, int ny) {
   // (adaptive segments: tail segments have at least 4 rows, see tail_nb;
   // the band layout adds at most one shorter segment per band: bounded by
   // counting segments of 2 rows)
-  const dim3 g[8] = {grid_cols(nx, ny, 2),          grid_strip(nx, LW, ny, 2),
+  const dim3 g[7] = {grid_strip(nx, LW, ny, 2),
                      grid_strip(nx, CW_X, ny, CKS),    grid_cols(nx, ny, CKS_Y),
                      grid_strip(nx + 1, MW_X, ny + 1, MKS), grid_cols(nx + 1, ny + 1, MKS_Y),
                      grid_strip(nx + 1, XW, ny + 1, 2), grid_strip(nx + 1, YW, ny + 1, 2)};
-  int64_t m = 0;
+  const dim3 gv = grid_cols_v(nx, ny, 2);  // visc_dt: SBV-thread blocks
+  int64_t m = (int64_t)gv.x * gv.y * (SBV / 32);
   for (const dim3& d : g) m = std::max<int64_t>(m, (int64_t)d.x * d.y * (SB / 32));
   return m;
 }
@@ -1007,15 +1010,15 @@ void band_layout(bool on, int ks, int64_t colblocks, int rows, int64_t slots, in
 }
 
 void set_segs(Chunk& c, int nsm, const int occ[4], bool chain) {
-  c.vks = seg_rows(VKS, grid_cols(c.nx, c.ny, VKS).x, c.ny);
+  c.vks = seg_rows(VKS, grid_cols_v(c.nx, c.ny, VKS).x, c.ny);
   c.lks = seg_rows(LKS, grid_strip(c.nx, LW, c.ny, LKS).x, c.ny);
   c.xks = seg_rows(XKS, grid_strip(c.nx + 1, XW, c.ny + 1, XKS).x, c.ny + 1);
   c.yks = seg_rows(YKS, grid_strip(c.nx + 1, YW, c.ny + 1, YKS).x, c.ny + 1);
-  c.vnb = tail_nb(c.vks, grid_cols(c.nx, c.ny, c.vks).x, c.ny, (int64_t)nsm * occ[0]);
+  c.vnb = tail_nb(c.vks, grid_cols_v(c.nx, c.ny, c.vks).x, c.ny, (int64_t)nsm * occ[0]);
   c.lnb = tail_nb(c.lks, grid_strip(c.nx, LW, c.ny, c.lks).x, c.ny, (int64_t)nsm * occ[1]);
   c.xnb = tail_nb(c.xks, grid_strip(c.nx + 1, XW, c.ny + 1, c.xks).x, c.ny + 1, (int64_t)nsm * occ[2]);
   c.ynb = tail_nb(c.yks, grid_strip(c.nx + 1, YW, c.ny + 1, c.yks).x, c.ny + 1, (int64_t)nsm * occ[3]);
-  band_layout(chain, c.vks, grid_cols(c.nx, c.ny, c.vks).x, c.ny, (int64_t)nsm * occ[0], &c.vch, &c.vcf);
+  band_layout(chain, c.vks, grid_cols_v(c.nx, c.ny, c.vks).x, c.ny, (int64_t)nsm * occ[0], &c.vch, &c.vcf);
   band_layout(chain, c.lks, grid_strip(c.nx, LW, c.ny, c.lks).x, c.ny, (int64_t)nsm * occ[1], &c.lch, &c.lcf);
   band_layout(chain, c.xks, grid_strip(c.nx + 1, XW, c.ny + 1, c.xks).x, c.ny + 1, (int64_t)nsm * occ[2],
               &c.xch, &c.xcf);
@@ -1189,12 +1192,12 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
       vb.a[t].tm = v.tm_visc;
       vb.a[t].q = v.buf[B_Q];
       vb.a[t].fix = v.fix;
-      g.x = std::max(g.x, grid_cols(v.c.nx, v.c.ny, v.c.vks).x);
+      g.x = std::max(g.x, grid_cols_v(v.c.nx, v.c.ny, v.c.vks).x);
       g.y = std::max<unsigned>(g.y, (unsigned)seg_count_lay(v.c.vks, v.c.vnb, v.c.vch, v.c.vcf, v.c.ny));
     }
-    launch_step(ks_visc_dt_b, g, SB, st, vb, ctx->scal, ctx->dtp);
+    launch_step(ks_visc_dt_b, g, SBV, st, vb, ctx->scal, ctx->dtp);
     STEP_LAUNCH_CHECK();
-    launch_fix(kf_visc_dt_b, dim3(FIX_BLOCKS, 1, g.z), SB, st, vb, ctx->scal, ctx->dtp);
+    launch_fix(kf_visc_dt_b, dim3(FIX_BLOCKS, 1, g.z), SBV, st, vb, ctx->scal, ctx->dtp);
     FIX_LAUNCH_CHECK();
     if (needs_exchange(ctx) && !deep) {
       int rc = exchange_axis(ctx, {B_Q}, 0);
@@ -1209,10 +1212,10 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
       if (deep) view = deep_view(ctx, cs0, DEEP_EXT_VISC);
       const ChunkState& cs = deep ? view : cs0;
       const Chunk c = with_rev(cs.c, CLOVER_SERP);  // top-down: sweep 2 wrote these rows last
-      launch_step(ks_visc_dt, dim3(grid_cols(c.nx, c.ny, c.vks).x, seg_count_lay(c.vks, c.vnb, c.vch, c.vcf, c.ny)), SB, st, c, cs.tm_visc, cs.buf[B_Q],
+      launch_step(ks_visc_dt, dim3(grid_cols_v(c.nx, c.ny, c.vks).x, seg_count_lay(c.vks, c.vnb, c.vch, c.vcf, c.ny)), SBV, st, c, cs.tm_visc, cs.buf[B_Q],
                   ctx->scal, ctx->dtp, cs.fix);
       STEP_LAUNCH_CHECK();
-      launch_fix(kf_visc_dt, FIX_BLOCKS, SB, st, c, cs.tm_visc, cs.buf[B_Q], ctx->scal, ctx->dtp,
+      launch_fix(kf_visc_dt, FIX_BLOCKS, SBV, st, c, cs.tm_visc, cs.buf[B_Q], ctx->scal, ctx->dtp,
                   cs.fix, ctx->hist, fold_fin);
       FIX_LAUNCH_CHECK();
     }
@@ -1896,7 +1899,7 @@ int clover_init(const clover_grid* grid, const clover_state* states, int32_t nst
     int dev = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&ctx->nsm, cudaDevAttrMultiProcessorCount, dev);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&ctx->occ[0], ks_visc_dt, SB, 0);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&ctx->occ[0], ks_visc_dt, SBV, 0);
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&ctx->occ[1], ks_lagrangian, SB, 0);
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&ctx->occ[2], ks_advec_x<1>, SB, 0);
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&ctx->occ[3], ks_advec_y<1>, SB, 0);

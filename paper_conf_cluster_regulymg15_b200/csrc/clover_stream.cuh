@@ -27,9 +27,16 @@ namespace clover {
 
 constexpr unsigned FULL = 0xffffffffu;
 #ifndef CLOVER_SB
-#define CLOVER_SB 64
+#define CLOVER_SB 32
 #endif
-constexpr int SB = CLOVER_SB;  // threads per block
+constexpr int SB = CLOVER_SB;  // threads per block (one warp: a block slot frees as soon as its
+                               // warp's segment is done; measured faster than 2-warp blocks for the
+                               // Lagrangian and both sweeps)
+#ifndef CLOVER_SBV
+#define CLOVER_SBV 64
+#endif
+constexpr int SBV = CLOVER_SBV;  // visc_dt threads per block (its streaming-only bm segments are
+                                 // short: 1-warp blocks cost more in block launches than they save)
 
 // Tunables (defaults = measured best; scripts/ab_variants.py builds others).
 #define CLOVER_STR2(x) #x
@@ -44,11 +51,15 @@ constexpr int SB = CLOVER_SB;  // threads per block
 // 3840^2 (scripts/ab_variants.py), 64-thread blocks: lagrangian 10 (96 regs),
 // visc_dt uncapped, advection 16 (64 regs), mom_y 14.  Short row segments
 // (8-16 rows) measured 6 % faster than 16-32 (more, shorter blocks).
+// Round 2, 32-thread blocks: the Lagrangian at (32, 10), which ptxas
+// compiles to 108 registers (18 warps/SM: 0.262 -> 0.253 ms; plain (32)
+// gives 80), the unfused advection kernels at the same warps per SM as
+// before (the counts scale with 64 / SB).
 #ifndef CLOVER_MINB_HEAVY
 #define CLOVER_MINB_HEAVY 10
 #endif
 #ifndef CLOVER_MINB_ADV
-#define CLOVER_MINB_ADV 16
+#define CLOVER_MINB_ADV (16 * 64 / CLOVER_SB)
 #endif
 #ifndef CLOVER_MINB_VISC
 #define CLOVER_MINB_VISC 0
@@ -70,7 +81,7 @@ constexpr int SB = CLOVER_SB;  // threads per block
 #define LB_ADVY __launch_bounds__(SB)
 #endif
 #ifndef CLOVER_MINB_MOMY
-#define CLOVER_MINB_MOMY 14
+#define CLOVER_MINB_MOMY (14 * 64 / CLOVER_SB)
 #endif
 #if CLOVER_MINB_MOMY > 0
 #define LB_MOMY __launch_bounds__(SB, CLOVER_MINB_MOMY)
@@ -83,9 +94,9 @@ constexpr int SB = CLOVER_SB;  // threads per block
 #define LB_HEAVY __launch_bounds__(SB)
 #endif
 #if CLOVER_MINB_VISC > 0
-#define LB_VISC __launch_bounds__(SB, CLOVER_MINB_VISC)
+#define LB_VISC __launch_bounds__(SBV, CLOVER_MINB_VISC)
 #else
-#define LB_VISC __launch_bounds__(SB)
+#define LB_VISC __launch_bounds__(SBV)
 #endif
 #if CLOVER_MINB_ADV > 0
 #define LB_ADV __launch_bounds__(SB, CLOVER_MINB_ADV)
@@ -147,7 +158,7 @@ struct NoLast {
 #define CLOVER_FIX_BLOCKS 148
 #endif
 constexpr int FIX_BLOCKS = CLOVER_FIX_BLOCKS;  // fixup blocks (one per SM); a launch may add y-wall blocks
-template <class Run, class Last = NoLast>
+template <int BS = SB, class Run, class Last = NoLast>
 __device__ __forceinline__ void fix_loop(FixSlot f, int ks, int nb, int ch, int cf, int lim, Run&& run,
                                          Last last = {}) {
   const unsigned n = *(volatile unsigned*)f.hdr;  // the same value in every thread
@@ -158,7 +169,7 @@ __device__ __forceinline__ void fix_loop(FixSlot f, int ks, int nb, int ch, int 
   }
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const unsigned items = n * (unsigned)ks;
-  for (unsigned it = blockIdx.x * (SB / 32) + w; it < items; it += FIX_BLOCKS * (SB / 32)) {
+  for (unsigned it = blockIdx.x * (BS / 32) + w; it < items; it += FIX_BLOCKS * (BS / 32)) {
     const uint2 t = f.e[it / ks];
     int ks0, len;
     seg_rows_lay((int)t.y, ks, nb, ch, cf, lim - 1, ks0, len);
@@ -407,10 +418,10 @@ ks_visc_dt(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__
            StepScalars* __restrict__ s, DtParams prm, FixSlot fix) {
   pdl_trigger();
   pdl_wait();
-  __shared__ __align__(128) double ring[SB / 32][VSTG * VSLOT];
-  __shared__ __align__(8) unsigned long long bars[SB / 32][VSTG];
+  __shared__ __align__(128) double ring[SBV / 32][VSTG * VSLOT];
+  __shared__ __align__(8) unsigned long long bars[SBV / 32][VSTG];
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  const int gw = blockIdx.x * (SB / 32) + warp;
+  const int gw = blockIdx.x * (SBV / 32) + warp;
   double dtw = G_BIG;
   int k0, len;
   const int sg = seg_y(c);
@@ -424,33 +435,33 @@ ks_visc_dt(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__
       dtw = G_BIG;  // this warp's dt comes from the fixup
     }
   }
-  __shared__ double wmin[SB / 32];
+  __shared__ double wmin[SBV / 32];
   if (lane == 0) wmin[warp] = dtw;
   __syncthreads();
   if (threadIdx.x == 0) {
     double m = wmin[0];
-    for (int w = 1; w < SB / 32; ++w) m = fmin(m, wmin[w]);
-    atomicMin(&s->dt_slot, (unsigned long long)__double_as_longlong(m));
+    for (int w = 1; w < SBV / 32; ++w) m = fmin(m, wmin[w]);
+    dt_slot_min(s, m);
   }
 }
 
-__global__ void __launch_bounds__(SB)
+__global__ void __launch_bounds__(SBV)
 kf_visc_dt(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__ q,
            StepScalars* __restrict__ s, DtParams prm, FixSlot fix, double* __restrict__ hist,
            int fin) {
   pdl_trigger();
   pdl_wait();
-  __shared__ __align__(128) double ring[SB / 32][VSTG * VSLOT];
-  __shared__ __align__(8) unsigned long long bars[SB / 32][VSTG];
+  __shared__ __align__(128) double ring[SBV / 32][VSTG * VSLOT];
+  __shared__ __align__(8) unsigned long long bars[SBV / 32][VSTG];
   // fin: single chunk on one rank -- the last block also finalises dt
   // (k_dt_finalize's work, once every contribution to the slot is in)
-  fix_loop(
+  fix_loop<SBV>(
       fix, c.vks, c.vnb, c.vch, c.vcf, c.ny + 1,
       [&](int gw, int k0, int k1, int lane, int w) {
         double dtw;
         visc_ring_rows(c, k0, k1);  // rows 1 / ny redo their ring row too
         visc_seg<DivIEEE>(c, &tm, q, prm, gw, k0, k1, lane, ring[w], bars[w], dtw);
-        if (lane == 0) atomicMin(&s->dt_slot, (unsigned long long)__double_as_longlong(dtw));
+        if (lane == 0) dt_slot_min(s, dtw);
       },
       [&]() {
         if (fin) dt_finalize(s, hist, prm);
@@ -1527,8 +1538,8 @@ constexpr int YKS = CLOVER_YKS;
 #ifndef CLOVER_YRING2
 #define CLOVER_YRING2 7
 #endif
-#ifndef CLOVER_YMINB1
-#define CLOVER_YMINB1 9
+#ifndef CLOVER_YMINB1  // (18 one-warp blocks: 94 registers; uncapped it takes 106, 2 % slower)
+#define CLOVER_YMINB1 (9 * 64 / CLOVER_SB)
 #endif
 #ifndef CLOVER_L2HINT  // y sweep: L2 policy for the ring rows shared with the segment below
 #define CLOVER_L2HINT 0
@@ -1862,10 +1873,10 @@ ks_visc_dt_b(const __grid_constant__ KBatch<VArgs> b, StepScalars* __restrict__ 
   const VArgs& a = b.a[blockIdx.z];
   const Chunk& c = a.c;
   if ((int)blockIdx.y >= seg_count_lay(c.vks, c.vnb, c.vch, c.vcf, c.ny)) return;
-  __shared__ __align__(128) double ring[SB / 32][VSTG * VSLOT];
-  __shared__ __align__(8) unsigned long long bars[SB / 32][VSTG];
+  __shared__ __align__(128) double ring[SBV / 32][VSTG * VSLOT];
+  __shared__ __align__(8) unsigned long long bars[SBV / 32][VSTG];
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  const int gw = blockIdx.x * (SB / 32) + warp;
+  const int gw = blockIdx.x * (SBV / 32) + warp;
   double dtw = G_BIG;
   int k0, len;
   const int sg = (int)blockIdx.y;
@@ -1879,28 +1890,28 @@ ks_visc_dt_b(const __grid_constant__ KBatch<VArgs> b, StepScalars* __restrict__ 
       dtw = G_BIG;
     }
   }
-  __shared__ double wmin[SB / 32];
+  __shared__ double wmin[SBV / 32];
   if (lane == 0) wmin[warp] = dtw;
   __syncthreads();
   if (threadIdx.x == 0) {
     double m = wmin[0];
-    for (int w = 1; w < SB / 32; ++w) m = fmin(m, wmin[w]);
-    atomicMin(&s->dt_slot, (unsigned long long)__double_as_longlong(m));
+    for (int w = 1; w < SBV / 32; ++w) m = fmin(m, wmin[w]);
+    dt_slot_min(s, m);
   }
 }
-__global__ void __launch_bounds__(SB)
+__global__ void __launch_bounds__(SBV)
 kf_visc_dt_b(const __grid_constant__ KBatch<VArgs> b, StepScalars* __restrict__ s, DtParams prm) {
   pdl_trigger();
   pdl_wait();
   const VArgs& a = b.a[blockIdx.z];
   const Chunk& c = a.c;
-  __shared__ __align__(128) double ring[SB / 32][VSTG * VSLOT];
-  __shared__ __align__(8) unsigned long long bars[SB / 32][VSTG];
-  fix_loop(a.fix, c.vks, c.vnb, c.vch, c.vcf, c.ny + 1, [&](int gw, int k0, int k1, int lane, int w) {
+  __shared__ __align__(128) double ring[SBV / 32][VSTG * VSLOT];
+  __shared__ __align__(8) unsigned long long bars[SBV / 32][VSTG];
+  fix_loop<SBV>(a.fix, c.vks, c.vnb, c.vch, c.vcf, c.ny + 1, [&](int gw, int k0, int k1, int lane, int w) {
     double dtw;
     visc_ring_rows(c, k0, k1);
     visc_seg<DivIEEE>(c, &a.tm, a.q, prm, gw, k0, k1, lane, ring[w], bars[w], dtw);
-    if (lane == 0) atomicMin(&s->dt_slot, (unsigned long long)__double_as_longlong(dtw));
+    if (lane == 0) dt_slot_min(s, dtw);
   });
 }
 
