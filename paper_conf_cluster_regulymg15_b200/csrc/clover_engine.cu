@@ -234,12 +234,12 @@ EncodeTiledFn encode_tiled() {
 // staged row of a kernel's ring.  Out-of-range columns (the last warp strip)
 // read as zeros.
 int encode_rows_map(CUtensorMap* m, const double* base, int pitch, int rows, int64_t fstride,
-                    int nf, int boxw) {
+                    int nf, int boxw, int boxh = 1) {
   EncodeTiledFn fn = encode_tiled();
   if (!fn) return fail(CLOVER_ERR_CUDA, "cuTensorMapEncodeTiled unavailable");
   const cuuint64_t dims[3] = {(cuuint64_t)pitch, (cuuint64_t)rows, (cuuint64_t)nf};
   const cuuint64_t strides[2] = {(cuuint64_t)pitch * 8, (cuuint64_t)fstride};
-  const cuuint32_t box[3] = {(cuuint32_t)boxw, 1, (cuuint32_t)nf};
+  const cuuint32_t box[3] = {(cuuint32_t)boxw, (cuuint32_t)boxh, (cuuint32_t)nf};
   const cuuint32_t es[3] = {1, 1, 1};
   CUresult r = fn(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 3, (void*)base, dims, strides, box, es,
                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
@@ -1951,9 +1951,9 @@ int clover_init(const clover_grid* grid, const clover_state* states, int32_t nst
     {
       const double* base = cs.buf[B_D0] - (int64_t)ROW0 * c.pitch - COL0;
       const int rows = c.ny + 2 + 2 * HALO_ROWS;
-      int rc = encode_rows_map(&cs.tm_lag, base, c.pitch, rows, align_up(fe * 8, kAlign), LNF, LRW);
+      int rc = encode_rows_map(&cs.tm_lag, base, c.pitch, rows, align_up(fe * 8, kAlign), LNF, LRW, LBOX);
       const int64_t fs = align_up(fe * 8, kAlign);
-      if (!rc) rc = encode_rows_map(&cs.tm_visc, base, c.pitch, rows, fs, VNF, VRW);
+      if (!rc) rc = encode_rows_map(&cs.tm_visc, base, c.pitch, rows, fs, VNF, VRW, VBOX);
       if (!rc) rc = encode_rows_map(&cs.tm_x1, base + (B_D1 - B_D0) * (fs / 8), c.pitch, rows, fs,
                                     XF<1>::NF, XRW);
       if (!rc) rc = encode_rows_map(&cs.tm_x2, base + (B_FX - B_D0) * (fs / 8), c.pitch, rows, fs,

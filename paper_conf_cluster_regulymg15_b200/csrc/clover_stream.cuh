@@ -276,8 +276,8 @@ __device__ __forceinline__ bool y_walls_after_fix(const Chunk& c, FixSlot f, con
 
 // ================================================================ visc_dt
 // Warp w of the grid owns columns j = 32*w + lane + 1 over rows [k0, k0+VKS).
-// Rows of d0, e0, u0, v0 stream through a per-warp VSTG-row shared-memory
-// ring, one 3D TMA tensor copy per row (the four fields are consecutive
+// Rows of d0, e0, u0, v0 stream through a per-warp shared-memory ring of
+// VSTG slots of VBOX rows, one 3D TMA tensor copy per slot (the four fields are consecutive
 // equally spaced buffers); smem column t of a slot holds memory column
 // COL0 - 1 + 32*w + t, so lane l reads its column at t = l+2 and both x
 // neighbours.  Iteration k reads rows k and k+1 (the pressures of rows k-1
@@ -286,14 +286,26 @@ __device__ __forceinline__ bool y_walls_after_fix(const Chunk& c, FixSlot f, con
 // memory (an odd start column faults with an illegal instruction on B200;
 // scripts/tma_probe.cu).
 constexpr int VKS = CLOVER_VKS;
-#ifndef CLOVER_VSTG
-#define CLOVER_VSTG 4
+#ifndef CLOVER_VSTG  // ring slots (boxes of VBOX rows)
+#define CLOVER_VSTG 2
 #endif
 constexpr int VSTG = CLOVER_VSTG;
 constexpr int VRW = 36;
+// rows per tensor copy (ring slot): one copy brings VBOX consecutive rows of
+// the four fields (box {VRW, VBOX, 4}; smem slot [field][row][column]).
+// Round 2: 2 slots of 4 rows instead of 4 slots of 1 row -- the same
+// bytes in flight in a quarter of the copies: bm window 0.136 -> 0.127 ms
+// (profiles/r2_vbox_ab.jsonl; 2x4 and 3x2 rows 0.130 / 0.133, 2x8 0.145,
+// 3x4 0.134); the kernel streams more than it computes there, and fewer,
+// larger copies reach the data sooner.
+#ifndef CLOVER_VBOX
+#define CLOVER_VBOX 4
+#endif
+constexpr int VBOX = CLOVER_VBOX;
 enum { VF_R, VF_E, VF_U, VF_V, VNF };  // = buffer order B_D0 B_E0 B_U0 B_V0
-constexpr int VSLOT = VNF * VRW;       // 1152 B: a multiple of 128 B
-constexpr unsigned VBYTES = VNF * VRW * 8;
+constexpr int VFS = VBOX * VRW;        // field stride in a slot (doubles)
+constexpr int VSLOT = VNF * VFS;       // 1152 B per row: a multiple of 128 B
+constexpr unsigned VBYTES = VNF * VFS * 8;
 static_assert((VSLOT * 8) % 128 == 0 && VSTG >= 2, "visc ring");
 static_assert(COL0 % 2 == 1, "visc ring box starts on an even (16-B aligned) column");
 
@@ -311,39 +323,51 @@ __device__ __forceinline__ bool visc_body(const Chunk& c, const CUtensorMap* __r
   D dv;
   const int r_first = k0 - 1, r_last = k1;
   const int xcol = COL0 - 1 + gw * 32;  // even (COL0 = 15)
-  auto slot_of = [&](int r) { return (unsigned)(r - r_first) % (unsigned)VSTG; };
-  auto issue = [&](int r) {
+  // ring slot of a row: its box (VBOX rows from r_first) modulo VSTG
+  auto slot_of = [&](int r) { return ((unsigned)(r - r_first) / (unsigned)VBOX) % (unsigned)VSTG; };
+  auto issue = [&](int r) {  // the box whose first row is r
     const unsigned sl = slot_of(r);
     mbar_arrive_expect_tx(&bars[sl], VBYTES);
     tma_load_3d(ring + sl * VSLOT, tm, xcol, c.row0 + r, 0, &bars[sl]);
   };
   auto wait_row = [&](int r) {
-    const unsigned rel = (unsigned)(r - r_first);
-    mbar_wait(&bars[rel % VSTG], (rel / VSTG) & 1u);
+    const unsigned box = (unsigned)(r - r_first) / (unsigned)VBOX;
+    mbar_wait(&bars[box % VSTG], (box / VSTG) & 1u);
   };
-  auto row = [&](int r) -> const double* { return ring + slot_of(r) * VSLOT + lane + 2; };
+  auto row = [&](int r) -> const double* {
+    return ring + slot_of(r) * VSLOT + ((unsigned)(r - r_first) % (unsigned)VBOX) * VRW + lane + 2;
+  };
+  // row r consumed: when it is its box's last row, refill the slot with the
+  // box VSTG boxes further on
+  auto release = [&](int r) {
+    const unsigned rel = (unsigned)(r - r_first);
+    if (rel % VBOX == VBOX - 1 && lane == 0) {
+      const int nr = r + 1 + (VSTG - 1) * VBOX;
+      if (nr <= r_last) issue(nr);
+    }
+  };
   if (lane == 0) {
     for (int t = 0; t < VSTG; ++t) mbar_init(&bars[t], 1);
     fence_mbar_init();
     fence_proxy_async();
-    for (int r = r_first; r < r_first + VSTG && r <= r_last; ++r) issue(r);
+    for (int r = r_first; r < r_first + VSTG * VBOX && r <= r_last; r += VBOX) issue(r);
   }
   __syncwarp();
   const bool ncol = EDGE && near_wall_col(c, j);
   wait_row(r_first);
   wait_row(k0);
-  double pcm = eos_pressure(row(r_first)[VF_R * VRW], row(r_first)[VF_E * VRW]);  // p(k-1)
-  double pc = eos_pressure(row(k0)[VF_R * VRW], row(k0)[VF_E * VRW]);            // p(k)
+  double pcm = eos_pressure(row(r_first)[VF_R * VFS], row(r_first)[VF_E * VFS]);  // p(k-1)
+  double pc = eos_pressure(row(k0)[VF_R * VFS], row(k0)[VF_E * VFS]);            // p(k)
 #if CLOVER_TMA_RELEASE_FENCE
   fence_proxy_async();
 #endif
   __syncwarp();
-  if (lane == 0 && r_first + VSTG <= r_last) issue(r_first + VSTG);  // row k0-1 is consumed
+  release(r_first);  // row k0-1 is consumed
   DtAcc acc;
   // rows 0 / ny+1 at a y chunk boundary are ring rows (q only, no dt): the
   // Lagrangian phase reads q on ring 1, so no q exchange is needed in y
   if ((!EDGE || j <= c.nx) && k1 > k0 && (!EDGE || k0 >= 1))
-    acc.bottom(row(k0)[VF_V * VRW], row(k0)[VF_V * VRW + 1], c);
+    acc.bottom(row(k0)[VF_V * VFS], row(k0)[VF_V * VFS + 1], c);
   const bool left = EDGE && j == 1;  // column 1: no left neighbour takes this face
   int i = idx(c, j, k0);
   // (ring slots by mask: VSTG is a power of two; rotating the row pointers
@@ -355,15 +379,15 @@ __device__ __forceinline__ bool visc_body(const Chunk& c, const CUtensorMap* __r
     const bool owned_row = !EDGE || (k >= 1 && k <= c.ny);
     if (!EDGE || j <= c.nx) {
       ViscIn I;
-      I.rho = rc[VF_R * VRW]; I.e = rc[VF_E * VRW];
+      I.rho = rc[VF_R * VFS]; I.e = rc[VF_E * VFS];
       I.pb = pcm;
-      I.pt = eos_pressure(rn[VF_R * VRW], rn[VF_E * VRW]);
-      I.pl = eos_pressure(rc[VF_R * VRW - 1], rc[VF_E * VRW - 1]);
-      I.pr = eos_pressure(rc[VF_R * VRW + 1], rc[VF_E * VRW + 1]);
-      I.u00 = rc[VF_U * VRW]; I.u10 = rc[VF_U * VRW + 1];
-      I.u01 = rn[VF_U * VRW]; I.u11 = rn[VF_U * VRW + 1];
-      I.v00 = rc[VF_V * VRW]; I.v10 = rc[VF_V * VRW + 1];
-      I.v01 = rn[VF_V * VRW]; I.v11 = rn[VF_V * VRW + 1];
+      I.pt = eos_pressure(rn[VF_R * VFS], rn[VF_E * VFS]);
+      I.pl = eos_pressure(rc[VF_R * VFS - 1], rc[VF_E * VFS - 1]);
+      I.pr = eos_pressure(rc[VF_R * VFS + 1], rc[VF_E * VFS + 1]);
+      I.u00 = rc[VF_U * VFS]; I.u10 = rc[VF_U * VFS + 1];
+      I.u01 = rn[VF_U * VFS]; I.u11 = rn[VF_U * VFS + 1];
+      I.v00 = rc[VF_V * VFS]; I.v10 = rc[VF_V * VFS + 1];
+      I.v01 = rn[VF_V * VFS]; I.v11 = rn[VF_V * VFS + 1];
       double qv, cc2, c2;
       visc_cell(dv, I, c, qv, cc2, c2);
       if (owned_row) {
@@ -379,7 +403,7 @@ __device__ __forceinline__ bool visc_body(const Chunk& c, const CUtensorMap* __r
     fence_proxy_async();
 #endif
     __syncwarp();
-    if (lane == 0 && k + VSTG <= r_last) issue(k + VSTG);
+    release(k);
   }
   __syncwarp();
   if (lane == 0)
@@ -496,9 +520,16 @@ constexpr int LKS = CLOVER_LKS;  // rows per segment
 constexpr int LSTG = CLOVER_LSTG;  // ring rows
 constexpr int LRW = 36;            // staged columns (>= 34, 16-B multiple)
 enum { LF_R, LF_E, LF_U, LF_V, LF_Q, LNF };  // = buffer order B_D0 B_E0 B_U0 B_V0 B_Q
-constexpr int LSLOT = 192;         // doubles per slot: LNF*LRW = 180 padded to 128 B
-constexpr unsigned LBYTES = LNF * LRW * 8;
-static_assert(LSLOT >= LNF * LRW && (LSLOT * 8) % 128 == 0, "slot");
+// rows per tensor copy (ring slot), as for visc_dt (VBOX): box {LRW, LBOX, 5},
+// smem slot [field][row][column]
+#ifndef CLOVER_LBOX
+#define CLOVER_LBOX 1
+#endif
+constexpr int LBOX = CLOVER_LBOX;
+constexpr int LFS = LBOX * LRW;    // field stride in a slot (doubles)
+constexpr int LSLOT = (LNF * LFS + 15) / 16 * 16;  // doubles per slot, padded to 128 B (192 at LBOX 1)
+constexpr unsigned LBYTES = LNF * LFS * 8;
+static_assert(LSLOT >= LNF * LFS && (LSLOT * 8) % 128 == 0, "slot");
 static_assert(LSTG >= 3, "ring");
 
 // EDGE = false: a warp segment whose stencil reach is at least HALO+2 away
@@ -526,29 +557,31 @@ __device__ __forceinline__ bool lagr_body(const Chunk& c, const CUtensorMap* __r
 
   const int r_first = k0 - 1, r_last = k1 + 1;  // staged rows
   const int xcol = COL0 + J0 - 2;  // = 14 + 30*gw: even, 16-B aligned (see visc_body)
-  auto slot_of = [&](int r) { return (unsigned)(r - r_first) % (unsigned)LSTG; };
+  auto slot_of = [&](int r) { return ((unsigned)(r - r_first) / (unsigned)LBOX) % (unsigned)LSTG; };
   auto issue_at = [&](unsigned sl, int r) {  // row r into slot sl
     mbar_arrive_expect_tx(&bars[sl], LBYTES);
     tma_load_3d(ring + sl * LSLOT, tm, xcol, c.row0 + r, 0, &bars[sl]);
   };
   auto issue = [&](int r) { issue_at(slot_of(r), r); };
   auto wait_row = [&](int r) {
-    const unsigned rel = (unsigned)(r - r_first);
-    mbar_wait(&bars[rel % LSTG], (rel / LSTG) & 1u);
+    const unsigned box = (unsigned)(r - r_first) / (unsigned)LBOX;
+    mbar_wait(&bars[box % LSTG], (box / LSTG) & 1u);
   };
-  auto row = [&](int r) -> const double* { return ring + slot_of(r) * LSLOT + lane + 1; };
+  auto row = [&](int r) -> const double* {
+    return ring + slot_of(r) * LSLOT + ((unsigned)(r - r_first) % (unsigned)LBOX) * LRW + lane + 1;
+  };
   // PdV predictor + EOS of the cell in row rc, node rows rc and rn (c.5)
   auto predict = [&](const double* rc, const double* rn) -> double {
-    return pdv_predict_pressure(dv, rc[LF_R * LRW], rc[LF_E * LRW], rc[LF_Q * LRW],
-                                rc[LF_U * LRW], rn[LF_U * LRW], rc[LF_U * LRW + 1],
-                                rn[LF_U * LRW + 1], rc[LF_V * LRW], rc[LF_V * LRW + 1],
-                                rn[LF_V * LRW], rn[LF_V * LRW + 1], dx, dy, c.rvol, dt);
+    return pdv_predict_pressure(dv, rc[LF_R * LFS], rc[LF_E * LFS], rc[LF_Q * LFS],
+                                rc[LF_U * LFS], rn[LF_U * LFS], rc[LF_U * LFS + 1],
+                                rn[LF_U * LFS + 1], rc[LF_V * LFS], rc[LF_V * LFS + 1],
+                                rn[LF_V * LFS], rn[LF_V * LFS + 1], dx, dy, c.rvol, dt);
   };
   if (lane == 0) {
     for (int t = 0; t < LSTG; ++t) mbar_init(&bars[t], 1);
     fence_mbar_init();
     fence_proxy_async();
-    for (int r = r_first; r < r_first + LSTG && r <= r_last; ++r) issue(r);
+    for (int r = r_first; r < r_first + LSTG * LBOX && r <= r_last; r += LBOX) issue(r);
   }
   __syncwarp();
 
@@ -568,10 +601,10 @@ __device__ __forceinline__ bool lagr_body(const Chunk& c, const CUtensorMap* __r
     } else {
       const double* a = row(kp);
       const double* b = row(kp + 1);
-      tfp = pdv_face_pred(b[LF_V * LRW], b[LF_V * LRW + 1], dx, dt);
-      ph = pdv_predict_pressure_bt(dv, a[LF_R * LRW], a[LF_E * LRW], a[LF_Q * LRW], a[LF_U * LRW],
-                                   b[LF_U * LRW], a[LF_U * LRW + 1], b[LF_U * LRW + 1],
-                                   pdv_face_pred(a[LF_V * LRW], a[LF_V * LRW + 1], dx, dt), tfp,
+      tfp = pdv_face_pred(b[LF_V * LFS], b[LF_V * LFS + 1], dx, dt);
+      ph = pdv_predict_pressure_bt(dv, a[LF_R * LFS], a[LF_E * LFS], a[LF_Q * LFS], a[LF_U * LFS],
+                                   b[LF_U * LFS], a[LF_U * LFS + 1], b[LF_U * LFS + 1],
+                                   pdv_face_pred(a[LF_V * LFS], a[LF_V * LFS + 1], dx, dt), tfp,
                                    dx, dy, c.rvol, dt);
     }
     if (xwall_warp) ph = __shfl_sync(FULL, ph, src);
@@ -584,8 +617,8 @@ __device__ __forceinline__ bool lagr_body(const Chunk& c, const CUtensorMap* __r
   double mass_m = 0.0, massl_m = 0.0, mass_c = 0.0, massl_c = 0.0;
   if constexpr (!EDGE) {
     const double* a = row(k0 - 1);
-    mass_m = a[LF_R * LRW] * vol;
-    massl_m = a[LF_R * LRW - 1] * vol;
+    mass_m = a[LF_R * LFS] * vol;
+    massl_m = a[LF_R * LFS - 1] * vol;
   }
   double u1_m = 0.0, v1_m = 0.0, u1r_m = 0.0, v1r_m = 0.0;
   // ring rows k-1, k, k+1 of the iteration, rotated at its end (one slot
@@ -596,7 +629,11 @@ __device__ __forceinline__ bool lagr_body(const Chunk& c, const CUtensorMap* __r
   unsigned wsl = 2u % (unsigned)LSTG, wph = 0u;
   unsigned isl = 0u;  // slot of row k-1, refilled at the end of iteration k
   for (int k = k0; k <= k1; ++k) {
-    mbar_wait(&bars[wsl], wph);  // row k+1
+    if constexpr (LBOX == 1) {
+      mbar_wait(&bars[wsl], wph);  // row k+1
+    } else {
+      if ((unsigned)(k + 1 - r_first) % (unsigned)LBOX == 0u) wait_row(k + 1);  // its box
+    }
     const double* rm = Pm;
     const double* rc = Pc;
     double ph = 0.0;
@@ -607,10 +644,10 @@ __device__ __forceinline__ bool lagr_body(const Chunk& c, const CUtensorMap* __r
         ph = predict(rc, Pn);
     } else {
       const double* rn = Pn;
-      const double tf = pdv_face_pred(rn[LF_V * LRW], rn[LF_V * LRW + 1], dx, dt);
-      ph = pdv_predict_pressure_bt(dv, rc[LF_R * LRW], rc[LF_E * LRW], rc[LF_Q * LRW],
-                                   rc[LF_U * LRW], rn[LF_U * LRW], rc[LF_U * LRW + 1],
-                                   rn[LF_U * LRW + 1], tfp, tf, dx, dy, c.rvol, dt);
+      const double tf = pdv_face_pred(rn[LF_V * LFS], rn[LF_V * LFS + 1], dx, dt);
+      ph = pdv_predict_pressure_bt(dv, rc[LF_R * LFS], rc[LF_E * LFS], rc[LF_Q * LFS],
+                                   rc[LF_U * LFS], rn[LF_U * LFS], rc[LF_U * LFS + 1],
+                                   rn[LF_U * LFS + 1], tfp, tf, dx, dy, c.rvol, dt);
       tfp = tf;
     }
     if (xwall_warp) ph = __shfl_sync(FULL, ph, src);
@@ -620,16 +657,16 @@ __device__ __forceinline__ bool lagr_body(const Chunk& c, const CUtensorMap* __r
     double u1_c = 0.0, v1_c = 0.0;
     if (colok) {
       const double pp[4] = {phl_m, ph_m, ph, phl};
-      const double qv[4] = {rm[LF_Q * LRW - 1], rm[LF_Q * LRW], rc[LF_Q * LRW], rc[LF_Q * LRW - 1]};
+      const double qv[4] = {rm[LF_Q * LFS - 1], rm[LF_Q * LFS], rc[LF_Q * LFS], rc[LF_Q * LFS - 1]};
       if constexpr (EDGE) {
-        const double rr[4] = {rm[LF_R * LRW - 1], rm[LF_R * LRW], rc[LF_R * LRW], rc[LF_R * LRW - 1]};
-        accelerate_node(dv, rr, pp, qv, rc[LF_U * LRW], rc[LF_V * LRW], dx, dy, dt, u1_c, v1_c);
+        const double rr[4] = {rm[LF_R * LFS - 1], rm[LF_R * LFS], rc[LF_R * LFS], rc[LF_R * LFS - 1]};
+        accelerate_node(dv, rr, pp, qv, rc[LF_U * LFS], rc[LF_V * LFS], dx, dy, dt, u1_c, v1_c);
       } else {
         // cell masses of row k; those of row k-1 are carried from the last row
-        mass_c = rc[LF_R * LRW] * vol;
-        massl_c = rc[LF_R * LRW - 1] * vol;
+        mass_c = rc[LF_R * LFS] * vol;
+        massl_c = rc[LF_R * LFS - 1] * vol;
         const double mm[4] = {massl_m, mass_m, mass_c, massl_c};
-        accelerate_node_m(dv, mm, pp, qv, rc[LF_U * LRW], rc[LF_V * LRW], dx, dy, dt, u1_c, v1_c);
+        accelerate_node_m(dv, mm, pp, qv, rc[LF_U * LFS], rc[LF_V * LFS], dx, dy, dt, u1_c, v1_c);
       }
     }
     const double u1r_c = __shfl_down_sync(FULL, u1_c, 1);
@@ -640,18 +677,18 @@ __device__ __forceinline__ bool lagr_body(const Chunk& c, const CUtensorMap* __r
     double tsum_c = 0.0, tfc_c = 0.0;
     if constexpr (!EDGE) {
       // top face of cell row k-1 = bottom face of row k (carried to k+1)
-      tsum_c = rc[LF_V * LRW] + rc[LF_V * LRW + 1] + v1_c + v1r_c;
+      tsum_c = rc[LF_V * LFS] + rc[LF_V * LFS + 1] + v1_c + v1r_c;
       tfc_c = pdv_face_corr(tsum_c, dx, dt);
     }
     if (kc >= k0 && lane >= 1 && lane <= LW && (!EDGE || j <= c.nx)) {
-      const double u0_m = rm[LF_U * LRW], u0r_m = rm[LF_U * LRW + 1];
-      const double u0_c = rc[LF_U * LRW], u0r_c = rc[LF_U * LRW + 1];
+      const double u0_m = rm[LF_U * LFS], u0r_m = rm[LF_U * LFS + 1];
+      const double u0_c = rc[LF_U * LFS], u0r_c = rc[LF_U * LFS + 1];
       const double lsum = u0_m + u0_c + u1_m + u1_c;
       const double rsum = u0r_m + u0r_c + u1r_m + u1r_c;
       double bsum, tsum, bfc, tfc;
       if constexpr (EDGE) {
-        const double v0_m = rm[LF_V * LRW], v0r_m = rm[LF_V * LRW + 1];
-        const double v0_c = rc[LF_V * LRW], v0r_c = rc[LF_V * LRW + 1];
+        const double v0_m = rm[LF_V * LFS], v0r_m = rm[LF_V * LFS + 1];
+        const double v0_c = rc[LF_V * LFS], v0r_c = rc[LF_V * LFS + 1];
         bsum = v0_m + v0r_m + v1_m + v1r_m;
         tsum = v0_c + v0r_c + v1_c + v1r_c;
         bfc = pdv_face_corr(bsum, dx, dt);
@@ -661,7 +698,7 @@ __device__ __forceinline__ bool lagr_body(const Chunk& c, const CUtensorMap* __r
         bfc = tfc_m; tfc = tfc_c;
       }
       double ev, dvv;
-      pdv_correct_bt(dv, rm[LF_R * LRW], rm[LF_E * LRW], ph_m, rm[LF_Q * LRW], lsum, rsum, bfc, tfc,
+      pdv_correct_bt(dv, rm[LF_R * LFS], rm[LF_E * LFS], ph_m, rm[LF_Q * LFS], lsum, rsum, bfc, tfc,
                      dx, dy, c.rvol, dt, ev, dvv);
       const int ic = idx(c, j, kc);
       const double cx = 0.25 * dt * dy, cy = 0.25 * dt * dx;
@@ -707,11 +744,20 @@ __device__ __forceinline__ bool lagr_body(const Chunk& c, const CUtensorMap* __r
     fence_proxy_async();
 #endif
     __syncwarp();
-    if (lane == 0 && k - 1 + LSTG <= r_last) issue_at(isl, k - 1 + LSTG);
-    if (++isl == (unsigned)LSTG) isl = 0u;
-    Pm = Pc; Pc = Pn;
-    if (++wsl == (unsigned)LSTG) { wsl = 0u; wph ^= 1u; }
-    Pn = ring + wsl * LSLOT + lane + 1;
+    if constexpr (LBOX == 1) {
+      if (lane == 0 && k - 1 + LSTG <= r_last) issue_at(isl, k - 1 + LSTG);
+      if (++isl == (unsigned)LSTG) isl = 0u;
+      Pm = Pc; Pc = Pn;
+      if (++wsl == (unsigned)LSTG) { wsl = 0u; wph ^= 1u; }
+      Pn = ring + wsl * LSLOT + lane + 1;
+    } else {
+      // row k-1 ends its box: refill the slot with the box LSTG boxes on
+      if ((unsigned)(k - 1 - r_first) % (unsigned)LBOX == (unsigned)(LBOX - 1) && lane == 0 &&
+          k + (LSTG - 1) * LBOX <= r_last)
+        issue(k + (LSTG - 1) * LBOX);
+      Pm = Pc; Pc = Pn;
+      Pn = row(k + 2);
+    }
   }
   __syncwarp();
   if (lane == 0)
