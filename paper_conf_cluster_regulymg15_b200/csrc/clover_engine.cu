@@ -106,7 +106,8 @@ struct ChunkState {
   FixSlot fix_b;     // the same for boundary segments running beside the interior (run_phase)
   CUtensorMap tm_lag;   // d0 e0 u0 v0 q as one {pitch, rows, 5} fp64 tensor, box {LRW, 1, 5}
   CUtensorMap tm_visc;  // d0 e0 u0 v0 as {pitch, rows, 4}, box {VRW, 1, 4}
-  CUtensorMap tm_x1;    // d1 e1 u1 v1 fy fx, box {XRW, 1, 6} (fused x sweep 1)
+  CUtensorMap tm_x1;    // d1 e1 u1 v1 fy fx, box {XRW, 1, 6} (fused y sweep 1)
+  CUtensorMap tm_x1x;   // the same tensor, box {XRW, XBOX, 6} (fused x sweep 1)
   CUtensorMap tm_x2;    // fx d2 e2 u2 v2, box {XRW, 1, 5} (fused x sweep 2)
   CUtensorMap tm_fy;    // fy, box {YRW, 1, 1} (fused y sweep 2)
   CUtensorMap tm_c4;    // d2 e2 u2 v2, box {YRW, 1, 4} (fused y sweep 2)
@@ -1311,7 +1312,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
           c = with_rev(c, serp);
           const dim3 g(grid_strip(c.nx + 1, XW, c.ny + 1, c.xks).x, n);
           if (sweep == 1)
-            launch_step(ks_advec_x<1>, g, SB, sm, c, cs.tm_x1, cs.buf[rout], cs.buf[eout],
+            launch_step(ks_advec_x<1>, g, SB, sm, c, cs.tm_x1x, cs.buf[rout], cs.buf[eout],
                         cs.buf[uout], cs.buf[vout], fx);
           else
             launch_step(ks_advec_x<2>, g, SB, sm, c, cs.tm_x2, cs.buf[rout], cs.buf[eout],
@@ -1323,7 +1324,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
           c = with_rev(c, serp);
           if (sweep == 1) {
             const YWalls yw = walls_in_x1 ? ywalls_of(cs, 2) : kNoWalls;
-            launch_fix(kf_advec_x<1>, FIX_BLOCKS + 5 * yw.nbx, SB, sm, c, cs.tm_x1, cs.buf[rout],
+            launch_fix(kf_advec_x<1>, FIX_BLOCKS + 5 * yw.nbx, SB, sm, c, cs.tm_x1x, cs.buf[rout],
                         cs.buf[eout], cs.buf[uout], cs.buf[vout], fx, yw);
           } else {
             launch_fix(kf_advec_x<2>, FIX_BLOCKS, SB, sm, c, cs.tm_x2, cs.buf[rout], cs.buf[eout],
@@ -1337,7 +1338,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
           dim3 g(1, 1, (unsigned)vs.size());
           for (size_t t = 0; t < vs.size(); ++t) {
             const ChunkState& v = vs[t];
-            xb.a[t] = XArgs{v.c, sweep == 1 ? v.tm_x1 : v.tm_x2, v.buf[rout], v.buf[eout],
+            xb.a[t] = XArgs{v.c, sweep == 1 ? v.tm_x1x : v.tm_x2, v.buf[rout], v.buf[eout],
                             v.buf[uout], v.buf[vout], v.fix};
             g.x = std::max(g.x, grid_strip(v.c.nx + 1, XW, v.c.ny + 1, v.c.xks).x);
             g.y = std::max<unsigned>(g.y, (unsigned)seg_count_lay(v.c.xks, v.c.xnb, v.c.xch, v.c.xcf, v.c.ny + 1));
@@ -1956,8 +1957,10 @@ int clover_init(const clover_grid* grid, const clover_state* states, int32_t nst
       if (!rc) rc = encode_rows_map(&cs.tm_visc, base, c.pitch, rows, fs, VNF, VRW, VBOX);
       if (!rc) rc = encode_rows_map(&cs.tm_x1, base + (B_D1 - B_D0) * (fs / 8), c.pitch, rows, fs,
                                     XF<1>::NF, XRW);
+      if (!rc) rc = encode_rows_map(&cs.tm_x1x, base + (B_D1 - B_D0) * (fs / 8), c.pitch, rows, fs,
+                                    XF<1>::NF, XRW, XBOX);
       if (!rc) rc = encode_rows_map(&cs.tm_x2, base + (B_FX - B_D0) * (fs / 8), c.pitch, rows, fs,
-                                    XF<2>::NF, XRW);
+                                    XF<2>::NF, XRW, XBOX);
       if (!rc) rc = encode_rows_map(&cs.tm_fy, base + (B_FY - B_D0) * (fs / 8), c.pitch, rows, fs,
                                     1, YRW);
       if (!rc) rc = encode_rows_map(&cs.tm_c4, base + (B_D2 - B_D0) * (fs / 8), c.pitch, rows, fs,

@@ -33,10 +33,11 @@ constexpr int SB = CLOVER_SB;  // threads per block (one warp: a block slot free
                                // warp's segment is done; measured faster than 2-warp blocks for the
                                // Lagrangian and both sweeps)
 #ifndef CLOVER_SBV
-#define CLOVER_SBV 64
+#define CLOVER_SBV 32
 #endif
-constexpr int SBV = CLOVER_SBV;  // visc_dt threads per block (its streaming-only bm segments are
-                                 // short: 1-warp blocks cost more in block launches than they save)
+constexpr int SBV = CLOVER_SBV;  // visc_dt threads per block (64 was faster on the bm window with
+                                 // 1-row ring slots; with 4-row slots 32 is as fast there and 5 %
+                                 // faster on active flow: profiles/r2_sbv_box_ab.jsonl)
 
 // Tunables (defaults = measured best; scripts/ab_variants.py builds others).
 #define CLOVER_STR2(x) #x
@@ -1172,8 +1173,14 @@ constexpr int XRW = 36;
 #define CLOVER_XSTG 4
 #endif
 constexpr int XSTG = CLOVER_XSTG;
+// rows per tensor copy (ring slot), as for visc_dt (VBOX); slot [field][row][column]
+#ifndef CLOVER_XBOX
+#define CLOVER_XBOX 1
+#endif
+constexpr int XBOX = CLOVER_XBOX;
+constexpr int XFS = XBOX * XRW;  // field stride in a slot (doubles)
 template <int SWEEP>
-__host__ __device__ constexpr int xslot() { return (XF<SWEEP>::NF * XRW + 15) / 16 * 16; }  // 128-B multiple
+__host__ __device__ constexpr int xslot() { return (XF<SWEEP>::NF * XFS + 15) / 16 * 16; }  // 128-B multiple
 static_assert((COL0 + 1 - 4) % 2 == 0 && XW % 2 == 0, "fused x ring box starts on an even column");
 
 // EDGE = false: a warp segment whose columns and rows are all at least
@@ -1188,7 +1195,7 @@ __device__ __forceinline__ bool advec_x_body(const Chunk& c, const CUtensorMap* 
                                              int lane, double* ring, unsigned long long* bars) {
   using F = XF<SWEEP>;
   constexpr int SL = xslot<SWEEP>();
-  constexpr unsigned BYTES = F::NF * XRW * 8;
+  constexpr unsigned BYTES = F::NF * XFS * 8;
   D dv;
   const int J0 = 1 + XW * gw;
   if (J0 > c.nx + 1) return false;
@@ -1218,27 +1225,29 @@ __device__ __forceinline__ bool advec_x_body(const Chunk& c, const CUtensorMap* 
 
   const int r_first = k0 - 1, r_last = k1;  // staged rows (fy of row r+1 is read at row r)
   const int xcol = COL0 + J0 - 4;
-  auto slot_of = [&](int r) { return (unsigned)(r - r_first) % (unsigned)XSTG; };
+  auto slot_of = [&](int r) { return ((unsigned)(r - r_first) / (unsigned)XBOX) % (unsigned)XSTG; };
   auto issue = [&](int r) {
     const unsigned sl = slot_of(r);
     mbar_arrive_expect_tx(&bars[sl], BYTES);
     tma_load_3d(ring + sl * SL, tm, xcol, c.row0 + r, 0, &bars[sl]);
   };
   auto wait_row = [&](int r) {
-    const unsigned rel = (unsigned)(r - r_first);
-    mbar_wait(&bars[rel % XSTG], (rel / XSTG) & 1u);
+    const unsigned box = (unsigned)(r - r_first) / (unsigned)XBOX;
+    mbar_wait(&bars[box % XSTG], (box / XSTG) & 1u);
   };
-  auto row = [&](int r) -> const double* { return ring + slot_of(r) * SL + lane + 2; };
+  auto row = [&](int r) -> const double* {
+    return ring + slot_of(r) * SL + ((unsigned)(r - r_first) % (unsigned)XBOX) * XRW + lane + 2;
+  };
   // post-sweep cell volume of the node-mass term
   auto pv_mom = [&](const double* rc, const double* rn) -> double {
-    if constexpr (SWEEP == 1) return vol + rn[F::FY * XRW] - rc[F::FY * XRW];
+    if constexpr (SWEEP == 1) return vol + rn[F::FY * XFS] - rc[F::FY * XFS];
     else return vol;
   };
   if (lane == 0) {
     for (int t = 0; t < XSTG; ++t) mbar_init(&bars[t], 1);
     fence_mbar_init();
     fence_proxy_async();
-    for (int r = r_first; r < r_first + XSTG && r <= r_last; ++r) issue(r);
+    for (int r = r_first; r < r_first + XSTG * XBOX && r <= r_last; r += XBOX) issue(r);
   }
   __syncwarp();
   wait_row(r_first);
@@ -1263,13 +1272,13 @@ __device__ __forceinline__ bool advec_x_body(const Chunk& c, const CUtensorMap* 
         // ---- advec_cell x, row r
         double pv = 0.0, F = 0.0, m = 0.0, ef = 0.0, rr = 0.0, ee = 0.0, flo = 0.0, fhi = 0.0;
         if (cellok) {
-          flo = rc[F::FX * XRW]; fhi = rc[F::FX * XRW + 1];
+          flo = rc[F::FX * XFS]; fhi = rc[F::FX * XFS + 1];
           F = flo;
           if constexpr (SWEEP == 1)
-            pv = vol + (fhi - flo + rn[F::FY * XRW] - rc[F::FY * XRW]);
+            pv = vol + (fhi - flo + rn[F::FY * XFS] - rc[F::FY * XFS]);
           else
             pv = vol + fhi - flo;
-          rr = rc[F::R * XRW]; ee = rc[F::E * XRW];
+          rr = rc[F::R * XFS]; ee = rc[F::E * XFS];
         }
         if (faceok) {
           // pre_vol of cell j-1 from the ring (the same expression lane j-1
@@ -1277,9 +1286,9 @@ __device__ __forceinline__ bool advec_x_body(const Chunk& c, const CUtensorMap* 
           // divergent lane-0 path)
           double pvl;
           {
-            const double fl = rc[F::FX * XRW - 1];
+            const double fl = rc[F::FX * XFS - 1];
             if constexpr (SWEEP == 1)
-              pvl = vol + (flo - fl + rn[F::FY * XRW - 1] - rc[F::FY * XRW - 1]);
+              pvl = vol + (flo - fl + rn[F::FY * XFS - 1] - rc[F::FY * XFS - 1]);
             else
               pvl = vol + flo - fl;
           }
@@ -1290,8 +1299,8 @@ __device__ __forceinline__ bool advec_x_body(const Chunk& c, const CUtensorMap* 
           const double* pu = pos ? rc - 2 : rc + ((EDGE && c.wr) ? min(j + 1, nx + 2) - j : 1);
           const double* pd = pos ? rc - 1 : rc;
           const double* pw = pos ? rc : rc - 1;
-          cell_face_flux(dv, F, pos ? pvl : pv, pu[F::R * XRW], pd[F::R * XRW], pw[F::R * XRW],
-                         pu[F::E * XRW], pd[F::E * XRW], pw[F::E * XRW], m, ef);
+          cell_face_flux(dv, F, pos ? pvl : pv, pu[F::R * XFS], pd[F::R * XFS], pw[F::R * XFS],
+                         pu[F::E * XFS], pd[F::E * XFS], pw[F::E * XFS], m, ef);
         }
         const double mh = __shfl_down_sync(FULL, m, 1);
         const double efh = __shfl_down_sync(FULL, ef, 1);
@@ -1338,14 +1347,14 @@ __device__ __forceinline__ bool advec_x_body(const Chunk& c, const CUtensorMap* 
           } else {
             up = -1; don = 0; dw = 1; nmp = pre;
           }
-          const double uu[3] = {rc[F::U * XRW + up], rc[F::U * XRW + don], rc[F::U * XRW + dw]};
-          const double vv[3] = {rc[F::V * XRW + up], rc[F::V * XRW + don], rc[F::V * XRW + dw]};
+          const double uu[3] = {rc[F::U * XFS + up], rc[F::U * XFS + don], rc[F::U * XFS + dw]};
+          const double vv[3] = {rc[F::V * XFS + up], rc[F::V * XFS + don], rc[F::V * XFS + dw]};
           mom_flux2(dv, nf, nmp, uu, vv, c.dx, c.rdx, mu, mv);
         }
         const double mul = __shfl_up_sync(FULL, mu, 1);
         const double mvl = __shfl_up_sync(FULL, mv, 1);
         if (own && (!EDGE || (j >= 1 && j <= nx + 1))) {
-          const double u = rc[F::U * XRW], v = rc[F::V * XRW];
+          const double u = rc[F::U * XFS], v = rc[F::V * XFS];
           double un, vn;
           mom_update(dv, u, v, pre, post, mul, mu, mvl, mv, un, vn);
           const bool near = EDGE && (ncol || near_wall_row(c, r));
@@ -1361,7 +1370,13 @@ __device__ __forceinline__ bool advec_x_body(const Chunk& c, const CUtensorMap* 
       fence_proxy_async();
 #endif
       __syncwarp();
-      if (lane == 0 && r - 1 + XSTG <= r_last) issue(r - 1 + XSTG);
+      if constexpr (XBOX == 1) {
+        if (lane == 0 && r - 1 + XSTG <= r_last) issue(r - 1 + XSTG);
+      } else {  // row r-1 ends its box: refill the slot with the box XSTG boxes on
+        if ((unsigned)(r - 1 - r_first) % (unsigned)XBOX == (unsigned)(XBOX - 1) && lane == 0 &&
+            r + (XSTG - 1) * XBOX <= r_last)
+          issue(r + (XSTG - 1) * XBOX);
+      }
     }
   }
   __syncwarp();
