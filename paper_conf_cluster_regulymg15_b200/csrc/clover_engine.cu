@@ -111,6 +111,7 @@ struct ChunkState {
   CUtensorMap tm_x2;    // fx d2 e2 u2 v2, box {XRW, 1, 5} (fused x sweep 2)
   CUtensorMap tm_fy;    // fy, box {YRW, 1, 1} (fused y sweep 2)
   CUtensorMap tm_c4;    // d2 e2 u2 v2, box {YRW, 1, 4} (fused y sweep 2)
+  CUtensorMap tm_y2;    // fy fx d2 e2 u2 v2, box {YRW, 1, 6} (fused y sweep 2, CLOVER_Y2ONE)
 };
 
 struct Layout {
@@ -1387,8 +1388,8 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
         auto launch = [&](ChunkState& cs, Chunk c, int n, cudaStream_t sm, FixSlot fx) -> int {
           c = with_rev(c, serp);
           const dim3 g(grid_strip(c.nx + 1, YW, c.ny + 1, c.yks).x, n);
-          const CUtensorMap& ta = sweep == 1 ? cs.tm_x1 : cs.tm_fy;
-          const CUtensorMap& tb = sweep == 1 ? cs.tm_x1 : cs.tm_c4;
+          const CUtensorMap& ta = sweep == 1 ? cs.tm_x1 : (CLOVER_Y2ONE ? cs.tm_y2 : cs.tm_fy);
+          const CUtensorMap& tb = sweep == 1 ? cs.tm_x1 : (CLOVER_Y2ONE ? cs.tm_y2 : cs.tm_c4);
           if (sweep == 1) {
             launch_step(ks_advec_y<1>, g, SB, sm, c, ta, tb, cs.buf[rout], cs.buf[eout], cs.buf[B_MY],
                         cs.buf[uout], cs.buf[vout], fx);
@@ -1401,8 +1402,8 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
         };
         auto fixup = [&](ChunkState& cs, Chunk c, cudaStream_t sm, FixSlot fx) -> int {
           c = with_rev(c, serp);
-          const CUtensorMap& ta = sweep == 1 ? cs.tm_x1 : cs.tm_fy;
-          const CUtensorMap& tb = sweep == 1 ? cs.tm_x1 : cs.tm_c4;
+          const CUtensorMap& ta = sweep == 1 ? cs.tm_x1 : (CLOVER_Y2ONE ? cs.tm_y2 : cs.tm_fy);
+          const CUtensorMap& tb = sweep == 1 ? cs.tm_x1 : (CLOVER_Y2ONE ? cs.tm_y2 : cs.tm_c4);
           if (sweep == 1)
             launch_fix(kf_advec_y<1>, FIX_BLOCKS, SB, sm, c, ta, tb, cs.buf[rout], cs.buf[eout],
                         cs.buf[B_MY], cs.buf[uout], cs.buf[vout], fx);
@@ -1420,7 +1421,8 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
           dim3 g(1, 1, (unsigned)vs.size());
           for (size_t t = 0; t < vs.size(); ++t) {
             const ChunkState& v = vs[t];
-            yb.a[t] = YArgs{v.c, sweep == 1 ? v.tm_x1 : v.tm_fy, sweep == 1 ? v.tm_x1 : v.tm_c4,
+            yb.a[t] = YArgs{v.c, sweep == 1 ? v.tm_x1 : (CLOVER_Y2ONE ? v.tm_y2 : v.tm_fy),
+                            sweep == 1 ? v.tm_x1 : (CLOVER_Y2ONE ? v.tm_y2 : v.tm_c4),
                             v.buf[rout], v.buf[eout], v.buf[B_MY], v.buf[uout], v.buf[vout],
                             v.fix};
             g.x = std::max(g.x, grid_strip(v.c.nx + 1, YW, v.c.ny + 1, v.c.yks).x);
@@ -1965,6 +1967,8 @@ int clover_init(const clover_grid* grid, const clover_state* states, int32_t nst
                                     1, YRW);
       if (!rc) rc = encode_rows_map(&cs.tm_c4, base + (B_D2 - B_D0) * (fs / 8), c.pitch, rows, fs,
                                     4, YRW);
+      if (!rc) rc = encode_rows_map(&cs.tm_y2, base + (B_FY - B_D0) * (fs / 8), c.pitch, rows, fs,
+                                    6, YRW);
       if (rc) return bail(rc);
     }
     cs.ntx = (c.nx + ST - 1) / ST; cs.nty = (c.ny + ST - 1) / ST;

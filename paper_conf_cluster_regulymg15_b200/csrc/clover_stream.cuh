@@ -1615,13 +1615,30 @@ template <> struct YL<1> {  // tensor d1 e1 u1 v1 fy fx
   enum { R = 0, E = YRW, U = 2 * YRW, V = 3 * YRW, FY = 4 * YRW, FX = 5 * YRW, B = 0,
          SLOT = (6 * YRW + 15) / 16 * 16 };
   static constexpr unsigned BYTES = 6 * YRW * 8;
+  static constexpr bool TWO = false;
 };
+// CLOVER_Y2ONE: sweep 2 reads fy fx d2 e2 u2 v2 as one tensor copy per row
+// (fx is not used: one copy instead of two for 20 % more bytes)
+#ifndef CLOVER_Y2ONE
+#define CLOVER_Y2ONE 0
+#endif
+#if CLOVER_Y2ONE
+template <> struct YL<2> {  // tensor fy fx d2 e2 u2 v2
+  static constexpr int RING = CLOVER_YRING2, MINB = 0;
+  enum { FY = 0, FX = YRW, B = 0, R = 2 * YRW, E = 3 * YRW, U = 4 * YRW, V = 5 * YRW,
+         SLOT = (6 * YRW + 15) / 16 * 16 };
+  static constexpr unsigned BYTES = 6 * YRW * 8;
+  static constexpr bool TWO = false;
+};
+#else
 template <> struct YL<2> {  // tensors fy | d2 e2 u2 v2
   static constexpr int RING = CLOVER_YRING2, MINB = 0;  // 0: no cap
   enum { FY = 0, B = (YRW + 15) / 16 * 16, R = B, E = B + YRW, U = B + 2 * YRW, V = B + 3 * YRW,
          FX = -1, SLOT = (B + 4 * YRW + 15) / 16 * 16 };
   static constexpr unsigned BYTES = 5 * YRW * 8;
+  static constexpr bool TWO = true;
 };
+#endif
 
 template <int SWEEP, class D, bool EDGE>
 __device__ __forceinline__ bool advec_y_body(const Chunk& c, const CUtensorMap* __restrict__ ta,
@@ -1667,17 +1684,17 @@ __device__ __forceinline__ bool advec_y_body(const Chunk& c, const CUtensorMap* 
 #if CLOVER_L2HINT
     if (r <= k0 + 2) {
       tma_load_3d_hint(d, ta, xcol, c.row0 + r, 0, &bars[sl], pol_keep);
-      if constexpr (SWEEP == 2) tma_load_3d_hint(d + L::B, tb, xcol, c.row0 + r, 0, &bars[sl], pol_keep);
+      if constexpr (SWEEP == 2 && L::TWO) tma_load_3d_hint(d + L::B, tb, xcol, c.row0 + r, 0, &bars[sl], pol_keep);
       return;
     }
 #if CLOVER_L2HINT > 1
     tma_load_3d_hint(d, ta, xcol, c.row0 + r, 0, &bars[sl], pol_once);
-    if constexpr (SWEEP == 2) tma_load_3d_hint(d + L::B, tb, xcol, c.row0 + r, 0, &bars[sl], pol_once);
+    if constexpr (SWEEP == 2 && L::TWO) tma_load_3d_hint(d + L::B, tb, xcol, c.row0 + r, 0, &bars[sl], pol_once);
     return;
 #endif
 #endif
     tma_load_3d(d, ta, xcol, c.row0 + r, 0, &bars[sl]);
-    if constexpr (SWEEP == 2) tma_load_3d(d + L::B, tb, xcol, c.row0 + r, 0, &bars[sl]);
+    if constexpr (SWEEP == 2 && L::TWO) tma_load_3d(d + L::B, tb, xcol, c.row0 + r, 0, &bars[sl]);
   };
   auto issue = [&](int r) { issue_at((unsigned)(r - r_first) % (unsigned)L::RING, r); };
   auto row = [&](int r) -> const double* {
