@@ -162,7 +162,7 @@ dim3 grid_strip(int ncols, int width, int nrows, int ks) {
 // bounds the step there.  Never below MIN_KS (fix-list capacity).
 constexpr int MIN_KS = 8;
 #ifndef CLOVER_SEG_FILL
-#define CLOVER_SEG_FILL 8
+#define CLOVER_SEG_FILL (8 * 64 / CLOVER_SB)  // blocks per SM: 16 warps/SM, as tuned on 2-warp blocks
 #endif
 int seg_rows(int ks, int64_t colblocks, int nrows) {
   while (ks > MIN_KS && colblocks * cdiv(nrows, ks) < 148 * CLOVER_SEG_FILL) ks /= 2;
