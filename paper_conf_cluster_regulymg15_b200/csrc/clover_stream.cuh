@@ -155,11 +155,13 @@ __device__ __forceinline__ void fix_push(FixSlot f, int lane, unsigned gw, unsig
 struct NoLast {
   __device__ void operator()() const {}
 };
-// Fixup blocks (one warp each since the blocks have one warp: three per SM;
+// Fixup blocks (one warp each since the blocks have one warp: six per SM;
 // 148 -> 444 warps redo the flagged rows, bm 3840^2 step 0.858 -> 0.847 ms,
-// profiles/r2_fixblocks_ab.jsonl); a launch may add y-wall blocks.
+// profiles/r2_fixblocks_ab.jsonl; 888 for the late steps, where 25-76
+// segments a step are flagged: 300-step run 0.871 -> 0.868 ms,
+// profiles/r2_fixblocks_full_ab.txt); a launch may add y-wall blocks.
 #ifndef CLOVER_FIX_BLOCKS
-#define CLOVER_FIX_BLOCKS 444
+#define CLOVER_FIX_BLOCKS 888
 #endif
 constexpr int FIX_BLOCKS = CLOVER_FIX_BLOCKS;
 template <int BS = SB, class Run, class Last = NoLast>
