@@ -1597,12 +1597,14 @@ constexpr int YKS = CLOVER_YKS;
 // sweep 2 (5 fields) at 7 rows uncapped (10 blocks/SM) -- measured best
 // after the ring-pointer rotation (round 2, same box, 3 repeats: step
 // 0.8737 -> 0.8693 ms against 6/10 and 8/uncapped; round 1's best were 6
-// and 8 rows).
+// and 8 rows).  On one-warp blocks sweep 2 takes 6 rows (24 warps/SM by
+// shared memory instead of 21; y sweep 2 0.2464 -> 0.2444 ms on the bm
+// window, 0.328 -> 0.320 on active flow: profiles/r2_yring2_ab.jsonl).
 #ifndef CLOVER_YRING1
 #define CLOVER_YRING1 7
 #endif
 #ifndef CLOVER_YRING2
-#define CLOVER_YRING2 7
+#define CLOVER_YRING2 6
 #endif
 #ifndef CLOVER_YMINB1  // (18 one-warp blocks: 94 registers; uncapped it takes 106, 2 % slower)
 #define CLOVER_YMINB1 (9 * 64 / CLOVER_SB)
