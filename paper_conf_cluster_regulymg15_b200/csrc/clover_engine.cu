@@ -182,11 +182,11 @@ int seg_rows(int ks, int64_t colblocks, int nrows) {
 #ifndef CLOVER_TAIL_WAVES
 #define CLOVER_TAIL_WAVES 2
 #endif
-int tail_nb(int ks, int64_t colblocks, int rows, int64_t slots) {
-  if (!CLOVER_TAIL || ks < 4 * CLOVER_TAIL_DIV || slots <= 0) return 0x3fffffff;
+int tail_nb(int ks, int64_t colblocks, int rows, int64_t slots, int td = CLOVER_TAIL_DIV) {
+  if (!CLOVER_TAIL || ks < 4 * td || slots <= 0) return 0x3fffffff;
   const int64_t tail_rows = (int64_t)CLOVER_TAIL_WAVES *
                             cdiv((int)std::min<int64_t>(slots, 1 << 30), (int)colblocks) *
-                            (int64_t)(ks / CLOVER_TAIL_DIV);
+                            (int64_t)(ks / td);
   if (rows <= tail_rows) return 0;
   return (int)((rows - tail_rows) / ks);
 }
@@ -999,33 +999,57 @@ bool batch_ok(const clover_ctx* ctx) {
 #ifndef CLOVER_CHAIN
 #define CLOVER_CHAIN 1
 #endif
+// Tail segments per kernel: ks / td rows (visc_dt, Lagrangian, x sweep,
+// y sweep).  Quarter-height tails measured faster for visc_dt and the x
+// sweeps, half-height for the Lagrangian and the y sweeps.
+#ifndef CLOVER_TD_V
+#define CLOVER_TD_V 4
+#endif
+#ifndef CLOVER_TD_L
+#define CLOVER_TD_L 2
+#endif
+#ifndef CLOVER_TD_X
+#define CLOVER_TD_X 4
+#endif
+#ifndef CLOVER_TD_Y
+#define CLOVER_TD_Y 2
+#endif
 #ifndef CLOVER_CHAIN_ADJ
 #define CLOVER_CHAIN_ADJ 0
 #endif
-void band_layout(bool on, int ks, int64_t colblocks, int rows, int64_t slots, int* ch, int* cf) {
+void band_layout(bool on, int ks, int64_t colblocks, int rows, int64_t slots, int* ch, int* cf,
+                 int td) {
   *ch = 0;
   *cf = 0;
-  if (!on || !CLOVER_TAIL || ks < 4 * CLOVER_TAIL_DIV || colblocks <= 0 || slots <= 0) return;
+  if (!on || !CLOVER_TAIL || ks < 4 * td || colblocks <= 0 || slots <= 0) return;
   const int64_t C = (slots + colblocks - 1) / colblocks + CLOVER_CHAIN_ADJ;
   if (C < 2 || C > rows) return;
-  band_params(ks, (int)C, rows, ch, cf);
+  band_params(ks, (int)C, rows, ch, cf, td);
 }
 
 void set_segs(Chunk& c, int nsm, const int occ[4], bool chain) {
+  c.vtd = CLOVER_TD_V; c.ltd = CLOVER_TD_L; c.xtd = CLOVER_TD_X; c.ytd = CLOVER_TD_Y;
   c.vks = seg_rows(VKS, grid_cols_v(c.nx, c.ny, VKS).x, c.ny);
   c.lks = seg_rows(LKS, grid_strip(c.nx, LW, c.ny, LKS).x, c.ny);
   c.xks = seg_rows(XKS, grid_strip(c.nx + 1, XW, c.ny + 1, XKS).x, c.ny + 1);
   c.yks = seg_rows(YKS, grid_strip(c.nx + 1, YW, c.ny + 1, YKS).x, c.ny + 1);
-  c.vnb = tail_nb(c.vks, grid_cols_v(c.nx, c.ny, c.vks).x, c.ny, (int64_t)nsm * occ[0]);
-  c.lnb = tail_nb(c.lks, grid_strip(c.nx, LW, c.ny, c.lks).x, c.ny, (int64_t)nsm * occ[1]);
-  c.xnb = tail_nb(c.xks, grid_strip(c.nx + 1, XW, c.ny + 1, c.xks).x, c.ny + 1, (int64_t)nsm * occ[2]);
-  c.ynb = tail_nb(c.yks, grid_strip(c.nx + 1, YW, c.ny + 1, c.yks).x, c.ny + 1, (int64_t)nsm * occ[3]);
-  band_layout(chain, c.vks, grid_cols_v(c.nx, c.ny, c.vks).x, c.ny, (int64_t)nsm * occ[0], &c.vch, &c.vcf);
-  band_layout(chain, c.lks, grid_strip(c.nx, LW, c.ny, c.lks).x, c.ny, (int64_t)nsm * occ[1], &c.lch, &c.lcf);
+  // (short segments on small meshes: keep tail segments >= 4 rows)
+  if (c.vks < 4 * c.vtd) c.vtd = CLOVER_TAIL_DIV;
+  if (c.lks < 4 * c.ltd) c.ltd = CLOVER_TAIL_DIV;
+  if (c.xks < 4 * c.xtd) c.xtd = CLOVER_TAIL_DIV;
+  if (c.yks < 4 * c.ytd) c.ytd = CLOVER_TAIL_DIV;
+  c.vnb = tail_nb(c.vks, grid_cols_v(c.nx, c.ny, c.vks).x, c.ny, (int64_t)nsm * occ[0], c.vtd);
+  c.lnb = tail_nb(c.lks, grid_strip(c.nx, LW, c.ny, c.lks).x, c.ny, (int64_t)nsm * occ[1], c.ltd);
+  c.xnb = tail_nb(c.xks, grid_strip(c.nx + 1, XW, c.ny + 1, c.xks).x, c.ny + 1, (int64_t)nsm * occ[2], c.xtd);
+  c.ynb = tail_nb(c.yks, grid_strip(c.nx + 1, YW, c.ny + 1, c.yks).x, c.ny + 1, (int64_t)nsm * occ[3], c.ytd);
+  band_layout(chain, c.vks, grid_cols_v(c.nx, c.ny, c.vks).x, c.ny, (int64_t)nsm * occ[0], &c.vch, &c.vcf,
+              c.vtd);
+  band_layout(chain, c.lks, grid_strip(c.nx, LW, c.ny, c.lks).x, c.ny, (int64_t)nsm * occ[1], &c.lch, &c.lcf,
+              c.ltd);
   band_layout(chain, c.xks, grid_strip(c.nx + 1, XW, c.ny + 1, c.xks).x, c.ny + 1, (int64_t)nsm * occ[2],
-              &c.xch, &c.xcf);
+              &c.xch, &c.xcf, c.xtd);
   band_layout(chain, c.yks, grid_strip(c.nx + 1, YW, c.ny + 1, c.yks).x, c.ny + 1, (int64_t)nsm * occ[3],
-              &c.ych, &c.ycf);
+              &c.ych, &c.ycf, c.ytd);
 }
 
 // The chunk seen from `e` rows beyond each of its non-wall y sides: rows
@@ -1046,27 +1070,27 @@ ChunkState deep_view(const clover_ctx* ctx, const ChunkState& cs, int e) {
 // Row-segment geometry of a streaming kernel kind on a chunk: rows per
 // segment, full-height segments, rows covered (seg_rows_of).
 enum { SEG_LAGR, SEG_X, SEG_Y };
-void seg_geom(const Chunk& c, int kind, int* ks, int* nb, int* rows, int* ch, int* cf) {
-  if (kind == SEG_LAGR) { *ks = c.lks; *nb = c.lnb; *rows = c.ny; *ch = c.lch; *cf = c.lcf; }
-  else if (kind == SEG_X) { *ks = c.xks; *nb = c.xnb; *rows = c.ny + 1; *ch = c.xch; *cf = c.xcf; }
-  else { *ks = c.yks; *nb = c.ynb; *rows = c.ny + 1; *ch = c.ych; *cf = c.ycf; }
+void seg_geom(const Chunk& c, int kind, int* ks, int* nb, int* rows, int* ch, int* cf, int* td) {
+  if (kind == SEG_LAGR) { *ks = c.lks; *nb = c.lnb; *rows = c.ny; *ch = c.lch; *cf = c.lcf; *td = c.ltd; }
+  else if (kind == SEG_X) { *ks = c.xks; *nb = c.xnb; *rows = c.ny + 1; *ch = c.xch; *cf = c.xcf; *td = c.xtd; }
+  else { *ks = c.yks; *nb = c.ynb; *rows = c.ny + 1; *ch = c.ych; *cf = c.ycf; *td = c.ytd; }
 }
 // the segment holding row r (1-based), inverse of seg_rows_of
-int seg_of_row(int r, int ks, int nb) {
+int seg_of_row(int r, int ks, int nb, int td) {
   if (r < 1) r = 1;
   if ((int64_t)(r - 1) < (int64_t)nb * ks) return (r - 1) / ks;
-  return nb + (int)(((int64_t)(r - 1) - (int64_t)nb * ks) / (ks / CLOVER_TAIL_DIV));
+  return nb + (int)(((int64_t)(r - 1) - (int64_t)nb * ks) / (ks / td));
 }
 // Boundary / interior split of a chunk's segments [0, n) for an exchange of
 // depth yd: [0, lo) holds the rows sent to the neighbour below (1 .. yd+1),
 // [hi, n) those sent up (ny+1-yd .. ny); [lo, hi) is the interior.
 void phase_ranges(const Chunk& c, int kind, int yd, int* lo, int* hi, int* n) {
-  int ks, nb, rows, ch, cf;
-  seg_geom(c, kind, &ks, &nb, &rows, &ch, &cf);
-  *n = seg_count_lay(ks, nb, ch, cf, rows);
+  int ks, nb, rows, ch, cf, td;
+  seg_geom(c, kind, &ks, &nb, &rows, &ch, &cf, &td);
+  *n = seg_count_lay(ks, nb, ch, cf, rows, td);
   // (lo / hi: sub-range launches, row layout only -- callers pass ch = 0)
-  *lo = c.wb ? 0 : std::min(*n, seg_of_row(yd + 1, ks, nb) + 1);
-  *hi = c.wt ? *n : std::min(*n, std::max(*lo, seg_of_row(std::max(1, c.ny + 1 - yd), ks, nb)));
+  *lo = c.wb ? 0 : std::min(*n, seg_of_row(yd + 1, ks, nb, td) + 1);
+  *hi = c.wt ? *n : std::min(*n, std::max(*lo, seg_of_row(std::max(1, c.ny + 1 - yd), ks, nb, td)));
 }
 
 // Enqueue kernel phases [0, nphase) of one step (7 = full step).
@@ -1195,7 +1219,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
       vb.a[t].q = v.buf[B_Q];
       vb.a[t].fix = v.fix;
       g.x = std::max(g.x, grid_cols_v(v.c.nx, v.c.ny, v.c.vks).x);
-      g.y = std::max<unsigned>(g.y, (unsigned)seg_count_lay(v.c.vks, v.c.vnb, v.c.vch, v.c.vcf, v.c.ny));
+      g.y = std::max<unsigned>(g.y, (unsigned)seg_count_lay(v.c.vks, v.c.vnb, v.c.vch, v.c.vcf, v.c.ny, v.c.vtd));
     }
     launch_step(ks_visc_dt_b, g, SBV, st, vb, ctx->scal, ctx->dtp);
     STEP_LAUNCH_CHECK();
@@ -1214,7 +1238,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
       if (deep) view = deep_view(ctx, cs0, DEEP_EXT_VISC);
       const ChunkState& cs = deep ? view : cs0;
       const Chunk c = with_rev(cs.c, CLOVER_SERP);  // top-down: sweep 2 wrote these rows last
-      launch_step(ks_visc_dt, dim3(grid_cols_v(c.nx, c.ny, c.vks).x, seg_count_lay(c.vks, c.vnb, c.vch, c.vcf, c.ny)), SBV, st, c, cs.tm_visc, cs.buf[B_Q],
+      launch_step(ks_visc_dt, dim3(grid_cols_v(c.nx, c.ny, c.vks).x, seg_count_lay(c.vks, c.vnb, c.vch, c.vcf, c.ny, c.vtd)), SBV, st, c, cs.tm_visc, cs.buf[B_Q],
                   ctx->scal, ctx->dtp, cs.fix);
       STEP_LAUNCH_CHECK();
       launch_fix(kf_visc_dt, FIX_BLOCKS, SBV, st, c, cs.tm_visc, cs.buf[B_Q], ctx->scal, ctx->dtp,
@@ -1277,7 +1301,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
         lb.a[t] = LArgs{v.c, v.tm_lag, v.buf[B_D1], v.buf[B_E1], v.buf[B_U1], v.buf[B_V1],
                         v.buf[B_FX], v.buf[B_FY], v.fix};
         g.x = std::max(g.x, grid_strip(v.c.nx, LW, v.c.ny, v.c.lks).x);
-        g.y = std::max<unsigned>(g.y, (unsigned)seg_count_lay(v.c.lks, v.c.lnb, v.c.lch, v.c.lcf, v.c.ny));
+        g.y = std::max<unsigned>(g.y, (unsigned)seg_count_lay(v.c.lks, v.c.lnb, v.c.lch, v.c.lcf, v.c.ny, v.c.ltd));
       }
       launch_step(ks_lagrangian_b, g, SB, st, lb, ctx->scal);
       STEP_LAUNCH_CHECK();
@@ -1342,7 +1366,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
             xb.a[t] = XArgs{v.c, sweep == 1 ? v.tm_x1x : v.tm_x2, v.buf[rout], v.buf[eout],
                             v.buf[uout], v.buf[vout], v.fix};
             g.x = std::max(g.x, grid_strip(v.c.nx + 1, XW, v.c.ny + 1, v.c.xks).x);
-            g.y = std::max<unsigned>(g.y, (unsigned)seg_count_lay(v.c.xks, v.c.xnb, v.c.xch, v.c.xcf, v.c.ny + 1));
+            g.y = std::max<unsigned>(g.y, (unsigned)seg_count_lay(v.c.xks, v.c.xnb, v.c.xch, v.c.xcf, v.c.ny + 1, v.c.xtd));
           }
           if (sweep == 1) launch_step(ks_advec_x_b<1>, g, SB, st, xb);
           else launch_step(ks_advec_x_b<2>, g, SB, st, xb);
@@ -1426,7 +1450,7 @@ int enqueue_step(clover_ctx* ctx, bool advect_x, int nphase) {
                             v.buf[rout], v.buf[eout], v.buf[B_MY], v.buf[uout], v.buf[vout],
                             v.fix};
             g.x = std::max(g.x, grid_strip(v.c.nx + 1, YW, v.c.ny + 1, v.c.yks).x);
-            g.y = std::max<unsigned>(g.y, (unsigned)seg_count_lay(v.c.yks, v.c.ynb, v.c.ych, v.c.ycf, v.c.ny + 1));
+            g.y = std::max<unsigned>(g.y, (unsigned)seg_count_lay(v.c.yks, v.c.ynb, v.c.ych, v.c.ycf, v.c.ny + 1, v.c.ytd));
           }
           if (sweep == 1) launch_step(ks_advec_y_b<1>, g, SB, st, yb);
           else launch_step(ks_advec_y_b<2>, g, SB, st, yb);

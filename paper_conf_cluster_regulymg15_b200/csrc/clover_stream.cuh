@@ -165,7 +165,7 @@ struct NoLast {
 #endif
 constexpr int FIX_BLOCKS = CLOVER_FIX_BLOCKS;
 template <int BS = SB, class Run, class Last = NoLast>
-__device__ __forceinline__ void fix_loop(FixSlot f, int ks, int nb, int ch, int cf, int lim, Run&& run,
+__device__ __forceinline__ void fix_loop(FixSlot f, int ks, int nb, int ch, int cf, int td, int lim, Run&& run,
                                          Last last = {}) {
   const unsigned n = *(volatile unsigned*)f.hdr;  // the same value in every thread
   if (n == 0u) {
@@ -178,7 +178,7 @@ __device__ __forceinline__ void fix_loop(FixSlot f, int ks, int nb, int ch, int 
   for (unsigned it = blockIdx.x * (BS / 32) + w; it < items; it += FIX_BLOCKS * (BS / 32)) {
     const uint2 t = f.e[it / ks];
     int ks0, len;
-    seg_rows_lay((int)t.y, ks, nb, ch, cf, lim - 1, ks0, len);
+    seg_rows_lay((int)t.y, ks, nb, ch, cf, lim - 1, ks0, len, td);
     const int r = (int)(it % ks);
     const int k0 = ks0 + r;
     if (r < len && k0 < lim) run((int)t.x, k0, k0 + 1, lane, w);
@@ -455,7 +455,7 @@ ks_visc_dt(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__
   double dtw = G_BIG;
   int k0, len;
   const int sg = seg_y(c);
-  seg_rows_lay(sg, c.vks, c.vnb, c.vch, c.vcf, c.ny, k0, len);
+  seg_rows_lay(sg, c.vks, c.vnb, c.vch, c.vcf, c.ny, k0, len, c.vtd);
   if (len <= 0) return;  // empty band segment
   int k1 = min(k0 + len, c.ny + 1);
   visc_ring_rows(c, k0, k1);
@@ -486,7 +486,7 @@ kf_visc_dt(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__
   // fin: single chunk on one rank -- the last block also finalises dt
   // (k_dt_finalize's work, once every contribution to the slot is in)
   fix_loop<SBV>(
-      fix, c.vks, c.vnb, c.vch, c.vcf, c.ny + 1,
+      fix, c.vks, c.vnb, c.vch, c.vcf, c.vtd, c.ny + 1,
       [&](int gw, int k0, int k1, int lane, int w) {
         double dtw;
         visc_ring_rows(c, k0, k1);  // rows 1 / ny redo their ring row too
@@ -803,7 +803,7 @@ ks_lagrangian(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restric
   const int gw = blockIdx.x * (SB / 32) + w;
   int k0, len;
   const int sg = seg_y(c);
-  seg_rows_lay(sg, c.lks, c.lnb, c.lch, c.lcf, c.ny, k0, len);
+  seg_rows_lay(sg, c.lks, c.lnb, c.lch, c.lcf, c.ny, k0, len, c.ltd);
   if (len <= 0) return;  // empty band segment
   const int k1 = min(k0 + len, c.ny + 1);
   if (lagr_seg<DivFast>(c, &tm, d1, e1, u1, v1, fx, fy, s, gw, k0, k1, lane, ring[w], bars[w]))
@@ -820,7 +820,7 @@ kf_lagrangian(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restric
   if (y_walls_after_fix<1>(c, fix, yw)) return;
   __shared__ __align__(128) double ring[SB / 32][LSTG * LSLOT];
   __shared__ __align__(8) unsigned long long bars[SB / 32][LSTG];
-  fix_loop(fix, c.lks, c.lnb, c.lch, c.lcf, c.ny + 1, [&](int gw, int k0, int k1, int lane, int w) {
+  fix_loop(fix, c.lks, c.lnb, c.lch, c.lcf, c.ltd, c.ny + 1, [&](int gw, int k0, int k1, int lane, int w) {
     // the IEEE redo's flag is the exact PdV volume test (DivIEEE::vol_check)
     if (lagr_seg<DivIEEE>(c, &tm, d1, e1, u1, v1, fx, fy, s, gw, k0, k1, lane, ring[w], bars[w]) &&
         lane == 0)
@@ -918,7 +918,7 @@ kf_advec_cell_x(Chunk c, const double* __restrict__ rho, const double* __restric
                 double* __restrict__ mfx, FixSlot fix) {
   pdl_trigger();
   pdl_wait();
-  fix_loop(fix, CKS, 0x7fffffff, 0, 0, c.ny + 1, [&](int gw, int k0, int k1, int lane, int) {
+  fix_loop(fix, CKS, 0x7fffffff, 0, 0, CLOVER_TAIL_DIV, c.ny + 1, [&](int gw, int k0, int k1, int lane, int) {
     advec_cell_x_body<SWEEP, DivIEEE>(c, rho, en, fx, fy, rho_out, en_out, mfx, gw, k0, k1, lane);
   });
 }
@@ -1034,7 +1034,7 @@ kf_advec_cell_y(Chunk c, const double* __restrict__ rho, const double* __restric
                 double* __restrict__ mfy, FixSlot fix) {
   pdl_trigger();
   pdl_wait();
-  fix_loop(fix, CKS_Y, 0x7fffffff, 0, 0, c.ny + 1, [&](int gw, int k0, int k1, int lane, int) {
+  fix_loop(fix, CKS_Y, 0x7fffffff, 0, 0, CLOVER_TAIL_DIV, c.ny + 1, [&](int gw, int k0, int k1, int lane, int) {
     advec_cell_y_body<SWEEP, DivIEEE, true>(c, rho, en, fx, fy, rho_out, en_out, mfy, gw, k0, k1, lane);
   });
 }
@@ -1136,7 +1136,7 @@ kf_advec_mom_x(Chunk c, const double* __restrict__ rho, const double* __restrict
                double* __restrict__ vout, FixSlot fix) {
   pdl_trigger();
   pdl_wait();
-  fix_loop(fix, MKS, 0x7fffffff, 0, 0, c.ny + 2, [&](int gw, int k0, int k1, int lane, int) {
+  fix_loop(fix, MKS, 0x7fffffff, 0, 0, CLOVER_TAIL_DIV, c.ny + 2, [&](int gw, int k0, int k1, int lane, int) {
     advec_mom_x_body<SWEEP, DivIEEE>(c, rho, mfx, fy, uin, vin, uout, vout, gw, k0, k1, lane);
   });
 }
@@ -1428,7 +1428,7 @@ ks_advec_x(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__
   const int gw = blockIdx.x * (SB / 32) + w;
   int k0, len;
   const int sg = seg_y(c);
-  seg_rows_lay(sg, c.xks, c.xnb, c.xch, c.xcf, c.ny + 1, k0, len);
+  seg_rows_lay(sg, c.xks, c.xnb, c.xch, c.xcf, c.ny + 1, k0, len, c.xtd);
   if (len <= 0) return;  // empty band segment
   const int k1 = min(k0 + len, c.ny + 2);
   if (advec_x_seg<SWEEP, DivFast>(c, &tm, rho_out, en_out, uout, vout, gw, k0, k1, lane, ring[w],
@@ -1447,7 +1447,7 @@ kf_advec_x(Chunk c, const __grid_constant__ CUtensorMap tm, double* __restrict__
     if (y_walls_after_fix<2>(c, fix, yw)) return;
   __shared__ __align__(128) double ring[SB / 32][XSTG * xslot<SWEEP>()];
   __shared__ __align__(8) unsigned long long bars[SB / 32][XSTG];
-  fix_loop(fix, c.xks, c.xnb, c.xch, c.xcf, c.ny + 2, [&](int gw, int k0, int k1, int lane, int w) {
+  fix_loop(fix, c.xks, c.xnb, c.xch, c.xcf, c.xtd, c.ny + 2, [&](int gw, int k0, int k1, int lane, int w) {
     advec_x_seg<SWEEP, DivIEEE>(c, &tm, rho_out, en_out, uout, vout, gw, k0, k1, lane, ring[w],
                                  bars[w]);
   });
@@ -1564,7 +1564,7 @@ kf_advec_mom_y(Chunk c, const double* __restrict__ rho, const double* __restrict
                double* __restrict__ vout, FixSlot fix) {
   pdl_trigger();
   pdl_wait();
-  fix_loop(fix, MKS_Y, 0x7fffffff, 0, 0, c.ny + 2, [&](int gw, int k0, int k1, int lane, int) {
+  fix_loop(fix, MKS_Y, 0x7fffffff, 0, 0, CLOVER_TAIL_DIV, c.ny + 2, [&](int gw, int k0, int k1, int lane, int) {
     advec_mom_y_body<SWEEP, DivIEEE, true>(c, rho, mfy, fx, uin, vin, uout, vout, gw, k0, k1, lane);
   });
 }
@@ -1911,7 +1911,7 @@ ks_advec_y(Chunk c, const __grid_constant__ CUtensorMap ta, const __grid_constan
   const int gw = blockIdx.x * (SB / 32) + w;
   int k0, len;
   const int sg = seg_y(c);
-  seg_rows_lay(sg, c.yks, c.ynb, c.ych, c.ycf, c.ny + 1, k0, len);
+  seg_rows_lay(sg, c.yks, c.ynb, c.ych, c.ycf, c.ny + 1, k0, len, c.ytd);
   if (len <= 0) return;  // empty band segment
   const int k1 = min(k0 + len, c.ny + 2);
   if (advec_y_seg<SWEEP, DivFast>(c, &ta, &tb, rho_out, en_out, mfy, uout, vout, gw, k0, k1, lane,
@@ -1928,7 +1928,7 @@ kf_advec_y(Chunk c, const __grid_constant__ CUtensorMap ta, const __grid_constan
   pdl_wait();
   __shared__ __align__(128) double ring[SB / 32][YL<SWEEP>::RING * YL<SWEEP>::SLOT];
   __shared__ __align__(8) unsigned long long bars[SB / 32][YL<SWEEP>::RING];
-  fix_loop(fix, c.yks, c.ynb, c.ych, c.ycf, c.ny + 2, [&](int gw, int k0, int k1, int lane, int w) {
+  fix_loop(fix, c.yks, c.ynb, c.ych, c.ycf, c.ytd, c.ny + 2, [&](int gw, int k0, int k1, int lane, int w) {
     advec_y_seg<SWEEP, DivIEEE>(c, &ta, &tb, rho_out, en_out, mfy, uout, vout, gw, k0, k1, lane,
                                 ring[w], bars[w]);
   });
@@ -1957,7 +1957,7 @@ ks_visc_dt_b(const __grid_constant__ KBatch<VArgs> b, StepScalars* __restrict__ 
   pdl_wait();
   const VArgs& a = b.a[blockIdx.z];
   const Chunk& c = a.c;
-  if ((int)blockIdx.y >= seg_count_lay(c.vks, c.vnb, c.vch, c.vcf, c.ny)) return;
+  if ((int)blockIdx.y >= seg_count_lay(c.vks, c.vnb, c.vch, c.vcf, c.ny, c.vtd)) return;
   __shared__ __align__(128) double ring[SBV / 32][VSTG * VSLOT];
   __shared__ __align__(8) unsigned long long bars[SBV / 32][VSTG];
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
@@ -1965,7 +1965,7 @@ ks_visc_dt_b(const __grid_constant__ KBatch<VArgs> b, StepScalars* __restrict__ 
   double dtw = G_BIG;
   int k0, len;
   const int sg = (int)blockIdx.y;
-  seg_rows_lay(sg, c.vks, c.vnb, c.vch, c.vcf, c.ny, k0, len);
+  seg_rows_lay(sg, c.vks, c.vnb, c.vch, c.vcf, c.ny, k0, len, c.vtd);
   if (len <= 0) return;
   int k1 = min(k0 + len, c.ny + 1);
   visc_ring_rows(c, k0, k1);
@@ -1992,7 +1992,7 @@ kf_visc_dt_b(const __grid_constant__ KBatch<VArgs> b, StepScalars* __restrict__ 
   const Chunk& c = a.c;
   __shared__ __align__(128) double ring[SBV / 32][VSTG * VSLOT];
   __shared__ __align__(8) unsigned long long bars[SBV / 32][VSTG];
-  fix_loop<SBV>(a.fix, c.vks, c.vnb, c.vch, c.vcf, c.ny + 1, [&](int gw, int k0, int k1, int lane, int w) {
+  fix_loop<SBV>(a.fix, c.vks, c.vnb, c.vch, c.vcf, c.vtd, c.ny + 1, [&](int gw, int k0, int k1, int lane, int w) {
     double dtw;
     visc_ring_rows(c, k0, k1);
     visc_seg<DivIEEE>(c, &a.tm, a.q, prm, gw, k0, k1, lane, ring[w], bars[w], dtw);
@@ -2006,14 +2006,14 @@ ks_lagrangian_b(const __grid_constant__ KBatch<LArgs> b, const StepScalars* __re
   pdl_wait();
   const LArgs& a = b.a[blockIdx.z];
   const Chunk& c = a.c;
-  if ((int)blockIdx.y >= seg_count_lay(c.lks, c.lnb, c.lch, c.lcf, c.ny)) return;
+  if ((int)blockIdx.y >= seg_count_lay(c.lks, c.lnb, c.lch, c.lcf, c.ny, c.ltd)) return;
   __shared__ __align__(128) double ring[SB / 32][LSTG * LSLOT];
   __shared__ __align__(8) unsigned long long bars[SB / 32][LSTG];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const int gw = blockIdx.x * (SB / 32) + w;
   int k0, len;
   const int sg = (int)blockIdx.y;
-  seg_rows_lay(sg, c.lks, c.lnb, c.lch, c.lcf, c.ny, k0, len);
+  seg_rows_lay(sg, c.lks, c.lnb, c.lch, c.lcf, c.ny, k0, len, c.ltd);
   if (len <= 0) return;
   const int k1 = min(k0 + len, c.ny + 1);
   if (lagr_seg<DivFast>(c, &a.tm, a.d1, a.e1, a.u1, a.v1, a.fx, a.fy, s, gw, k0, k1, lane, ring[w],
@@ -2028,7 +2028,7 @@ kf_lagrangian_b(const __grid_constant__ KBatch<LArgs> b, StepScalars* __restrict
   const Chunk& c = a.c;
   __shared__ __align__(128) double ring[SB / 32][LSTG * LSLOT];
   __shared__ __align__(8) unsigned long long bars[SB / 32][LSTG];
-  fix_loop(a.fix, c.lks, c.lnb, c.lch, c.lcf, c.ny + 1, [&](int gw, int k0, int k1, int lane, int w) {
+  fix_loop(a.fix, c.lks, c.lnb, c.lch, c.lcf, c.ltd, c.ny + 1, [&](int gw, int k0, int k1, int lane, int w) {
     if (lagr_seg<DivIEEE>(c, &a.tm, a.d1, a.e1, a.u1, a.v1, a.fx, a.fy, s, gw, k0, k1, lane,
                           ring[w], bars[w]) &&
         lane == 0)
@@ -2042,14 +2042,14 @@ __global__ void LB_ADVX ks_advec_x_b(const __grid_constant__ KBatch<XArgs> b) {
   pdl_wait();
   const XArgs& a = b.a[blockIdx.z];
   const Chunk& c = a.c;
-  if ((int)blockIdx.y >= seg_count_lay(c.xks, c.xnb, c.xch, c.xcf, c.ny + 1)) return;
+  if ((int)blockIdx.y >= seg_count_lay(c.xks, c.xnb, c.xch, c.xcf, c.ny + 1, c.xtd)) return;
   __shared__ __align__(128) double ring[SB / 32][XSTG * xslot<SWEEP>()];
   __shared__ __align__(8) unsigned long long bars[SB / 32][XSTG];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const int gw = blockIdx.x * (SB / 32) + w;
   int k0, len;
   const int sg = (int)blockIdx.y;
-  seg_rows_lay(sg, c.xks, c.xnb, c.xch, c.xcf, c.ny + 1, k0, len);
+  seg_rows_lay(sg, c.xks, c.xnb, c.xch, c.xcf, c.ny + 1, k0, len, c.xtd);
   if (len <= 0) return;
   const int k1 = min(k0 + len, c.ny + 2);
   if (advec_x_seg<SWEEP, DivFast>(c, &a.tm, a.rho, a.en, a.u, a.v, gw, k0, k1, lane, ring[w],
@@ -2064,7 +2064,7 @@ __global__ void __launch_bounds__(SB) kf_advec_x_b(const __grid_constant__ KBatc
   const Chunk& c = a.c;
   __shared__ __align__(128) double ring[SB / 32][XSTG * xslot<SWEEP>()];
   __shared__ __align__(8) unsigned long long bars[SB / 32][XSTG];
-  fix_loop(a.fix, c.xks, c.xnb, c.xch, c.xcf, c.ny + 2, [&](int gw, int k0, int k1, int lane, int w) {
+  fix_loop(a.fix, c.xks, c.xnb, c.xch, c.xcf, c.xtd, c.ny + 2, [&](int gw, int k0, int k1, int lane, int w) {
     advec_x_seg<SWEEP, DivIEEE>(c, &a.tm, a.rho, a.en, a.u, a.v, gw, k0, k1, lane, ring[w],
                                  bars[w]);
   });
@@ -2077,14 +2077,14 @@ ks_advec_y_b(const __grid_constant__ KBatch<YArgs> b) {
   pdl_wait();
   const YArgs& a = b.a[blockIdx.z];
   const Chunk& c = a.c;
-  if ((int)blockIdx.y >= seg_count_lay(c.yks, c.ynb, c.ych, c.ycf, c.ny + 1)) return;
+  if ((int)blockIdx.y >= seg_count_lay(c.yks, c.ynb, c.ych, c.ycf, c.ny + 1, c.ytd)) return;
   __shared__ __align__(128) double ring[SB / 32][YL<SWEEP>::RING * YL<SWEEP>::SLOT];
   __shared__ __align__(8) unsigned long long bars[SB / 32][YL<SWEEP>::RING];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const int gw = blockIdx.x * (SB / 32) + w;
   int k0, len;
   const int sg = (int)blockIdx.y;
-  seg_rows_lay(sg, c.yks, c.ynb, c.ych, c.ycf, c.ny + 1, k0, len);
+  seg_rows_lay(sg, c.yks, c.ynb, c.ych, c.ycf, c.ny + 1, k0, len, c.ytd);
   if (len <= 0) return;
   const int k1 = min(k0 + len, c.ny + 2);
   if (advec_y_seg<SWEEP, DivFast>(c, &a.ta, &a.tb, a.rho, a.en, a.mfy, a.u, a.v, gw, k0, k1, lane,
@@ -2099,7 +2099,7 @@ __global__ void __launch_bounds__(SB) kf_advec_y_b(const __grid_constant__ KBatc
   const Chunk& c = a.c;
   __shared__ __align__(128) double ring[SB / 32][YL<SWEEP>::RING * YL<SWEEP>::SLOT];
   __shared__ __align__(8) unsigned long long bars[SB / 32][YL<SWEEP>::RING];
-  fix_loop(a.fix, c.yks, c.ynb, c.ych, c.ycf, c.ny + 2, [&](int gw, int k0, int k1, int lane, int w) {
+  fix_loop(a.fix, c.yks, c.ynb, c.ych, c.ycf, c.ytd, c.ny + 2, [&](int gw, int k0, int k1, int lane, int w) {
     advec_y_seg<SWEEP, DivIEEE>(c, &a.ta, &a.tb, a.rho, a.en, a.mfy, a.u, a.v, gw, k0, k1, lane,
                                 ring[w], bars[w]);
   });

@@ -32,14 +32,15 @@ int main() {
   // within a band the segments ascend with the launch slot (consecutive
   // rows), the band's first segment is in wave 0 and its last
   // CLOVER_TAIL_WAVES segments have ks / CLOVER_TAIL_DIV rows
+  for (int td = 2; td <= 4; td += 2)
   for (int ks = 8; ks <= 64; ks *= 2)
     for (int rows = 1; rows <= 4200; rows += (rows < 300 ? 1 : 97))
       for (int C = 0; C <= 40; ++C) {
         int ch, cf;
-        band_params(ks, C, rows, &ch, &cf);
+        band_params(ks, C, rows, &ch, &cf, td);
         if (ch == 0) continue;
         ++banded;
-        const int n = seg_count_lay(ks, 0, ch, cf, rows);
+        const int n = seg_count_lay(ks, 0, ch, cf, rows, td);
         if (n != (cf + CLOVER_TAIL_WAVES) * ch) return fail("count", ks, rows, ch, n);
         std::vector<int> cover(rows + 2, 0);
         for (int c = 0; c < ch; ++c) {
@@ -47,9 +48,9 @@ int main() {
           for (int w = 0; w < cf + CLOVER_TAIL_WAVES; ++w) {
             const int s = w * ch + c;
             int k0, len;
-            seg_rows_lay(s, ks, 0, ch, cf, rows, k0, len);
+            seg_rows_lay(s, ks, 0, ch, cf, rows, k0, len, td);
             if (len > ks) return fail("len", ks, rows, ch, s);
-            if (w >= cf && len != ks / CLOVER_TAIL_DIV) return fail("tail", ks, rows, ch, s);
+            if (w >= cf && len != ks / td) return fail("tail", ks, rows, ch, s);
             if (len <= 0) continue;
             if (next >= 0 && k0 != next) return fail("band order", ks, rows, ch, s);
             next = k0 + len;
@@ -63,14 +64,15 @@ int main() {
           if (cover[k] != 1) return fail("cover", ks, rows, ch, k);
       }
   // row layout (ch = 0): full segments then half-height tail segments
-  for (int ks = 8; ks <= 64; ks *= 2)
+  for (int td = 2; td <= 4; td += 2)
+  for (int ks = 16; ks <= 64; ks *= 2)
     for (int nb = 0; nb <= 40; ++nb)
       for (int rows = 1; rows <= 2000; rows += 37) {
-        const int n = seg_count_lay(ks, nb, 0, 0, rows);
+        const int n = seg_count_lay(ks, nb, 0, 0, rows, td);
         int next = 1;
         for (int s = 0; s < n; ++s) {
           int k0, len;
-          seg_rows_lay(s, ks, nb, 0, 0, rows, k0, len);
+          seg_rows_lay(s, ks, nb, 0, 0, rows, k0, len, td);
           if (k0 != next || len <= 0) return fail("rows", ks, rows, nb, s);
           next = k0 + len;
         }
